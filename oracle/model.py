@@ -1,0 +1,398 @@
+"""CPU ORACLE (test infrastructure only) — plain fp64 forward/backward of the workload models.
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl reference legs may
+import this module. It shares no code with the CUDA path (paper_conf_eurosys_stratimk24_b200/).
+
+What it computes. Orion's numeric outputs have a plain definition independent of scheduling
+(§5.1: Orion only decides *when* each client's kernels launch; stream order keeps each
+client's data dependencies). So the oracle is each client's model written out with
+PyTorch/TorchVision semantics, which is what the paper ran (TorchVision ResNet50 /
+MobileNet-v2, full precision):
+  * every op computes in float64 with plain torch CPU primitives (a conv, a matmul, a sum);
+  * every op's output is rounded to the GPU's storage dtype (float32) before the next op uses it,
+    exactly as the unfused GPU op stream materialises it (DESIGN.md §3 R22-R24);
+  * backward passes are written out op by op (no autograd), in the reverse order of the forward.
+Layouts follow the GPU's HBM layout so buffers can be compared element by element:
+activations NHWC, conv weights OHWI ([Cout, kh, kw, Cin/groups]), linear weights [out, in].
+
+Pins (tests/test_oracle_model.py): explicit-loop brute force of every forward op on tiny shapes,
+central finite differences (fp64) of every backward op, closed forms (BN output moments, CE of
+uniform logits = log C, MSE), and model-level gradients against fp64 autograd of the same forward.
+"""
+import math
+
+import torch
+import torch.nn.functional as F
+
+F64 = torch.float64
+F32 = torch.float32
+
+
+def _r(t):
+    """Round an fp64 result to the fp32 storage dtype (the unfused GPU op writes fp32)."""
+    return t.to(F32)
+
+
+def _d(t):
+    return t.to(F64)
+
+
+def _nchw(x):   # NHWC -> NCHW view for torch primitives
+    return x.permute(0, 3, 1, 2)
+
+
+def _nhwc(x):
+    return x.permute(0, 2, 3, 1).contiguous()
+
+
+def _w_oihw(w):  # OHWI -> OIHW
+    return w.permute(0, 3, 1, 2)
+
+
+# ----------------------------------------------------------------------------------- linear
+def linear_fwd(x, w, b):
+    """y = x W^T + b  (torch.nn.Linear). x [B, in], w [out, in], b [out]."""
+    return _r(_d(x) @ _d(w).t() + (_d(b) if b is not None else 0.0))
+
+
+def linear_bwd(x, w, dy):
+    """dx = dy W, dW = dy^T x, db = sum_b dy."""
+    dyd = _d(dy)
+    return _r(dyd @ _d(w)), _r(dyd.t() @ _d(x)), _r(dyd.sum(0))
+
+
+# ------------------------------------------------------------------------------------- conv
+def conv2d_fwd(x, w, stride=1, pad=0, groups=1):
+    """Conv2d, zero padding, no bias (TorchVision convs are bias-free). x NHWC, w OHWI."""
+    y = F.conv2d(_nchw(_d(x)), _w_oihw(_d(w)), None, stride, pad, 1, groups)
+    return _r(_nhwc(y))
+
+
+def conv2d_bwd_data(dy, w, x_shape, stride=1, pad=0, groups=1):
+    dx = torch.nn.grad.conv2d_input((x_shape[0], x_shape[3], x_shape[1], x_shape[2]), _w_oihw(_d(w)),
+                                    _nchw(_d(dy)), stride, pad, 1, groups)
+    return _r(_nhwc(dx))
+
+
+def conv2d_bwd_weight(x, dy, w_shape, stride=1, pad=0, groups=1):
+    o, kh, kw, ig = w_shape
+    dw = torch.nn.grad.conv2d_weight(_nchw(_d(x)), (o, ig, kh, kw), _nchw(_d(dy)), stride, pad, 1, groups)
+    return _r(dw.permute(0, 2, 3, 1).contiguous())
+
+
+# --------------------------------------------------------------------------------------- BN
+def bn_eval(x, gamma, beta, rmean, rvar, eps=1e-5):
+    """BatchNorm2d eval: (x - rm) / sqrt(rv + eps) * gamma + beta, per channel (last dim)."""
+    inv = 1.0 / torch.sqrt(_d(rvar) + eps)
+    return _r((_d(x) - _d(rmean)) * inv * _d(gamma) + _d(beta))
+
+
+def bn_train_fwd(x, gamma, beta, rmean, rvar, eps=1e-5, momentum=0.1):
+    """BatchNorm2d train: normalise with the batch mean and biased variance; update running stats
+    with momentum and the *unbiased* variance (torch semantics). Returns y, mean, invstd, rm', rv'."""
+    xd = _d(x)
+    c = x.shape[-1]
+    flat = xd.reshape(-1, c)
+    n = flat.shape[0]
+    mean = flat.mean(0)
+    var = ((flat - mean) ** 2).mean(0)
+    invstd = 1.0 / torch.sqrt(var + eps)
+    y = (xd - mean) * invstd * _d(gamma) + _d(beta)
+    rm = (1 - momentum) * _d(rmean) + momentum * mean
+    rv = (1 - momentum) * _d(rvar) + momentum * var * n / (n - 1)
+    return _r(y), _r(mean), _r(invstd), _r(rm), _r(rv)
+
+
+def bn_bwd(x, dy, gamma, mean, invstd):
+    """Backward of training-mode BN given the saved (fp32) batch mean / invstd.
+    xhat = (x-mean)*invstd; dbeta = sum dy; dgamma = sum dy*xhat;
+    dx = gamma*invstd/N * (N dy - dbeta - xhat dgamma)."""
+    c = x.shape[-1]
+    xd = _d(x).reshape(-1, c)
+    dyd = _d(dy).reshape(-1, c)
+    n = xd.shape[0]
+    xhat = (xd - _d(mean)) * _d(invstd)
+    dbeta = dyd.sum(0)
+    dgamma = (dyd * xhat).sum(0)
+    dx = _d(gamma) * _d(invstd) / n * (n * dyd - dbeta - xhat * dgamma)
+    return _r(dx.reshape(x.shape)), _r(dgamma), _r(dbeta)
+
+
+# ------------------------------------------------------------------------------ elementwise
+def relu(x):
+    return _r(torch.clamp(_d(x), min=0.0))
+
+
+def relu_bwd(x, dy):
+    """Gradient passes where x > 0 (torch threshold_backward)."""
+    return _r(torch.where(_d(x) > 0, _d(dy), torch.zeros((), dtype=F64)))
+
+
+def relu6(x):
+    return _r(torch.clamp(_d(x), 0.0, 6.0))
+
+
+def relu6_bwd(x, dy):
+    """hardtanh_backward(0, 6): gradient passes where 0 < x < 6."""
+    xd = _d(x)
+    return _r(torch.where((xd > 0) & (xd < 6), _d(dy), torch.zeros((), dtype=F64)))
+
+
+def add(a, b):
+    return _r(_d(a) + _d(b))
+
+
+# ---------------------------------------------------------------------------------- pooling
+def maxpool3x3s2(x):
+    """MaxPool2d(3, stride 2, padding 1), -inf padding. NHWC."""
+    y = F.max_pool2d(_nchw(_d(x)), 3, 2, 1)
+    return _r(_nhwc(y))
+
+
+def avgpool_fwd(x):
+    """Global average pool (AdaptiveAvgPool2d(1) + flatten): [N,H,W,C] -> [N,C]."""
+    return _r(_d(x).mean(dim=(1, 2)))
+
+
+def avgpool_bwd(dy, x_shape):
+    n, h, w, c = x_shape
+    return _r((_d(dy) / (h * w)).reshape(n, 1, 1, c).expand(n, h, w, c).contiguous())
+
+
+# ------------------------------------------------------------------------------------ losses
+def ce_fwd_bwd(z, labels):
+    """Cross entropy, mean over batch: L = mean_i(logsumexp(z_i) - z_i[y_i]);
+    dz = (softmax(z) - onehot(y)) / B."""
+    zd = _d(z)
+    b = zd.shape[0]
+    lse = torch.logsumexp(zd, dim=1)
+    loss = (lse - zd[torch.arange(b), labels.long()]).mean()
+    p = torch.exp(zd - lse[:, None])
+    p[torch.arange(b), labels.long()] -= 1.0
+    return _r(loss), _r(p / b)
+
+
+def mse_fwd_bwd(y, t):
+    """MSE, mean over all elements: L = mean((y-t)^2); dy = 2 (y-t) / numel."""
+    diff = _d(y) - _d(t)
+    return _r((diff ** 2).mean()), _r(2.0 * diff / diff.numel())
+
+
+# ---------------------------------------------------------------------------------- optimizer
+def sgd(p, g, v, lr, momentum, first):
+    """torch.optim.SGD (dampening 0, no weight decay): v <- g (first step) else mu v + g;
+    p <- p - lr v. With momentum == 0 the buffer is unused: p <- p - lr g."""
+    if momentum == 0.0:
+        return _r(_d(p) - lr * _d(g)), v
+    vn = _d(g) if first else momentum * _d(v) + _d(g)
+    return _r(_d(p) - lr * _r(vn).to(F64)), _r(vn)
+
+
+# ================================================================================== models
+# Parameter specs: ordered list of (name, shape, init). `init` names a distribution that the
+# seeded generator (synth/inputs.py) draws from; the oracle never draws random numbers itself.
+
+def mlp_spec(width=512, layers=3):
+    spec = []
+    for i in range(layers):
+        spec.append((f"fc{i}.w", (width, width), ("uniform_fan_in", width)))
+        spec.append((f"fc{i}.b", (width,), ("uniform_fan_in", width)))
+    return spec
+
+
+def mlp_fwd(P, x, layers=3, keep=False):
+    """Toy MLP (BASELINE config 1): Linear-ReLU-Linear-ReLU-Linear."""
+    acts = [x]
+    h = x
+    for i in range(layers):
+        h = linear_fwd(h, P[f"fc{i}.w"], P[f"fc{i}.b"])
+        acts.append(h)
+        if i < layers - 1:
+            h = relu(h)
+            acts.append(h)
+    return (h, acts) if keep else h
+
+
+def mlp_train_step(P, x, t, lr=0.01, layers=3):
+    """One SGD(momentum 0) step with MSE loss. Returns (loss, new params)."""
+    y, acts = mlp_fwd(P, x, layers, keep=True)
+    loss, dy = mse_fwd_bwd(y, t)
+    grads = {}
+    # acts: [x, z0, h0, z1, h1, z2]
+    for i in reversed(range(layers)):
+        inp = acts[2 * i]
+        dx, dw, db = linear_bwd(inp, P[f"fc{i}.w"], dy)
+        grads[f"fc{i}.w"], grads[f"fc{i}.b"] = dw, db
+        if i > 0:
+            dy = relu_bwd(acts[2 * i - 1], dx)
+    newP = {k: sgd(P[k], grads[k], None, lr, 0.0, True)[0] for k in P}
+    return loss, newP, grads
+
+
+# ------------------------------------------------------------------------------ ResNet-50
+RESNET50_LAYERS = [(64, 3, 1), (128, 4, 2), (256, 6, 2), (512, 3, 2)]   # (width, blocks, stride)
+RESNET101_LAYERS = [(64, 3, 1), (128, 4, 2), (256, 23, 2), (512, 3, 2)]
+
+
+def _bn_spec(name, c, eval_stats):
+    s = [(f"{name}.gamma", (c,), ("const", 1.0)), (f"{name}.beta", (c,), ("const", 0.0))]
+    if eval_stats:
+        s += [(f"{name}.rmean", (c,), ("normal", 0.1)), (f"{name}.rvar", (c,), ("uniform", 0.5, 1.5))]
+    else:
+        s += [(f"{name}.rmean", (c,), ("const", 0.0)), (f"{name}.rvar", (c,), ("const", 1.0))]
+    return s
+
+
+def _conv_spec(name, cout, k, cin_g):
+    # kaiming_normal_(mode='fan_out', relu): std = sqrt(2 / (cout * k * k))
+    return [(f"{name}.w", (cout, k, k, cin_g), ("kaiming_fan_out", cout * k * k))]
+
+
+def resnet_spec(layers=RESNET50_LAYERS, num_classes=1000, eval_stats=True):
+    s = _conv_spec("conv1", 64, 7, 3) + _bn_spec("bn1", 64, eval_stats)
+    cin = 64
+    for li, (w, nb, stride) in enumerate(layers):
+        for bi in range(nb):
+            p = f"layer{li + 1}.{bi}"
+            s += _conv_spec(f"{p}.conv1", w, 1, cin) + _bn_spec(f"{p}.bn1", w, eval_stats)
+            s += _conv_spec(f"{p}.conv2", w, 3, w) + _bn_spec(f"{p}.bn2", w, eval_stats)
+            s += _conv_spec(f"{p}.conv3", 4 * w, 1, w) + _bn_spec(f"{p}.bn3", 4 * w, eval_stats)
+            if bi == 0:
+                s += _conv_spec(f"{p}.down", 4 * w, 1, cin) + _bn_spec(f"{p}.downbn", 4 * w, eval_stats)
+            cin = 4 * w
+    s += [("fc.w", (num_classes, cin), ("uniform_fan_in", cin)), ("fc.b", (num_classes,), ("uniform_fan_in", cin))]
+    return s
+
+
+def resnet_infer(P, x, layers=RESNET50_LAYERS):
+    """TorchVision ResNet v1.5 (stride on the 3x3), eval-mode BN. x NHWC [N,H,W,3] -> logits [N,1000]."""
+    def cbr(h, name, bn, stride, pad, act=True):
+        h = conv2d_fwd(h, P[f"{name}.w"], stride, pad)
+        h = bn_eval(h, P[f"{bn}.gamma"], P[f"{bn}.beta"], P[f"{bn}.rmean"], P[f"{bn}.rvar"])
+        return relu(h) if act else h
+    h = cbr(x, "conv1", "bn1", 2, 3)
+    h = maxpool3x3s2(h)
+    for li, (w, nb, stride) in enumerate(layers):
+        for bi in range(nb):
+            p = f"layer{li + 1}.{bi}"
+            s = stride if bi == 0 else 1
+            o = cbr(h, f"{p}.conv1", f"{p}.bn1", 1, 0)
+            o = cbr(o, f"{p}.conv2", f"{p}.bn2", s, 1)
+            o = cbr(o, f"{p}.conv3", f"{p}.bn3", 1, 0, act=False)
+            idn = cbr(h, f"{p}.down", f"{p}.downbn", s, 0, act=False) if bi == 0 else h
+            h = relu(add(o, idn))
+    h = avgpool_fwd(h)
+    return linear_fwd(h, P["fc.w"], P["fc.b"])
+
+
+# ---------------------------------------------------------------------------- MobileNetV2
+MNV2_SETTINGS = [(1, 16, 1, 1), (6, 24, 2, 2), (6, 32, 3, 2), (6, 64, 4, 2), (6, 96, 3, 1),
+                 (6, 160, 3, 2), (6, 320, 1, 1)]   # torchvision (t, c, n, s)
+
+
+def mnv2_blocks(width_mult=1.0):
+    """Block list: (name, cin, hidden, cout, stride, expand, residual)."""
+    blocks = []
+    cin = 32
+    i = 1
+    for t, c, n, s in MNV2_SETTINGS:
+        for j in range(n):
+            stride = s if j == 0 else 1
+            hidden = cin * t
+            blocks.append((f"features.{i}", cin, hidden, c, stride, t != 1, stride == 1 and cin == c))
+            cin = c
+            i += 1
+    return blocks
+
+
+def mnv2_spec(num_classes=1000):
+    s = _conv_spec("features.0", 32, 3, 3) + _bn_spec("features.0.bn", 32, False)
+    for name, cin, hid, cout, stride, expand, res in mnv2_blocks():
+        if expand:
+            s += _conv_spec(f"{name}.expand", hid, 1, cin) + _bn_spec(f"{name}.expand_bn", hid, False)
+        s += _conv_spec(f"{name}.dw", hid, 3, 1) + _bn_spec(f"{name}.dw_bn", hid, False)
+        s += _conv_spec(f"{name}.project", cout, 1, hid) + _bn_spec(f"{name}.project_bn", cout, False)
+    s += _conv_spec("features.18", 1280, 1, 320) + _bn_spec("features.18.bn", 1280, False)
+    # torchvision MobileNetV2 classifier init: normal(0, 0.01), bias zeros
+    s += [("classifier.w", (num_classes, 1280), ("normal", 0.01)), ("classifier.b", (num_classes,), ("const", 0.0))]
+    return s
+
+
+def mnv2_trainable(spec):
+    """Names of the parameters SGD updates (BN running stats are buffers, not parameters)."""
+    return [n for n, _, _ in spec if not (n.endswith(".rmean") or n.endswith(".rvar"))]
+
+
+def mnv2_train_step(P, V, x, labels, first, lr=0.01, momentum=0.9, eps=1e-5, bn_momentum=0.1):
+    """One training iteration of torchvision MobileNetV2 (dropout p=0, reading R22) with
+    CE loss and SGD(momentum). P: params + BN running stats (dict of fp32 tensors);
+    V: momentum buffers (dict). Returns (loss, newP, newV, grads)."""
+    newP = dict(P)
+
+    def conv_bn(h, cname, bname, k, stride, groups, act):
+        z = conv2d_fwd(h, P[f"{cname}.w"], stride, k // 2, groups)
+        y, mean, invstd, rm, rv = bn_train_fwd(z, P[f"{bname}.gamma"], P[f"{bname}.beta"],
+                                               P[f"{bname}.rmean"], P[f"{bname}.rvar"], eps, bn_momentum)
+        newP[f"{bname}.rmean"], newP[f"{bname}.rvar"] = rm, rv
+        rec = (cname, bname, k, stride, groups, act, h, z, y, mean, invstd)
+        return (relu6(y) if act else y), rec
+
+    g = {}
+
+    def conv_bn_bwd(rec, dout, need_dx=True):
+        cname, bname, k, stride, groups, act, hin, z, y, mean, invstd = rec
+        dy = relu6_bwd(y, dout) if act else dout
+        dz, g[f"{bname}.gamma"], g[f"{bname}.beta"] = bn_bwd(z, dy, P[f"{bname}.gamma"], mean, invstd)
+        w = P[f"{cname}.w"]
+        g[f"{cname}.w"] = conv2d_bwd_weight(hin, dz, tuple(w.shape), stride, k // 2, groups)
+        return conv2d_bwd_data(dz, w, tuple(hin.shape), stride, k // 2, groups) if need_dx else None
+
+    # ---- forward
+    h, stem = conv_bn(x, "features.0", "features.0.bn", 3, 2, 1, True)
+    recs = []
+    for name, cin, hid, cout, stride, expand, res in mnv2_blocks():
+        inp = h
+        r = {}
+        if expand:
+            h, r["expand"] = conv_bn(h, f"{name}.expand", f"{name}.expand_bn", 1, 1, 1, True)
+        h, r["dw"] = conv_bn(h, f"{name}.dw", f"{name}.dw_bn", 3, stride, hid, True)
+        h, r["project"] = conv_bn(h, f"{name}.project", f"{name}.project_bn", 1, 1, 1, False)
+        if res:
+            h = add(h, inp)
+        recs.append((res, r))
+    h, last = conv_bn(h, "features.18", "features.18.bn", 1, 1, 1, True)
+    feat_shape = tuple(h.shape)
+    pooled = avgpool_fwd(h)
+    logits = linear_fwd(pooled, P["classifier.w"], P["classifier.b"])
+    loss, dlogits = ce_fwd_bwd(logits, labels)
+
+    # ---- backward (reverse op order)
+    dpooled, g["classifier.w"], g["classifier.b"] = linear_bwd(pooled, P["classifier.w"], dlogits)
+    dh = avgpool_bwd(dpooled, feat_shape)
+    dh = conv_bn_bwd(last, dh)
+    for res, r in reversed(recs):
+        d = conv_bn_bwd(r["project"], dh)
+        d = conv_bn_bwd(r["dw"], d)
+        if "expand" in r:
+            d = conv_bn_bwd(r["expand"], d)
+        dh = add(d, dh) if res else d
+    conv_bn_bwd(stem, dh, need_dx=False)
+
+    # ---- optimizer
+    newV = {}
+    for n in sorted(g):
+        newP[n], newV[n] = sgd(P[n], g[n], V.get(n), lr, momentum, first)
+    return loss, newP, newV, g
+
+
+# ------------------------------------------------------------------------- small helpers
+def count_flops_conv(n, ho, wo, cout, k, cin_g):
+    return 2 * n * ho * wo * cout * k * k * cin_g
+
+
+def out_hw(h, k, s, p):
+    return (h + 2 * p - k) // s + 1
+
+
+def logsumexp_uniform(c):
+    return math.log(c)
