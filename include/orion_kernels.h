@@ -1,0 +1,98 @@
+/*
+ * orion_kernels.h — the operator table of liborion: hand-written sm_100a kernels that an
+ * orion_op names through orion_op.fn (part of the C ABI, see orion.h).
+ *
+ * The paper's operators are cuDNN/cuBLAS/PyTorch kernels of TorchVision models run in fp32
+ * (P:888-899); here each is an explicit kernel with the PyTorch semantics written out in
+ * oracle/model.py. Layouts in HBM: activations NHWC fp32, conv weights OHWI fp32
+ * ([Cout][kh][kw][Cin/groups]), linear weights [out][in], labels int32. All pointers are device
+ * pointers owned by the caller (torch tensors) and must stay alive until the op completes.
+ *
+ * Every kernel is deterministic and independent of the SM partition it runs in (no float
+ * atomics, fixed reduction order, no SM-count-dependent tiling), so a client's outputs are
+ * bitwise identical solo and collocated.
+ *
+ * Arg layouts: args[i] as listed (u64; floats as their fp32 bit pattern in the low 32 bits).
+ */
+#ifndef ORION_KERNELS_H
+#define ORION_KERNELS_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum orion_fn {
+  /* C[M,N] = op(A) op(B) (+ bias[N]); row-major; op = transpose if flag set.
+     args: A, B, C, bias (0 = none), M, N, K, lda, ldb, ldc, flags (1 = A^T, 2 = B^T).
+     y = x W^T + b (Linear fwd) is flags=2; dx = dy W is flags=0; dW = dy^T x is flags=1. */
+  ORION_FN_GEMM = 0,
+  /* Column sum: out[n] = sum_m A[m, n]  (bias gradient). args: A, out, M, N */
+  ORION_FN_COLSUM = 1,
+  /* y = max(x, 0). args: x, y, n */
+  ORION_FN_RELU = 2,
+  /* dx = dy * (x > 0). args: x, dy, dx, n */
+  ORION_FN_RELU_BWD = 3,
+  /* y = min(max(x, 0), 6). args: x, y, n */
+  ORION_FN_RELU6 = 4,
+  /* dx = dy * (0 < x < 6). args: x, dy, dx, n */
+  ORION_FN_RELU6_BWD = 5,
+  /* c = a + b. args: a, b, c, n */
+  ORION_FN_ADD = 6,
+  /* MSE loss mean((y-t)^2) and dy = 2(y-t)/n. args: y, t, loss (1 float), dy, n */
+  ORION_FN_MSE = 7,
+  /* SGD with momentum (torch semantics, dampening 0): v = mu v + g; p -= lr v. With v
+     initialised to 0 the first step equals torch's v = g. mu = 0: p -= lr g (v unused).
+     args: p, g, v, n, lr_bits, mu_bits */
+  ORION_FN_SGD = 8,
+  /* Conv2d forward, implicit GEMM, groups = 1, no bias. args: x, w, y, N, H, W, C, K(=Cout),
+     R, S (kernel h, w), stride, pad, P, Q (out h, w) */
+  ORION_FN_CONV_FWD = 9,
+  /* Conv2d backward data: dx[N,H,W,C] from dy[N,P,Q,K], w. args: dy, w, dx, N,H,W,C,K,R,S,stride,pad,P,Q */
+  ORION_FN_CONV_DGRAD = 10,
+  /* Conv2d backward weight: dw[K,R,S,C] from x, dy. args: x, dy, dw, N,H,W,C,K,R,S,stride,pad,P,Q */
+  ORION_FN_CONV_WGRAD = 11,
+  /* Depthwise 3x3 conv (groups = C): args as CONV_* with K = C */
+  ORION_FN_DW_FWD = 12,
+  ORION_FN_DW_DGRAD = 13,
+  ORION_FN_DW_WGRAD = 14,
+  /* BN eval: y = (x - rm) * rsqrt(rv + eps) * gamma + beta. args: x, y, gamma, beta, rm, rv, rows, C, eps_bits */
+  ORION_FN_BN_EVAL = 15,
+  /* BN train statistics (batch mean, biased var) + running-stat update (momentum, unbiased var).
+     args: x, mean, invstd, rm, rv, rows, C, eps_bits, momentum_bits, workspace, ws_bytes */
+  ORION_FN_BN_STATS = 16,
+  /* BN train apply: y = (x - mean) * invstd * gamma + beta. args: x, y, gamma, beta, mean, invstd, rows, C */
+  ORION_FN_BN_APPLY = 17,
+  /* BN backward reduce: dgamma = sum dy*xhat, dbeta = sum dy. args: x, dy, mean, invstd, dgamma, dbeta,
+     rows, C, workspace, ws_bytes */
+  ORION_FN_BN_BWD_REDUCE = 18,
+  /* BN backward dx = gamma*invstd/N (N dy - dbeta - xhat dgamma). args: x, dy, dx, gamma, mean, invstd,
+     dgamma, dbeta, rows, C */
+  ORION_FN_BN_BWD_DX = 19,
+  /* MaxPool 3x3 stride 2 pad 1. args: x, y, N, H, W, C, P, Q */
+  ORION_FN_MAXPOOL = 20,
+  /* Global average pool [N,H,W,C] -> [N,C]. args: x, y, N, HW, C */
+  ORION_FN_AVGPOOL = 21,
+  /* Its backward: dx[n,hw,c] = dy[n,c] / HW. args: dy, dx, N, HW, C */
+  ORION_FN_AVGPOOL_BWD = 22,
+  /* Softmax cross entropy (mean over batch) and dz = (softmax - onehot)/B.
+     args: z, labels(int32), loss (1 float), dz, B, classes */
+  ORION_FN_CE = 23,
+  ORION_FN_COUNT = 24
+};
+
+/* Number of table entries, and a stable name for each (for profiles and logs). */
+int orion_kernel_count(void);
+const char* orion_kernel_name(uint32_t fn);
+/* Launch one operator directly on `cu_stream` (no scheduler; the "native" path, R20, and the
+   offline profiler's solo runner). */
+int orion_kernel_launch(uint32_t fn, const uint64_t* args, uint32_t nargs, void* cu_stream);
+/* Launch geometry of an operator as it would launch: total CTAs and the occupancy-limited
+   CTAs per SM (cudaOccupancyMaxActiveBlocksPerMultiprocessor), for sm_needed (R17). */
+int orion_kernel_geometry(uint32_t fn, const uint64_t* args, uint32_t nargs, uint64_t* grid_ctas,
+                          int32_t* blocks_per_sm, int32_t* threads_per_cta, int32_t* smem_bytes);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ORION_KERNELS_H */

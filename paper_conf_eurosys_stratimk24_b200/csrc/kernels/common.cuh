@@ -1,0 +1,103 @@
+// Shared device/host plumbing of the operator kernels (not of the oracle).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include "orion.h"
+#include "orion_kernels.h"
+
+// Completion signal fused into every kernel: the last CTA of a launch publishes `seq` (the
+// client's completed-op count) to a host-mapped counter, so the scheduler observes completion by a
+// plain load instead of a CUDA event query (P:778-786 uses cudaEventQuery).
+struct OrionSig {
+  unsigned long long* ticket;  // per-stream device counter of finished CTAs (monotone)
+  unsigned long long* done;    // host-mapped completion counter of the stream
+  unsigned long long target;   // ticket value reached when the last CTA of this launch finishes
+  unsigned long long seq;      // value to publish
+};
+
+__device__ __forceinline__ void orion_signal(const OrionSig& sig) {
+  if (sig.ticket == nullptr) return;  // direct launch (no scheduler)
+  __threadfence();                    // this thread's global writes visible GPU-wide
+  __syncthreads();
+  if (threadIdx.x == 0 && threadIdx.y == 0 && threadIdx.z == 0) {
+    unsigned long long t = atomicAdd(sig.ticket, 1ull) + 1ull;
+    if (t == sig.target) {
+      __threadfence_system();
+      asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(sig.done), "l"(sig.seq) : "memory");
+    }
+  }
+}
+
+// Launch geometry computed from the op's args (identical for geometry queries and launches).
+struct LaunchGeom {
+  dim3 grid{1, 1, 1}, block{1, 1, 1};
+  int smem = 0;
+  const void* func = nullptr;
+  unsigned long long ctas() const { return (unsigned long long)grid.x * grid.y * grid.z; }
+};
+
+typedef int (*geom_fn)(const uint64_t* a, LaunchGeom* g);
+typedef int (*launch_fn)(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
+
+struct KernelEntry {
+  const char* name;
+  int nargs;
+  geom_fn geom;
+  launch_fn launch;
+};
+
+__host__ __device__ __forceinline__ float u2f(uint64_t v) {
+  union { uint32_t u; float f; } c; c.u = (uint32_t)v; return c.f;
+}
+
+__host__ __device__ __forceinline__ uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+
+// Last-CTA-of-a-group detection for deterministic two-phase reductions: every CTA of the group
+// calls this after writing its partials; returns true in exactly one CTA (the last), which then
+// reduces the partials in a fixed order. The ticket is reset by the last CTA.
+__device__ __forceinline__ bool last_cta_of(unsigned int* ticket, unsigned int count) {
+  __shared__ unsigned int s_last;
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned int t = atomicAdd(ticket, 1u) + 1u;
+    s_last = (t == count);
+    if (t == count) *ticket = 0u;  // reset for the next launch (stream order serialises launches)
+  }
+  __syncthreads();
+  if (s_last) __threadfence();
+  return s_last != 0;
+}
+
+// Kernel table (table.cu)
+extern const KernelEntry g_kernels[ORION_FN_COUNT];
+int kernel_launch_sig(uint32_t fn, const uint64_t* args, uint32_t nargs, OrionSig sig, cudaStream_t s,
+                      unsigned long long* ctas_out);
+
+#define ENTRY_DECL(name) \
+  int name##_geom(const uint64_t* a, LaunchGeom* g); \
+  int name##_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
+ENTRY_DECL(gemm)
+ENTRY_DECL(colsum)
+ENTRY_DECL(relu)
+ENTRY_DECL(relu_bwd)
+ENTRY_DECL(relu6)
+ENTRY_DECL(relu6_bwd)
+ENTRY_DECL(add)
+ENTRY_DECL(mse)
+ENTRY_DECL(sgd)
+ENTRY_DECL(conv_fwd)
+ENTRY_DECL(conv_dgrad)
+ENTRY_DECL(conv_wgrad)
+ENTRY_DECL(dw_fwd)
+ENTRY_DECL(dw_dgrad)
+ENTRY_DECL(dw_wgrad)
+ENTRY_DECL(bn_eval)
+ENTRY_DECL(bn_stats)
+ENTRY_DECL(bn_apply)
+ENTRY_DECL(bn_bwd_reduce)
+ENTRY_DECL(bn_bwd_dx)
+ENTRY_DECL(maxpool)
+ENTRY_DECL(avgpool)
+ENTRY_DECL(avgpool_bwd)
+ENTRY_DECL(ce)
