@@ -1,0 +1,370 @@
+"""Orion-on-B200 benchmark (BASELINE.json metric: HP p99 latency vs dedicated; BE iters/s under
+collocation, 1-8 B200).
+
+Workload (default, BASELINE configs[1]): HP ResNet-50 inference batch 4 with Poisson arrivals at
+15 RPS (Table 3 inf-train ResNet50) + BE MobileNetV2 training batch 96 closed loop,
+fp32, synthetic seeded data. `--config toy` runs BASELINE configs[0].
+
+A "step" is one HP request interval: K steps = K Poisson HP requests while BE trains closed loop.
+`value` = BE iterations/s under collocation summed over ranks (inputs resident in HBM);
+HP p50/p99 collocated vs dedicated are reported beside it. Each rank is an independent Orion
+instance on its own GPU (replicas, no data-path collective): scaling "weak".
+
+--impl reference runs the CPU oracle (oracle/model.py) on the host cores on a bounded sample of
+the same workload (the reference arm of this tier; no GPU).
+"""
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0}
+FFMA_TFLOPS = 148 * 128 * 2 * 1.965e9 / 1e12   # fp32 FFMA peak at max SM clock
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured"
+    return PEAKS_FALLBACK, "fallback"
+
+
+# --------------------------------------------------------------------------------- workloads
+def build_config(name, rank):
+    from paper_conf_eurosys_stratimk24_b200 import workloads as W
+    from synth import inputs as si
+    if name == "toy":
+        P = si.make_params(W.mlp_spec())
+        n_in = 64
+        hp_inputs = [si.normal((1, 512), si.HP_SEED, sub=r) for r in range(n_in)]
+        hpg = W.mlp_infer_graph(P, batch=1)
+        xs = [si.normal((32, 512), si.BE_SEED, sub=i) for i in range(8)]
+        ts = [si.normal((32, 512), si.BE_SEED, sub=100 + i) for i in range(8)]
+        beg = W.mlp_train_graph(P, xs, ts)
+        return dict(hpg=hpg, beg=beg, hp_inputs=hp_inputs, rate=1000.0, be_inputs=xs,
+                    cfg={"workload": "toy: HP MLP 3x512 fp32 inference b1 + BE MLP training b32",
+                         "hp_model": "mlp3x512", "hp_batch": 1, "be_model": "mlp3x512", "be_batch": 32,
+                         "arrivals": "poisson 1000 rps"})
+    Prn = si.make_params(W.resnet_spec())
+    hp_inputs = [si.normal((4, 224, 224, 3), si.HP_SEED, sub=r) for r in range(16)]
+    hpg = W.resnet_infer_graph(Prn, batch=4)
+    Pmn = si.make_params(W.mnv2_spec())
+    xs = [si.normal((96, 224, 224, 3), si.BE_SEED, sub=i) for i in range(8)]
+    labels = [si.labels(96, 1000, si.BE_SEED, sub=i) for i in range(8)]
+    beg = W.mnv2_train_graph(Pmn, xs, labels)
+    return dict(hpg=hpg, beg=beg, hp_inputs=hp_inputs, rate=15.0, be_inputs=xs,
+                cfg={"workload": "HP ResNet-50 inference b4 (Poisson 15 rps) + BE MobileNetV2 training b96, 1 B200 per instance",
+                     "hp_model": "resnet50", "hp_batch": 4, "be_model": "mobilenet_v2", "be_batch": 96,
+                     "image": "224x224x3 NHWC fp32", "arrivals": "poisson 15 rps (PAPER Table 3)"})
+
+
+def with_be_h2d(graph, xs_host):
+    """E2E variant of the BE client: each iteration first copies its batch from pinned host memory
+    (H2D memop) and finally reads the loss back (D2H memop)."""
+    from paper_conf_eurosys_stratimk24_b200 import _lib as L
+    pinned = [x.contiguous().pin_memory() for x in xs_host]
+    loss_host = torch.zeros(len(graph.variants), dtype=torch.float32).pin_memory()
+    xbufs = [graph.bufs[f"x{i}"] for i in range(len(graph.variants))]
+    variants = []
+    for i, v in enumerate(graph.variants):
+        ops = [(L.OP_MEMCPY_H2D, [xbufs[i].data_ptr(), pinned[i].data_ptr(), pinned[i].numel() * 4], "h2d_batch")]
+        ops += list(v)
+        ops.append((L.OP_MEMCPY_D2H, [loss_host.data_ptr() + 4 * i, graph.loss.data_ptr(), 4], "d2h_loss"))
+        variants.append(ops)
+    return variants, pinned, loss_host, sum(p.numel() * 4 for p in pinned) / len(pinned)
+
+
+# ------------------------------------------------------------------------------------ clocks
+class ClockSampler:
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,power.draw,"
+                 "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+                 "--format=csv,noheader,nounits", "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.th = threading.Thread(target=self._read, daemon=True)
+            self.th.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], 0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in self.lines:
+            f = [x.strip() for x in l.split(",")]
+            if len(f) < 7:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = max(mx, float(f[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, f[3:7]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx or None, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# --------------------------------------------------------------------------------- CPU oracle
+def cpu_oracle_sample(cfg_name, budget_s=15.0):
+    """Time the oracle (as it stands) on the host cores on a bounded sample of the BE workload;
+    return it/s scaled to the full batch, the sample description and the cores used."""
+    from oracle import model as om
+    from synth import inputs as si
+    cores = torch.get_num_threads()
+    if cfg_name == "toy":
+        P = si.make_params(om.mlp_spec())
+        x, t = si.normal((32, 512), si.BE_SEED), si.normal((32, 512), si.BE_SEED, sub=100)
+        n, t0 = 0, time.time()
+        while time.time() - t0 < budget_s and n < 2000:
+            _, P, _ = om.mlp_train_step(P, x, t)
+            n += 1
+        dt = time.time() - t0
+        return n / dt, f"{n} full MLP b32 training iterations (fp64 oracle)", cores
+    P = si.make_params(om.mnv2_spec())
+    b = 2
+    x, lab = si.normal((b, 224, 224, 3), si.BE_SEED), si.labels(b, 1000, si.BE_SEED)
+    n, t0 = 0, time.time()
+    V = {}
+    while True:
+        _, P, V, _ = om.mnv2_train_step(P, V, x, lab, first=(n == 0))
+        n += 1
+        if time.time() - t0 > budget_s:
+            break
+    dt = time.time() - t0
+    return n / dt * b / 96.0, f"{n} MobileNetV2 training iterations at batch {b} (224x224, fp64 oracle), scaled x{b}/96 to batch 96", cores
+
+
+# ------------------------------------------------------------------------------------- main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=300, help="HP requests timed under collocation")
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="orion", choices=["orion", "reference"])
+    ap.add_argument("--config", default="rn50_mnv2", choices=["rn50_mnv2", "toy"])
+    ap.add_argument("--dur-ppm", type=int, default=25000)
+    ap.add_argument("--be-partition", type=int, default=0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--rate", type=float, default=0.0, help="override HP arrival rate (rps)")
+    args = ap.parse_args()
+
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    metric = "HP p99 latency vs dedicated; BE iters/s under collocation, 1-8 B200"
+
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        v, sample, cores = cpu_oracle_sample(args.config, budget_s=max(10.0, min(30.0, 2.0 * args.steps)))
+        _, _, cfgd = None, None, None
+        line = {"impl": "reference", "metric": metric, "value": v, "unit": "it/s", "n_gpus": args.gpus,
+                "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": "oracle (CPU, fp64) BE training iterations of the same config", "config": args.config},
+                "cpu_baseline": {"value": v, "unit": "it/s", "cores": cores, "kind": "oracle", "sample": sample},
+                "e2e": {"value": v, "unit": "it/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(line), flush=True)
+        return
+
+    import torch.distributed as dist
+    if world > 1:
+        dist.init_process_group("gloo")
+    torch.cuda.set_device(local)
+    from paper_conf_eurosys_stratimk24_b200 import collocate as C, profiler as PR, _lib as L
+    from paper_conf_eurosys_stratimk24_b200.profiler import op_work
+    from synth import inputs as si
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def allmax(x):
+        if world == 1:
+            return [x]
+        t = [None] * world
+        dist.all_gather_object(t, x)
+        return t
+
+    W_ = build_config(args.config, rank)
+    rate = args.rate or W_["rate"]
+    hpg, beg = W_["hpg"], W_["beg"]
+    # ---- offline profile: solo op durations, sm_needed, class
+    prof_hp, rows_hp = PR.build_profiles(hpg, 0, reps=5)
+    prof_be, rows_be = PR.build_profiles(beg, 10000, reps=5)
+    beg.params.reset()
+    hp = C.HPClient(hpg, W_["hp_inputs"], max(args.steps, 64), prof_hp, 0)
+    be = C.BEClient(beg, prof_be, 10000)
+    n_hp_k = sum(1 for o in hp.ops if o.kind == L.OP_KERNEL)
+    n_be_k = sum(1 for o in be.variants[0] if o.kind == L.OP_KERNEL)
+    sched_cpu = 2 + 4 * local if (os.cpu_count() or 1) >= 8 else -1
+
+    def session(**kw):
+        return C.run_session(sched_cpu=sched_cpu, device=local, **kw)
+
+    # ---- HP solo request latency -> DUR_THRESHOLD base (R9)
+    spaced = (np.arange(1, 41) * 20e6).astype(np.int64)
+    r0 = session(hp=hp, arrivals_ns=spaced)
+    lat0 = np.sort(r0["t_done"] - r0["t_arrival"])
+    hp_lat_ns = int(lat0[len(lat0) // 2])
+    # ---- warm-up (untimed)
+    if args.warmup:
+        session(hp=hp, be=be, arrivals_ns=si.poisson_arrivals_ns(rate, args.warmup, seed=99, gpu_index=rank),
+                hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm)
+    arrivals = si.poisson_arrivals_ns(rate, args.steps, gpu_index=rank)
+    # ---- dedicated HP (Ideal latency)
+    barrier()
+    rd = session(hp=hp, arrivals_ns=arrivals)
+    ded = C.latency_stats(rd)
+    # ---- dedicated BE throughput
+    beg.params.reset()
+    t0 = time.time()
+    rb = session(be=be, be_iters=3)
+    per_it = (time.time() - t0) / 3
+    n_it = int(max(5, min(200, 6.0 / max(per_it, 1e-6))))
+    rb = session(be=be, be_iters=n_it)
+    tb = rb["be_t_end"]
+    be_ded = (len(tb) - 1) / ((tb[-1] - tb[0]) / 1e9) if len(tb) > 1 else float("nan")
+    # ---- dominant BE kernel (largest share of solo time) for the roofline
+    shares = {}
+    for r in rows_be:
+        shares[r["kernel_id"]] = r["dur_ns"]
+    top_kid = max(shares, key=shares.get)
+    top_row = next(r for r in rows_be if r["kernel_id"] == top_kid)
+    # ---- collocated (timed region)
+    beg.params.reset()
+    barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        e0.record()
+        rc = session(hp=hp, be=be, arrivals_ns=arrivals, hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm,
+                     be_partition_sms=args.be_partition, trace_kernel_id=top_kid)
+        torch.cuda.synchronize()
+        e1.record()
+        torch.cuda.synchronize()
+    barrier()
+    win_ms = e0.elapsed_time(e1)
+    col = C.latency_stats(rc)
+    be_col, be_n = C.be_throughput(rc, rc["t0"], rc["t_hp_end"])
+    clocks = clk.summary()
+    # roofline of the dominant kernel from its live launches inside the timed region
+    tr = rc.get("trace_ms", [])
+    flops, nbytes = top_row["flops"], top_row["bytes"]
+    pk, pk_src = peaks()
+    if tr:
+        avg_s = float(np.mean(tr)) / 1e3
+        if top_row["cls"] == "M":
+            achieved, peak, unit, bound = nbytes / avg_s / 1e9, pk["hbm_gbs"], "GB/s", "hbm"
+        else:
+            achieved, peak, unit, bound = flops / avg_s / 1e12, FFMA_TFLOPS, "TFLOP/s", "alu"
+    else:
+        achieved, peak, unit, bound, avg_s = None, None, None, None, None
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get(top_row["label"])
+        except Exception:
+            traffic = None
+    # ---- e2e: BE inputs copied from pinned host each iteration (H2D) + loss read back (D2H)
+    e2e = None
+    if not args.no_e2e:
+        variants, pinned, loss_host, be_h2d = with_be_h2d(beg, W_["be_inputs"])
+        from paper_conf_eurosys_stratimk24_b200.workloads import Graph  # noqa: F401
+        be_e2e = C.BEClient.__new__(C.BEClient)
+        be_e2e.graph = beg
+        saved = beg.variants
+        beg.variants = variants
+        be_e2e.set_profiles(prof_be_e2e(prof_be, 10000), 10000)
+        beg.variants = saved
+        beg.ops = saved[0]
+        beg.params.reset()
+        barrier()
+        re2 = session(hp=hp, be=be_e2e, arrivals_ns=arrivals, hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm,
+                      be_partition_sms=args.be_partition)
+        e2e_its, e2e_n = C.be_throughput(re2, re2["t0"], re2["t_hp_end"])
+        hp_in = hp.inp[0].numel() * 4
+        hp_out = hp.out[0].numel() * 4
+        e2e = {"value": e2e_its, "unit": "it/s", "hp_p99_ms": C.latency_stats(re2)["p99_ns"] / 1e6,
+               "h2d_bytes_per_step": int(hp_in + be_h2d * e2e_n / max(args.steps, 1)),
+               "d2h_bytes_per_step": int(hp_out + 4 * e2e_n / max(args.steps, 1))}
+    # ---- aggregate over ranks
+    mine = dict(be_col=be_col, be_ded=be_ded, win_ms=win_ms, p99=col["p99_ns"], p50=col["p50_ns"], p99d=ded["p99_ns"],
+                p50d=ded["p50_ns"], e2e=(e2e or {}).get("value", 0.0), be_n=be_n)
+    allr = allmax(mine)
+    if rank != 0:
+        return
+    value = sum(r["be_col"] for r in allr)
+    cpu = None
+    if not args.no_cpu_baseline:
+        v, sample, cores = cpu_oracle_sample(args.config)
+        cpu = {"value": v, "unit": "it/s", "cores": cores, "kind": "oracle", "sample": sample}
+    ms_per_step = max(r["win_ms"] for r in allr) / args.steps
+    line = {
+        "metric": metric, "value": value, "unit": "it/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic (seeded; DESIGN.md §5)",
+        "config": dict(W_["cfg"], parallelism=f"replicas x{world} (independent Orion instance per GPU)",
+                       hp_rate_rps=rate, dur_threshold_pct=args.dur_ppm / 1e4, be_partition_sms=args.be_partition,
+                       l2="inputs > L2 (BE batch 57.8 MB x 8 staged; no flush)"),
+        "hp": {"p50_ms": col["p50_ns"] / 1e6, "p99_ms": col["p99_ns"] / 1e6, "dedicated_p50_ms": ded["p50_ns"] / 1e6,
+               "dedicated_p99_ms": ded["p99_ns"] / 1e6, "p99_vs_dedicated": col["p99_ns"] / ded["p99_ns"],
+               "p50_vs_dedicated": col["p50_ns"] / ded["p50_ns"], "solo_latency_ms": hp_lat_ns / 1e6,
+               "requests": col["n"], "per_rank_p99_ratio": [r["p99"] / r["p99d"] for r in allr]},
+        "be": {"collocated_its": value, "dedicated_its": sum(r["be_ded"] for r in allr),
+               "fraction_of_dedicated": value / max(sum(r["be_ded"] for r in allr), 1e-9),
+               "iterations_in_window": sum(r["be_n"] for r in allr)},
+        "target": {"hp_p99_ratio_max": 1.15, "be_fraction_min": 0.5},
+        "roofline": {"kernel": top_row["label"], "bound": bound, "achieved": achieved, "peak": peak, "unit": unit,
+                     "frac": (achieved / peak) if achieved and peak else None, "traffic": traffic,
+                     "launches": len(tr), "avg_launch_us": avg_s * 1e6 if avg_s else None,
+                     "algorithmic_bytes": nbytes, "algorithmic_flops": flops, "peak_source": pk_src},
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": int(args.steps * n_hp_k + sum(r["be_n"] for r in allr) // max(world, 1) * n_be_k),
+        "clocks": clocks,
+        "scheduler": rc["stats"],
+    }
+    print(json.dumps(line), flush=True)
+
+
+def prof_be_e2e(prof, base):
+    """Profiles of the e2e BE op list: one H2D memop prepended shifts kernel ids by one."""
+    return {k + 1: v for k, v in prof.items()}
+
+
+if __name__ == "__main__":
+    main()

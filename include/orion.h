@@ -95,7 +95,10 @@ typedef struct {
   int32_t sched_cpu;          /* core to pin the scheduler thread to; -1 = no pinning */
   uint64_t log_capacity;      /* records per section; 0 = logging off */
   uint32_t fake_time_scale_pct; /* FAKE backend: op duration = dur_ns * pct/100 (0 -> 100) */
-  uint32_t reserved[7];
+  uint32_t trace_kernel_id_plus1; /* CUDA backend: 0 = off; else record a CUDA event pair around every
+                                     launch of kernel_id (trace_kernel_id_plus1 - 1) on its own stream
+                                     (bench roofline: live launch durations, read by orion_trace_read) */
+  uint32_t reserved[6];
 } orion_config;
 
 /* Create an instance on `cuda_device` (ignored by the FAKE backend). Returns ORION_E_NODEV if the
@@ -128,6 +131,9 @@ int orion_read_log(orion_t h, void* buf, size_t cap, size_t* written);
 int orion_stats(orion_t h, uint64_t* out, uint32_t n);
 int orion_destroy(orion_t h);
 const char* orion_strerror(int code);
+/* After orion_stop: durations (ms) of the traced kernel's launches (trace_kernel_id_plus1), in
+ * launch order. *n = number available (up to 8192); copies min(*n, cap) into ms_out. */
+int orion_trace_read(orion_t h, float* ms_out, uint32_t cap, uint32_t* n);
 
 /* ---------------------------------------------------------------------------------------------
  * Native client drivers (the bench's clients; C++ loops so no Python sits on the hot path).

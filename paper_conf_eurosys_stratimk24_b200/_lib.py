@@ -39,7 +39,8 @@ class Config(ctypes.Structure):
                 ("dur_threshold_ppm", ctypes.c_uint32), ("be_partition_sms", ctypes.c_uint32),
                 ("hp_latency_ns", ctypes.c_uint64), ("flags", ctypes.c_uint32), ("queue_capacity", ctypes.c_uint32),
                 ("backend", ctypes.c_uint32), ("sched_cpu", ctypes.c_int32), ("log_capacity", ctypes.c_uint64),
-                ("fake_time_scale_pct", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 7)]
+                ("fake_time_scale_pct", ctypes.c_uint32), ("trace_kernel_id_plus1", ctypes.c_uint32),
+                ("reserved", ctypes.c_uint32 * 6)]
 
 
 assert ctypes.sizeof(Op) == 224 and ctypes.sizeof(Profile) == 24
@@ -65,6 +66,7 @@ _sig = {
                                             ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint64,
                                             ctypes.POINTER(ctypes.c_uint64)]),
     "orion_now_ns": (ctypes.c_int64, []),
+    "orion_trace_read": (ctypes.c_int, [_h, ctypes.POINTER(ctypes.c_float), ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint32)]),
     "orion_kernel_count": (ctypes.c_int, []),
     "orion_kernel_name": (ctypes.c_char_p, [ctypes.c_uint32]),
     "orion_kernel_launch": (ctypes.c_int, [ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint64), ctypes.c_uint32, ctypes.c_void_p]),

@@ -1,0 +1,122 @@
+"""Collocation sessions: one Orion instance, one HP client (open-loop inference requests) and BE
+clients (closed-loop training iterations), driven by liborion's native client drivers
+(orion_run_requests / orion_run_iterations) so no Python sits between the clients and the
+scheduler (P:1082-1085 notes Python client threads contend on the GIL).
+
+Dedicated runs (the "Ideal" baseline) use the same binary with the other client
+absent (R20).
+"""
+import ctypes
+import threading
+
+import numpy as np
+import torch
+
+from . import _lib as L
+from .runtime import Orion
+
+
+class HPClient:
+    """Inference client: graph with an H2D input memop first and a D2H output memop last."""
+
+    def __init__(self, graph, inputs_host, n_req, profiles=None, kid_base=0):
+        self.graph = graph
+        self.n_req = n_req
+        in_elems = graph.ops[0][1][2] // 4
+        out_elems = graph.ops[-1][1][2] // 4
+        self.inp = torch.empty((len(inputs_host), in_elems), dtype=torch.float32).pin_memory()
+        for i, x in enumerate(inputs_host):
+            self.inp[i].copy_(x.reshape(-1))
+        self.out = torch.zeros((n_req, out_elems), dtype=torch.float32).pin_memory()
+        self.set_profiles(profiles, kid_base)
+
+    def set_profiles(self, profiles, kid_base=0):
+        ops = self.graph.orion_ops(profiles, kid_base)
+        ops[0].args[1] = self.inp.data_ptr()      # H2D src: request r uses input r % in_cycle
+        ops[-1].args[0] = self.out.data_ptr()     # D2H dst: request r writes row r
+        self.ops = ops
+
+
+class BEClient:
+    """Training client: op-list variants (one per pre-staged batch), run closed loop."""
+
+    def __init__(self, graph, profiles=None, kid_base=0):
+        self.graph = graph
+        self.set_profiles(profiles, kid_base)
+
+    def set_profiles(self, profiles, kid_base=0):
+        self.variants = []
+        for v in self.graph.variants:
+            self.graph.ops = v
+            self.variants.append(self.graph.orion_ops(profiles, kid_base))
+        self.graph.ops = self.graph.variants[0]
+
+
+def run_session(hp=None, be=None, arrivals_ns=None, be_iters=0, log_capacity=0, hp_latency_ns=0,
+                dur_threshold_ppm=25000, sm_threshold=0, be_partition_sms=0, flags=0, sched_cpu=-1,
+                backend=L.BACKEND_CUDA, device=0, trace_kernel_id=None):
+    """Run one session. HP (if given) issues len(arrivals_ns) requests open loop; BE (if given) runs
+    closed loop until HP finishes (or be_iters iterations if HP is absent / be_iters > 0 and no HP).
+    Returns dict with HP arrival/completion ns, BE iteration end times, window, log bytes, stats."""
+    o = Orion(device=device, backend=backend, hp_latency_ns=hp_latency_ns, dur_threshold_ppm=dur_threshold_ppm,
+              sm_threshold=sm_threshold, be_partition_sms=be_partition_sms, flags=flags, sched_cpu=sched_cpu,
+              log_capacity=log_capacity, trace_kernel_id=trace_kernel_id)
+    hp_id = o.register_client(L.HP) if hp is not None else None
+    be_id = o.register_client(L.BE) if be is not None else None
+    torch.cuda.synchronize()
+    o.start()
+    res = {}
+    stop = ctypes.c_int32(0)
+    th = None
+    if be is not None:
+        max_iters = be_iters if (hp is None or be_iters) else 0
+
+        def be_main():
+            try:
+                res["be_t_end"] = o.run_iterations(be_id, be.variants, stop_flag=stop, max_iters=max_iters)
+            except Exception as e:  # surfaced below
+                res["be_err"] = e
+        th = threading.Thread(target=be_main)
+        res["t0"] = o_now = L.lib.orion_now_ns()
+        th.start()
+    else:
+        res["t0"] = o_now = L.lib.orion_now_ns()
+    if hp is not None:
+        ta, td = o.run_requests(hp_id, hp.ops, arrivals_ns, in_cycle=hp.inp.shape[0], out_cycle=hp.n_req)
+        res["t_arrival"], res["t_done"] = ta, td
+        res["t_hp_end"] = L.lib.orion_now_ns()
+        stop.value = 1
+    if th is not None:
+        th.join()
+        if "be_err" in res:
+            o.stop()
+            raise res["be_err"]
+    res["t1"] = L.lib.orion_now_ns()
+    o.stop()
+    res["stats"] = o.stats()
+    if trace_kernel_id is not None:
+        res["trace_ms"] = o.trace_read()
+    if log_capacity:
+        res["log"] = o.read_log()
+    o.destroy()
+    del o_now
+    return res
+
+
+def latency_stats(res):
+    lat = (res["t_done"] - res["t_arrival"]).astype(np.float64)
+    s = np.sort(lat)
+    n = len(s)
+
+    def pct(p):   # nearest rank (R19)
+        return float(s[max(0, int(np.ceil(p / 100.0 * n)) - 1)])
+    return dict(n=n, p50_ns=pct(50), p95_ns=pct(95), p99_ns=pct(99), mean_ns=float(lat.mean()))
+
+
+def be_throughput(res, t_from=None, t_to=None):
+    """BE iterations completed inside [t_from, t_to] per second (SURVEY §8(d) BE throughput)."""
+    t = res.get("be_t_end", np.zeros(0, dtype=np.int64))
+    t_from = res["t0"] if t_from is None else t_from
+    t_to = res["t1"] if t_to is None else t_to
+    n = int(((t >= t_from) & (t <= t_to)).sum())
+    return n / ((t_to - t_from) / 1e9), n

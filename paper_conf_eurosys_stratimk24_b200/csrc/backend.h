@@ -20,6 +20,8 @@ struct Backend {
   virtual uint64_t read_done(StreamHandle* s) = 0;  // plain load, no API call
   virtual void thread_init() {}                     // called on the scheduler thread
   virtual void finish() {}
+  // live per-kernel tracing (CUDA backend): durations in ms of traced launches, after finish()
+  virtual int trace_read(float* ms, uint32_t cap, uint32_t* n) { (void)ms; (void)cap; *n = 0; return 0; }
 };
 
 int make_backend(const orion_config& cfg, int device, std::unique_ptr<Backend>* out);

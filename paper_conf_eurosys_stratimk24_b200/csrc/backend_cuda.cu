@@ -9,6 +9,7 @@
 
 #include <cstring>
 #include <mutex>
+#include <vector>
 
 #include "backend.h"
 #include "kernels/common.cuh"
@@ -55,8 +56,14 @@ struct CudaBackend : Backend {
   Drv drv;
   unsigned long long* host_counters = nullptr;  // one 64-byte line per stream
   int next_counter = 0;
+  // live tracing of one kernel id: event pairs recorded on the launching stream
+  uint32_t trace_kid_p1 = 0;
+  static constexpr int kTraceCap = 8192;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> trace_ev;
+  int trace_n = 0;
 
   ~CudaBackend() override {
+    for (auto& e : trace_ev) { cudaEventDestroy(e.first); cudaEventDestroy(e.second); }
     if (host_counters) cudaFreeHost(host_counters);
   }
   uint32_t num_sms() override { return sms; }
@@ -85,6 +92,12 @@ struct CudaBackend : Backend {
     if (cudaHostAlloc((void**)&host_counters, 64 * 8 * 16, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)
       return ORION_E_CUDA;
     memset(host_counters, 0, 64 * 8 * 16);
+    trace_kid_p1 = cfg.trace_kernel_id_plus1;
+    if (trace_kid_p1) {
+      trace_ev.resize(kTraceCap);
+      for (auto& e : trace_ev)
+        if (cudaEventCreate(&e.first) != cudaSuccess || cudaEventCreate(&e.second) != cudaSuccess) return ORION_E_CUDA;
+    }
     return 0;
   }
 
@@ -141,8 +154,11 @@ struct CudaBackend : Backend {
     if (op.kind == ORION_OP_KERNEL) {
       OrionSig sig{s->ticket, s->done_dev, s->ticket_base, seq + 1};
       unsigned long long ctas = 0;
+      const bool tr = trace_kid_p1 && op.prof.kernel_id + 1 == trace_kid_p1 && trace_n < kTraceCap;
+      if (tr) cudaEventRecord(trace_ev[trace_n].first, s->stream);
       int r = kernel_launch_sig(op.fn, op.args, op.nargs, sig, s->stream, &ctas);
       if (r) return r;
+      if (tr) cudaEventRecord(trace_ev[trace_n++].second, s->stream);
       s->ticket_base += ctas;
       return 0;
     }
@@ -166,6 +182,16 @@ struct CudaBackend : Backend {
   void finish() override {
     cudaSetDevice(device);
     cudaDeviceSynchronize();
+  }
+
+  int trace_read(float* ms, uint32_t cap, uint32_t* n) override {
+    *n = (uint32_t)trace_n;
+    for (int i = 0; i < trace_n && (uint32_t)i < cap; i++) {
+      float t = 0.f;
+      if (cudaEventElapsedTime(&t, trace_ev[i].first, trace_ev[i].second) != cudaSuccess) return ORION_E_CUDA;
+      ms[i] = t;
+    }
+    return 0;
   }
 };
 

@@ -474,6 +474,12 @@ int orion_stats(orion_t h, uint64_t* out, uint32_t n) {
   return ORION_OK;
 }
 
+int orion_trace_read(orion_t h, float* ms_out, uint32_t cap, uint32_t* n) {
+  if (!h || !n) return ORION_E_INVAL;
+  if (h->state.load() == STARTED) return ORION_E_STATE;
+  return h->backend->trace_read(ms_out, ms_out ? cap : 0, n);
+}
+
 int orion_destroy(orion_t h) {
   if (!h) return ORION_E_INVAL;
   if (h->state.load() == STARTED) {

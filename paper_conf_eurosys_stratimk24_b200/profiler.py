@@ -1,0 +1,159 @@
+"""Offline workload profiler (§5.2), B200 edition.
+
+For every operator of a client's op list it produces the profile row Orion's policy consumes:
+  * dur_ns     — solo execution time, median of CUDA-event-timed solo launches;
+  * sm_needed  — ceil(num_blocks / blocks_per_sm) with blocks_per_sm the occupancy limit of the
+                 kernel as launched (reading R17);
+  * cls        — compute (C) / memory (M) / unknown (U) (reading R16): roofline first
+                 (algorithmic FLOPs / measured DRAM bytes vs the ridge of the pipe the kernel uses),
+                 else >60% compute or memory throughput from ncu, else unknown.
+ncu counters come from tools/profile/ncu_profile.py (run on the GPU box; CSV committed under
+profiles/). Without a capture the classifier falls back to the analytic roofline of the op
+(algorithmic bytes and FLOPs computed here from the op's shape), and says so in the row.
+"""
+import csv
+import math
+import os
+
+import torch
+
+from . import _lib as L
+from .runtime import kernel_launch, kernel_geometry
+
+# B200 peaks (MEASURED_PEAKS.json; FFMA peak derived: 148 SMs x 128 FMA x 2 x 1.965 GHz)
+HBM_GBS = 6554.2
+FFMA_TFLOPS = 148 * 128 * 2 * 1.965e9 / 1e12
+RIDGE_FFMA = FFMA_TFLOPS * 1e12 / (HBM_GBS * 1e9)   # flop per DRAM byte
+
+
+def op_work(fn, a):
+    """Algorithmic FLOPs and compulsory DRAM bytes of one op (each input read once, each output
+    written once; fp32). The per-op numbers DESIGN.md §7 tabulates."""
+    f = L.kernel_names()[fn] if isinstance(fn, int) else fn
+    if f == "gemm":
+        M, N, K = a[4], a[5], a[6]
+        return 2 * M * N * K, 4 * (M * K + K * N + M * N + (N if a[3] else 0))
+    if f in ("conv_fwd", "conv_dgrad", "conv_wgrad"):
+        n, h, w, c, k, r, s, st, pad, p, q = a[3:14]
+        return 2 * n * p * q * k * r * s * c, 4 * (n * h * w * c + k * r * s * c + n * p * q * k)
+    if f in ("dw_fwd", "dw_dgrad", "dw_wgrad"):
+        n, h, w, c, k, r, s, st, pad, p, q = a[3:14]
+        return 2 * n * p * q * c * 9, 4 * (n * h * w * c + 9 * c + n * p * q * c)
+    if f in ("relu", "relu6"):
+        return a[2], 8 * a[2]
+    if f in ("relu_bwd", "relu6_bwd", "add"):
+        return a[3], 12 * a[3]
+    if f == "bn_eval":
+        return 2 * a[6] * a[7], 8 * a[6] * a[7]
+    if f == "bn_stats":
+        return 3 * a[5] * a[6], 4 * a[5] * a[6]
+    if f == "bn_apply":
+        return 2 * a[6] * a[7], 8 * a[6] * a[7]
+    if f == "bn_bwd_reduce":
+        return 4 * a[6] * a[7], 8 * a[6] * a[7]
+    if f == "bn_bwd_dx":
+        return 6 * a[8] * a[9], 12 * a[8] * a[9]
+    if f == "maxpool":
+        n, h, w, c, p, q = a[2:8]
+        return 9 * n * p * q * c, 4 * (n * h * w * c + n * p * q * c)
+    if f == "avgpool":
+        return a[2] * a[3] * a[4], 4 * (a[2] * a[3] * a[4] + a[2] * a[4])
+    if f == "avgpool_bwd":
+        return a[2] * a[3] * a[4], 4 * (a[2] * a[3] * a[4] + a[2] * a[4])
+    if f == "ce":
+        return 5 * a[4] * a[5], 4 * 2 * a[4] * a[5]
+    if f == "mse":
+        return 3 * a[4], 12 * a[4]
+    if f == "sgd":
+        return 3 * a[3], (20 if a[5] else 12) * a[3]
+    if f == "colsum":
+        return a[2] * a[3], 4 * (a[2] * a[3] + a[3])
+    return 0, 0
+
+
+def classify(c_pct=None, m_pct=None, flops=0, dram_bytes=0, ridge=RIDGE_FFMA):
+    """R16. (1) roofline when defined: C iff arithmetic intensity >= ridge; (2) else >60% compute or
+    memory throughput (ncu's own threshold): C iff c >= m; (3) else unknown."""
+    if flops > 0 and dram_bytes > 0:
+        return L.CLS_C if flops / dram_bytes >= ridge else L.CLS_M
+    if c_pct is not None and m_pct is not None and (c_pct > 60 or m_pct > 60):
+        return L.CLS_C if c_pct >= m_pct else L.CLS_M
+    return L.CLS_U
+
+
+def sm_needed(fn, args, num_sms=148):
+    grid, bps, _, _ = kernel_geometry(fn, args)
+    return int(math.ceil(grid / max(bps, 1)))
+
+
+def time_ops(graph, reps=10, warmup=2, stream=None):
+    """Median solo duration (ns) of every kernel op in the graph, each timed alone with CUDA events
+    on the launching stream (per-kernel execution time)."""
+    s = stream or torch.cuda.Stream()
+    out = {}
+    kops = graph.kernel_ops()
+    with torch.cuda.stream(s):
+        for i, fn, args, lab in kops:          # warm everything once (first-touch, module load)
+            for _ in range(warmup):
+                kernel_launch(fn, args, s.cuda_stream)
+        torch.cuda.synchronize()
+        for i, fn, args, lab in kops:
+            ts = []
+            for _ in range(reps):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                kernel_launch(fn, args, s.cuda_stream)
+                e1.record(s)
+                e1.synchronize()
+                ts.append(e0.elapsed_time(e1) * 1e6)
+            ts.sort()
+            out[i] = int(ts[len(ts) // 2])
+    return out
+
+
+def load_ncu_csv(path):
+    """{kernel_id: (c_pct, m_pct, dram_bytes)} from tools/profile/ncu_profile.py's summary CSV."""
+    if not path or not os.path.exists(path):
+        return {}
+    rows = {}
+    with open(path) as f:
+        for r in csv.DictReader(f):
+            rows[int(r["kernel_id"])] = (float(r["sm_pct"]), float(r["mem_pct"]), float(r["dram_bytes"]))
+    return rows
+
+
+def build_profiles(graph, kid_base=0, reps=10, ncu_csv=None):
+    """Profile table {kernel_id: (cls, sm_needed, dur_ns)} + rows for the CSV."""
+    durs = time_ops(graph, reps=reps)
+    ncu = load_ncu_csv(ncu_csv)
+    table, rows = {}, []
+    for i, fn, args, lab in graph.kernel_ops():
+        kid = kid_base + i
+        flops, nbytes = op_work(fn, args)
+        if kid in ncu:
+            c, m, dram = ncu[kid]
+            cls = classify(c, m, flops, dram)
+            src = "ncu"
+        else:
+            c = m = None
+            cls = classify(None, None, flops, nbytes)
+            src = "analytic"
+        sm = sm_needed(fn, args)
+        table[kid] = (cls, sm, durs[i])
+        rows.append(dict(kernel_id=kid, label=lab, fn=fn, cls="UCM"[cls], sm_needed=sm, dur_ns=durs[i],
+                         flops=flops, bytes=nbytes, source=src))
+    return table, rows
+
+
+def write_profile_csv(path, rows):
+    os.makedirs(os.path.dirname(path) or ".", exist_ok=True)
+    with open(path, "w", newline="") as f:
+        w = csv.DictWriter(f, fieldnames=list(rows[0].keys()))
+        w.writeheader()
+        w.writerows(rows)
+
+
+def request_latency(run_once, n=100):
+    """Median solo HP request latency (R9): run_once() returns one request's latency ns."""
+    lats = sorted(run_once() for _ in range(n))
+    return lats[len(lats) // 2]

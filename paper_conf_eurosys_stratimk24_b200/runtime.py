@@ -41,12 +41,13 @@ class Orion:
 
     def __init__(self, device=0, backend=L.BACKEND_CUDA, num_sms=0, sm_threshold=0, dur_threshold_ppm=25000,
                  hp_latency_ns=0, be_partition_sms=0, flags=0, queue_capacity=4096, sched_cpu=-1, log_capacity=0,
-                 fake_time_scale_pct=100):
+                 fake_time_scale_pct=100, trace_kernel_id=None):
         cfg = Config()
         cfg.num_sms, cfg.sm_threshold, cfg.dur_threshold_ppm = num_sms, sm_threshold, dur_threshold_ppm
         cfg.be_partition_sms, cfg.hp_latency_ns, cfg.flags = be_partition_sms, hp_latency_ns, flags
         cfg.queue_capacity, cfg.backend, cfg.sched_cpu = queue_capacity, backend, sched_cpu
         cfg.log_capacity, cfg.fake_time_scale_pct = log_capacity, fake_time_scale_pct
+        cfg.trace_kernel_id_plus1 = 0 if trace_kernel_id is None else trace_kernel_id + 1
         self.h = ctypes.c_void_p()
         check(L.lib.orion_create(device, ctypes.byref(cfg), ctypes.byref(self.h)), "orion_create")
         self.started = False
@@ -101,6 +102,14 @@ class Orion:
         buf = ctypes.create_string_buffer(need.value)
         check(L.lib.orion_read_log(self.h, buf, need.value, ctypes.byref(need)), "orion_read_log")
         return buf.raw[:need.value]
+
+    def trace_read(self):
+        """Live durations (ms) of the traced kernel's launches (config trace_kernel_id)."""
+        n = ctypes.c_uint32()
+        check(L.lib.orion_trace_read(self.h, None, 0, ctypes.byref(n)), "orion_trace_read")
+        buf = (ctypes.c_float * max(n.value, 1))()
+        check(L.lib.orion_trace_read(self.h, buf, n.value, ctypes.byref(n)), "orion_trace_read")
+        return [buf[i] for i in range(n.value)]
 
     def stats(self):
         out = (ctypes.c_uint64 * 8)()

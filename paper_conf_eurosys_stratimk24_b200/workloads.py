@@ -1,0 +1,519 @@
+"""Op-stream builders for the paper's client workloads (BASELINE.json configs):
+toy MLP (config 1), ResNet-50 inference (config 2 HP) and MobileNetV2 training (config 2 BE).
+
+A workload is a static list of liborion operators (R15: the unique kernel ID is the op's position
+in the list) over device buffers that torch allocates once (PyTorch is only the allocator here;
+every op runs in liborion's kernels). Layouts: activations NHWC fp32, conv weights OHWI, linear
+[out, in], parameters/gradients/momentum in flat buffers so SGD is one launch.
+
+The builders are independent of oracle/model.py (they define the same TorchVision architectures
+separately; tests compare parameter specs and outputs).
+"""
+import math
+
+import torch
+
+from . import _lib as L
+from .runtime import make_op, f32bits
+
+F32 = torch.float32
+EPS_BITS = f32bits(1e-5)
+
+
+class Graph:
+    """A client's op list plus the device buffers it references."""
+
+    def __init__(self, name, device="cuda"):
+        self.name = name
+        self.device = device
+        self.ops = []          # (fn_name or kind, args, label)
+        self.bufs = {}
+        self.ws_bytes = 256
+        self._ws = None
+        self._ws_ops = []      # (op index, arg index of ws ptr, arg index of ws bytes)
+
+    # ---- buffers
+    def buf(self, name, shape, dtype=F32, zero=True):
+        t = torch.zeros(shape, dtype=dtype, device=self.device) if zero else torch.empty(shape, dtype=dtype, device=self.device)
+        self.bufs[name] = t
+        return t
+
+    def need_ws(self, nbytes):
+        self.ws_bytes = max(self.ws_bytes, int(nbytes))
+
+    # ---- ops
+    def k(self, fn, args, label, ws_at=None):
+        self.ops.append((fn, list(args), label))
+        if ws_at is not None:
+            self._ws_ops.append((len(self.ops) - 1, ws_at))
+        return len(self.ops) - 1
+
+    def memcpy(self, kind, dst, src, nbytes, label):
+        self.ops.append((kind, [dst, src, nbytes], label))
+
+    def finalize(self):
+        """Allocate the shared split/reduction workspace (ops of one client run in stream order, and
+        every kernel leaves its tickets zeroed, so one workspace serves all of them)."""
+        self._ws = torch.zeros(self.ws_bytes // 4 + 64, dtype=F32, device=self.device)
+        for i, at in self._ws_ops:
+            self.ops[i][1][at] = self._ws.data_ptr()
+            self.ops[i][1][at + 1] = self.ws_bytes
+        return self
+
+    def orion_ops(self, profiles=None, kid_base=0):
+        """liborion op records; profiles: {kernel_id: (cls, sm_needed, dur_ns)} (offline profile)."""
+        out = []
+        for i, (fn, args, label) in enumerate(self.ops):
+            kid = kid_base + i
+            cls, sm, dur = (profiles or {}).get(kid, (L.CLS_U, 0, 0))
+            if isinstance(fn, str):
+                out.append(make_op(fn, args, kernel_id=kid, cls=cls, sm_needed=sm, dur_ns=dur))
+            else:
+                out.append(make_op(0, args, kernel_id=kid, kind=fn))
+        return out
+
+    def labels(self):
+        return [lab for _, _, lab in self.ops]
+
+    def kernel_ops(self):
+        return [(i, fn, args, lab) for i, (fn, args, lab) in enumerate(self.ops) if isinstance(fn, str)]
+
+
+def _p(t):
+    return t.data_ptr()
+
+
+# ------------------------------------------------------------------------ generic layer helpers
+def gemm(g, A, B, C, bias, M, N, K, lda, ldb, ldc, flags, label):
+    ws = L.lib.orion_gemm_workspace_bytes(M, N, K) if not (M <= 8 and flags == 2) else 0
+    args = [_p(A), _p(B), _p(C), _p(bias) if bias is not None else 0, M, N, K, lda, ldb, ldc, flags, 0, 0]
+    if ws:
+        g.need_ws(ws)
+        return g.k("gemm", args, label, ws_at=11)
+    return g.k("gemm", args, label)
+
+
+def linear_fwd(g, x, w, b, y, label):
+    """y[B, out] = x[B, in] W^T + b (flags = B^T)."""
+    Bn, fin = x.shape
+    fout = w.shape[0]
+    return gemm(g, x, w, y, b, Bn, fout, fin, fin, fin, fout, 2, label)
+
+
+def conv_args(x, w, y, stride, pad):
+    n, h, wd, c = x.shape
+    k, r, s, _ = w.shape
+    p, q = y.shape[1], y.shape[2]
+    return [n, h, wd, c, k, r, s, stride, pad, p, q]
+
+
+def conv_fwd(g, x, w, y, stride, pad, label, depthwise=False):
+    n, h, wd, c = x.shape
+    k, r, s, cg = w.shape
+    if depthwise:
+        return g.k("dw_fwd", [_p(x), _p(w), _p(y)] + conv_args(x, w, y, stride, pad), label)
+    if r == 1 and s == 1 and stride == 1 and pad == 0:   # 1x1 conv = GEMM [NHW, C] x [K, C]^T
+        return gemm(g, x, w, y, None, n * h * wd, k, c, c, c, k, 2, label)
+    return g.k("conv_fwd", [_p(x), _p(w), _p(y)] + conv_args(x, w, y, stride, pad), label)
+
+
+def conv_dgrad(g, dy, w, dx, stride, pad, label, depthwise=False):
+    n, h, wd, c = dx.shape
+    k, r, s, _ = w.shape
+    if depthwise:
+        return g.k("dw_dgrad", [_p(dy), _p(w), _p(dx)] + conv_args(dx, w, dy, stride, pad), label)
+    if r == 1 and s == 1 and stride == 1 and pad == 0:   # dx[NHW, C] = dy[NHW, K] W[K, C]
+        return gemm(g, dy, w, dx, None, n * h * wd, c, k, k, c, c, 0, label)
+    return g.k("conv_dgrad", [_p(dy), _p(w), _p(dx)] + conv_args(dx, w, dy, stride, pad), label)
+
+
+def conv_wgrad(g, x, dy, dw, stride, pad, label, depthwise=False):
+    n, h, wd, c = x.shape
+    k, r, s, _ = dw.shape
+    p, q = dy.shape[1], dy.shape[2]
+    if depthwise:
+        g.need_ws(L.lib.orion_dw_wgrad_workspace_bytes(n, c, p, q))
+        return g.k("dw_wgrad", [_p(x), _p(dy), _p(dw)] + conv_args(x, dw, dy, stride, pad) + [0, 0], label, ws_at=14)
+    if r == 1 and s == 1 and stride == 1 and pad == 0:   # dW[K, C] = dy^T[K, NHW] x[NHW, C]
+        return gemm(g, dy, x, dw, None, k, c, n * h * wd, k, c, c, 1, label)
+    g.need_ws(L.lib.orion_gemm_workspace_bytes(k, r * s * c, n * p * q))
+    return g.k("conv_wgrad", [_p(x), _p(dy), _p(dw)] + conv_args(x, dw, dy, stride, pad) + [0, 0], label, ws_at=14)
+
+
+# ============================================================================ toy MLP (config 1)
+def mlp_spec(width=512, layers=3):
+    spec = []
+    for i in range(layers):
+        spec.append((f"fc{i}.w", (width, width), ("uniform_fan_in", width)))
+        spec.append((f"fc{i}.b", (width,), ("uniform_fan_in", width)))
+    return spec
+
+
+class FlatParams:
+    """Parameters (and their gradients / momentum) as views of flat device buffers."""
+
+    def __init__(self, g, spec, host_params, trainable=None, grads=True, momentum=False):
+        names = [n for n, _, _ in spec if trainable is None or n in trainable]
+        self.spec = {n: s for n, s, _ in spec}
+        total = sum(math.prod(self.spec[n]) for n in names)
+        self.flat = g.buf("params.flat", (max(total, 1),))
+        self.gflat = g.buf("grads.flat", (max(total, 1),)) if grads else None
+        self.vflat = g.buf("momentum.flat", (max(total, 1),)) if momentum else None
+        self.total = total
+        self.p, self.g = {}, {}
+        off = 0
+        for n in names:
+            sz = math.prod(self.spec[n])
+            self.p[n] = self.flat[off:off + sz].view(self.spec[n])
+            if grads:
+                self.g[n] = self.gflat[off:off + sz].view(self.spec[n])
+            off += sz
+        for n, s, _ in spec:         # non-trainable tensors (BN running stats)
+            if n not in self.p:
+                self.p[n] = g.buf(n, s)
+        self.host = host_params
+        self.reset()
+
+    def reset(self):
+        """Restore the initial parameters / running stats and zero gradients and momentum."""
+        with torch.no_grad():
+            for n in self.p:
+                self.p[n].copy_(self.host[n].to(self.p[n].device))
+            if self.gflat is not None:
+                self.gflat.zero_()
+            if self.vflat is not None:
+                self.vflat.zero_()
+
+
+def mlp_infer_graph(host_params, batch=1, width=512, layers=3, device="cuda"):
+    """HP: Linear-ReLU-Linear-ReLU-Linear inference with H2D input and D2H output memops."""
+    g = Graph("mlp_infer", device)
+    P = FlatParams(g, mlp_spec(width, layers), host_params, grads=False)
+    x = g.buf("x", (batch, width))
+    g.memcpy(L.OP_MEMCPY_H2D, _p(x), 0, x.numel() * 4, "h2d_input")
+    h = x
+    for i in range(layers):
+        z = g.buf(f"z{i}", (batch, width))
+        linear_fwd(g, h, P.p[f"fc{i}.w"], P.p[f"fc{i}.b"], z, f"fc{i}")
+        h = z
+        if i < layers - 1:
+            a = g.buf(f"a{i}", (batch, width))
+            g.k("relu", [_p(z), _p(a), z.numel()], f"relu{i}")
+            h = a
+    g.out = h
+    g.memcpy(L.OP_MEMCPY_D2H, 0, _p(h), h.numel() * 4, "d2h_output")
+    g.params = P
+    return g.finalize()
+
+
+def mlp_train_graph(host_params, xs, ts, lr=0.01, width=512, layers=3, device="cuda"):
+    """BE: MLP training step (MSE loss, SGD momentum 0), one op-list variant per pre-staged batch.
+    Returns (graph, variants) where variants[i] are the op lists for batch i."""
+    g = Graph("mlp_train", device)
+    P = FlatParams(g, mlp_spec(width, layers), host_params, grads=True, momentum=False)
+    batch = xs[0].shape[0]
+    xb = [g.buf(f"x{i}", tuple(x.shape)) for i, x in enumerate(xs)]
+    tb = [g.buf(f"t{i}", tuple(t.shape)) for i, t in enumerate(ts)]
+    with torch.no_grad():
+        for d, s in zip(xb + tb, list(xs) + list(ts)):
+            d.copy_(s.to(d.device))
+    loss = g.buf("loss", (1,))
+    z = [g.buf(f"z{i}", (batch, width)) for i in range(layers)]
+    a = [g.buf(f"a{i}", (batch, width)) for i in range(layers - 1)]
+    dz = [g.buf(f"dz{i}", (batch, width)) for i in range(layers)]
+    da = [g.buf(f"da{i}", (batch, width)) for i in range(layers - 1)]
+    g.need_ws(256 + 8 * 148 * 8)
+    variants = []
+    for vi in range(len(xs)):
+        g.ops = []
+        g._ws_ops = []
+        x, t = xb[vi], tb[vi]
+        h = x
+        for i in range(layers):
+            linear_fwd(g, h, P.p[f"fc{i}.w"], P.p[f"fc{i}.b"], z[i], f"fc{i}")
+            h = z[i]
+            if i < layers - 1:
+                g.k("relu", [_p(z[i]), _p(a[i]), z[i].numel()], f"relu{i}")
+                h = a[i]
+        g.k("mse", [_p(z[-1]), _p(t), _p(loss), _p(dz[-1]), z[-1].numel(), 0, 0], "mse", ws_at=5)
+        for i in reversed(range(layers)):
+            inp = x if i == 0 else a[i - 1]
+            w = P.p[f"fc{i}.w"]
+            # dW = dz^T inp ; db = colsum(dz) ; d(inp) = dz W
+            gemm(g, dz[i], inp, P.g[f"fc{i}.w"], None, width, width, batch, width, width, width, 1, f"fc{i}.wgrad")
+            g.k("colsum", [_p(dz[i]), _p(P.g[f"fc{i}.b"]), batch, width], f"fc{i}.bgrad")
+            if i > 0:
+                gemm(g, dz[i], w, da[i - 1], None, batch, width, width, width, width, width, 0, f"fc{i}.dgrad")
+                g.k("relu_bwd", [_p(z[i - 1]), _p(da[i - 1]), _p(dz[i - 1]), z[i - 1].numel()], f"relu{i - 1}.bwd")
+        g.k("sgd", [_p(P.flat), _p(P.gflat), 0, P.total, f32bits(lr), f32bits(0.0)], "sgd")
+        variants.append((g.ops, g._ws_ops))
+    g.variants = []
+    for ops, wso in variants:
+        g.ops, g._ws_ops = ops, wso
+        g.finalize()
+        g.variants.append(list(g.ops))
+    g.ops = g.variants[0]
+    g.loss = loss
+    g.params = P
+    return g
+
+
+# ====================================================================== ResNet-50 inference (HP)
+RESNET50_LAYERS = [(64, 3, 1), (128, 4, 2), (256, 6, 2), (512, 3, 2)]
+
+
+def resnet_spec(layers=RESNET50_LAYERS, num_classes=1000):
+    def bn(name, c):
+        return [(f"{name}.gamma", (c,), ("const", 1.0)), (f"{name}.beta", (c,), ("const", 0.0)),
+                (f"{name}.rmean", (c,), ("normal", 0.1)), (f"{name}.rvar", (c,), ("uniform", 0.5, 1.5))]
+
+    def conv(name, cout, k, cin):
+        return [(f"{name}.w", (cout, k, k, cin), ("kaiming_fan_out", cout * k * k))]
+    s = conv("conv1", 64, 7, 3) + bn("bn1", 64)
+    cin = 64
+    for li, (w, nb, stride) in enumerate(layers):
+        for bi in range(nb):
+            p = f"layer{li + 1}.{bi}"
+            s += conv(f"{p}.conv1", w, 1, cin) + bn(f"{p}.bn1", w)
+            s += conv(f"{p}.conv2", w, 3, w) + bn(f"{p}.bn2", w)
+            s += conv(f"{p}.conv3", 4 * w, 1, w) + bn(f"{p}.bn3", 4 * w)
+            if bi == 0:
+                s += conv(f"{p}.down", 4 * w, 1, cin) + bn(f"{p}.downbn", 4 * w)
+            cin = 4 * w
+    s += [("fc.w", (num_classes, cin), ("uniform_fan_in", cin)), ("fc.b", (num_classes,), ("uniform_fan_in", cin))]
+    return s
+
+
+def resnet_infer_graph(host_params, batch=4, hw=224, layers=RESNET50_LAYERS, num_classes=1000, device="cuda"):
+    """HP: TorchVision ResNet v1.5 inference, eval BN, unfused ops (conv, BN, ReLU, add each a kernel,
+    as PyTorch eager dispatches them: P:888-899), H2D input and D2H logits."""
+    g = Graph("resnet_infer", device)
+    spec = resnet_spec(layers, num_classes)
+    P = FlatParams(g, spec, host_params, grads=False)
+    x = g.buf("x", (batch, hw, hw, 3))
+    g.memcpy(L.OP_MEMCPY_H2D, _p(x), 0, x.numel() * 4, "h2d_input")
+    cnt = [0]
+
+    def new(shape):
+        cnt[0] += 1
+        return g.buf(f"t{cnt[0]}", shape)
+
+    def cbr(h, name, bn, stride, pad, act=True):
+        w = P.p[f"{name}.w"]
+        n, hh, ww, _ = h.shape
+        k = w.shape[1]
+        ho, wo = (hh + 2 * pad - k) // stride + 1, (ww + 2 * pad - k) // stride + 1
+        z = new((n, ho, wo, w.shape[0]))
+        conv_fwd(g, h, w, z, stride, pad, name)
+        y = new(z.shape)
+        g.k("bn_eval", [_p(z), _p(y), _p(P.p[f"{bn}.gamma"]), _p(P.p[f"{bn}.beta"]), _p(P.p[f"{bn}.rmean"]),
+                        _p(P.p[f"{bn}.rvar"]), n * ho * wo, w.shape[0], EPS_BITS], bn)
+        if not act:
+            return y
+        a = new(y.shape)
+        g.k("relu", [_p(y), _p(a), y.numel()], f"{bn}.relu")
+        return a
+
+    h = cbr(x, "conv1", "bn1", 2, 3)
+    n, hh, ww, c = h.shape
+    pq = (hh + 2 - 3) // 2 + 1
+    m = new((n, pq, pq, c))
+    g.k("maxpool", [_p(h), _p(m), n, hh, ww, c, pq, pq], "maxpool")
+    h = m
+    for li, (w, nb, stride) in enumerate(layers):
+        for bi in range(nb):
+            p = f"layer{li + 1}.{bi}"
+            s = stride if bi == 0 else 1
+            o = cbr(h, f"{p}.conv1", f"{p}.bn1", 1, 0)
+            o = cbr(o, f"{p}.conv2", f"{p}.bn2", s, 1)
+            o = cbr(o, f"{p}.conv3", f"{p}.bn3", 1, 0, act=False)
+            idn = cbr(h, f"{p}.down", f"{p}.downbn", s, 0, act=False) if bi == 0 else h
+            sm = new(o.shape)
+            g.k("add", [_p(o), _p(idn), _p(sm), o.numel()], f"{p}.add")
+            r = new(o.shape)
+            g.k("relu", [_p(sm), _p(r), sm.numel()], f"{p}.relu")
+            h = r
+    n, hh, ww, c = h.shape
+    pooled = new((n, c))
+    g.k("avgpool", [_p(h), _p(pooled), n, hh * ww, c], "avgpool")
+    logits = new((n, num_classes))
+    linear_fwd(g, pooled, P.p["fc.w"], P.p["fc.b"], logits, "fc")
+    g.memcpy(L.OP_MEMCPY_D2H, 0, _p(logits), logits.numel() * 4, "d2h_logits")
+    g.out = logits
+    g.x = x
+    g.params = P
+    return g.finalize()
+
+
+# ================================================================= MobileNetV2 training (BE)
+MNV2_SETTINGS = [(1, 16, 1, 1), (6, 24, 2, 2), (6, 32, 3, 2), (6, 64, 4, 2), (6, 96, 3, 1), (6, 160, 3, 2), (6, 320, 1, 1)]
+
+
+def mnv2_blocks():
+    blocks, cin, i = [], 32, 1
+    for t, c, n, s in MNV2_SETTINGS:
+        for j in range(n):
+            stride = s if j == 0 else 1
+            blocks.append((f"features.{i}", cin, cin * t, c, stride, t != 1, stride == 1 and cin == c))
+            cin = c
+            i += 1
+    return blocks
+
+
+def mnv2_spec(num_classes=1000):
+    def bn(name, c):
+        return [(f"{name}.gamma", (c,), ("const", 1.0)), (f"{name}.beta", (c,), ("const", 0.0)),
+                (f"{name}.rmean", (c,), ("const", 0.0)), (f"{name}.rvar", (c,), ("const", 1.0))]
+
+    def conv(name, cout, k, cin):
+        return [(f"{name}.w", (cout, k, k, cin), ("kaiming_fan_out", cout * k * k))]
+    s = conv("features.0", 32, 3, 3) + bn("features.0.bn", 32)
+    for name, cin, hid, cout, stride, expand, res in mnv2_blocks():
+        if expand:
+            s += conv(f"{name}.expand", hid, 1, cin) + bn(f"{name}.expand_bn", hid)
+        s += conv(f"{name}.dw", hid, 3, 1) + bn(f"{name}.dw_bn", hid)
+        s += conv(f"{name}.project", cout, 1, hid) + bn(f"{name}.project_bn", cout)
+    s += conv("features.18", 1280, 1, 320) + bn("features.18.bn", 1280)
+    s += [("classifier.w", (num_classes, 1280), ("normal", 0.01)), ("classifier.b", (num_classes,), ("const", 0.0))]
+    return s
+
+
+def mnv2_train_graph(host_params, xs, labels, lr=0.01, momentum=0.9, num_classes=1000, device="cuda"):
+    """BE: one MobileNetV2 training iteration (train-mode BN, ReLU6, CE, SGD momentum), dropout p=0
+    (reading R22). One op-list variant per pre-staged batch (8 batches cycled)."""
+    g = Graph("mnv2_train", device)
+    spec = mnv2_spec(num_classes)
+    trainable = {n for n, _, _ in spec if not n.endswith((".rmean", ".rvar"))}
+    P = FlatParams(g, spec, host_params, trainable=trainable, grads=True, momentum=True)
+    batch, hw = xs[0].shape[0], xs[0].shape[1]
+    xb = [g.buf(f"x{i}", tuple(x.shape)) for i, x in enumerate(xs)]
+    lb = [g.buf(f"lab{i}", (batch,), dtype=torch.int32) for i in range(len(xs))]
+    with torch.no_grad():
+        for d, s in zip(xb, xs):
+            d.copy_(s.to(d.device))
+        for d, s in zip(lb, labels):
+            d.copy_(s.to(d.device))
+    loss = g.buf("loss", (1,))
+    cnt = [0]
+
+    def new(shape):
+        cnt[0] += 1
+        return g.buf(f"t{cnt[0]}", shape)
+
+    # ---- allocate activations / gradient buffers once (shared by all variants)
+    layers = []   # (cname, bname, k, stride, depthwise, act, in_shape, out_shape)
+
+    def plan(cname, bname, cin_shape, cout, k, stride, dw, act):
+        n, h, w, c = cin_shape
+        pad = k // 2
+        ho, wo = (h + 2 * pad - k) // stride + 1, (w + 2 * pad - k) // stride + 1
+        L_ = dict(cname=cname, bname=bname, k=k, stride=stride, pad=pad, dw=dw, act=act, cout=cout, in_shape=cin_shape,
+                  z=new((n, ho, wo, cout)), y=new((n, ho, wo, cout)),
+                  mean=new((cout,)), invstd=new((cout,)),
+                  a=new((n, ho, wo, cout)) if act else None,
+                  dy=new((n, ho, wo, cout)) if act else None, dz=new((n, ho, wo, cout)))
+        layers.append(L_)
+        return (n, ho, wo, cout)
+
+    shape = plan("features.0", "features.0.bn", (batch, hw, hw, 3), 32, 3, 2, False, True)
+    blocks = []
+    for name, cin, hid, cout, stride, expand, res in mnv2_blocks():
+        first = len(layers)
+        in_shape = shape
+        if expand:
+            shape = plan(f"{name}.expand", f"{name}.expand_bn", shape, hid, 1, 1, False, True)
+        shape = plan(f"{name}.dw", f"{name}.dw_bn", shape, hid, 3, stride, True, True)
+        shape = plan(f"{name}.project", f"{name}.project_bn", shape, cout, 1, 1, False, False)
+        blk = dict(first=first, last=len(layers) - 1, res=res, out=new(shape) if res else None,
+                   in_shape=in_shape, dres=new(in_shape) if res else None)
+        blocks.append(blk)
+    shape = plan("features.18", "features.18.bn", shape, 1280, 1, 1, False, True)
+    gin = [new(b["in_shape"]) for b in blocks] + [new(layers[-1]["in_shape"])]
+    dtmp = {li: new(layers[li]["in_shape"]) for b in blocks for li in range(b["first"] + 1, b["last"] + 1)}
+    n, hh, ww, c = shape
+    pooled, logits, dlogits, dpooled, dfeat = new((n, c)), new((n, num_classes)), new((n, num_classes)), new((n, c)), new(shape)
+    for L_ in layers:
+        g.need_ws(L.lib.orion_bn_workspace_bytes(L_["z"].shape[0] * L_["z"].shape[1] * L_["z"].shape[2], L_["cout"]))
+    g.need_ws(256 + 4 * batch)
+
+    def conv_bn_fwd(L_, h):
+        w = P.p[f"{L_['cname']}.w"]
+        conv_fwd(g, h, w, L_["z"], L_["stride"], L_["pad"], L_["cname"], depthwise=L_["dw"])
+        rows = L_["z"].numel() // L_["cout"]
+        b = L_["bname"]
+        g.k("bn_stats", [_p(L_["z"]), _p(L_["mean"]), _p(L_["invstd"]), _p(P.p[f"{b}.rmean"]), _p(P.p[f"{b}.rvar"]),
+                         rows, L_["cout"], EPS_BITS, f32bits(0.1), 0, 0], f"{b}.stats", ws_at=9)
+        g.k("bn_apply", [_p(L_["z"]), _p(L_["y"]), _p(P.p[f"{b}.gamma"]), _p(P.p[f"{b}.beta"]), _p(L_["mean"]),
+                         _p(L_["invstd"]), rows, L_["cout"]], f"{b}.apply")
+        L_["in"] = h
+        if L_["act"]:
+            g.k("relu6", [_p(L_["y"]), _p(L_["a"]), L_["y"].numel()], f"{b}.relu6")
+            return L_["a"]
+        return L_["y"]
+
+    def conv_bn_bwd(L_, dout, dx):
+        b = L_["bname"]
+        rows = L_["z"].numel() // L_["cout"]
+        dy = dout
+        if L_["act"]:
+            g.k("relu6_bwd", [_p(L_["y"]), _p(dout), _p(L_["dy"]), dout.numel()], f"{b}.relu6_bwd")
+            dy = L_["dy"]
+        g.k("bn_bwd_reduce", [_p(L_["z"]), _p(dy), _p(L_["mean"]), _p(L_["invstd"]), _p(P.g[f"{b}.gamma"]),
+                              _p(P.g[f"{b}.beta"]), rows, L_["cout"], 0, 0], f"{b}.bwd_reduce", ws_at=8)
+        g.k("bn_bwd_dx", [_p(L_["z"]), _p(dy), _p(L_["dz"]), _p(P.p[f"{b}.gamma"]), _p(L_["mean"]), _p(L_["invstd"]),
+                          _p(P.g[f"{b}.gamma"]), _p(P.g[f"{b}.beta"]), rows, L_["cout"]], f"{b}.bwd_dx")
+        w = P.p[f"{L_['cname']}.w"]
+        conv_wgrad(g, L_["in"], L_["dz"], P.g[f"{L_['cname']}.w"], L_["stride"], L_["pad"], f"{L_['cname']}.wgrad",
+                   depthwise=L_["dw"])
+        if dx is not None:
+            conv_dgrad(g, L_["dz"], w, dx, L_["stride"], L_["pad"], f"{L_['cname']}.dgrad", depthwise=L_["dw"])
+
+    variants, ws_ops = [], None
+    for vi in range(len(xs)):
+        g.ops, g._ws_ops = [], []
+        h = conv_bn_fwd(layers[0], xb[vi])
+        for blk in blocks:
+            inp = h
+            for li in range(blk["first"], blk["last"] + 1):
+                h = conv_bn_fwd(layers[li], h)
+            if blk["res"]:
+                g.k("add", [_p(h), _p(inp), _p(blk["out"]), h.numel()], f"block{blk['first']}.add")
+                h = blk["out"]
+        h = conv_bn_fwd(layers[-1], h)
+        g.k("avgpool", [_p(h), _p(pooled), n, hh * ww, c], "avgpool")
+        linear_fwd(g, pooled, P.p["classifier.w"], P.p["classifier.b"], logits, "classifier")
+        g.k("ce", [_p(logits), _p(lb[vi]), _p(loss), _p(dlogits), n, num_classes, 0, 0], "ce", ws_at=6)
+        gemm(g, dlogits, pooled, P.g["classifier.w"], None, num_classes, c, n, num_classes, c, c, 1, "classifier.wgrad")
+        g.k("colsum", [_p(dlogits), _p(P.g["classifier.b"]), n, num_classes], "classifier.bgrad")
+        gemm(g, dlogits, P.p["classifier.w"], dpooled, None, n, c, num_classes, num_classes, c, c, 0, "classifier.dgrad")
+        g.k("avgpool_bwd", [_p(dpooled), _p(dfeat), n, hh * ww, c], "avgpool_bwd")
+        # gin[b] = gradient w.r.t. the input of block b; gin[len(blocks)] = w.r.t. features.18's input
+        conv_bn_bwd(layers[-1], dfeat, gin[len(blocks)])
+        for bi in reversed(range(len(blocks))):
+            blk = blocks[bi]
+            dout = gin[bi + 1]
+            dd = dout
+            for li in range(blk["last"], blk["first"] - 1, -1):
+                if li == blk["first"]:
+                    out = blk["dres"] if blk["res"] else gin[bi]
+                else:
+                    out = dtmp[li]
+                conv_bn_bwd(layers[li], dd, out)
+                dd = out
+            if blk["res"]:
+                g.k("add", [_p(blk["dres"]), _p(dout), _p(gin[bi]), dout.numel()], f"block{bi}.add_bwd")
+        d = gin[0]
+        conv_bn_bwd(layers[0], d, None)
+        g.k("sgd", [_p(P.flat), _p(P.gflat), _p(P.vflat), P.total, f32bits(lr), f32bits(momentum)], "sgd")
+        variants.append(g.ops)
+        ws_ops = g._ws_ops
+    g.variants = []
+    for ops in variants:
+        g.ops, g._ws_ops = ops, list(ws_ops)
+        g.finalize()
+        g.variants.append(list(g.ops))
+    g.ops = g.variants[0]
+    g.loss = loss
+    g.params = P
+    g.logits = logits
+    return g

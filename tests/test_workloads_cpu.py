@@ -1,0 +1,74 @@
+"""Op-list builders (workloads.py) on the CPU: structure only (no kernels run). Parameter specs
+must equal the oracle's independently written specs; every kernel op must carry at least the
+args its table entry needs, with non-null device pointers where the kernel dereferences them."""
+import pytest
+import torch
+
+from oracle import model as om
+from synth import inputs as si
+from paper_conf_eurosys_stratimk24_b200 import workloads as W, _lib as L
+
+
+def test_specs_match_oracle():
+    assert W.mlp_spec() == om.mlp_spec()
+    assert W.resnet_spec() == om.resnet_spec()
+    assert W.mnv2_spec() == om.mnv2_spec()
+    assert W.mnv2_blocks() == om.mnv2_blocks()
+
+
+NARGS = {"gemm": 13, "colsum": 4, "relu": 3, "relu_bwd": 4, "relu6": 3, "relu6_bwd": 4, "add": 4, "mse": 6, "sgd": 6,
+         "conv_fwd": 14, "conv_dgrad": 14, "conv_wgrad": 16, "dw_fwd": 14, "dw_dgrad": 14, "dw_wgrad": 16,
+         "bn_eval": 9, "bn_stats": 11, "bn_apply": 8, "bn_bwd_reduce": 10, "bn_bwd_dx": 10, "maxpool": 8,
+         "avgpool": 5, "avgpool_bwd": 5, "ce": 7}
+
+
+def _check(g):
+    for fn, args, lab in g.ops:
+        if isinstance(fn, str):
+            assert fn in L.FN, fn
+            assert len(args) >= NARGS[fn], (lab, fn, len(args))
+            assert all(isinstance(a, int) for a in args), lab
+            assert args[0] != 0, lab
+
+
+def test_mlp_graphs():
+    P = si.make_params(W.mlp_spec(64))
+    hp = W.mlp_infer_graph(P, batch=1, width=64, device="cpu")
+    assert [o[2] for o in hp.ops] == ["h2d_input", "fc0", "relu0", "fc1", "relu1", "fc2", "d2h_output"]
+    _check(hp)
+    xs = [si.normal((4, 64), 2, sub=i) for i in range(2)]
+    be = W.mlp_train_graph(P, xs, xs, width=64, device="cpu")
+    assert len(be.variants) == 2 and len(be.variants[0]) == len(be.variants[1]) == 17
+    for v in be.variants:
+        be.ops = v
+        _check(be)
+
+
+def test_resnet_graph_structure():
+    P = si.make_params(W.resnet_spec())
+    g = W.resnet_infer_graph(P, batch=1, hw=32, device="cpu")
+    _check(g)
+    labs = [o[2] for o in g.ops]
+    kern = [o for o in g.ops if isinstance(o[0], str)]
+    # 53 convs (+ fc), 53 BN, 49 ReLU, 16 add, maxpool, avgpool -> 174 ops + 2 memops
+    assert sum(1 for o in kern if o[2].endswith(".relu") or o[2] == "bn1.relu") == 49
+    assert sum(1 for o in kern if o[0] == "bn_eval") == 53
+    assert sum(1 for o in kern if o[0] == "add") == 16
+    assert len(kern) == 174, len(kern)
+    assert labs[0] == "h2d_input" and labs[-1] == "d2h_logits"
+
+
+def test_mnv2_graph_structure():
+    P = si.make_params(W.mnv2_spec(num_classes=10))
+    xs = [si.normal((2, 32, 32, 3), 2, sub=i) for i in range(2)]
+    labels = [si.labels(2, 10, 2, sub=i) for i in range(2)]
+    g = W.mnv2_train_graph(P, xs, labels, num_classes=10, device="cpu")
+    assert len(g.variants) == 2
+    for v in g.variants:
+        g.ops = v
+        _check(g)
+    fns = [o[0] for o in g.variants[0]]
+    assert fns.count("bn_stats") == 52 and fns.count("bn_bwd_dx") == 52
+    assert fns.count("sgd") == 1 and fns.count("ce") == 1
+    assert fns.count("dw_fwd") == 17 and fns.count("dw_wgrad") == 17 and fns.count("dw_dgrad") == 17
+    assert 350 <= len(fns) <= 520, len(fns)
