@@ -22,6 +22,7 @@ OPF_REQ_BEGIN, OPF_REQ_END = 1, 2
 F_HP_BUSY_REQUEST, F_HP_REF_ALL, F_HP_UNKNOWN_STRICT, F_THROTTLE_ONLY_HP_BUSY, F_FREE_SMS = 1, 2, 4, 8, 16
 BACKEND_CUDA, BACKEND_FAKE = 0, 1
 MAX_ARGS = 24
+WS_TICKET_BYTES = 65536   # kernels/common.cuh: ticket region at the start of every workspace
 
 
 class Profile(ctypes.Structure):

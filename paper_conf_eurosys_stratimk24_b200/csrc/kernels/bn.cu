@@ -30,7 +30,7 @@ BnSplit bn_split(long long rows, int C) {
 
 uint64_t bn_ws_bytes(long long rows, int C, int nvals) {
   BnSplit s = bn_split(rows, C);
-  return 256 * cdiv((uint64_t)s.cblocks * 4, 256) * 1 + (uint64_t)s.rs * C * nvals * 8;
+  return WS_TICKET_BYTES + (uint64_t)s.rs * C * nvals * 8;
 }
 
 // Reduce per-thread double accumulators v[NV] over the row-lanes of the CTA (fixed order) and
@@ -43,8 +43,7 @@ __device__ bool bn_partial(double (&v)[NV], int C, int cb, int c0, int rs_count,
   for (int j = 0; j < NV; j++) sh[(rl * cb + cl) * NV + j] = v[j];
   __syncthreads();
   unsigned int* tickets = reinterpret_cast<unsigned int*>(ws);
-  const int cblocks = (C + cb - 1) / cb;
-  double* part = reinterpret_cast<double*>(ws + 256 * ((cblocks * 4 + 255) / 256));
+  double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
   if (rl == 0) {
     double t[NV];
     for (int j = 0; j < NV; j++) t[j] = 0.0;
@@ -59,8 +58,8 @@ __device__ bool bn_partial(double (&v)[NV], int C, int cb, int c0, int rs_count,
 
 template <int NV>
 __device__ void bn_combine(double (&t)[NV], int C, int c, int rs_count, unsigned char* ws, int cb) {
-  const int cblocks = (C + cb - 1) / cb;
-  const double* part = reinterpret_cast<const double*>(ws + 256 * ((cblocks * 4 + 255) / 256));
+  (void)cb;
+  const double* part = reinterpret_cast<const double*>(ws + WS_TICKET_BYTES);
   for (int j = 0; j < NV; j++) t[j] = 0.0;
   for (int r = 0; r < rs_count; r++)
     for (int j = 0; j < NV; j++) t[j] += __ldcg(part + ((long long)r * C + c) * NV + j);

@@ -69,6 +69,12 @@ __device__ __forceinline__ bool last_cta_of(unsigned int* ticket, unsigned int c
   return s_last != 0;
 }
 
+// Workspace layout shared by all ops of a client (they run in stream order): the first
+// WS_TICKET_BYTES hold u32 tickets, always zero between launches (each group's last CTA resets its
+// ticket); per-launch partials follow. Separating the two keeps one op's partials from ever
+// aliasing another op's tickets.
+constexpr uint64_t WS_TICKET_BYTES = 65536;
+
 // Kernel table (table.cu)
 extern const KernelEntry g_kernels[ORION_FN_COUNT];
 int kernel_launch_sig(uint32_t fn, const uint64_t* args, uint32_t nargs, OrionSig sig, cudaStream_t s,

@@ -110,9 +110,8 @@ __global__ void __launch_bounds__(DW_THREADS) dw_wgrad_kernel(const float* __res
 #pragma unroll
   for (int j = 0; j < 9; j++) sh[threadIdx.x][j] = acc[j];
   __syncthreads();
-  const int cblocks = (s.C + WG_CB - 1) / WG_CB;
   unsigned int* tickets = reinterpret_cast<unsigned int*>(ws);
-  double* part = reinterpret_cast<double*>(ws + 256 * ((cblocks * 4 + 255) / 256));
+  double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
   if (pl == 0 && c < s.C) {
     for (int j = 0; j < 9; j++) {
       double t = 0.0;
@@ -165,7 +164,7 @@ WgSplit wg_split(const DwShape& s) {
 extern "C" uint64_t orion_dw_wgrad_workspace_bytes(uint64_t N, uint64_t C, uint64_t P, uint64_t Q) {
   DwShape s{(int)N, 0, 0, (int)C, 1, (int)P, (int)Q};
   WgSplit w = wg_split(s);
-  return 256 * cdiv((uint64_t)w.cblocks * 4, 256) + (uint64_t)w.rs * C * 9 * 8;
+  return WS_TICKET_BYTES + (uint64_t)w.rs * C * 9 * 8;
 }
 
 #define CHECK_LAUNCH() return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA

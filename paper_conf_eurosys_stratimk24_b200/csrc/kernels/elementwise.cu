@@ -150,7 +150,7 @@ __global__ void __launch_bounds__(EW_THREADS) mse_kernel(const float* __restrict
                                                          float* __restrict__ dy, long long n, unsigned char* ws, OrionSig sig) {
   __shared__ double sh[32];
   unsigned int* ticket = reinterpret_cast<unsigned int*>(ws);
-  double* part = reinterpret_cast<double*>(ws + 256);
+  double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
   long long i0 = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   long long stride = (long long)gridDim.x * blockDim.x;
   double acc = 0.0;
@@ -177,7 +177,7 @@ __global__ void __launch_bounds__(EW_THREADS) ce_kernel(const float* __restrict_
                                                         float* __restrict__ dz, int B, int Cn, unsigned char* ws, OrionSig sig) {
   __shared__ float sh[32];
   unsigned int* ticket = reinterpret_cast<unsigned int*>(ws);
-  float* rowloss = reinterpret_cast<float*>(ws + 256);
+  float* rowloss = reinterpret_cast<float*>(ws + WS_TICKET_BYTES);
   const int b = blockIdx.x;
   const float* zr = z + (long long)b * Cn;
   float m = -FLT_MAX;
@@ -291,7 +291,7 @@ int colsum_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStre
   CHECK_LAUNCH();
 }
 
-// ---- MSE: args y, t, loss, dy, n, ws (>= 256 + 8 * ctas bytes, zeroed once)
+// ---- MSE: args y, t, loss, dy, n, ws (>= WS_TICKET_BYTES + 8 * ctas bytes, zeroed once)
 int mse_geom(const uint64_t* a, LaunchGeom* g) { ew_geom(g, a[4], (const void*)mse_kernel); return 0; }
 int mse_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   mse_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (const float*)a[1], (float*)a[2], (float*)a[3], (long long)a[4],
@@ -299,7 +299,7 @@ int mse_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_
   CHECK_LAUNCH();
 }
 
-// ---- CE: args z, labels, loss, dz, B, classes, ws (>= 256 + 4 * B bytes, zeroed once)
+// ---- CE: args z, labels, loss, dz, B, classes, ws (>= WS_TICKET_BYTES + 4 * B bytes, zeroed once)
 int ce_geom(const uint64_t* a, LaunchGeom* g) {
   g->grid = dim3((unsigned)a[4]); g->block = dim3(EW_THREADS); g->smem = 0; g->func = (const void*)ce_kernel;
   return 0;

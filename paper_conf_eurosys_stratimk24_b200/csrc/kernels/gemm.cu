@@ -334,11 +334,9 @@ GemmParams make_params(long long M, long long N, long long K, float* C, long lon
   p.ws = ws;
   p.tickets = nullptr;
   if (split > 1) {
-    // workspace layout: [tickets (256 B aligned)][partials]
-    long long tiles = cdiv(M, BM) * cdiv(N, BN);
-    long long tk_bytes = ((tiles * 4 + 255) / 256) * 256;
+    // workspace layout: [tickets (WS_TICKET_BYTES)][partials]
     p.tickets = reinterpret_cast<unsigned int*>(ws);
-    p.ws = reinterpret_cast<float*>(reinterpret_cast<char*>(ws) + tk_bytes);
+    p.ws = reinterpret_cast<float*>(reinterpret_cast<char*>(ws) + WS_TICKET_BYTES);
     (void)ws_bytes;
   }
   return p;
@@ -350,8 +348,7 @@ GemmParams make_params(long long M, long long N, long long K, float* C, long lon
 extern "C" uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t K) {
   int split = choose_split(M, N, K);
   if (split == 1) return 0;
-  long long tiles = cdiv(M, BM) * cdiv(N, BN);
-  return ((tiles * 4 + 255) / 256) * 256 + (uint64_t)split * M * N * 4;
+  return WS_TICKET_BYTES + (uint64_t)split * M * N * 4;
 }
 
 // ------------------------------------------------------------------------- GEMM entry

@@ -28,7 +28,7 @@ class Graph:
         self.device = device
         self.ops = []          # (fn_name or kind, args, label)
         self.bufs = {}
-        self.ws_bytes = 256
+        self.ws_bytes = L.WS_TICKET_BYTES + 256
         self._ws = None
         self._ws_ops = []      # (op index, arg index of ws ptr, arg index of ws bytes)
 
@@ -222,7 +222,7 @@ def mlp_train_graph(host_params, xs, ts, lr=0.01, width=512, layers=3, device="c
     a = [g.buf(f"a{i}", (batch, width)) for i in range(layers - 1)]
     dz = [g.buf(f"dz{i}", (batch, width)) for i in range(layers)]
     da = [g.buf(f"da{i}", (batch, width)) for i in range(layers - 1)]
-    g.need_ws(256 + 8 * 148 * 8)
+    g.need_ws(L.WS_TICKET_BYTES + 8 * 148 * 8)
     variants = []
     for vi in range(len(xs)):
         g.ops = []
@@ -434,7 +434,7 @@ def mnv2_train_graph(host_params, xs, labels, lr=0.01, momentum=0.9, num_classes
     pooled, logits, dlogits, dpooled, dfeat = new((n, c)), new((n, num_classes)), new((n, num_classes)), new((n, c)), new(shape)
     for L_ in layers:
         g.need_ws(L.lib.orion_bn_workspace_bytes(L_["z"].shape[0] * L_["z"].shape[1] * L_["z"].shape[2], L_["cout"]))
-    g.need_ws(256 + 4 * batch)
+    g.need_ws(L.WS_TICKET_BYTES + 4 * batch)
 
     def conv_bn_fwd(L_, h):
         w = P.p[f"{L_['cname']}.w"]

@@ -1,0 +1,90 @@
+"""End-to-end at BASELINE config 2's full sizes: HP ResNet-50 inference b4 (224x224) collocated with
+BE MobileNetV2 training b96 under liborion on the GPU, in the bench's launch configuration.
+  * HP logits of 16 requests vs the fp64 oracle (rel L2 1e-4, north_star);
+  * one BE training iteration (loss, every gradient, BN running stats, SGD-updated parameters) vs
+    the fp64 oracle (rel L2 1e-4; BN betas feeding conv->train-BN have an exactly-zero true gradient
+    and are compared against an absolute floor);
+  * decision log == oracle replay, byte for byte;
+  * HP logits and BE parameters bitwise identical between collocated and solo runs."""
+import numpy as np
+import pytest
+import torch
+
+from oracle import model as om
+from oracle import policy_ffi as po
+from synth import inputs as si
+import logfmt as lf
+
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    from paper_conf_eurosys_stratimk24_b200 import workloads as W, collocate as C, profiler as PR
+
+
+def rel(a, b, floor=1e-30):
+    a, b = torch.as_tensor(a).double().cpu(), torch.as_tensor(b).double().cpu()
+    return float((a - b).norm() / max(float(b.norm()), floor))
+
+
+@pytest.fixture(scope="module")
+def cfg2():
+    torch.cuda.set_device(0)
+    Prn = si.make_params(W.resnet_spec())
+    hp_inputs = [si.normal((4, 224, 224, 3), si.HP_SEED, sub=r) for r in range(16)]
+    hpg = W.resnet_infer_graph(Prn, batch=4)
+    Pmn = si.make_params(W.mnv2_spec())
+    xs = [si.normal((96, 224, 224, 3), si.BE_SEED, sub=i) for i in range(8)]
+    labels = [si.labels(96, 1000, si.BE_SEED, sub=i) for i in range(8)]
+    beg = W.mnv2_train_graph(Pmn, xs, labels)
+    ph, _ = PR.build_profiles(hpg, 0, reps=3)
+    pb, _ = PR.build_profiles(beg, 10000, reps=3)
+    beg.params.reset()
+    hp = C.HPClient(hpg, hp_inputs, 16, ph, 0)
+    be = C.BEClient(beg, pb, 10000)
+    lat = C.latency_stats(C.run_session(hp=hp, arrivals_ns=(np.arange(1, 11) * 30e6).astype(np.int64)))["p50_ns"]
+    return dict(Prn=Prn, Pmn=Pmn, hp=hp, be=be, xs=xs, labels=labels, hp_inputs=hp_inputs, lat=int(lat))
+
+
+def test_be_one_iteration_vs_oracle(cfg2):
+    be, Pmn = cfg2["be"], cfg2["Pmn"]
+    be.graph.params.reset()
+    C.run_session(be=be, be_iters=1)
+    G = be.graph.params
+    loss_ref, newP, newV, g_ref = om.mnv2_train_step(Pmn, {}, cfg2["xs"][0], cfg2["labels"][0], first=True)
+    assert rel(be.graph.loss, loss_ref.reshape(1)) < 1e-5
+    worst = {}
+    for name, ref in g_ref.items():
+        floor = 1e-3 if name.endswith(".beta") else 1e-30
+        worst[name] = rel(G.g[name], ref, floor)
+    bad = {k: v for k, v in worst.items() if v > 1e-4}
+    assert not bad, sorted(bad.items(), key=lambda x: -x[1])[:10]
+    for name in newP:
+        assert rel(G.p[name], newP[name]) < 1e-5, name
+    # first step: v = mu*0 + g = g exactly (torch's v <- g), so the momentum buffer equals the grads
+    assert torch.equal(G.vflat, G.gflat)
+
+
+def test_collocated_parity_and_log(cfg2):
+    hp, be = cfg2["hp"], cfg2["be"]
+    be.graph.params.reset()
+    hp.out.zero_()
+    arrivals = si.poisson_arrivals_ns(40.0, 16)
+    res = C.run_session(hp=hp, be=be, arrivals_ns=arrivals, log_capacity=1 << 22, hp_latency_ns=cfg2["lat"])
+    out_col = hp.out.clone()
+    K = len(res["be_t_end"])
+    p_col = be.graph.params.flat.cpu().clone()
+    assert K >= 1
+    # decision log bit-exact vs oracle replay of the recorded tape
+    _, prefix, _, decs = lf.split_log(res["log"])
+    assert decs == po.replay(prefix)
+    # HP logits vs oracle
+    for r in range(16):
+        ref = om.resnet_infer(cfg2["Prn"], cfg2["hp_inputs"][r])
+        assert rel(out_col[r].view(4, 1000), ref) < 1e-4, r
+    # solo runs: bitwise equal
+    hp.out.zero_()
+    C.run_session(hp=hp, arrivals_ns=arrivals)
+    assert torch.equal(hp.out, out_col)
+    be.graph.params.reset()
+    C.run_session(be=be, be_iters=K)
+    assert torch.equal(be.graph.params.flat.cpu(), p_col)
