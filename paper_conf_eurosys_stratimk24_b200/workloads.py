@@ -52,9 +52,12 @@ class Graph:
         self.ops.append((kind, [dst, src, nbytes], label))
 
     def finalize(self):
-        """Allocate the shared split/reduction workspace (ops of one client run in stream order, and
-        every kernel leaves its tickets zeroed, so one workspace serves all of them)."""
-        self._ws = torch.zeros(self.ws_bytes // 4 + 64, dtype=F32, device=self.device)
+        """Allocate the shared split/reduction workspace once per graph (ops of one client run in
+        stream order, and every kernel leaves its tickets zeroed, so one workspace serves all ops and
+        all variants) and patch its pointer into the ops that use it."""
+        if self._ws is None or self._ws.numel() * 4 < self.ws_bytes:
+            assert self._ws is None, "workspace grew after ops were patched"
+            self._ws = torch.zeros(self.ws_bytes // 4 + 64, dtype=F32, device=self.device)
         for i, at in self._ws_ops:
             self.ops[i][1][at] = self._ws.data_ptr()
             self.ops[i][1][at + 1] = self.ws_bytes

@@ -13,6 +13,7 @@ pytestmark = pytest.mark.gpu
 
 if torch.cuda.is_available():
     import paper_conf_eurosys_stratimk24_b200 as orion
+    import paper_conf_eurosys_stratimk24_b200.profiler  # noqa: F401
     from paper_conf_eurosys_stratimk24_b200 import _lib as L
 
 
@@ -191,4 +192,5 @@ def test_geometry_and_sm_needed():
     grid, bps, thr, smem = orion.kernel_geometry("gemm", [A.data_ptr(), A.data_ptr(), A.data_ptr(), 0, 4096, 256, 256, 256, 256, 256, 2, 0, 0])
     assert grid == 32 * 2 and thr == 256 and bps >= 1
     grid, bps, thr, smem = orion.kernel_geometry("relu", [A.data_ptr(), A.data_ptr(), A.numel()])
-    assert grid == min((A.numel() // 4 + 255) // 256, 148 * 8) and bps == 8
+    assert grid == min((A.numel() // 4 + 255) // 256, 148 * 8) and 1 <= bps <= 8
+    assert orion.profiler.sm_needed("relu", [A.data_ptr(), A.data_ptr(), A.numel()]) == -(-grid // bps)

@@ -72,3 +72,25 @@ def test_mnv2_graph_structure():
     assert fns.count("sgd") == 1 and fns.count("ce") == 1
     assert fns.count("dw_fwd") == 17 and fns.count("dw_wgrad") == 17 and fns.count("dw_dgrad") == 17
     assert 350 <= len(fns) <= 520, len(fns)
+
+
+def test_variants_share_one_live_workspace():
+    """Every variant's ops must point at the one workspace the graph keeps alive (a freed workspace
+    would be reused by the allocator: a dangling-pointer race)."""
+    P = si.make_params(W.mnv2_spec(num_classes=10))
+    xs = [si.normal((2, 32, 32, 3), 2, sub=i) for i in range(3)]
+    labels = [si.labels(2, 10, 2, sub=i) for i in range(3)]
+    g = W.mnv2_train_graph(P, xs, labels, num_classes=10, device="cpu")
+    ws = g._ws.data_ptr()
+    for v in g.variants:
+        for fn, args, lab in v:
+            if fn in ("bn_stats", "dw_wgrad", "ce", "conv_wgrad"):
+                at = {"bn_stats": 9, "dw_wgrad": 14, "ce": 6, "conv_wgrad": 14}[fn]
+                assert args[at] == ws, lab
+    Pm = si.make_params(W.mlp_spec(64))
+    xm = [si.normal((4, 64), 2, sub=i) for i in range(3)]
+    gm = W.mlp_train_graph(Pm, xm, xm, width=64, device="cpu")
+    for v in gm.variants:
+        for fn, args, lab in v:
+            if fn == "mse":
+                assert args[5] == gm._ws.data_ptr()
