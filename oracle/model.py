@@ -323,10 +323,15 @@ def mnv2_trainable(spec):
     return [n for n, _, _ in spec if not (n.endswith(".rmean") or n.endswith(".rvar"))]
 
 
-def mnv2_train_step(P, V, x, labels, first, lr=0.01, momentum=0.9, eps=1e-5, bn_momentum=0.1):
+def mnv2_train_step(P, V, x, labels, first, lr=0.01, momentum=0.9, eps=1e-5, bn_momentum=0.1, masks=None):
     """One training iteration of torchvision MobileNetV2 (dropout p=0, reading R22) with
     CE loss and SGD(momentum). P: params + BN running stats (dict of fp32 tensors);
-    V: momentum buffers (dict). Returns (loss, newP, newV, grads)."""
+    V: momentum buffers (dict). Returns (loss, newP, newV, grads).
+
+    masks (optional): {bn name: fp32 tensor} — the values on which the ReLU6 backward takes its
+    pass/stop decision (0 < y < 6). A decision is an integer decided by floating point; to compare
+    a fp32 GPU backward with this fp64 oracle both must decide on the same value, so
+    parity tests pass the GPU's own BN outputs here. All arithmetic stays the oracle's."""
     newP = dict(P)
 
     def conv_bn(h, cname, bname, k, stride, groups, act):
@@ -341,7 +346,7 @@ def mnv2_train_step(P, V, x, labels, first, lr=0.01, momentum=0.9, eps=1e-5, bn_
 
     def conv_bn_bwd(rec, dout, need_dx=True):
         cname, bname, k, stride, groups, act, hin, z, y, mean, invstd = rec
-        dy = relu6_bwd(y, dout) if act else dout
+        dy = relu6_bwd(masks[bname] if masks is not None else y, dout) if act else dout
         dz, g[f"{bname}.gamma"], g[f"{bname}.beta"] = bn_bwd(z, dy, P[f"{bname}.gamma"], mean, invstd)
         w = P[f"{cname}.w"]
         g[f"{cname}.w"] = conv2d_bwd_weight(hin, dz, tuple(w.shape), stride, k // 2, groups)

@@ -172,14 +172,16 @@ __global__ void __launch_bounds__(BN_THREADS) bn_bwd_dx_kernel(const float* __re
                                                                const float* __restrict__ gamma, const float* __restrict__ mean,
                                                                const float* __restrict__ invstd, const float* __restrict__ dgamma,
                                                                const float* __restrict__ dbeta, long long rows, int C, OrionSig sig) {
+  // fp64 per element: dy and (dbeta + xhat*dgamma)/N nearly cancel, and fp32 would amplify the
+  // rounding of each term through every BN layer of the backward pass (memory-bound: free)
   const long long total = rows * C;
-  const float invN = 1.0f / (float)rows;
+  const double invN = 1.0 / (double)rows;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
     int c = (int)(i % C);
-    float is = invstd[c];
-    float xh = (x[i] - mean[c]) * is;
-    float k = gamma[c] * is;
-    dx[i] = k * (dy[i] - (dbeta[c] + xh * dgamma[c]) * invN);
+    double is = invstd[c];
+    double xh = ((double)x[i] - (double)mean[c]) * is;
+    double k = (double)gamma[c] * is;
+    dx[i] = (float)(k * ((double)dy[i] - ((double)dbeta[c] + xh * (double)dgamma[c]) * invN));
   }
   orion_signal(sig);
 }

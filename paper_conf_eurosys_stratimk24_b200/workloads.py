@@ -519,4 +519,5 @@ def mnv2_train_graph(host_params, xs, labels, lr=0.01, momentum=0.9, num_classes
     g.loss = loss
     g.params = P
     g.logits = logits
+    g.bn_out = {L_["bname"]: L_["y"] for L_ in layers}   # BN outputs (ReLU6 inputs), for parity tests
     return g

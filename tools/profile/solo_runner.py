@@ -1,0 +1,40 @@
+"""Solo op runner for the offline profiler (§5.2): launches every kernel op of one client's
+op list once, in order, directly through the C ABI (no scheduler), so that
+`ncu --csv` captures exactly one launch per kernel_id (launch i <-> i-th kernel op)."""
+import argparse
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import bench  # noqa: E402
+import paper_conf_eurosys_stratimk24_b200 as orion  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="rn50_mnv2")
+    ap.add_argument("--client", default="be", choices=["hp", "be"])
+    ap.add_argument("--only", default=None, help="substring of op labels to launch (others skipped)")
+    ap.add_argument("--repeat", type=int, default=1)
+    a = ap.parse_args()
+    torch.cuda.set_device(0)
+    W = bench.build_config(a.config, 0)
+    g = W["hpg"] if a.client == "hp" else W["beg"]
+    s = torch.cuda.current_stream().cuda_stream
+    for _ in range(a.repeat):
+        for fn, args, lab in g.ops:
+            if isinstance(fn, str) and (a.only is None or a.only in lab):
+                orion.kernel_launch(fn, args, s)
+    torch.cuda.synchronize()
+    with open(os.path.join(ROOT, "gpurun_out", f"oplist_{a.config}_{a.client}.txt"), "w") as f:
+        for i, (fn, args, lab) in enumerate(g.ops):
+            if isinstance(fn, str):
+                f.write(f"{i}\t{fn}\t{lab}\n")
+
+
+if __name__ == "__main__":
+    main()
