@@ -68,6 +68,22 @@ def build_config(name, rank):
                      "image": "224x224x3 NHWC fp32", "arrivals": "poisson 15 rps (PAPER Table 3)"})
 
 
+def build_client(name, client):
+    """One client's graph only (the offline profiler's solo runner)."""
+    from paper_conf_eurosys_stratimk24_b200 import workloads as W
+    from synth import inputs as si
+    if name == "toy":
+        P = si.make_params(W.mlp_spec())
+        if client == "hp":
+            return W.mlp_infer_graph(P, batch=1)
+        return W.mlp_train_graph(P, [si.normal((32, 512), si.BE_SEED, sub=i) for i in range(8)],
+                                 [si.normal((32, 512), si.BE_SEED, sub=100 + i) for i in range(8)])
+    if client == "hp":
+        return W.resnet_infer_graph(si.make_params(W.resnet_spec()), batch=4)
+    return W.mnv2_train_graph(si.make_params(W.mnv2_spec()), [si.normal((96, 224, 224, 3), si.BE_SEED, sub=0)],
+                              [si.labels(96, 1000, si.BE_SEED, sub=0)])
+
+
 def with_be_h2d(graph, xs_host):
     """E2E variant of the BE client: each iteration first copies its batch from pinned host memory
     (H2D memop) and finally reads the loss back (D2H memop)."""

@@ -76,6 +76,8 @@ def test_be_one_iteration_vs_oracle(cfg2):
     bad = {k: v for k, v in worst.items() if v > 3e-4}
     assert not bad, sorted(bad.items(), key=lambda x: -x[1])[:10]
     for name in newP:
+        if name.endswith("project_bn.beta"):
+            continue   # init 0 and exactly-zero true gradient: the value is pure rounding noise (checked above)
         assert rel(G.p[name], newP[name]) < 1e-5, name
     # first step: v = mu*0 + g = g exactly (torch's v <- g), so the momentum buffer equals the grads
     assert torch.equal(G.vflat, G.gflat)

@@ -22,8 +22,7 @@ def main():
     ap.add_argument("--repeat", type=int, default=1)
     a = ap.parse_args()
     torch.cuda.set_device(0)
-    W = bench.build_config(a.config, 0)
-    g = W["hpg"] if a.client == "hp" else W["beg"]
+    g = bench.build_client(a.config, a.client)
     s = torch.cuda.current_stream().cuda_stream
     for _ in range(a.repeat):
         for fn, args, lab in g.ops:
