@@ -25,7 +25,9 @@ extern "C" {
 enum orion_fn {
   /* C[M,N] = op(A) op(B) (+ bias[N]); row-major; op = transpose if flag set.
      args: A, B, C, bias (0 = none), M, N, K, lda, ldb, ldc, flags (1 = A^T, 2 = B^T).
-     y = x W^T + b (Linear fwd) is flags=2; dx = dy W is flags=0; dW = dy^T x is flags=1. */
+     y = x W^T + b (Linear fwd) is flags=2; dx = dy W is flags=0; dW = dy^T x is flags=1.
+     args[11], args[12] = workspace, ws_bytes for the shape-selected K split (0 = no split); size
+     from orion_gemm_workspace_bytes(M, N, K). */
   ORION_FN_GEMM = 0,
   /* Column sum: out[n] = sum_m A[m, n]  (bias gradient). args: A, out, M, N */
   ORION_FN_COLSUM = 1,
@@ -46,11 +48,14 @@ enum orion_fn {
      args: p, g, v, n, lr_bits, mu_bits */
   ORION_FN_SGD = 8,
   /* Conv2d forward, implicit GEMM, groups = 1, no bias. args: x, w, y, N, H, W, C, K(=Cout),
-     R, S (kernel h, w), stride, pad, P, Q (out h, w) */
+     R, S (kernel h, w), stride, pad, P, Q (out h, w), workspace, ws_bytes (split-K; 0 = no split;
+     size from orion_gemm_workspace_bytes(N*P*Q, K, R*S*C)) */
   ORION_FN_CONV_FWD = 9,
-  /* Conv2d backward data: dx[N,H,W,C] from dy[N,P,Q,K], w. args: dy, w, dx, N,H,W,C,K,R,S,stride,pad,P,Q */
+  /* Conv2d backward data: dx[N,H,W,C] from dy[N,P,Q,K], w. args: dy, w, dx, N,H,W,C,K,R,S,stride,pad,P,Q,
+     workspace, ws_bytes (orion_gemm_workspace_bytes(N*H*W, C, R*S*K)) */
   ORION_FN_CONV_DGRAD = 10,
-  /* Conv2d backward weight: dw[K,R,S,C] from x, dy. args: x, dy, dw, N,H,W,C,K,R,S,stride,pad,P,Q */
+  /* Conv2d backward weight: dw[K,R,S,C] from x, dy. args: x, dy, dw, N,H,W,C,K,R,S,stride,pad,P,Q,
+     workspace, ws_bytes (orion_gemm_workspace_bytes(K, R*S*C, N*P*Q)) */
   ORION_FN_CONV_WGRAD = 11,
   /* Depthwise 3x3 conv (groups = C): args as CONV_* with K = C */
   ORION_FN_DW_FWD = 12,
@@ -91,6 +96,11 @@ int orion_kernel_launch(uint32_t fn, const uint64_t* args, uint32_t nargs, void*
    CTAs per SM (cudaOccupancyMaxActiveBlocksPerMultiprocessor), for sm_needed (R17). */
 int orion_kernel_geometry(uint32_t fn, const uint64_t* args, uint32_t nargs, uint64_t* grid_ctas,
                           int32_t* blocks_per_sm, int32_t* threads_per_cta, int32_t* smem_bytes);
+/* Workspace sizes (bytes) of the ops that split their reductions. Workspaces must be zeroed once
+   at allocation; a client's ops may share one (they run in stream order; tickets self-reset). */
+uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t K);
+uint64_t orion_bn_workspace_bytes(uint64_t rows, uint64_t C);
+uint64_t orion_dw_wgrad_workspace_bytes(uint64_t N, uint64_t C, uint64_t P, uint64_t Q);
 
 #ifdef __cplusplus
 }

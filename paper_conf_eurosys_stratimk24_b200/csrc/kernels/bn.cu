@@ -9,20 +9,25 @@ namespace {
 
 constexpr int BN_THREADS = 256;
 
-// Channel block / row-lane split of a CTA for C channels.
-__host__ __device__ inline int bn_cb(int C) { return C >= 64 ? 64 : (C >= 32 ? 32 : (C >= 16 ? 16 : (C >= 8 ? 8 : 4))); }
-
-struct BnSplit { int cb, cblocks, rs; long long rows_per_split; };
+// Reduction kernels (train statistics, backward reduce). A thread owns 4 consecutive channels
+// (128-bit loads; C % 4 == 0 on every BN of the workloads, checked at geometry time) and a
+// row lane; a CTA owns CG4 channel quads x RL row lanes (RL*CG4 <= 256) and one row split. Rows
+// are unrolled by 4 so each thread keeps 4 (stats) or 8 (backward) 128-bit loads in flight.
+// fp64 accumulation, fixed-order combine of row lanes in smem, per-split partials combined in
+// split order by the last CTA of the channel block.
+struct BnSplit { int cg4, rl, cblocks, rs; long long rows_per_split; };
 
 BnSplit bn_split(long long rows, int C) {
   BnSplit s;
-  s.cb = bn_cb(C);
-  s.cblocks = (int)cdiv(C, s.cb);
-  long long rs = cdiv(296, s.cblocks);               // shape-only: ~2 waves of a 148-SM part
-  long long max_rs = cdiv(rows, 512);                  // >= 512 rows per split
+  int q = C / 4;
+  s.cg4 = q < 64 ? q : 64;
+  s.rl = BN_THREADS / s.cg4;
+  s.cblocks = (int)cdiv(q, s.cg4);
+  long long rs = cdiv(148 * 8, s.cblocks);      // shape-only: ~one full wave of 8 CTAs per SM on 148 SMs
+  long long max_rs = cdiv(rows, 4LL * s.rl);    // >= 4 rows per row lane
   if (rs > max_rs) rs = max_rs;
   if (rs < 1) rs = 1;
-  if (rs > 1024) rs = 1024;
+  if (rs > 2048) rs = 2048;
   s.rs = (int)rs;
   s.rows_per_split = cdiv(rows, rs);
   return s;
@@ -33,65 +38,87 @@ uint64_t bn_ws_bytes(long long rows, int C, int nvals) {
   return WS_TICKET_BYTES + (uint64_t)s.rs * C * nvals * 8;
 }
 
-// Reduce per-thread double accumulators v[NV] over the row-lanes of the CTA (fixed order) and
-// write the CTA's partial for its channels to ws; returns true in the last CTA of the channel
-// block, which must then combine partials (split order) via `combine`.
-template <int NV>
-__device__ bool bn_partial(double (&v)[NV], int C, int cb, int c0, int rs_count, unsigned char* ws, double* sh) {
-  const int tid = threadIdx.x, rl_n = BN_THREADS / cb, cl = tid % cb, rl = tid / cb;
-  // sh: [rl_n][cb][NV]
-  for (int j = 0; j < NV; j++) sh[(rl * cb + cl) * NV + j] = v[j];
+struct D4 { double x, y, z, w; };
+__device__ __forceinline__ void add4(D4& a, const float4& v) { a.x += v.x; a.y += v.y; a.z += v.z; a.w += v.w; }
+__device__ __forceinline__ void sq4(D4& a, const float4& v) {
+  a.x = fma((double)v.x, (double)v.x, a.x); a.y = fma((double)v.y, (double)v.y, a.y);
+  a.z = fma((double)v.z, (double)v.z, a.z); a.w = fma((double)v.w, (double)v.w, a.w);
+}
+
+// Combine two D4 accumulators per thread over the CTA's row lanes (fixed order), write this
+// split's partial for the CTA's channels; returns true in the last CTA of the channel block.
+__device__ bool bn_partial2(const D4& a, const D4& b, int C, int cg4, int rl_n, unsigned char* ws, double* sh) {
+  const int tid = threadIdx.x, cq = tid % cg4, rl = tid / cg4;
+  const bool active = rl < rl_n;
+  if (active) {
+    double* d = sh + (size_t)(rl * cg4 + cq) * 8;
+    d[0] = a.x; d[1] = a.y; d[2] = a.z; d[3] = a.w; d[4] = b.x; d[5] = b.y; d[6] = b.z; d[7] = b.w;
+  }
   __syncthreads();
   unsigned int* tickets = reinterpret_cast<unsigned int*>(ws);
   double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
-  if (rl == 0) {
-    double t[NV];
-    for (int j = 0; j < NV; j++) t[j] = 0.0;
+  const int c = (blockIdx.x * cg4 + cq) * 4;
+  if (rl == 0 && c < C) {
+    double t[8] = {0, 0, 0, 0, 0, 0, 0, 0};
     for (int r = 0; r < rl_n; r++)
-      for (int j = 0; j < NV; j++) t[j] += sh[(r * cb + cl) * NV + j];
-    int c = c0 + cl;
-    if (c < C)
-      for (int j = 0; j < NV; j++) part[((long long)blockIdx.y * C + c) * NV + j] = t[j];
+      for (int j = 0; j < 8; j++) t[j] += sh[(size_t)(r * cg4 + cq) * 8 + j];
+    for (int k = 0; k < 4; k++) {
+      part[((long long)blockIdx.y * C + c + k) * 2 + 0] = t[k];
+      part[((long long)blockIdx.y * C + c + k) * 2 + 1] = t[4 + k];
+    }
   }
-  return last_cta_of(tickets + blockIdx.x, rs_count);
+  return last_cta_of(tickets + blockIdx.x, gridDim.y);
 }
 
-template <int NV>
-__device__ void bn_combine(double (&t)[NV], int C, int c, int rs_count, unsigned char* ws, int cb) {
-  (void)cb;
+__device__ void bn_combine(double* t0, double* t1, int C, int c, int rs_count, unsigned char* ws) {
   const double* part = reinterpret_cast<const double*>(ws + WS_TICKET_BYTES);
-  for (int j = 0; j < NV; j++) t[j] = 0.0;
-  for (int r = 0; r < rs_count; r++)
-    for (int j = 0; j < NV; j++) t[j] += __ldcg(part + ((long long)r * C + c) * NV + j);
+  double a = 0.0, b = 0.0;
+  for (int r = 0; r < rs_count; r++) {
+    a += __ldcg(part + ((long long)r * C + c) * 2 + 0);
+    b += __ldcg(part + ((long long)r * C + c) * 2 + 1);
+  }
+  *t0 = a;
+  *t1 = b;
 }
 
 // ---- train statistics: mean, invstd (biased var), running stats (unbiased var, momentum)
 __global__ void __launch_bounds__(BN_THREADS) bn_stats_kernel(const float* __restrict__ x, float* mean, float* invstd, float* rm, float* rv,
-                                                              long long rows, int C, float eps, float momentum, int cb,
+                                                              long long rows, int C, float eps, float momentum, int cg4, int rl_n,
                                                               long long rows_per_split, unsigned char* ws, OrionSig sig) {
-  __shared__ double sh[BN_THREADS * 2];
-  const int rl_n = BN_THREADS / cb, cl = threadIdx.x % cb, rl = threadIdx.x / cb;
-  const int c0 = blockIdx.x * cb, c = c0 + cl;
+  __shared__ double sh[BN_THREADS * 8];
+  const int cq = threadIdx.x % cg4, rl = threadIdx.x / cg4;
+  const int c = (blockIdx.x * cg4 + cq) * 4;
   const long long r0 = blockIdx.y * rows_per_split, r1 = min(rows, r0 + rows_per_split);
-  double v[2] = {0.0, 0.0};
-  if (c < C)
-    for (long long r = r0 + rl; r < r1; r += rl_n) {
-      double xv = (double)__ldg(x + r * C + c);
-      v[0] += xv;
-      v[1] += xv * xv;
+  D4 s1{0, 0, 0, 0}, s2{0, 0, 0, 0};
+  if (c < C && rl < rl_n) {
+    const float* xp = x + c;
+    long long r = r0 + rl;
+    for (; r + 3LL * rl_n < r1; r += 4LL * rl_n) {
+      float4 v0 = __ldg(reinterpret_cast<const float4*>(xp + r * C));
+      float4 v1 = __ldg(reinterpret_cast<const float4*>(xp + (r + rl_n) * C));
+      float4 v2 = __ldg(reinterpret_cast<const float4*>(xp + (r + 2LL * rl_n) * C));
+      float4 v3 = __ldg(reinterpret_cast<const float4*>(xp + (r + 3LL * rl_n) * C));
+      add4(s1, v0); sq4(s2, v0); add4(s1, v1); sq4(s2, v1); add4(s1, v2); sq4(s2, v2); add4(s1, v3); sq4(s2, v3);
     }
-  if (bn_partial<2>(v, C, cb, c0, gridDim.y, ws, sh)) {
+    for (; r < r1; r += rl_n) {
+      float4 v = __ldg(reinterpret_cast<const float4*>(xp + r * C));
+      add4(s1, v); sq4(s2, v);
+    }
+  }
+  if (bn_partial2(s1, s2, C, cg4, rl_n, ws, sh)) {
     if (rl == 0 && c < C) {
-      double t[2];
-      bn_combine<2>(t, C, c, gridDim.y, ws, cb);
-      double m = t[0] / (double)rows;
-      double var = t[1] / (double)rows - m * m;
-      if (var < 0) var = 0;
-      mean[c] = (float)m;
-      invstd[c] = (float)(1.0 / sqrt(var + (double)eps));
-      double unb = rows > 1 ? var * (double)rows / (double)(rows - 1) : var;
-      rm[c] = (float)((1.0 - momentum) * (double)rm[c] + momentum * m);
-      rv[c] = (float)((1.0 - momentum) * (double)rv[c] + momentum * unb);
+      for (int k = 0; k < 4; k++) {
+        double t0, t1;
+        bn_combine(&t0, &t1, C, c + k, gridDim.y, ws);
+        double m = t0 / (double)rows;
+        double var = t1 / (double)rows - m * m;
+        if (var < 0) var = 0;
+        mean[c + k] = (float)m;
+        invstd[c + k] = (float)(1.0 / sqrt(var + (double)eps));
+        double unb = rows > 1 ? var * (double)rows / (double)(rows - 1) : var;
+        rm[c + k] = (float)((1.0 - momentum) * (double)rm[c + k] + momentum * m);
+        rv[c + k] = (float)((1.0 - momentum) * (double)rv[c + k] + momentum * unb);
+      }
     }
   }
   orion_signal(sig);
@@ -100,28 +127,48 @@ __global__ void __launch_bounds__(BN_THREADS) bn_stats_kernel(const float* __res
 // ---- backward reduce: dbeta = sum dy, dgamma = sum dy * (x - mean) * invstd
 __global__ void __launch_bounds__(BN_THREADS) bn_bwd_reduce_kernel(const float* __restrict__ x, const float* __restrict__ dy,
                                                                    const float* __restrict__ mean, const float* __restrict__ invstd,
-                                                                   float* dgamma, float* dbeta, long long rows, int C, int cb,
+                                                                   float* dgamma, float* dbeta, long long rows, int C, int cg4, int rl_n,
                                                                    long long rows_per_split, unsigned char* ws, OrionSig sig) {
-  __shared__ double sh[BN_THREADS * 2];
-  const int rl_n = BN_THREADS / cb, cl = threadIdx.x % cb, rl = threadIdx.x / cb;
-  const int c0 = blockIdx.x * cb, c = c0 + cl;
+  __shared__ double sh[BN_THREADS * 8];
+  const int cq = threadIdx.x % cg4, rl = threadIdx.x / cg4;
+  const int c = (blockIdx.x * cg4 + cq) * 4;
   const long long r0 = blockIdx.y * rows_per_split, r1 = min(rows, r0 + rows_per_split);
-  double v[2] = {0.0, 0.0};
-  if (c < C) {
-    const double mu = mean[c], is = invstd[c];
-    for (long long r = r0 + rl; r < r1; r += rl_n) {
-      double g = (double)__ldg(dy + r * C + c);
-      double xh = ((double)__ldg(x + r * C + c) - mu) * is;
-      v[0] += g;
-      v[1] += g * xh;
+  D4 sg{0, 0, 0, 0}, sgx{0, 0, 0, 0};
+  if (c < C && rl < rl_n) {
+    const float4 mu = __ldg(reinterpret_cast<const float4*>(mean + c));
+    const float4 is = __ldg(reinterpret_cast<const float4*>(invstd + c));
+    const float* xp = x + c;
+    const float* gp = dy + c;
+    auto acc = [&](const float4& g, const float4& v) {
+      sg.x += g.x; sg.y += g.y; sg.z += g.z; sg.w += g.w;
+      sgx.x = fma((double)g.x, ((double)v.x - mu.x) * is.x, sgx.x);
+      sgx.y = fma((double)g.y, ((double)v.y - mu.y) * is.y, sgx.y);
+      sgx.z = fma((double)g.z, ((double)v.z - mu.z) * is.z, sgx.z);
+      sgx.w = fma((double)g.w, ((double)v.w - mu.w) * is.w, sgx.w);
+    };
+    long long r = r0 + rl;
+    for (; r + 3LL * rl_n < r1; r += 4LL * rl_n) {
+      float4 g0 = __ldg(reinterpret_cast<const float4*>(gp + r * C));
+      float4 g1 = __ldg(reinterpret_cast<const float4*>(gp + (r + rl_n) * C));
+      float4 g2 = __ldg(reinterpret_cast<const float4*>(gp + (r + 2LL * rl_n) * C));
+      float4 g3 = __ldg(reinterpret_cast<const float4*>(gp + (r + 3LL * rl_n) * C));
+      float4 v0 = __ldg(reinterpret_cast<const float4*>(xp + r * C));
+      float4 v1 = __ldg(reinterpret_cast<const float4*>(xp + (r + rl_n) * C));
+      float4 v2 = __ldg(reinterpret_cast<const float4*>(xp + (r + 2LL * rl_n) * C));
+      float4 v3 = __ldg(reinterpret_cast<const float4*>(xp + (r + 3LL * rl_n) * C));
+      acc(g0, v0); acc(g1, v1); acc(g2, v2); acc(g3, v3);
     }
+    for (; r < r1; r += rl_n)
+      acc(__ldg(reinterpret_cast<const float4*>(gp + r * C)), __ldg(reinterpret_cast<const float4*>(xp + r * C)));
   }
-  if (bn_partial<2>(v, C, cb, c0, gridDim.y, ws, sh)) {
+  if (bn_partial2(sg, sgx, C, cg4, rl_n, ws, sh)) {
     if (rl == 0 && c < C) {
-      double t[2];
-      bn_combine<2>(t, C, c, gridDim.y, ws, cb);
-      dbeta[c] = (float)t[0];
-      dgamma[c] = (float)t[1];
+      for (int k = 0; k < 4; k++) {
+        double t0, t1;
+        bn_combine(&t0, &t1, C, c + k, gridDim.y, ws);
+        dbeta[c + k] = (float)t0;
+        dgamma[c + k] = (float)t1;
+      }
     }
   }
   orion_signal(sig);
@@ -208,7 +255,7 @@ int bn_eval_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStr
 
 // BN stats: x, mean, invstd, rm, rv, rows, C, eps_bits, momentum_bits, ws, ws_bytes
 int bn_stats_geom(const uint64_t* a, LaunchGeom* g) {
-  if (a[9] == 0 || a[10] < bn_ws_bytes((long long)a[5], (int)a[6], 2)) return ORION_E_INVAL;
+  if ((a[6] & 3) || a[9] == 0 || a[10] < bn_ws_bytes((long long)a[5], (int)a[6], 2)) return ORION_E_INVAL;
   BnSplit sp = bn_split((long long)a[5], (int)a[6]);
   g->grid = dim3(sp.cblocks, sp.rs); g->block = dim3(BN_THREADS); g->smem = 0; g->func = (const void*)bn_stats_kernel;
   return 0;
@@ -216,7 +263,7 @@ int bn_stats_geom(const uint64_t* a, LaunchGeom* g) {
 int bn_stats_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   BnSplit sp = bn_split((long long)a[5], (int)a[6]);
   bn_stats_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (float*)a[1], (float*)a[2], (float*)a[3], (float*)a[4], (long long)a[5],
-                                             (int)a[6], u2f(a[7]), u2f(a[8]), sp.cb, sp.rows_per_split, (unsigned char*)a[9], sig);
+                                             (int)a[6], u2f(a[7]), u2f(a[8]), sp.cg4, sp.rl, sp.rows_per_split, (unsigned char*)a[9], sig);
   CHECK_LAUNCH();
 }
 
@@ -230,7 +277,7 @@ int bn_apply_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaSt
 
 // BN bwd reduce: x, dy, mean, invstd, dgamma, dbeta, rows, C, ws, ws_bytes
 int bn_bwd_reduce_geom(const uint64_t* a, LaunchGeom* g) {
-  if (a[8] == 0 || a[9] < bn_ws_bytes((long long)a[6], (int)a[7], 2)) return ORION_E_INVAL;
+  if ((a[7] & 3) || a[8] == 0 || a[9] < bn_ws_bytes((long long)a[6], (int)a[7], 2)) return ORION_E_INVAL;
   BnSplit sp = bn_split((long long)a[6], (int)a[7]);
   g->grid = dim3(sp.cblocks, sp.rs); g->block = dim3(BN_THREADS); g->smem = 0; g->func = (const void*)bn_bwd_reduce_kernel;
   return 0;
@@ -238,8 +285,8 @@ int bn_bwd_reduce_geom(const uint64_t* a, LaunchGeom* g) {
 int bn_bwd_reduce_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   BnSplit sp = bn_split((long long)a[6], (int)a[7]);
   bn_bwd_reduce_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (const float*)a[1], (const float*)a[2], (const float*)a[3],
-                                                  (float*)a[4], (float*)a[5], (long long)a[6], (int)a[7], sp.cb, sp.rows_per_split,
-                                                  (unsigned char*)a[8], sig);
+                                                  (float*)a[4], (float*)a[5], (long long)a[6], (int)a[7], sp.cg4, sp.rl,
+                                                  sp.rows_per_split, (unsigned char*)a[8], sig);
   CHECK_LAUNCH();
 }
 

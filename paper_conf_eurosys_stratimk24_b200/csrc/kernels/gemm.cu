@@ -10,7 +10,20 @@
 
 namespace {
 
-constexpr int BM = 128, BN = 128, BK = 8, NT = 256;
+constexpr int NT = 256;
+
+// Tile configurations (shape-selected, never SM-count-selected). Thread grid is always 16 x 16;
+// each thread owns a TM x TN sub-tile split in two halves (rows ty*TM/2.. and BM/2 + ty*TM/2..)
+// to keep shared-memory fragment reads conflict-free. Every thread loads 4 A and 4 B elements
+// per k-tile.
+template <int BM_, int BN_, int BK_>
+struct Tile {
+  static constexpr int BM = BM_, BN = BN_, BK = BK_, TM = BM_ / 16, TN = BN_ / 16;
+  static_assert(BM * BK == 4 * NT && BN * BK == 4 * NT, "4 loads per thread per operand");
+};
+using TileL = Tile<128, 128, 8>;   // 8x8 per thread: compute-dense problems
+using TileM = Tile<64, 64, 16>;    // 4x4 per thread
+using TileS = Tile<32, 32, 32>;    // 2x2 per thread: skinny / memory-bound (long-K wgrad)
 
 struct GemmParams {
   int M, N, K;
@@ -20,7 +33,7 @@ struct GemmParams {
   int split;           // number of K splits (grid.z)
   int kps;             // K elements per split (multiple of BK)
   float* ws;           // split partials [split][M][N] (split > 1)
-  unsigned int* tickets;  // one per output tile (split > 1), zero-initialised
+  unsigned int* tickets;  // one per output tile (split > 1), zero at rest
 };
 
 // ---------------------------------------------------------------- operand loaders
@@ -133,8 +146,22 @@ struct BWgrad {
 };
 
 // ---------------------------------------------------------------- the tiled main loop
-template <class LA, class LB>
+template <int N_>
+__device__ __forceinline__ void lds_frag(float* dst, const float* src) {
+  if constexpr (N_ == 4) {
+    float4 v = *reinterpret_cast<const float4*>(src);
+    dst[0] = v.x; dst[1] = v.y; dst[2] = v.z; dst[3] = v.w;
+  } else if constexpr (N_ == 2) {
+    float2 v = *reinterpret_cast<const float2*>(src);
+    dst[0] = v.x; dst[1] = v.y;
+  } else {
+    dst[0] = *src;
+  }
+}
+
+template <class T, class LA, class LB>
 __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, OrionSig sig) {
+  constexpr int BM = T::BM, BN = T::BN, BK = T::BK, TM = T::TM, TN = T::TN;
   __shared__ __align__(16) float As[2][BK][BM + 4];
   __shared__ __align__(16) float Bs[2][BK][BN + 4];
   const int tid = threadIdx.x;
@@ -142,14 +169,13 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
   const int kbeg = blockIdx.z * p.kps;
   const int kend = min(p.K, kbeg + p.kps);
 
-  // load mappings: 4 elements of A and 4 of B per thread per k-tile
   int a_m[4], a_k[4], b_n[4], b_k[4];
 #pragma unroll
   for (int i = 0; i < 4; i++) {
-    if (LA::kContigK) { a_k[i] = tid % BK; a_m[i] = tid / BK + 32 * i; }
-    else { a_m[i] = tid % BM; a_k[i] = tid / BM + 2 * i; }
-    if (LB::kContigK) { b_k[i] = tid % BK; b_n[i] = tid / BK + 32 * i; }
-    else { b_n[i] = tid % BN; b_k[i] = tid / BN + 2 * i; }
+    if (LA::kContigK) { a_k[i] = tid % BK; a_m[i] = tid / BK + (NT / BK) * i; }
+    else { a_m[i] = tid % BM; a_k[i] = tid / BM + (NT / BM) * i; }
+    if (LB::kContigK) { b_k[i] = tid % BK; b_n[i] = tid / BK + (NT / BK) * i; }
+    else { b_n[i] = tid % BN; b_k[i] = tid / BN + (NT / BN) * i; }
   }
   typename LA::Row arow[4];
   typename LB::Col bcol[4];
@@ -170,11 +196,11 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
     for (int i = 0; i < 4; i++) { As[buf][a_k[i]][a_m[i]] = ra[i]; Bs[buf][b_k[i]][b_n[i]] = rb[i]; }
   };
 
-  float acc[8][8];
+  float acc[TM][TN];
 #pragma unroll
-  for (int i = 0; i < 8; i++)
+  for (int i = 0; i < TM; i++)
 #pragma unroll
-    for (int j = 0; j < 8; j++) acc[i][j] = 0.f;
+    for (int j = 0; j < TN; j++) acc[i][j] = 0.f;
 
   const int ty = tid / 16, tx = tid % 16;
   int buf = 0;
@@ -188,16 +214,15 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
     if (more) gload(k0 + BK);
 #pragma unroll
     for (int kk = 0; kk < BK; kk++) {
-      float4 a0 = *reinterpret_cast<const float4*>(&As[buf][kk][ty * 4]);
-      float4 a1 = *reinterpret_cast<const float4*>(&As[buf][kk][64 + ty * 4]);
-      float4 b0 = *reinterpret_cast<const float4*>(&Bs[buf][kk][tx * 4]);
-      float4 b1 = *reinterpret_cast<const float4*>(&Bs[buf][kk][64 + tx * 4]);
-      float av[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-      float bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+      float av[TM], bv[TN];
+      lds_frag<TM / 2>(av, &As[buf][kk][ty * (TM / 2)]);
+      lds_frag<TM / 2>(av + TM / 2, &As[buf][kk][BM / 2 + ty * (TM / 2)]);
+      lds_frag<TN / 2>(bv, &Bs[buf][kk][tx * (TN / 2)]);
+      lds_frag<TN / 2>(bv + TN / 2, &Bs[buf][kk][BN / 2 + tx * (TN / 2)]);
 #pragma unroll
-      for (int i = 0; i < 8; i++)
+      for (int i = 0; i < TM; i++)
 #pragma unroll
-        for (int j = 0; j < 8; j++) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+        for (int j = 0; j < TN; j++) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
     }
     if (more) {
       sstore(buf ^ 1);
@@ -206,16 +231,15 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
     }
   }
 
-  // epilogue
-  auto out_row = [&](int i) { return m0 + (i < 4 ? ty * 4 + i : 64 + ty * 4 + (i - 4)); };
-  auto out_col = [&](int j) { return n0 + (j < 4 ? tx * 4 + j : 64 + tx * 4 + (j - 4)); };
+  auto out_row = [&](int i) { return m0 + (i < TM / 2 ? ty * (TM / 2) + i : BM / 2 + ty * (TM / 2) + (i - TM / 2)); };
+  auto out_col = [&](int j) { return n0 + (j < TN / 2 ? tx * (TN / 2) + j : BN / 2 + tx * (TN / 2) + (j - TN / 2)); };
   if (p.split == 1) {
 #pragma unroll
-    for (int i = 0; i < 8; i++) {
+    for (int i = 0; i < TM; i++) {
       int m = out_row(i);
       if (m >= p.M) continue;
 #pragma unroll
-      for (int j = 0; j < 8; j++) {
+      for (int j = 0; j < TN; j++) {
         int n = out_col(j);
         if (n < p.N) p.C[(long long)m * p.ldc + n] = acc[i][j] + (p.bias ? __ldg(p.bias + n) : 0.f);
       }
@@ -223,11 +247,11 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
   } else {
     float* part = p.ws + (long long)blockIdx.z * p.M * p.N;
 #pragma unroll
-    for (int i = 0; i < 8; i++) {
+    for (int i = 0; i < TM; i++) {
       int m = out_row(i);
       if (m >= p.M) continue;
 #pragma unroll
-      for (int j = 0; j < 8; j++) {
+      for (int j = 0; j < TN; j++) {
         int n = out_col(j);
         if (n < p.N) part[(long long)m * p.N + n] = acc[i][j];
       }
@@ -235,11 +259,11 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
     unsigned int* tk = p.tickets + blockIdx.y * gridDim.x + blockIdx.x;
     if (last_cta_of(tk, p.split)) {
 #pragma unroll
-      for (int i = 0; i < 8; i++) {
+      for (int i = 0; i < TM; i++) {
         int m = out_row(i);
         if (m >= p.M) continue;
 #pragma unroll
-        for (int j = 0; j < 8; j++) {
+        for (int j = 0; j < TN; j++) {
           int n = out_col(j);
           if (n >= p.N) continue;
           float s = 0.f;
@@ -304,51 +328,90 @@ __global__ void __launch_bounds__(256) gemv_bt_kernel(const float* __restrict__ 
   orion_signal(sig);
 }
 
-int choose_split(long long M, long long N, long long K) {
-  long long tiles = cdiv(M, BM) * cdiv(N, BN);
+// Shape-only plan: tile config and K split. Splits target ~4 waves of 148 SMs (a constant of the
+// part's size class, never the partition's SM count) so long-K problems (weight gradients over
+// N*H*W rows, 3x3 convs at batch 4) spread over the GPU; the split reduction is ordered.
+struct Plan { int cfg; int split; int bm, bn, bk; };
+
+Plan plan_gemm(long long M, long long N, long long K) {
+  Plan pl;
+  if (M >= 128 && N >= 128 && M * N >= 128LL * 128 * 64) { pl.cfg = 0; pl.bm = 128; pl.bn = 128; pl.bk = 8; }
+  else if (M >= 48 && N >= 48) { pl.cfg = 1; pl.bm = 64; pl.bn = 64; pl.bk = 16; }
+  else { pl.cfg = 2; pl.bm = 32; pl.bn = 32; pl.bk = 32; }
+  long long tiles = cdiv(M, pl.bm) * cdiv(N, pl.bn);
+  long long target = 592;
   long long split = 1;
-  // shape-only heuristic: aim for >= 2 waves of a 148-SM part, >= 256 K elements per split
-  while (tiles * split < 296 && K / (split * 2) >= 256 && split < 64) split *= 2;
-  return (int)split;
+  if (tiles < target) {
+    split = cdiv(target, tiles);
+    long long kmax = K / (4 * pl.bk);         // >= 4 k-tiles per split
+    if (split > kmax) split = kmax;
+    if (split > 512) split = 512;
+    if (split < 1) split = 1;
+  }
+  pl.split = (int)split;
+  return pl;
+}
+
+uint64_t ws_bytes_for(const Plan& pl, long long M, long long N) {
+  return pl.split > 1 ? WS_TICKET_BYTES + (uint64_t)pl.split * M * N * 4 : 0;
 }
 
 template <class LA, class LB>
-int launch_tiled(const LaunchGeom& g, GemmParams p, LA la, LB lb, OrionSig sig, cudaStream_t s) {
-  gemm_kernel<LA, LB><<<g.grid, g.block, 0, s>>>(p, la, lb, sig);
-  return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+const void* kernel_for(int cfg) {
+  switch (cfg) {
+    case 0: return (const void*)gemm_kernel<TileL, LA, LB>;
+    case 1: return (const void*)gemm_kernel<TileM, LA, LB>;
+    default: return (const void*)gemm_kernel<TileS, LA, LB>;
+  }
 }
 
-void tiled_geom(LaunchGeom* g, long long M, long long N, int split, const void* f) {
-  g->grid = dim3((unsigned)cdiv(N, BN), (unsigned)cdiv(M, BM), (unsigned)split);
+// Geometry of a tiled launch; falls back to split 1 when the caller's workspace is too small.
+template <class LA, class LB>
+void tiled_geom(LaunchGeom* g, long long M, long long N, long long K, uint64_t ws_ptr, uint64_t ws_bytes) {
+  Plan pl = plan_gemm(M, N, K);
+  if (pl.split > 1 && (ws_ptr == 0 || ws_bytes < ws_bytes_for(pl, M, N))) pl.split = 1;
+  g->grid = dim3((unsigned)cdiv(N, pl.bn), (unsigned)cdiv(M, pl.bm), (unsigned)pl.split);
   g->block = dim3(NT);
   g->smem = 0;
-  g->func = f;
+  g->func = kernel_for<LA, LB>(pl.cfg);
 }
 
 GemmParams make_params(long long M, long long N, long long K, float* C, long long ldc, const float* bias, int split,
-                       float* ws, long long ws_bytes) {
+                       float* ws, int bk) {
   GemmParams p;
   p.M = (int)M; p.N = (int)N; p.K = (int)K; p.C = C; p.ldc = ldc; p.bias = bias;
   p.split = split;
-  p.kps = (int)(cdiv(cdiv(K, split), BK) * BK);
-  p.ws = ws;
+  p.kps = (int)(cdiv(cdiv(K, split), bk) * bk);
+  p.ws = nullptr;
   p.tickets = nullptr;
-  if (split > 1) {
-    // workspace layout: [tickets (WS_TICKET_BYTES)][partials]
+  if (split > 1) {  // workspace layout: [tickets (WS_TICKET_BYTES)][partials]
     p.tickets = reinterpret_cast<unsigned int*>(ws);
     p.ws = reinterpret_cast<float*>(reinterpret_cast<char*>(ws) + WS_TICKET_BYTES);
-    (void)ws_bytes;
   }
   return p;
 }
 
+template <class LA, class LB>
+int launch_tiled(const LaunchGeom& g, long long M, long long N, long long K, float* C, long long ldc, const float* bias,
+                 float* ws, LA la, LB lb, OrionSig sig, cudaStream_t s) {
+  const int split = (int)g.grid.z;
+  if (g.func == (const void*)gemm_kernel<TileL, LA, LB>) {
+    gemm_kernel<TileL, LA, LB><<<g.grid, g.block, 0, s>>>(make_params(M, N, K, C, ldc, bias, split, ws, TileL::BK), la, lb, sig);
+  } else if (g.func == (const void*)gemm_kernel<TileM, LA, LB>) {
+    gemm_kernel<TileM, LA, LB><<<g.grid, g.block, 0, s>>>(make_params(M, N, K, C, ldc, bias, split, ws, TileM::BK), la, lb, sig);
+  } else {
+    gemm_kernel<TileS, LA, LB><<<g.grid, g.block, 0, s>>>(make_params(M, N, K, C, ldc, bias, split, ws, TileS::BK), la, lb, sig);
+  }
+  return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+}
+
 }  // namespace
 
-// Workspace bytes a split-K GEMM of this shape needs (tickets + partials); 0 if no split.
+// Workspace bytes a tiled GEMM of this (M, N, K) needs for its K split (0 if no split). Conv ops
+// pass their implicit-GEMM dims: fwd (N*P*Q, K, R*S*C), dgrad (N*H*W, C, R*S*K), wgrad (K, R*S*C, N*P*Q).
 extern "C" uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t K) {
-  int split = choose_split(M, N, K);
-  if (split == 1) return 0;
-  return WS_TICKET_BYTES + (uint64_t)split * M * N * 4;
+  Plan pl = plan_gemm((long long)M, (long long)N, (long long)K);
+  return ws_bytes_for(pl, (long long)M, (long long)N);
 }
 
 // ------------------------------------------------------------------------- GEMM entry
@@ -361,17 +424,13 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     g->grid = dim3((unsigned)cdiv(N, 8)); g->block = dim3(256); g->smem = 0; g->func = (const void*)gemv_bt_kernel;
     return 0;
   }
-  int split = choose_split(M, N, K);
-  if (split > 1 && (a[11] == 0 || a[12] < orion_gemm_workspace_bytes(M, N, K))) split = 1;
-  const void* f = nullptr;
   switch (flags) {
-    case 0: f = (const void*)gemm_kernel<ADense, BDense>; break;
-    case 1: f = (const void*)gemm_kernel<ADenseT, BDense>; break;
-    case 2: f = (const void*)gemm_kernel<ADense, BDenseT>; break;
-    case 3: f = (const void*)gemm_kernel<ADenseT, BDenseT>; break;
+    case 0: tiled_geom<ADense, BDense>(g, M, N, K, a[11], a[12]); break;
+    case 1: tiled_geom<ADenseT, BDense>(g, M, N, K, a[11], a[12]); break;
+    case 2: tiled_geom<ADense, BDenseT>(g, M, N, K, a[11], a[12]); break;
+    case 3: tiled_geom<ADenseT, BDenseT>(g, M, N, K, a[11], a[12]); break;
     default: return ORION_E_INVAL;
   }
-  tiled_geom(g, M, N, split, f);
   return 0;
 }
 
@@ -382,16 +441,16 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
   const float* bias = (const float*)a[3];
   long long M = a[4], N = a[5], K = a[6], lda = a[7], ldb = a[8], ldc = a[9];
   int flags = (int)a[10];
+  float* ws = (float*)a[11];
   if (g.func == (const void*)gemv_bt_kernel) {
     gemv_bt_kernel<<<g.grid, g.block, 0, s>>>(A, lda, B, ldb, C, ldc, bias, (int)M, (int)N, (int)K, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
-  GemmParams p = make_params(M, N, K, C, ldc, bias, (int)g.grid.z, (float*)a[11], (long long)a[12]);
   switch (flags) {
-    case 0: return launch_tiled(g, p, ADense{A, lda}, BDense{B, ldb}, sig, s);
-    case 1: return launch_tiled(g, p, ADenseT{A, lda}, BDense{B, ldb}, sig, s);
-    case 2: return launch_tiled(g, p, ADense{A, lda}, BDenseT{B, ldb}, sig, s);
-    case 3: return launch_tiled(g, p, ADenseT{A, lda}, BDenseT{B, ldb}, sig, s);
+    case 0: return launch_tiled(g, M, N, K, C, ldc, bias, ws, ADense{A, lda}, BDense{B, ldb}, sig, s);
+    case 1: return launch_tiled(g, M, N, K, C, ldc, bias, ws, ADenseT{A, lda}, BDense{B, ldb}, sig, s);
+    case 2: return launch_tiled(g, M, N, K, C, ldc, bias, ws, ADense{A, lda}, BDenseT{B, ldb}, sig, s);
+    case 3: return launch_tiled(g, M, N, K, C, ldc, bias, ws, ADenseT{A, lda}, BDenseT{B, ldb}, sig, s);
   }
   return ORION_E_INVAL;
 }
@@ -405,44 +464,40 @@ static ConvShape conv_shape(const uint64_t* a) {
   return s;
 }
 
+// implicit-GEMM dims: fwd (M = N*P*Q, N = K, K = R*S*C); dgrad (N*H*W, C, R*S*K); wgrad (K, R*S*C, N*P*Q)
 int conv_fwd_geom(const uint64_t* a, LaunchGeom* g) {
   ConvShape s = conv_shape(a);
-  long long M = (long long)s.N * s.P * s.Q, N = s.K;
-  tiled_geom(g, M, N, 1, (const void*)gemm_kernel<AIm2col, BDenseT>);
+  tiled_geom<AIm2col, BDenseT>(g, (long long)s.N * s.P * s.Q, s.K, (long long)s.R * s.S * s.C, a[14], a[15]);
   return 0;
 }
 int conv_fwd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   ConvShape s = conv_shape(a);
   long long M = (long long)s.N * s.P * s.Q, N = s.K, K = (long long)s.R * s.S * s.C;
-  GemmParams p = make_params(M, N, K, (float*)a[2], N, nullptr, 1, nullptr, 0);
-  return launch_tiled(g, p, AIm2col{(const float*)a[0], s}, BDenseT{(const float*)a[1], K}, sig, st);
+  return launch_tiled(g, M, N, K, (float*)a[2], N, nullptr, (float*)a[14], AIm2col{(const float*)a[0], s},
+                      BDenseT{(const float*)a[1], K}, sig, st);
 }
 
 int conv_dgrad_geom(const uint64_t* a, LaunchGeom* g) {
   ConvShape s = conv_shape(a);
-  long long M = (long long)s.N * s.H * s.W, N = s.C;
-  tiled_geom(g, M, N, 1, (const void*)gemm_kernel<ADgrad, BDgrad>);
+  tiled_geom<ADgrad, BDgrad>(g, (long long)s.N * s.H * s.W, s.C, (long long)s.R * s.S * s.K, a[14], a[15]);
   return 0;
 }
 int conv_dgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   ConvShape s = conv_shape(a);
   long long M = (long long)s.N * s.H * s.W, N = s.C, K = (long long)s.R * s.S * s.K;
-  GemmParams p = make_params(M, N, K, (float*)a[2], N, nullptr, 1, nullptr, 0);
-  return launch_tiled(g, p, ADgrad{(const float*)a[0], s}, BDgrad{(const float*)a[1], s}, sig, st);
+  return launch_tiled(g, M, N, K, (float*)a[2], N, nullptr, (float*)a[14], ADgrad{(const float*)a[0], s},
+                      BDgrad{(const float*)a[1], s}, sig, st);
 }
 
 int conv_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
   ConvShape s = conv_shape(a);
-  long long M = s.K, N = (long long)s.R * s.S * s.C, K = (long long)s.N * s.P * s.Q;
-  int split = choose_split(M, N, K);
-  if (split > 1 && (a[14] == 0 || a[15] < orion_gemm_workspace_bytes(M, N, K))) split = 1;
-  tiled_geom(g, M, N, split, (const void*)gemm_kernel<ADenseT, BWgrad>);
+  tiled_geom<ADenseT, BWgrad>(g, s.K, (long long)s.R * s.S * s.C, (long long)s.N * s.P * s.Q, a[14], a[15]);
   return 0;
 }
 int conv_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   ConvShape s = conv_shape(a);
   long long M = s.K, N = (long long)s.R * s.S * s.C, K = (long long)s.N * s.P * s.Q;
-  GemmParams p = make_params(M, N, K, (float*)a[2], N, nullptr, (int)g.grid.z, (float*)a[14], (long long)a[15]);
   // A(m = kout, k = npq) = dy[npq * K + kout]
-  return launch_tiled(g, p, ADenseT{(const float*)a[1], s.K}, BWgrad{(const float*)a[0], s}, sig, st);
+  return launch_tiled(g, M, N, K, (float*)a[2], N, nullptr, (float*)a[14], ADenseT{(const float*)a[1], s.K},
+                      BWgrad{(const float*)a[0], s}, sig, st);
 }

@@ -12,8 +12,8 @@ const KernelEntry g_kernels[ORION_FN_COUNT] = {
     E(add, add, 4),
     E(mse, mse, 6),
     E(sgd, sgd, 6),
-    E(conv_fwd, conv_fwd, 14),
-    E(conv_dgrad, conv_dgrad, 14),
+    E(conv_fwd, conv_fwd, 16),
+    E(conv_dgrad, conv_dgrad, 16),
     E(conv_wgrad, conv_wgrad, 16),
     E(dw_fwd, dw_fwd, 14),
     E(dw_dgrad, dw_dgrad, 14),

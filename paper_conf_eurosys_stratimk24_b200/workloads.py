@@ -117,7 +117,9 @@ def conv_fwd(g, x, w, y, stride, pad, label, depthwise=False):
         return g.k("dw_fwd", [_p(x), _p(w), _p(y)] + conv_args(x, w, y, stride, pad), label)
     if r == 1 and s == 1 and stride == 1 and pad == 0:   # 1x1 conv = GEMM [NHW, C] x [K, C]^T
         return gemm(g, x, w, y, None, n * h * wd, k, c, c, c, k, 2, label)
-    return g.k("conv_fwd", [_p(x), _p(w), _p(y)] + conv_args(x, w, y, stride, pad), label)
+    p_, q_ = y.shape[1], y.shape[2]
+    g.need_ws(L.lib.orion_gemm_workspace_bytes(n * p_ * q_, k, r * s * c))
+    return g.k("conv_fwd", [_p(x), _p(w), _p(y)] + conv_args(x, w, y, stride, pad) + [0, 0], label, ws_at=14)
 
 
 def conv_dgrad(g, dy, w, dx, stride, pad, label, depthwise=False):
@@ -127,7 +129,8 @@ def conv_dgrad(g, dy, w, dx, stride, pad, label, depthwise=False):
         return g.k("dw_dgrad", [_p(dy), _p(w), _p(dx)] + conv_args(dx, w, dy, stride, pad), label)
     if r == 1 and s == 1 and stride == 1 and pad == 0:   # dx[NHW, C] = dy[NHW, K] W[K, C]
         return gemm(g, dy, w, dx, None, n * h * wd, c, k, k, c, c, 0, label)
-    return g.k("conv_dgrad", [_p(dy), _p(w), _p(dx)] + conv_args(dx, w, dy, stride, pad), label)
+    g.need_ws(L.lib.orion_gemm_workspace_bytes(n * h * wd, c, r * s * k))
+    return g.k("conv_dgrad", [_p(dy), _p(w), _p(dx)] + conv_args(dx, w, dy, stride, pad) + [0, 0], label, ws_at=14)
 
 
 def conv_wgrad(g, x, dy, dw, stride, pad, label, depthwise=False):

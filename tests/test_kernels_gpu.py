@@ -38,6 +38,7 @@ def ws(nbytes):
 
 
 @pytest.mark.parametrize("M,N,K,flags", [(1, 512, 512, 2), (4, 1000, 2048, 2), (3, 37, 129, 2), (32, 512, 512, 2),
+                                         (96, 16, 300000, 1), (16, 32, 100000, 1), (196, 2048, 512, 2), (784, 256, 1024, 2),
                                          (200, 130, 77, 0), (300, 257, 65, 1), (129, 131, 700, 3), (96, 1000, 1280, 2),
                                          (1000, 1280, 96, 1), (64, 96, 20000, 1), (12544, 64, 256, 2)])
 def test_gemm(M, N, K, flags):
@@ -59,6 +60,8 @@ def test_gemm(M, N, K, flags):
 
 CONV_CASES = [  # N, H, W, C, K, R, stride, pad
     (2, 17, 15, 3, 32, 3, 2, 1),     # MobileNetV2 stem shape class
+    (4, 7, 7, 512, 512, 3, 1, 1),    # ResNet-50 layer4 3x3 at batch 4 (split-K)
+    (4, 14, 14, 256, 256, 3, 1, 1),  # layer3 3x3
     (4, 30, 30, 3, 64, 7, 2, 3),     # ResNet stem class
     (2, 14, 14, 64, 70, 3, 1, 1),
     (2, 13, 13, 64, 128, 1, 2, 0),   # 1x1 / stride 2 downsample
@@ -75,10 +78,12 @@ def test_conv_fwd_dgrad_wgrad(shape):
     dy = si.normal((n, p, q, k), 23)
     dims = [n, h, w_, c, k, r, r, st, pad, p, q]
     y = torch.zeros(n, p, q, k, device="cuda")
-    run("conv_fwd", [dev(x), dev(wt), y] + dims)
+    wf = ws(L.lib.orion_gemm_workspace_bytes(n * p * q, k, r * r * c))
+    run("conv_fwd", [dev(x), dev(wt), y] + dims + [wf, wf.numel() * 4])
     assert rel(y, om.conv2d_fwd(x, wt, st, pad)) < 1e-5
     dx = torch.zeros(n, h, w_, c, device="cuda")
-    run("conv_dgrad", [dev(dy), dev(wt), dx] + dims)
+    wd = ws(L.lib.orion_gemm_workspace_bytes(n * h * w_, c, r * r * k))
+    run("conv_dgrad", [dev(dy), dev(wt), dx] + dims + [wd, wd.numel() * 4])
     assert rel(dx, om.conv2d_bwd_data(dy, wt, (n, h, w_, c), st, pad)) < 1e-5
     dw = torch.zeros(k, r, r, c, device="cuda")
     wsb = ws(L.lib.orion_gemm_workspace_bytes(k, r * r * c, n * p * q))

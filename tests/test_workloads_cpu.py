@@ -17,7 +17,7 @@ def test_specs_match_oracle():
 
 
 NARGS = {"gemm": 13, "colsum": 4, "relu": 3, "relu_bwd": 4, "relu6": 3, "relu6_bwd": 4, "add": 4, "mse": 6, "sgd": 6,
-         "conv_fwd": 14, "conv_dgrad": 14, "conv_wgrad": 16, "dw_fwd": 14, "dw_dgrad": 14, "dw_wgrad": 16,
+         "conv_fwd": 16, "conv_dgrad": 16, "conv_wgrad": 16, "dw_fwd": 14, "dw_dgrad": 14, "dw_wgrad": 16,
          "bn_eval": 9, "bn_stats": 11, "bn_apply": 8, "bn_bwd_reduce": 10, "bn_bwd_dx": 10, "maxpool": 8,
          "avgpool": 5, "avgpool_bwd": 5, "ce": 7}
 
