@@ -178,10 +178,26 @@ __global__ void __launch_bounds__(BN_THREADS) bn_bwd_reduce_kernel(const float* 
 __global__ void __launch_bounds__(BN_THREADS) bn_eval_kernel(const float* __restrict__ x, float* __restrict__ y, const float* __restrict__ gamma,
                                                              const float* __restrict__ beta, const float* __restrict__ rm,
                                                              const float* __restrict__ rv, long long total, int C, float eps, OrionSig sig) {
-  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
-    int c = (int)(i % C);
-    float sc = gamma[c] * rsqrtf(rv[c] + eps);
-    y[i] = fmaf(x[i] - rm[c], sc, beta[c]);
+  if ((C & 3) == 0) {
+    const long long nv = total / 4;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nv; i += (long long)gridDim.x * blockDim.x) {
+      const int c = (int)((i * 4) % C);
+      float4 xv = __ldg(reinterpret_cast<const float4*>(x) + i);
+      float4 g = __ldg(reinterpret_cast<const float4*>(gamma + c)), b = __ldg(reinterpret_cast<const float4*>(beta + c));
+      float4 m = __ldg(reinterpret_cast<const float4*>(rm + c)), v = __ldg(reinterpret_cast<const float4*>(rv + c));
+      float4 o;
+      o.x = fmaf(xv.x - m.x, g.x * rsqrtf(v.x + eps), b.x);
+      o.y = fmaf(xv.y - m.y, g.y * rsqrtf(v.y + eps), b.y);
+      o.z = fmaf(xv.z - m.z, g.z * rsqrtf(v.z + eps), b.z);
+      o.w = fmaf(xv.w - m.w, g.w * rsqrtf(v.w + eps), b.w);
+      reinterpret_cast<float4*>(y)[i] = o;
+    }
+  } else {
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+      int c = (int)(i % C);
+      float sc = gamma[c] * rsqrtf(rv[c] + eps);
+      y[i] = fmaf(x[i] - rm[c], sc, beta[c]);
+    }
   }
   orion_signal(sig);
 }
@@ -214,21 +230,39 @@ __global__ void __launch_bounds__(BN_THREADS) bn_apply_kernel(const float* __res
   orion_signal(sig);
 }
 
-// dx = gamma*invstd/N * (N dy - dbeta - xhat dgamma)
+// dx = gamma*invstd/N (N dy - dbeta - xhat dgamma), evaluated in fp64 per element: dy and
+// (dbeta + xhat*dgamma)/N nearly cancel, and fp32 would amplify the rounding of each term through
+// every BN layer of the backward pass (memory-bound kernel: the fp64 math is free).
+__device__ __forceinline__ float bn_dx1(float x, float dy, float g, float m, float is, float dg, float db, double invN) {
+  double xh = ((double)x - (double)m) * (double)is;
+  return (float)((double)g * (double)is * ((double)dy - ((double)db + xh * (double)dg) * invN));
+}
 __global__ void __launch_bounds__(BN_THREADS) bn_bwd_dx_kernel(const float* __restrict__ x, const float* __restrict__ dy, float* __restrict__ dx,
                                                                const float* __restrict__ gamma, const float* __restrict__ mean,
                                                                const float* __restrict__ invstd, const float* __restrict__ dgamma,
                                                                const float* __restrict__ dbeta, long long rows, int C, OrionSig sig) {
-  // fp64 per element: dy and (dbeta + xhat*dgamma)/N nearly cancel, and fp32 would amplify the
-  // rounding of each term through every BN layer of the backward pass (memory-bound: free)
   const long long total = rows * C;
   const double invN = 1.0 / (double)rows;
-  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
-    int c = (int)(i % C);
-    double is = invstd[c];
-    double xh = ((double)x[i] - (double)mean[c]) * is;
-    double k = (double)gamma[c] * is;
-    dx[i] = (float)(k * ((double)dy[i] - ((double)dbeta[c] + xh * (double)dgamma[c]) * invN));
+  if ((C & 3) == 0) {
+    const long long nv = total / 4;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nv; i += (long long)gridDim.x * blockDim.x) {
+      const int c = (int)((i * 4) % C);
+      float4 xv = __ldg(reinterpret_cast<const float4*>(x) + i), gv = __ldg(reinterpret_cast<const float4*>(dy) + i);
+      float4 ga = __ldg(reinterpret_cast<const float4*>(gamma + c)), mu = __ldg(reinterpret_cast<const float4*>(mean + c));
+      float4 is = __ldg(reinterpret_cast<const float4*>(invstd + c)), dg = __ldg(reinterpret_cast<const float4*>(dgamma + c));
+      float4 db = __ldg(reinterpret_cast<const float4*>(dbeta + c));
+      float4 o;
+      o.x = bn_dx1(xv.x, gv.x, ga.x, mu.x, is.x, dg.x, db.x, invN);
+      o.y = bn_dx1(xv.y, gv.y, ga.y, mu.y, is.y, dg.y, db.y, invN);
+      o.z = bn_dx1(xv.z, gv.z, ga.z, mu.z, is.z, dg.z, db.z, invN);
+      o.w = bn_dx1(xv.w, gv.w, ga.w, mu.w, is.w, dg.w, db.w, invN);
+      reinterpret_cast<float4*>(dx)[i] = o;
+    }
+  } else {
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
+      int c = (int)(i % C);
+      dx[i] = bn_dx1(x[i], dy[i], gamma[c], mean[c], invstd[c], dgamma[c], dbeta[c], invN);
+    }
   }
   orion_signal(sig);
 }
@@ -246,7 +280,7 @@ extern "C" uint64_t orion_bn_workspace_bytes(uint64_t rows, uint64_t C) { return
 #define CHECK_LAUNCH() return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA
 
 // BN eval: x, y, gamma, beta, rm, rv, rows, C, eps_bits
-int bn_eval_geom(const uint64_t* a, LaunchGeom* g) { ew(g, a[6] * a[7], (const void*)bn_eval_kernel); return 0; }
+int bn_eval_geom(const uint64_t* a, LaunchGeom* g) { ew(g, (a[7] & 3) == 0 ? a[6] * a[7] / 4 : a[6] * a[7], (const void*)bn_eval_kernel); return 0; }
 int bn_eval_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   bn_eval_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (float*)a[1], (const float*)a[2], (const float*)a[3], (const float*)a[4],
                                             (const float*)a[5], (long long)(a[6] * a[7]), (int)a[7], u2f(a[8]), sig);
@@ -291,7 +325,7 @@ int bn_bwd_reduce_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, c
 }
 
 // BN bwd dx: x, dy, dx, gamma, mean, invstd, dgamma, dbeta, rows, C
-int bn_bwd_dx_geom(const uint64_t* a, LaunchGeom* g) { ew(g, a[8] * a[9], (const void*)bn_bwd_dx_kernel); return 0; }
+int bn_bwd_dx_geom(const uint64_t* a, LaunchGeom* g) { ew(g, (a[9] & 3) == 0 ? a[8] * a[9] / 4 : a[8] * a[9], (const void*)bn_bwd_dx_kernel); return 0; }
 int bn_bwd_dx_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   bn_bwd_dx_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (const float*)a[1], (float*)a[2], (const float*)a[3], (const float*)a[4],
                                               (const float*)a[5], (const float*)a[6], (const float*)a[7], (long long)a[8], (int)a[9], sig);
