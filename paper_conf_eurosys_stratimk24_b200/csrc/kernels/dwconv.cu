@@ -1,7 +1,8 @@
-// Depthwise 3x3 convolution (groups = C; MobileNetV2's memory-bound conv, "MobileNet-v2"),
-// NHWC activations, weights [C][3][3][1]. fwd / dgrad: one thread per 4 channels of an output
-// pixel (128-bit loads along C). wgrad: per-thread fp64 accumulation of the 9 taps over a row
-// split, fixed-order CTA combine, last CTA per channel block sums splits in order.
+// Depthwise 3x3 convolution (groups = C; MobileNetV2's memory-bound conv), NHWC activations,
+// weights [C][3][3][1]. fwd, stride-1 dgrad and wgrad slide a 3x3 register window along output
+// rows (one warp = 32 channels x one row); stride-2 dgrad gathers per output pixel (4 channels per
+// thread). wgrad reductions: fp32 per row, fp64 across rows, fixed-order CTA combine, ordered
+// split reduction by the last CTA per channel block.
 #include "common.cuh"
 
 namespace {
@@ -10,33 +11,173 @@ constexpr int DW_THREADS = 256;
 
 struct DwShape { int N, H, W, C, stride, P, Q; };
 
-__global__ void __launch_bounds__(DW_THREADS) dw_fwd_kernel(const float* __restrict__ x, const float* __restrict__ w, float* __restrict__ y,
-                                                            DwShape s, OrionSig sig) {
-  const int C4 = s.C / 4;
-  const long long total = (long long)s.N * s.P * s.Q * C4;
-  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
-    int c4 = (int)(i % C4); long long t = i / C4;
-    int q = (int)(t % s.Q); t /= s.Q;
-    int p = (int)(t % s.P); int n = (int)(t / s.P);
-    int c = c4 * 4;
-    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+// Row-sliding depthwise kernels: a warp owns 32 consecutive channels (128-byte coalesced rows of
+// the NHWC tensor) and one output row (n, p); each lane walks q = 0..Q-1 keeping a 3x3 window
+// of its input column values in registers, so each input element is loaded once per output row
+// that uses it (3x for the 3 kernel rows) instead of 9x. Weights live in registers.
+constexpr int ROW_WARPS = 8;
+
+__global__ void __launch_bounds__(DW_THREADS) dw_fwd_rows_kernel(const float* __restrict__ x, const float* __restrict__ w,
+                                                                 float* __restrict__ y, DwShape s, OrionSig sig) {
+  const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
+  const int cblocks = (s.C + 31) / 32;
+  const long long nrows = (long long)s.N * s.P;
+  for (long long item = (long long)blockIdx.x * ROW_WARPS + warp; item < nrows * cblocks; item += (long long)gridDim.x * ROW_WARPS) {
+    const int cb = (int)(item % cblocks);
+    const long long row = item / cblocks;
+    const int p = (int)(row % s.P), n = (int)(row / s.P);
+    const int c = cb * 32 + lane;
+    if (c >= s.C) continue;
+    float wr[9];
+#pragma unroll
+    for (int t = 0; t < 9; t++) wr[t] = __ldg(w + c * 9 + t);
+    const float* xr[3];
+    bool rv[3];
 #pragma unroll
     for (int r = 0; r < 3; r++) {
       int h = p * s.stride - 1 + r;
-      if ((unsigned)h >= (unsigned)s.H) continue;
-#pragma unroll
-      for (int u = 0; u < 3; u++) {
-        int ww = q * s.stride - 1 + u;
-        if ((unsigned)ww >= (unsigned)s.W) continue;
-        float4 xv = __ldg(reinterpret_cast<const float4*>(x + (((long long)n * s.H + h) * s.W + ww) * s.C + c));
-        int tap = r * 3 + u;
-        acc.x = fmaf(xv.x, __ldg(w + (c + 0) * 9 + tap), acc.x);
-        acc.y = fmaf(xv.y, __ldg(w + (c + 1) * 9 + tap), acc.y);
-        acc.z = fmaf(xv.z, __ldg(w + (c + 2) * 9 + tap), acc.z);
-        acc.w = fmaf(xv.w, __ldg(w + (c + 3) * 9 + tap), acc.w);
+      rv[r] = (unsigned)h < (unsigned)s.H;
+      xr[r] = x + (((long long)n * s.H + (rv[r] ? h : 0)) * s.W) * s.C + c;
+    }
+    auto ld = [&](int r, int col) -> float {
+      return (rv[r] && (unsigned)col < (unsigned)s.W) ? __ldg(xr[r] + (long long)col * s.C) : 0.f;
+    };
+    float* yr = y + (((long long)n * s.P + p) * s.Q) * s.C + c;
+    // window columns a (= q*st-1), b (= q*st), c2 (= q*st+1)
+    float a0 = ld(0, -1), a1 = ld(1, -1), a2 = ld(2, -1);
+    float b0 = ld(0, 0), b1 = ld(1, 0), b2 = ld(2, 0);
+    for (int q = 0; q < s.Q; q++) {
+      const int col = q * s.stride + 1;
+      float c0 = ld(0, col), c1 = ld(1, col), c2 = ld(2, col);
+      float acc = a0 * wr[0];
+      acc = fmaf(b0, wr[1], acc); acc = fmaf(c0, wr[2], acc);
+      acc = fmaf(a1, wr[3], acc); acc = fmaf(b1, wr[4], acc); acc = fmaf(c1, wr[5], acc);
+      acc = fmaf(a2, wr[6], acc); acc = fmaf(b2, wr[7], acc); acc = fmaf(c2, wr[8], acc);
+      yr[(long long)q * s.C] = acc;
+      if (s.stride == 1) {
+        a0 = b0; a1 = b1; a2 = b2; b0 = c0; b1 = c1; b2 = c2;
+      } else {  // stride 2: next window starts at col (q+1)*2-1 = current c column
+        a0 = c0; a1 = c1; a2 = c2;
+        b0 = ld(0, col + 1); b1 = ld(1, col + 1); b2 = ld(2, col + 1);
       }
     }
-    reinterpret_cast<float4*>(y)[i] = acc;
+  }
+  orion_signal(sig);
+}
+
+// Stride-1 dgrad is a correlation with the flipped kernel: dx(h, w) = sum_{r,u} dy(h+1-r, w+1-u) k(r,u).
+__global__ void __launch_bounds__(DW_THREADS) dw_dgrad_rows_s1_kernel(const float* __restrict__ dy, const float* __restrict__ w,
+                                                                      float* __restrict__ dx, DwShape s, OrionSig sig) {
+  const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
+  const int cblocks = (s.C + 31) / 32;
+  const long long nrows = (long long)s.N * s.H;
+  for (long long item = (long long)blockIdx.x * ROW_WARPS + warp; item < nrows * cblocks; item += (long long)gridDim.x * ROW_WARPS) {
+    const int cb = (int)(item % cblocks);
+    const long long row = item / cblocks;
+    const int h = (int)(row % s.H), n = (int)(row / s.H);
+    const int c = cb * 32 + lane;
+    if (c >= s.C) continue;
+    float wr[9];
+#pragma unroll
+    for (int t = 0; t < 9; t++) wr[t] = __ldg(w + c * 9 + t);
+    const float* gr[3];
+    bool rv[3];
+#pragma unroll
+    for (int r = 0; r < 3; r++) {   // kernel row r reads dy row p = h + 1 - r
+      int pp = h + 1 - r;
+      rv[r] = (unsigned)pp < (unsigned)s.P;
+      gr[r] = dy + (((long long)n * s.P + (rv[r] ? pp : 0)) * s.Q) * s.C + c;
+    }
+    auto ld = [&](int r, int col) -> float {
+      return (rv[r] && (unsigned)col < (unsigned)s.Q) ? __ldg(gr[r] + (long long)col * s.C) : 0.f;
+    };
+    float* dr = dx + (((long long)n * s.H + h) * s.W) * s.C + c;
+    // dx(h, wq) = sum_r sum_u dy(r-row, wq+1-u) k(r,u): columns wq+1 (u=0), wq (u=1), wq-1 (u=2)
+    float m0 = ld(0, -1), m1 = ld(1, -1), m2 = ld(2, -1);   // column wq-1
+    float z0 = ld(0, 0), z1 = ld(1, 0), z2 = ld(2, 0);      // column wq
+    for (int wq = 0; wq < s.W; wq++) {
+      float p0 = ld(0, wq + 1), p1 = ld(1, wq + 1), p2 = ld(2, wq + 1);
+      float acc = p0 * wr[0];
+      acc = fmaf(z0, wr[1], acc); acc = fmaf(m0, wr[2], acc);
+      acc = fmaf(p1, wr[3], acc); acc = fmaf(z1, wr[4], acc); acc = fmaf(m1, wr[5], acc);
+      acc = fmaf(p2, wr[6], acc); acc = fmaf(z2, wr[7], acc); acc = fmaf(m2, wr[8], acc);
+      dr[(long long)wq * s.C] = acc;
+      m0 = z0; m1 = z1; m2 = z2; z0 = p0; z1 = p1; z2 = p2;
+    }
+  }
+  orion_signal(sig);
+}
+
+// wgrad: a warp accumulates the 9 taps of its 32 channels over whole output rows with a sliding
+// window of x, in fp32 per row and fp64 across rows; warps combine in smem in fixed order, CTAs
+// write per-split partials, the last CTA of the channel block sums them in split order.
+__global__ void __launch_bounds__(DW_THREADS) dw_wgrad_rows_kernel(const float* __restrict__ x, const float* __restrict__ dy,
+                                                                   float* __restrict__ dw, DwShape s, unsigned char* ws, OrionSig sig) {
+  __shared__ double sh[ROW_WARPS][9][32];
+  const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
+  const int c = blockIdx.x * 32 + lane;
+  const long long nrows = (long long)s.N * s.P;
+  double acc[9];
+#pragma unroll
+  for (int t = 0; t < 9; t++) acc[t] = 0.0;
+  if (c < s.C) {
+    for (long long row = (long long)blockIdx.y * ROW_WARPS + warp; row < nrows; row += (long long)gridDim.y * ROW_WARPS) {
+      const int p = (int)(row % s.P), n = (int)(row / s.P);
+      const float* xr[3];
+      bool rv[3];
+#pragma unroll
+      for (int r = 0; r < 3; r++) {
+        int h = p * s.stride - 1 + r;
+        rv[r] = (unsigned)h < (unsigned)s.H;
+        xr[r] = x + (((long long)n * s.H + (rv[r] ? h : 0)) * s.W) * s.C + c;
+      }
+      auto ld = [&](int r, int col) -> float {
+        return (rv[r] && (unsigned)col < (unsigned)s.W) ? __ldg(xr[r] + (long long)col * s.C) : 0.f;
+      };
+      const float* gr = dy + (((long long)n * s.P + p) * s.Q) * s.C + c;
+      float f[9];
+#pragma unroll
+      for (int t = 0; t < 9; t++) f[t] = 0.f;
+      float a0 = ld(0, -1), a1 = ld(1, -1), a2 = ld(2, -1);
+      float b0 = ld(0, 0), b1 = ld(1, 0), b2 = ld(2, 0);
+      for (int q = 0; q < s.Q; q++) {
+        const int col = q * s.stride + 1;
+        float c0 = ld(0, col), c1 = ld(1, col), c2 = ld(2, col);
+        float g = __ldg(gr + (long long)q * s.C);
+        f[0] = fmaf(g, a0, f[0]); f[1] = fmaf(g, b0, f[1]); f[2] = fmaf(g, c0, f[2]);
+        f[3] = fmaf(g, a1, f[3]); f[4] = fmaf(g, b1, f[4]); f[5] = fmaf(g, c1, f[5]);
+        f[6] = fmaf(g, a2, f[6]); f[7] = fmaf(g, b2, f[7]); f[8] = fmaf(g, c2, f[8]);
+        if (s.stride == 1) {
+          a0 = b0; a1 = b1; a2 = b2; b0 = c0; b1 = c1; b2 = c2;
+        } else {
+          a0 = c0; a1 = c1; a2 = c2;
+          b0 = ld(0, col + 1); b1 = ld(1, col + 1); b2 = ld(2, col + 1);
+        }
+      }
+#pragma unroll
+      for (int t = 0; t < 9; t++) acc[t] += (double)f[t];
+    }
+  }
+#pragma unroll
+  for (int t = 0; t < 9; t++) sh[warp][t][lane] = acc[t];
+  __syncthreads();
+  unsigned int* tickets = reinterpret_cast<unsigned int*>(ws);
+  double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
+  if (warp == 0 && c < s.C) {
+    for (int t = 0; t < 9; t++) {
+      double v = 0.0;
+      for (int wv = 0; wv < ROW_WARPS; wv++) v += sh[wv][t][lane];
+      part[((long long)blockIdx.y * s.C + c) * 9 + t] = v;
+    }
+  }
+  if (last_cta_of(tickets + blockIdx.x, gridDim.y)) {
+    if (warp == 0 && c < s.C) {
+      for (int t = 0; t < 9; t++) {
+        double v = 0.0;
+        for (unsigned r = 0; r < gridDim.y; r++) v += __ldcg(part + ((long long)r * s.C + c) * 9 + t);
+        dw[c * 9 + t] = (float)v;
+      }
+    }
   }
   orion_signal(sig);
 }
@@ -77,60 +218,6 @@ __global__ void __launch_bounds__(DW_THREADS) dw_dgrad_kernel(const float* __res
   orion_signal(sig);
 }
 
-// dw[c, r, u] = sum_{n,p,q} dy[n,p,q,c] x[n, p*st-1+r, q*st-1+u, c]
-constexpr int WG_CB = 32;  // channels per CTA (one per lane), 8 position-lanes
-__global__ void __launch_bounds__(DW_THREADS) dw_wgrad_kernel(const float* __restrict__ x, const float* __restrict__ dy, float* __restrict__ dw,
-                                                              DwShape s, long long pos_per_split, unsigned char* ws, OrionSig sig) {
-  __shared__ double sh[DW_THREADS][9];
-  const int cl = threadIdx.x % WG_CB, pl = threadIdx.x / WG_CB, PL = DW_THREADS / WG_CB;
-  const int c = blockIdx.x * WG_CB + cl;
-  const long long npos = (long long)s.N * s.P * s.Q;
-  const long long p0 = blockIdx.y * pos_per_split, p1 = min(npos, p0 + pos_per_split);
-  double acc[9];
-#pragma unroll
-  for (int j = 0; j < 9; j++) acc[j] = 0.0;
-  if (c < s.C) {
-    for (long long pos = p0 + pl; pos < p1; pos += PL) {
-      int q = (int)(pos % s.Q); long long t = pos / s.Q;
-      int p = (int)(t % s.P); int n = (int)(t / s.P);
-      float g = __ldg(dy + pos * s.C + c);
-#pragma unroll
-      for (int r = 0; r < 3; r++) {
-        int h = p * s.stride - 1 + r;
-        if ((unsigned)h >= (unsigned)s.H) continue;
-#pragma unroll
-        for (int u = 0; u < 3; u++) {
-          int ww = q * s.stride - 1 + u;
-          if ((unsigned)ww >= (unsigned)s.W) continue;
-          acc[r * 3 + u] += (double)g * (double)__ldg(x + (((long long)n * s.H + h) * s.W + ww) * s.C + c);
-        }
-      }
-    }
-  }
-#pragma unroll
-  for (int j = 0; j < 9; j++) sh[threadIdx.x][j] = acc[j];
-  __syncthreads();
-  unsigned int* tickets = reinterpret_cast<unsigned int*>(ws);
-  double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
-  if (pl == 0 && c < s.C) {
-    for (int j = 0; j < 9; j++) {
-      double t = 0.0;
-      for (int r = 0; r < PL; r++) t += sh[r * WG_CB + cl][j];
-      part[((long long)blockIdx.y * s.C + c) * 9 + j] = t;
-    }
-  }
-  if (last_cta_of(tickets + blockIdx.x, gridDim.y)) {
-    if (pl == 0 && c < s.C) {
-      for (int j = 0; j < 9; j++) {
-        double t = 0.0;
-        for (unsigned r = 0; r < gridDim.y; r++) t += __ldcg(part + ((long long)r * s.C + c) * 9 + j);
-        dw[c * 9 + j] = (float)t;
-      }
-    }
-  }
-  orion_signal(sig);
-}
-
 DwShape dw_shape(const uint64_t* a) {
   // args: x|dy, w|dy, y|dx|dw, N, H, W, C, K(=C), R(=3), S(=3), stride, pad(=1), P, Q, [ws, ws_bytes]
   DwShape s;
@@ -145,26 +232,27 @@ void ew(LaunchGeom* g, uint64_t n, const void* f) {
   g->grid = dim3((unsigned)ctas); g->block = dim3(DW_THREADS); g->smem = 0; g->func = f;
 }
 
-struct WgSplit { int cblocks, rs; long long per; };
-WgSplit wg_split(const DwShape& s) {
-  WgSplit w;
-  w.cblocks = (s.C + WG_CB - 1) / WG_CB;
-  long long npos = (long long)s.N * s.P * s.Q;
-  long long rs = cdiv(296, w.cblocks);
-  long long max_rs = cdiv(npos, 256);
+void rows_geom(LaunchGeom* g, long long items, const void* f) {
+  long long ctas = cdiv(items, ROW_WARPS);
+  if (ctas > 148 * 8) ctas = 148 * 8;
+  if (ctas < 1) ctas = 1;
+  g->grid = dim3((unsigned)ctas); g->block = dim3(DW_THREADS); g->smem = 0; g->func = f;
+}
+
+int wg_splits(const DwShape& s) {
+  long long cblocks = (s.C + 31) / 32;
+  long long rs = cdiv(148 * 8, cblocks);
+  long long max_rs = cdiv((long long)s.N * s.P, ROW_WARPS);
   if (rs > max_rs) rs = max_rs;
   if (rs < 1) rs = 1;
-  w.rs = (int)rs;
-  w.per = cdiv(npos, rs);
-  return w;
+  return (int)rs;
 }
 
 }  // namespace
 
 extern "C" uint64_t orion_dw_wgrad_workspace_bytes(uint64_t N, uint64_t C, uint64_t P, uint64_t Q) {
   DwShape s{(int)N, 0, 0, (int)C, 1, (int)P, (int)Q};
-  WgSplit w = wg_split(s);
-  return WS_TICKET_BYTES + (uint64_t)w.rs * C * 9 * 8;
+  return WS_TICKET_BYTES + (uint64_t)wg_splits(s) * C * 9 * 8;
 }
 
 #define CHECK_LAUNCH() return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA
@@ -172,21 +260,25 @@ extern "C" uint64_t orion_dw_wgrad_workspace_bytes(uint64_t N, uint64_t C, uint6
 int dw_fwd_geom(const uint64_t* a, LaunchGeom* g) {
   if (!dw_ok(a)) return ORION_E_INVAL;
   DwShape s = dw_shape(a);
-  ew(g, (uint64_t)s.N * s.P * s.Q * (s.C / 4), (const void*)dw_fwd_kernel);
+  rows_geom(g, (long long)s.N * s.P * ((s.C + 31) / 32), (const void*)dw_fwd_rows_kernel);
   return 0;
 }
 int dw_fwd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
-  dw_fwd_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
+  dw_fwd_rows_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
   CHECK_LAUNCH();
 }
 int dw_dgrad_geom(const uint64_t* a, LaunchGeom* g) {
   if (!dw_ok(a)) return ORION_E_INVAL;
   DwShape s = dw_shape(a);
-  ew(g, (uint64_t)s.N * s.H * s.W * (s.C / 4), (const void*)dw_dgrad_kernel);
+  if (s.stride == 1) rows_geom(g, (long long)s.N * s.H * ((s.C + 31) / 32), (const void*)dw_dgrad_rows_s1_kernel);
+  else ew(g, (uint64_t)s.N * s.H * s.W * (s.C / 4), (const void*)dw_dgrad_kernel);
   return 0;
 }
 int dw_dgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
-  dw_dgrad_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
+  if (g.func == (const void*)dw_dgrad_rows_s1_kernel)
+    dw_dgrad_rows_s1_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
+  else
+    dw_dgrad_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
   CHECK_LAUNCH();
 }
 // wgrad args: x, dy, dw, N, H, W, C, C, 3, 3, stride, 1, P, Q, ws, ws_bytes
@@ -194,13 +286,11 @@ int dw_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
   if (!dw_ok(a)) return ORION_E_INVAL;
   DwShape s = dw_shape(a);
   if (a[14] == 0 || a[15] < orion_dw_wgrad_workspace_bytes(s.N, s.C, s.P, s.Q)) return ORION_E_INVAL;
-  WgSplit w = wg_split(s);
-  g->grid = dim3(w.cblocks, w.rs); g->block = dim3(DW_THREADS); g->smem = 0; g->func = (const void*)dw_wgrad_kernel;
+  g->grid = dim3((s.C + 31) / 32, wg_splits(s)); g->block = dim3(DW_THREADS); g->smem = 0; g->func = (const void*)dw_wgrad_rows_kernel;
   return 0;
 }
 int dw_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
-  DwShape s = dw_shape(a);
-  WgSplit w = wg_split(s);
-  dw_wgrad_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s, w.per, (unsigned char*)a[14], sig);
+  dw_wgrad_rows_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a),
+                                                   (unsigned char*)a[14], sig);
   CHECK_LAUNCH();
 }
