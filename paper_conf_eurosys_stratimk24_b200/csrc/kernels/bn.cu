@@ -23,8 +23,8 @@ BnSplit bn_split(long long rows, int C) {
   s.cg4 = q < 64 ? q : 64;
   s.rl = BN_THREADS / s.cg4;
   s.cblocks = (int)cdiv(q, s.cg4);
-  long long rs = cdiv(148 * 8, s.cblocks);      // shape-only: ~one full wave of 8 CTAs per SM on 148 SMs
-  long long max_rs = cdiv(rows, 4LL * s.rl);    // >= 4 rows per row lane
+  long long rs = cdiv(148 * 4, s.cblocks);      // shape-only: ~4 CTAs per SM of a 148-SM part
+  long long max_rs = cdiv(rows, 32LL * s.rl);   // >= 32 rows per row lane (8 unrolled trips)
   if (rs > max_rs) rs = max_rs;
   if (rs < 1) rs = 1;
   if (rs > 2048) rs = 2048;
@@ -70,15 +70,43 @@ __device__ bool bn_partial2(const D4& a, const D4& b, int C, int cg4, int rl_n, 
   return last_cta_of(tickets + blockIdx.x, gridDim.y);
 }
 
-__device__ void bn_combine(double* t0, double* t1, int C, int c, int rs_count, unsigned char* ws) {
+// Parallel ordered combine in the last CTA: each of the CTA's CB = 4*cg4 channels gets
+// T = 256/CB threads; thread j sums splits j, j+T, j+2T, ... in order, then the T partial sums
+// are added in thread order. Fixed by shape, so deterministic. Results for channel
+// (blockIdx.x*cg4 + cq)*4 + k land in tot[(cq*4 + k)*2 + {0,1}] (smem, valid after return).
+__device__ void bn_combine_all(double* tot, double* sh, int C, int cg4, int rs_count, unsigned char* ws) {
   const double* part = reinterpret_cast<const double*>(ws + WS_TICKET_BYTES);
+  const int CB = 4 * cg4;
+  const int T = BN_THREADS / CB;
+  const int tid = threadIdx.x;
+  const int ch = tid % CB, j = tid / CB;
+  const int c = blockIdx.x * CB + ch;
   double a = 0.0, b = 0.0;
-  for (int r = 0; r < rs_count; r++) {
-    a += __ldcg(part + ((long long)r * C + c) * 2 + 0);
-    b += __ldcg(part + ((long long)r * C + c) * 2 + 1);
+  if (j < T && c < C) {
+    int r = j;
+    for (; r + 3 * T < rs_count; r += 4 * T) {   // 4 independent loads in flight, fixed order
+      double a0 = __ldcg(part + ((long long)r * C + c) * 2), b0 = __ldcg(part + ((long long)r * C + c) * 2 + 1);
+      double a1 = __ldcg(part + ((long long)(r + T) * C + c) * 2), b1 = __ldcg(part + ((long long)(r + T) * C + c) * 2 + 1);
+      double a2 = __ldcg(part + ((long long)(r + 2 * T) * C + c) * 2), b2 = __ldcg(part + ((long long)(r + 2 * T) * C + c) * 2 + 1);
+      double a3 = __ldcg(part + ((long long)(r + 3 * T) * C + c) * 2), b3 = __ldcg(part + ((long long)(r + 3 * T) * C + c) * 2 + 1);
+      a += a0; a += a1; a += a2; a += a3;
+      b += b0; b += b1; b += b2; b += b3;
+    }
+    for (; r < rs_count; r += T) {
+      a += __ldcg(part + ((long long)r * C + c) * 2);
+      b += __ldcg(part + ((long long)r * C + c) * 2 + 1);
+    }
   }
-  *t0 = a;
-  *t1 = b;
+  __syncthreads();
+  if (j < T) { sh[(j * CB + ch) * 2] = a; sh[(j * CB + ch) * 2 + 1] = b; }
+  __syncthreads();
+  if (j == 0) {
+    double ta = 0.0, tb = 0.0;
+    for (int k = 0; k < T; k++) { ta += sh[(k * CB + ch) * 2]; tb += sh[(k * CB + ch) * 2 + 1]; }
+    tot[ch * 2] = ta;
+    tot[ch * 2 + 1] = tb;
+  }
+  __syncthreads();
 }
 
 // ---- train statistics: mean, invstd (biased var), running stats (unbiased var, momentum)
@@ -105,11 +133,12 @@ __global__ void __launch_bounds__(BN_THREADS) bn_stats_kernel(const float* __res
       add4(s1, v); sq4(s2, v);
     }
   }
+  __shared__ double tot[BN_THREADS * 2];
   if (bn_partial2(s1, s2, C, cg4, rl_n, ws, sh)) {
+    bn_combine_all(tot, sh, C, cg4, gridDim.y, ws);
     if (rl == 0 && c < C) {
       for (int k = 0; k < 4; k++) {
-        double t0, t1;
-        bn_combine(&t0, &t1, C, c + k, gridDim.y, ws);
+        double t0 = tot[(cq * 4 + k) * 2], t1 = tot[(cq * 4 + k) * 2 + 1];
         double m = t0 / (double)rows;
         double var = t1 / (double)rows - m * m;
         if (var < 0) var = 0;
@@ -161,11 +190,12 @@ __global__ void __launch_bounds__(BN_THREADS) bn_bwd_reduce_kernel(const float* 
     for (; r < r1; r += rl_n)
       acc(__ldg(reinterpret_cast<const float4*>(gp + r * C)), __ldg(reinterpret_cast<const float4*>(xp + r * C)));
   }
+  __shared__ double tot[BN_THREADS * 2];
   if (bn_partial2(sg, sgx, C, cg4, rl_n, ws, sh)) {
+    bn_combine_all(tot, sh, C, cg4, gridDim.y, ws);
     if (rl == 0 && c < C) {
       for (int k = 0; k < 4; k++) {
-        double t0, t1;
-        bn_combine(&t0, &t1, C, c + k, gridDim.y, ws);
+        double t0 = tot[(cq * 4 + k) * 2], t1 = tot[(cq * 4 + k) * 2 + 1];
         dbeta[c + k] = (float)t0;
         dgamma[c + k] = (float)t1;
       }

@@ -6,6 +6,8 @@
 // Determinism: each output element is accumulated by one thread in k order; split-K partials are
 // reduced by the last CTA of each tile in split order; the split count is a function of the
 // shape only (never of the SM partition), so results are identical solo and collocated.
+#include <atomic>
+
 #include "common.cuh"
 
 namespace {
@@ -266,8 +268,17 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
         for (int j = 0; j < TN; j++) {
           int n = out_col(j);
           if (n >= p.N) continue;
+          // ordered sum over splits, 4 loads in flight: ((s + p0) + p1) + p2 ...
+          const float* q = p.ws + (long long)m * p.N + n;
+          const long long stride = (long long)p.M * p.N;
           float s = 0.f;
-          for (int z = 0; z < p.split; z++) s += __ldcg(p.ws + (long long)z * p.M * p.N + (long long)m * p.N + n);
+          int z = 0;
+          for (; z + 3 < p.split; z += 4) {
+            float v0 = __ldcg(q + z * stride), v1 = __ldcg(q + (z + 1) * stride);
+            float v2 = __ldcg(q + (z + 2) * stride), v3 = __ldcg(q + (z + 3) * stride);
+            s += v0; s += v1; s += v2; s += v3;
+          }
+          for (; z < p.split; z++) s += __ldcg(q + z * stride);
           p.C[(long long)m * p.ldc + n] = s + (p.bias ? __ldg(p.bias + n) : 0.f);
         }
       }
@@ -275,6 +286,243 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
   }
   orion_signal(sig);
 }
+
+// ---------------------------------------------------------------- tcgen05 path (sm_100a)
+// fp32 GEMM on the 5th-generation tensor cores with a 3xTF32 split: every operand
+// x = hi + lo with hi = rna_tf32(x), lo = x - hi, and D += A_lo B_hi + A_hi B_lo + A_hi B_hi per
+// k-step (kind::tf32, fp32 accumulators in TMEM). This keeps fp32-level accuracy (~2^-21 relative
+// per product) where plain TF32 would miss the 1e-4 parity bar.
+// Warp roles (160 threads): warps 0-3 stage operands (loader -> hi/lo split -> UMMA K-major
+// SWIZZLE_NONE core-matrix layout in shared memory) and later run the epilogue (TMEM lanes
+// 32w..32w+31 -> registers -> global); warp 4 owns TMEM and one elected lane issues tcgen05.mma,
+// releasing each stage with tcgen05.commit onto an mbarrier. The operand loaders are the same
+// im2col / transposed-view functors as the FFMA path, so every conv kind runs on this kernel.
+namespace tc {
+
+constexpr int BM = 128, BK = 32, NPROD = 128, NTHR = 160;
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint32_t a, uint32_t cnt) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(cnt) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t a) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(a) : "memory");
+}
+__device__ __forceinline__ bool mbar_try(uint32_t a, uint32_t parity) {
+  uint32_t ok;
+  asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+               : "=r"(ok) : "r"(a), "r"(parity) : "memory");
+  return ok != 0;
+}
+__device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity) { while (!mbar_try(a, parity)) {} }
+__device__ __forceinline__ float tf32_rna(float x) {
+  uint32_t u;
+  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(u) : "f"(x));
+  return __uint_as_float(u);
+}
+// UMMA shared-memory descriptor, K-major, no swizzle: LBO = byte stride between the two 16-byte
+// K halves of an 8x(32 B) core-matrix pair, SBO = byte stride between 8-row groups; version 1.
+__device__ __forceinline__ uint64_t sdesc(uint32_t addr, uint32_t lbo, uint32_t sbo) {
+  return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) | ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) |
+         (1ull << 46);
+}
+__device__ __forceinline__ void mma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}"
+               ::"r"(d), "l"(a), "l"(b), "r"(idesc), "r"(acc) : "memory");
+}
+__device__ __forceinline__ void mma_commit(uint32_t mbar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(mbar) : "memory");
+}
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
+  uint32_t r[32];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
+        "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]),
+        "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+        "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+#pragma unroll
+  for (int i = 0; i < 32; i++) v[i] = __uint_as_float(r[i]);
+}
+
+template <int BN>
+struct TcCfg {
+  static constexpr int STAGES = BN >= 128 ? 3 : 4;
+  static constexpr int A_BYTES = BM * BK * 4;   // one of hi / lo
+  static constexpr int B_BYTES = BN * BK * 4;
+  static constexpr int STAGE_BYTES = 2 * (A_BYTES + B_BYTES);
+  static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 256;
+  static constexpr int TMEM_COLS = BN < 32 ? 32 : BN;
+  // instruction descriptor: D f32 (bits 4-5 = 1), A/B tf32 (2 at bits 7-9 / 10-12), K-major A/B,
+  // N>>3 at bits 17-22, M>>4 at bits 24-28
+  static constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+};
+
+// Byte offset of the 4 consecutive k (quad kq of the 32-k tile) of operand row `row` in a stage
+// buffer of `rows` rows: k-chunk j = kq/2 (one MMA K-step of 8 tf32, rows x 32 B), then the
+// core-matrix layout ((8 rows, row groups), 2 halves): row group stride SBO = 256 B, half stride
+// LBO = 128 B, row stride 16 B inside a core matrix.
+__device__ __forceinline__ uint32_t elem_off(int row, int kq, int rows) {
+  return (uint32_t)((kq >> 1) * (rows * 32) + (row >> 3) * 256 + (kq & 1) * 128 + (row & 7) * 16);
+}
+
+template <int BN, class LA, class LB>
+__global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, LB lb, OrionSig sig) {
+  using Cfg = TcCfg<BN>;
+  extern __shared__ __align__(1024) unsigned char smem_raw[];
+  unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + Cfg::STAGES * Cfg::STAGE_BYTES);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * Cfg::STAGES + 1);
+  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + Cfg::STAGES), done_bar = smem_u32(bars + 2 * Cfg::STAGES);
+  const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
+  const int m0 = blockIdx.y * BM, n0 = blockIdx.x * BN;
+  const int kbeg = blockIdx.z * p.kps;
+  const int kend = min(p.K, kbeg + p.kps);
+  const int nk = kend > kbeg ? (kend - kbeg + BK - 1) / BK : 0;
+
+  if (tid == 0) {
+    for (int s = 0; s < Cfg::STAGES; s++) { mbar_init(full0 + 8 * s, NPROD); mbar_init(empty0 + 8 * s, 1); }
+    mbar_init(done_bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 4) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)), "r"(Cfg::TMEM_COLS) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp < 4) {
+    // ---------------- producers: row-per-thread staging of A (128 rows) and B (BN rows)
+    const int arow_i = tid;                      // A row m0 + tid
+    typename LA::Row arow = la.row(m0 + arow_i, p.M);
+    constexpr int BROWS = (BN + NPROD - 1) / NPROD;
+    typename LB::Col bcol[BROWS];
+#pragma unroll
+    for (int j = 0; j < BROWS; j++) bcol[j] = lb.col(n0 + tid + j * NPROD, p.N);
+    for (int kt = 0; kt < nk; kt++) {
+      const int s = kt % Cfg::STAGES;
+      const uint32_t ph = (uint32_t)(kt / Cfg::STAGES) & 1u;
+      mbar_wait(empty0 + 8 * s, ph ^ 1u);
+      unsigned char* st = smem + s * Cfg::STAGE_BYTES;
+      unsigned char* a_hi = st;
+      unsigned char* a_lo = st + Cfg::A_BYTES;
+      unsigned char* b_hi = st + 2 * Cfg::A_BYTES;
+      unsigned char* b_lo = b_hi + Cfg::B_BYTES;
+      const int k0 = kbeg + kt * BK;
+#pragma unroll
+      for (int kq = 0; kq < BK / 4; kq++) {     // 8 quads of 4 consecutive k
+        float4 h, l;
+        float v[4];
+#pragma unroll
+        for (int e = 0; e < 4; e++) { int k = k0 + kq * 4 + e; v[e] = k < kend ? la.at(arow, k, p.K) : 0.f; }
+        h.x = tf32_rna(v[0]); h.y = tf32_rna(v[1]); h.z = tf32_rna(v[2]); h.w = tf32_rna(v[3]);
+        l.x = v[0] - h.x; l.y = v[1] - h.y; l.z = v[2] - h.z; l.w = v[3] - h.w;
+        const uint32_t off = elem_off(arow_i, kq, BM);
+        *reinterpret_cast<float4*>(a_hi + off) = h;
+        *reinterpret_cast<float4*>(a_lo + off) = l;
+#pragma unroll
+        for (int j = 0; j < BROWS; j++) {
+          const int brow = tid + j * NPROD;
+          if (brow < BN) {
+#pragma unroll
+            for (int e = 0; e < 4; e++) { int k = k0 + kq * 4 + e; v[e] = k < kend ? lb.at(bcol[j], k, p.K) : 0.f; }
+            h.x = tf32_rna(v[0]); h.y = tf32_rna(v[1]); h.z = tf32_rna(v[2]); h.w = tf32_rna(v[3]);
+            l.x = v[0] - h.x; l.y = v[1] - h.y; l.z = v[2] - h.z; l.w = v[3] - h.w;
+            const uint32_t boff = elem_off(brow, kq, BN);
+            *reinterpret_cast<float4*>(b_hi + boff) = h;
+            *reinterpret_cast<float4*>(b_lo + boff) = l;
+          }
+        }
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic-proxy writes -> tensor core
+      mbar_arrive(full0 + 8 * s);
+    }
+  } else if (lane == 0) {
+    // ---------------- MMA issuer (one thread)
+    for (int kt = 0; kt < nk; kt++) {
+      const int s = kt % Cfg::STAGES;
+      const uint32_t ph = (uint32_t)(kt / Cfg::STAGES) & 1u;
+      mbar_wait(full0 + 8 * s, ph);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      const uint32_t st = smem_u32(smem + s * Cfg::STAGE_BYTES);
+      const uint32_t a_hi = st, a_lo = st + Cfg::A_BYTES, b_hi = st + 2 * Cfg::A_BYTES, b_lo = b_hi + Cfg::B_BYTES;
+#pragma unroll
+      for (int j = 0; j < BK / 8; j++) {
+        const uint64_t dah = sdesc(a_hi + j * BM * 32, 128, 256), dal = sdesc(a_lo + j * BM * 32, 128, 256);
+        const uint64_t dbh = sdesc(b_hi + j * BN * 32, 128, 256), dbl = sdesc(b_lo + j * BN * 32, 128, 256);
+        mma_tf32(tmem, dal, dbh, Cfg::IDESC, (kt | j) != 0);
+        mma_tf32(tmem, dah, dbl, Cfg::IDESC, 1);
+        mma_tf32(tmem, dah, dbh, Cfg::IDESC, 1);
+      }
+      mma_commit(empty0 + 8 * s);   // frees the stage once these MMAs have read it
+    }
+    mma_commit(done_bar);           // accumulator complete
+  }
+
+  // ---------------- epilogue: TMEM -> registers -> global (or split partials)
+  if (warp < 4) {
+    mbar_wait(done_bar, 0);
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const int m = m0 + tid;
+    float* dst = p.split == 1 ? (p.C + (long long)m * p.ldc) : (p.ws + (long long)blockIdx.z * p.M * p.N + (long long)m * p.N);
+#pragma unroll 1
+    for (int c0 = 0; c0 < BN; c0 += 32) {
+      float v[32];
+      if (nk > 0) {
+        tmem_ld32(tmem + ((uint32_t)(32 * warp) << 16) + (uint32_t)c0, v);
+      } else {
+#pragma unroll
+        for (int i = 0; i < 32; i++) v[i] = 0.f;
+      }
+      if (m < p.M) {
+#pragma unroll
+        for (int i = 0; i < 32; i++) {
+          const int n = n0 + c0 + i;
+          if (n < p.N) dst[n] = p.split == 1 ? v[i] + (p.bias ? __ldg(p.bias + n) : 0.f) : v[i];
+        }
+      }
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  if (p.split > 1) {
+    unsigned int* tk = p.tickets + blockIdx.y * gridDim.x + blockIdx.x;
+    if (last_cta_of(tk, p.split)) {
+      if (tid < BM && m0 + tid < p.M) {
+        const int m = m0 + tid;
+        const long long stride = (long long)p.M * p.N;
+        for (int c = 0; c < BN; c++) {
+          const int n = n0 + c;
+          if (n >= p.N) break;
+          const float* q = p.ws + (long long)m * p.N + n;
+          float sum = 0.f;
+          int z = 0;
+          for (; z + 3 < p.split; z += 4) {
+            float v0 = __ldcg(q + z * stride), v1 = __ldcg(q + (z + 1) * stride);
+            float v2 = __ldcg(q + (z + 2) * stride), v3 = __ldcg(q + (z + 3) * stride);
+            sum += v0; sum += v1; sum += v2; sum += v3;
+          }
+          for (; z < p.split; z++) sum += __ldcg(q + z * stride);
+          p.C[(long long)m * p.ldc + n] = sum + (p.bias ? __ldg(p.bias + n) : 0.f);
+        }
+      }
+    }
+  } else {
+    __syncthreads();
+  }
+  if (warp == 4) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(Cfg::TMEM_COLS) : "memory");
+  }
+  orion_signal(sig);
+}
+
+}  // namespace tc
 
 // ---------------------------------------------------------------- small-M GEMM (GEMV-like)
 // For M <= 8 with B transposed (weights [N][K], the Linear layout): one warp per output column n,
@@ -332,9 +580,25 @@ __global__ void __launch_bounds__(256) gemv_bt_kernel(const float* __restrict__ 
 // part's size class, never the partition's SM count) so long-K problems (weight gradients over
 // N*H*W rows, 3x3 convs at batch 4) spread over the GPU; the split reduction is ordered.
 struct Plan { int cfg; int split; int bm, bn, bk; };
+// cfg: 0/1/2 = FFMA tiles L/M/S; 3/4 = tcgen05 3xTF32 with BN = 128 / 64.
 
 Plan plan_gemm(long long M, long long N, long long K) {
   Plan pl;
+  const bool tc_ok = M >= 64 && N >= 32 && K >= 64 && M * N * K >= (1LL << 22);
+  if (tc_ok) {
+    pl.cfg = N >= 96 ? 3 : 4; pl.bm = 128; pl.bn = N >= 96 ? 128 : 64; pl.bk = 32;
+    long long tiles = cdiv(M, pl.bm) * cdiv(N, pl.bn);
+    long long ktiles = cdiv(K, pl.bk);
+    long long split = 1;
+    if (tiles < 148) {              // one CTA per SM (~196 KB smem each): fill a 148-SM part once
+      split = cdiv(148, tiles);
+      if (split > ktiles / 2) split = ktiles / 2;   // >= 2 k-tiles per split
+      if (split > 64) split = 64;
+      if (split < 1) split = 1;
+    }
+    pl.split = (int)split;
+    return pl;
+  }
   if (M >= 128 && N >= 128 && M * N >= 128LL * 128 * 64) { pl.cfg = 0; pl.bm = 128; pl.bn = 128; pl.bk = 8; }
   else if (M >= 48 && N >= 48) { pl.cfg = 1; pl.bm = 64; pl.bn = 64; pl.bk = 16; }
   else { pl.cfg = 2; pl.bm = 32; pl.bn = 32; pl.bk = 32; }
@@ -361,8 +625,21 @@ const void* kernel_for(int cfg) {
   switch (cfg) {
     case 0: return (const void*)gemm_kernel<TileL, LA, LB>;
     case 1: return (const void*)gemm_kernel<TileM, LA, LB>;
-    default: return (const void*)gemm_kernel<TileS, LA, LB>;
+    case 2: return (const void*)gemm_kernel<TileS, LA, LB>;
+    case 3: return (const void*)tc::gemm_tc_kernel<128, LA, LB>;
+    default: return (const void*)tc::gemm_tc_kernel<64, LA, LB>;
   }
+}
+
+// Opt the tcgen05 kernels into > 48 KB dynamic shared memory once per instantiation.
+template <int BN, class LA, class LB>
+bool tc_prepare() {
+  static std::atomic<int> done{0};
+  if (done.load(std::memory_order_acquire)) return true;
+  bool ok = cudaFuncSetAttribute((const void*)tc::gemm_tc_kernel<BN, LA, LB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 tc::TcCfg<BN>::SMEM) == cudaSuccess;
+  if (ok) done.store(1, std::memory_order_release);
+  return ok;
 }
 
 // Geometry of a tiled launch; falls back to split 1 when the caller's workspace is too small.
@@ -371,9 +648,10 @@ void tiled_geom(LaunchGeom* g, long long M, long long N, long long K, uint64_t w
   Plan pl = plan_gemm(M, N, K);
   if (pl.split > 1 && (ws_ptr == 0 || ws_bytes < ws_bytes_for(pl, M, N))) pl.split = 1;
   g->grid = dim3((unsigned)cdiv(N, pl.bn), (unsigned)cdiv(M, pl.bm), (unsigned)pl.split);
-  g->block = dim3(NT);
-  g->smem = 0;
   g->func = kernel_for<LA, LB>(pl.cfg);
+  if (pl.cfg == 3) { tc_prepare<128, LA, LB>(); g->block = dim3(tc::NTHR); g->smem = tc::TcCfg<128>::SMEM; }
+  else if (pl.cfg == 4) { tc_prepare<64, LA, LB>(); g->block = dim3(tc::NTHR); g->smem = tc::TcCfg<64>::SMEM; }
+  else { g->block = dim3(NT); g->smem = 0; }
 }
 
 GemmParams make_params(long long M, long long N, long long K, float* C, long long ldc, const float* bias, int split,
@@ -399,8 +677,14 @@ int launch_tiled(const LaunchGeom& g, long long M, long long N, long long K, flo
     gemm_kernel<TileL, LA, LB><<<g.grid, g.block, 0, s>>>(make_params(M, N, K, C, ldc, bias, split, ws, TileL::BK), la, lb, sig);
   } else if (g.func == (const void*)gemm_kernel<TileM, LA, LB>) {
     gemm_kernel<TileM, LA, LB><<<g.grid, g.block, 0, s>>>(make_params(M, N, K, C, ldc, bias, split, ws, TileM::BK), la, lb, sig);
-  } else {
+  } else if (g.func == (const void*)gemm_kernel<TileS, LA, LB>) {
     gemm_kernel<TileS, LA, LB><<<g.grid, g.block, 0, s>>>(make_params(M, N, K, C, ldc, bias, split, ws, TileS::BK), la, lb, sig);
+  } else if (g.func == (const void*)tc::gemm_tc_kernel<128, LA, LB>) {
+    if (!tc_prepare<128, LA, LB>()) return ORION_E_CUDA;
+    tc::gemm_tc_kernel<128, LA, LB><<<g.grid, g.block, g.smem, s>>>(make_params(M, N, K, C, ldc, bias, split, ws, tc::BK), la, lb, sig);
+  } else {
+    if (!tc_prepare<64, LA, LB>()) return ORION_E_CUDA;
+    tc::gemm_tc_kernel<64, LA, LB><<<g.grid, g.block, g.smem, s>>>(make_params(M, N, K, C, ldc, bias, split, ws, tc::BK), la, lb, sig);
   }
   return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
 }
