@@ -41,12 +41,21 @@ struct GemmParams {
 // ---------------------------------------------------------------- operand loaders
 // A(m, k) and B(k, n). kContigK says whether consecutive k are adjacent in memory; it picks the
 // global->smem load mapping that keeps warps coalesced.
+// at4(r, k, kend): the 4 values at k..k+3 (k % 4 == 0), zero beyond kend; one 128-bit load when the
+// 4 are contiguous and aligned, else 4 scalar loads.
+__device__ __forceinline__ bool al16(const float* q) { return (reinterpret_cast<uintptr_t>(q) & 15) == 0; }
+
 struct ADense {          // A row-major [M][lda]
   static constexpr bool kContigK = true;
   const float* p; long long ld;
   struct Row { long long base; bool ok; };
   __device__ Row row(int m, int M) const { return {(long long)m * ld, m < M}; }
   __device__ float at(const Row& r, int k, int K) const { return (r.ok && k < K) ? __ldg(p + r.base + k) : 0.f; }
+  __device__ float4 at4(const Row& r, int k, int kend) const {
+    const float* q = p + r.base + k;
+    if (r.ok && k + 3 < kend && al16(q)) return __ldg(reinterpret_cast<const float4*>(q));
+    return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
+  }
 };
 struct ADenseT {         // A stored transposed: A(m,k) = p[k*ld + m]
   static constexpr bool kContigK = false;
@@ -54,6 +63,9 @@ struct ADenseT {         // A stored transposed: A(m,k) = p[k*ld + m]
   struct Row { int m; bool ok; };
   __device__ Row row(int m, int M) const { return {m, m < M}; }
   __device__ float at(const Row& r, int k, int K) const { return (r.ok && k < K) ? __ldg(p + (long long)k * ld + r.m) : 0.f; }
+  __device__ float4 at4(const Row& r, int k, int kend) const {
+    return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
+  }
 };
 struct BDense {          // B row-major [K][ldb]: B(k,n) = p[k*ld + n]
   static constexpr bool kContigK = false;
@@ -61,6 +73,9 @@ struct BDense {          // B row-major [K][ldb]: B(k,n) = p[k*ld + n]
   struct Col { int n; bool ok; };
   __device__ Col col(int n, int N) const { return {n, n < N}; }
   __device__ float at(const Col& c, int k, int K) const { return (c.ok && k < K) ? __ldg(p + (long long)k * ld + c.n) : 0.f; }
+  __device__ float4 at4(const Col& c, int k, int kend) const {
+    return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
+  }
 };
 struct BDenseT {         // B stored transposed [N][ldb]: B(k,n) = p[n*ld + k]
   static constexpr bool kContigK = true;
@@ -68,6 +83,11 @@ struct BDenseT {         // B stored transposed [N][ldb]: B(k,n) = p[n*ld + k]
   struct Col { long long base; bool ok; };
   __device__ Col col(int n, int N) const { return {(long long)n * ld, n < N}; }
   __device__ float at(const Col& c, int k, int K) const { return (c.ok && k < K) ? __ldg(p + c.base + k) : 0.f; }
+  __device__ float4 at4(const Col& c, int k, int kend) const {
+    const float* q = p + c.base + k;
+    if (c.ok && k + 3 < kend && al16(q)) return __ldg(reinterpret_cast<const float4*>(q));
+    return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
+  }
 };
 
 struct ConvShape { int N, H, W, C, K, R, S, stride, pad, P, Q; };
@@ -90,6 +110,18 @@ struct AIm2col {
     int h = r.h0 + rr, w = r.w0 + ss;
     if ((unsigned)h >= (unsigned)s.H || (unsigned)w >= (unsigned)s.W) return 0.f;
     return __ldg(x + r.nbase + ((long long)h * s.W + w) * s.C + c);
+  }
+  __device__ float4 at4(const Row& r, int k, int kend) const {
+    if ((s.C & 3) == 0 && k + 3 < kend) {   // same (r, s) tap, 4 consecutive channels
+      if (!r.ok) return make_float4(0.f, 0.f, 0.f, 0.f);
+      int c = k % s.C; int t = k / s.C; int ss = t % s.S; int rr = t / s.S;
+      int h = r.h0 + rr, w = r.w0 + ss;
+      if ((unsigned)h >= (unsigned)s.H || (unsigned)w >= (unsigned)s.W) return make_float4(0.f, 0.f, 0.f, 0.f);
+      const float* q = x + r.nbase + ((long long)h * s.W + w) * s.C + c;
+      if (al16(q)) return __ldg(reinterpret_cast<const float4*>(q));
+      return make_float4(__ldg(q), __ldg(q + 1), __ldg(q + 2), __ldg(q + 3));
+    }
+    return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
   }
 };
 
@@ -115,6 +147,20 @@ struct ADgrad {
     if (p >= s.P || q >= s.Q) return 0.f;
     return __ldg(dy + r.nbase + ((long long)p * s.Q + q) * s.K + ko);
   }
+  __device__ float4 at4(const Row& r, int k, int kend) const {
+    if ((s.K & 3) == 0 && k + 3 < kend) {   // same tap, 4 consecutive output channels
+      if (!r.ok) return make_float4(0.f, 0.f, 0.f, 0.f);
+      int ko = k % s.K; int t = k / s.K; int ss = t % s.S; int rr = t / s.S;
+      int ph = r.hp - rr, pw = r.wp - ss;
+      if (ph < 0 || pw < 0 || ph % s.stride || pw % s.stride) return make_float4(0.f, 0.f, 0.f, 0.f);
+      int p = ph / s.stride, q = pw / s.stride;
+      if (p >= s.P || q >= s.Q) return make_float4(0.f, 0.f, 0.f, 0.f);
+      const float* qq = dy + r.nbase + ((long long)p * s.Q + q) * s.K + ko;
+      if (al16(qq)) return __ldg(reinterpret_cast<const float4*>(qq));
+      return make_float4(__ldg(qq), __ldg(qq + 1), __ldg(qq + 2), __ldg(qq + 3));
+    }
+    return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
+  }
 };
 // Conv dgrad B: B(k = (r,s,kout), n = c) = w[kout][r][s][c]
 struct BDgrad {
@@ -126,6 +172,9 @@ struct BDgrad {
     if (!cc.ok || k >= K) return 0.f;
     int ko = k % s.K; int t = k / s.K; int ss = t % s.S; int rr = t / s.S;
     return __ldg(w + (((long long)ko * s.R + rr) * s.S + ss) * s.C + cc.c);
+  }
+  __device__ float4 at4(const Col& c, int k, int kend) const {
+    return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
   }
 };
 // Conv wgrad B: B(k = (n,p,q), col = (r,s,c)) = x[n, p*st-pad+r, q*st-pad+s, c]
@@ -144,6 +193,9 @@ struct BWgrad {
     int h = p * s.stride - s.pad + cc.r, w = q * s.stride - s.pad + cc.ss;
     if ((unsigned)h >= (unsigned)s.H || (unsigned)w >= (unsigned)s.W) return 0.f;
     return __ldg(x + (((long long)n * s.H + h) * s.W + w) * s.C + cc.c);
+  }
+  __device__ float4 at4(const Col& c, int k, int kend) const {
+    return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
   }
 };
 
@@ -299,7 +351,7 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
 // im2col / transposed-view functors as the FFMA path, so every conv kind runs on this kernel.
 namespace tc {
 
-constexpr int BM = 128, BK = 32, NPROD = 128, NTHR = 160;
+constexpr int BM = 128, BK = 32, NPROD = 256, NTHR = 288;   // 8 producer warps + 1 MMA warp
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint32_t a, uint32_t cnt) {
@@ -388,7 +440,7 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
     mbar_init(done_bar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == 4) {
+  if (warp == NPROD / 32) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)), "r"(Cfg::TMEM_COLS) : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
@@ -397,53 +449,55 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   const uint32_t tmem = *tmem_slot;
 
-  if (warp < 4) {
-    // ---------------- producers: row-per-thread staging of A (128 rows) and B (BN rows)
-    const int arow_i = tid;                      // A row m0 + tid
-    typename LA::Row arow = la.row(m0 + arow_i, p.M);
-    constexpr int BROWS = (BN + NPROD - 1) / NPROD;
-    typename LB::Col bcol[BROWS];
+  if (warp < NPROD / 32) {
+    // ---------------- producers: TPR threads per operand row, each staging 8/TPR k-quads per stage.
+    // All of a stage's global loads are issued before any hi/lo split or shared store.
+    constexpr int A_TPR = NPROD / BM, A_QPT = 8 / A_TPR;           // 2 threads per A row, 4 quads each
+    constexpr int B_TPR = NPROD / BN >= 1 ? NPROD / BN : 1;
+    constexpr int B_QPT = 8 / B_TPR >= 1 ? 8 / B_TPR : 1;
+    constexpr int B_RPT = BN > NPROD ? BN / NPROD : 1;             // rows per thread (BN > 256 only)
+    const int a_row = tid % BM, a_q0 = (tid / BM) * A_QPT;
+    typename LA::Row arow = la.row(m0 + a_row, p.M);
+    const int b_row = tid % (BN < NPROD ? BN : NPROD), b_q0 = (tid / (BN < NPROD ? BN : NPROD)) * B_QPT;
+    typename LB::Col bcol[B_RPT];
 #pragma unroll
-    for (int j = 0; j < BROWS; j++) bcol[j] = lb.col(n0 + tid + j * NPROD, p.N);
+    for (int j = 0; j < B_RPT; j++) bcol[j] = lb.col(n0 + b_row + j * NPROD, p.N);
     for (int kt = 0; kt < nk; kt++) {
       const int s = kt % Cfg::STAGES;
       const uint32_t ph = (uint32_t)(kt / Cfg::STAGES) & 1u;
+      const int k0 = kbeg + kt * BK;
+      float4 va[A_QPT], vb[B_RPT][B_QPT];
+#pragma unroll
+      for (int q = 0; q < A_QPT; q++) va[q] = la.at4(arow, k0 + (a_q0 + q) * 4, kend);
+#pragma unroll
+      for (int j = 0; j < B_RPT; j++)
+#pragma unroll
+        for (int q = 0; q < B_QPT; q++) vb[j][q] = lb.at4(bcol[j], k0 + (b_q0 + q) * 4, kend);
       mbar_wait(empty0 + 8 * s, ph ^ 1u);
       unsigned char* st = smem + s * Cfg::STAGE_BYTES;
       unsigned char* a_hi = st;
       unsigned char* a_lo = st + Cfg::A_BYTES;
       unsigned char* b_hi = st + 2 * Cfg::A_BYTES;
       unsigned char* b_lo = b_hi + Cfg::B_BYTES;
-      const int k0 = kbeg + kt * BK;
-#pragma unroll
-      for (int kq = 0; kq < BK / 4; kq++) {     // 8 quads of 4 consecutive k
+      auto split_store = [](unsigned char* hi, unsigned char* lo, uint32_t off, const float4& v) {
         float4 h, l;
-        float v[4];
+        h.x = tf32_rna(v.x); h.y = tf32_rna(v.y); h.z = tf32_rna(v.z); h.w = tf32_rna(v.w);
+        l.x = v.x - h.x; l.y = v.y - h.y; l.z = v.z - h.z; l.w = v.w - h.w;
+        *reinterpret_cast<float4*>(hi + off) = h;
+        *reinterpret_cast<float4*>(lo + off) = l;
+      };
 #pragma unroll
-        for (int e = 0; e < 4; e++) { int k = k0 + kq * 4 + e; v[e] = k < kend ? la.at(arow, k, p.K) : 0.f; }
-        h.x = tf32_rna(v[0]); h.y = tf32_rna(v[1]); h.z = tf32_rna(v[2]); h.w = tf32_rna(v[3]);
-        l.x = v[0] - h.x; l.y = v[1] - h.y; l.z = v[2] - h.z; l.w = v[3] - h.w;
-        const uint32_t off = elem_off(arow_i, kq, BM);
-        *reinterpret_cast<float4*>(a_hi + off) = h;
-        *reinterpret_cast<float4*>(a_lo + off) = l;
+      for (int q = 0; q < A_QPT; q++) split_store(a_hi, a_lo, elem_off(a_row, a_q0 + q, BM), va[q]);
+      if (tid < B_TPR * (BN < NPROD ? BN : NPROD)) {
 #pragma unroll
-        for (int j = 0; j < BROWS; j++) {
-          const int brow = tid + j * NPROD;
-          if (brow < BN) {
+        for (int j = 0; j < B_RPT; j++)
 #pragma unroll
-            for (int e = 0; e < 4; e++) { int k = k0 + kq * 4 + e; v[e] = k < kend ? lb.at(bcol[j], k, p.K) : 0.f; }
-            h.x = tf32_rna(v[0]); h.y = tf32_rna(v[1]); h.z = tf32_rna(v[2]); h.w = tf32_rna(v[3]);
-            l.x = v[0] - h.x; l.y = v[1] - h.y; l.z = v[2] - h.z; l.w = v[3] - h.w;
-            const uint32_t boff = elem_off(brow, kq, BN);
-            *reinterpret_cast<float4*>(b_hi + boff) = h;
-            *reinterpret_cast<float4*>(b_lo + boff) = l;
-          }
-        }
+          for (int q = 0; q < B_QPT; q++) split_store(b_hi, b_lo, elem_off(b_row + j * NPROD, b_q0 + q, BN), vb[j][q]);
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic-proxy writes -> tensor core
       mbar_arrive(full0 + 8 * s);
     }
-  } else if (lane == 0) {
+  } else if (warp == NPROD / 32 && lane == 0) {
     // ---------------- MMA issuer (one thread)
     for (int kt = 0; kt < nk; kt++) {
       const int s = kt % Cfg::STAGES;
@@ -515,7 +569,7 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
   } else {
     __syncthreads();
   }
-  if (warp == 4) {
+  if (warp == NPROD / 32) {
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(Cfg::TMEM_COLS) : "memory");
   }

@@ -39,6 +39,14 @@ def ws(nbytes):
 
 @pytest.mark.parametrize("M,N,K,flags", [(1, 512, 512, 2), (4, 1000, 2048, 2), (3, 37, 129, 2), (32, 512, 512, 2),
                                          (96, 16, 300000, 1), (16, 32, 100000, 1), (196, 2048, 512, 2), (784, 256, 1024, 2),
+                                         (256, 256, 256, 0), (300, 200, 520, 1), (130, 70, 300, 2), (257, 129, 333, 3),
+                                         (4704, 1280, 320, 2), (1280, 320, 4704, 1), (18816, 96, 576, 2)],
+                         ids=lambda v: str(v))
+def test_gemm_shapes(M, N, K, flags):
+    test_gemm(M, N, K, flags)
+
+
+@pytest.mark.parametrize("M,N,K,flags", [(1, 512, 512, 2),
                                          (200, 130, 77, 0), (300, 257, 65, 1), (129, 131, 700, 3), (96, 1000, 1280, 2),
                                          (1000, 1280, 96, 1), (64, 96, 20000, 1), (12544, 64, 256, 2)])
 def test_gemm(M, N, K, flags):
@@ -194,8 +202,11 @@ def test_losses_sgd_colsum():
 def test_geometry_and_sm_needed():
     """sm_needed = ceil(grid / blocks_per_sm) from the kernel's own launch geometry."""
     A = torch.zeros(4096, 256, device="cuda")
-    grid, bps, thr, smem = orion.kernel_geometry("gemm", [A.data_ptr(), A.data_ptr(), A.data_ptr(), 0, 4096, 256, 256, 256, 256, 256, 2, 0, 0])
-    assert grid == 32 * 2 and thr == 256 and bps >= 1
+    grid, bps, thr, smem = orion.kernel_geometry("gemm", [A.data_ptr(), A.data_ptr(), A.data_ptr(), 0, 4096, 16, 16, 16, 16, 16, 2, 0, 0])
+    assert grid == 4096 // 32 and thr == 256 and bps >= 1
+    # a compute-dense shape routes to the tcgen05 kernel (160 threads, ~196 KB dynamic smem)
+    grid, bps, thr, smem = orion.kernel_geometry("gemm", [A.data_ptr(), A.data_ptr(), A.data_ptr(), 0, 4096, 256, 256, 256, 256, 256, 0, 0, 0])
+    assert thr == 160 and smem > 100_000 and bps == 1
     grid, bps, thr, smem = orion.kernel_geometry("relu", [A.data_ptr(), A.data_ptr(), A.numel()])
     assert grid == min((A.numel() // 4 + 255) // 256, 148 * 8) and 1 <= bps <= 8
     assert orion.profiler.sm_needed("relu", [A.data_ptr(), A.data_ptr(), A.numel()]) == -(-grid // bps)
