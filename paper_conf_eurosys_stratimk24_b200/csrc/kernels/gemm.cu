@@ -199,6 +199,61 @@ struct BWgrad {
   }
 };
 
+// ---------------------------------------------------------------- ordered split-K reduction
+// Run by every thread of the last CTA of a tile: C[m0:m0+bm, n0:n0+bn] = sum_{z < split} ws[z] (+bias),
+// summed in split order (((p0 + p1) + p2) + ...), so the result depends only on the shape.
+// Elements are spread over the CTA's threads with consecutive threads on consecutive columns
+// (coalesced), 4 columns (128 bits) per thread when possible and 4 splits in flight.
+__device__ void split_reduce_tile(const GemmParams& p, int m0, int n0, int bm, int bn) {
+  const long long stride = (long long)p.M * p.N;
+  const int rows = min(bm, p.M - m0), cols = min(bn, p.N - n0);
+  const bool vec = (cols % 4 == 0) && (p.N % 4 == 0) && (n0 % 4 == 0) && (p.ldc % 4 == 0) &&
+                   ((reinterpret_cast<uintptr_t>(p.ws) & 15) == 0) && ((reinterpret_cast<uintptr_t>(p.C) & 15) == 0);
+  if (vec) {
+    const int cq = cols / 4, total = rows * cq;
+    for (int e = threadIdx.x; e < total; e += blockDim.x) {
+      const int r = e / cq, c = (e % cq) * 4;
+      const float* q = p.ws + (long long)(m0 + r) * p.N + n0 + c;
+      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+      int z = 0;
+      for (; z + 3 < p.split; z += 4) {
+        float4 v0 = __ldcg(reinterpret_cast<const float4*>(q + z * stride));
+        float4 v1 = __ldcg(reinterpret_cast<const float4*>(q + (z + 1) * stride));
+        float4 v2 = __ldcg(reinterpret_cast<const float4*>(q + (z + 2) * stride));
+        float4 v3 = __ldcg(reinterpret_cast<const float4*>(q + (z + 3) * stride));
+        acc.x += v0.x; acc.x += v1.x; acc.x += v2.x; acc.x += v3.x;
+        acc.y += v0.y; acc.y += v1.y; acc.y += v2.y; acc.y += v3.y;
+        acc.z += v0.z; acc.z += v1.z; acc.z += v2.z; acc.z += v3.z;
+        acc.w += v0.w; acc.w += v1.w; acc.w += v2.w; acc.w += v3.w;
+      }
+      for (; z < p.split; z++) {
+        float4 v = __ldcg(reinterpret_cast<const float4*>(q + z * stride));
+        acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+      }
+      const int n = n0 + c;
+      if (p.bias) {
+        acc.x += __ldg(p.bias + n); acc.y += __ldg(p.bias + n + 1); acc.z += __ldg(p.bias + n + 2); acc.w += __ldg(p.bias + n + 3);
+      }
+      *reinterpret_cast<float4*>(p.C + (long long)(m0 + r) * p.ldc + n) = acc;
+    }
+  } else {
+    const int total = rows * cols;
+    for (int e = threadIdx.x; e < total; e += blockDim.x) {
+      const int r = e / cols, c = e % cols;
+      const float* q = p.ws + (long long)(m0 + r) * p.N + n0 + c;
+      float acc = 0.f;
+      int z = 0;
+      for (; z + 3 < p.split; z += 4) {
+        float v0 = __ldcg(q + z * stride), v1 = __ldcg(q + (z + 1) * stride);
+        float v2 = __ldcg(q + (z + 2) * stride), v3 = __ldcg(q + (z + 3) * stride);
+        acc += v0; acc += v1; acc += v2; acc += v3;
+      }
+      for (; z < p.split; z++) acc += __ldcg(q + z * stride);
+      p.C[(long long)(m0 + r) * p.ldc + n0 + c] = acc + (p.bias ? __ldg(p.bias + n0 + c) : 0.f);
+    }
+  }
+}
+
 // ---------------------------------------------------------------- the tiled main loop
 template <int N_>
 __device__ __forceinline__ void lds_frag(float* dst, const float* src) {
@@ -311,30 +366,7 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
       }
     }
     unsigned int* tk = p.tickets + blockIdx.y * gridDim.x + blockIdx.x;
-    if (last_cta_of(tk, p.split)) {
-#pragma unroll
-      for (int i = 0; i < TM; i++) {
-        int m = out_row(i);
-        if (m >= p.M) continue;
-#pragma unroll
-        for (int j = 0; j < TN; j++) {
-          int n = out_col(j);
-          if (n >= p.N) continue;
-          // ordered sum over splits, 4 loads in flight: ((s + p0) + p1) + p2 ...
-          const float* q = p.ws + (long long)m * p.N + n;
-          const long long stride = (long long)p.M * p.N;
-          float s = 0.f;
-          int z = 0;
-          for (; z + 3 < p.split; z += 4) {
-            float v0 = __ldcg(q + z * stride), v1 = __ldcg(q + (z + 1) * stride);
-            float v2 = __ldcg(q + (z + 2) * stride), v3 = __ldcg(q + (z + 3) * stride);
-            s += v0; s += v1; s += v2; s += v3;
-          }
-          for (; z < p.split; z++) s += __ldcg(q + z * stride);
-          p.C[(long long)m * p.ldc + n] = s + (p.bias ? __ldg(p.bias + n) : 0.f);
-        }
-      }
-    }
+    if (last_cta_of(tk, p.split)) split_reduce_tile(p, m0, n0, BM, BN);
   }
   orion_signal(sig);
 }
@@ -546,26 +578,7 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   if (p.split > 1) {
     unsigned int* tk = p.tickets + blockIdx.y * gridDim.x + blockIdx.x;
-    if (last_cta_of(tk, p.split)) {
-      if (tid < BM && m0 + tid < p.M) {
-        const int m = m0 + tid;
-        const long long stride = (long long)p.M * p.N;
-        for (int c = 0; c < BN; c++) {
-          const int n = n0 + c;
-          if (n >= p.N) break;
-          const float* q = p.ws + (long long)m * p.N + n;
-          float sum = 0.f;
-          int z = 0;
-          for (; z + 3 < p.split; z += 4) {
-            float v0 = __ldcg(q + z * stride), v1 = __ldcg(q + (z + 1) * stride);
-            float v2 = __ldcg(q + (z + 2) * stride), v3 = __ldcg(q + (z + 3) * stride);
-            sum += v0; sum += v1; sum += v2; sum += v3;
-          }
-          for (; z < p.split; z++) sum += __ldcg(q + z * stride);
-          p.C[(long long)m * p.ldc + n] = sum + (p.bias ? __ldg(p.bias + n) : 0.f);
-        }
-      }
-    }
+    if (last_cta_of(tk, p.split)) split_reduce_tile(p, m0, n0, BM, BN);
   } else {
     __syncthreads();
   }
@@ -640,14 +653,17 @@ Plan plan_gemm(long long M, long long N, long long K) {
   Plan pl;
   const bool tc_ok = M >= 64 && N >= 32 && K >= 64 && M * N * K >= (1LL << 22);
   if (tc_ok) {
-    pl.cfg = N >= 96 ? 3 : 4; pl.bm = 128; pl.bn = N >= 96 ? 128 : 64; pl.bk = 32;
+    // BN = 128 only when that already yields >= 74 tiles; otherwise BN = 64 doubles the tiles so
+    // fewer K splits are needed (each split adds bm*bn*4 bytes the last CTA must re-read).
+    const bool wide = N >= 96 && cdiv(M, 128) * cdiv(N, 128) >= 74;
+    pl.cfg = wide ? 3 : 4; pl.bm = 128; pl.bn = wide ? 128 : 64; pl.bk = 32;
     long long tiles = cdiv(M, pl.bm) * cdiv(N, pl.bn);
     long long ktiles = cdiv(K, pl.bk);
     long long split = 1;
     if (tiles < 148) {              // one CTA per SM (~196 KB smem each): fill a 148-SM part once
       split = cdiv(148, tiles);
-      if (split > ktiles / 2) split = ktiles / 2;   // >= 2 k-tiles per split
-      if (split > 64) split = 64;
+      if (split > ktiles / 4) split = ktiles / 4;   // >= 4 k-tiles per split
+      if (split > 16) split = 16;                   // bounded ordered reduction (<= 512 KB per tile)
       if (split < 1) split = 1;
     }
     pl.split = (int)split;
@@ -657,13 +673,13 @@ Plan plan_gemm(long long M, long long N, long long K) {
   else if (M >= 48 && N >= 48) { pl.cfg = 1; pl.bm = 64; pl.bn = 64; pl.bk = 16; }
   else { pl.cfg = 2; pl.bm = 32; pl.bn = 32; pl.bk = 32; }
   long long tiles = cdiv(M, pl.bm) * cdiv(N, pl.bn);
-  long long target = 592;
+  long long target = 148 * 8;                 // long-K (weight-gradient) GEMMs are HBM-bound: many CTAs
   long long split = 1;
   if (tiles < target) {
     split = cdiv(target, tiles);
     long long kmax = K / (4 * pl.bk);         // >= 4 k-tiles per split
     if (split > kmax) split = kmax;
-    if (split > 512) split = 512;
+    if (split > 1024) split = 1024;
     if (split < 1) split = 1;
   }
   pl.split = (int)split;

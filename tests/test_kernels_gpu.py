@@ -206,7 +206,7 @@ def test_geometry_and_sm_needed():
     assert grid == 4096 // 32 and thr == 256 and bps >= 1
     # a compute-dense shape routes to the tcgen05 kernel (160 threads, ~196 KB dynamic smem)
     grid, bps, thr, smem = orion.kernel_geometry("gemm", [A.data_ptr(), A.data_ptr(), A.data_ptr(), 0, 4096, 256, 256, 256, 256, 256, 0, 0, 0])
-    assert thr == 160 and smem > 100_000 and bps == 1
+    assert thr == 288 and smem > 100_000 and bps == 1
     grid, bps, thr, smem = orion.kernel_geometry("relu", [A.data_ptr(), A.data_ptr(), A.numel()])
     assert grid == min((A.numel() // 4 + 255) // 256, 148 * 8) and 1 <= bps <= 8
     assert orion.profiler.sm_needed("relu", [A.data_ptr(), A.data_ptr(), A.numel()]) == -(-grid // bps)
