@@ -439,7 +439,11 @@ struct TcCfg {
   static constexpr int B_BYTES = BN * BK * 4;
   static constexpr int STAGE_BYTES = 2 * (A_BYTES + B_BYTES);
   static constexpr int SMEM = STAGES * STAGE_BYTES + 1024 + 256;
-  static constexpr int TMEM_COLS = BN < 32 ? 32 : BN;
+  // three fp32 accumulators of BN columns: hi*hi for even / odd k-steps, and the two correction
+  // products. The tensor core's fp32 accumulation truncates, so each chain's bias grows with its
+  // length; splitting the chains keeps the GEMM within ~1e-6 of fp64.
+  static constexpr int ACC_COLS = 3 * BN;
+  static constexpr int TMEM_COLS = ACC_COLS <= 32 ? 32 : ACC_COLS <= 64 ? 64 : ACC_COLS <= 128 ? 128 : ACC_COLS <= 256 ? 256 : 512;
   // instruction descriptor: D f32 (bits 4-5 = 1), A/B tf32 (2 at bits 7-9 / 10-12), K-major A/B,
   // N>>3 at bits 17-22, M>>4 at bits 24-28
   static constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
@@ -542,9 +546,10 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
       for (int j = 0; j < BK / 8; j++) {
         const uint64_t dah = sdesc(a_hi + j * BM * 32, 128, 256), dal = sdesc(a_lo + j * BM * 32, 128, 256);
         const uint64_t dbh = sdesc(b_hi + j * BN * 32, 128, 256), dbl = sdesc(b_lo + j * BN * 32, 128, 256);
-        mma_tf32(tmem, dal, dbh, Cfg::IDESC, (kt | j) != 0);
-        mma_tf32(tmem, dah, dbl, Cfg::IDESC, 1);
-        mma_tf32(tmem, dah, dbh, Cfg::IDESC, 1);
+        const uint32_t d_main = tmem + (uint32_t)((j & 1) * BN), d_corr = tmem + (uint32_t)(2 * BN);
+        mma_tf32(d_corr, dal, dbh, Cfg::IDESC, (kt | j) != 0);
+        mma_tf32(d_corr, dah, dbl, Cfg::IDESC, 1);
+        mma_tf32(d_main, dah, dbh, Cfg::IDESC, (kt | (j >> 1)) != 0);
       }
       mma_commit(empty0 + 8 * s);   // frees the stage once these MMAs have read it
     }
@@ -561,7 +566,13 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
     for (int c0 = 0; c0 < BN; c0 += 32) {
       float v[32];
       if (nk > 0) {
-        tmem_ld32(tmem + ((uint32_t)(32 * warp) << 16) + (uint32_t)c0, v);
+        const uint32_t lane_base = tmem + ((uint32_t)(32 * warp) << 16) + (uint32_t)c0;
+        float e[32], o[32];
+        tmem_ld32(lane_base, e);
+        tmem_ld32(lane_base + BN, o);
+        tmem_ld32(lane_base + 2 * BN, v);
+#pragma unroll
+        for (int i = 0; i < 32; i++) v[i] = (e[i] + o[i]) + v[i];
       } else {
 #pragma unroll
         for (int i = 0; i < 32; i++) v[i] = 0.f;
