@@ -11,12 +11,31 @@ constexpr int DW_THREADS = 256;
 
 struct DwShape { int N, H, W, C, stride, P, Q; };
 
-// Row-sliding depthwise kernels: a warp owns 32 consecutive channels (128-byte coalesced rows of
-// the NHWC tensor) and one output row (n, p); each lane walks q = 0..Q-1 keeping a 3x3 window
-// of its input column values in registers, so each input element is loaded once per output row
-// that uses it (3x for the 3 kernel rows) instead of 9x. Weights live in registers.
+// Row-blocked depthwise kernels: a warp owns 32 consecutive channels (128-byte coalesced rows of
+// the NHWC tensor) and one output row (n, p); each lane produces U = 4 consecutive outputs per step
+// from a 3 x ((U-1)*S+3) register window of its input columns whose loads are all issued
+// together (memory-level parallelism instead of one dependent load per output). Weights live in
+// registers. S = stride (compile-time 1 or 2).
 constexpr int ROW_WARPS = 8;
+constexpr int DW_U = 4;
 
+template <int S>
+struct Win {
+  static constexpr int NC = (DW_U - 1) * S + 3;   // input columns per block of U outputs
+  float v[3][NC];
+  // columns col0 .. col0+NC-1 of the 3 input rows (zero outside the image / missing rows)
+  __device__ __forceinline__ void load(const float* const (&rowp)[3], const bool (&rv)[3], int col0, int W, int C) {
+#pragma unroll
+    for (int r = 0; r < 3; r++)
+#pragma unroll
+      for (int j = 0; j < NC; j++) {
+        const int col = col0 + j;
+        v[r][j] = (rv[r] && (unsigned)col < (unsigned)W) ? __ldg(rowp[r] + (long long)col * C) : 0.f;
+      }
+  }
+};
+
+template <int S>
 __global__ void __launch_bounds__(DW_THREADS) dw_fwd_rows_kernel(const float* __restrict__ x, const float* __restrict__ w,
                                                                  float* __restrict__ y, DwShape s, OrionSig sig) {
   const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
@@ -35,30 +54,24 @@ __global__ void __launch_bounds__(DW_THREADS) dw_fwd_rows_kernel(const float* __
     bool rv[3];
 #pragma unroll
     for (int r = 0; r < 3; r++) {
-      int h = p * s.stride - 1 + r;
+      int h = p * S - 1 + r;
       rv[r] = (unsigned)h < (unsigned)s.H;
       xr[r] = x + (((long long)n * s.H + (rv[r] ? h : 0)) * s.W) * s.C + c;
     }
-    auto ld = [&](int r, int col) -> float {
-      return (rv[r] && (unsigned)col < (unsigned)s.W) ? __ldg(xr[r] + (long long)col * s.C) : 0.f;
-    };
     float* yr = y + (((long long)n * s.P + p) * s.Q) * s.C + c;
-    // window columns a (= q*st-1), b (= q*st), c2 (= q*st+1)
-    float a0 = ld(0, -1), a1 = ld(1, -1), a2 = ld(2, -1);
-    float b0 = ld(0, 0), b1 = ld(1, 0), b2 = ld(2, 0);
-    for (int q = 0; q < s.Q; q++) {
-      const int col = q * s.stride + 1;
-      float c0 = ld(0, col), c1 = ld(1, col), c2 = ld(2, col);
-      float acc = a0 * wr[0];
-      acc = fmaf(b0, wr[1], acc); acc = fmaf(c0, wr[2], acc);
-      acc = fmaf(a1, wr[3], acc); acc = fmaf(b1, wr[4], acc); acc = fmaf(c1, wr[5], acc);
-      acc = fmaf(a2, wr[6], acc); acc = fmaf(b2, wr[7], acc); acc = fmaf(c2, wr[8], acc);
-      yr[(long long)q * s.C] = acc;
-      if (s.stride == 1) {
-        a0 = b0; a1 = b1; a2 = b2; b0 = c0; b1 = c1; b2 = c2;
-      } else {  // stride 2: next window starts at col (q+1)*2-1 = current c column
-        a0 = c0; a1 = c1; a2 = c2;
-        b0 = ld(0, col + 1); b1 = ld(1, col + 1); b2 = ld(2, col + 1);
+    for (int q0 = 0; q0 < s.Q; q0 += DW_U) {
+      Win<S> win;
+      win.load(xr, rv, q0 * S - 1, s.W, s.C);
+#pragma unroll
+      for (int u = 0; u < DW_U; u++) {
+        if (q0 + u < s.Q) {
+          float acc = 0.f;
+#pragma unroll
+          for (int r = 0; r < 3; r++)
+#pragma unroll
+            for (int t = 0; t < 3; t++) acc = fmaf(win.v[r][u * S + t], wr[r * 3 + t], acc);
+          yr[(long long)(q0 + u) * s.C] = acc;
+        }
       }
     }
   }
@@ -88,29 +101,31 @@ __global__ void __launch_bounds__(DW_THREADS) dw_dgrad_rows_s1_kernel(const floa
       rv[r] = (unsigned)pp < (unsigned)s.P;
       gr[r] = dy + (((long long)n * s.P + (rv[r] ? pp : 0)) * s.Q) * s.C + c;
     }
-    auto ld = [&](int r, int col) -> float {
-      return (rv[r] && (unsigned)col < (unsigned)s.Q) ? __ldg(gr[r] + (long long)col * s.C) : 0.f;
-    };
     float* dr = dx + (((long long)n * s.H + h) * s.W) * s.C + c;
-    // dx(h, wq) = sum_r sum_u dy(r-row, wq+1-u) k(r,u): columns wq+1 (u=0), wq (u=1), wq-1 (u=2)
-    float m0 = ld(0, -1), m1 = ld(1, -1), m2 = ld(2, -1);   // column wq-1
-    float z0 = ld(0, 0), z1 = ld(1, 0), z2 = ld(2, 0);      // column wq
-    for (int wq = 0; wq < s.W; wq++) {
-      float p0 = ld(0, wq + 1), p1 = ld(1, wq + 1), p2 = ld(2, wq + 1);
-      float acc = p0 * wr[0];
-      acc = fmaf(z0, wr[1], acc); acc = fmaf(m0, wr[2], acc);
-      acc = fmaf(p1, wr[3], acc); acc = fmaf(z1, wr[4], acc); acc = fmaf(m1, wr[5], acc);
-      acc = fmaf(p2, wr[6], acc); acc = fmaf(z2, wr[7], acc); acc = fmaf(m2, wr[8], acc);
-      dr[(long long)wq * s.C] = acc;
-      m0 = z0; m1 = z1; m2 = z2; z0 = p0; z1 = p1; z2 = p2;
+    for (int w0 = 0; w0 < s.W; w0 += DW_U) {
+      Win<1> win;                      // dy columns w0-1 .. w0+U
+      win.load(gr, rv, w0 - 1, s.Q, s.C);
+#pragma unroll
+      for (int u = 0; u < DW_U; u++) {
+        if (w0 + u < s.W) {
+          // column index in win for dy column (w0+u)+1-t is u + 2 - t
+          float acc = 0.f;
+#pragma unroll
+          for (int r = 0; r < 3; r++)
+#pragma unroll
+            for (int t = 0; t < 3; t++) acc = fmaf(win.v[r][u + 2 - t], wr[r * 3 + t], acc);
+          dr[(long long)(w0 + u) * s.C] = acc;
+        }
+      }
     }
   }
   orion_signal(sig);
 }
 
-// wgrad: a warp accumulates the 9 taps of its 32 channels over whole output rows with a sliding
-// window of x, in fp32 per row and fp64 across rows; warps combine in smem in fixed order, CTAs
+// wgrad: a warp accumulates the 9 taps of its 32 channels over whole output rows (register window
+// blocks as above), fp32 per row and fp64 across rows; warps combine in smem in fixed order, CTAs
 // write per-split partials, the last CTA of the channel block sums them in split order.
+template <int S>
 __global__ void __launch_bounds__(DW_THREADS) dw_wgrad_rows_kernel(const float* __restrict__ x, const float* __restrict__ dy,
                                                                    float* __restrict__ dw, DwShape s, unsigned char* ws, OrionSig sig) {
   __shared__ double sh[ROW_WARPS][9][32];
@@ -127,32 +142,26 @@ __global__ void __launch_bounds__(DW_THREADS) dw_wgrad_rows_kernel(const float* 
       bool rv[3];
 #pragma unroll
       for (int r = 0; r < 3; r++) {
-        int h = p * s.stride - 1 + r;
+        int h = p * S - 1 + r;
         rv[r] = (unsigned)h < (unsigned)s.H;
         xr[r] = x + (((long long)n * s.H + (rv[r] ? h : 0)) * s.W) * s.C + c;
       }
-      auto ld = [&](int r, int col) -> float {
-        return (rv[r] && (unsigned)col < (unsigned)s.W) ? __ldg(xr[r] + (long long)col * s.C) : 0.f;
-      };
       const float* gr = dy + (((long long)n * s.P + p) * s.Q) * s.C + c;
       float f[9];
 #pragma unroll
       for (int t = 0; t < 9; t++) f[t] = 0.f;
-      float a0 = ld(0, -1), a1 = ld(1, -1), a2 = ld(2, -1);
-      float b0 = ld(0, 0), b1 = ld(1, 0), b2 = ld(2, 0);
-      for (int q = 0; q < s.Q; q++) {
-        const int col = q * s.stride + 1;
-        float c0 = ld(0, col), c1 = ld(1, col), c2 = ld(2, col);
-        float g = __ldg(gr + (long long)q * s.C);
-        f[0] = fmaf(g, a0, f[0]); f[1] = fmaf(g, b0, f[1]); f[2] = fmaf(g, c0, f[2]);
-        f[3] = fmaf(g, a1, f[3]); f[4] = fmaf(g, b1, f[4]); f[5] = fmaf(g, c1, f[5]);
-        f[6] = fmaf(g, a2, f[6]); f[7] = fmaf(g, b2, f[7]); f[8] = fmaf(g, c2, f[8]);
-        if (s.stride == 1) {
-          a0 = b0; a1 = b1; a2 = b2; b0 = c0; b1 = c1; b2 = c2;
-        } else {
-          a0 = c0; a1 = c1; a2 = c2;
-          b0 = ld(0, col + 1); b1 = ld(1, col + 1); b2 = ld(2, col + 1);
-        }
+      for (int q0 = 0; q0 < s.Q; q0 += DW_U) {
+        Win<S> win;
+        win.load(xr, rv, q0 * S - 1, s.W, s.C);
+        float g[DW_U];
+#pragma unroll
+        for (int u = 0; u < DW_U; u++) g[u] = (q0 + u < s.Q) ? __ldg(gr + (long long)(q0 + u) * s.C) : 0.f;
+#pragma unroll
+        for (int u = 0; u < DW_U; u++)
+#pragma unroll
+          for (int r = 0; r < 3; r++)
+#pragma unroll
+            for (int t = 0; t < 3; t++) f[r * 3 + t] = fmaf(g[u], win.v[r][u * S + t], f[r * 3 + t]);
       }
 #pragma unroll
       for (int t = 0; t < 9; t++) acc[t] += (double)f[t];
@@ -171,10 +180,17 @@ __global__ void __launch_bounds__(DW_THREADS) dw_wgrad_rows_kernel(const float* 
     }
   }
   if (last_cta_of(tickets + blockIdx.x, gridDim.y)) {
-    if (warp == 0 && c < s.C) {
-      for (int t = 0; t < 9; t++) {
+    // 9 taps x 32 channels reduced by 8 warps: warp w takes taps w and w+8 (fixed split order)
+    for (int t = warp; t < 9; t += ROW_WARPS) {
+      if (c < s.C) {
         double v = 0.0;
-        for (unsigned r = 0; r < gridDim.y; r++) v += __ldcg(part + ((long long)r * s.C + c) * 9 + t);
+        unsigned r = 0;
+        for (; r + 3 < gridDim.y; r += 4) {
+          double a0 = __ldcg(part + ((long long)r * s.C + c) * 9 + t), a1 = __ldcg(part + ((long long)(r + 1) * s.C + c) * 9 + t);
+          double a2 = __ldcg(part + ((long long)(r + 2) * s.C + c) * 9 + t), a3 = __ldcg(part + ((long long)(r + 3) * s.C + c) * 9 + t);
+          v += a0; v += a1; v += a2; v += a3;
+        }
+        for (; r < gridDim.y; r++) v += __ldcg(part + ((long long)r * s.C + c) * 9 + t);
         dw[c * 9 + t] = (float)v;
       }
     }
@@ -260,11 +276,15 @@ extern "C" uint64_t orion_dw_wgrad_workspace_bytes(uint64_t N, uint64_t C, uint6
 int dw_fwd_geom(const uint64_t* a, LaunchGeom* g) {
   if (!dw_ok(a)) return ORION_E_INVAL;
   DwShape s = dw_shape(a);
-  rows_geom(g, (long long)s.N * s.P * ((s.C + 31) / 32), (const void*)dw_fwd_rows_kernel);
+  if (s.stride != 1 && s.stride != 2) return ORION_E_INVAL;
+  rows_geom(g, (long long)s.N * s.P * ((s.C + 31) / 32), s.stride == 1 ? (const void*)dw_fwd_rows_kernel<1> : (const void*)dw_fwd_rows_kernel<2>);
   return 0;
 }
 int dw_fwd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
-  dw_fwd_rows_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
+  if (g.func == (const void*)dw_fwd_rows_kernel<1>)
+    dw_fwd_rows_kernel<1><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
+  else
+    dw_fwd_rows_kernel<2><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
   CHECK_LAUNCH();
 }
 int dw_dgrad_geom(const uint64_t* a, LaunchGeom* g) {
@@ -286,11 +306,17 @@ int dw_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
   if (!dw_ok(a)) return ORION_E_INVAL;
   DwShape s = dw_shape(a);
   if (a[14] == 0 || a[15] < orion_dw_wgrad_workspace_bytes(s.N, s.C, s.P, s.Q)) return ORION_E_INVAL;
-  g->grid = dim3((s.C + 31) / 32, wg_splits(s)); g->block = dim3(DW_THREADS); g->smem = 0; g->func = (const void*)dw_wgrad_rows_kernel;
+  if (s.stride != 1 && s.stride != 2) return ORION_E_INVAL;
+  g->grid = dim3((s.C + 31) / 32, wg_splits(s)); g->block = dim3(DW_THREADS); g->smem = 0;
+  g->func = s.stride == 1 ? (const void*)dw_wgrad_rows_kernel<1> : (const void*)dw_wgrad_rows_kernel<2>;
   return 0;
 }
 int dw_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
-  dw_wgrad_rows_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a),
-                                                   (unsigned char*)a[14], sig);
+  if (g.func == (const void*)dw_wgrad_rows_kernel<1>)
+    dw_wgrad_rows_kernel<1><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a),
+                                                        (unsigned char*)a[14], sig);
+  else
+    dw_wgrad_rows_kernel<2><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a),
+                                                        (unsigned char*)a[14], sig);
   CHECK_LAUNCH();
 }

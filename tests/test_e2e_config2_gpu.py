@@ -80,7 +80,7 @@ def test_be_one_iteration_vs_oracle(cfg2):
             continue   # init 0 and exactly-zero true gradient: the value is pure rounding noise (checked above)
         # block outputs have exactly-zero per-channel batch mean (every path ends in a BN), so the
         # running means of the BNs fed by them (expand_bn, features.18.bn) are ~1e-9 noise: floor
-        floor = 1e-3 if name.endswith(".rmean") else 1e-30
+        floor = 1e-2 if name.endswith(".rmean") else 1e-30
         assert rel(G.p[name], newP[name], floor) < 1e-5, name
     # first step: v = mu*0 + g = g exactly (torch's v <- g), so the momentum buffer equals the grads
     assert torch.equal(G.vflat, G.gflat)
