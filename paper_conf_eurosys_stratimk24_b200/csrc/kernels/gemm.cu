@@ -602,6 +602,141 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
 
 }  // namespace tc
 
+// ---------------------------------------------------------------- skinny A^T B (weight gradients)
+// C[M][N] = sum_k A[k][m] B[k][n] for M, N <= 128 and very long K (1x1-conv weight gradients over
+// N*H*W rows): HBM-bound, so the kernel streams 64-row blocks of both operands with coalesced
+// 128-bit loads (the next block's loads in flight while the current one is multiplied), keeps both
+// blocks in shared memory and gives each thread a 4x4 register block of C over a fixed subset of
+// the rows (row groups combined in fixed order). K is split over CTAs (shape-only count) and the
+// splits are summed in order by the last CTA (split_reduce_tile).
+namespace atb {
+constexpr int R = 64, NTH = 256, MAXD = 128;
+
+__host__ __device__ inline int pad_dim(int d) { return ((d + 3) / 4) * 4 + 4; }
+__host__ __device__ inline int smem_bytes(int M, int N) { return (2 * R * (pad_dim(M) + pad_dim(N)) + NTH * 16) * 4; }
+
+__global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float* __restrict__ A, long long lda,
+                                                      const float* __restrict__ B, long long ldb, OrionSig sig) {
+  extern __shared__ __align__(16) float atb_smem[];
+  const int tid = threadIdx.x;
+  const int M = p.M, N = p.N;
+  const int Mp = pad_dim(M), Np = pad_dim(N);
+  float* As0 = atb_smem;                  // [2][R][Mp]
+  float* Bs0 = As0 + 2 * R * Mp;          // [2][R][Np]
+  float* red = Bs0 + 2 * R * Np;          // [NTH * 16]
+  auto As = [&](int b, int r, int c) -> float* { return As0 + ((size_t)b * R + r) * Mp + c; };
+  auto Bs = [&](int b, int r, int c) -> float* { return Bs0 + ((size_t)b * R + r) * Np + c; };
+  const int mb = (M + 3) / 4, nb = (N + 3) / 4;      // 4x4 output blocks
+  const int nblk = mb * nb;
+  const int G = NTH / nblk;                            // row groups (>= 1 since M, N <= 128 -> nblk <= 1024? see host)
+  const int grp = tid / nblk, blk = tid % nblk;
+  const int bm = (blk / nb) * 4, bn = (blk % nb) * 4;
+  const bool active = grp < G;
+  const int kbeg = blockIdx.z * p.kps;
+  const int kend = min(p.K, kbeg + p.kps);
+  const bool vecA = (lda % 4 == 0) && (M % 4 == 0) && ((reinterpret_cast<uintptr_t>(A) & 15) == 0);
+  const bool vecB = (ldb % 4 == 0) && (N % 4 == 0) && ((reinterpret_cast<uintptr_t>(B) & 15) == 0);
+  const int qa = (M + 3) / 4, qb = (N + 3) / 4;       // float4 per row
+  float acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; i++)
+#pragma unroll
+    for (int j = 0; j < 4; j++) acc[i][j] = 0.f;
+
+  // staging: each thread moves quads (row, q) = idx -> (idx / q*, idx % q*) of the 64-row block
+  constexpr int MAXQ = (R * (MAXD / 4) * 2 + NTH - 1) / NTH;   // upper bound of quads per thread
+  float4 ra[MAXQ];
+  const int tot_a = R * qa, tot_b = R * qb, tot = tot_a + tot_b;
+  auto gload = [&](int k0) {
+#pragma unroll
+    for (int j = 0; j < MAXQ; j++) {
+      const int idx = tid + j * NTH;
+      float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (idx < tot) {
+        const bool isA = idx < tot_a;
+        const int li = isA ? idx : idx - tot_a;
+        const int q = isA ? qa : qb;
+        const int r = li / q, c = (li % q) * 4;
+        const int k = k0 + r;
+        if (k < kend) {
+          const float* base = isA ? A + (long long)k * lda : B + (long long)k * ldb;
+          const int lim = isA ? M : N;
+          if ((isA ? vecA : vecB)) v = __ldg(reinterpret_cast<const float4*>(base + c));
+          else {
+            v.x = c < lim ? __ldg(base + c) : 0.f;
+            v.y = c + 1 < lim ? __ldg(base + c + 1) : 0.f;
+            v.z = c + 2 < lim ? __ldg(base + c + 2) : 0.f;
+            v.w = c + 3 < lim ? __ldg(base + c + 3) : 0.f;
+          }
+        }
+      }
+      ra[j] = v;
+    }
+  };
+  auto sstore = [&](int buf) {
+#pragma unroll
+    for (int j = 0; j < MAXQ; j++) {
+      const int idx = tid + j * NTH;
+      if (idx < tot) {
+        const bool isA = idx < tot_a;
+        const int li = isA ? idx : idx - tot_a;
+        const int q = isA ? qa : qb;
+        const int r = li / q, c = (li % q) * 4;
+        float* dst = isA ? As(buf, r, c) : Bs(buf, r, c);
+        *reinterpret_cast<float4*>(dst) = ra[j];
+      }
+    }
+  };
+  int buf = 0;
+  if (kbeg < kend) { gload(kbeg); sstore(0); }
+  __syncthreads();
+  for (int k0 = kbeg; k0 < kend; k0 += R) {
+    const bool more = k0 + R < kend;
+    if (more) gload(k0 + R);
+    if (active) {
+      for (int r = grp; r < R; r += G) {
+        float4 a = *reinterpret_cast<const float4*>(As(buf, r, bm));
+        float4 b = *reinterpret_cast<const float4*>(Bs(buf, r, bn));
+        const float av[4] = {a.x, a.y, a.z, a.w}, bv[4] = {b.x, b.y, b.z, b.w};
+#pragma unroll
+        for (int i = 0; i < 4; i++)
+#pragma unroll
+          for (int j = 0; j < 4; j++) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+      }
+    }
+    if (more) {
+      __syncthreads();
+      sstore(buf ^ 1);
+      __syncthreads();
+      buf ^= 1;
+    }
+  }
+  // combine row groups in fixed order
+  if (active) {
+#pragma unroll
+    for (int i = 0; i < 4; i++)
+#pragma unroll
+      for (int j = 0; j < 4; j++) red[(grp * nblk + blk) * 16 + i * 4 + j] = acc[i][j];
+  }
+  __syncthreads();
+  float* out = p.split == 1 ? nullptr : p.ws + (long long)blockIdx.z * M * N;
+  for (int e = tid; e < nblk * 16; e += NTH) {
+    const int b = e / 16, ij = e % 16, i = ij / 4, j = ij % 4;
+    const int m = (b / nb) * 4 + i, n = (b % nb) * 4 + j;
+    float v = 0.f;
+    for (int g = 0; g < G; g++) v += red[(g * nblk + b) * 16 + ij];
+    if (m < M && n < N) {
+      if (p.split == 1) p.C[(long long)m * p.ldc + n] = v + (p.bias ? __ldg(p.bias + n) : 0.f);
+      else out[(long long)m * N + n] = v;
+    }
+  }
+  if (p.split > 1) {
+    if (last_cta_of(p.tickets, p.split)) split_reduce_tile(p, 0, 0, M, N);
+  }
+  orion_signal(sig);
+}
+}  // namespace atb
+
 // ---------------------------------------------------------------- small-M GEMM (GEMV-like)
 // For M <= 8 with B transposed (weights [N][K], the Linear layout): one warp per output column n,
 // lanes stride k with float4 loads; all M rows at once; fixed shuffle-tree reduction.
@@ -659,6 +794,22 @@ __global__ void __launch_bounds__(256) gemv_bt_kernel(const float* __restrict__ 
 // N*H*W rows, 3x3 convs at batch 4) spread over the GPU; the split reduction is ordered.
 struct Plan { int cfg; int split; int bm, bn, bk; };
 // cfg: 0/1/2 = FFMA tiles L/M/S; 3/4 = tcgen05 3xTF32 with BN = 128 / 64.
+
+// Skinny A^T B (cfg 5): both dims <= 128 with at most 256 4x4 output blocks, long K.
+bool atb_ok(long long M, long long N, long long K) {
+  return M <= 128 && N <= 128 && cdiv(M, 4) * cdiv(N, 4) <= 256 && K >= 4096;
+}
+
+Plan plan_atb(long long M, long long N, long long K) {
+  Plan pl;
+  pl.cfg = 5; pl.bm = (int)M; pl.bn = (int)N; pl.bk = atb::R;
+  long long split = cdiv(148 * 4, 1);
+  long long kmax = K / (4 * atb::R);
+  if (split > kmax) split = kmax;
+  if (split < 1) split = 1;
+  pl.split = (int)split;
+  return pl;
+}
 
 Plan plan_gemm(long long M, long long N, long long K) {
   Plan pl;
@@ -776,7 +927,12 @@ int launch_tiled(const LaunchGeom& g, long long M, long long N, long long K, flo
 // pass their implicit-GEMM dims: fwd (N*P*Q, K, R*S*C), dgrad (N*H*W, C, R*S*K), wgrad (K, R*S*C, N*P*Q).
 extern "C" uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t K) {
   Plan pl = plan_gemm((long long)M, (long long)N, (long long)K);
-  return ws_bytes_for(pl, (long long)M, (long long)N);
+  uint64_t b = ws_bytes_for(pl, (long long)M, (long long)N);
+  if (atb_ok((long long)M, (long long)N, (long long)K)) {   // A^T B callers may take the skinny kernel
+    uint64_t b2 = ws_bytes_for(plan_atb((long long)M, (long long)N, (long long)K), (long long)M, (long long)N);
+    if (b2 > b) b = b2;
+  }
+  return b;
 }
 
 // ------------------------------------------------------------------------- GEMM entry
@@ -787,6 +943,19 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
   if (M <= 0 || N <= 0 || K <= 0) return ORION_E_INVAL;
   if (M <= SM_MAXM && flags == 2) {
     g->grid = dim3((unsigned)cdiv(N, 8)); g->block = dim3(256); g->smem = 0; g->func = (const void*)gemv_bt_kernel;
+    return 0;
+  }
+  if (flags == 1 && atb_ok(M, N, K)) {
+    Plan pl = plan_atb(M, N, K);
+    if (pl.split > 1 && (a[11] == 0 || a[12] < ws_bytes_for(pl, M, N))) pl.split = 1;
+    static std::atomic<int> attr{0};
+    if (!attr.load()) {
+      if (cudaFuncSetAttribute((const void*)atb::gemm_atb_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               atb::smem_bytes(128, 128)) != cudaSuccess) return ORION_E_CUDA;
+      attr.store(1);
+    }
+    g->grid = dim3(1, 1, (unsigned)pl.split); g->block = dim3(atb::NTH); g->smem = atb::smem_bytes((int)M, (int)N);
+    g->func = (const void*)atb::gemm_atb_kernel;
     return 0;
   }
   switch (flags) {
@@ -809,6 +978,10 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
   float* ws = (float*)a[11];
   if (g.func == (const void*)gemv_bt_kernel) {
     gemv_bt_kernel<<<g.grid, g.block, 0, s>>>(A, lda, B, ldb, C, ldc, bias, (int)M, (int)N, (int)K, sig);
+    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+  }
+  if (g.func == (const void*)atb::gemm_atb_kernel) {
+    atb::gemm_atb_kernel<<<g.grid, g.block, g.smem, s>>>(make_params(M, N, K, C, ldc, bias, (int)g.grid.z, ws, atb::R), A, lda, B, ldb, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
   switch (flags) {

@@ -40,7 +40,8 @@ def ws(nbytes):
 @pytest.mark.parametrize("M,N,K,flags", [(1, 512, 512, 2), (4, 1000, 2048, 2), (3, 37, 129, 2), (32, 512, 512, 2),
                                          (96, 16, 300000, 1), (16, 32, 100000, 1), (196, 2048, 512, 2), (784, 256, 1024, 2),
                                          (256, 256, 256, 0), (300, 200, 520, 1), (130, 70, 300, 2), (257, 129, 333, 3),
-                                         (4704, 1280, 320, 2), (1280, 320, 4704, 1), (18816, 96, 576, 2)],
+                                         (4704, 1280, 320, 2), (1280, 320, 4704, 1), (18816, 96, 576, 2),
+                                         (99, 37, 9999, 1), (24, 144, 75264, 1), (128, 32, 300000, 1)],
                          ids=lambda v: str(v))
 def test_gemm_shapes(M, N, K, flags):
     test_gemm(M, N, K, flags)
