@@ -56,6 +56,13 @@ struct ADense {          // A row-major [M][lda]
     if (r.ok && k + 3 < kend && al16(q)) return __ldg(reinterpret_cast<const float4*>(q));
     return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
   }
+  // address of element k (nullptr = zero) and of an aligned contiguous quad (true + ptr/nullptr)
+  __device__ const float* addr(const Row& r, int k, int kend) const { return (r.ok && k < kend) ? p + r.base + k : nullptr; }
+  __device__ bool addr4(const Row& r, int k, int kend, const float*& q) const {
+    if (!r.ok || k >= kend) { q = nullptr; return true; }
+    q = p + r.base + k;
+    return k + 3 < kend && al16(q);
+  }
 };
 struct ADenseT {         // A stored transposed: A(m,k) = p[k*ld + m]
   static constexpr bool kContigK = false;
@@ -66,6 +73,11 @@ struct ADenseT {         // A stored transposed: A(m,k) = p[k*ld + m]
   __device__ float4 at4(const Row& r, int k, int kend) const {
     return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
   }
+  __device__ const float* addr(const Row& r, int k, int kend) const { return (r.ok && k < kend) ? p + (long long)k * ld + r.m : nullptr; }
+  __device__ bool addr4(const Row& r, int k, int kend, const float*& q) const {
+    if (!r.ok || k >= kend) { q = nullptr; return true; }
+    return false;
+  }
 };
 struct BDense {          // B row-major [K][ldb]: B(k,n) = p[k*ld + n]
   static constexpr bool kContigK = false;
@@ -75,6 +87,11 @@ struct BDense {          // B row-major [K][ldb]: B(k,n) = p[k*ld + n]
   __device__ float at(const Col& c, int k, int K) const { return (c.ok && k < K) ? __ldg(p + (long long)k * ld + c.n) : 0.f; }
   __device__ float4 at4(const Col& c, int k, int kend) const {
     return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
+  }
+  __device__ const float* addr(const Col& c, int k, int kend) const { return (c.ok && k < kend) ? p + (long long)k * ld + c.n : nullptr; }
+  __device__ bool addr4(const Col& c, int k, int kend, const float*& q) const {
+    if (!c.ok || k >= kend) { q = nullptr; return true; }
+    return false;
   }
 };
 struct BDenseT {         // B stored transposed [N][ldb]: B(k,n) = p[n*ld + k]
@@ -87,6 +104,12 @@ struct BDenseT {         // B stored transposed [N][ldb]: B(k,n) = p[n*ld + k]
     const float* q = p + c.base + k;
     if (c.ok && k + 3 < kend && al16(q)) return __ldg(reinterpret_cast<const float4*>(q));
     return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
+  }
+  __device__ const float* addr(const Col& c, int k, int kend) const { return (c.ok && k < kend) ? p + c.base + k : nullptr; }
+  __device__ bool addr4(const Col& c, int k, int kend, const float*& q) const {
+    if (!c.ok || k >= kend) { q = nullptr; return true; }
+    q = p + c.base + k;
+    return k + 3 < kend && al16(q);
   }
 };
 
@@ -122,6 +145,19 @@ struct AIm2col {
       return make_float4(__ldg(q), __ldg(q + 1), __ldg(q + 2), __ldg(q + 3));
     }
     return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
+  }
+  __device__ const float* addr(const Row& r, int k, int kend) const {
+    if (!r.ok || k >= kend) return nullptr;
+    int c = k % s.C; int t = k / s.C; int ss = t % s.S; int rr = t / s.S;
+    int h = r.h0 + rr, w = r.w0 + ss;
+    if ((unsigned)h >= (unsigned)s.H || (unsigned)w >= (unsigned)s.W) return nullptr;
+    return x + r.nbase + ((long long)h * s.W + w) * s.C + c;
+  }
+  __device__ bool addr4(const Row& r, int k, int kend, const float*& q) const {
+    if (!r.ok || k >= kend) { q = nullptr; return true; }
+    if ((s.C & 3) != 0 || k + 3 >= kend) return false;
+    q = addr(r, k, kend);   // same tap for the 4 channels; nullptr = padding
+    return q == nullptr || al16(q);
   }
 };
 
@@ -161,6 +197,21 @@ struct ADgrad {
     }
     return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
   }
+  __device__ const float* addr(const Row& r, int k, int kend) const {
+    if (!r.ok || k >= kend) return nullptr;
+    int ko = k % s.K; int t = k / s.K; int ss = t % s.S; int rr = t / s.S;
+    int ph = r.hp - rr, pw = r.wp - ss;
+    if (ph < 0 || pw < 0 || ph % s.stride || pw % s.stride) return nullptr;
+    int p = ph / s.stride, q = pw / s.stride;
+    if (p >= s.P || q >= s.Q) return nullptr;
+    return dy + r.nbase + ((long long)p * s.Q + q) * s.K + ko;
+  }
+  __device__ bool addr4(const Row& r, int k, int kend, const float*& q) const {
+    if (!r.ok || k >= kend) { q = nullptr; return true; }
+    if ((s.K & 3) != 0 || k + 3 >= kend) return false;
+    q = addr(r, k, kend);
+    return q == nullptr || al16(q);
+  }
 };
 // Conv dgrad B: B(k = (r,s,kout), n = c) = w[kout][r][s][c]
 struct BDgrad {
@@ -175,6 +226,15 @@ struct BDgrad {
   }
   __device__ float4 at4(const Col& c, int k, int kend) const {
     return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
+  }
+  __device__ const float* addr(const Col& cc, int k, int kend) const {
+    if (!cc.ok || k >= kend) return nullptr;
+    int ko = k % s.K; int t = k / s.K; int ss = t % s.S; int rr = t / s.S;
+    return w + (((long long)ko * s.R + rr) * s.S + ss) * s.C + cc.c;
+  }
+  __device__ bool addr4(const Col& c, int k, int kend, const float*& q) const {
+    if (!c.ok || k >= kend) { q = nullptr; return true; }
+    return false;
   }
 };
 // Conv wgrad B: B(k = (n,p,q), col = (r,s,c)) = x[n, p*st-pad+r, q*st-pad+s, c]
@@ -196,6 +256,17 @@ struct BWgrad {
   }
   __device__ float4 at4(const Col& c, int k, int kend) const {
     return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
+  }
+  __device__ const float* addr(const Col& cc, int k, int kend) const {
+    if (!cc.ok || k >= kend) return nullptr;
+    int q = k % s.Q; int t = k / s.Q; int p = t % s.P; int n = t / s.P;
+    int h = p * s.stride - s.pad + cc.r, w = q * s.stride - s.pad + cc.ss;
+    if ((unsigned)h >= (unsigned)s.H || (unsigned)w >= (unsigned)s.W) return nullptr;
+    return x + (((long long)n * s.H + h) * s.W + w) * s.C + cc.c;
+  }
+  __device__ bool addr4(const Col& c, int k, int kend, const float*& q) const {
+    if (!c.ok || k >= kend) { q = nullptr; return true; }
+    return false;
   }
 };
 
@@ -399,6 +470,18 @@ __device__ __forceinline__ bool mbar_try(uint32_t a, uint32_t parity) {
   return ok != 0;
 }
 __device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity) { while (!mbar_try(a, parity)) {} }
+__device__ __forceinline__ void cp_async16(uint32_t dst, const float* src) {
+  // zero-fill when src == nullptr (src-size 0 reads nothing; the address operand must still be valid)
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src ? src : reinterpret_cast<const float*>(&cp_async16)),
+               "r"(src ? 16 : 0) : "memory");
+}
+__device__ __forceinline__ void cp_async4(uint32_t dst, const float* src) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(dst), "l"(src ? src : reinterpret_cast<const float*>(&cp_async16)),
+               "r"(src ? 4 : 0) : "memory");
+}
+__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N_>
+__device__ __forceinline__ void cp_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N_) : "memory"); }
 __device__ __forceinline__ float tf32_rna(float x) {
   uint32_t u;
   asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(u) : "f"(x));
@@ -486,52 +569,85 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
   const uint32_t tmem = *tmem_slot;
 
   if (warp < NPROD / 32) {
-    // ---------------- producers: TPR threads per operand row, each staging 8/TPR k-quads per stage.
-    // All of a stage's global loads are issued before any hi/lo split or shared store.
+    // ---------------- producers. Each thread owns fixed k-quads of one A row and one B row per
+    // stage. Raw fp32 quads are copied global -> shared with cp.async (STAGES-1 stages in flight,
+    // zero-fill for padding / out-of-range), then each thread splits its own quads in place
+    // (hi = rna_tf32(x) over the raw copy, lo = x - hi into the lo buffer) and arrives on the
+    // stage's full barrier after a proxy fence.
+    constexpr int S = Cfg::STAGES;
     constexpr int A_TPR = NPROD / BM, A_QPT = 8 / A_TPR;           // 2 threads per A row, 4 quads each
-    constexpr int B_TPR = NPROD / BN >= 1 ? NPROD / BN : 1;
+    constexpr int BROWS = BN < NPROD ? BN : NPROD;
+    constexpr int B_TPR = NPROD / BROWS;
     constexpr int B_QPT = 8 / B_TPR >= 1 ? 8 / B_TPR : 1;
-    constexpr int B_RPT = BN > NPROD ? BN / NPROD : 1;             // rows per thread (BN > 256 only)
     const int a_row = tid % BM, a_q0 = (tid / BM) * A_QPT;
     typename LA::Row arow = la.row(m0 + a_row, p.M);
-    const int b_row = tid % (BN < NPROD ? BN : NPROD), b_q0 = (tid / (BN < NPROD ? BN : NPROD)) * B_QPT;
-    typename LB::Col bcol[B_RPT];
-#pragma unroll
-    for (int j = 0; j < B_RPT; j++) bcol[j] = lb.col(n0 + b_row + j * NPROD, p.N);
-    for (int kt = 0; kt < nk; kt++) {
-      const int s = kt % Cfg::STAGES;
-      const uint32_t ph = (uint32_t)(kt / Cfg::STAGES) & 1u;
+    const int b_row = tid % BROWS, b_q0 = (tid / BROWS) * B_QPT;
+    const bool b_on = tid < B_TPR * BROWS && b_row < BN;
+    typename LB::Col bcol = lb.col(n0 + b_row, p.N);
+    auto issue = [&](int kt) {
+      const int s = kt % S;
+      const uint32_t st = smem_u32(smem + s * Cfg::STAGE_BYTES);
+      const uint32_t a_hi = st, b_hi = st + 2 * Cfg::A_BYTES;
       const int k0 = kbeg + kt * BK;
-      float4 va[A_QPT], vb[B_RPT][B_QPT];
 #pragma unroll
-      for (int q = 0; q < A_QPT; q++) va[q] = la.at4(arow, k0 + (a_q0 + q) * 4, kend);
+      for (int q = 0; q < A_QPT; q++) {
+        const int k = k0 + (a_q0 + q) * 4;
+        const uint32_t dst = a_hi + elem_off(a_row, a_q0 + q, BM);
+        const float* src;
+        if (la.addr4(arow, k, kend, src)) cp_async16(dst, src);
+        else {
 #pragma unroll
-      for (int j = 0; j < B_RPT; j++)
+          for (int e = 0; e < 4; e++) cp_async4(dst + 4 * e, la.addr(arow, k + e, kend));
+        }
+      }
+      if (b_on) {
 #pragma unroll
-        for (int q = 0; q < B_QPT; q++) vb[j][q] = lb.at4(bcol[j], k0 + (b_q0 + q) * 4, kend);
-      mbar_wait(empty0 + 8 * s, ph ^ 1u);
+        for (int q = 0; q < B_QPT; q++) {
+          const int k = k0 + (b_q0 + q) * 4;
+          const uint32_t dst = b_hi + elem_off(b_row, b_q0 + q, BN);
+          const float* src;
+          if (lb.addr4(bcol, k, kend, src)) cp_async16(dst, src);
+          else {
+#pragma unroll
+            for (int e = 0; e < 4; e++) cp_async4(dst + 4 * e, lb.addr(bcol, k + e, kend));
+          }
+        }
+      }
+    };
+    auto split = [](unsigned char* hi, unsigned char* lo, uint32_t off) {
+      float4 v = *reinterpret_cast<float4*>(hi + off), h, l;
+      h.x = tf32_rna(v.x); h.y = tf32_rna(v.y); h.z = tf32_rna(v.z); h.w = tf32_rna(v.w);
+      l.x = v.x - h.x; l.y = v.y - h.y; l.z = v.z - h.z; l.w = v.w - h.w;
+      *reinterpret_cast<float4*>(hi + off) = h;
+      *reinterpret_cast<float4*>(lo + off) = l;
+    };
+    // prologue: stages 0 .. S-2 (fresh barriers: the empty waits pass at once)
+#pragma unroll 1
+    for (int kt = 0; kt < S - 1; kt++) {
+      if (kt < nk) issue(kt);
+      cp_commit();
+    }
+#pragma unroll 1
+    for (int kt = 0; kt < nk; kt++) {
+      cp_wait<S - 2>();                                  // this thread's copies for stage kt landed
+      const int s = kt % S;
       unsigned char* st = smem + s * Cfg::STAGE_BYTES;
-      unsigned char* a_hi = st;
-      unsigned char* a_lo = st + Cfg::A_BYTES;
-      unsigned char* b_hi = st + 2 * Cfg::A_BYTES;
-      unsigned char* b_lo = b_hi + Cfg::B_BYTES;
-      auto split_store = [](unsigned char* hi, unsigned char* lo, uint32_t off, const float4& v) {
-        float4 h, l;
-        h.x = tf32_rna(v.x); h.y = tf32_rna(v.y); h.z = tf32_rna(v.z); h.w = tf32_rna(v.w);
-        l.x = v.x - h.x; l.y = v.y - h.y; l.z = v.z - h.z; l.w = v.w - h.w;
-        *reinterpret_cast<float4*>(hi + off) = h;
-        *reinterpret_cast<float4*>(lo + off) = l;
-      };
 #pragma unroll
-      for (int q = 0; q < A_QPT; q++) split_store(a_hi, a_lo, elem_off(a_row, a_q0 + q, BM), va[q]);
-      if (tid < B_TPR * (BN < NPROD ? BN : NPROD)) {
+      for (int q = 0; q < A_QPT; q++) split(st, st + Cfg::A_BYTES, elem_off(a_row, a_q0 + q, BM));
+      if (b_on) {
 #pragma unroll
-        for (int j = 0; j < B_RPT; j++)
-#pragma unroll
-          for (int q = 0; q < B_QPT; q++) split_store(b_hi, b_lo, elem_off(b_row + j * NPROD, b_q0 + q, BN), vb[j][q]);
+        for (int q = 0; q < B_QPT; q++)
+          split(st + 2 * Cfg::A_BYTES, st + 2 * Cfg::A_BYTES + Cfg::B_BYTES, elem_off(b_row, b_q0 + q, BN));
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic-proxy writes -> tensor core
       mbar_arrive(full0 + 8 * s);
+      const int nxt = kt + S - 1;
+      if (nxt < nk) {
+        const int sn = nxt % S;
+        mbar_wait(empty0 + 8 * sn, ((uint32_t)(nxt / S) & 1u) ^ 1u);   // MMA finished reading it
+        issue(nxt);
+      }
+      cp_commit();
     }
   } else if (warp == NPROD / 32 && lane == 0) {
     // ---------------- MMA issuer (one thread)

@@ -1,0 +1,12 @@
+#!/bin/bash
+# ncu --set full on a few named ops (solo runner), reports under gpurun_out/
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+OURS='(gemm_kernel|gemm_tc_kernel|gemm_atb_kernel|gemv_bt_kernel|unary_kernel|binary_kernel|bn_|dw_|maxpool_kernel|avgpool|ce_kernel|mse_kernel|sgd_kernel|colsum_kernel)'
+for spec in $FOCUS; do
+  client=${spec%%:*}; only=${spec#*:}
+  tag=$(echo "$only" | tr -c 'a-zA-Z0-9\n' '_')
+  timeout -s KILL 600 ncu --set full --clock-control none --import-source on --kernel-name-base function -k "regex:$OURS" -c ${NCU_C:-4} \
+     -o gpurun_out/ncu_${client}_${tag} python tools/profile/solo_runner.py --client $client --only "$only" > gpurun_out/ncu_${client}_${tag}.out 2>&1
+  echo "$spec rc=$?"
+done
