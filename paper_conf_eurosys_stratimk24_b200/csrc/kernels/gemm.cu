@@ -454,7 +454,7 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
 // im2col / transposed-view functors as the FFMA path, so every conv kind runs on this kernel.
 namespace tc {
 
-constexpr int BM = 128, BK = 32, NPROD = 256, NTHR = 288;   // 8 producer warps + 1 MMA warp
+constexpr int BM = 128, BK = 16, NPROD = 256, NTHR = 288;   // 8 producer warps + 1 MMA warp
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint32_t a, uint32_t cnt) {
@@ -517,7 +517,7 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
 
 template <int BN>
 struct TcCfg {
-  static constexpr int STAGES = BN >= 128 ? 3 : 4;
+  static constexpr int STAGES = BN >= 128 ? 6 : 8;   // ~192 KB of stages: deep enough to cover L2/HBM latency
   static constexpr int A_BYTES = BM * BK * 4;   // one of hi / lo
   static constexpr int B_BYTES = BN * BK * 4;
   static constexpr int STAGE_BYTES = 2 * (A_BYTES + B_BYTES);
@@ -575,10 +575,11 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
     // (hi = rna_tf32(x) over the raw copy, lo = x - hi into the lo buffer) and arrives on the
     // stage's full barrier after a proxy fence.
     constexpr int S = Cfg::STAGES;
-    constexpr int A_TPR = NPROD / BM, A_QPT = 8 / A_TPR;           // 2 threads per A row, 4 quads each
+    constexpr int KQ = BK / 4;                                    // k-quads per row per stage
+    constexpr int A_TPR = NPROD / BM, A_QPT = KQ / A_TPR;          // 2 threads per A row
     constexpr int BROWS = BN < NPROD ? BN : NPROD;
     constexpr int B_TPR = NPROD / BROWS;
-    constexpr int B_QPT = 8 / B_TPR >= 1 ? 8 / B_TPR : 1;
+    constexpr int B_QPT = KQ / B_TPR >= 1 ? KQ / B_TPR : 1;
     const int a_row = tid % BM, a_q0 = (tid / BM) * A_QPT;
     typename LA::Row arow = la.row(m0 + a_row, p.M);
     const int b_row = tid % BROWS, b_q0 = (tid / BROWS) * B_QPT;
