@@ -45,17 +45,18 @@ struct GemmParams {
 // 4 are contiguous and aligned, else 4 scalar loads.
 __device__ __forceinline__ bool al16(const float* q) { return (reinterpret_cast<uintptr_t>(q) & 15) == 0; }
 
+// Per-k-tile address helpers for the tensor-core producer: tile(k0, kend, bk) precomputes what is
+// uniform over the tile (a conv tap when the tile lies inside one tap's channels); quad(row, t,
+// kq, kend, q) then resolves quad kq of the tile for one row with a few adds. Loaders without a
+// fast path fall back to addr4 / addr.
+struct NoTile { int k0; };
+
 struct ADense {          // A row-major [M][lda]
   static constexpr bool kContigK = true;
   const float* p; long long ld;
   struct Row { long long base; bool ok; };
   __device__ Row row(int m, int M) const { return {(long long)m * ld, m < M}; }
   __device__ float at(const Row& r, int k, int K) const { return (r.ok && k < K) ? __ldg(p + r.base + k) : 0.f; }
-  __device__ float4 at4(const Row& r, int k, int kend) const {
-    const float* q = p + r.base + k;
-    if (r.ok && k + 3 < kend && al16(q)) return __ldg(reinterpret_cast<const float4*>(q));
-    return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
-  }
   // address of element k (nullptr = zero) and of an aligned contiguous quad (true + ptr/nullptr)
   __device__ const float* addr(const Row& r, int k, int kend) const { return (r.ok && k < kend) ? p + r.base + k : nullptr; }
   __device__ bool addr4(const Row& r, int k, int kend, const float*& q) const {
@@ -63,6 +64,9 @@ struct ADense {          // A row-major [M][lda]
     q = p + r.base + k;
     return k + 3 < kend && al16(q);
   }
+  __device__ NoTile tile(int k0, int, int) const { return {k0}; }
+  template <class RC>
+  __device__ bool quad(const RC& r, const NoTile& t, int kq, int kend, const float*& q) const { return addr4(r, t.k0 + 4 * kq, kend, q); }
 };
 struct ADenseT {         // A stored transposed: A(m,k) = p[k*ld + m]
   static constexpr bool kContigK = false;
@@ -70,14 +74,14 @@ struct ADenseT {         // A stored transposed: A(m,k) = p[k*ld + m]
   struct Row { int m; bool ok; };
   __device__ Row row(int m, int M) const { return {m, m < M}; }
   __device__ float at(const Row& r, int k, int K) const { return (r.ok && k < K) ? __ldg(p + (long long)k * ld + r.m) : 0.f; }
-  __device__ float4 at4(const Row& r, int k, int kend) const {
-    return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
-  }
   __device__ const float* addr(const Row& r, int k, int kend) const { return (r.ok && k < kend) ? p + (long long)k * ld + r.m : nullptr; }
   __device__ bool addr4(const Row& r, int k, int kend, const float*& q) const {
     if (!r.ok || k >= kend) { q = nullptr; return true; }
     return false;
   }
+  __device__ NoTile tile(int k0, int, int) const { return {k0}; }
+  template <class RC>
+  __device__ bool quad(const RC& r, const NoTile& t, int kq, int kend, const float*& q) const { return addr4(r, t.k0 + 4 * kq, kend, q); }
 };
 struct BDense {          // B row-major [K][ldb]: B(k,n) = p[k*ld + n]
   static constexpr bool kContigK = false;
@@ -85,14 +89,14 @@ struct BDense {          // B row-major [K][ldb]: B(k,n) = p[k*ld + n]
   struct Col { int n; bool ok; };
   __device__ Col col(int n, int N) const { return {n, n < N}; }
   __device__ float at(const Col& c, int k, int K) const { return (c.ok && k < K) ? __ldg(p + (long long)k * ld + c.n) : 0.f; }
-  __device__ float4 at4(const Col& c, int k, int kend) const {
-    return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
-  }
   __device__ const float* addr(const Col& c, int k, int kend) const { return (c.ok && k < kend) ? p + (long long)k * ld + c.n : nullptr; }
   __device__ bool addr4(const Col& c, int k, int kend, const float*& q) const {
     if (!c.ok || k >= kend) { q = nullptr; return true; }
     return false;
   }
+  __device__ NoTile tile(int k0, int, int) const { return {k0}; }
+  template <class RC>
+  __device__ bool quad(const RC& r, const NoTile& t, int kq, int kend, const float*& q) const { return addr4(r, t.k0 + 4 * kq, kend, q); }
 };
 struct BDenseT {         // B stored transposed [N][ldb]: B(k,n) = p[n*ld + k]
   static constexpr bool kContigK = true;
@@ -100,17 +104,15 @@ struct BDenseT {         // B stored transposed [N][ldb]: B(k,n) = p[n*ld + k]
   struct Col { long long base; bool ok; };
   __device__ Col col(int n, int N) const { return {(long long)n * ld, n < N}; }
   __device__ float at(const Col& c, int k, int K) const { return (c.ok && k < K) ? __ldg(p + c.base + k) : 0.f; }
-  __device__ float4 at4(const Col& c, int k, int kend) const {
-    const float* q = p + c.base + k;
-    if (c.ok && k + 3 < kend && al16(q)) return __ldg(reinterpret_cast<const float4*>(q));
-    return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
-  }
   __device__ const float* addr(const Col& c, int k, int kend) const { return (c.ok && k < kend) ? p + c.base + k : nullptr; }
   __device__ bool addr4(const Col& c, int k, int kend, const float*& q) const {
     if (!c.ok || k >= kend) { q = nullptr; return true; }
     q = p + c.base + k;
     return k + 3 < kend && al16(q);
   }
+  __device__ NoTile tile(int k0, int, int) const { return {k0}; }
+  template <class RC>
+  __device__ bool quad(const RC& r, const NoTile& t, int kq, int kend, const float*& q) const { return addr4(r, t.k0 + 4 * kq, kend, q); }
 };
 
 struct ConvShape { int N, H, W, C, K, R, S, stride, pad, P, Q; };
@@ -134,18 +136,6 @@ struct AIm2col {
     if ((unsigned)h >= (unsigned)s.H || (unsigned)w >= (unsigned)s.W) return 0.f;
     return __ldg(x + r.nbase + ((long long)h * s.W + w) * s.C + c);
   }
-  __device__ float4 at4(const Row& r, int k, int kend) const {
-    if ((s.C & 3) == 0 && k + 3 < kend) {   // same (r, s) tap, 4 consecutive channels
-      if (!r.ok) return make_float4(0.f, 0.f, 0.f, 0.f);
-      int c = k % s.C; int t = k / s.C; int ss = t % s.S; int rr = t / s.S;
-      int h = r.h0 + rr, w = r.w0 + ss;
-      if ((unsigned)h >= (unsigned)s.H || (unsigned)w >= (unsigned)s.W) return make_float4(0.f, 0.f, 0.f, 0.f);
-      const float* q = x + r.nbase + ((long long)h * s.W + w) * s.C + c;
-      if (al16(q)) return __ldg(reinterpret_cast<const float4*>(q));
-      return make_float4(__ldg(q), __ldg(q + 1), __ldg(q + 2), __ldg(q + 3));
-    }
-    return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
-  }
   __device__ const float* addr(const Row& r, int k, int kend) const {
     if (!r.ok || k >= kend) return nullptr;
     int c = k % s.C; int t = k / s.C; int ss = t % s.S; int rr = t / s.S;
@@ -158,6 +148,20 @@ struct AIm2col {
     if ((s.C & 3) != 0 || k + 3 >= kend) return false;
     q = addr(r, k, kend);   // same tap for the 4 channels; nullptr = padding
     return q == nullptr || al16(q);
+  }
+  // tile inside one tap (C % bk == 0): every row's quad kq is 4 consecutive channels at one pixel
+  struct Tile { int k0, rr, ss, c0; bool fast; };
+  __device__ Tile tile(int k0, int kend, int bk) const {
+    Tile t; t.k0 = k0; t.fast = (s.C % bk) == 0 && k0 + bk <= kend;
+    int c = k0 % s.C, u = k0 / s.C; t.c0 = c; t.ss = u % s.S; t.rr = u / s.S;
+    return t;
+  }
+  __device__ bool quad(const Row& r, const Tile& t, int kq, int kend, const float*& q) const {
+    if (!t.fast) return addr4(r, t.k0 + 4 * kq, kend, q);
+    const int h = r.h0 + t.rr, w = r.w0 + t.ss;
+    if (!r.ok || (unsigned)h >= (unsigned)s.H || (unsigned)w >= (unsigned)s.W) { q = nullptr; return true; }
+    q = x + r.nbase + ((long long)h * s.W + w) * s.C + t.c0 + 4 * kq;
+    return al16(q);
   }
 };
 
@@ -183,20 +187,6 @@ struct ADgrad {
     if (p >= s.P || q >= s.Q) return 0.f;
     return __ldg(dy + r.nbase + ((long long)p * s.Q + q) * s.K + ko);
   }
-  __device__ float4 at4(const Row& r, int k, int kend) const {
-    if ((s.K & 3) == 0 && k + 3 < kend) {   // same tap, 4 consecutive output channels
-      if (!r.ok) return make_float4(0.f, 0.f, 0.f, 0.f);
-      int ko = k % s.K; int t = k / s.K; int ss = t % s.S; int rr = t / s.S;
-      int ph = r.hp - rr, pw = r.wp - ss;
-      if (ph < 0 || pw < 0 || ph % s.stride || pw % s.stride) return make_float4(0.f, 0.f, 0.f, 0.f);
-      int p = ph / s.stride, q = pw / s.stride;
-      if (p >= s.P || q >= s.Q) return make_float4(0.f, 0.f, 0.f, 0.f);
-      const float* qq = dy + r.nbase + ((long long)p * s.Q + q) * s.K + ko;
-      if (al16(qq)) return __ldg(reinterpret_cast<const float4*>(qq));
-      return make_float4(__ldg(qq), __ldg(qq + 1), __ldg(qq + 2), __ldg(qq + 3));
-    }
-    return make_float4(at(r, k, kend), at(r, k + 1, kend), at(r, k + 2, kend), at(r, k + 3, kend));
-  }
   __device__ const float* addr(const Row& r, int k, int kend) const {
     if (!r.ok || k >= kend) return nullptr;
     int ko = k % s.K; int t = k / s.K; int ss = t % s.S; int rr = t / s.S;
@@ -212,6 +202,21 @@ struct ADgrad {
     q = addr(r, k, kend);
     return q == nullptr || al16(q);
   }
+  struct Tile { int k0, rr, ss, ko0; bool fast; };
+  __device__ Tile tile(int k0, int kend, int bk) const {
+    Tile t; t.k0 = k0; t.fast = (s.K % bk) == 0 && k0 + bk <= kend;
+    int c = k0 % s.K, u = k0 / s.K; t.ko0 = c; t.ss = u % s.S; t.rr = u / s.S;
+    return t;
+  }
+  __device__ bool quad(const Row& r, const Tile& t, int kq, int kend, const float*& q) const {
+    if (!t.fast) return addr4(r, t.k0 + 4 * kq, kend, q);
+    const int ph = r.hp - t.rr, pw = r.wp - t.ss;
+    if (!r.ok || ph < 0 || pw < 0 || ph % s.stride || pw % s.stride) { q = nullptr; return true; }
+    const int p = ph / s.stride, qq = pw / s.stride;
+    if (p >= s.P || qq >= s.Q) { q = nullptr; return true; }
+    q = dy + r.nbase + ((long long)p * s.Q + qq) * s.K + t.ko0 + 4 * kq;
+    return al16(q);
+  }
 };
 // Conv dgrad B: B(k = (r,s,kout), n = c) = w[kout][r][s][c]
 struct BDgrad {
@@ -224,9 +229,6 @@ struct BDgrad {
     int ko = k % s.K; int t = k / s.K; int ss = t % s.S; int rr = t / s.S;
     return __ldg(w + (((long long)ko * s.R + rr) * s.S + ss) * s.C + cc.c);
   }
-  __device__ float4 at4(const Col& c, int k, int kend) const {
-    return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
-  }
   __device__ const float* addr(const Col& cc, int k, int kend) const {
     if (!cc.ok || k >= kend) return nullptr;
     int ko = k % s.K; int t = k / s.K; int ss = t % s.S; int rr = t / s.S;
@@ -236,6 +238,9 @@ struct BDgrad {
     if (!c.ok || k >= kend) { q = nullptr; return true; }
     return false;
   }
+  __device__ NoTile tile(int k0, int, int) const { return {k0}; }
+  template <class RC>
+  __device__ bool quad(const RC& r, const NoTile& t, int kq, int kend, const float*& q) const { return addr4(r, t.k0 + 4 * kq, kend, q); }
 };
 // Conv wgrad B: B(k = (n,p,q), col = (r,s,c)) = x[n, p*st-pad+r, q*st-pad+s, c]
 struct BWgrad {
@@ -254,9 +259,6 @@ struct BWgrad {
     if ((unsigned)h >= (unsigned)s.H || (unsigned)w >= (unsigned)s.W) return 0.f;
     return __ldg(x + (((long long)n * s.H + h) * s.W + w) * s.C + cc.c);
   }
-  __device__ float4 at4(const Col& c, int k, int kend) const {
-    return make_float4(at(c, k, kend), at(c, k + 1, kend), at(c, k + 2, kend), at(c, k + 3, kend));
-  }
   __device__ const float* addr(const Col& cc, int k, int kend) const {
     if (!cc.ok || k >= kend) return nullptr;
     int q = k % s.Q; int t = k / s.Q; int p = t % s.P; int n = t / s.P;
@@ -268,6 +270,9 @@ struct BWgrad {
     if (!c.ok || k >= kend) { q = nullptr; return true; }
     return false;
   }
+  __device__ NoTile tile(int k0, int, int) const { return {k0}; }
+  template <class RC>
+  __device__ bool quad(const RC& r, const NoTile& t, int kq, int kend, const float*& q) const { return addr4(r, t.k0 + 4 * kq, kend, q); }
 };
 
 // ---------------------------------------------------------------- ordered split-K reduction
@@ -590,12 +595,14 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
       const uint32_t st = smem_u32(smem + s * Cfg::STAGE_BYTES);
       const uint32_t a_hi = st, b_hi = st + 2 * Cfg::A_BYTES;
       const int k0 = kbeg + kt * BK;
+      const auto ta = la.tile(k0, kend, BK);
+      const auto tb = lb.tile(k0, kend, BK);
 #pragma unroll
       for (int q = 0; q < A_QPT; q++) {
         const int k = k0 + (a_q0 + q) * 4;
         const uint32_t dst = a_hi + elem_off(a_row, a_q0 + q, BM);
         const float* src;
-        if (la.addr4(arow, k, kend, src)) cp_async16(dst, src);
+        if (la.quad(arow, ta, a_q0 + q, kend, src)) cp_async16(dst, src);
         else {
 #pragma unroll
           for (int e = 0; e < 4; e++) cp_async4(dst + 4 * e, la.addr(arow, k + e, kend));
@@ -607,7 +614,7 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
           const int k = k0 + (b_q0 + q) * 4;
           const uint32_t dst = b_hi + elem_off(b_row, b_q0 + q, BN);
           const float* src;
-          if (lb.addr4(bcol, k, kend, src)) cp_async16(dst, src);
+          if (lb.quad(bcol, tb, b_q0 + q, kend, src)) cp_async16(dst, src);
           else {
 #pragma unroll
             for (int e = 0; e < 4; e++) cp_async4(dst + 4 * e, lb.addr(bcol, k + e, kend));
@@ -854,6 +861,72 @@ __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float
 }
 }  // namespace atb
 
+// ---------------------------------------------------------------- tall-skinny rows GEMM
+// C[M][N] = A[M][K] B for M >> N (N <= 32): 1x1-conv forward into few channels and the data
+// gradient of expand convs. HBM-bound on A and C, so each CTA streams a contiguous block of 256 rows
+// of A (coalesced 128-bit loads, transposed into shared memory so each thread reads its own row
+// conflict-free), B lives in shared memory for the whole CTA (broadcast reads), and each thread
+// accumulates its row's N outputs in registers in k order (deterministic, no split).
+namespace rows {
+constexpr int NTH = 256, KC = 32, MAXN = 32, MAXKN = 16384;
+
+template <bool BT>
+__global__ void __launch_bounds__(NTH) gemm_rows_kernel(const float* __restrict__ A, long long lda, const float* __restrict__ B,
+                                                       long long ldb, float* __restrict__ C, long long ldc,
+                                                       const float* __restrict__ bias, int M, int N, int K, OrionSig sig) {
+  extern __shared__ __align__(16) float rows_smem[];
+  float* Bs = rows_smem;                 // [K][N]
+  float* As = Bs + K * N;                // [KC][NTH + 1]
+  const int tid = threadIdx.x;
+  for (int i = tid; i < K * N; i += NTH) {
+    const int k = i / N, n = i % N;
+    Bs[i] = BT ? __ldg(B + (long long)n * ldb + k) : __ldg(B + (long long)k * ldb + n);
+  }
+  const long long r0 = (long long)blockIdx.x * NTH;
+  const int rows_here = (int)min((long long)NTH, (long long)M - r0);
+  float acc[MAXN];
+#pragma unroll
+  for (int n = 0; n < MAXN; n++) acc[n] = 0.f;
+  const bool vec = (lda % 4 == 0) && ((reinterpret_cast<uintptr_t>(A) & 15) == 0);
+  for (int k0 = 0; k0 < K; k0 += KC) {
+    const int kc = min(KC, K - k0);
+    __syncthreads();   // previous chunk consumed (and Bs staged on the first pass)
+    if (vec && (kc % 4) == 0) {
+      const int q = kc / 4;
+      for (int i = tid; i < rows_here * q; i += NTH) {
+        const int r = i / q, c = (i % q) * 4;
+        const float4 v = __ldg(reinterpret_cast<const float4*>(A + (r0 + r) * lda + k0 + c));
+        As[(c + 0) * (NTH + 1) + r] = v.x; As[(c + 1) * (NTH + 1) + r] = v.y;
+        As[(c + 2) * (NTH + 1) + r] = v.z; As[(c + 3) * (NTH + 1) + r] = v.w;
+      }
+    } else {
+      for (int i = tid; i < rows_here * kc; i += NTH) {
+        const int r = i / kc, c = i % kc;
+        As[c * (NTH + 1) + r] = __ldg(A + (r0 + r) * lda + k0 + c);
+      }
+    }
+    __syncthreads();
+    if (tid < rows_here) {
+      for (int kk = 0; kk < kc; kk++) {
+        const float a = As[kk * (NTH + 1) + tid];
+        const float* b = Bs + (k0 + kk) * N;
+#pragma unroll
+        for (int n = 0; n < MAXN; n++)
+          if (n < N) acc[n] = fmaf(a, b[n], acc[n]);
+      }
+    }
+  }
+  if (tid < rows_here) {
+    float* c = C + (r0 + tid) * ldc;
+#pragma unroll
+    for (int n = 0; n < MAXN; n++)
+      if (n < N) c[n] = acc[n] + (bias ? __ldg(bias + n) : 0.f);
+  }
+  orion_signal(sig);
+}
+inline int smem_bytes(int K, int N) { return (K * N + KC * (NTH + 1)) * 4; }
+}  // namespace rows
+
 // ---------------------------------------------------------------- small-M GEMM (GEMV-like)
 // For M <= 8 with B transposed (weights [N][K], the Linear layout): one warp per output column n,
 // lanes stride k with float4 loads; all M rows at once; fixed shuffle-tree reduction.
@@ -1062,6 +1135,20 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     g->grid = dim3((unsigned)cdiv(N, 8)); g->block = dim3(256); g->smem = 0; g->func = (const void*)gemv_bt_kernel;
     return 0;
   }
+  if ((flags == 0 || flags == 2) && M >= 4096 && N <= rows::MAXN && K * N <= rows::MAXKN) {
+    const void* f = flags == 2 ? (const void*)rows::gemm_rows_kernel<true> : (const void*)rows::gemm_rows_kernel<false>;
+    static std::atomic<int> attr{0};
+    if (!attr.load()) {
+      if (cudaFuncSetAttribute((const void*)rows::gemm_rows_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               rows::smem_bytes(rows::MAXKN, 1)) != cudaSuccess ||
+          cudaFuncSetAttribute((const void*)rows::gemm_rows_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               rows::smem_bytes(rows::MAXKN, 1)) != cudaSuccess)
+        return ORION_E_CUDA;
+      attr.store(1);
+    }
+    g->grid = dim3((unsigned)cdiv(M, rows::NTH)); g->block = dim3(rows::NTH); g->smem = rows::smem_bytes((int)K, (int)N); g->func = f;
+    return 0;
+  }
   if (flags == 1 && atb_ok(M, N, K)) {
     Plan pl = plan_atb(M, N, K);
     if (pl.split > 1 && (a[11] == 0 || a[12] < ws_bytes_for(pl, M, N))) pl.split = 1;
@@ -1095,6 +1182,13 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
   float* ws = (float*)a[11];
   if (g.func == (const void*)gemv_bt_kernel) {
     gemv_bt_kernel<<<g.grid, g.block, 0, s>>>(A, lda, B, ldb, C, ldc, bias, (int)M, (int)N, (int)K, sig);
+    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+  }
+  if (g.func == (const void*)rows::gemm_rows_kernel<true> || g.func == (const void*)rows::gemm_rows_kernel<false>) {
+    if (flags == 2)
+      rows::gemm_rows_kernel<true><<<g.grid, g.block, g.smem, s>>>(A, lda, B, ldb, C, ldc, bias, (int)M, (int)N, (int)K, sig);
+    else
+      rows::gemm_rows_kernel<false><<<g.grid, g.block, g.smem, s>>>(A, lda, B, ldb, C, ldc, bias, (int)M, (int)N, (int)K, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
   if (g.func == (const void*)atb::gemm_atb_kernel) {

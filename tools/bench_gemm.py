@@ -23,6 +23,6 @@ def run(M, N, K, flags, reps=10):
     print(f"M={M:6d} N={N:5d} K={K:6d} fl={flags} grid={grid:5d} thr={thr} smem={smem:6d}  {t*1e6:9.1f} us  {2*M*N*K/t/1e12:7.2f} TF/s")
 
 torch.cuda.set_device(0)
-for shp in [(4096, 4096, 4096, 2), (8192, 1024, 2048, 2), (2048, 2048, 8192, 0), (196, 512, 4608, 2), (784, 256, 2304, 2), (3136, 128, 1152, 2),
+for shp in [(128, 64, 64, 2), (128, 64, 1024, 2), (128, 128, 4096, 2), (256, 128, 1024, 2), (4096, 4096, 4096, 2), (8192, 1024, 2048, 2), (2048, 2048, 8192, 0), (196, 512, 4608, 2), (784, 256, 2304, 2), (3136, 128, 1152, 2),
             (4704, 1280, 320, 2), (1280, 320, 4704, 1), (12544, 64, 576, 2)]:
     run(*shp)

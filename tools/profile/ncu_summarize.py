@@ -6,23 +6,23 @@ import sys
 
 
 def parse(path):
+    """ncu --csv --page raw: one row per launch, metric names as columns (second row = units)."""
     txt = open(path).read()
     start = txt.find('"ID"')
-    rows = list(csv.DictReader(io.StringIO(txt[start:])))
-    out = {}
-    for r in rows:
-        try:
-            i = int(r["ID"])
-        except (KeyError, ValueError):
-            continue
-        d = out.setdefault(i, {"name": r.get("Kernel Name", "")})
-        name, val = r.get("Metric Name"), r.get("Metric Value", "").replace(",", "")
-        if name:
+    rows = list(csv.reader(io.StringIO(txt[start:])))
+    hdr = rows[0]
+    out = []
+    for r in rows[1:]:
+        if not r or not r[0].isdigit():
+            continue   # units row
+        d = {"name": r[hdr.index("Kernel Name")]}
+        for k, v in zip(hdr, r):
             try:
-                d[name] = float(val)
+                d[k] = float(v.replace(",", ""))
             except ValueError:
-                d[name] = val
-    return [out[k] for k in sorted(out)]
+                pass
+        out.append(d)
+    return out
 
 
 def main(ncu_log, oplist, base, out_csv):
