@@ -9,7 +9,7 @@ timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smok
 fi
 timeout 1200 python bench.py ${BENCH_ARGS} > gpurun_out/bench.log 2>&1; echo "rc=$?" >> gpurun_out/bench.log
 if [ -z "$SKIP_NCU" ]; then
-OURS='(gemm_kernel|gemv_bt_kernel|unary_kernel|binary_kernel|bn_|dw_|maxpool_kernel|avgpool|ce_kernel|mse_kernel|sgd_kernel|colsum_kernel)'
+OURS='(gemm_kernel|gemm_tc_kernel|gemm_atb_kernel|gemm_rows_kernel|gemv_bt_kernel|unary_kernel|binary_kernel|bn_|dw_|maxpool_kernel|avgpool|ce_kernel|mse_kernel|sgd_kernel|colsum_kernel)'
 M=gpu__time_duration.sum,sm__throughput.avg.pct_of_peak_sustained_elapsed,gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed,dram__bytes_read.sum,dram__bytes_write.sum,launch__grid_size
 for c in hp be; do
   timeout 1200 ncu --metrics $M --clock-control none --csv --page raw --kernel-name-base function -k "regex:$OURS" --log-file gpurun_out/ncu_${c}.csv python tools/profile/solo_runner.py --client $c > gpurun_out/ncu_${c}.out 2>&1
