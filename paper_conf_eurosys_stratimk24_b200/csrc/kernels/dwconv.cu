@@ -122,6 +122,68 @@ __global__ void __launch_bounds__(DW_THREADS) dw_dgrad_rows_s1_kernel(const floa
   orion_signal(sig);
 }
 
+// Stride-2 dgrad, row-blocked: for input row h only kernel rows r with (h+1-r) even contribute
+// (one row for even h, two for odd h), and along w the pair (w = 2j, 2j+1) reads dy columns j and
+// j+1 only: dx(2j) = sum_r dy(p_r, j) k(r,1); dx(2j+1) = sum_r dy(p_r, j+1) k(r,0) + dy(p_r, j) k(r,2).
+__global__ void __launch_bounds__(DW_THREADS) dw_dgrad_rows_s2_kernel(const float* __restrict__ dy, const float* __restrict__ w,
+                                                                      float* __restrict__ dx, DwShape s, OrionSig sig) {
+  const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
+  const int cblocks = (s.C + 31) / 32;
+  const long long nrows = (long long)s.N * s.H;
+  for (long long item = (long long)blockIdx.x * ROW_WARPS + warp; item < nrows * cblocks; item += (long long)gridDim.x * ROW_WARPS) {
+    const int cb = (int)(item % cblocks);
+    const long long row = item / cblocks;
+    const int h = (int)(row % s.H), n = (int)(row / s.H);
+    const int c = cb * 32 + lane;
+    if (c >= s.C) continue;
+    // up to two contributing kernel rows
+    int rr[2], pp[2], nr = 0;
+#pragma unroll
+    for (int r = 0; r < 3; r++) {
+      const int ph = h + 1 - r;
+      if (ph >= 0 && (ph & 1) == 0 && ph / 2 < s.P) { rr[nr] = r; pp[nr] = ph / 2; nr++; }
+    }
+    float k0[2], k1[2], k2[2];
+    const float* gr[2];
+#pragma unroll
+    for (int i = 0; i < 2; i++) {
+      const bool on = i < nr;
+      k0[i] = on ? __ldg(w + c * 9 + rr[i] * 3 + 0) : 0.f;
+      k1[i] = on ? __ldg(w + c * 9 + rr[i] * 3 + 1) : 0.f;
+      k2[i] = on ? __ldg(w + c * 9 + rr[i] * 3 + 2) : 0.f;
+      gr[i] = dy + (((long long)n * s.P + (on ? pp[i] : 0)) * s.Q) * s.C + c;
+    }
+    auto ld = [&](int i, int col) -> float {
+      return (i < nr && (unsigned)col < (unsigned)s.Q) ? __ldg(gr[i] + (long long)col * s.C) : 0.f;
+    };
+    float* dr = dx + (((long long)n * s.H + h) * s.W) * s.C + c;
+    const int npairs = (s.W + 1) / 2;
+    for (int j0 = 0; j0 < npairs; j0 += DW_U) {
+      float col[2][DW_U + 1];
+#pragma unroll
+      for (int i = 0; i < 2; i++)
+#pragma unroll
+        for (int u = 0; u <= DW_U; u++) col[i][u] = ld(i, j0 + u);
+#pragma unroll
+      for (int u = 0; u < DW_U; u++) {
+        const int we = 2 * (j0 + u);
+        if (we < s.W) {
+          float e = 0.f, o = 0.f;
+#pragma unroll
+          for (int i = 0; i < 2; i++) {
+            e = fmaf(col[i][u], k1[i], e);
+            o = fmaf(col[i][u + 1], k0[i], o);
+            o = fmaf(col[i][u], k2[i], o);
+          }
+          dr[(long long)we * s.C] = e;
+          if (we + 1 < s.W) dr[(long long)(we + 1) * s.C] = o;
+        }
+      }
+    }
+  }
+  orion_signal(sig);
+}
+
 // wgrad: a warp accumulates the 9 taps of its 32 channels over whole output rows (register window
 // blocks as above), fp32 per row and fp64 across rows; warps combine in smem in fixed order, CTAs
 // write per-split partials, the last CTA of the channel block sums them in split order.
@@ -291,12 +353,15 @@ int dw_dgrad_geom(const uint64_t* a, LaunchGeom* g) {
   if (!dw_ok(a)) return ORION_E_INVAL;
   DwShape s = dw_shape(a);
   if (s.stride == 1) rows_geom(g, (long long)s.N * s.H * ((s.C + 31) / 32), (const void*)dw_dgrad_rows_s1_kernel);
+  else if (s.stride == 2) rows_geom(g, (long long)s.N * s.H * ((s.C + 31) / 32), (const void*)dw_dgrad_rows_s2_kernel);
   else ew(g, (uint64_t)s.N * s.H * s.W * (s.C / 4), (const void*)dw_dgrad_kernel);
   return 0;
 }
 int dw_dgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   if (g.func == (const void*)dw_dgrad_rows_s1_kernel)
     dw_dgrad_rows_s1_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
+  else if (g.func == (const void*)dw_dgrad_rows_s2_kernel)
+    dw_dgrad_rows_s2_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
   else
     dw_dgrad_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
   CHECK_LAUNCH();
