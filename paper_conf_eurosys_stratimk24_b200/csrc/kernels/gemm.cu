@@ -771,7 +771,26 @@ __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float
   constexpr int MAXQ = (R * (MAXD / 4) * 2 + NTH - 1) / NTH;   // upper bound of quads per thread
   float4 ra[MAXQ];
   const int tot_a = R * qa, tot_b = R * qb, tot = tot_a + tot_b;
+  // Flat path: when both operands are dense with ld == width (the weight-gradient case), a 64-row
+  // block of each is one contiguous range, copied float4 by float4 with no index decomposition
+  // (rows past kend are zero-filled by comparing the flat offset with the valid length).
+  const bool flat = vecA && vecB && lda == M && ldb == N;
   auto gload = [&](int k0) {
+    if (flat) {
+      const int rows_ok = max(0, min(R, kend - k0));
+      const int lim_a = rows_ok * M / 4, lim_b = rows_ok * N / 4;
+      const float4* ga = reinterpret_cast<const float4*>(A + (long long)k0 * lda);
+      const float4* gb = reinterpret_cast<const float4*>(B + (long long)k0 * ldb);
+#pragma unroll
+      for (int j = 0; j < MAXQ; j++) {
+        const int idx = tid + j * NTH;
+        float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (idx < tot_a) { if (idx < lim_a) v = __ldg(ga + idx); }
+        else if (idx < tot) { if (idx - tot_a < lim_b) v = __ldg(gb + (idx - tot_a)); }
+        ra[j] = v;
+      }
+      return;
+    }
 #pragma unroll
     for (int j = 0; j < MAXQ; j++) {
       const int idx = tid + j * NTH;
@@ -798,6 +817,15 @@ __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float
     }
   };
   auto sstore = [&](int buf) {
+    if (flat) {   // smem rows unpadded (stride M / N) in flat mode
+#pragma unroll
+      for (int j = 0; j < MAXQ; j++) {
+        const int idx = tid + j * NTH;
+        if (idx < tot_a) reinterpret_cast<float4*>(As0 + (size_t)buf * R * Mp)[idx] = ra[j];
+        else if (idx < tot) reinterpret_cast<float4*>(Bs0 + (size_t)buf * R * Np)[idx - tot_a] = ra[j];
+      }
+      return;
+    }
 #pragma unroll
     for (int j = 0; j < MAXQ; j++) {
       const int idx = tid + j * NTH;
@@ -811,6 +839,8 @@ __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float
       }
     }
   };
+  // row stride of the staged blocks (flat mode stores rows unpadded)
+  const int sA = flat ? M : Mp, sB = flat ? N : Np;
   int buf = 0;
   if (kbeg < kend) { gload(kbeg); sstore(0); }
   __syncthreads();
@@ -819,8 +849,8 @@ __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float
     if (more) gload(k0 + R);
     if (active) {
       for (int r = grp; r < R; r += G) {
-        float4 a = *reinterpret_cast<const float4*>(As(buf, r, bm));
-        float4 b = *reinterpret_cast<const float4*>(Bs(buf, r, bn));
+        float4 a = *reinterpret_cast<const float4*>(As0 + ((size_t)buf * R * Mp) + (size_t)r * sA + bm);
+        float4 b = *reinterpret_cast<const float4*>(Bs0 + ((size_t)buf * R * Np) + (size_t)r * sB + bn);
         const float av[4] = {a.x, a.y, a.z, a.w}, bv[4] = {b.x, b.y, b.z, b.w};
 #pragma unroll
         for (int i = 0; i < 4; i++)
@@ -875,18 +905,19 @@ __global__ void __launch_bounds__(NTH) gemm_rows_kernel(const float* __restrict_
                                                        long long ldb, float* __restrict__ C, long long ldc,
                                                        const float* __restrict__ bias, int M, int N, int K, OrionSig sig) {
   extern __shared__ __align__(16) float rows_smem[];
-  float* Bs = rows_smem;                 // [K][N]
-  float* As = Bs + K * N;                // [KC][NTH + 1]
+  const int NP = (N + 3) & ~3, nq = NP / 4;      // B rows padded to whole float4
+  float* Bs = rows_smem;                          // [K][NP]
+  float* As = Bs + K * NP;                        // [KC][NTH + 1]
   const int tid = threadIdx.x;
-  for (int i = tid; i < K * N; i += NTH) {
-    const int k = i / N, n = i % N;
-    Bs[i] = BT ? __ldg(B + (long long)n * ldb + k) : __ldg(B + (long long)k * ldb + n);
+  for (int i = tid; i < K * NP; i += NTH) {
+    const int k = i / NP, n = i % NP;
+    Bs[i] = n < N ? (BT ? __ldg(B + (long long)n * ldb + k) : __ldg(B + (long long)k * ldb + n)) : 0.f;
   }
   const long long r0 = (long long)blockIdx.x * NTH;
   const int rows_here = (int)min((long long)NTH, (long long)M - r0);
-  float acc[MAXN];
+  float4 acc[MAXN / 4];
 #pragma unroll
-  for (int n = 0; n < MAXN; n++) acc[n] = 0.f;
+  for (int j = 0; j < MAXN / 4; j++) acc[j] = make_float4(0.f, 0.f, 0.f, 0.f);
   const bool vec = (lda % 4 == 0) && ((reinterpret_cast<uintptr_t>(A) & 15) == 0);
   for (int k0 = 0; k0 < K; k0 += KC) {
     const int kc = min(KC, K - k0);
@@ -909,22 +940,40 @@ __global__ void __launch_bounds__(NTH) gemm_rows_kernel(const float* __restrict_
     if (tid < rows_here) {
       for (int kk = 0; kk < kc; kk++) {
         const float a = As[kk * (NTH + 1) + tid];
-        const float* b = Bs + (k0 + kk) * N;
+        const float4* b = reinterpret_cast<const float4*>(Bs + (k0 + kk) * NP);
 #pragma unroll
-        for (int n = 0; n < MAXN; n++)
-          if (n < N) acc[n] = fmaf(a, b[n], acc[n]);
+        for (int j = 0; j < MAXN / 4; j++) {
+          if (j < nq) {
+            const float4 bv = b[j];
+            acc[j].x = fmaf(a, bv.x, acc[j].x); acc[j].y = fmaf(a, bv.y, acc[j].y);
+            acc[j].z = fmaf(a, bv.z, acc[j].z); acc[j].w = fmaf(a, bv.w, acc[j].w);
+          }
+        }
       }
     }
   }
   if (tid < rows_here) {
     float* c = C + (r0 + tid) * ldc;
+    const bool vc = (N % 4 == 0) && (ldc % 4 == 0) && ((reinterpret_cast<uintptr_t>(C) & 15) == 0) && bias == nullptr;
 #pragma unroll
-    for (int n = 0; n < MAXN; n++)
-      if (n < N) c[n] = acc[n] + (bias ? __ldg(bias + n) : 0.f);
+    for (int j = 0; j < MAXN / 4; j++) {
+      if (j < nq) {
+        if (vc) {
+          reinterpret_cast<float4*>(c)[j] = acc[j];
+        } else {
+          const float v[4] = {acc[j].x, acc[j].y, acc[j].z, acc[j].w};
+#pragma unroll
+          for (int e = 0; e < 4; e++) {
+            const int n = 4 * j + e;
+            if (n < N) c[n] = v[e] + (bias ? __ldg(bias + n) : 0.f);
+          }
+        }
+      }
+    }
   }
   orion_signal(sig);
 }
-inline int smem_bytes(int K, int N) { return (K * N + KC * (NTH + 1)) * 4; }
+inline int smem_bytes(int K, int N) { return (K * ((N + 3) & ~3) + KC * (NTH + 1)) * 4; }
 }  // namespace rows
 
 // ---------------------------------------------------------------- small-M GEMM (GEMV-like)
@@ -1135,14 +1184,14 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     g->grid = dim3((unsigned)cdiv(N, 8)); g->block = dim3(256); g->smem = 0; g->func = (const void*)gemv_bt_kernel;
     return 0;
   }
-  if ((flags == 0 || flags == 2) && M >= 4096 && N <= rows::MAXN && K * N <= rows::MAXKN) {
+  if ((flags == 0 || flags == 2) && M >= 4096 && N <= rows::MAXN && K * ((N + 3) & ~3) <= rows::MAXKN) {
     const void* f = flags == 2 ? (const void*)rows::gemm_rows_kernel<true> : (const void*)rows::gemm_rows_kernel<false>;
     static std::atomic<int> attr{0};
     if (!attr.load()) {
       if (cudaFuncSetAttribute((const void*)rows::gemm_rows_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               rows::smem_bytes(rows::MAXKN, 1)) != cudaSuccess ||
+                               rows::smem_bytes(rows::MAXKN, 4)) != cudaSuccess ||
           cudaFuncSetAttribute((const void*)rows::gemm_rows_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               rows::smem_bytes(rows::MAXKN, 1)) != cudaSuccess)
+                               rows::smem_bytes(rows::MAXKN, 4)) != cudaSuccess)
         return ORION_E_CUDA;
       attr.store(1);
     }
