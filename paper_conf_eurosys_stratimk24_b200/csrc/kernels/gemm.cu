@@ -1189,9 +1189,9 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     static std::atomic<int> attr{0};
     if (!attr.load()) {
       if (cudaFuncSetAttribute((const void*)rows::gemm_rows_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               rows::smem_bytes(rows::MAXKN, 4)) != cudaSuccess ||
+                               (rows::MAXKN + rows::KC * (rows::NTH + 1)) * 4) != cudaSuccess ||
           cudaFuncSetAttribute((const void*)rows::gemm_rows_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               rows::smem_bytes(rows::MAXKN, 4)) != cudaSuccess)
+                               (rows::MAXKN + rows::KC * (rows::NTH + 1)) * 4) != cudaSuccess)
         return ORION_E_CUDA;
       attr.store(1);
     }
