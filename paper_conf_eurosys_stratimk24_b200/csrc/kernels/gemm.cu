@@ -276,57 +276,79 @@ struct BWgrad {
 };
 
 // ---------------------------------------------------------------- ordered split-K reduction
-// Run by every thread of the last CTA of a tile: C[m0:m0+bm, n0:n0+bn] = sum_{z < split} ws[z] (+bias),
-// summed in split order (((p0 + p1) + p2) + ...), so the result depends only on the shape.
-// Elements are spread over the CTA's threads with consecutive threads on consecutive columns
-// (coalesced), 4 columns (128 bits) per thread when possible and 4 splits in flight.
-__device__ void split_reduce_tile(const GemmParams& p, int m0, int n0, int bm, int bn) {
-  const long long stride = (long long)p.M * p.N;
-  const int rows = min(bm, p.M - m0), cols = min(bn, p.N - n0);
-  const bool vec = (cols % 4 == 0) && (p.N % 4 == 0) && (n0 % 4 == 0) && (p.ldc % 4 == 0) &&
-                   ((reinterpret_cast<uintptr_t>(p.ws) & 15) == 0) && ((reinterpret_cast<uintptr_t>(p.C) & 15) == 0);
+// dst[m0:m0+bm, n0:n0+bn] = sum_{z < count} src[z] (+ bias), summed in z order (((s0 + s1) + s2) + ...)
+// by every thread of the calling CTA: consecutive threads on consecutive columns (coalesced),
+// 128-bit where possible, 4 partials in flight.
+__device__ void reduce_range(const float* src, long long zstride, int count, float* dst, long long ldd, const float* bias,
+                             int M, int N, int m0, int n0, int bm, int bn) {
+  const int rows = min(bm, M - m0), cols = min(bn, N - n0);
+  const bool vec = (cols % 4 == 0) && (N % 4 == 0) && (n0 % 4 == 0) && (ldd % 4 == 0) &&
+                   ((reinterpret_cast<uintptr_t>(src) & 15) == 0) && ((reinterpret_cast<uintptr_t>(dst) & 15) == 0) &&
+                   (zstride % 4 == 0);
   if (vec) {
     const int cq = cols / 4, total = rows * cq;
     for (int e = threadIdx.x; e < total; e += blockDim.x) {
       const int r = e / cq, c = (e % cq) * 4;
-      const float* q = p.ws + (long long)(m0 + r) * p.N + n0 + c;
+      const float* q = src + (long long)(m0 + r) * N + n0 + c;
       float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
       int z = 0;
-      for (; z + 3 < p.split; z += 4) {
-        float4 v0 = __ldcg(reinterpret_cast<const float4*>(q + z * stride));
-        float4 v1 = __ldcg(reinterpret_cast<const float4*>(q + (z + 1) * stride));
-        float4 v2 = __ldcg(reinterpret_cast<const float4*>(q + (z + 2) * stride));
-        float4 v3 = __ldcg(reinterpret_cast<const float4*>(q + (z + 3) * stride));
+      for (; z + 3 < count; z += 4) {
+        float4 v0 = __ldcg(reinterpret_cast<const float4*>(q + z * zstride));
+        float4 v1 = __ldcg(reinterpret_cast<const float4*>(q + (z + 1) * zstride));
+        float4 v2 = __ldcg(reinterpret_cast<const float4*>(q + (z + 2) * zstride));
+        float4 v3 = __ldcg(reinterpret_cast<const float4*>(q + (z + 3) * zstride));
         acc.x += v0.x; acc.x += v1.x; acc.x += v2.x; acc.x += v3.x;
         acc.y += v0.y; acc.y += v1.y; acc.y += v2.y; acc.y += v3.y;
         acc.z += v0.z; acc.z += v1.z; acc.z += v2.z; acc.z += v3.z;
         acc.w += v0.w; acc.w += v1.w; acc.w += v2.w; acc.w += v3.w;
       }
-      for (; z < p.split; z++) {
-        float4 v = __ldcg(reinterpret_cast<const float4*>(q + z * stride));
+      for (; z < count; z++) {
+        float4 v = __ldcg(reinterpret_cast<const float4*>(q + z * zstride));
         acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
       }
       const int n = n0 + c;
-      if (p.bias) {
-        acc.x += __ldg(p.bias + n); acc.y += __ldg(p.bias + n + 1); acc.z += __ldg(p.bias + n + 2); acc.w += __ldg(p.bias + n + 3);
+      if (bias) {
+        acc.x += __ldg(bias + n); acc.y += __ldg(bias + n + 1); acc.z += __ldg(bias + n + 2); acc.w += __ldg(bias + n + 3);
       }
-      *reinterpret_cast<float4*>(p.C + (long long)(m0 + r) * p.ldc + n) = acc;
+      *reinterpret_cast<float4*>(dst + (long long)(m0 + r) * ldd + n) = acc;
     }
   } else {
     const int total = rows * cols;
     for (int e = threadIdx.x; e < total; e += blockDim.x) {
       const int r = e / cols, c = e % cols;
-      const float* q = p.ws + (long long)(m0 + r) * p.N + n0 + c;
+      const float* q = src + (long long)(m0 + r) * N + n0 + c;
       float acc = 0.f;
       int z = 0;
-      for (; z + 3 < p.split; z += 4) {
-        float v0 = __ldcg(q + z * stride), v1 = __ldcg(q + (z + 1) * stride);
-        float v2 = __ldcg(q + (z + 2) * stride), v3 = __ldcg(q + (z + 3) * stride);
+      for (; z + 3 < count; z += 4) {
+        float v0 = __ldcg(q + z * zstride), v1 = __ldcg(q + (z + 1) * zstride);
+        float v2 = __ldcg(q + (z + 2) * zstride), v3 = __ldcg(q + (z + 3) * zstride);
         acc += v0; acc += v1; acc += v2; acc += v3;
       }
-      for (; z < p.split; z++) acc += __ldcg(q + z * stride);
-      p.C[(long long)(m0 + r) * p.ldc + n0 + c] = acc + (p.bias ? __ldg(p.bias + n0 + c) : 0.f);
+      for (; z < count; z++) acc += __ldcg(q + z * zstride);
+      dst[(long long)(m0 + r) * ldd + n0 + c] = acc + (bias ? __ldg(bias + n0 + c) : 0.f);
     }
+  }
+}
+
+// Finish a split-K tile after this CTA wrote its partial p.ws[blockIdx.z]. Up to 32 splits: the
+// last CTA of the tile sums all partials in order. More: a fixed two-level tree — the last CTA of
+// each group of 16 consecutive splits sums the group into a group partial (after the split
+// partials in the workspace), and the last group to finish sums the group partials in order.
+constexpr int SPLIT_GROUP = 16, SPLIT_FLAT_MAX = 32, TICKETS_PER_TILE = 64;
+__device__ void split_finish(const GemmParams& p, int tile, int m0, int n0, int bm, int bn) {
+  const long long MN = (long long)p.M * p.N;
+  if (p.split <= SPLIT_FLAT_MAX) {
+    if (last_cta_of(p.tickets + tile, p.split)) reduce_range(p.ws, MN, p.split, p.C, p.ldc, p.bias, p.M, p.N, m0, n0, bm, bn);
+    return;
+  }
+  const int ng = (p.split + SPLIT_GROUP - 1) / SPLIT_GROUP;
+  const int g = blockIdx.z / SPLIT_GROUP;
+  const int gsize = min(SPLIT_GROUP, p.split - g * SPLIT_GROUP);
+  unsigned int* tb = p.tickets + (long long)tile * TICKETS_PER_TILE;
+  float* gws = p.ws + (long long)p.split * MN;
+  if (last_cta_of(tb + 1 + g, gsize)) {
+    reduce_range(p.ws + (long long)g * SPLIT_GROUP * MN, MN, gsize, gws + (long long)g * MN, p.N, nullptr, p.M, p.N, m0, n0, bm, bn);
+    if (last_cta_of(tb, ng)) reduce_range(gws, MN, ng, p.C, p.ldc, p.bias, p.M, p.N, m0, n0, bm, bn);
   }
 }
 
@@ -441,8 +463,7 @@ __global__ void __launch_bounds__(NT) gemm_kernel(GemmParams p, LA la, LB lb, Or
         if (n < p.N) part[(long long)m * p.N + n] = acc[i][j];
       }
     }
-    unsigned int* tk = p.tickets + blockIdx.y * gridDim.x + blockIdx.x;
-    if (last_cta_of(tk, p.split)) split_reduce_tile(p, m0, n0, BM, BN);
+    split_finish(p, blockIdx.y * gridDim.x + blockIdx.x, m0, n0, BM, BN);
   }
   orion_signal(sig);
 }
@@ -712,8 +733,7 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   if (p.split > 1) {
-    unsigned int* tk = p.tickets + blockIdx.y * gridDim.x + blockIdx.x;
-    if (last_cta_of(tk, p.split)) split_reduce_tile(p, m0, n0, BM, BN);
+    split_finish(p, blockIdx.y * gridDim.x + blockIdx.x, m0, n0, BM, BN);
   } else {
     __syncthreads();
   }
@@ -732,7 +752,7 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
 // 128-bit loads (the next block's loads in flight while the current one is multiplied), keeps both
 // blocks in shared memory and gives each thread a 4x4 register block of C over a fixed subset of
 // the rows (row groups combined in fixed order). K is split over CTAs (shape-only count) and the
-// splits are summed in order by the last CTA (split_reduce_tile).
+// splits are summed in order (split_finish).
 namespace atb {
 constexpr int R = 64, NTH = 256, MAXD = 128;
 
@@ -884,9 +904,7 @@ __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float
       else out[(long long)m * N + n] = v;
     }
   }
-  if (p.split > 1) {
-    if (last_cta_of(p.tickets, p.split)) split_reduce_tile(p, 0, 0, M, N);
-  }
+  if (p.split > 1) split_finish(p, 0, 0, 0, M, N);
   orion_signal(sig);
 }
 }  // namespace atb
@@ -1080,7 +1098,7 @@ Plan plan_gemm(long long M, long long N, long long K) {
     split = cdiv(target, tiles);
     long long kmax = K / (4 * pl.bk);         // >= 4 k-tiles per split
     if (split > kmax) split = kmax;
-    if (split > 1024) split = 1024;
+    if (split > 1008) split = 1008;                 // two-level reduction: <= 63 groups of 16
     if (split < 1) split = 1;
   }
   pl.split = (int)split;
@@ -1088,7 +1106,10 @@ Plan plan_gemm(long long M, long long N, long long K) {
 }
 
 uint64_t ws_bytes_for(const Plan& pl, long long M, long long N) {
-  return pl.split > 1 ? WS_TICKET_BYTES + (uint64_t)pl.split * M * N * 4 : 0;
+  if (pl.split <= 1) return 0;
+  uint64_t parts = (uint64_t)pl.split;
+  if (pl.split > SPLIT_FLAT_MAX) parts += (uint64_t)((pl.split + SPLIT_GROUP - 1) / SPLIT_GROUP);   // group partials
+  return WS_TICKET_BYTES + parts * M * N * 4;
 }
 
 template <class LA, class LB>
