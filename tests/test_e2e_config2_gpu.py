@@ -81,7 +81,9 @@ def test_be_one_iteration_vs_oracle(cfg2):
         # block outputs have exactly-zero per-channel batch mean (every path ends in a BN), so the
         # running means of the BNs fed by them (expand_bn, features.18.bn) are ~1e-9 noise: floor
         floor = 1e-2 if name.endswith(".rmean") else 1e-30
-        assert rel(G.p[name], newP[name], floor) < 1e-5, name
+        # BN betas start at 0: after one step the value is -lr * grad, i.e. a gradient check
+        tol = 3e-4 if name.endswith(".beta") else 1e-5
+        assert rel(G.p[name], newP[name], floor) < tol, name
     # first step: v = mu*0 + g = g exactly (torch's v <- g), so the momentum buffer equals the grads
     assert torch.equal(G.vflat, G.gflat)
 
