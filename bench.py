@@ -238,8 +238,12 @@ def main():
     rate = args.rate or W_["rate"]
     hpg, beg = W_["hpg"], W_["beg"]
     # ---- offline profile: solo op durations, sm_needed, class
-    prof_hp, rows_hp = PR.build_profiles(hpg, 0, reps=5)
-    prof_be, rows_be = PR.build_profiles(beg, 10000, reps=5)
+    # offline profile: event-timed durations, occupancy sm_needed, class from the committed per-op
+    # ncu counters (profiles/<config>_<client>_ncu.csv, R16) or the analytic roofline without one
+    ncu_hp = os.path.join(ROOT, "profiles", f"{args.config}_hp_ncu.csv")
+    ncu_be = os.path.join(ROOT, "profiles", f"{args.config}_be_ncu.csv")
+    prof_hp, rows_hp = PR.build_profiles(hpg, 0, reps=5, ncu_csv=ncu_hp)
+    prof_be, rows_be = PR.build_profiles(beg, 10000, reps=5, ncu_csv=ncu_be)
     beg.params.reset()
     hp = C.HPClient(hpg, W_["hp_inputs"], max(args.steps, 64), prof_hp, 0)
     be = C.BEClient(beg, prof_be, 10000)

@@ -112,13 +112,15 @@ def time_ops(graph, reps=10, warmup=2, stream=None):
 
 
 def load_ncu_csv(path):
-    """{kernel_id: (c_pct, m_pct, dram_bytes)} from tools/profile/ncu_profile.py's summary CSV."""
+    """{kernel_id: (c_pct, m_pct, dram_bytes, dur_ns)} from tools/profile/ncu_summarize.py's CSV
+    (one solo launch per op under ncu: sm__throughput, gpu__compute_memory_throughput, DRAM bytes,
+    gpu__time_duration)."""
     if not path or not os.path.exists(path):
         return {}
     rows = {}
     with open(path) as f:
         for r in csv.DictReader(f):
-            rows[int(r["kernel_id"])] = (float(r["sm_pct"]), float(r["mem_pct"]), float(r["dram_bytes"]))
+            rows[int(r["kernel_id"])] = (float(r["sm_pct"]), float(r["mem_pct"]), float(r["dram_bytes"]), float(r["dur_ns"]))
     return rows
 
 
@@ -130,17 +132,18 @@ def build_profiles(graph, kid_base=0, reps=10, ncu_csv=None):
     for i, fn, args, lab in graph.kernel_ops():
         kid = kid_base + i
         flops, nbytes = op_work(fn, args)
+        dur = durs[i]
         if kid in ncu:
-            c, m, dram = ncu[kid]
+            c, m, dram, ndur = ncu[kid]
             cls = classify(c, m, flops, dram)
+            dur = int(ndur) if ndur > 0 else dur   # device time of the kernel alone
             src = "ncu"
         else:
-            c = m = None
             cls = classify(None, None, flops, nbytes)
             src = "analytic"
         sm = sm_needed(fn, args)
-        table[kid] = (cls, sm, durs[i])
-        rows.append(dict(kernel_id=kid, label=lab, fn=fn, cls="UCM"[cls], sm_needed=sm, dur_ns=durs[i],
+        table[kid] = (cls, sm, dur)
+        rows.append(dict(kernel_id=kid, label=lab, fn=fn, cls="UCM"[cls], sm_needed=sm, dur_ns=dur,
                          flops=flops, bytes=nbytes, source=src))
     return table, rows
 
