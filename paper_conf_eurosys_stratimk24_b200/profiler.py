@@ -135,7 +135,10 @@ def build_profiles(graph, kid_base=0, reps=10, ncu_csv=None):
         dur = durs[i]
         if kid in ncu:
             c, m, dram, ndur = ncu[kid]
-            cls = classify(c, m, flops, dram)
+            # arithmetic intensity over max(measured DRAM bytes, compulsory bytes): on B200 the 126 MB
+            # L2 often holds an op's inputs, and DRAM bytes alone would call a memory-bound op
+            # compute-bound (DESIGN.md §3 R16)
+            cls = classify(c, m, flops, max(dram, nbytes))
             dur = int(ndur) if ndur > 0 else dur   # device time of the kernel alone
             src = "ncu"
         else:
