@@ -754,46 +754,55 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
 // the rows (row groups combined in fixed order). K is split over CTAs (shape-only count) and the
 // splits are summed in order (split_finish).
 namespace atb {
-constexpr int R = 64, NTH = 256, MAXD = 128;
+constexpr int NTH = 256;
 
-__host__ __device__ inline int pad_dim(int d) { return ((d + 3) / 4) * 4 + 4; }
-__host__ __device__ inline int smem_bytes(int M, int N) { return (2 * R * (pad_dim(M) + pad_dim(N)) + NTH * 16) * 4; }
+// Variant <TMB, TNB, R, MAXM, MAXN>: each thread owns a TMB x TNB register block of C; R rows of
+// both operands are staged per step. MAXQ = float4s each thread stages per step.
+template <int TMB, int TNB, int R, int MAXM, int MAXN>
+struct V {
+  static constexpr int MAXQ = (R * ((MAXM + MAXN) / 4) + NTH - 1) / NTH;
+  __host__ __device__ static int pad_dim(int d) { return ((d + 3) / 4) * 4 + 4; }
+  __host__ __device__ static int smem_bytes(int M, int N) { return (2 * R * (pad_dim(M) + pad_dim(N)) + NTH * TMB * TNB) * 4; }
+  __host__ __device__ static bool fits(long long M, long long N) {
+    return M <= MAXM && N <= MAXN && ((M + TMB - 1) / TMB) * ((N + TNB - 1) / TNB) <= NTH;
+  }
+};
+using V44 = V<4, 4, 64, 128, 128>;
+using V84 = V<8, 4, 32, 192, 64>;
+using V48 = V<4, 8, 32, 64, 192>;
 
+template <class VV, int TMB, int TNB, int R>
 __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float* __restrict__ A, long long lda,
                                                       const float* __restrict__ B, long long ldb, OrionSig sig) {
   extern __shared__ __align__(16) float atb_smem[];
+  constexpr int MAXQ = VV::MAXQ;
   const int tid = threadIdx.x;
   const int M = p.M, N = p.N;
-  const int Mp = pad_dim(M), Np = pad_dim(N);
+  const int Mp = VV::pad_dim(M), Np = VV::pad_dim(N);
   float* As0 = atb_smem;                  // [2][R][Mp]
   float* Bs0 = As0 + 2 * R * Mp;          // [2][R][Np]
-  float* red = Bs0 + 2 * R * Np;          // [NTH * 16]
-  auto As = [&](int b, int r, int c) -> float* { return As0 + ((size_t)b * R + r) * Mp + c; };
-  auto Bs = [&](int b, int r, int c) -> float* { return Bs0 + ((size_t)b * R + r) * Np + c; };
-  const int mb = (M + 3) / 4, nb = (N + 3) / 4;      // 4x4 output blocks
+  float* red = Bs0 + 2 * R * Np;          // [NTH * TMB * TNB]
+  const int mb = (M + TMB - 1) / TMB, nb = (N + TNB - 1) / TNB;
   const int nblk = mb * nb;
-  const int G = NTH / nblk;                            // row groups (>= 1 since M, N <= 128 -> nblk <= 1024? see host)
+  const int G = NTH / nblk;                            // row groups
   const int grp = tid / nblk, blk = tid % nblk;
-  const int bm = (blk / nb) * 4, bn = (blk % nb) * 4;
+  const int bm = (blk / nb) * TMB, bn = (blk % nb) * TNB;
   const bool active = grp < G;
   const int kbeg = blockIdx.z * p.kps;
   const int kend = min(p.K, kbeg + p.kps);
   const bool vecA = (lda % 4 == 0) && (M % 4 == 0) && ((reinterpret_cast<uintptr_t>(A) & 15) == 0);
   const bool vecB = (ldb % 4 == 0) && (N % 4 == 0) && ((reinterpret_cast<uintptr_t>(B) & 15) == 0);
-  const int qa = (M + 3) / 4, qb = (N + 3) / 4;       // float4 per row
-  float acc[4][4];
+  const int qa = (M + 3) / 4, qb = (N + 3) / 4;
+  float acc[TMB][TNB];
 #pragma unroll
-  for (int i = 0; i < 4; i++)
+  for (int i = 0; i < TMB; i++)
 #pragma unroll
-    for (int j = 0; j < 4; j++) acc[i][j] = 0.f;
+    for (int j = 0; j < TNB; j++) acc[i][j] = 0.f;
 
-  // staging: each thread moves quads (row, q) = idx -> (idx / q*, idx % q*) of the 64-row block
-  constexpr int MAXQ = (R * (MAXD / 4) * 2 + NTH - 1) / NTH;   // upper bound of quads per thread
   float4 ra[MAXQ];
   const int tot_a = R * qa, tot_b = R * qb, tot = tot_a + tot_b;
-  // Flat path: when both operands are dense with ld == width (the weight-gradient case), a 64-row
-  // block of each is one contiguous range, copied float4 by float4 with no index decomposition
-  // (rows past kend are zero-filled by comparing the flat offset with the valid length).
+  // Flat path: dense operands with ld == width (the weight-gradient case): an R-row block of each is
+  // one contiguous range, copied float4 by float4 (rows past kend zero-filled by offset compare).
   const bool flat = vecA && vecB && lda == M && ldb == N;
   auto gload = [&](int k0) {
     if (flat) {
@@ -836,31 +845,26 @@ __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float
       ra[j] = v;
     }
   };
+  const int sA = flat ? M : Mp, sB = flat ? N : Np;   // staged row strides
   auto sstore = [&](int buf) {
-    if (flat) {   // smem rows unpadded (stride M / N) in flat mode
-#pragma unroll
-      for (int j = 0; j < MAXQ; j++) {
-        const int idx = tid + j * NTH;
-        if (idx < tot_a) reinterpret_cast<float4*>(As0 + (size_t)buf * R * Mp)[idx] = ra[j];
-        else if (idx < tot) reinterpret_cast<float4*>(Bs0 + (size_t)buf * R * Np)[idx - tot_a] = ra[j];
-      }
-      return;
-    }
 #pragma unroll
     for (int j = 0; j < MAXQ; j++) {
       const int idx = tid + j * NTH;
       if (idx < tot) {
         const bool isA = idx < tot_a;
         const int li = isA ? idx : idx - tot_a;
-        const int q = isA ? qa : qb;
-        const int r = li / q, c = (li % q) * 4;
-        float* dst = isA ? As(buf, r, c) : Bs(buf, r, c);
-        *reinterpret_cast<float4*>(dst) = ra[j];
+        if (flat) {
+          if (isA) reinterpret_cast<float4*>(As0 + (size_t)buf * R * Mp)[li] = ra[j];
+          else reinterpret_cast<float4*>(Bs0 + (size_t)buf * R * Np)[li] = ra[j];
+        } else {
+          const int q = isA ? qa : qb;
+          const int r = li / q, c = (li % q) * 4;
+          float* dst = isA ? As0 + ((size_t)buf * R + r) * Mp + c : Bs0 + ((size_t)buf * R + r) * Np + c;
+          *reinterpret_cast<float4*>(dst) = ra[j];
+        }
       }
     }
   };
-  // row stride of the staged blocks (flat mode stores rows unpadded)
-  const int sA = flat ? M : Mp, sB = flat ? N : Np;
   int buf = 0;
   if (kbeg < kend) { gload(kbeg); sstore(0); }
   __syncthreads();
@@ -868,14 +872,24 @@ __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float
     const bool more = k0 + R < kend;
     if (more) gload(k0 + R);
     if (active) {
+      const float* ab = As0 + (size_t)buf * R * Mp + bm;
+      const float* bb = Bs0 + (size_t)buf * R * Np + bn;
       for (int r = grp; r < R; r += G) {
-        float4 a = *reinterpret_cast<const float4*>(As0 + ((size_t)buf * R * Mp) + (size_t)r * sA + bm);
-        float4 b = *reinterpret_cast<const float4*>(Bs0 + ((size_t)buf * R * Np) + (size_t)r * sB + bn);
-        const float av[4] = {a.x, a.y, a.z, a.w}, bv[4] = {b.x, b.y, b.z, b.w};
+        float av[TMB], bv[TNB];
 #pragma unroll
-        for (int i = 0; i < 4; i++)
+        for (int i = 0; i < TMB; i += 4) {
+          const float4 a = *reinterpret_cast<const float4*>(ab + (size_t)r * sA + i);
+          av[i] = a.x; av[i + 1] = a.y; av[i + 2] = a.z; av[i + 3] = a.w;
+        }
 #pragma unroll
-          for (int j = 0; j < 4; j++) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+        for (int j = 0; j < TNB; j += 4) {
+          const float4 b = *reinterpret_cast<const float4*>(bb + (size_t)r * sB + j);
+          bv[j] = b.x; bv[j + 1] = b.y; bv[j + 2] = b.z; bv[j + 3] = b.w;
+        }
+#pragma unroll
+        for (int i = 0; i < TMB; i++)
+#pragma unroll
+          for (int j = 0; j < TNB; j++) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
       }
     }
     if (more) {
@@ -886,19 +900,20 @@ __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float
     }
   }
   // combine row groups in fixed order
+  constexpr int BLK = TMB * TNB;
   if (active) {
 #pragma unroll
-    for (int i = 0; i < 4; i++)
+    for (int i = 0; i < TMB; i++)
 #pragma unroll
-      for (int j = 0; j < 4; j++) red[(grp * nblk + blk) * 16 + i * 4 + j] = acc[i][j];
+      for (int j = 0; j < TNB; j++) red[(grp * nblk + blk) * BLK + i * TNB + j] = acc[i][j];
   }
   __syncthreads();
   float* out = p.split == 1 ? nullptr : p.ws + (long long)blockIdx.z * M * N;
-  for (int e = tid; e < nblk * 16; e += NTH) {
-    const int b = e / 16, ij = e % 16, i = ij / 4, j = ij % 4;
-    const int m = (b / nb) * 4 + i, n = (b % nb) * 4 + j;
+  for (int e = tid; e < nblk * BLK; e += NTH) {
+    const int b = e / BLK, ij = e % BLK, i = ij / TNB, j = ij % TNB;
+    const int m = (b / nb) * TMB + i, n = (b % nb) * TNB + j;
     float v = 0.f;
-    for (int g = 0; g < G; g++) v += red[(g * nblk + b) * 16 + ij];
+    for (int g = 0; g < G; g++) v += red[(g * nblk + b) * BLK + ij];
     if (m < M && n < N) {
       if (p.split == 1) p.C[(long long)m * p.ldc + n] = v + (p.bias ? __ldg(p.bias + n) : 0.f);
       else out[(long long)m * N + n] = v;
@@ -1052,16 +1067,22 @@ __global__ void __launch_bounds__(256) gemv_bt_kernel(const float* __restrict__ 
 struct Plan { int cfg; int split; int bm, bn, bk; };
 // cfg: 0/1/2 = FFMA tiles L/M/S; 3/4 = tcgen05 3xTF32 with BN = 128 / 64.
 
-// Skinny A^T B (cfg 5): both dims <= 128 with at most 256 4x4 output blocks, long K.
-bool atb_ok(long long M, long long N, long long K) {
-  return M <= 128 && N <= 128 && cdiv(M, 4) * cdiv(N, 4) <= 256 && K >= 4096;
+// Skinny A^T B (cfg 5/6/7 = variants V44/V84/V48): the whole M x N fits one CTA's register
+// blocks (<= 256 of them), long K.
+int atb_variant(long long M, long long N, long long K) {
+  if (K < 4096) return -1;
+  if (atb::V44::fits(M, N)) return 5;
+  if (atb::V84::fits(M, N)) return 6;
+  if (atb::V48::fits(M, N)) return 7;
+  return -1;
 }
+bool atb_ok(long long M, long long N, long long K) { return atb_variant(M, N, K) >= 0; }
 
 Plan plan_atb(long long M, long long N, long long K) {
   Plan pl;
-  pl.cfg = 5; pl.bm = (int)M; pl.bn = (int)N; pl.bk = atb::R;
+  pl.cfg = atb_variant(M, N, K); pl.bm = (int)M; pl.bn = (int)N; pl.bk = pl.cfg == 5 ? 64 : 32;
   long long split = cdiv(148 * 4, 1);
-  long long kmax = K / (4 * atb::R);
+  long long kmax = K / (4 * pl.bk);
   if (split > kmax) split = kmax;
   if (split < 1) split = 1;
   pl.split = (int)split;
@@ -1224,12 +1245,19 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     if (pl.split > 1 && (a[11] == 0 || a[12] < ws_bytes_for(pl, M, N))) pl.split = 1;
     static std::atomic<int> attr{0};
     if (!attr.load()) {
-      if (cudaFuncSetAttribute((const void*)atb::gemm_atb_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               atb::smem_bytes(128, 128)) != cudaSuccess) return ORION_E_CUDA;
+      if (cudaFuncSetAttribute((const void*)atb::gemm_atb_kernel<atb::V44, 4, 4, 64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               atb::V44::smem_bytes(128, 128)) != cudaSuccess ||
+          cudaFuncSetAttribute((const void*)atb::gemm_atb_kernel<atb::V84, 8, 4, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               atb::V84::smem_bytes(192, 64)) != cudaSuccess ||
+          cudaFuncSetAttribute((const void*)atb::gemm_atb_kernel<atb::V48, 4, 8, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               atb::V48::smem_bytes(64, 192)) != cudaSuccess)
+        return ORION_E_CUDA;
       attr.store(1);
     }
-    g->grid = dim3(1, 1, (unsigned)pl.split); g->block = dim3(atb::NTH); g->smem = atb::smem_bytes((int)M, (int)N);
-    g->func = (const void*)atb::gemm_atb_kernel;
+    g->grid = dim3(1, 1, (unsigned)pl.split); g->block = dim3(atb::NTH);
+    if (pl.cfg == 5) { g->smem = atb::V44::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V44, 4, 4, 64>; }
+    else if (pl.cfg == 6) { g->smem = atb::V84::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V84, 8, 4, 32>; }
+    else { g->smem = atb::V48::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V48, 4, 8, 32>; }
     return 0;
   }
   switch (flags) {
@@ -1261,8 +1289,16 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
       rows::gemm_rows_kernel<false><<<g.grid, g.block, g.smem, s>>>(A, lda, B, ldb, C, ldc, bias, (int)M, (int)N, (int)K, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
-  if (g.func == (const void*)atb::gemm_atb_kernel) {
-    atb::gemm_atb_kernel<<<g.grid, g.block, g.smem, s>>>(make_params(M, N, K, C, ldc, bias, (int)g.grid.z, ws, atb::R), A, lda, B, ldb, sig);
+  if (g.func == (const void*)atb::gemm_atb_kernel<atb::V44, 4, 4, 64>) {
+    atb::gemm_atb_kernel<atb::V44, 4, 4, 64><<<g.grid, g.block, g.smem, s>>>(make_params(M, N, K, C, ldc, bias, (int)g.grid.z, ws, 64), A, lda, B, ldb, sig);
+    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+  }
+  if (g.func == (const void*)atb::gemm_atb_kernel<atb::V84, 8, 4, 32>) {
+    atb::gemm_atb_kernel<atb::V84, 8, 4, 32><<<g.grid, g.block, g.smem, s>>>(make_params(M, N, K, C, ldc, bias, (int)g.grid.z, ws, 32), A, lda, B, ldb, sig);
+    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+  }
+  if (g.func == (const void*)atb::gemm_atb_kernel<atb::V48, 4, 8, 32>) {
+    atb::gemm_atb_kernel<atb::V48, 4, 8, 32><<<g.grid, g.block, g.smem, s>>>(make_params(M, N, K, C, ldc, bias, (int)g.grid.z, ws, 32), A, lda, B, ldb, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
   switch (flags) {

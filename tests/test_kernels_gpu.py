@@ -42,7 +42,8 @@ def ws(nbytes):
                                          (256, 256, 256, 0), (300, 200, 520, 1), (130, 70, 300, 2), (257, 129, 333, 3),
                                          (4704, 1280, 320, 2), (1280, 320, 4704, 1), (18816, 96, 576, 2),
                                          (99, 37, 9999, 1), (24, 144, 75264, 1), (128, 32, 300000, 1),
-                                         (12544, 16, 96, 0), (20000, 24, 144, 2), (5000, 7, 33, 0), (4097, 32, 512, 2)],
+                                         (12544, 16, 96, 0), (20000, 24, 144, 2), (5000, 7, 33, 0), (4097, 32, 512, 2),
+                                         (144, 24, 75264, 1), (192, 32, 75264, 1), (32, 192, 75264, 1), (150, 22, 5000, 1)],
                          ids=lambda v: str(v))
 def test_gemm_shapes(M, N, K, flags):
     test_gemm(M, N, K, flags)
