@@ -931,26 +931,34 @@ __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float
 // conflict-free), B lives in shared memory for the whole CTA (broadcast reads), and each thread
 // accumulates its row's N outputs in registers in k order (deterministic, no split).
 namespace rows {
-constexpr int NTH = 256, KC = 32, MAXN = 32, MAXKN = 16384;
+constexpr int NTH = 256, KC = 32, NCH = 32, MAXN = 128, MAXKN = 16384;
 
+// Threads are (row, chunk): each thread owns NCH = 32 consecutive outputs of one row; a CTA holds
+// RPC = 256 / nchunk rows (nchunk = ceil(N / 32) <= 4).
 template <bool BT>
 __global__ void __launch_bounds__(NTH) gemm_rows_kernel(const float* __restrict__ A, long long lda, const float* __restrict__ B,
                                                        long long ldb, float* __restrict__ C, long long ldc,
                                                        const float* __restrict__ bias, int M, int N, int K, OrionSig sig) {
   extern __shared__ __align__(16) float rows_smem[];
-  const int NP = (N + 3) & ~3, nq = NP / 4;      // B rows padded to whole float4
+  const int NP = (N + 3) & ~3;                    // B rows padded to whole float4
+  const int nchunk = (N + NCH - 1) / NCH;
+  const int RPC = NTH / nchunk;
   float* Bs = rows_smem;                          // [K][NP]
-  float* As = Bs + K * NP;                        // [KC][NTH + 1]
+  float* As = Bs + K * NP;                        // [KC][RPC + 1]
   const int tid = threadIdx.x;
+  const int row = tid % RPC, chunk = tid / RPC;
+  const bool thr_on = chunk < nchunk;
+  const int n0 = chunk * NCH;
+  const int nq = thr_on ? (min(NCH, NP - n0) + 3) / 4 : 0;   // float4 columns of this thread
   for (int i = tid; i < K * NP; i += NTH) {
     const int k = i / NP, n = i % NP;
     Bs[i] = n < N ? (BT ? __ldg(B + (long long)n * ldb + k) : __ldg(B + (long long)k * ldb + n)) : 0.f;
   }
-  const long long r0 = (long long)blockIdx.x * NTH;
-  const int rows_here = (int)min((long long)NTH, (long long)M - r0);
-  float4 acc[MAXN / 4];
+  const long long r0 = (long long)blockIdx.x * RPC;
+  const int rows_here = (int)min((long long)RPC, (long long)M - r0);
+  float4 acc[NCH / 4];
 #pragma unroll
-  for (int j = 0; j < MAXN / 4; j++) acc[j] = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int j = 0; j < NCH / 4; j++) acc[j] = make_float4(0.f, 0.f, 0.f, 0.f);
   const bool vec = (lda % 4 == 0) && ((reinterpret_cast<uintptr_t>(A) & 15) == 0);
   for (int k0 = 0; k0 < K; k0 += KC) {
     const int kc = min(KC, K - k0);
@@ -960,22 +968,22 @@ __global__ void __launch_bounds__(NTH) gemm_rows_kernel(const float* __restrict_
       for (int i = tid; i < rows_here * q; i += NTH) {
         const int r = i / q, c = (i % q) * 4;
         const float4 v = __ldg(reinterpret_cast<const float4*>(A + (r0 + r) * lda + k0 + c));
-        As[(c + 0) * (NTH + 1) + r] = v.x; As[(c + 1) * (NTH + 1) + r] = v.y;
-        As[(c + 2) * (NTH + 1) + r] = v.z; As[(c + 3) * (NTH + 1) + r] = v.w;
+        As[(c + 0) * (RPC + 1) + r] = v.x; As[(c + 1) * (RPC + 1) + r] = v.y;
+        As[(c + 2) * (RPC + 1) + r] = v.z; As[(c + 3) * (RPC + 1) + r] = v.w;
       }
     } else {
       for (int i = tid; i < rows_here * kc; i += NTH) {
         const int r = i / kc, c = i % kc;
-        As[c * (NTH + 1) + r] = __ldg(A + (r0 + r) * lda + k0 + c);
+        As[c * (RPC + 1) + r] = __ldg(A + (r0 + r) * lda + k0 + c);
       }
     }
     __syncthreads();
-    if (tid < rows_here) {
+    if (thr_on && row < rows_here) {
       for (int kk = 0; kk < kc; kk++) {
-        const float a = As[kk * (NTH + 1) + tid];
-        const float4* b = reinterpret_cast<const float4*>(Bs + (k0 + kk) * NP);
+        const float a = As[kk * (RPC + 1) + row];
+        const float4* b = reinterpret_cast<const float4*>(Bs + (k0 + kk) * NP + n0);
 #pragma unroll
-        for (int j = 0; j < MAXN / 4; j++) {
+        for (int j = 0; j < NCH / 4; j++) {
           if (j < nq) {
             const float4 bv = b[j];
             acc[j].x = fmaf(a, bv.x, acc[j].x); acc[j].y = fmaf(a, bv.y, acc[j].y);
@@ -985,11 +993,11 @@ __global__ void __launch_bounds__(NTH) gemm_rows_kernel(const float* __restrict_
       }
     }
   }
-  if (tid < rows_here) {
-    float* c = C + (r0 + tid) * ldc;
+  if (thr_on && row < rows_here) {
+    float* c = C + (r0 + row) * ldc + n0;
     const bool vc = (N % 4 == 0) && (ldc % 4 == 0) && ((reinterpret_cast<uintptr_t>(C) & 15) == 0) && bias == nullptr;
 #pragma unroll
-    for (int j = 0; j < MAXN / 4; j++) {
+    for (int j = 0; j < NCH / 4; j++) {
       if (j < nq) {
         if (vc) {
           reinterpret_cast<float4*>(c)[j] = acc[j];
@@ -997,8 +1005,8 @@ __global__ void __launch_bounds__(NTH) gemm_rows_kernel(const float* __restrict_
           const float v[4] = {acc[j].x, acc[j].y, acc[j].z, acc[j].w};
 #pragma unroll
           for (int e = 0; e < 4; e++) {
-            const int n = 4 * j + e;
-            if (n < N) c[n] = v[e] + (bias ? __ldg(bias + n) : 0.f);
+            const int n = n0 + 4 * j + e;
+            if (n < N) c[4 * j + e] = v[e] + (bias ? __ldg(bias + n) : 0.f);
           }
         }
       }
@@ -1006,7 +1014,8 @@ __global__ void __launch_bounds__(NTH) gemm_rows_kernel(const float* __restrict_
   }
   orion_signal(sig);
 }
-inline int smem_bytes(int K, int N) { return (K * ((N + 3) & ~3) + KC * (NTH + 1)) * 4; }
+inline int rpc(int N) { return NTH / ((N + NCH - 1) / NCH); }
+inline int smem_bytes(int K, int N) { return (K * ((N + 3) & ~3) + KC * (rpc(N) + 1)) * 4; }
 }  // namespace rows
 
 // ---------------------------------------------------------------- small-M GEMM (GEMV-like)
@@ -1202,6 +1211,161 @@ int launch_tiled(const LaunchGeom& g, long long M, long long N, long long K, flo
   return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
 }
 
+// ---------------------------------------------------------------- few-input-channel convs (stem)
+// The network stem (C = 3 input channels) makes a poor implicit GEMM (K = R*S*C = 27). Forward: one
+// thread per output pixel gathers its R*S*C window into registers and produces all K outputs
+// (weights in shared memory, 128-bit stores of the output row). Weight gradient: a CTA streams
+// blocks of 64 output pixels, staging dy rows (contiguous) and the gathered input patches in
+// shared memory; each thread owns a 4x4 block of dW over a fixed subset of the pixels; splits are
+// combined with the ordered split reduction.
+namespace smallc {
+constexpr int NTH = 256, MAXK = 64, MAXRSC = 64, PB = 32;
+
+template <int R, int S, int C>
+__global__ void __launch_bounds__(NTH) conv_fwd_smallc_kernel(const float* __restrict__ x, const float* __restrict__ w,
+                                                              float* __restrict__ y, ConvShape s, OrionSig sig) {
+  constexpr int RSC = R * S * C;
+  __shared__ float ws_[MAXK * RSC];
+  for (int i = threadIdx.x; i < s.K * RSC; i += NTH) ws_[i] = __ldg(w + i);
+  __syncthreads();
+  const long long npix = (long long)s.N * s.P * s.Q;
+  for (long long pix = (long long)blockIdx.x * NTH + threadIdx.x; pix < npix; pix += (long long)gridDim.x * NTH) {
+    const int q = (int)(pix % s.Q); const long long t = pix / s.Q;
+    const int p = (int)(t % s.P); const int n = (int)(t / s.P);
+    float patch[RSC];
+#pragma unroll
+    for (int r = 0; r < R; r++) {
+      const int h = p * s.stride - s.pad + r;
+#pragma unroll
+      for (int u = 0; u < S; u++) {
+        const int ww = q * s.stride - s.pad + u;
+        const bool ok = (unsigned)h < (unsigned)s.H && (unsigned)ww < (unsigned)s.W;
+        const float* src = x + (((long long)n * s.H + (ok ? h : 0)) * s.W + (ok ? ww : 0)) * C;
+#pragma unroll
+        for (int c = 0; c < C; c++) patch[(r * S + u) * C + c] = ok ? __ldg(src + c) : 0.f;
+      }
+    }
+    float* dst = y + pix * s.K;
+    for (int k0 = 0; k0 < s.K; k0 += 4) {
+      float o[4];
+#pragma unroll
+      for (int j = 0; j < 4; j++) {
+        const float* wr = ws_ + (k0 + j) * RSC;
+        float acc = 0.f;
+#pragma unroll
+        for (int i = 0; i < RSC; i++) acc = fmaf(patch[i], wr[i], acc);
+        o[j] = acc;
+      }
+      *reinterpret_cast<float4*>(dst + k0) = make_float4(o[0], o[1], o[2], o[3]);
+    }
+  }
+  orion_signal(sig);
+}
+
+template <int R, int S, int C>
+__global__ void __launch_bounds__(NTH) conv_wgrad_smallc_kernel(GemmParams p, const float* __restrict__ x, const float* __restrict__ dy,
+                                                                ConvShape s, OrionSig sig) {
+  __shared__ __align__(16) float dys[PB][MAXK];
+  __shared__ __align__(16) float pat[PB][MAXRSC + 4];
+  __shared__ float red[NTH * 16];
+  const int tid = threadIdx.x;
+  constexpr int RSC = R * S * C;
+  const int K = s.K;
+  const int mb = (K + 3) / 4, nb = (RSC + 3) / 4, nblk = mb * nb;
+  const int G = NTH / nblk, grp = tid / nblk, blk = tid % nblk;
+  const int bm = (blk / nb) * 4, bn = (blk % nb) * 4;
+  const bool active = grp < G;
+  const int kbeg = blockIdx.z * p.kps, kend = min(p.K, kbeg + p.kps);
+  float acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; i++)
+#pragma unroll
+    for (int j = 0; j < 4; j++) acc[i][j] = 0.f;
+  for (int b0 = kbeg; b0 < kend; b0 += PB) {
+    const int nb_pix = min(PB, kend - b0);
+    __syncthreads();
+    for (int i = tid; i < PB * K; i += NTH) {
+      const int r = i / K, c = i % K;
+      dys[r][c] = r < nb_pix ? __ldg(dy + (long long)(b0 + r) * K + c) : 0.f;
+    }
+    // gather the patches: one thread per (pixel, tap), C consecutive channels each
+    for (int i = tid; i < PB * R * S; i += NTH) {
+      const int r = i / (R * S), tap = i % (R * S), rr = tap / S, u = tap % S;
+      float v[C];
+#pragma unroll
+      for (int c = 0; c < C; c++) v[c] = 0.f;
+      if (r < nb_pix) {
+        const long long pix = b0 + r;
+        const int q = (int)(pix % s.Q); const long long t = pix / s.Q;
+        const int pp = (int)(t % s.P); const int n = (int)(t / s.P);
+        const int h = pp * s.stride - s.pad + rr, ww = q * s.stride - s.pad + u;
+        if ((unsigned)h < (unsigned)s.H && (unsigned)ww < (unsigned)s.W) {
+          const float* src = x + (((long long)n * s.H + h) * s.W + ww) * C;
+#pragma unroll
+          for (int c = 0; c < C; c++) v[c] = __ldg(src + c);
+        }
+      }
+#pragma unroll
+      for (int c = 0; c < C; c++) pat[r][tap * C + c] = v[c];
+    }
+    for (int i = tid; i < PB * (MAXRSC + 4 - RSC); i += NTH) {   // zero the padding columns
+      const int r = i / (MAXRSC + 4 - RSC), e = RSC + i % (MAXRSC + 4 - RSC);
+      pat[r][e] = 0.f;
+    }
+    __syncthreads();
+    if (active) {
+      for (int r = grp; r < nb_pix; r += G) {
+        const float4 a = *reinterpret_cast<const float4*>(&dys[r][bm]);
+        const float4 b = *reinterpret_cast<const float4*>(&pat[r][bn]);
+        const float av[4] = {a.x, a.y, a.z, a.w}, bv[4] = {b.x, b.y, b.z, b.w};
+#pragma unroll
+        for (int i = 0; i < 4; i++)
+#pragma unroll
+          for (int j = 0; j < 4; j++) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
+      }
+    }
+  }
+  if (active) {
+#pragma unroll
+    for (int i = 0; i < 4; i++)
+#pragma unroll
+      for (int j = 0; j < 4; j++) red[(grp * nblk + blk) * 16 + i * 4 + j] = acc[i][j];
+  }
+  __syncthreads();
+  float* out = p.split == 1 ? nullptr : p.ws + (long long)blockIdx.z * p.M * p.N;
+  for (int e = tid; e < nblk * 16; e += NTH) {
+    const int b = e / 16, ij = e % 16, i = ij / 4, j = ij % 4;
+    const int m = (b / nb) * 4 + i, n = (b % nb) * 4 + j;
+    float v = 0.f;
+    for (int g = 0; g < G; g++) v += red[(g * nblk + b) * 16 + ij];
+    if (m < p.M && n < p.N) {
+      if (p.split == 1) p.C[(long long)m * p.ldc + n] = v;
+      else out[(long long)m * p.N + n] = v;
+    }
+  }
+  if (p.split > 1) split_finish(p, 0, 0, 0, p.M, p.N);
+  orion_signal(sig);
+}
+
+// specialised for the 3x3, 3-channel stem (the only few-channel conv of the workloads)
+inline bool fwd_ok(const ConvShape& s) { return s.C == 3 && s.R == 3 && s.S == 3 && s.K % 4 == 0 && s.K <= MAXK; }
+inline bool wgrad_ok(const ConvShape& s) {
+  const int nblk = ((s.K + 3) / 4) * ((s.R * s.S * s.C + 3) / 4);
+  return s.C == 3 && s.R == 3 && s.S == 3 && s.K <= MAXK && nblk <= NTH;
+}
+Plan wgrad_plan(const ConvShape& s) {
+  Plan pl;
+  pl.cfg = 8; pl.bm = s.K; pl.bn = s.R * s.S * s.C; pl.bk = PB;
+  long long npix = (long long)s.N * s.P * s.Q;
+  long long split = 148 * 4;
+  if (split > npix / (4 * PB)) split = npix / (4 * PB);
+  if (split > 1008) split = 1008;
+  if (split < 1) split = 1;
+  pl.split = (int)split;
+  return pl;
+}
+}  // namespace smallc
+
 }  // namespace
 
 // Workspace bytes a tiled GEMM of this (M, N, K) needs for its K split (0 if no split). Conv ops
@@ -1209,6 +1373,12 @@ int launch_tiled(const LaunchGeom& g, long long M, long long N, long long K, flo
 extern "C" uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t K) {
   Plan pl = plan_gemm((long long)M, (long long)N, (long long)K);
   uint64_t b = ws_bytes_for(pl, (long long)M, (long long)N);
+  if (M <= (uint64_t)smallc::MAXK && N <= (uint64_t)smallc::MAXRSC) {   // stem conv wgrad (few input channels)
+    ConvShape st{};
+    st.N = 1; st.P = 1; st.Q = (int)K; st.K = (int)M; st.R = 1; st.S = 1; st.C = (int)N;
+    uint64_t b3 = ws_bytes_for(smallc::wgrad_plan(st), (long long)M, (long long)N);
+    if (b3 > b) b = b3;
+  }
   if (atb_ok((long long)M, (long long)N, (long long)K)) {   // A^T B callers may take the skinny kernel
     uint64_t b2 = ws_bytes_for(plan_atb((long long)M, (long long)N, (long long)K), (long long)M, (long long)N);
     if (b2 > b) b = b2;
@@ -1237,7 +1407,7 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
         return ORION_E_CUDA;
       attr.store(1);
     }
-    g->grid = dim3((unsigned)cdiv(M, rows::NTH)); g->block = dim3(rows::NTH); g->smem = rows::smem_bytes((int)K, (int)N); g->func = f;
+    g->grid = dim3((unsigned)cdiv(M, rows::rpc((int)N))); g->block = dim3(rows::NTH); g->smem = rows::smem_bytes((int)K, (int)N); g->func = f;
     return 0;
   }
   if (flags == 1 && atb_ok(M, N, K)) {
@@ -1319,14 +1489,25 @@ static ConvShape conv_shape(const uint64_t* a) {
   return s;
 }
 
+
 // implicit-GEMM dims: fwd (M = N*P*Q, N = K, K = R*S*C); dgrad (N*H*W, C, R*S*K); wgrad (K, R*S*C, N*P*Q)
 int conv_fwd_geom(const uint64_t* a, LaunchGeom* g) {
   ConvShape s = conv_shape(a);
+  if (smallc::fwd_ok(s)) {
+    long long ctas = cdiv((long long)s.N * s.P * s.Q, smallc::NTH);
+    g->grid = dim3((unsigned)(ctas < 148 * 16 ? ctas : 148 * 16)); g->block = dim3(smallc::NTH); g->smem = 0;
+    g->func = (const void*)smallc::conv_fwd_smallc_kernel<3, 3, 3>;
+    return 0;
+  }
   tiled_geom<AIm2col, BDenseT>(g, (long long)s.N * s.P * s.Q, s.K, (long long)s.R * s.S * s.C, a[14], a[15]);
   return 0;
 }
 int conv_fwd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   ConvShape s = conv_shape(a);
+  if (g.func == (const void*)smallc::conv_fwd_smallc_kernel<3, 3, 3>) {
+    smallc::conv_fwd_smallc_kernel<3, 3, 3><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s, sig);
+    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+  }
   long long M = (long long)s.N * s.P * s.Q, N = s.K, K = (long long)s.R * s.S * s.C;
   return launch_tiled(g, M, N, K, (float*)a[2], N, nullptr, (float*)a[14], AIm2col{(const float*)a[0], s},
                       BDenseT{(const float*)a[1], K}, sig, st);
@@ -1346,11 +1527,25 @@ int conv_dgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cuda
 
 int conv_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
   ConvShape s = conv_shape(a);
+  if (smallc::wgrad_ok(s)) {
+    Plan pl = smallc::wgrad_plan(s);
+    if (pl.split > 1 && (a[14] == 0 || a[15] < ws_bytes_for(pl, pl.bm, pl.bn))) pl.split = 1;
+    g->grid = dim3(1, 1, (unsigned)pl.split); g->block = dim3(smallc::NTH); g->smem = 0;
+    g->func = (const void*)smallc::conv_wgrad_smallc_kernel<3, 3, 3>;
+    return 0;
+  }
   tiled_geom<ADenseT, BWgrad>(g, s.K, (long long)s.R * s.S * s.C, (long long)s.N * s.P * s.Q, a[14], a[15]);
   return 0;
 }
 int conv_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   ConvShape s = conv_shape(a);
+  if (g.func == (const void*)smallc::conv_wgrad_smallc_kernel<3, 3, 3>) {
+    const long long M = s.K, N = (long long)s.R * s.S * s.C, K = (long long)s.N * s.P * s.Q;
+    smallc::conv_wgrad_smallc_kernel<3, 3, 3><<<g.grid, g.block, 0, st>>>(
+        make_params(M, N, K, (float*)a[2], N, nullptr, (int)g.grid.z, (float*)a[14], smallc::PB), (const float*)a[0],
+        (const float*)a[1], s, sig);
+    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+  }
   long long M = s.K, N = (long long)s.R * s.S * s.C, K = (long long)s.N * s.P * s.Q;
   // A(m = kout, k = npq) = dy[npq * K + kout]
   return launch_tiled(g, M, N, K, (float*)a[2], N, nullptr, (float*)a[14], ADenseT{(const float*)a[1], s.K},
