@@ -4,7 +4,7 @@ mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
 OURS='(gemm_kernel|gemm_tc_kernel|gemm_atb_kernel|gemm_rows_kernel|gemv_bt_kernel|unary_kernel|binary_kernel|bn_|dw_|maxpool_kernel|avgpool|ce_kernel|mse_kernel|sgd_kernel|colsum_kernel)'
 for c in ${CLIENTS:-hp be}; do
-  timeout -s KILL 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,launch__grid_size,sm__throughput.avg.pct_of_peak_sustained_elapsed,gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed --clock-control none --csv --page raw \
+  timeout -s KILL 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,launch__grid_size --clock-control none --csv --page raw \
      --kernel-name-base function -k "regex:$OURS" --log-file gpurun_out/ncu_times_${c}.csv python tools/profile/solo_runner.py --client $c > gpurun_out/ncu_times_${c}.out 2>&1
   base=0; [ "$c" = be ] && base=10000
   python tools/profile/ncu_summarize.py gpurun_out/ncu_times_${c}.csv gpurun_out/oplist_rn50_mnv2_${c}.txt 0 gpurun_out/times_${c}.csv
