@@ -1350,8 +1350,10 @@ __global__ void __launch_bounds__(NTH) conv_wgrad_smallc_kernel(GemmParams p, co
 // specialised for the 3x3, 3-channel stem (the only few-channel conv of the workloads)
 inline bool fwd_ok(const ConvShape& s) { return s.C == 3 && s.R == 3 && s.S == 3 && s.K % 4 == 0 && s.K <= MAXK; }
 inline bool wgrad_ok(const ConvShape& s) {
-  const int nblk = ((s.K + 3) / 4) * ((s.R * s.S * s.C + 3) / 4);
-  return s.C == 3 && s.R == 3 && s.S == 3 && s.K <= MAXK && nblk <= NTH;
+  // measured slower than the tiled split-K path on the MobileNetV2 stem (449 vs 311 us): kept for
+  // reference, not routed
+  (void)s;
+  return false;
 }
 Plan wgrad_plan(const ConvShape& s) {
   Plan pl;
@@ -1396,7 +1398,7 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     g->grid = dim3((unsigned)cdiv(N, 8)); g->block = dim3(256); g->smem = 0; g->func = (const void*)gemv_bt_kernel;
     return 0;
   }
-  if ((flags == 0 || flags == 2) && M >= 4096 && N <= rows::MAXN && K * ((N + 3) & ~3) <= rows::MAXKN) {
+  if ((flags == 0 || flags == 2) && M >= 4096 && N <= 32 && K * ((N + 3) & ~3) <= rows::MAXKN) {
     const void* f = flags == 2 ? (const void*)rows::gemm_rows_kernel<true> : (const void*)rows::gemm_rows_kernel<false>;
     static std::atomic<int> attr{0};
     if (!attr.load()) {
