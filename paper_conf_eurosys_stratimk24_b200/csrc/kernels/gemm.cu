@@ -931,7 +931,7 @@ __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float
 // conflict-free), B lives in shared memory for the whole CTA (broadcast reads), and each thread
 // accumulates its row's N outputs in registers in k order (deterministic, no split).
 namespace rows {
-constexpr int NTH = 256, KC = 32, NCH = 32, MAXN = 128, MAXKN = 16384;
+constexpr int NTH = 256, KC = 32, NCH = 32, MAXKN = 16384;
 
 // Threads are (row, chunk): each thread owns NCH = 32 consecutive outputs of one row; a CTA holds
 // RPC = 256 / nchunk rows (nchunk = ceil(N / 32) <= 4).
@@ -1214,12 +1214,10 @@ int launch_tiled(const LaunchGeom& g, long long M, long long N, long long K, flo
 // ---------------------------------------------------------------- few-input-channel convs (stem)
 // The network stem (C = 3 input channels) makes a poor implicit GEMM (K = R*S*C = 27). Forward: one
 // thread per output pixel gathers its R*S*C window into registers and produces all K outputs
-// (weights in shared memory, 128-bit stores of the output row). Weight gradient: a CTA streams
-// blocks of 64 output pixels, staging dy rows (contiguous) and the gathered input patches in
-// shared memory; each thread owns a 4x4 block of dW over a fixed subset of the pixels; splits are
-// combined with the ordered split reduction.
+// (weights in shared memory, 128-bit stores of the output row). (The stem's weight gradient stays
+// on the tiled split-K path, which measured faster.)
 namespace smallc {
-constexpr int NTH = 256, MAXK = 64, MAXRSC = 64, PB = 32;
+constexpr int NTH = 256, MAXK = 64;
 
 template <int R, int S, int C>
 __global__ void __launch_bounds__(NTH) conv_fwd_smallc_kernel(const float* __restrict__ x, const float* __restrict__ w,
@@ -1262,110 +1260,8 @@ __global__ void __launch_bounds__(NTH) conv_fwd_smallc_kernel(const float* __res
   orion_signal(sig);
 }
 
-template <int R, int S, int C>
-__global__ void __launch_bounds__(NTH) conv_wgrad_smallc_kernel(GemmParams p, const float* __restrict__ x, const float* __restrict__ dy,
-                                                                ConvShape s, OrionSig sig) {
-  __shared__ __align__(16) float dys[PB][MAXK];
-  __shared__ __align__(16) float pat[PB][MAXRSC + 4];
-  __shared__ float red[NTH * 16];
-  const int tid = threadIdx.x;
-  constexpr int RSC = R * S * C;
-  const int K = s.K;
-  const int mb = (K + 3) / 4, nb = (RSC + 3) / 4, nblk = mb * nb;
-  const int G = NTH / nblk, grp = tid / nblk, blk = tid % nblk;
-  const int bm = (blk / nb) * 4, bn = (blk % nb) * 4;
-  const bool active = grp < G;
-  const int kbeg = blockIdx.z * p.kps, kend = min(p.K, kbeg + p.kps);
-  float acc[4][4];
-#pragma unroll
-  for (int i = 0; i < 4; i++)
-#pragma unroll
-    for (int j = 0; j < 4; j++) acc[i][j] = 0.f;
-  for (int b0 = kbeg; b0 < kend; b0 += PB) {
-    const int nb_pix = min(PB, kend - b0);
-    __syncthreads();
-    for (int i = tid; i < PB * K; i += NTH) {
-      const int r = i / K, c = i % K;
-      dys[r][c] = r < nb_pix ? __ldg(dy + (long long)(b0 + r) * K + c) : 0.f;
-    }
-    // gather the patches: one thread per (pixel, tap), C consecutive channels each
-    for (int i = tid; i < PB * R * S; i += NTH) {
-      const int r = i / (R * S), tap = i % (R * S), rr = tap / S, u = tap % S;
-      float v[C];
-#pragma unroll
-      for (int c = 0; c < C; c++) v[c] = 0.f;
-      if (r < nb_pix) {
-        const long long pix = b0 + r;
-        const int q = (int)(pix % s.Q); const long long t = pix / s.Q;
-        const int pp = (int)(t % s.P); const int n = (int)(t / s.P);
-        const int h = pp * s.stride - s.pad + rr, ww = q * s.stride - s.pad + u;
-        if ((unsigned)h < (unsigned)s.H && (unsigned)ww < (unsigned)s.W) {
-          const float* src = x + (((long long)n * s.H + h) * s.W + ww) * C;
-#pragma unroll
-          for (int c = 0; c < C; c++) v[c] = __ldg(src + c);
-        }
-      }
-#pragma unroll
-      for (int c = 0; c < C; c++) pat[r][tap * C + c] = v[c];
-    }
-    for (int i = tid; i < PB * (MAXRSC + 4 - RSC); i += NTH) {   // zero the padding columns
-      const int r = i / (MAXRSC + 4 - RSC), e = RSC + i % (MAXRSC + 4 - RSC);
-      pat[r][e] = 0.f;
-    }
-    __syncthreads();
-    if (active) {
-      for (int r = grp; r < nb_pix; r += G) {
-        const float4 a = *reinterpret_cast<const float4*>(&dys[r][bm]);
-        const float4 b = *reinterpret_cast<const float4*>(&pat[r][bn]);
-        const float av[4] = {a.x, a.y, a.z, a.w}, bv[4] = {b.x, b.y, b.z, b.w};
-#pragma unroll
-        for (int i = 0; i < 4; i++)
-#pragma unroll
-          for (int j = 0; j < 4; j++) acc[i][j] = fmaf(av[i], bv[j], acc[i][j]);
-      }
-    }
-  }
-  if (active) {
-#pragma unroll
-    for (int i = 0; i < 4; i++)
-#pragma unroll
-      for (int j = 0; j < 4; j++) red[(grp * nblk + blk) * 16 + i * 4 + j] = acc[i][j];
-  }
-  __syncthreads();
-  float* out = p.split == 1 ? nullptr : p.ws + (long long)blockIdx.z * p.M * p.N;
-  for (int e = tid; e < nblk * 16; e += NTH) {
-    const int b = e / 16, ij = e % 16, i = ij / 4, j = ij % 4;
-    const int m = (b / nb) * 4 + i, n = (b % nb) * 4 + j;
-    float v = 0.f;
-    for (int g = 0; g < G; g++) v += red[(g * nblk + b) * 16 + ij];
-    if (m < p.M && n < p.N) {
-      if (p.split == 1) p.C[(long long)m * p.ldc + n] = v;
-      else out[(long long)m * p.N + n] = v;
-    }
-  }
-  if (p.split > 1) split_finish(p, 0, 0, 0, p.M, p.N);
-  orion_signal(sig);
-}
-
 // specialised for the 3x3, 3-channel stem (the only few-channel conv of the workloads)
 inline bool fwd_ok(const ConvShape& s) { return s.C == 3 && s.R == 3 && s.S == 3 && s.K % 4 == 0 && s.K <= MAXK; }
-inline bool wgrad_ok(const ConvShape& s) {
-  // measured slower than the tiled split-K path on the MobileNetV2 stem (449 vs 311 us): kept for
-  // reference, not routed
-  (void)s;
-  return false;
-}
-Plan wgrad_plan(const ConvShape& s) {
-  Plan pl;
-  pl.cfg = 8; pl.bm = s.K; pl.bn = s.R * s.S * s.C; pl.bk = PB;
-  long long npix = (long long)s.N * s.P * s.Q;
-  long long split = 148 * 4;
-  if (split > npix / (4 * PB)) split = npix / (4 * PB);
-  if (split > 1008) split = 1008;
-  if (split < 1) split = 1;
-  pl.split = (int)split;
-  return pl;
-}
 }  // namespace smallc
 
 }  // namespace
@@ -1375,12 +1271,6 @@ Plan wgrad_plan(const ConvShape& s) {
 extern "C" uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t K) {
   Plan pl = plan_gemm((long long)M, (long long)N, (long long)K);
   uint64_t b = ws_bytes_for(pl, (long long)M, (long long)N);
-  if (M <= (uint64_t)smallc::MAXK && N <= (uint64_t)smallc::MAXRSC) {   // stem conv wgrad (few input channels)
-    ConvShape st{};
-    st.N = 1; st.P = 1; st.Q = (int)K; st.K = (int)M; st.R = 1; st.S = 1; st.C = (int)N;
-    uint64_t b3 = ws_bytes_for(smallc::wgrad_plan(st), (long long)M, (long long)N);
-    if (b3 > b) b = b3;
-  }
   if (atb_ok((long long)M, (long long)N, (long long)K)) {   // A^T B callers may take the skinny kernel
     uint64_t b2 = ws_bytes_for(plan_atb((long long)M, (long long)N, (long long)K), (long long)M, (long long)N);
     if (b2 > b) b = b2;
@@ -1529,26 +1419,11 @@ int conv_dgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cuda
 
 int conv_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
   ConvShape s = conv_shape(a);
-  if (smallc::wgrad_ok(s)) {
-    Plan pl = smallc::wgrad_plan(s);
-    if (pl.split > 1 && (a[14] == 0 || a[15] < ws_bytes_for(pl, pl.bm, pl.bn))) pl.split = 1;
-    g->grid = dim3(1, 1, (unsigned)pl.split); g->block = dim3(smallc::NTH); g->smem = 0;
-    g->func = (const void*)smallc::conv_wgrad_smallc_kernel<3, 3, 3>;
-    return 0;
-  }
   tiled_geom<ADenseT, BWgrad>(g, s.K, (long long)s.R * s.S * s.C, (long long)s.N * s.P * s.Q, a[14], a[15]);
   return 0;
 }
 int conv_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   ConvShape s = conv_shape(a);
-  if (g.func == (const void*)smallc::conv_wgrad_smallc_kernel<3, 3, 3>) {
-    const long long M = s.K, N = (long long)s.R * s.S * s.C, K = (long long)s.N * s.P * s.Q;
-    smallc::conv_wgrad_smallc_kernel<3, 3, 3><<<g.grid, g.block, 0, st>>>(
-        make_params(M, N, K, (float*)a[2], N, nullptr, (int)g.grid.z, (float*)a[14], smallc::PB), (const float*)a[0],
-        (const float*)a[1], s, sig);
-    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
-  }
-  long long M = s.K, N = (long long)s.R * s.S * s.C, K = (long long)s.N * s.P * s.Q;
   // A(m = kout, k = npq) = dy[npq * K + kout]
   return launch_tiled(g, M, N, K, (float*)a[2], N, nullptr, (float*)a[14], ADenseT{(const float*)a[1], s.K},
                       BWgrad{(const float*)a[0], s}, sig, st);
