@@ -1424,6 +1424,7 @@ int conv_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
 }
 int conv_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   ConvShape s = conv_shape(a);
+  long long M = s.K, N = (long long)s.R * s.S * s.C, K = (long long)s.N * s.P * s.Q;
   // A(m = kout, k = npq) = dy[npq * K + kout]
   return launch_tiled(g, M, N, K, (float*)a[2], N, nullptr, (float*)a[14], ADenseT{(const float*)a[1], s.K},
                       BWgrad{(const float*)a[0], s}, sig, st);
