@@ -81,12 +81,12 @@ struct CudaBackend : Backend {
     if (!resolve("cuStreamWriteValue64", &drv.streamWriteValue64, 12000)) return ORION_E_CUDA;
     be_partition = cfg.be_partition_sms;
     if (be_partition) {
-      bool ok = resolve("cuDeviceGetDevResource", &drv.deviceGetDevResource, 12040) &&
-                resolve("cuDevSmResourceSplitByCount", &drv.devSmResourceSplitByCount, 12040) &&
-                resolve("cuDevResourceGenerateDesc", &drv.devResourceGenerateDesc, 12040) &&
-                resolve("cuGreenCtxCreate", &drv.greenCtxCreate, 12040) &&
-                resolve("cuGreenCtxStreamCreate", &drv.greenCtxStreamCreate, 12040) &&
-                resolve("cuGreenCtxDestroy", &drv.greenCtxDestroy, 12040);
+      bool ok = resolve("cuDeviceGetDevResource", &drv.deviceGetDevResource, 12080) &&
+                resolve("cuDevSmResourceSplitByCount", &drv.devSmResourceSplitByCount, 12080) &&
+                resolve("cuDevResourceGenerateDesc", &drv.devResourceGenerateDesc, 12080) &&
+                resolve("cuGreenCtxCreate", &drv.greenCtxCreate, 12080) &&
+                resolve("cuGreenCtxStreamCreate", &drv.greenCtxStreamCreate, 12080) &&
+                resolve("cuGreenCtxDestroy", &drv.greenCtxDestroy, 12080);
       if (!ok) return ORION_E_CUDA;
     }
     if (cudaHostAlloc((void**)&host_counters, 64 * 8 * 16, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess)

@@ -213,3 +213,19 @@ def test_geometry_and_sm_needed():
     grid, bps, thr, smem = orion.kernel_geometry("relu", [A.data_ptr(), A.data_ptr(), A.numel()])
     assert grid == min((A.numel() // 4 + 255) // 256, 148 * 8) and 1 <= bps <= 8
     assert orion.profiler.sm_needed("relu", [A.data_ptr(), A.data_ptr(), A.numel()]) == -(-grid // bps)
+
+
+def test_green_context_partition_runs_and_is_bitwise_equal():
+    """A BE client confined to a green-context SM partition (cuGreenCtxCreate, 8-SM granularity)
+    produces bitwise the same parameters as on the full GPU (partition-independent kernels)."""
+    from paper_conf_eurosys_stratimk24_b200 import workloads as W, collocate as C
+    from synth import inputs as si
+    P = si.make_params(W.mlp_spec())
+    xs = [si.normal((32, 512), si.BE_SEED, sub=i) for i in range(2)]
+    g = W.mlp_train_graph(P, xs, xs)
+    be = C.BEClient(g)
+    C.run_session(be=be, be_iters=6)
+    ref = g.params.flat.cpu().clone()
+    g.params.reset()
+    C.run_session(be=be, be_iters=6, be_partition_sms=16)
+    assert torch.equal(g.params.flat.cpu(), ref)
