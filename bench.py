@@ -197,8 +197,6 @@ def main():
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", 0))
-    world = int(os.environ.get("WORLD_SIZE", 1))
-    local = int(os.environ.get("LOCAL_RANK", 0))
     metric = "HP p99 latency vs dedicated; BE iters/s under collocation, 1-8 B200"
 
     if args.impl == "reference":
@@ -215,24 +213,12 @@ def main():
         print(json.dumps(line), flush=True)
         return
 
-    import torch.distributed as dist
-    if world > 1:
-        dist.init_process_group("gloo")
+    from paper_conf_eurosys_stratimk24_b200 import replicas as RP
+    rank, world, local = RP.init_from_env()
     torch.cuda.set_device(local)
     from paper_conf_eurosys_stratimk24_b200 import collocate as C, profiler as PR, _lib as L
-    from paper_conf_eurosys_stratimk24_b200.profiler import op_work
     from synth import inputs as si
-
-    def barrier():
-        if world > 1:
-            dist.barrier()
-
-    def allmax(x):
-        if world == 1:
-            return [x]
-        t = [None] * world
-        dist.all_gather_object(t, x)
-        return t
+    barrier = RP.barrier
 
     W_ = build_config(args.config, rank)
     rate = args.rate or W_["rate"]
@@ -344,15 +330,16 @@ def main():
     # ---- aggregate over ranks
     mine = dict(be_col=be_col, be_ded=be_ded, win_ms=win_ms, p99=col["p99_ns"], p50=col["p50_ns"], p99d=ded["p99_ns"],
                 p50d=ded["p50_ns"], e2e=(e2e or {}).get("value", 0.0), be_n=be_n)
-    allr = allmax(mine)
+    allr = RP.gather(mine)
     if rank != 0:
         return
-    value = sum(r["be_col"] for r in allr)
+    agg = RP.aggregate(allr, args.steps)
+    value = agg["value"]
     cpu = None
     if not args.no_cpu_baseline:
         v, sample, cores = cpu_oracle_sample(args.config)
         cpu = {"value": v, "unit": "it/s", "cores": cores, "kind": "oracle", "sample": sample}
-    ms_per_step = max(r["win_ms"] for r in allr) / args.steps
+    ms_per_step = agg["ms_per_step"]
     line = {
         "metric": metric, "value": value, "unit": "it/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
@@ -363,10 +350,11 @@ def main():
         "hp": {"p50_ms": col["p50_ns"] / 1e6, "p99_ms": col["p99_ns"] / 1e6, "dedicated_p50_ms": ded["p50_ns"] / 1e6,
                "dedicated_p99_ms": ded["p99_ns"] / 1e6, "p99_vs_dedicated": col["p99_ns"] / ded["p99_ns"],
                "p50_vs_dedicated": col["p50_ns"] / ded["p50_ns"], "solo_latency_ms": hp_lat_ns / 1e6,
-               "requests": col["n"], "per_rank_p99_ratio": [r["p99"] / r["p99d"] for r in allr]},
-        "be": {"collocated_its": value, "dedicated_its": sum(r["be_ded"] for r in allr),
-               "fraction_of_dedicated": value / max(sum(r["be_ded"] for r in allr), 1e-9),
-               "iterations_in_window": sum(r["be_n"] for r in allr)},
+               "requests": col["n"], "per_rank_p99_ratio": agg["hp_p99_ratio_per_rank"],
+               "worst_rank_p99_ratio": agg["hp_p99_ratio_max"]},
+        "be": {"collocated_its": value, "dedicated_its": agg["be_dedicated"],
+               "fraction_of_dedicated": value / max(agg["be_dedicated"], 1e-9),
+               "iterations_in_window": agg["be_iterations"]},
         "target": {"hp_p99_ratio_max": 1.15, "be_fraction_min": 0.5},
         "roofline": {"kernel": top_row["label"], "bound": bound, "achieved": achieved, "peak": peak, "unit": unit,
                      "frac": (achieved / peak) if achieved and peak else None, "traffic": traffic,
