@@ -362,7 +362,7 @@ def main():
                      "algorithmic_bytes": nbytes, "algorithmic_flops": flops, "peak_source": pk_src},
         "cpu_baseline": cpu,
         "e2e": e2e,
-        "gpu_launches": int(args.steps * n_hp_k + sum(r["be_n"] for r in allr) // max(world, 1) * n_be_k),
+        "gpu_launches": int(world * args.steps * n_hp_k + sum(r["be_n"] for r in allr) * n_be_k),
         "clocks": clocks,
         "scheduler": rc["stats"],
     }
