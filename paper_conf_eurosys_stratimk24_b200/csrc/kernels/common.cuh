@@ -17,9 +17,11 @@ struct OrionSig {
 
 __device__ __forceinline__ void orion_signal(const OrionSig& sig) {
   if (sig.ticket == nullptr) return;  // direct launch (no scheduler)
-  __threadfence();                    // this thread's global writes visible GPU-wide
+  // bar.sync orders the CTA's writes before thread 0; its gpu-scope fence is cumulative over what
+  // it observed through the barrier (the release pattern CUTLASS semaphores use)
   __syncthreads();
   if (threadIdx.x == 0 && threadIdx.y == 0 && threadIdx.z == 0) {
+    __threadfence();
     unsigned long long t = atomicAdd(sig.ticket, 1ull) + 1ull;
     if (t == sig.target) {
       __threadfence_system();
@@ -57,9 +59,9 @@ __host__ __device__ __forceinline__ uint64_t cdiv(uint64_t a, uint64_t b) { retu
 // reduces the partials in a fixed order. The ticket is reset by the last CTA.
 __device__ __forceinline__ bool last_cta_of(unsigned int* ticket, unsigned int count) {
   __shared__ unsigned int s_last;
-  __threadfence();
   __syncthreads();
   if (threadIdx.x == 0) {
+    __threadfence();   // cumulative over the CTA's writes ordered before it by bar.sync
     unsigned int t = atomicAdd(ticket, 1u) + 1u;
     s_last = (t == count);
     if (t == count) *ticket = 0u;  // reset for the next launch (stream order serialises launches)

@@ -701,12 +701,15 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
     mma_commit(done_bar);           // accumulator complete
   }
 
-  // ---------------- epilogue: TMEM -> registers -> global (or split partials)
+  // ---------------- epilogue: TMEM -> registers -> shared tile -> coalesced global (or split partials)
+  // The stage buffers are free once the accumulator is complete; the 128 epilogue threads (TMEM
+  // lanes 0..127 = tile rows) park their rows in a padded shared tile, then write it out row-major
+  // with 128-bit stores (consecutive threads on consecutive columns).
   if (warp < 4) {
     mbar_wait(done_bar, 0);
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-    const int m = m0 + tid;
-    float* dst = p.split == 1 ? (p.C + (long long)m * p.ldc) : (p.ws + (long long)blockIdx.z * p.M * p.N + (long long)m * p.N);
+    constexpr int TS = BN + 4;   // padded row stride (floats): conflict-free 128-bit row writes
+    float* tile = reinterpret_cast<float*>(smem);
 #pragma unroll 1
     for (int c0 = 0; c0 < BN; c0 += 32) {
       float v[32];
@@ -722,12 +725,29 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
 #pragma unroll
         for (int i = 0; i < 32; i++) v[i] = 0.f;
       }
-      if (m < p.M) {
 #pragma unroll
-        for (int i = 0; i < 32; i++) {
-          const int n = n0 + c0 + i;
-          if (n < p.N) dst[n] = p.split == 1 ? v[i] + (p.bias ? __ldg(p.bias + n) : 0.f) : v[i];
-        }
+      for (int i = 0; i < 32; i += 4)
+        *reinterpret_cast<float4*>(tile + tid * TS + c0 + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+    }
+    asm volatile("bar.sync 1, 128;" ::: "memory");   // epilogue warps only
+    float* base = p.split == 1 ? p.C : p.ws + (long long)blockIdx.z * p.M * p.N;
+    const long long ld = p.split == 1 ? p.ldc : p.N;
+    const bool vec = ((ld & 3) == 0) && ((n0 & 3) == 0) && ((reinterpret_cast<uintptr_t>(base) & 15) == 0) &&
+                     (p.split > 1 || p.bias == nullptr);
+    constexpr int QPR = BN / 4;   // float4 per tile row
+    for (int e = tid; e < BM * QPR; e += 128) {
+      const int r = e / QPR, c = (e % QPR) * 4;
+      const int m = m0 + r, n = n0 + c;
+      if (m >= p.M) continue;
+      const float4 t4 = *reinterpret_cast<const float4*>(tile + r * TS + c);
+      float* dst = base + (long long)m * ld + n;
+      if (vec && n + 3 < p.N) {
+        *reinterpret_cast<float4*>(dst) = t4;
+      } else {
+        const float tv[4] = {t4.x, t4.y, t4.z, t4.w};
+#pragma unroll
+        for (int i = 0; i < 4; i++)
+          if (n + i < p.N) dst[i] = p.split == 1 ? tv[i] + (p.bias ? __ldg(p.bias + n + i) : 0.f) : tv[i];
       }
     }
   }
@@ -1109,8 +1129,8 @@ Plan plan_gemm(long long M, long long N, long long K) {
     long long tiles = cdiv(M, pl.bm) * cdiv(N, pl.bn);
     long long ktiles = cdiv(K, pl.bk);
     long long split = 1;
-    if (tiles < 148) {              // one CTA per SM (~196 KB smem each): fill a 148-SM part once
-      split = cdiv(148, tiles);
+    if (tiles < 148) {              // one CTA per SM (~196 KB smem each): fill a 148-SM part once,
+      split = 148 / tiles;          // never spilling into a second wave
       if (split > ktiles / 4) split = ktiles / 4;   // >= 4 k-tiles per split
       if (split > 16) split = 16;                   // bounded ordered reduction (<= 512 KB per tile)
       if (split < 1) split = 1;
