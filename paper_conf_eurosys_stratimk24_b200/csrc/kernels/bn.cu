@@ -24,18 +24,19 @@ BnSplit bn_split(long long rows, int C) {
   s.rl = BN_THREADS / s.cg4;
   s.cblocks = (int)cdiv(q, s.cg4);
   long long rs = cdiv(148 * 4, s.cblocks);      // shape-only: ~4 CTAs per SM of a 148-SM part
-  long long max_rs = cdiv(rows, 32LL * s.rl);   // >= 32 rows per row lane (8 unrolled trips)
+  long long max_rs = cdiv(rows, 16LL * s.rl);   // >= 16 rows per row lane (2 trips of 8 loads)
   if (rs > max_rs) rs = max_rs;
   if (rs < 1) rs = 1;
-  if (rs > 2048) rs = 2048;
+  if (rs > 1024) rs = 1024;
   s.rs = (int)rs;
   s.rows_per_split = cdiv(rows, rs);
   return s;
 }
 
+// workspace: [tickets][split partials rs x C x nvals][group partials combine_rows(rs) x C x nvals]
 uint64_t bn_ws_bytes(long long rows, int C, int nvals) {
   BnSplit s = bn_split(rows, C);
-  return WS_TICKET_BYTES + (uint64_t)s.rs * C * nvals * 8;
+  return WS_TICKET_BYTES + (uint64_t)(s.rs + combine_rows(s.rs)) * C * nvals * 8;
 }
 
 struct D4 { double x, y, z, w; };
@@ -46,8 +47,10 @@ __device__ __forceinline__ void sq4(D4& a, const float4& v) {
 }
 
 // Combine two D4 accumulators per thread over the CTA's row lanes (fixed order), write this
-// split's partial for the CTA's channels; returns true in the last CTA of the channel block.
-__device__ bool bn_partial2(const D4& a, const D4& b, int C, int cg4, int rl_n, unsigned char* ws, double* sh) {
+// split's partial for the CTA's channels, then combine the splits of the channel block in order
+// (combine_splits). Returns true in the one CTA per channel block whose tot[(ch*2) + {0,1}]
+// (ch = channel within the block) holds the totals.
+__device__ bool bn_partial2(const D4& a, const D4& b, int C, int cg4, int rl_n, unsigned char* ws, double* sh, double* tot) {
   const int tid = threadIdx.x, cq = tid % cg4, rl = tid / cg4;
   const bool active = rl < rl_n;
   if (active) {
@@ -67,46 +70,10 @@ __device__ bool bn_partial2(const D4& a, const D4& b, int C, int cg4, int rl_n, 
       part[((long long)blockIdx.y * C + c + k) * 2 + 1] = t[4 + k];
     }
   }
-  return last_cta_of(tickets + blockIdx.x, gridDim.y);
-}
-
-// Parallel ordered combine in the last CTA: each of the CTA's CB = 4*cg4 channels gets
-// T = 256/CB threads; thread j sums splits j, j+T, j+2T, ... in order, then the T partial sums
-// are added in thread order. Fixed by shape, so deterministic. Results for channel
-// (blockIdx.x*cg4 + cq)*4 + k land in tot[(cq*4 + k)*2 + {0,1}] (smem, valid after return).
-__device__ void bn_combine_all(double* tot, double* sh, int C, int cg4, int rs_count, unsigned char* ws) {
-  const double* part = reinterpret_cast<const double*>(ws + WS_TICKET_BYTES);
-  const int CB = 4 * cg4;
-  const int T = BN_THREADS / CB;
-  const int tid = threadIdx.x;
-  const int ch = tid % CB, j = tid / CB;
-  const int c = blockIdx.x * CB + ch;
-  double a = 0.0, b = 0.0;
-  if (j < T && c < C) {
-    int r = j;
-    for (; r + 3 * T < rs_count; r += 4 * T) {   // 4 independent loads in flight, fixed order
-      double a0 = __ldcg(part + ((long long)r * C + c) * 2), b0 = __ldcg(part + ((long long)r * C + c) * 2 + 1);
-      double a1 = __ldcg(part + ((long long)(r + T) * C + c) * 2), b1 = __ldcg(part + ((long long)(r + T) * C + c) * 2 + 1);
-      double a2 = __ldcg(part + ((long long)(r + 2 * T) * C + c) * 2), b2 = __ldcg(part + ((long long)(r + 2 * T) * C + c) * 2 + 1);
-      double a3 = __ldcg(part + ((long long)(r + 3 * T) * C + c) * 2), b3 = __ldcg(part + ((long long)(r + 3 * T) * C + c) * 2 + 1);
-      a += a0; a += a1; a += a2; a += a3;
-      b += b0; b += b1; b += b2; b += b3;
-    }
-    for (; r < rs_count; r += T) {
-      a += __ldcg(part + ((long long)r * C + c) * 2);
-      b += __ldcg(part + ((long long)r * C + c) * 2 + 1);
-    }
-  }
-  __syncthreads();
-  if (j < T) { sh[(j * CB + ch) * 2] = a; sh[(j * CB + ch) * 2 + 1] = b; }
-  __syncthreads();
-  if (j == 0) {
-    double ta = 0.0, tb = 0.0;
-    for (int k = 0; k < T; k++) { ta += sh[(k * CB + ch) * 2]; tb += sh[(k * CB + ch) * 2 + 1]; }
-    tot[ch * 2] = ta;
-    tot[ch * 2 + 1] = tb;
-  }
-  __syncthreads();
+  const int rs = gridDim.y, cb0 = blockIdx.x * cg4 * 4;
+  const int V = 2 * min(4 * cg4, C - cb0);
+  return combine_splits(tickets + blockIdx.x * (combine_rows(rs) + 1), part + 2LL * cb0, part + 2LL * rs * C + 2LL * cb0, 2LL * C, rs,
+                        blockIdx.y, V, tot, sh);
 }
 
 // ---- train statistics: mean, invstd (biased var), running stats (unbiased var, momentum)
@@ -121,12 +88,12 @@ __global__ void __launch_bounds__(BN_THREADS) bn_stats_kernel(const float* __res
   if (c < C && rl < rl_n) {
     const float* xp = x + c;
     long long r = r0 + rl;
-    for (; r + 3LL * rl_n < r1; r += 4LL * rl_n) {
-      float4 v0 = __ldg(reinterpret_cast<const float4*>(xp + r * C));
-      float4 v1 = __ldg(reinterpret_cast<const float4*>(xp + (r + rl_n) * C));
-      float4 v2 = __ldg(reinterpret_cast<const float4*>(xp + (r + 2LL * rl_n) * C));
-      float4 v3 = __ldg(reinterpret_cast<const float4*>(xp + (r + 3LL * rl_n) * C));
-      add4(s1, v0); sq4(s2, v0); add4(s1, v1); sq4(s2, v1); add4(s1, v2); sq4(s2, v2); add4(s1, v3); sq4(s2, v3);
+    for (; r + 7LL * rl_n < r1; r += 8LL * rl_n) {
+      float4 v[8];
+#pragma unroll
+      for (int i = 0; i < 8; i++) v[i] = __ldg(reinterpret_cast<const float4*>(xp + (r + i * (long long)rl_n) * C));
+#pragma unroll
+      for (int i = 0; i < 8; i++) { add4(s1, v[i]); sq4(s2, v[i]); }
     }
     for (; r < r1; r += rl_n) {
       float4 v = __ldg(reinterpret_cast<const float4*>(xp + r * C));
@@ -134,8 +101,7 @@ __global__ void __launch_bounds__(BN_THREADS) bn_stats_kernel(const float* __res
     }
   }
   __shared__ double tot[BN_THREADS * 2];
-  if (bn_partial2(s1, s2, C, cg4, rl_n, ws, sh)) {
-    bn_combine_all(tot, sh, C, cg4, gridDim.y, ws);
+  if (bn_partial2(s1, s2, C, cg4, rl_n, ws, sh, tot)) {
     if (rl == 0 && c < C) {
       for (int k = 0; k < 4; k++) {
         double t0 = tot[(cq * 4 + k) * 2], t1 = tot[(cq * 4 + k) * 2 + 1];
@@ -191,8 +157,7 @@ __global__ void __launch_bounds__(BN_THREADS) bn_bwd_reduce_kernel(const float* 
       acc(__ldg(reinterpret_cast<const float4*>(gp + r * C)), __ldg(reinterpret_cast<const float4*>(xp + r * C)));
   }
   __shared__ double tot[BN_THREADS * 2];
-  if (bn_partial2(sg, sgx, C, cg4, rl_n, ws, sh)) {
-    bn_combine_all(tot, sh, C, cg4, gridDim.y, ws);
+  if (bn_partial2(sg, sgx, C, cg4, rl_n, ws, sh, tot)) {
     if (rl == 0 && c < C) {
       for (int k = 0; k < 4; k++) {
         double t0 = tot[(cq * 4 + k) * 2], t1 = tot[(cq * 4 + k) * 2 + 1];

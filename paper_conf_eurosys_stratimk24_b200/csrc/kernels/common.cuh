@@ -77,6 +77,76 @@ __device__ __forceinline__ bool last_cta_of(unsigned int* ticket, unsigned int c
 // aliasing another op's tickets.
 constexpr uint64_t WS_TICKET_BYTES = 65536;
 
+// dst[v] = sum_{z < n} src[z * stride + v] for v < V, summed in z order, by all threads of the
+// CTA: value v gets T = blockDim / V threads (at least 1), thread j of them sums the fixed
+// contiguous chunk j of the n rows (8 loads in flight), and the T chunk sums are added in chunk
+// order. The split into chunks depends on (n, V, blockDim) only, so the result is deterministic.
+// scratch: >= blockDim doubles of shared memory. dst may be global or shared; on return (after
+// a barrier) dst is complete.
+__device__ __forceinline__ double sum_chunk(const double* src, long long stride, int z0, int z1, int v) {
+  double s = 0.0;
+  int z = z0;
+  for (; z + 7 < z1; z += 8) {
+    double a[8];
+#pragma unroll
+    for (int i = 0; i < 8; i++) a[i] = __ldcg(src + (long long)(z + i) * stride + v);
+#pragma unroll
+    for (int i = 0; i < 8; i++) s += a[i];
+  }
+  for (; z < z1; z++) s += __ldcg(src + (long long)z * stride + v);
+  return s;
+}
+__device__ inline void sum_rows_ordered(const double* src, long long stride, int n, int V, double* dst, double* scratch) {
+  const int nt = blockDim.x, t = threadIdx.x;
+  if (V >= nt / 2) {
+    for (int v = t; v < V; v += nt) dst[v] = sum_chunk(src, stride, 0, n, v);
+  } else {
+    int T = nt / V;
+    if (T > n) T = n > 0 ? n : 1;
+    const int v = t % V, j = t / V;
+    if (j < T) scratch[j * V + v] = sum_chunk(src, stride, (int)((long long)j * n / T), (int)((long long)(j + 1) * n / T), v);
+    __syncthreads();
+    if (t < V) {
+      double s = 0.0;
+      for (int k = 0; k < T; k++) s += scratch[k * V + t];
+      dst[t] = s;
+    }
+  }
+  __syncthreads();
+}
+
+// Ordered combine of per-split partial vectors, two levels when there are many splits. Split z of
+// a reduction (nz splits) has written its V values at part[z * stride ..]; the group partials
+// live at gpart[g * stride ..] (ng = ceil(nz / G) rows). Tickets: tk[0] final, tk[1 + g] per
+// group (zero at rest; reset by their last CTA). Level 1: the last CTA of each run of G
+// consecutive splits sums the run in order into gpart[g]; level 2: the last run sums the gpart
+// rows in order into out (shared, V doubles). Returns true in exactly one CTA, with out complete.
+// G is a function of nz only (combine_group), so results do not depend on the SM partition.
+__host__ __device__ __forceinline__ int combine_group(int nz) {
+  if (nz <= 16) return nz;
+  int g = 8;
+  while (g * g < nz) g++;
+  return g;
+}
+__host__ __device__ __forceinline__ int combine_rows(int nz) {   // gpart rows needed (0: one level)
+  return nz <= 16 ? 0 : (nz + combine_group(nz) - 1) / combine_group(nz);
+}
+__device__ inline bool combine_splits(unsigned int* tk, const double* part, double* gpart, long long stride, int nz, int z, int V,
+                                      double* out, double* scratch) {
+  if (nz <= 16) {
+    if (!last_cta_of(tk, (unsigned)nz)) return false;
+    sum_rows_ordered(part, stride, nz, V, out, scratch);
+    return true;
+  }
+  const int G = combine_group(nz), ng = (nz + G - 1) / G, g = z / G;
+  const int gsize = min(G, nz - g * G);
+  if (!last_cta_of(tk + 1 + g, (unsigned)gsize)) return false;
+  sum_rows_ordered(part + (long long)g * G * stride, stride, gsize, V, gpart + (long long)g * stride, scratch);
+  if (!last_cta_of(tk, (unsigned)ng)) return false;
+  sum_rows_ordered(gpart, stride, ng, V, out, scratch);
+  return true;
+}
+
 // Kernel table (table.cu)
 extern const KernelEntry g_kernels[ORION_FN_COUNT];
 int kernel_launch_sig(uint32_t fn, const uint64_t* args, uint32_t nargs, OrionSig sig, cudaStream_t s,

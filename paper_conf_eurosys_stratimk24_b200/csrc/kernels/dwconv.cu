@@ -2,7 +2,7 @@
 // weights [C][3][3][1]. fwd, stride-1 dgrad and wgrad slide a 3x3 register window along output
 // rows (one warp = 32 channels x one row); stride-2 dgrad gathers per output pixel (4 channels per
 // thread). wgrad reductions: fp32 per row, fp64 across rows, fixed-order CTA combine, ordered
-// split reduction by the last CTA per channel block.
+// split reduction (combine_splits) per channel block.
 #include "common.cuh"
 
 namespace {
@@ -241,21 +241,12 @@ __global__ void __launch_bounds__(DW_THREADS) dw_wgrad_rows_kernel(const float* 
       part[((long long)blockIdx.y * s.C + c) * 9 + t] = v;
     }
   }
-  if (last_cta_of(tickets + blockIdx.x, gridDim.y)) {
-    // 9 taps x 32 channels reduced by 8 warps: warp w takes taps w and w+8 (fixed split order)
-    for (int t = warp; t < 9; t += ROW_WARPS) {
-      if (c < s.C) {
-        double v = 0.0;
-        unsigned r = 0;
-        for (; r + 3 < gridDim.y; r += 4) {
-          double a0 = __ldcg(part + ((long long)r * s.C + c) * 9 + t), a1 = __ldcg(part + ((long long)(r + 1) * s.C + c) * 9 + t);
-          double a2 = __ldcg(part + ((long long)(r + 2) * s.C + c) * 9 + t), a3 = __ldcg(part + ((long long)(r + 3) * s.C + c) * 9 + t);
-          v += a0; v += a1; v += a2; v += a3;
-        }
-        for (; r < gridDim.y; r++) v += __ldcg(part + ((long long)r * s.C + c) * 9 + t);
-        dw[c * 9 + t] = (float)v;
-      }
-    }
+  __shared__ double out[9 * 32];
+  const int rs = gridDim.y, c0 = blockIdx.x * 32;
+  const int V = 9 * min(32, s.C - c0);
+  if (combine_splits(tickets + blockIdx.x * (combine_rows(rs) + 1), part + 9LL * c0, part + 9LL * rs * s.C + 9LL * c0, 9LL * s.C, rs,
+                     blockIdx.y, V, out, &sh[0][0][0])) {
+    for (int v = threadIdx.x; v < V; v += blockDim.x) dw[9LL * c0 + v] = (float)out[v];
   }
   orion_signal(sig);
 }
@@ -330,7 +321,8 @@ int wg_splits(const DwShape& s) {
 
 extern "C" uint64_t orion_dw_wgrad_workspace_bytes(uint64_t N, uint64_t C, uint64_t P, uint64_t Q) {
   DwShape s{(int)N, 0, 0, (int)C, 1, (int)P, (int)Q};
-  return WS_TICKET_BYTES + (uint64_t)wg_splits(s) * C * 9 * 8;
+  const int rs = wg_splits(s);
+  return WS_TICKET_BYTES + (uint64_t)(rs + combine_rows(rs)) * C * 9 * 8;
 }
 
 #define CHECK_LAUNCH() return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA

@@ -7,6 +7,7 @@
 // reduced by the last CTA of each tile in split order; the split count is a function of the
 // shape only (never of the SM partition), so results are identical solo and collocated.
 #include <atomic>
+#include <cstdlib>
 
 #include "common.cuh"
 
@@ -292,15 +293,12 @@ __device__ void reduce_range(const float* src, long long zstride, int count, flo
       const float* q = src + (long long)(m0 + r) * N + n0 + c;
       float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
       int z = 0;
-      for (; z + 3 < count; z += 4) {
-        float4 v0 = __ldcg(reinterpret_cast<const float4*>(q + z * zstride));
-        float4 v1 = __ldcg(reinterpret_cast<const float4*>(q + (z + 1) * zstride));
-        float4 v2 = __ldcg(reinterpret_cast<const float4*>(q + (z + 2) * zstride));
-        float4 v3 = __ldcg(reinterpret_cast<const float4*>(q + (z + 3) * zstride));
-        acc.x += v0.x; acc.x += v1.x; acc.x += v2.x; acc.x += v3.x;
-        acc.y += v0.y; acc.y += v1.y; acc.y += v2.y; acc.y += v3.y;
-        acc.z += v0.z; acc.z += v1.z; acc.z += v2.z; acc.z += v3.z;
-        acc.w += v0.w; acc.w += v1.w; acc.w += v2.w; acc.w += v3.w;
+      for (; z + 7 < count; z += 8) {
+        float4 v[8];
+#pragma unroll
+        for (int i = 0; i < 8; i++) v[i] = __ldcg(reinterpret_cast<const float4*>(q + (z + i) * zstride));
+#pragma unroll
+        for (int i = 0; i < 8; i++) { acc.x += v[i].x; acc.y += v[i].y; acc.z += v[i].z; acc.w += v[i].w; }
       }
       for (; z < count; z++) {
         float4 v = __ldcg(reinterpret_cast<const float4*>(q + z * zstride));
@@ -334,13 +332,18 @@ __device__ void reduce_range(const float* src, long long zstride, int count, flo
 // last CTA of the tile sums all partials in order. More: a fixed two-level tree — the last CTA of
 // each group of 16 consecutive splits sums the group into a group partial (after the split
 // partials in the workspace), and the last group to finish sums the group partials in order.
-constexpr int SPLIT_GROUP = 16, SPLIT_FLAT_MAX = 32, TICKETS_PER_TILE = 64;
+// The group size is ~sqrt(split) (combine_group: both levels sum ~sqrt(split) partials).
+constexpr int SPLIT_FLAT_MAX = 32, TICKETS_PER_TILE = 64;
+__host__ __device__ __forceinline__ int split_groups(int split) {   // group partials (0: flat)
+  return split <= SPLIT_FLAT_MAX ? 0 : (split + combine_group(split) - 1) / combine_group(split);
+}
 __device__ void split_finish(const GemmParams& p, int tile, int m0, int n0, int bm, int bn) {
   const long long MN = (long long)p.M * p.N;
   if (p.split <= SPLIT_FLAT_MAX) {
     if (last_cta_of(p.tickets + tile, p.split)) reduce_range(p.ws, MN, p.split, p.C, p.ldc, p.bias, p.M, p.N, m0, n0, bm, bn);
     return;
   }
+  const int SPLIT_GROUP = combine_group(p.split);
   const int ng = (p.split + SPLIT_GROUP - 1) / SPLIT_GROUP;
   const int g = blockIdx.z / SPLIT_GROUP;
   const int gsize = min(SPLIT_GROUP, p.split - g * SPLIT_GROUP);
@@ -526,6 +529,19 @@ __device__ __forceinline__ void mma_tf32(uint32_t d, uint64_t a, uint64_t b, uin
 __device__ __forceinline__ void mma_commit(uint32_t mbar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(mbar) : "memory");
 }
+// 32 consecutive TMEM columns of this thread's lane; tmem_ld32_nw leaves the wait to the caller
+// (tmem_wait_ld) so several loads can be in flight.
+#define TMEM_LD32_ASM(taddr, r)                                                                                   \
+  asm volatile(                                                                                                 \
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"           \
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"                                \
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]), \
+        "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]),    \
+        "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),   \
+        "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])                 \
+      : "r"(taddr))
+__device__ __forceinline__ void tmem_ld32_nw(uint32_t taddr, uint32_t* r) { TMEM_LD32_ASM(taddr, r); }
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
   uint32_t r[32];
   asm volatile(
@@ -650,15 +666,23 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
       *reinterpret_cast<float4*>(hi + off) = h;
       *reinterpret_cast<float4*>(lo + off) = l;
     };
-    // prologue: stages 0 .. S-2 (fresh barriers: the empty waits pass at once)
+    // prologue: stages 0 .. L-1 with L = S-2 loads in flight ahead of the stage being split; a refill
+    // targets the stage the MMA released two steps earlier (never the one just handed to it)
+    constexpr int L = S - 2;
 #pragma unroll 1
-    for (int kt = 0; kt < S - 1; kt++) {
+    for (int kt = 0; kt < L; kt++) {
       if (kt < nk) issue(kt);
       cp_commit();
     }
 #pragma unroll 1
     for (int kt = 0; kt < nk; kt++) {
-      cp_wait<S - 2>();                                  // this thread's copies for stage kt landed
+      const int nxt = kt + L;
+      if (nxt < nk) {
+        if (nxt >= S) mbar_wait(empty0 + 8 * (nxt % S), ((uint32_t)(nxt / S) & 1u) ^ 1u);
+        issue(nxt);
+      }
+      cp_commit();
+      cp_wait<L>();                                      // this thread's copies for stage kt landed
       const int s = kt % S;
       unsigned char* st = smem + s * Cfg::STAGE_BYTES;
 #pragma unroll
@@ -670,13 +694,6 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // generic-proxy writes -> tensor core
       mbar_arrive(full0 + 8 * s);
-      const int nxt = kt + S - 1;
-      if (nxt < nk) {
-        const int sn = nxt % S;
-        mbar_wait(empty0 + 8 * sn, ((uint32_t)(nxt / S) & 1u) ^ 1u);   // MMA finished reading it
-        issue(nxt);
-      }
-      cp_commit();
     }
   } else if (warp == NPROD / 32 && lane == 0) {
     // ---------------- MMA issuer (one thread)
@@ -765,6 +782,289 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, L
 }
 
 }  // namespace tc
+
+// ---------------------------------------------------------------- multi-tile tcgen05 kernel
+// Streaming GEMMs (M >> 128 with modest K and N: MobileNetV2's 1x1 convs and their data gradients
+// at batch 96, ResNet's 1x1 convs) are HBM-bound, and a one-tile CTA spends most of its life in
+// setup, pipeline fill and a serial epilogue. Here a CTA owns TPC consecutive output tiles (a
+// shape-only count) with two TMEM accumulator buffers, so the epilogue of tile i (dedicated warps
+// 0-3: TMEM -> registers -> per-warp padded staging -> coalesced 128-bit stores) runs while the
+// producers (warps 4-11: cp.async -> in-place 3xTF32 hi/lo split) and the MMA thread (warp 12) work
+// on tile i+1, with 6-8 operand stages in flight. A CTA lives for TPC tiles only: no whole-GPU persistent grid,
+// so an HP kernel's CTAs find a free SM within a few microseconds (kernels are not preemptible,
+// P:670-689). Each tile is computed by one CTA in fixed k order: results do not depend on which
+// CTA or SM runs it. Accumulators: one chain for hi*hi, one for the two correction products.
+namespace tcm {
+using namespace tc;
+constexpr int BM = 128, BK = 16, NPROD = 256, NTHR = 416;   // 4 epilogue + 8 producer + 1 MMA warps
+constexpr int MMA_WARP = 4 + NPROD / 32;
+constexpr int EPI_LD = 36;                                   // padded staging row (floats): conflict-free
+constexpr int EPI_BYTES = 4 * 32 * EPI_LD * 4;
+// BN = 64 or 128 output columns per tile; one CTA per SM with STAGES deep enough to keep ~80 KB of
+// operand loads in flight per SM (an HBM-bound stream needs latency x bandwidth / #SM bytes).
+template <int BN_>
+struct Cfg {
+  static constexpr int BN = BN_;
+  static constexpr int A_BYTES = BM * BK * 4, B_BYTES = BN * BK * 4, STAGE_BYTES = 2 * (A_BYTES + B_BYTES);
+  // RAW_STAGES landing slots (raw fp32, cp.async) feed STAGES split slots (hi/lo, read by the MMA):
+  // ~100 KB of loads in flight per SM for HBM-bound streams.
+  static constexpr int RAW_BYTES = A_BYTES + B_BYTES;
+  static constexpr int RAW_STAGES = BN == 64 ? 10 : 8, STAGES = BN == 64 ? 3 : 2;
+  static constexpr int SMEM = RAW_STAGES * RAW_BYTES + STAGES * STAGE_BYTES + EPI_BYTES + 256 + 1024;
+  static constexpr int TMEM_COLS = 4 * BN;                   // 2 buffers x (main, corr)
+  static constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+};
+
+struct Params { int M, N, K; float* C; long long ldc; const float* bias; int tiles_n, tiles, tpc, dbg; };
+
+template <int BN_, class LA, class LB>
+__global__ void __launch_bounds__(NTHR, 1) gemm_tcm_kernel(Params p, LA la, LB lb, OrionSig sig) {
+  using C_ = Cfg<BN_>;
+  constexpr int BN = C_::BN, A_BYTES = C_::A_BYTES, B_BYTES = C_::B_BYTES, STAGE_BYTES = C_::STAGE_BYTES, STAGES = C_::STAGES;
+  constexpr int RAW_BYTES = C_::RAW_BYTES, RAW_STAGES = C_::RAW_STAGES;
+  constexpr int TMEM_COLS = C_::TMEM_COLS;
+  constexpr uint32_t IDESC = C_::IDESC;
+  extern __shared__ __align__(1024) unsigned char smem_raw[];
+  unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  unsigned char* raw = smem + STAGES * STAGE_BYTES;
+  float* epi = reinterpret_cast<float*>(raw + RAW_STAGES * RAW_BYTES);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(raw + RAW_STAGES * RAW_BYTES + EPI_BYTES);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 4);
+  const uint32_t full0 = smem_u32(bars), empty0 = full0 + 8 * STAGES, tfull0 = empty0 + 8 * STAGES, tempty0 = tfull0 + 16;
+  const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
+  const int t0 = blockIdx.x * p.tpc;
+  const int ntl = min(p.tpc, p.tiles - t0);
+  const int nk = (p.K + BK - 1) / BK;
+  const int G = ntl * nk;   // (tile, k-tile) steps of this CTA
+
+  if (tid == 0) {
+    for (int s = 0; s < STAGES; s++) { mbar_init(full0 + 8 * s, NPROD); mbar_init(empty0 + 8 * s, 1); }
+    for (int b = 0; b < 2; b++) { mbar_init(tfull0 + 8 * b, 1); mbar_init(tempty0 + 8 * b, 4); }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == MMA_WARP) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)), "r"(TMEM_COLS) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp >= 4 && warp < MMA_WARP) {
+    // ---------------- producers: thread pt stages the quads idx = pt + 128 j with row = 8 (idx / 32)
+    // + idx % 8 and quad = (idx / 8) % 4: a warp instruction covers 8 rows x 4 quads (whole 64-byte
+    // row pieces, coalesced), and the 8 threads of each shared-memory phase hit 8 rows of one core
+    // matrix column (16 B apart in the K-major layout): conflict-free.
+    const int pt = tid - 128;
+    auto row_of = [](int idx) { return ((idx >> 5) << 3) | (idx & 7); };
+    auto quad_of = [](int idx) { return (idx >> 3) & 3; };
+    auto issue = [&](int g) {
+      const int t = t0 + g / nk, kt = g % nk;
+      const int m0 = (t / p.tiles_n) * BM, n0 = (t % p.tiles_n) * BN;
+      const uint32_t st = smem_u32(raw + (g % RAW_STAGES) * RAW_BYTES);
+      const uint32_t a_hi = st, b_hi = st + A_BYTES;
+      const int k0 = kt * BK;
+      const auto ta = la.tile(k0, p.K, BK);
+      const auto tb = lb.tile(k0, p.K, BK);
+#pragma unroll
+      for (int j = 0; j < BM * 4 / NPROD; j++) {
+        const int idx = pt + NPROD * j, row = row_of(idx), q = quad_of(idx);
+        const typename LA::Row ar = la.row(m0 + row, p.M);
+        const uint32_t dst = a_hi + elem_off(row, q, BM);
+        const float* src;
+        if (la.quad(ar, ta, q, p.K, src)) cp_async16(dst, src);
+        else {
+#pragma unroll
+          for (int e = 0; e < 4; e++) cp_async4(dst + 4 * e, la.addr(ar, k0 + 4 * q + e, p.K));
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < BN * 4 / NPROD; j++) {
+        const int idx = pt + NPROD * j, row = row_of(idx), q = quad_of(idx);
+        const typename LB::Col bc = lb.col(n0 + row, p.N);
+        const uint32_t dst = b_hi + elem_off(row, q, BN);
+        const float* src;
+        if (lb.quad(bc, tb, q, p.K, src)) cp_async16(dst, src);
+        else {
+#pragma unroll
+          for (int e = 0; e < 4; e++) cp_async4(dst + 4 * e, lb.addr(bc, k0 + 4 * q + e, p.K));
+        }
+      }
+    };
+    auto split = [](const unsigned char* src, unsigned char* hi, unsigned char* lo, uint32_t off) {
+      float4 v = *reinterpret_cast<const float4*>(src + off), h, l;
+      h.x = tf32_rna(v.x); h.y = tf32_rna(v.y); h.z = tf32_rna(v.z); h.w = tf32_rna(v.w);
+      l.x = v.x - h.x; l.y = v.y - h.y; l.z = v.z - h.z; l.w = v.w - h.w;
+      *reinterpret_cast<float4*>(hi + off) = h;
+      *reinterpret_cast<float4*>(lo + off) = l;
+    };
+    // Each thread splits exactly the quads it copied, so a raw slot is free for this thread's next
+    // copy as soon as its own split of that slot is done (program order): L = RAW_STAGES - 1 steps of
+    // loads in flight without any cross-thread wait; only the split slots wait for the MMA.
+    constexpr int L = RAW_STAGES - 1;
+#pragma unroll 1
+    for (int g = 0; g < L; g++) {
+      if (g < G) issue(g);
+      cp_commit();
+    }
+#pragma unroll 1
+    for (int g = 0; g < G; g++) {
+      if (g + L < G && !(p.dbg & 2)) issue(g + L);
+      cp_commit();
+      cp_wait<L>();                                   // this thread's copies for step g landed
+      const int s = g % STAGES;
+      if (g >= STAGES) mbar_wait(empty0 + 8 * s, ((uint32_t)(g / STAGES) & 1u) ^ 1u);   // MMA released slot s
+      const unsigned char* rw = raw + (g % RAW_STAGES) * RAW_BYTES;
+      unsigned char* st = smem + s * STAGE_BYTES;
+#pragma unroll
+      for (int j = 0; j < BM * 4 / NPROD; j++) {
+        const int idx = pt + NPROD * j;
+        split(rw, st, st + A_BYTES, elem_off(row_of(idx), quad_of(idx), BM));
+      }
+#pragma unroll
+      for (int j = 0; j < BN * 4 / NPROD; j++) {
+        const int idx = pt + NPROD * j;
+        split(rw + A_BYTES, st + 2 * A_BYTES, st + 2 * A_BYTES + B_BYTES, elem_off(row_of(idx), quad_of(idx), BN));
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      mbar_arrive(full0 + 8 * s);
+    }
+  } else if (warp == MMA_WARP && lane == 0) {
+    // ---------------- MMA issuer
+#pragma unroll 1
+    for (int g = 0; g < G; g++) {
+      const int i = g / nk, kt = g % nk, buf = i & 1;
+      if (kt == 0) {
+        mbar_wait(tempty0 + 8 * buf, ((uint32_t)(i >> 1) & 1u) ^ 1u);   // epilogue drained this buffer
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      }
+      const int s = g % STAGES;
+      mbar_wait(full0 + 8 * s, (uint32_t)(g / STAGES) & 1u);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      const uint32_t st = smem_u32(smem + s * STAGE_BYTES);
+      const uint32_t a_hi = st, a_lo = st + A_BYTES, b_hi = st + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
+      const uint32_t d_main = tmem + (uint32_t)(buf * 2 * BN), d_corr = d_main + BN;
+#pragma unroll
+      for (int j = 0; j < BK / 8; j++) {
+        const uint64_t dah = sdesc(a_hi + j * BM * 32, 128, 256), dal = sdesc(a_lo + j * BM * 32, 128, 256);
+        const uint64_t dbh = sdesc(b_hi + j * BN * 32, 128, 256), dbl = sdesc(b_lo + j * BN * 32, 128, 256);
+        mma_tf32(d_corr, dal, dbh, IDESC, (kt | j) != 0);
+        mma_tf32(d_corr, dah, dbl, IDESC, 1);
+        mma_tf32(d_main, dah, dbh, IDESC, (kt | j) != 0);
+      }
+      mma_commit(empty0 + 8 * s);
+      if (kt == nk - 1) mma_commit(tfull0 + 8 * buf);
+    }
+  } else if (warp < 4) {
+    // ---------------- epilogue: warp w owns tile rows 32w..32w+31 (TMEM lanes)
+    float* stg = epi + warp * 32 * EPI_LD;
+    const bool vec = ((p.ldc & 3) == 0) && ((reinterpret_cast<uintptr_t>(p.C) & 15) == 0);
+    const int rr = lane >> 3, cq = (lane & 7) * 4;
+#pragma unroll 1
+    for (int i = 0; i < ntl; i++) {
+      const int buf = i & 1, t = t0 + i;
+      const int m0 = (t / p.tiles_n) * BM, n0 = (t % p.tiles_n) * BN;
+      mbar_wait(tfull0 + 8 * buf, (uint32_t)(i >> 1) & 1u);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+#pragma unroll 1
+      for (int c0 = 0; c0 < BN && n0 + c0 < p.N && !(p.dbg & 4); c0 += 32) {
+        uint32_t mv[32], cv[32];
+        const uint32_t base = tmem + ((uint32_t)(32 * warp) << 16) + (uint32_t)(buf * 2 * BN + c0);
+        tmem_ld32_nw(base, mv);
+        tmem_ld32_nw(base + BN, cv);
+        tmem_wait_ld();
+#pragma unroll
+        for (int j = 0; j < 32; j += 4)
+          *reinterpret_cast<float4*>(stg + lane * EPI_LD + j) =
+              make_float4(__uint_as_float(mv[j]) + __uint_as_float(cv[j]), __uint_as_float(mv[j + 1]) + __uint_as_float(cv[j + 1]),
+                          __uint_as_float(mv[j + 2]) + __uint_as_float(cv[j + 2]), __uint_as_float(mv[j + 3]) + __uint_as_float(cv[j + 3]));
+        __syncwarp();
+        // all 8 staged rows into distinct registers first, then the 8 stores: a store's source
+        // registers are not recycled by the next load (no serialisation on store data read-out)
+        float4 vv[8];
+#pragma unroll
+        for (int it = 0; it < 8; it++) vv[it] = *reinterpret_cast<const float4*>(stg + (it * 4 + rr) * EPI_LD + cq);
+#pragma unroll
+        for (int it = 0; it < 8; it++) {
+          const int r = it * 4 + rr;
+          const int m = m0 + 32 * warp + r, n = n0 + c0 + cq;
+          if (m < p.M && n < p.N && !(p.dbg & 1)) {
+            float4 v = vv[it];
+            float* dst = p.C + (long long)m * p.ldc + n;
+            if (vec && n + 3 < p.N) {
+              if (p.bias) { v.x += __ldg(p.bias + n); v.y += __ldg(p.bias + n + 1); v.z += __ldg(p.bias + n + 2); v.w += __ldg(p.bias + n + 3); }
+              *reinterpret_cast<float4*>(dst) = v;
+            } else {
+              const float tv[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+              for (int e = 0; e < 4; e++)
+                if (n + e < p.N) dst[e] = tv[e] + (p.bias ? __ldg(p.bias + n + e) : 0.f);
+            }
+          }
+        }
+        __syncwarp();
+      }
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(tempty0 + 8 * buf);
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == MMA_WARP) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS) : "memory");
+  }
+  orion_signal(sig);
+}
+
+// Shape-only plan: the kernel takes streaming shapes with enough tiles to fill the part's 148 SMs
+// without a K split; BN = 128 when N > 64 (A read once for N <= 128); a CTA's tile count targets
+// ~4 waves (<= 16 tiles, so a CTA lives a few microseconds).
+inline int bn_for(long long N) { return N > 64 ? 128 : 64; }
+inline long long tiles_of(long long M, long long N) { return cdiv(M, BM) * cdiv(N, bn_for(N)); }
+inline bool ok(long long M, long long N, long long K) { return K >= 8 && K <= 2048 && tiles_of(M, N) >= 2 * 148; }
+inline int tpc_of(long long tiles) {
+  long long t = cdiv(tiles, 148 * 4);
+  return (int)(t < 1 ? 1 : t > 16 ? 16 : t);
+}
+template <int BN, class LA, class LB>
+bool prepare() {
+  static std::atomic<int> done{0};
+  if (done.load(std::memory_order_acquire)) return true;
+  bool okk = cudaFuncSetAttribute((const void*)gemm_tcm_kernel<BN, LA, LB>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<BN>::SMEM) ==
+             cudaSuccess;
+  if (okk) done.store(1, std::memory_order_release);
+  return okk;
+}
+template <class LA, class LB>
+void geom(LaunchGeom* g, long long M, long long N) {
+  const long long tiles = tiles_of(M, N);
+  g->grid = dim3((unsigned)cdiv(tiles, tpc_of(tiles))); g->block = dim3(NTHR);
+  if (bn_for(N) == 128) { prepare<128, LA, LB>(); g->smem = Cfg<128>::SMEM; g->func = (const void*)gemm_tcm_kernel<128, LA, LB>; }
+  else { prepare<64, LA, LB>(); g->smem = Cfg<64>::SMEM; g->func = (const void*)gemm_tcm_kernel<64, LA, LB>; }
+}
+template <class LA, class LB>
+bool is(const void* f) { return f == (const void*)gemm_tcm_kernel<128, LA, LB> || f == (const void*)gemm_tcm_kernel<64, LA, LB>; }
+template <class LA, class LB>
+int launch(const LaunchGeom& g, long long M, long long N, long long K, float* C, long long ldc, const float* bias, LA la, LB lb,
+           OrionSig sig, cudaStream_t s) {
+  Params p;
+  p.M = (int)M; p.N = (int)N; p.K = (int)K; p.C = C; p.ldc = ldc; p.bias = bias;
+  p.tiles_n = (int)cdiv(N, bn_for(N)); p.tiles = (int)tiles_of(M, N); p.tpc = tpc_of(p.tiles);
+  static const int dbg = getenv("ORION_TCM_DEBUG") ? atoi(getenv("ORION_TCM_DEBUG")) : 0;   // 1 no stores, 2 no loads, 4 no epilogue
+  p.dbg = dbg;
+  if (bn_for(N) == 128) {
+    if (!prepare<128, LA, LB>()) return ORION_E_CUDA;
+    gemm_tcm_kernel<128, LA, LB><<<g.grid, g.block, g.smem, s>>>(p, la, lb, sig);
+  } else {
+    if (!prepare<64, LA, LB>()) return ORION_E_CUDA;
+    gemm_tcm_kernel<64, LA, LB><<<g.grid, g.block, g.smem, s>>>(p, la, lb, sig);
+  }
+  return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+}
+}  // namespace tcm
 
 // ---------------------------------------------------------------- skinny A^T B (weight gradients)
 // C[M][N] = sum_k A[k][m] B[k][n] for M, N <= 128 and very long K (1x1-conv weight gradients over
@@ -1148,7 +1448,7 @@ Plan plan_gemm(long long M, long long N, long long K) {
     split = cdiv(target, tiles);
     long long kmax = K / (4 * pl.bk);         // >= 4 k-tiles per split
     if (split > kmax) split = kmax;
-    if (split > 1008) split = 1008;                 // two-level reduction: <= 63 groups of 16
+    if (split > 1008) split = 1008;                 // two-level reduction: <= 32 groups of <= 32
     if (split < 1) split = 1;
   }
   pl.split = (int)split;
@@ -1158,7 +1458,7 @@ Plan plan_gemm(long long M, long long N, long long K) {
 uint64_t ws_bytes_for(const Plan& pl, long long M, long long N) {
   if (pl.split <= 1) return 0;
   uint64_t parts = (uint64_t)pl.split;
-  if (pl.split > SPLIT_FLAT_MAX) parts += (uint64_t)((pl.split + SPLIT_GROUP - 1) / SPLIT_GROUP);   // group partials
+  parts += (uint64_t)split_groups(pl.split);   // group partials
   return WS_TICKET_BYTES + parts * M * N * 4;
 }
 
@@ -1308,6 +1608,11 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     g->grid = dim3((unsigned)cdiv(N, 8)); g->block = dim3(256); g->smem = 0; g->func = (const void*)gemv_bt_kernel;
     return 0;
   }
+  if ((flags == 0 || flags == 2) && tcm::ok(M, N, K)) {   // streaming shapes: multi-tile tcgen05 kernel
+    if (flags == 2) tcm::geom<ADense, BDenseT>(g, M, N);
+    else tcm::geom<ADense, BDense>(g, M, N);
+    return 0;
+  }
   if ((flags == 0 || flags == 2) && M >= 4096 && N <= 32 && K * ((N + 3) & ~3) <= rows::MAXKN) {
     const void* f = flags == 2 ? (const void*)rows::gemm_rows_kernel<true> : (const void*)rows::gemm_rows_kernel<false>;
     static std::atomic<int> attr{0};
@@ -1364,6 +1669,10 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
     gemv_bt_kernel<<<g.grid, g.block, 0, s>>>(A, lda, B, ldb, C, ldc, bias, (int)M, (int)N, (int)K, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
+  if (tcm::is<ADense, BDenseT>(g.func))
+    return tcm::launch(g, M, N, K, C, ldc, bias, ADense{A, lda}, BDenseT{B, ldb}, sig, s);
+  if (tcm::is<ADense, BDense>(g.func))
+    return tcm::launch(g, M, N, K, C, ldc, bias, ADense{A, lda}, BDense{B, ldb}, sig, s);
   if (g.func == (const void*)rows::gemm_rows_kernel<true> || g.func == (const void*)rows::gemm_rows_kernel<false>) {
     if (flags == 2)
       rows::gemm_rows_kernel<true><<<g.grid, g.block, g.smem, s>>>(A, lda, B, ldb, C, ldc, bias, (int)M, (int)N, (int)K, sig);

@@ -43,7 +43,10 @@ def ws(nbytes):
                                          (4704, 1280, 320, 2), (1280, 320, 4704, 1), (18816, 96, 576, 2),
                                          (99, 37, 9999, 1), (24, 144, 75264, 1), (128, 32, 300000, 1),
                                          (12544, 16, 96, 0), (20000, 24, 144, 2), (5000, 7, 33, 0), (4097, 32, 512, 2),
-                                         (144, 24, 75264, 1), (192, 32, 75264, 1), (32, 192, 75264, 1), (150, 22, 5000, 1)],
+                                         (144, 24, 75264, 1), (192, 32, 75264, 1), (32, 192, 75264, 1), (150, 22, 5000, 1),
+                                         # multi-tile tcgen05 kernel (>= 296 tiles): ragged M / N / K, unaligned K
+                                         (40000, 96, 16, 2), (30000, 144, 20, 0), (20000, 200, 40, 2), (40000, 64, 33, 2),
+                                         (301056, 24, 144, 0), (38000, 33, 24, 0), (18816, 384, 64, 2), (4704, 1280, 320, 0)],
                          ids=lambda v: str(v))
 def test_gemm_shapes(M, N, K, flags):
     test_gemm(M, N, K, flags)

@@ -23,6 +23,17 @@ def run(M, N, K, flags, reps=10):
     print(f"M={M:6d} N={N:5d} K={K:6d} fl={flags} grid={grid:5d} thr={thr} smem={smem:6d}  {t*1e6:9.1f} us  {2*M*N*K/t/1e12:7.2f} TF/s")
 
 torch.cuda.set_device(0)
-for shp in [(128, 64, 64, 2), (128, 64, 1024, 2), (128, 128, 4096, 2), (256, 128, 1024, 2), (4096, 4096, 4096, 2), (8192, 1024, 2048, 2), (2048, 2048, 8192, 0), (196, 512, 4608, 2), (784, 256, 2304, 2), (3136, 128, 1152, 2),
-            (4704, 1280, 320, 2), (1280, 320, 4704, 1), (12544, 64, 576, 2)]:
-    run(*shp)
+SHAPES = {
+    "generic": [(4096, 4096, 4096, 2), (8192, 1024, 2048, 2), (196, 512, 4608, 2), (784, 256, 2304, 2), (3136, 128, 1152, 2),
+                (4704, 1280, 320, 2), (1280, 320, 4704, 1), (12544, 64, 576, 2)],
+    # MobileNetV2 b96 1x1 convs: fwd (flags 2: x [M][Cin] . W[Cout][Cin]^T) and dgrad (flags 0: dy [M][Cout] . W[Cout][Cin])
+    "dbg": [(1204224, 96, 16, 2), (1204224, 16, 96, 0), (4704, 1280, 320, 2)],
+    "mnv2": [(1204224, 16, 32, 2), (1204224, 96, 16, 2), (301056, 24, 96, 2), (301056, 144, 24, 2), (301056, 24, 144, 2),
+             (75264, 32, 144, 2), (75264, 192, 32, 2), (75264, 32, 192, 2), (18816, 384, 64, 2), (18816, 64, 384, 2),
+             (18816, 576, 96, 2), (4704, 960, 160, 2), (4704, 160, 960, 2), (4704, 1280, 320, 2),
+             (1204224, 32, 16, 0), (1204224, 16, 96, 0), (301056, 96, 24, 0), (301056, 24, 144, 0), (75264, 144, 32, 0),
+             (75264, 32, 192, 0), (18816, 64, 384, 0), (4704, 160, 960, 0), (4704, 320, 1280, 0)],
+}
+for name in (sys.argv[1:] or ["generic", "mnv2"]):
+    for shp in SHAPES[name]:
+        run(*shp)
