@@ -9,6 +9,8 @@
 #include <atomic>
 #include <cstdlib>
 
+#include <cuda.h>
+
 #include "common.cuh"
 
 namespace {
@@ -498,7 +500,19 @@ __device__ __forceinline__ bool mbar_try(uint32_t a, uint32_t parity) {
                : "=r"(ok) : "r"(a), "r"(parity) : "memory");
   return ok != 0;
 }
-__device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity) { while (!mbar_try(a, parity)) {} }
+__device__ __forceinline__ bool mbar_test(uint32_t a, uint32_t parity) {
+  uint32_t ok;
+  asm volatile("{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+               : "=r"(ok) : "r"(a), "r"(parity) : "memory");
+  return ok != 0;
+}
+#ifndef ORION_MBAR_SPIN
+#define ORION_MBAR_SPIN 0
+#endif
+__device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity) {
+  if (ORION_MBAR_SPIN) { while (!mbar_test(a, parity)) {} }
+  else { while (!mbar_try(a, parity)) {} }
+}
 __device__ __forceinline__ void cp_async16(uint32_t dst, const float* src) {
   // zero-fill when src == nullptr (src-size 0 reads nothing; the address operand must still be valid)
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(src ? src : reinterpret_cast<const float*>(&cp_async16)),
@@ -1066,6 +1080,321 @@ int launch(const LaunchGeom& g, long long M, long long N, long long K, float* C,
 }
 }  // namespace tcm
 
+// ---------------------------------------------------------------- TMA-fed multi-tile tcgen05 kernel
+// The dense streaming case (row-major A with K % 4 == 0: 1x1-conv forward and data gradient), fed
+// and drained by the Tensor Memory Accelerator. A 2-D tensor map with 128-byte swizzle lands a
+// BM x 32 tile directly in the UMMA K-major SWIZZLE_128B layout, so the raw fp32 tile IS the "hi"
+// operand: the tensor core reads tf32 by truncating the low 13 mantissa bits (measured,
+// tools/probe/tma_tf32.cu). Converter warps only form lo = x - trunc_tf32(x) (exact in fp32) at
+// the same offsets; D += A_lo B_hi + A_hi B_lo + A_hi B_hi (dropped A_lo B_lo < 2^-20 |ab|). B given
+// [K][N] (data gradient: W) lands as [32][BN] and the converters transpose it into the K-major
+// layout (hi and lo). The epilogue stages 32 x 32 blocks in 128B-swizzled shared memory (conflict
+// free) and stores them with TMA (double-buffered per warp), so no thread waits on global stores.
+// Roles: warps 0-3 epilogue (TMEM lanes), 4-7 converters, warp 8 lane 0 TMA producer, warp 9 lane 0
+// MMA issuer and TMEM owner. Each tile is computed by one CTA in fixed k order (deterministic).
+namespace tmk {
+using namespace tc;
+constexpr int BM = 128, BK = 32, NCONV = 128, NTHR = 320, CONV_WARPS = NCONV / 32;
+constexpr int TMA_WARP = 4 + CONV_WARPS, MMA_WARP = TMA_WARP + 1;
+constexpr int EPI_BUF = 32 * 32 * 4, EPI_BYTES = 4 * 2 * EPI_BUF;   // per warp: 2 staging blocks of 32 x 32
+template <int BN_, bool BMN_>
+struct Cfg {
+  static constexpr int BN = BN_;
+  static constexpr int A_BYTES = BM * BK * 4, B_BYTES = BN * BK * 4;
+  // stage: [A hi (TMA)][A lo][B hi][B lo][B raw (MN-major B only)]
+  static constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES + (BMN_ ? B_BYTES : 0);
+  static constexpr int STAGES = (194 * 1024) / STAGE_BYTES;
+  static constexpr int SMEM = STAGES * STAGE_BYTES + EPI_BYTES + 256 + 1024;
+  static constexpr int TMEM_COLS = 4 * BN;
+  static constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+  static constexpr uint32_t TX_BYTES = A_BYTES + B_BYTES;
+};
+struct Params { int M, N, K; const float* bias; int tiles_n, tiles, tpc; };
+
+__device__ __forceinline__ void tma2d(uint32_t dst, const CUtensorMap* tm, int c0, int c1, uint32_t bar) {
+  asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(dst), "l"(tm),
+               "r"(c0), "r"(c1), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void tma2d_store(const CUtensorMap* tm, int c0, int c1, uint32_t src) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(tm), "r"(c0), "r"(c1), "r"(src) : "memory");
+}
+__device__ __forceinline__ void mbar_expect(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ float trunc_tf32(float x) { return __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
+__device__ __forceinline__ float4 lo4(const float4 v) {
+  return make_float4(v.x - trunc_tf32(v.x), v.y - trunc_tf32(v.y), v.z - trunc_tf32(v.z), v.w - trunc_tf32(v.w));
+}
+// UMMA descriptor, K-major SWIZZLE_128B: 8-row atoms of 128-byte rows (32 tf32), SBO = 1024 B between
+// atoms, LBO unused; layout type 2 at bits 61-63; k-step j advances the start address by 32 B.
+__device__ __forceinline__ uint64_t sdesc128(uint32_t addr) {
+  return (uint64_t)((addr >> 4) & 0x3FFF) | (1ull << 16) | ((uint64_t)(1024 >> 4) << 32) | (1ull << 46) | (2ull << 61);
+}
+// byte offset of element (row, col < 32) of a 32-float-wide SWIZZLE_128B tile (what TMA writes / reads)
+__device__ __forceinline__ uint32_t sw128_off(int row, int col) {
+  return (uint32_t)((row >> 3) * 1024 + (row & 7) * 128 + (((col >> 2) ^ (row & 7)) << 4) + (col & 3) * 4);
+}
+
+template <int BN_, bool BMN>
+__global__ void __launch_bounds__(NTHR, 1) gemm_tmk_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                                                          const __grid_constant__ CUtensorMap tmC, Params p, OrionSig sig) {
+  using C_ = Cfg<BN_, BMN>;
+  constexpr int BN = C_::BN, A_BYTES = C_::A_BYTES, B_BYTES = C_::B_BYTES, STAGE_BYTES = C_::STAGE_BYTES, STAGES = C_::STAGES;
+  extern __shared__ __align__(1024) unsigned char smem_raw[];
+  unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  unsigned char* epi = smem + STAGES * STAGE_BYTES;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(epi + EPI_BYTES);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 3 * STAGES + 4);
+  const uint32_t tfull0 = smem_u32(bars), cfull0 = tfull0 + 8 * STAGES, empty0 = cfull0 + 8 * STAGES;
+  const uint32_t afull0 = empty0 + 8 * STAGES, aempty0 = afull0 + 16;   // TMEM accumulator buffers
+  const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
+  const int t0 = blockIdx.x * p.tpc;
+  const int ntl = min(p.tpc, p.tiles - t0);
+  const int nk = (p.K + BK - 1) / BK;
+  const int G = ntl * nk;
+
+  if (tid == 0) {
+    for (int s = 0; s < STAGES; s++) { mbar_init(tfull0 + 8 * s, 1); mbar_init(cfull0 + 8 * s, CONV_WARPS); mbar_init(empty0 + 8 * s, 1); }
+    for (int b = 0; b < 2; b++) { mbar_init(afull0 + 8 * b, 1); mbar_init(aempty0 + 8 * b, 4); }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == TMA_WARP && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmB) : "memory");
+  }
+  if (warp == 0 && lane == 0) asm volatile("prefetch.tensormap [%0];" ::"l"(&tmC) : "memory");
+  if (warp == MMA_WARP) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)), "r"(C_::TMEM_COLS) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == TMA_WARP) {
+    if (lane == 0) {
+#pragma unroll 1
+      for (int g = 0; g < G; g++) {
+        const int s = g % STAGES;
+        if (g >= STAGES) mbar_wait(empty0 + 8 * s, ((uint32_t)(g / STAGES) & 1u) ^ 1u);
+        const int t = t0 + g / nk, kt = g % nk;
+        const int m0 = (t / p.tiles_n) * BM, n0 = (t % p.tiles_n) * BN;
+        const uint32_t st = smem_u32(smem + s * STAGE_BYTES), bar = tfull0 + 8 * s;
+        mbar_expect(bar, C_::TX_BYTES);
+        tma2d(st, &tmA, kt * BK, m0, bar);
+        if (BMN) tma2d(st + 2 * A_BYTES + 2 * B_BYTES, &tmB, n0, kt * BK, bar);
+        else tma2d(st + 2 * A_BYTES, &tmB, kt * BK, n0, bar);
+      }
+    }
+  } else if (warp >= 4 && warp < TMA_WARP) {
+    // ---------------- converters: lo = x - trunc(x) for A (and B); B transposed when MN-major
+    const int ct = tid - 128;
+#pragma unroll 1
+    for (int g = 0; g < G; g++) {
+      const int s = g % STAGES;
+      mbar_wait(tfull0 + 8 * s, (uint32_t)(g / STAGES) & 1u);
+      unsigned char* st = smem + s * STAGE_BYTES;
+      const float4* ahi = reinterpret_cast<const float4*>(st);
+      float4* alo = reinterpret_cast<float4*>(st + A_BYTES);
+      constexpr int AQ = A_BYTES / 16 / NCONV;
+      float4 va[AQ];
+#pragma unroll
+      for (int j = 0; j < AQ; j++) va[j] = ahi[ct + NCONV * j];
+#pragma unroll
+      for (int j = 0; j < AQ; j++) alo[ct + NCONV * j] = lo4(va[j]);
+      constexpr int BQ = B_BYTES / 16 / NCONV;
+      if (!BMN) {
+        const float4* bhi = reinterpret_cast<const float4*>(st + 2 * A_BYTES);
+        float4* blo = reinterpret_cast<float4*>(st + 2 * A_BYTES + B_BYTES);
+        float4 vb[BQ];
+#pragma unroll
+        for (int j = 0; j < BQ; j++) vb[j] = bhi[ct + NCONV * j];
+#pragma unroll
+        for (int j = 0; j < BQ; j++) blo[ct + NCONV * j] = lo4(vb[j]);
+      } else {
+        // raw [32 k][BN n] -> K-major SWIZZLE_128B (n, k): thread item = (row n, k-quad kq); reads are
+        // consecutive n across lanes, writes one 16-byte chunk per row (swizzle spreads 8 rows over 8 chunks)
+        const float* braw = reinterpret_cast<const float*>(st + 2 * A_BYTES + 2 * B_BYTES);
+        unsigned char* bhi = st + 2 * A_BYTES;
+        unsigned char* blo = st + 2 * A_BYTES + B_BYTES;
+#pragma unroll
+        for (int j = 0; j < BQ; j++) {
+          const int idx = ct + NCONV * j;
+          const int n = idx % BN, kq = idx / BN;
+          const float4 v = make_float4(braw[(4 * kq) * BN + n], braw[(4 * kq + 1) * BN + n], braw[(4 * kq + 2) * BN + n], braw[(4 * kq + 3) * BN + n]);
+          const uint32_t off = sw128_off(n, 4 * kq);
+          *reinterpret_cast<float4*>(bhi + off) = make_float4(trunc_tf32(v.x), trunc_tf32(v.y), trunc_tf32(v.z), trunc_tf32(v.w));
+          *reinterpret_cast<float4*>(blo + off) = lo4(v);
+        }
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(cfull0 + 8 * s);
+    }
+  } else if (warp == MMA_WARP && lane == 0) {
+#pragma unroll 1
+    for (int g = 0; g < G; g++) {
+      const int i = g / nk, kt = g % nk, buf = i & 1;
+      if (kt == 0) {
+        mbar_wait(aempty0 + 8 * buf, ((uint32_t)(i >> 1) & 1u) ^ 1u);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      }
+      const int s = g % STAGES;
+      mbar_wait(tfull0 + 8 * s, (uint32_t)(g / STAGES) & 1u);
+      mbar_wait(cfull0 + 8 * s, (uint32_t)(g / STAGES) & 1u);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+      const uint32_t st = smem_u32(smem + s * STAGE_BYTES);
+      const uint32_t a_hi = st, a_lo = st + A_BYTES, b_hi = st + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
+      const uint32_t d_main = tmem + (uint32_t)(buf * 2 * BN), d_corr = d_main + BN;
+#pragma unroll
+      for (int j = 0; j < BK / 8; j++) {
+        const uint64_t dah = sdesc128(a_hi + 32 * j), dal = sdesc128(a_lo + 32 * j);
+        const uint64_t dbh = sdesc128(b_hi + 32 * j), dbl = sdesc128(b_lo + 32 * j);
+        mma_tf32(d_corr, dal, dbh, C_::IDESC, (kt | j) != 0);
+        mma_tf32(d_corr, dah, dbl, C_::IDESC, 1);
+        mma_tf32(d_main, dah, dbh, C_::IDESC, (kt | j) != 0);
+      }
+      mma_commit(empty0 + 8 * s);
+      if (kt == nk - 1) mma_commit(afull0 + 8 * buf);
+    }
+  } else if (warp < 4) {
+    // ---------------- epilogue: warp w owns tile rows 32w..32w+31 (TMEM lanes); per 32-column chunk:
+    // TMEM -> registers (+ bias) -> swizzled staging block -> TMA store (lane 0), two blocks in flight
+    unsigned char* stg0 = epi + warp * 2 * EPI_BUF;
+    int nst = 0;   // stores issued by this warp
+#pragma unroll 1
+    for (int i = 0; i < ntl; i++) {
+      const int buf = i & 1, t = t0 + i;
+      const int m0 = (t / p.tiles_n) * BM, n0 = (t % p.tiles_n) * BN;
+      mbar_wait(afull0 + 8 * buf, (uint32_t)(i >> 1) & 1u);
+      asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+#pragma unroll 1
+      for (int c0 = 0; c0 < BN && n0 + c0 < p.N; c0 += 32) {
+        uint32_t mv[32], cv[32];
+        const uint32_t base = tmem + ((uint32_t)(32 * warp) << 16) + (uint32_t)(buf * 2 * BN + c0);
+        tmem_ld32_nw(base, mv);
+        tmem_ld32_nw(base + BN, cv);
+        unsigned char* stg = stg0 + (nst & 1) * EPI_BUF;
+        if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");   // this block's previous store read it
+        tmem_wait_ld();
+        __syncwarp();
+#pragma unroll
+        for (int j = 0; j < 32; j += 4) {
+          float4 v = make_float4(__uint_as_float(mv[j]) + __uint_as_float(cv[j]), __uint_as_float(mv[j + 1]) + __uint_as_float(cv[j + 1]),
+                                 __uint_as_float(mv[j + 2]) + __uint_as_float(cv[j + 2]), __uint_as_float(mv[j + 3]) + __uint_as_float(cv[j + 3]));
+          if (p.bias) {
+            const int n = n0 + c0 + j;
+            if (n < p.N) v.x += __ldg(p.bias + n);
+            if (n + 1 < p.N) v.y += __ldg(p.bias + n + 1);
+            if (n + 2 < p.N) v.z += __ldg(p.bias + n + 2);
+            if (n + 3 < p.N) v.w += __ldg(p.bias + n + 3);
+          }
+          *reinterpret_cast<float4*>(stg + sw128_off(lane, j)) = v;
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        __syncwarp();
+        if (lane == 0) {
+          tma2d_store(&tmC, n0 + c0, m0 + 32 * warp, smem_u32(stg));
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+        nst++;
+      }
+      asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(aempty0 + 8 * buf);
+    }
+    if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");   // all of this warp's stores complete
+    __syncwarp();
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == MMA_WARP) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(C_::TMEM_COLS) : "memory");
+  }
+  orion_signal(sig);
+}
+
+// cuTensorMapEncodeTiled, resolved through cudart at first use (the library does not link libcuda)
+typedef CUresult (*encode_fn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                              const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+inline encode_fn encoder() {
+  static encode_fn fn = [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPointByVersion("cuTensorMapEncodeTiled", &p, 12000, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return (encode_fn) nullptr;
+    return (encode_fn)p;
+  }();
+  return fn;
+}
+// 2-D fp32 map of a row-major [rows][ld] array with `inner` columns, box {box_inner, box_rows}
+inline bool map2d(CUtensorMap* m, const float* base, long long rows, long long inner, long long ld, int box_inner, int box_rows,
+                  CUtensorMapSwizzle sw) {
+  cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
+  cuuint32_t box[2] = {(cuuint32_t)box_inner, (cuuint32_t)box_rows};
+  cuuint32_t es[2] = {1, 1};
+  return encoder()(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)base, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+inline bool al16p(const void* q) { return (reinterpret_cast<uintptr_t>(q) & 15) == 0; }
+// dense row-major A [M][lda] (K contiguous); B^T [N][ldb] (bmn = false) or B [K][ldb] (bmn = true); C [M][ldc]
+inline bool ok(long long M, long long N, long long K, long long lda, long long ldb, long long ldc, const float* A, const float* B,
+               const float* C) {
+  return tcm::ok(M, N, K) && K % 4 == 0 && lda % 4 == 0 && ldb % 4 == 0 && ldc % 4 == 0 && al16p(A) && al16p(B) && al16p(C) &&
+         encoder() != nullptr;
+}
+template <int BN, bool BMN>
+bool prepare() {
+  static std::atomic<int> done{0};
+  if (done.load(std::memory_order_acquire)) return true;
+  bool okk = cudaFuncSetAttribute((const void*)gemm_tmk_kernel<BN, BMN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<BN, BMN>::SMEM) ==
+             cudaSuccess;
+  if (okk) done.store(1, std::memory_order_release);
+  return okk;
+}
+template <int BN, bool BMN>
+void geom_t(LaunchGeom* g, long long tiles) {
+  prepare<BN, BMN>();
+  g->grid = dim3((unsigned)cdiv(tiles, tcm::tpc_of(tiles))); g->block = dim3(NTHR); g->smem = Cfg<BN, BMN>::SMEM;
+  g->func = (const void*)gemm_tmk_kernel<BN, BMN>;
+}
+inline void geom(LaunchGeom* g, long long M, long long N, bool bmn) {
+  const long long tiles = tcm::tiles_of(M, N);
+  if (tcm::bn_for(N) == 128) { if (bmn) geom_t<128, true>(g, tiles); else geom_t<128, false>(g, tiles); }
+  else { if (bmn) geom_t<64, true>(g, tiles); else geom_t<64, false>(g, tiles); }
+}
+inline bool is(const void* f) {
+  return f == (const void*)gemm_tmk_kernel<128, true> || f == (const void*)gemm_tmk_kernel<128, false> ||
+         f == (const void*)gemm_tmk_kernel<64, true> || f == (const void*)gemm_tmk_kernel<64, false>;
+}
+template <int BN, bool BMN>
+int launch_t(const LaunchGeom& g, const Params& p, const float* A, long long lda, const float* B, long long ldb, float* C, long long ldc,
+             OrionSig sig, cudaStream_t s) {
+  if (!prepare<BN, BMN>()) return ORION_E_CUDA;
+  CUtensorMap ma, mb, mc;
+  if (!map2d(&ma, A, p.M, p.K, lda, BK, BM, CU_TENSOR_MAP_SWIZZLE_128B)) return ORION_E_CUDA;
+  if (BMN ? !map2d(&mb, B, p.K, p.N, ldb, BN, BK, CU_TENSOR_MAP_SWIZZLE_NONE) : !map2d(&mb, B, p.N, p.K, ldb, BK, BN, CU_TENSOR_MAP_SWIZZLE_128B))
+    return ORION_E_CUDA;
+  if (!map2d(&mc, C, p.M, p.N, ldc, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B)) return ORION_E_CUDA;
+  gemm_tmk_kernel<BN, BMN><<<g.grid, g.block, g.smem, s>>>(ma, mb, mc, p, sig);
+  return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+}
+inline int launch(const LaunchGeom& g, long long M, long long N, long long K, float* C, long long ldc, const float* bias, const float* A,
+                  long long lda, const float* B, long long ldb, bool bmn, OrionSig sig, cudaStream_t s) {
+  Params p;
+  p.M = (int)M; p.N = (int)N; p.K = (int)K; p.bias = bias;
+  p.tiles_n = (int)cdiv(N, tcm::bn_for(N)); p.tiles = (int)tcm::tiles_of(M, N); p.tpc = tcm::tpc_of(p.tiles);
+  if (tcm::bn_for(N) == 128)
+    return bmn ? launch_t<128, true>(g, p, A, lda, B, ldb, C, ldc, sig, s) : launch_t<128, false>(g, p, A, lda, B, ldb, C, ldc, sig, s);
+  return bmn ? launch_t<64, true>(g, p, A, lda, B, ldb, C, ldc, sig, s) : launch_t<64, false>(g, p, A, lda, B, ldb, C, ldc, sig, s);
+}
+}  // namespace tmk
+
+
 // ---------------------------------------------------------------- skinny A^T B (weight gradients)
 // C[M][N] = sum_k A[k][m] B[k][n] for M, N <= 128 and very long K (1x1-conv weight gradients over
 // N*H*W rows): HBM-bound, so the kernel streams 64-row blocks of both operands with coalesced
@@ -1608,6 +1937,11 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     g->grid = dim3((unsigned)cdiv(N, 8)); g->block = dim3(256); g->smem = 0; g->func = (const void*)gemv_bt_kernel;
     return 0;
   }
+  if ((flags == 0 || flags == 2) &&
+      tmk::ok(M, N, K, (long long)a[7], (long long)a[8], (long long)a[9], (const float*)a[0], (const float*)a[1], (const float*)a[2])) {
+    tmk::geom(g, M, N, flags == 0);   // streaming shapes, TMA-fed
+    return 0;
+  }
   if ((flags == 0 || flags == 2) && tcm::ok(M, N, K)) {   // streaming shapes: multi-tile tcgen05 kernel
     if (flags == 2) tcm::geom<ADense, BDenseT>(g, M, N);
     else tcm::geom<ADense, BDense>(g, M, N);
@@ -1669,6 +2003,7 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
     gemv_bt_kernel<<<g.grid, g.block, 0, s>>>(A, lda, B, ldb, C, ldc, bias, (int)M, (int)N, (int)K, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
+  if (tmk::is(g.func)) return tmk::launch(g, M, N, K, C, ldc, bias, A, lda, B, ldb, flags == 0, sig, s);
   if (tcm::is<ADense, BDenseT>(g.func))
     return tcm::launch(g, M, N, K, C, ldc, bias, ADense{A, lda}, BDenseT{B, ldb}, sig, s);
   if (tcm::is<ADense, BDense>(g.func))

@@ -27,7 +27,7 @@ SHAPES = {
     "generic": [(4096, 4096, 4096, 2), (8192, 1024, 2048, 2), (196, 512, 4608, 2), (784, 256, 2304, 2), (3136, 128, 1152, 2),
                 (4704, 1280, 320, 2), (1280, 320, 4704, 1), (12544, 64, 576, 2)],
     # MobileNetV2 b96 1x1 convs: fwd (flags 2: x [M][Cin] . W[Cout][Cin]^T) and dgrad (flags 0: dy [M][Cout] . W[Cout][Cin])
-    "dbg": [(1204224, 96, 16, 2), (1204224, 16, 96, 0), (4704, 1280, 320, 2)],
+    "dbg": [(1204224, 96, 16, 2), (301056, 24, 144, 2), (1204224, 16, 96, 0), (4704, 1280, 320, 2)],
     "mnv2": [(1204224, 16, 32, 2), (1204224, 96, 16, 2), (301056, 24, 96, 2), (301056, 144, 24, 2), (301056, 24, 144, 2),
              (75264, 32, 144, 2), (75264, 192, 32, 2), (75264, 32, 192, 2), (18816, 384, 64, 2), (18816, 64, 384, 2),
              (18816, 576, 96, 2), (4704, 960, 160, 2), (4704, 160, 960, 2), (4704, 1280, 320, 2),
