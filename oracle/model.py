@@ -390,6 +390,214 @@ def mnv2_train_step(P, V, x, labels, first, lr=0.01, momentum=0.9, eps=1e-5, bn_
     return loss, newP, newV, g
 
 
+# ------------------------------------------------------------------- max-pool backward
+def maxpool3x3s2_bwd(x, dy):
+    """Backward of MaxPool2d(3, 2, 1): each output's gradient goes to the first maximum of its
+    window in row-major (u, v) order; contributions to one input add up. NHWC."""
+    xd, dyd = _d(x), _d(dy)
+    n, h, w, c = x.shape
+    p, q = dy.shape[1], dy.shape[2]
+    xp = torch.full((n, h + 2, w + 2, c), -math.inf, dtype=F64)
+    xp[:, 1:h + 1, 1:w + 1, :] = xd
+    best = torch.full((n, p, q, c), -math.inf, dtype=F64)
+    arg = torch.zeros((n, p, q, c), dtype=torch.long)
+    for u in range(3):
+        for v in range(3):
+            win = xp[:, u:u + 2 * p:2, v:v + 2 * q:2, :][:, :p, :q, :]
+            take = win > best                       # strict: the first maximum wins ties
+            best = torch.where(take, win, best)
+            arg = torch.where(take, torch.full_like(arg, u * 3 + v), arg)
+    dxp = torch.zeros((n, h + 2, w + 2, c), dtype=F64)
+    for u in range(3):
+        for v in range(3):
+            sel = torch.where(arg == u * 3 + v, dyd, torch.zeros((), dtype=F64))
+            dxp[:, u:u + 2 * p:2, v:v + 2 * q:2, :][:, :p, :q, :] += sel
+    return _r(dxp[:, 1:h + 1, 1:w + 1, :])
+
+
+# -------------------------------------------------------------------- ResNet training
+def resnet_train_step(P, V, x, labels, first, layers=RESNET50_LAYERS, lr=0.01, momentum=0.9, eps=1e-5,
+                      bn_momentum=0.1, masks=None):
+    """One training iteration of TorchVision ResNet v1.5 (train-mode BN, CE, SGD momentum), the
+    BE client of BASELINE config 3 (ResNet-50, batch 64) and HP of config 4 (ResNet-101).
+    Ops in PyTorch eager order, each rounded to fp32 (R22-R24). masks (optional): {name: fp32
+    tensor} of the values the GPU's ReLU backward decides on (its BN / residual-sum outputs), as in
+    mnv2_train_step. Returns (loss, newP, newV, grads)."""
+    newP = dict(P)
+    g = {}
+
+    def cb(h, cname, bname, stride, pad):
+        z = conv2d_fwd(h, P[f"{cname}.w"], stride, pad)
+        y, mean, invstd, rm, rv = bn_train_fwd(z, P[f"{bname}.gamma"], P[f"{bname}.beta"],
+                                               P[f"{bname}.rmean"], P[f"{bname}.rvar"], eps, bn_momentum)
+        newP[f"{bname}.rmean"], newP[f"{bname}.rvar"] = rm, rv
+        return y, (cname, bname, stride, pad, h, z, mean, invstd)
+
+    def cb_bwd(rec, dy, need_dx=True):
+        cname, bname, stride, pad, hin, z, mean, invstd = rec
+        dz, g[f"{bname}.gamma"], g[f"{bname}.beta"] = bn_bwd(z, dy, P[f"{bname}.gamma"], mean, invstd)
+        w = P[f"{cname}.w"]
+        g[f"{cname}.w"] = conv2d_bwd_weight(hin, dz, tuple(w.shape), stride, pad)
+        return conv2d_bwd_data(dz, w, tuple(hin.shape), stride, pad) if need_dx else None
+
+    def m(name, val):
+        return masks[name] if masks is not None else val
+
+    # ---- forward
+    y, stem = cb(x, "conv1", "bn1", 2, 3)
+    a = relu(y)
+    mp = maxpool3x3s2(a)
+    h = mp
+    blocks = []
+    for li, (w, nb, stride) in enumerate(layers):
+        for bi in range(nb):
+            p = f"layer{li + 1}.{bi}"
+            s = stride if bi == 0 else 1
+            y1, r1 = cb(h, f"{p}.conv1", f"{p}.bn1", 1, 0)
+            a1 = relu(y1)
+            y2, r2 = cb(a1, f"{p}.conv2", f"{p}.bn2", s, 1)
+            a2 = relu(y2)
+            y3, r3 = cb(a2, f"{p}.conv3", f"{p}.bn3", 1, 0)
+            if bi == 0:
+                idn, rd = cb(h, f"{p}.down", f"{p}.downbn", s, 0)
+            else:
+                idn, rd = h, None
+            sm = add(y3, idn)
+            out = relu(sm)
+            blocks.append((p, r1, y1, r2, y2, r3, rd, sm))
+            h = out
+    feat_shape = tuple(h.shape)
+    pooled = avgpool_fwd(h)
+    logits = linear_fwd(pooled, P["fc.w"], P["fc.b"])
+    loss, dlogits = ce_fwd_bwd(logits, labels)
+
+    # ---- backward (reverse op order)
+    dpooled, g["fc.w"], g["fc.b"] = linear_bwd(pooled, P["fc.w"], dlogits)
+    dh = avgpool_bwd(dpooled, feat_shape)
+    for p, r1, y1, r2, y2, r3, rd, sm in reversed(blocks):
+        dsm = relu_bwd(m(f"{p}.sum", sm), dh)
+        d = cb_bwd(r3, dsm)
+        d = relu_bwd(m(f"{p}.bn2", y2), d)
+        d = cb_bwd(r2, d)
+        d = relu_bwd(m(f"{p}.bn1", y1), d)
+        d = cb_bwd(r1, d)
+        didn = cb_bwd(rd, dsm) if rd is not None else dsm
+        dh = add(d, didn)
+    da = maxpool3x3s2_bwd(a, dh)
+    dy = relu_bwd(m("bn1", y), da)
+    cb_bwd(stem, dy, need_dx=False)
+
+    newV = {}
+    for n in sorted(g):
+        newP[n], newV[n] = sgd(P[n], g[n], V.get(n), lr, momentum, first)
+    return loss, newP, newV, g
+
+
+def resnet_train_spec(layers=RESNET50_LAYERS, num_classes=1000):
+    """Training ResNet: BN running stats start at torch's defaults (mean 0, var 1)."""
+    return resnet_spec(layers, num_classes, eval_stats=False)
+
+
+# ============================================================================ BERT (bf16)
+# HP of BASELINE config 3: BERT-base inference, batch 8, sequence 128, bf16 (HuggingFace
+# BertModel as PyTorch eager runs it with the model cast to bfloat16; readings R22, R29-R31 in
+# DESIGN.md §3). Every op computes in float64 from its bf16 inputs and rounds its output once to
+# bf16 (round-to-nearest-even), as the unfused GPU op stream materialises it. `store` selects the
+# storage dtype so the pins can run the same code unrounded (float64) against HF's fp64 model.
+BF16 = torch.bfloat16
+
+
+def _s(t, store):
+    return t.to(store)
+
+
+def bert_spec(layers=12, hidden=768, heads=12, ffn=3072, vocab=30522, max_pos=512, types=2):
+    """Parameter spec (names, shapes, init). Linear weights [out, in]. Init (reading R22): every
+    weight, embedding and bias N(0, 0.02); LayerNorm gamma U[0.9, 1.1], beta N(0, 0.02) (non-zero
+    biases / non-unit gammas so that every term of every op is exercised)."""
+    n = ("normal", 0.02)
+    s = [("emb.word", (vocab, hidden), n), ("emb.pos", (max_pos, hidden), n), ("emb.type", (types, hidden), n),
+         ("emb.ln.gamma", (hidden,), ("uniform", 0.9, 1.1)), ("emb.ln.beta", (hidden,), n)]
+    for i in range(layers):
+        p = f"layer{i}"
+        for nm, o, k in (("q", hidden, hidden), ("k", hidden, hidden), ("v", hidden, hidden), ("o", hidden, hidden),
+                         ("ffn1", ffn, hidden), ("ffn2", hidden, ffn)):
+            s += [(f"{p}.{nm}.w", (o, k), n), (f"{p}.{nm}.b", (o,), n)]
+        for ln in ("ln1", "ln2"):
+            s += [(f"{p}.{ln}.gamma", (hidden,), ("uniform", 0.9, 1.1)), (f"{p}.{ln}.beta", (hidden,), n)]
+    return s
+
+
+def bert_embed(ids, word, pos, typ, store=BF16):
+    """embeddings = word[ids] + type[0] + pos[s] (token type 0 everywhere, no padding: R22),
+    summed in fp64 and rounded once. ids [B, S] -> [B, S, H]."""
+    b, sq = ids.shape
+    e = _d(word)[ids.long()] + _d(typ)[0] + _d(pos)[:sq][None, :, :]
+    return _s(e, store)
+
+
+def layernorm(x, gamma, beta, eps=1e-12, store=BF16):
+    """LayerNorm over the last dim: (x - mean) / sqrt(var + eps) * gamma + beta, biased var."""
+    xd = _d(x)
+    mean = xd.mean(-1, keepdim=True)
+    var = ((xd - mean) ** 2).mean(-1, keepdim=True)
+    return _s((xd - mean) / torch.sqrt(var + eps) * _d(gamma) + _d(beta), store)
+
+
+def linear_any(x, w, b, store=BF16):
+    """y = x W^T + b over the last dim, fp64 accumulation, one rounding."""
+    return _s(_d(x) @ _d(w).t() + _d(b), store)
+
+
+def gelu(x, store=BF16):
+    """GELU, exact erf form: 0.5 x (1 + erf(x / sqrt 2)) (HF "gelu")."""
+    xd = _d(x)
+    return _s(0.5 * xd * (1.0 + torch.erf(xd / math.sqrt(2.0))), store)
+
+
+def add_any(a, b, store=BF16):
+    return _s(_d(a) + _d(b), store)
+
+
+def attention(q, k, v, heads, store=BF16):
+    """Multi-head scaled dot-product attention without mask (R22): per batch b and head h,
+    O = softmax(Q K^T / sqrt(d)) V with Q, K, V the head's d = H/heads columns of [B, S, H].
+    One op (the fused SDPA kernel PyTorch dispatches), fp64 inside, one rounding of O."""
+    b, sq, hd = q.shape
+    d = hd // heads
+    Q = _d(q).view(b, sq, heads, d).permute(0, 2, 1, 3)
+    K = _d(k).view(b, sq, heads, d).permute(0, 2, 1, 3)
+    Vv = _d(v).view(b, sq, heads, d).permute(0, 2, 1, 3)
+    sc = Q @ K.transpose(-1, -2) / math.sqrt(d)
+    pr = torch.softmax(sc, dim=-1)
+    o = (pr @ Vv).permute(0, 2, 1, 3).reshape(b, sq, hd)
+    return _s(o, store)
+
+
+def bert_infer(P, ids, layers=12, heads=12, store=BF16):
+    """BertModel forward (no pooler): last hidden state [B, S, H] in `store`. P holds the
+    parameters already in the model dtype (bf16, or fp64 for the pins)."""
+    h = bert_embed(ids, P["emb.word"], P["emb.pos"], P["emb.type"], store)
+    h = layernorm(h, P["emb.ln.gamma"], P["emb.ln.beta"], store=store)
+    for i in range(layers):
+        p = f"layer{i}"
+        q = linear_any(h, P[f"{p}.q.w"], P[f"{p}.q.b"], store)
+        k = linear_any(h, P[f"{p}.k.w"], P[f"{p}.k.b"], store)
+        v = linear_any(h, P[f"{p}.v.w"], P[f"{p}.v.b"], store)
+        a = attention(q, k, v, heads, store)
+        o = linear_any(a, P[f"{p}.o.w"], P[f"{p}.o.b"], store)
+        h1 = layernorm(add_any(o, h, store), P[f"{p}.ln1.gamma"], P[f"{p}.ln1.beta"], store=store)
+        f = gelu(linear_any(h1, P[f"{p}.ffn1.w"], P[f"{p}.ffn1.b"], store), store)
+        f2 = linear_any(f, P[f"{p}.ffn2.w"], P[f"{p}.ffn2.b"], store)
+        h = layernorm(add_any(f2, h1, store), P[f"{p}.ln2.gamma"], P[f"{p}.ln2.beta"], store=store)
+    return h
+
+
+def to_model_dtype(P, dtype=BF16):
+    """Cast drawn parameters to the model dtype (model.to(torch.bfloat16))."""
+    return {k: v.to(dtype) for k, v in P.items()}
+
+
 # ------------------------------------------------------------------------- small helpers
 def count_flops_conv(n, ho, wo, cout, k, cin_g):
     return 2 * n * ho * wo * cout * k * k * cin_g

@@ -66,3 +66,9 @@ def poisson_arrivals_ns(rate_rps, n, seed=ARRIVAL_SEED, gpu_index=0):
 
 def uniform_arrivals_ns(rate_rps, n):
     return (np.arange(1, n + 1) * (1e9 / rate_rps)).astype(np.int64)
+
+
+def token_ids(shape, vocab, seed, sub=0):
+    """Token ids U[0, vocab) as int32 (BERT inputs; token type 0, no padding: reading R22)."""
+    g = _gen(seed * 1_000_003 + 15_485_863 * (sub + 1))
+    return torch.randint(0, vocab, shape, generator=g, dtype=torch.int64).to(torch.int32)
