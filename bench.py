@@ -55,6 +55,18 @@ def build_config(name, rank):
                     cfg={"workload": "toy: HP MLP 3x512 fp32 inference b1 + BE MLP training b32",
                          "hp_model": "mlp3x512", "hp_batch": 1, "be_model": "mlp3x512", "be_batch": 32,
                          "arrivals": "poisson 1000 rps"})
+    if name == "bert_rn50":
+        Pb = si.make_params(W.bert_spec())
+        hp_inputs = [si.token_ids((8, 128), 30522, si.HP_SEED, sub=r).reshape(-1).view(torch.float32) for r in range(16)]
+        hpg = W.bert_infer_graph(Pb, batch=8, seq=128)
+        Prn = si.make_params(W.resnet_train_spec())
+        xs = [si.normal((64, 224, 224, 3), si.BE_SEED, sub=i) for i in range(8)]
+        labels = [si.labels(64, 1000, si.BE_SEED, sub=i) for i in range(8)]
+        beg = W.resnet_train_graph(Prn, xs, labels)
+        return dict(hpg=hpg, beg=beg, hp_inputs=hp_inputs, rate=4.0, be_inputs=xs, dtype="bf16 (HP) + f32 (BE)",
+                    cfg={"workload": "HP BERT-base inference b8 s128 bf16 (Poisson 4 rps) + BE ResNet-50 training b64, 1 B200 per instance",
+                         "hp_model": "bert-base", "hp_batch": 8, "seq_len": 128, "be_model": "resnet50", "be_batch": 64,
+                         "image": "224x224x3 NHWC fp32", "arrivals": "poisson 4 rps (PAPER Table 3 BERT)"})
     Prn = si.make_params(W.resnet_spec())
     hp_inputs = [si.normal((4, 224, 224, 3), si.HP_SEED, sub=r) for r in range(16)]
     hpg = W.resnet_infer_graph(Prn, batch=4)
@@ -78,6 +90,11 @@ def build_client(name, client):
             return W.mlp_infer_graph(P, batch=1)
         return W.mlp_train_graph(P, [si.normal((32, 512), si.BE_SEED, sub=i) for i in range(8)],
                                  [si.normal((32, 512), si.BE_SEED, sub=100 + i) for i in range(8)])
+    if name == "bert_rn50":
+        if client == "hp":
+            return W.bert_infer_graph(si.make_params(W.bert_spec()), batch=8, seq=128)
+        return W.resnet_train_graph(si.make_params(W.resnet_train_spec()), [si.normal((64, 224, 224, 3), si.BE_SEED, sub=0)],
+                                    [si.labels(64, 1000, si.BE_SEED, sub=0)])
     if client == "hp":
         return W.resnet_infer_graph(si.make_params(W.resnet_spec()), batch=4)
     return W.mnv2_train_graph(si.make_params(W.mnv2_spec()), [si.normal((96, 224, 224, 3), si.BE_SEED, sub=0)],
@@ -167,6 +184,18 @@ def cpu_oracle_sample(cfg_name, budget_s=15.0):
             n += 1
         dt = time.time() - t0
         return n / dt, f"{n} full MLP b32 training iterations (fp64 oracle)", cores
+    if cfg_name == "bert_rn50":
+        P = si.make_params(om.resnet_train_spec())
+        b = 2
+        x, lab = si.normal((b, 224, 224, 3), si.BE_SEED), si.labels(b, 1000, si.BE_SEED)
+        n, t0, V = 0, time.time(), {}
+        while True:
+            _, P, V, _ = om.resnet_train_step(P, V, x, lab, first=(n == 0))
+            n += 1
+            if time.time() - t0 > budget_s:
+                break
+        dt = time.time() - t0
+        return n / dt * b / 64.0, f"{n} ResNet-50 training iterations at batch {b} (224x224, fp64 oracle), scaled x{b}/64 to batch 64", cores
     P = si.make_params(om.mnv2_spec())
     b = 2
     x, lab = si.normal((b, 224, 224, 3), si.BE_SEED), si.labels(b, 1000, si.BE_SEED)
@@ -188,7 +217,7 @@ def main():
     ap.add_argument("--steps", type=int, default=300, help="HP requests timed under collocation")
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="orion", choices=["orion", "reference"])
-    ap.add_argument("--config", default="rn50_mnv2", choices=["rn50_mnv2", "toy"])
+    ap.add_argument("--config", default="rn50_mnv2", choices=["rn50_mnv2", "toy", "bert_rn50"])
     ap.add_argument("--dur-ppm", type=int, default=25000)
     ap.add_argument("--be-partition", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
@@ -294,6 +323,15 @@ def main():
         avg_s = float(np.mean(tr)) / 1e3
         if top_row["cls"] == "M":
             achieved, peak, unit, bound = nbytes / avg_s / 1e9, pk["hbm_gbs"], "GB/s", "hbm"
+        elif top_row["fn"] in ("gemm_bf16", "attention", "gemm", "conv_fwd", "conv_dgrad", "conv_wgrad"):
+            # timed inside a long collocated window: the sustained bf16 figure (B200_PROFILING.md)
+            tpk = pk.get("bf16_tflops_sustained", pk["bf16_tflops"])
+            if top_row["fn"] in ("gemm_bf16", "attention"):
+                achieved, peak, unit, bound = flops / avg_s / 1e12, tpk, "TFLOP/s", "tensor"
+            else:
+                # 3xTF32 on tcgen05: tf32 dense = bf16 x the guide's nominal 1/2, three MMAs per fp32
+                # product -> algorithmic fp32 peak = bf16 / 6
+                achieved, peak, unit, bound = flops / avg_s / 1e12, tpk / 6.0, "TFLOP/s", "tensor"
         else:
             achieved, peak, unit, bound = flops / avg_s / 1e12, FFMA_TFLOPS, "TFLOP/s", "alu"
     else:
@@ -342,11 +380,12 @@ def main():
     ms_per_step = agg["ms_per_step"]
     line = {
         "metric": metric, "value": value, "unit": "it/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "dtype": W_.get("dtype", "f32"),
         "data": "synthetic (seeded; DESIGN.md §5)",
         "config": dict(W_["cfg"], parallelism=f"replicas x{world} (independent Orion instance per GPU)",
                        hp_rate_rps=rate, dur_threshold_pct=args.dur_ppm / 1e4, be_partition_sms=args.be_partition,
-                       l2="inputs > L2 (BE batch 57.8 MB x 8 staged; no flush)"),
+                       l2=f"inputs > L2 (BE batch {W_['be_inputs'][0].numel() * 4 / 1e6:.1f} MB x 8 staged; no flush)"),
         "hp": {"p50_ms": col["p50_ns"] / 1e6, "p99_ms": col["p99_ns"] / 1e6, "dedicated_p50_ms": ded["p50_ns"] / 1e6,
                "dedicated_p99_ms": ded["p99_ns"] / 1e6, "p99_vs_dedicated": col["p99_ns"] / ded["p99_ns"],
                "p50_vs_dedicated": col["p50_ns"] / ded["p50_ns"], "solo_latency_ms": hp_lat_ns / 1e6,

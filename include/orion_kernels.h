@@ -83,7 +83,33 @@ enum orion_fn {
   /* Softmax cross entropy (mean over batch) and dz = (softmax - onehot)/B.
      args: z, labels(int32), loss (1 float), dz, B, classes */
   ORION_FN_CE = 23,
-  ORION_FN_COUNT = 24
+  /* ---- bf16 transformer operators (HP of BASELINE config 3: BERT-base inference as PyTorch
+     eager runs a bfloat16 HuggingFace BertModel; readings R22, R29-R31). bf16 tensors
+     are row-major, 16-byte aligned; arithmetic is fp32, each output rounded once (RNE).
+     Linear: y[M,N] = x[M,K] W[N,K]^T + b[N] on tcgen05 (kind::f16, fp32 TMEM accumulator).
+     args: x, W, y, b (0 = none), M, N, K. K % 8 == 0 (else ORION_E_INVAL). */
+  ORION_FN_GEMM_BF16 = 24,
+  /* Scaled dot-product attention without mask, one op: per batch b and head h,
+     O = softmax(Q K^T / sqrt(d)) V over the head's d columns. q, k, v, o: [B, S, ld] with head h at
+     columns h*d .. h*d+d-1. args: q, k, v, o, B, S, heads, d, ld. d == 64, S in {16, 32, 64, 128},
+     ld % 8 == 0 (else ORION_E_INVAL). P is rounded to bf16 before P V (flash-style). */
+  ORION_FN_ATTENTION = 25,
+  /* LayerNorm over the last dim (biased variance): y = (x - mean) / sqrt(var + eps) * gamma + beta.
+     args: x, y, gamma, beta, rows, C, eps_bits. C % 8 == 0, C <= 2048. */
+  ORION_FN_LAYERNORM = 26,
+  /* GELU, erf form: y = 0.5 x (1 + erf(x / sqrt 2)). args: x, y, n (n % 8 == 0) */
+  ORION_FN_GELU = 27,
+  /* bf16 residual add c = a + b. args: a, b, c, n (n % 8 == 0) */
+  ORION_FN_ADD_BF16 = 28,
+  /* Embedding sum: out[b, s, :] = word[ids[b, s]] + type[0] + pos[s] (token type 0, no padding).
+     args: ids (int32 [B*S]), word [vocab, H], pos [>= S, H], type [>= 1, H], out [B, S, H], B, S, H,
+     vocab. H % 8 == 0. Ids outside [0, vocab) are clamped into it. */
+  ORION_FN_EMBED = 29,
+  /* ---- fp32: MaxPool 3x3 / stride 2 / pad 1 backward. dx[n,h,w,c] = sum of dy over the windows
+     whose first maximum (row-major window order) is x[n,h,w,c]. args: x, dy, dx, N, H, W, C, P, Q.
+     C % 4 == 0; P, Q must be the forward's output size (else ORION_E_INVAL). */
+  ORION_FN_MAXPOOL_BWD = 30,
+  ORION_FN_COUNT = 31
 };
 
 /* Number of table entries, and a stable name for each (for profiles and logs). */

@@ -55,30 +55,35 @@ class BEClient:
 def run_session(hp=None, be=None, arrivals_ns=None, be_iters=0, log_capacity=0, hp_latency_ns=0,
                 dur_threshold_ppm=25000, sm_threshold=0, be_partition_sms=0, flags=0, sched_cpu=-1,
                 backend=L.BACKEND_CUDA, device=0, trace_kernel_id=None):
-    """Run one session. HP (if given) issues len(arrivals_ns) requests open loop; BE (if given) runs
-    closed loop until HP finishes (or be_iters iterations if HP is absent / be_iters > 0 and no HP).
+    """Run one session. HP (if given) issues len(arrivals_ns) requests open loop; BE (a client or a
+    list of clients, each on its own thread and stream) runs closed loop until HP finishes (or
+    be_iters iterations if HP is absent / be_iters > 0 and no HP).
     Returns dict with HP arrival/completion ns, BE iteration end times, window, log bytes, stats."""
     o = Orion(device=device, backend=backend, hp_latency_ns=hp_latency_ns, dur_threshold_ppm=dur_threshold_ppm,
               sm_threshold=sm_threshold, be_partition_sms=be_partition_sms, flags=flags, sched_cpu=sched_cpu,
               log_capacity=log_capacity, trace_kernel_id=trace_kernel_id)
+    # several BE clients (R11: one shared DUR budget, round robin) when `be` is a list
+    bes = [] if be is None else (list(be) if isinstance(be, (list, tuple)) else [be])
     hp_id = o.register_client(L.HP) if hp is not None else None
-    be_id = o.register_client(L.BE) if be is not None else None
+    be_ids = [o.register_client(L.BE) for _ in bes]
     torch.cuda.synchronize()
     o.start()
     res = {}
     stop = ctypes.c_int32(0)
-    th = None
-    if be is not None:
+    ths = []
+    if bes:
         max_iters = be_iters if (hp is None or be_iters) else 0
+        res["be_t_end_all"] = [None] * len(bes)
 
-        def be_main():
+        def be_main(j):
             try:
-                res["be_t_end"] = o.run_iterations(be_id, be.variants, stop_flag=stop, max_iters=max_iters)
+                res["be_t_end_all"][j] = o.run_iterations(be_ids[j], bes[j].variants, stop_flag=stop, max_iters=max_iters)
             except Exception as e:  # surfaced below
                 res["be_err"] = e
-        th = threading.Thread(target=be_main)
+        ths = [threading.Thread(target=be_main, args=(j,)) for j in range(len(bes))]
         res["t0"] = o_now = L.lib.orion_now_ns()
-        th.start()
+        for th in ths:
+            th.start()
     else:
         res["t0"] = o_now = L.lib.orion_now_ns()
     if hp is not None:
@@ -86,11 +91,13 @@ def run_session(hp=None, be=None, arrivals_ns=None, be_iters=0, log_capacity=0, 
         res["t_arrival"], res["t_done"] = ta, td
         res["t_hp_end"] = L.lib.orion_now_ns()
         stop.value = 1
-    if th is not None:
+    for th in ths:
         th.join()
-        if "be_err" in res:
-            o.stop()
-            raise res["be_err"]
+    if "be_err" in res:
+        o.stop()
+        raise res["be_err"]
+    if bes:
+        res["be_t_end"] = res["be_t_end_all"][0]
     res["t1"] = L.lib.orion_now_ns()
     o.stop()
     res["stats"] = o.stats()

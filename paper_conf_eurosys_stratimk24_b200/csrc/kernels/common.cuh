@@ -179,3 +179,10 @@ ENTRY_DECL(maxpool)
 ENTRY_DECL(avgpool)
 ENTRY_DECL(avgpool_bwd)
 ENTRY_DECL(ce)
+ENTRY_DECL(gemm_bf16)
+ENTRY_DECL(attention)
+ENTRY_DECL(layernorm)
+ENTRY_DECL(gelu)
+ENTRY_DECL(add_bf16)
+ENTRY_DECL(embed)
+ENTRY_DECL(maxpool_bwd)

@@ -27,6 +27,13 @@ const KernelEntry g_kernels[ORION_FN_COUNT] = {
     E(avgpool, avgpool, 5),
     E(avgpool_bwd, avgpool_bwd, 5),
     E(ce, ce, 7),
+    E(gemm_bf16, gemm_bf16, 7),
+    E(attention, attention, 9),
+    E(layernorm, layernorm, 7),
+    E(gelu, gelu, 3),
+    E(add_bf16, add_bf16, 4),
+    E(embed, embed, 9),
+    E(maxpool_bwd, maxpool_bwd, 9),
 };
 #undef E
 

@@ -24,6 +24,9 @@ from .runtime import kernel_launch, kernel_geometry
 HBM_GBS = 6554.2
 FFMA_TFLOPS = 148 * 128 * 2 * 1.965e9 / 1e12
 RIDGE_FFMA = FFMA_TFLOPS * 1e12 / (HBM_GBS * 1e9)   # flop per DRAM byte
+BF16_TFLOPS = 1669.2                                  # dense bf16 tensor pipe (MEASURED_PEAKS.json)
+RIDGE_BF16 = BF16_TFLOPS * 1e12 / (HBM_GBS * 1e9)
+TENSOR_OPS = ("gemm_bf16", "attention")               # ops on the bf16 tensor pipe: their own ridge
 
 
 def op_work(fn, a):
@@ -68,6 +71,25 @@ def op_work(fn, a):
         return 3 * a[3], (20 if a[5] else 12) * a[3]
     if f == "colsum":
         return a[2] * a[3], 4 * (a[2] * a[3] + a[3])
+    # bf16 transformer ops: 2 bytes per element
+    if f == "gemm_bf16":
+        M, N, K = a[4], a[5], a[6]
+        return 2 * M * N * K, 2 * (M * K + K * N + M * N + (N if a[3] else 0))
+    if f == "attention":
+        B, S, H, d = a[4], a[5], a[6], a[7]
+        return 4 * B * H * S * S * d + 5 * B * H * S * S, 2 * 4 * B * S * H * d
+    if f == "layernorm":
+        return 8 * a[4] * a[5], 2 * (2 * a[4] * a[5] + 2 * a[5])
+    if f == "gelu":
+        return 8 * a[2], 4 * a[2]
+    if f == "add_bf16":
+        return a[3], 6 * a[3]
+    if f == "embed":
+        B, S, H = a[5], a[6], a[7]
+        return 2 * B * S * H, 2 * (2 * B * S * H + S * H + H) + 4 * B * S
+    if f == "maxpool_bwd":
+        n, h, w, c, p, q = a[3:9]
+        return 9 * n * p * q * c, 4 * (2 * n * h * w * c + n * p * q * c)
     return 0, 0
 
 
@@ -138,11 +160,11 @@ def build_profiles(graph, kid_base=0, reps=10, ncu_csv=None):
             # arithmetic intensity over max(measured DRAM bytes, compulsory bytes): on B200 the 126 MB
             # L2 often holds an op's inputs, and DRAM bytes alone would call a memory-bound op
             # compute-bound (DESIGN.md §3 R16)
-            cls = classify(c, m, flops, max(dram, nbytes))
+            cls = classify(c, m, flops, max(dram, nbytes), RIDGE_BF16 if fn in TENSOR_OPS else RIDGE_FFMA)
             dur = int(ndur) if ndur > 0 else dur   # device time of the kernel alone
             src = "ncu"
         else:
-            cls = classify(None, None, flops, nbytes)
+            cls = classify(None, None, flops, nbytes, RIDGE_BF16 if fn in TENSOR_OPS else RIDGE_FFMA)
             src = "analytic"
         sm = sm_needed(fn, args)
         table[kid] = (cls, sm, dur)

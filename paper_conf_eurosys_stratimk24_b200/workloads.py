@@ -524,3 +524,266 @@ def mnv2_train_graph(host_params, xs, labels, lr=0.01, momentum=0.9, num_classes
     g.logits = logits
     g.bn_out = {L_["bname"]: L_["y"] for L_ in layers}   # BN outputs (ReLU6 inputs), for parity tests
     return g
+
+
+# ====================================================================== ResNet training (BE, config 3)
+def resnet_train_spec(layers=RESNET50_LAYERS, num_classes=1000):
+    """Training ResNet: BN running stats start at torch's defaults (mean 0, var 1)."""
+    spec = []
+    for n, s, init in resnet_spec(layers, num_classes):
+        if n.endswith(".rmean"):
+            init = ("const", 0.0)
+        elif n.endswith(".rvar"):
+            init = ("const", 1.0)
+        spec.append((n, s, init))
+    return spec
+
+
+def resnet_train_graph(host_params, xs, labels, layers=RESNET50_LAYERS, lr=0.01, momentum=0.9, num_classes=1000,
+                       device="cuda"):
+    """BE (config 3): one TorchVision ResNet v1.5 training iteration — conv, train-mode BN, ReLU,
+    residual add, max-pool, CE, SGD(momentum) — each op its own kernel, backward op by op in reverse
+    order. One op-list variant per pre-staged batch."""
+    g = Graph("resnet_train", device)
+    spec = resnet_train_spec(layers, num_classes)
+    trainable = {n for n, _, _ in spec if not n.endswith((".rmean", ".rvar"))}
+    P = FlatParams(g, spec, host_params, trainable=trainable, grads=True, momentum=True)
+    batch, hw = xs[0].shape[0], xs[0].shape[1]
+    xb = [g.buf(f"x{i}", tuple(x.shape)) for i, x in enumerate(xs)]
+    lb = [g.buf(f"lab{i}", (batch,), dtype=torch.int32) for i in range(len(xs))]
+    with torch.no_grad():
+        for d, s in zip(xb, xs):
+            d.copy_(s.to(d.device))
+        for d, s in zip(lb, labels):
+            d.copy_(s.to(d.device))
+    loss = g.buf("loss", (1,))
+    cnt = [0]
+
+    def new(shape):
+        cnt[0] += 1
+        return g.buf(f"t{cnt[0]}", shape)
+
+    def plan(cname, bname, in_shape, cout, k, stride, pad):
+        n, h, w, _ = in_shape
+        ho, wo = (h + 2 * pad - k) // stride + 1, (w + 2 * pad - k) // stride + 1
+        L_ = dict(cname=cname, bname=bname, stride=stride, pad=pad, cout=cout, in_shape=in_shape,
+                  z=new((n, ho, wo, cout)), y=new((n, ho, wo, cout)), mean=new((cout,)), invstd=new((cout,)),
+                  dz=new((n, ho, wo, cout)))
+        g.need_ws(L.lib.orion_bn_workspace_bytes(n * ho * wo, cout))
+        return L_
+
+    stem = plan("conv1", "bn1", (batch, hw, hw, 3), 64, 7, 2, 3)
+    s_shape = stem["y"].shape
+    a0, da0, dy0 = new(s_shape), new(s_shape), new(s_shape)
+    n_, h_, w_, c_ = s_shape
+    pq = (h_ + 2 - 3) // 2 + 1
+    mp = new((n_, pq, pq, c_))
+    shape = tuple(mp.shape)
+    blocks = []
+    cin = 64
+    for li, (wd, nb, stride) in enumerate(layers):
+        for bi in range(nb):
+            p = f"layer{li + 1}.{bi}"
+            s = stride if bi == 0 else 1
+            b = dict(name=p, in_shape=shape)
+            b["c1"] = plan(f"{p}.conv1", f"{p}.bn1", shape, wd, 1, 1, 0)
+            b["a1"], b["d1"] = new(b["c1"]["y"].shape), new(b["c1"]["y"].shape)
+            b["c2"] = plan(f"{p}.conv2", f"{p}.bn2", tuple(b["c1"]["y"].shape), wd, 3, s, 1)
+            b["a2"], b["d2"] = new(b["c2"]["y"].shape), new(b["c2"]["y"].shape)
+            b["c3"] = plan(f"{p}.conv3", f"{p}.bn3", tuple(b["c2"]["y"].shape), 4 * wd, 1, 1, 0)
+            b["down"] = plan(f"{p}.down", f"{p}.downbn", shape, 4 * wd, 1, s, 0) if bi == 0 else None
+            oshape = tuple(b["c3"]["y"].shape)
+            b["sum"], b["out"], b["dsum"] = new(oshape), new(oshape), new(oshape)
+            b["dmain"] = new(shape)
+            b["din"] = new(shape)          # gradient w.r.t. the block input
+            b["ddown"] = new(shape) if bi == 0 else None
+            b["da2"], b["da1"] = new(b["c2"]["y"].shape), new(b["c1"]["y"].shape)
+            blocks.append(b)
+            shape = oshape
+            cin = 4 * wd
+    n, hh, ww, c = shape
+    pooled, logits, dlogits, dpooled, dfeat = new((n, c)), new((n, num_classes)), new((n, num_classes)), new((n, c)), new(shape)
+    dmp = blocks[0]["din"]
+    g.need_ws(L.WS_TICKET_BYTES + 4 * batch)
+
+    def conv_bn(L_, h):
+        conv_fwd(g, h, P.p[f"{L_['cname']}.w"], L_["z"], L_["stride"], L_["pad"], L_["cname"])
+        rows = L_["z"].numel() // L_["cout"]
+        bn = L_["bname"]
+        g.k("bn_stats", [_p(L_["z"]), _p(L_["mean"]), _p(L_["invstd"]), _p(P.p[f"{bn}.rmean"]), _p(P.p[f"{bn}.rvar"]),
+                         rows, L_["cout"], EPS_BITS, f32bits(0.1), 0, 0], f"{bn}.stats", ws_at=9)
+        g.k("bn_apply", [_p(L_["z"]), _p(L_["y"]), _p(P.p[f"{bn}.gamma"]), _p(P.p[f"{bn}.beta"]), _p(L_["mean"]),
+                         _p(L_["invstd"]), rows, L_["cout"]], f"{bn}.apply")
+        L_["in"] = h
+        return L_["y"]
+
+    def conv_bn_bwd(L_, dy, dx):
+        bn = L_["bname"]
+        rows = L_["z"].numel() // L_["cout"]
+        g.k("bn_bwd_reduce", [_p(L_["z"]), _p(dy), _p(L_["mean"]), _p(L_["invstd"]), _p(P.g[f"{bn}.gamma"]),
+                              _p(P.g[f"{bn}.beta"]), rows, L_["cout"], 0, 0], f"{bn}.bwd_reduce", ws_at=8)
+        g.k("bn_bwd_dx", [_p(L_["z"]), _p(dy), _p(L_["dz"]), _p(P.p[f"{bn}.gamma"]), _p(L_["mean"]), _p(L_["invstd"]),
+                          _p(P.g[f"{bn}.gamma"]), _p(P.g[f"{bn}.beta"]), rows, L_["cout"]], f"{bn}.bwd_dx")
+        w = P.p[f"{L_['cname']}.w"]
+        conv_wgrad(g, L_["in"], L_["dz"], P.g[f"{L_['cname']}.w"], L_["stride"], L_["pad"], f"{L_['cname']}.wgrad")
+        if dx is not None:
+            conv_dgrad(g, L_["dz"], w, dx, L_["stride"], L_["pad"], f"{L_['cname']}.dgrad")
+
+    def relu(x, y, label):
+        g.k("relu", [_p(x), _p(y), x.numel()], label)
+
+    def relu_bwd(x, dy, dx, label):
+        g.k("relu_bwd", [_p(x), _p(dy), _p(dx), x.numel()], label)
+
+    def add(a, b, c, label):
+        g.k("add", [_p(a), _p(b), _p(c), a.numel()], label)
+
+    variants, ws_ops = [], None
+    for vi in range(len(xs)):
+        g.ops, g._ws_ops = [], []
+        y0 = conv_bn(stem, xb[vi])
+        relu(y0, a0, "bn1.relu")
+        g.k("maxpool", [_p(a0), _p(mp), n_, h_, w_, c_, pq, pq], "maxpool")
+        h = mp
+        for b in blocks:
+            p = b["name"]
+            relu(conv_bn(b["c1"], h), b["a1"], f"{p}.bn1.relu")
+            relu(conv_bn(b["c2"], b["a1"]), b["a2"], f"{p}.bn2.relu")
+            y3 = conv_bn(b["c3"], b["a2"])
+            idn = conv_bn(b["down"], h) if b["down"] is not None else h
+            add(y3, idn, b["sum"], f"{p}.add")
+            relu(b["sum"], b["out"], f"{p}.relu")
+            h = b["out"]
+        g.k("avgpool", [_p(h), _p(pooled), n, hh * ww, c], "avgpool")
+        linear_fwd(g, pooled, P.p["fc.w"], P.p["fc.b"], logits, "fc")
+        g.k("ce", [_p(logits), _p(lb[vi]), _p(loss), _p(dlogits), n, num_classes, 0, 0], "ce", ws_at=6)
+        gemm(g, dlogits, pooled, P.g["fc.w"], None, num_classes, c, n, num_classes, c, c, 1, "fc.wgrad")
+        g.k("colsum", [_p(dlogits), _p(P.g["fc.b"]), n, num_classes], "fc.bgrad")
+        gemm(g, dlogits, P.p["fc.w"], dpooled, None, n, c, num_classes, num_classes, c, c, 0, "fc.dgrad")
+        g.k("avgpool_bwd", [_p(dpooled), _p(dfeat), n, hh * ww, c], "avgpool_bwd")
+        dout = dfeat
+        for bi in reversed(range(len(blocks))):
+            b = blocks[bi]
+            p = b["name"]
+            relu_bwd(b["sum"], dout, b["dsum"], f"{p}.relu_bwd")
+            conv_bn_bwd(b["c3"], b["dsum"], b["da2"])
+            relu_bwd(b["c2"]["y"], b["da2"], b["d2"], f"{p}.bn2.relu_bwd")
+            conv_bn_bwd(b["c2"], b["d2"], b["da1"])
+            relu_bwd(b["c1"]["y"], b["da1"], b["d1"], f"{p}.bn1.relu_bwd")
+            conv_bn_bwd(b["c1"], b["d1"], b["dmain"])
+            if b["down"] is not None:
+                conv_bn_bwd(b["down"], b["dsum"], b["ddown"])
+                add(b["dmain"], b["ddown"], b["din"], f"{p}.add_bwd")
+            else:
+                add(b["dmain"], b["dsum"], b["din"], f"{p}.add_bwd")
+            dout = b["din"]
+        g.k("maxpool_bwd", [_p(a0), _p(dmp), _p(da0), n_, h_, w_, c_, pq, pq], "maxpool_bwd")
+        relu_bwd(y0, da0, dy0, "bn1.relu_bwd")
+        conv_bn_bwd(stem, dy0, None)
+        g.k("sgd", [_p(P.flat), _p(P.gflat), _p(P.vflat), P.total, f32bits(lr), f32bits(momentum)], "sgd")
+        variants.append(g.ops)
+        ws_ops = g._ws_ops
+    g.variants = []
+    for ops in variants:
+        g.ops, g._ws_ops = ops, list(ws_ops)
+        g.finalize()
+        g.variants.append(list(g.ops))
+    g.ops = g.variants[0]
+    g.loss = loss
+    g.params = P
+    g.logits = logits
+    # values the ReLU backward decides on (BN outputs and residual sums), for decision-aligned parity
+    g.relu_in = {"bn1": stem["y"]}
+    for b in blocks:
+        g.relu_in[f"{b['name']}.bn1"] = b["c1"]["y"]
+        g.relu_in[f"{b['name']}.bn2"] = b["c2"]["y"]
+        g.relu_in[f"{b['name']}.sum"] = b["sum"]
+    return g
+
+
+# ========================================================================= BERT inference (HP, config 3)
+BF16 = torch.bfloat16
+
+
+def bert_spec(layers=12, hidden=768, heads=12, ffn=3072, vocab=30522, max_pos=512, types=2):
+    """BERT-base parameters (HuggingFace BertModel without pooler), Linear weights [out, in].
+    Synthetic init (reading R22): weights, embeddings and biases N(0, 0.02); LayerNorm gamma
+    U[0.9, 1.1], beta N(0, 0.02)."""
+    nrm = ("normal", 0.02)
+    s = [("emb.word", (vocab, hidden), nrm), ("emb.pos", (max_pos, hidden), nrm), ("emb.type", (types, hidden), nrm),
+         ("emb.ln.gamma", (hidden,), ("uniform", 0.9, 1.1)), ("emb.ln.beta", (hidden,), nrm)]
+    for i in range(layers):
+        p = f"layer{i}"
+        for nm, o, k in (("q", hidden, hidden), ("k", hidden, hidden), ("v", hidden, hidden), ("o", hidden, hidden),
+                         ("ffn1", ffn, hidden), ("ffn2", hidden, ffn)):
+            s += [(f"{p}.{nm}.w", (o, k), nrm), (f"{p}.{nm}.b", (o,), nrm)]
+        for ln in ("ln1", "ln2"):
+            s += [(f"{p}.{ln}.gamma", (hidden,), ("uniform", 0.9, 1.1)), (f"{p}.{ln}.beta", (hidden,), nrm)]
+    return s
+
+
+class BF16Params:
+    """Inference parameters cast to bfloat16 (model.to(torch.bfloat16)), one device tensor each."""
+
+    def __init__(self, g, spec, host_params):
+        self.host = host_params
+        self.p = {n: g.buf(f"param.{n}", s, dtype=BF16) for n, s, _ in spec}
+        self.reset()
+
+    def reset(self):
+        with torch.no_grad():
+            for n, t in self.p.items():
+                t.copy_(self.host[n].to(BF16).to(t.device))
+
+
+def bert_infer_graph(host_params, batch=8, seq=128, layers=12, heads=12, hidden=768, ffn=3072, vocab=30522,
+                     device="cuda"):
+    """HP (config 3): BertModel forward in bf16, PyTorch-eager op granularity with the fused SDPA
+    attention kernel: per layer q, k, v projections, attention, output projection, residual add,
+    LayerNorm, FFN up, GELU, FFN down, residual add, LayerNorm (12 kernels). H2D of the token ids
+    (int32) first, D2H of the last hidden state (bf16) last."""
+    g = Graph("bert_infer", device)
+    spec = bert_spec(layers, hidden, heads, ffn, vocab)
+    P = BF16Params(g, spec, host_params)
+    rows = batch * seq
+    ids = g.buf("ids", (rows,), dtype=torch.int32)
+    g.memcpy(L.OP_MEMCPY_H2D, _p(ids), 0, rows * 4, "h2d_ids")
+    cnt = [0]
+
+    def new(cols):
+        cnt[0] += 1
+        return g.buf(f"t{cnt[0]}", (rows, cols), dtype=BF16)
+
+    def lin(x, name, out, k):
+        g.k("gemm_bf16", [_p(x), _p(P.p[f"{name}.w"]), _p(out), _p(P.p[f"{name}.b"]), rows, out.shape[1], k], name)
+
+    def ln(x, y, name):
+        g.k("layernorm", [_p(x), _p(y), _p(P.p[f"{name}.gamma"]), _p(P.p[f"{name}.beta"]), rows, hidden, f32bits(1e-12)], name)
+
+    e = new(hidden)
+    g.k("embed", [_p(ids), _p(P.p["emb.word"]), _p(P.p["emb.pos"]), _p(P.p["emb.type"]), _p(e), batch, seq, hidden, vocab],
+        "embed")
+    h = new(hidden)
+    ln(e, h, "emb.ln")
+    for i in range(layers):
+        p = f"layer{i}"
+        q, k, v, a, o, s1, h1 = (new(hidden) for _ in range(7))
+        f, fg, f2, s2, h2 = new(ffn), new(ffn), new(hidden), new(hidden), new(hidden)
+        lin(h, f"{p}.q", q, hidden)
+        lin(h, f"{p}.k", k, hidden)
+        lin(h, f"{p}.v", v, hidden)
+        g.k("attention", [_p(q), _p(k), _p(v), _p(a), batch, seq, heads, hidden // heads, hidden], f"{p}.attn")
+        lin(a, f"{p}.o", o, hidden)
+        g.k("add_bf16", [_p(o), _p(h), _p(s1), rows * hidden], f"{p}.add1")
+        ln(s1, h1, f"{p}.ln1")
+        lin(h1, f"{p}.ffn1", f, hidden)
+        g.k("gelu", [_p(f), _p(fg), rows * ffn], f"{p}.gelu")
+        lin(fg, f"{p}.ffn2", f2, ffn)
+        g.k("add_bf16", [_p(f2), _p(h1), _p(s2), rows * hidden], f"{p}.add2")
+        ln(s2, h2, f"{p}.ln2")
+        h = h2
+    g.memcpy(L.OP_MEMCPY_D2H, 0, _p(h), rows * hidden * 2, "d2h_hidden")
+    g.out = h
+    g.x = ids
+    g.params = P
+    return g.finalize()

@@ -125,6 +125,34 @@ def check_op(fn, a, R, snap=None, R_in=None):
         lab = R.get(a[1], B, None, torch.int32).cpu()
         loss, dz = om.ce_fwd_bwd(z, lab)
         return max(rel(R.get(a[2], 1), loss.reshape(1)), rel(R.get(a[3], B * Cn, (B, Cn)), dz))
+    BF = torch.bfloat16
+    if fn == "gemm_bf16":
+        M, N, K = a[4], a[5], a[6]
+        x, w = T(a[0], M * K, (M, K), BF), T(a[1], N * K, (N, K), BF)
+        b = T(a[3], N, None, BF) if a[3] else torch.zeros(N, dtype=BF)
+        return rel(R.get(a[2], M * N, (M, N), BF), om.linear_any(x, w, b))
+    if fn == "attention":
+        B, S, H, d, ld = a[4:9]
+        q, k, v = (T(a[i], B * S * ld, (B, S, ld), BF)[:, :, :H * d] for i in range(3))
+        return rel(R.get(a[3], B * S * ld, (B, S, ld), BF)[:, :, :H * d], om.attention(q, k, v, H))
+    if fn == "layernorm":
+        rows, C = a[4], a[5]
+        x = T(a[0], rows * C, (rows, C), BF)
+        ref = om.layernorm(x, T(a[2], C, None, BF), T(a[3], C, None, BF), eps=_u2f(a[6]))
+        return rel(R.get(a[1], rows * C, (rows, C), BF), ref)
+    if fn == "gelu":
+        return rel(R.get(a[1], a[2], None, BF), om.gelu(T(a[0], a[2], None, BF)))
+    if fn == "add_bf16":
+        return rel(R.get(a[2], a[3], None, BF), om.add_any(T(a[0], a[3], None, BF), T(a[1], a[3], None, BF)))
+    if fn == "embed":
+        B, S, H, V = a[5:9]
+        ids = R.get(a[0], B * S, (B, S), torch.int32).cpu()
+        ref = om.bert_embed(ids, T(a[1], V * H, (V, H), BF), T(a[2], S * H, (S, H), BF), T(a[3], H, (1, H), BF))
+        return rel(R.get(a[4], B * S * H, (B, S, H), BF), ref)
+    if fn == "maxpool_bwd":
+        n, h, w, c, p, q = a[3:9]
+        x, dy = T(a[0], n * h * w * c, (n, h, w, c)), T(a[1], n * p * q * c, (n, p, q, c))
+        return rel(R.get(a[2], n * h * w * c, (n, h, w, c)), om.maxpool3x3s2_bwd(x, dy))
     if fn == "colsum":
         M, N = a[2], a[3]
         return rel(R.get(a[1], N), om._r(T(a[0], M * N, (M, N)).double().sum(0)))

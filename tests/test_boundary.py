@@ -38,8 +38,13 @@ def test_no_libcuda_link_dependency():
 
 def test_kernel_table_names():
     from paper_conf_eurosys_stratimk24_b200 import _lib
+    import re
     names = _lib.kernel_names()
-    assert len(names) == 24 and names[0] == "gemm" and names[-1] == "ce"
+    hdr = open(os.path.join(ROOT, "include", "orion_kernels.h")).read()
+    enum = {int(v): k.lower() for k, v in re.findall(r"ORION_FN_(\w+) = (\d+)", hdr) if k != "COUNT"}
+    count = int(re.search(r"ORION_FN_COUNT = (\d+)", hdr).group(1))
+    assert len(names) == count == len(enum)
+    assert [enum[i] for i in range(count)] == names
 
 
 def test_cuda_backend_fails_cleanly_without_gpu():

@@ -76,3 +76,38 @@ def test_toy_collocated_parity(toy):
     be.graph.params.reset()
     C.run_session(be=be, be_iters=K)
     assert torch.equal(be.graph.params.flat.cpu(), p_col)
+
+
+def test_toy_three_be_clients(toy):
+    """one HP client and three BE training clients (each its own MLP,
+    buffers and stream) share one DUR budget round robin. The decision log must equal the oracle
+    replay byte for byte; every BE client's parameters after its K_j iterations must equal the
+    fp64 oracle's and be bitwise identical to a solo run of that client."""
+    hp = toy["hp"]
+    P = toy["P"]
+    bes = []
+    for j in range(3):
+        xs = [si.normal((32, 512), si.BE_SEED, sub=10 * (j + 1) + i) for i in range(2)]
+        ts = [si.normal((32, 512), si.BE_SEED, sub=200 + 10 * (j + 1) + i) for i in range(2)]
+        g = W.mlp_train_graph(P, xs, ts, lr=0.01)
+        prof, _ = PR.build_profiles(g, kid_base=1000 * (j + 1), reps=3)
+        g.params.reset()
+        bes.append((C.BEClient(g, prof, 1000 * (j + 1)), xs, ts))
+    res = C.run_session(hp=hp, be=[b for b, _, _ in bes], arrivals_ns=toy["arrivals"][:100], log_capacity=1 << 22,
+                        hp_latency_ns=20_000)
+    hdr, prefix, tape, decs = lf.split_log(res["log"])
+    assert decs == po.replay(prefix)
+    clients = {d[2] for d in lf.decode_decisions(decs) if d[1] in (3, 4)}
+    assert len(clients) == 3, clients          # every BE client was admitted
+    for j, (b, xs, ts) in enumerate(bes):
+        K = len(res["be_t_end_all"][j])
+        assert K >= 1
+        p_col = b.graph.params.flat.cpu().clone()
+        Po = dict(P)
+        for i in range(K):
+            _, Po, _ = om.mlp_train_step(Po, xs[i % 2], ts[i % 2], lr=0.01)
+        flat_ref = torch.cat([Po[n].reshape(-1) for n, _, _ in W.mlp_spec()])
+        assert rel(p_col, flat_ref) < 1e-4
+        b.graph.params.reset()
+        C.run_session(be=b, be_iters=K)
+        assert torch.equal(b.graph.params.flat.cpu(), p_col)
