@@ -223,6 +223,8 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--rate", type=float, default=0.0, help="override HP arrival rate (rps)")
+    ap.add_argument("--policy", default="orion", choices=["orion", "orion_noprio", "profiles", "priorities", "streams"],
+                    help="policy ablation (Fig. 14) / Streams baselines (P:1003-1014); orion = the full policy")
     args = ap.parse_args()
 
     rank = int(os.environ.get("RANK", 0))
@@ -266,8 +268,10 @@ def main():
     n_be_k = sum(1 for o in be.variants[0] if o.kind == L.OP_KERNEL)
     sched_cpu = 2 + 4 * local if (os.cpu_count() or 1) >= 8 else -1
 
+    pol_flags = L.POLICIES[args.policy]
+
     def session(**kw):
-        return C.run_session(sched_cpu=sched_cpu, device=local, **kw)
+        return C.run_session(sched_cpu=sched_cpu, device=local, flags=pol_flags, **kw)
 
     # ---- HP solo request latency -> DUR_THRESHOLD base (R9)
     spaced = (np.arange(1, 41) * 20e6).astype(np.int64)
@@ -385,6 +389,7 @@ def main():
         "data": "synthetic (seeded; DESIGN.md §5)",
         "config": dict(W_["cfg"], parallelism=f"replicas x{world} (independent Orion instance per GPU)",
                        hp_rate_rps=rate, dur_threshold_pct=args.dur_ppm / 1e4, be_partition_sms=args.be_partition,
+                       policy=args.policy,
                        l2=f"inputs > L2 (BE batch {W_['be_inputs'][0].numel() * 4 / 1e6:.1f} MB x 8 staged; no flush)"),
         "hp": {"p50_ms": col["p50_ns"] / 1e6, "p99_ms": col["p99_ns"] / 1e6, "dedicated_p50_ms": ded["p50_ns"] / 1e6,
                "dedicated_p99_ms": ded["p99_ns"] / 1e6, "p99_vs_dedicated": col["p99_ns"] / ded["p99_ns"],

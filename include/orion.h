@@ -77,7 +77,16 @@ enum {
   ORION_F_HP_REF_ALL = 2,            /* R3: profile test against every in-flight HP op */
   ORION_F_HP_UNKNOWN_STRICT = 4,     /* R4: HP-unknown admits only BE-unknown */
   ORION_F_THROTTLE_ONLY_HP_BUSY = 8, /* R7: DUR_THRESHOLD check only while HP is busy */
-  ORION_F_FREE_SMS = 16              /* R5: be.sm_needed + hp.sm_needed <= num_sms */
+  ORION_F_FREE_SMS = 16,             /* R5: be.sm_needed + hp.sm_needed <= num_sms */
+  /* Policy ablation (Fig. 14) and the Streams baselines: each switch
+     removes one component of the policy. NO_PROFILE | NO_SM | NO_THROTTLE admits every BE op
+     at once ("Stream Priorities"); adding NO_PRIORITY gives "GPU Streams" (every stream at the
+     default priority). NO_SM alone is the "Compute/Mem profiles" bar; NO_PRIORITY alone is
+     Orion without stream priorities. */
+  ORION_F_NO_PRIORITY = 32,          /* HP stream at the default (least) priority like the BE streams */
+  ORION_F_NO_PROFILE_TEST = 64,      /* schedule_be skips the compute/memory profile test (L28) */
+  ORION_F_NO_SM_TEST = 128,          /* schedule_be skips the SM-size test (L27) */
+  ORION_F_NO_THROTTLE = 256          /* no DUR_THRESHOLD throttle (L12-L16) */
 };
 
 enum { ORION_BACKEND_CUDA = 0, ORION_BACKEND_FAKE = 1 };

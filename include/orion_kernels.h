@@ -55,7 +55,7 @@ enum orion_fn {
      workspace, ws_bytes (orion_gemm_workspace_bytes(N*H*W, C, R*S*K)) */
   ORION_FN_CONV_DGRAD = 10,
   /* Conv2d backward weight: dw[K,R,S,C] from x, dy. args: x, dy, dw, N,H,W,C,K,R,S,stride,pad,P,Q,
-     workspace, ws_bytes (orion_gemm_workspace_bytes(K, R*S*C, N*P*Q)) */
+     workspace, ws_bytes (orion_conv_wgrad_workspace_bytes(N, H, W, C, K, R, S, stride, pad)) */
   ORION_FN_CONV_WGRAD = 11,
   /* Depthwise 3x3 conv (groups = C): args as CONV_* with K = C */
   ORION_FN_DW_FWD = 12,
@@ -125,6 +125,10 @@ int orion_kernel_geometry(uint32_t fn, const uint64_t* args, uint32_t nargs, uin
 /* Workspace sizes (bytes) of the ops that split their reductions. Workspaces must be zeroed once
    at allocation; a client's ops may share one (they run in stream order; tickets self-reset). */
 uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t K);
+/* CONV_WGRAD's workspace: the tiled split-K need, or (few-input-channel stems, C <= 4) the
+   per-CTA fp64 partials of the direct stem weight-gradient kernel, whichever is larger. */
+uint64_t orion_conv_wgrad_workspace_bytes(uint64_t N, uint64_t H, uint64_t W, uint64_t C, uint64_t K, uint64_t R, uint64_t S,
+                                          uint64_t stride, uint64_t pad);
 uint64_t orion_bn_workspace_bytes(uint64_t rows, uint64_t C);
 uint64_t orion_dw_wgrad_workspace_bytes(uint64_t N, uint64_t C, uint64_t P, uint64_t Q);
 

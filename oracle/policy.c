@@ -39,6 +39,10 @@
 #define F_HP_UNKNOWN_STRICT 4u
 #define F_THROTTLE_ONLY_HP_BUSY 8u
 #define F_FREE_SMS 16u
+#define F_NO_PRIORITY 32u        /* stream priorities only: no effect on decisions */
+#define F_NO_PROFILE_TEST 64u    /* ablation (Fig. 14): skip L28 */
+#define F_NO_SM_TEST 128u        /* ablation: skip L27 */
+#define F_NO_THROTTLE 256u       /* ablation / Streams baselines: skip L12-L16 */
 
 /* decision kinds */
 enum { D_HP_LAUNCH = 1, D_PASS = 2, D_ADMIT_IDLE = 3, D_ADMIT_COLOC = 4, D_DEFER_SM = 5,
@@ -155,6 +159,7 @@ static int parse_log(const uint8_t *b, size_t len, o_cfg *c, int want_tape) {
 /* differ(a, b): a = HP class, b = BE class. R4 (symmetric unknown optimism);
  * switch HP_UNKNOWN_STRICT keeps only BE-unknown optimism. */
 static int differ(const o_cfg *c, int a, int b) {
+  if (c->flags & F_NO_PROFILE_TEST) return 1;
   if (c->flags & F_HP_UNKNOWN_STRICT) return b == CLS_U || (a != CLS_U && a != b);
   if (ORACLE_MUTANT == 3) return a != b;   /* 'unknown' treated as a class of its own */
   return a == CLS_U || b == CLS_U || a != b;
@@ -162,6 +167,7 @@ static int differ(const o_cfg *c, int a, int b) {
 
 /* thr(h): R5. STATIC = SM_THRESHOLD; FREE_SMS: be.sm + hp.sm <= num_sms. */
 static int64_t thr(const o_cfg *c, const o_op *h) {
+  if (c->flags & F_NO_SM_TEST) return INT64_MAX;
   if (c->flags & F_FREE_SMS) {
     int64_t t = (int64_t)c->num_sms - (int64_t)h->sm_needed + 1;
     return t < 0 ? 0 : t;
@@ -244,7 +250,7 @@ static int iterate(const o_cfg *c, o_state *s, uint64_t k, o_out *out, int *err)
     }
     int reason = schedule_be(c, s, hp_busy, op);                            /* L11 */
     int sched = reason == R_NONE;
-    int throttle = !(c->flags & F_THROTTLE_ONLY_HP_BUSY) || hp_busy;        /* R7 */
+    int throttle = !(c->flags & F_NO_THROTTLE) && (!(c->flags & F_THROTTLE_ONLY_HP_BUSY) || hp_busy);   /* R7; ablation */
     if (throttle && (ORACLE_MUTANT == 4 ? s->be_dur >= (int64_t)c->dur_thr : s->be_dur > (int64_t)c->dur_thr)) { /* L12 (R6 strict >) */
       if (ORACLE_MUTANT == 5 ? 1 : all_be_drained(c, s)) {                  /* L13 */
         s->be_dur = 0;                                                      /* L14 */
@@ -387,7 +393,7 @@ static void check_iter(o_brute *b, const o_state *pre, const o_state *post, cons
         if (!((int64_t)op->sm_needed < thr(c, h) && differ(c, h->cls, op->cls))) bfail(b, "I3 (coloc admit violates SM/profile)", k);
       }
       /* I4: admission happens with be_dur <= thr, or after a RESET in this iteration */
-      int throttle = !(c->flags & F_THROTTLE_ONLY_HP_BUSY) || hp_busy_pre || hp_launches;
+      int throttle = !(c->flags & F_NO_THROTTLE) && (!(c->flags & F_THROTTLE_ONLY_HP_BUSY) || hp_busy_pre || hp_launches);
       if (throttle && !(be_dur <= (int64_t)c->dur_thr) && !reset_seen) bfail(b, "I4 (admit over threshold)", k);
       be_dur += (int64_t)op->dur_ns;
       if (r->be_dur != be_dur) bfail(b, "I4 (be_dur accounting)", k);
@@ -398,9 +404,10 @@ static void check_iter(o_brute *b, const o_state *pre, const o_state *post, cons
   /* I1: an HP op visible at k (earlier ones popped) is launched at k */
   if (c->hp >= 0 && pre->popped[c->hp] < pre->vis[c->hp] && hp_launches != 1) bfail(b, "I1 (visible HP op not launched)", k);
   /* I5: be_dur <= thr + max_dur always (overshoot bound) */
-  if (!(c->flags & F_THROTTLE_ONLY_HP_BUSY) && post->be_dur > (int64_t)c->dur_thr + b->max_dur) bfail(b, "I5 (overshoot bound)", k);
+  const int throttled = !(c->flags & (F_THROTTLE_ONLY_HP_BUSY | F_NO_THROTTLE));
+  if (throttled && post->be_dur > (int64_t)c->dur_thr + b->max_dur) bfail(b, "I5 (overshoot bound)", k);
   /* I6: outstanding profiled BE work <= thr + max_dur */
-  if (!(c->flags & F_THROTTLE_ONLY_HP_BUSY)) {
+  if (throttled) {
     int64_t outst = 0;
     for (int t = 0; t < c->n_be; t++) {
       int j = c->be_idx[t];

@@ -20,6 +20,10 @@ CLS_U, CLS_C, CLS_M = 0, 1, 2
 OP_KERNEL, OP_MEMCPY_H2D, OP_MEMCPY_D2H, OP_MEMSET, OP_MEMCPY_D2D = 0, 1, 2, 3, 4
 OPF_REQ_BEGIN, OPF_REQ_END = 1, 2
 F_HP_BUSY_REQUEST, F_HP_REF_ALL, F_HP_UNKNOWN_STRICT, F_THROTTLE_ONLY_HP_BUSY, F_FREE_SMS = 1, 2, 4, 8, 16
+F_NO_PRIORITY, F_NO_PROFILE_TEST, F_NO_SM_TEST, F_NO_THROTTLE = 32, 64, 128, 256
+# policy ablation (Fig. 14) and the Streams baselines
+POLICIES = {"orion": 0, "orion_noprio": F_NO_PRIORITY, "profiles": F_NO_SM_TEST, "priorities": F_NO_PROFILE_TEST | F_NO_SM_TEST | F_NO_THROTTLE,
+            "streams": F_NO_PRIORITY | F_NO_PROFILE_TEST | F_NO_SM_TEST | F_NO_THROTTLE}
 BACKEND_CUDA, BACKEND_FAKE = 0, 1
 MAX_ARGS = 24
 WS_TICKET_BYTES = 65536   # kernels/common.cuh: ticket region at the start of every workspace
@@ -75,6 +79,7 @@ _sig = {
                                              ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_int32),
                                              ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_int32)]),
     "orion_gemm_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64]),
+    "orion_conv_wgrad_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64] * 9),
     "orion_bn_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64, ctypes.c_uint64]),
     "orion_dw_wgrad_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64]),
 }

@@ -53,6 +53,7 @@ struct CudaBackend : Backend {
   uint32_t sms = 0;
   int prio_least = 0, prio_greatest = 0;
   uint32_t be_partition = 0;
+  uint32_t flags = 0;
   Drv drv;
   unsigned long long* host_counters = nullptr;  // one 64-byte line per stream
   int next_counter = 0;
@@ -80,6 +81,7 @@ struct CudaBackend : Backend {
     if (cudaDeviceGetStreamPriorityRange(&prio_least, &prio_greatest) != cudaSuccess) return ORION_E_CUDA;
     if (!resolve("cuStreamWriteValue64", &drv.streamWriteValue64, 12000)) return ORION_E_CUDA;
     be_partition = cfg.be_partition_sms;
+    flags = cfg.flags;
     if (be_partition) {
       bool ok = resolve("cuDeviceGetDevResource", &drv.deviceGetDevResource, 12080) &&
                 resolve("cuDevSmResourceSplitByCount", &drv.devSmResourceSplitByCount, 12080) &&
@@ -126,7 +128,8 @@ struct CudaBackend : Backend {
       }
       s->stream = (cudaStream_t)cs;
     } else {
-      if (cudaStreamCreateWithPriority(&s->stream, cudaStreamNonBlocking, prio == ORION_HP ? prio_greatest : prio_least) != cudaSuccess) {
+      const bool hp_prio = prio == ORION_HP && !(flags & ORION_F_NO_PRIORITY);   // NO_PRIORITY: "GPU Streams" baseline
+      if (cudaStreamCreateWithPriority(&s->stream, cudaStreamNonBlocking, hp_prio ? prio_greatest : prio_least) != cudaSuccess) {
         delete s;
         return ORION_E_CUDA;
       }

@@ -1911,6 +1911,139 @@ __global__ void __launch_bounds__(NTH) conv_fwd_smallc_kernel(const float* __res
 
 // specialised for the 3x3, 3-channel stem (the only few-channel conv of the workloads)
 inline bool fwd_ok(const ConvShape& s) { return s.C == 3 && s.R == 3 && s.S == 3 && s.K % 4 == 0 && s.K <= MAXK; }
+
+// Weight gradient of a few-input-channel stem (ResNet 7x7x3 / MobileNetV2 3x3x3):
+// dw[k][r][s][c] = sum_{n,p,q} dy[n,p,q,k] x[n, p*st-pad+r, q*st-pad+s, c]. As an implicit GEMM the
+// B operand (im2col of x, C = 3) cannot be loaded in 16-byte pieces and the problem has only
+// K x RSC = 64 x 147 outputs over 802816-long sums. Here a CTA walks tiles of QT consecutive
+// output pixels of one output row: the tile's dy rows (QT x K, contiguous) and the x window it
+// touches (R rows x ((QT-1)*st + S) columns x C, contiguous per row) are staged in shared memory
+// (the next tile's loads held in registers while the current one is multiplied), and each thread
+// owns a 4 (k) x <= WG_MAXR (rsc) register block. Partials (fp64) of the G CTAs (a shape-only
+// count) are combined in CTA order (combine_splits), so results are deterministic.
+constexpr int WG_QT = 32, WG_KPT = 4, WG_MAXR = 12, WG_G = 148;   // one CTA per SM of a full B200 (~166 registers)
+constexpr int WG_PF_DY = WG_QT * MAXK / 4 / NTH, WG_PF_X = 8;   // per-thread prefetch registers
+__host__ __device__ inline int wg_wwin(const ConvShape& s) { return (WG_QT - 1) * s.stride + s.S; }
+__host__ __device__ inline int wg_xwin(const ConvShape& s) { return s.R * wg_wwin(s) * s.C; }
+inline long long wg_tiles(const ConvShape& s) { return (long long)s.N * s.P * ((s.Q + WG_QT - 1) / WG_QT); }
+inline int wg_ctas(const ConvShape& s) { return (int)(wg_tiles(s) < WG_G ? wg_tiles(s) : WG_G); }
+inline bool wgrad_ok(const ConvShape& s) {
+  const int kg = s.K / WG_KPT, rsc = s.R * s.S * s.C;
+  return s.C <= 4 && s.K % WG_KPT == 0 && s.K <= MAXK && (kg & (kg - 1)) == 0 && rsc <= (NTH / kg) * WG_MAXR &&
+         wg_xwin(s) <= NTH * WG_PF_X && s.stride <= 2;
+}
+inline uint64_t wgrad_ws_bytes(const ConvShape& s) {
+  const int G = wg_ctas(s);
+  const uint64_t V = (uint64_t)s.K * s.R * s.S * s.C;
+  return WS_TICKET_BYTES + (uint64_t)(G + combine_rows(G) + 1) * V * 8;
+}
+
+__global__ void __launch_bounds__(NTH, 1) conv_wgrad_smallc_kernel(const float* __restrict__ x, const float* __restrict__ dy,
+                                                                float* __restrict__ dw, ConvShape s, unsigned char* ws, OrionSig sig) {
+  extern __shared__ __align__(16) float wsm[];
+  const int K = s.K, RSC = s.R * s.S * s.C, WW = wg_wwin(s), XW = wg_xwin(s);
+  float* dys = wsm;                      // [WG_QT][K]
+  float* xs = wsm + WG_QT * K;           // [R][WW][C]
+  const int kgroups = K / WG_KPT, rgroups = NTH / kgroups;
+  const int kg = threadIdx.x % kgroups, rg = threadIdx.x / kgroups;
+  int off[WG_MAXR];
+#pragma unroll
+  for (int i = 0; i < WG_MAXR; i++) {
+    const int j = rg + rgroups * i;
+    if (j < RSC) {
+      const int c = j % s.C, t = j / s.C, u = t % s.S, r = t / s.S;
+      off[i] = (r * WW + u) * s.C + c;
+    } else {
+      off[i] = -1;
+    }
+  }
+  float acc[WG_KPT][WG_MAXR];
+#pragma unroll
+  for (int a = 0; a < WG_KPT; a++)
+#pragma unroll
+    for (int i = 0; i < WG_MAXR; i++) acc[a][i] = 0.f;
+  const int qtiles = (s.Q + WG_QT - 1) / WG_QT;
+  const long long T = (long long)s.N * s.P * qtiles;
+  float4 pdy[WG_PF_DY];
+  float px[WG_PF_X];
+#define WG_FETCH(TT)                                                                                                    \
+  {                                                                                                                     \
+    const long long t_ = (TT);                                                                                          \
+    const int qt = (int)(t_ % qtiles); const long long np = t_ / qtiles;                                                \
+    const int p = (int)(np % s.P), n = (int)(np / s.P);                                                                 \
+    const int q0 = qt * WG_QT, qn = min(WG_QT, s.Q - q0);                                                               \
+    const float4* src = reinterpret_cast<const float4*>(dy + (((long long)n * s.P + p) * s.Q + q0) * K);                \
+    _Pragma("unroll") for (int e = 0; e < WG_PF_DY; e++) {                                                              \
+      const int idx = threadIdx.x + e * NTH;                                                                            \
+      pdy[e] = (idx * 4 < qn * K) ? __ldg(src + idx) : make_float4(0.f, 0.f, 0.f, 0.f);                                  \
+    }                                                                                                                   \
+    const int h0 = p * s.stride - s.pad, w0 = q0 * s.stride - s.pad;                                                    \
+    _Pragma("unroll") for (int e = 0; e < WG_PF_X; e++) {                                                               \
+      const int idx = threadIdx.x + e * NTH;                                                                            \
+      float v = 0.f;                                                                                                    \
+      if (idx < XW) {                                                                                                   \
+        const int c = idx % s.C, t2 = idx / s.C, u = t2 % WW, r = t2 / WW;                                              \
+        const int h = h0 + r, w = w0 + u;                                                                               \
+        if ((unsigned)h < (unsigned)s.H && (unsigned)w < (unsigned)s.W) v = __ldg(x + (((long long)n * s.H + h) * s.W + w) * s.C + c); \
+      }                                                                                                                 \
+      px[e] = v;                                                                                                        \
+    }                                                                                                                   \
+  }
+  long long t = blockIdx.x;
+  if (t < T) WG_FETCH(t);
+  for (; t < T; t += gridDim.x) {
+    __syncthreads();                                    // previous tile's compute done
+#pragma unroll
+    for (int e = 0; e < WG_PF_DY; e++) {
+      const int idx = threadIdx.x + e * NTH;
+      if (idx * 4 < WG_QT * K) reinterpret_cast<float4*>(dys)[idx] = pdy[e];
+    }
+#pragma unroll
+    for (int e = 0; e < WG_PF_X; e++) {
+      const int idx = threadIdx.x + e * NTH;
+      if (idx < XW) xs[idx] = px[e];
+    }
+    __syncthreads();
+    if (t + gridDim.x < T) WG_FETCH(t + gridDim.x);    // next tile's loads in flight during the math
+    const int xstep = s.stride * s.C;
+#pragma unroll 2
+    for (int i = 0; i < WG_QT; i++) {                   // zero dy rows beyond Q contribute nothing
+      const float4 d = *reinterpret_cast<const float4*>(dys + i * K + kg * WG_KPT);
+      const float* xr = xs + i * xstep;
+#pragma unroll
+      for (int j = 0; j < WG_MAXR; j++) {
+        if (off[j] >= 0) {
+          const float xv = xr[off[j]];
+          acc[0][j] = fmaf(d.x, xv, acc[0][j]);
+          acc[1][j] = fmaf(d.y, xv, acc[1][j]);
+          acc[2][j] = fmaf(d.z, xv, acc[2][j]);
+          acc[3][j] = fmaf(d.w, xv, acc[3][j]);
+        }
+      }
+    }
+  }
+  // partial of this CTA -> workspace (fp64), ordered combine over the G CTAs
+  const long long V = (long long)K * RSC;
+  unsigned int* tk = reinterpret_cast<unsigned int*>(ws);
+  double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
+  const int G = gridDim.x;
+  double* gpart = part + (long long)G * V;
+  double* out = gpart + (long long)combine_rows(G) * V;
+#pragma unroll
+  for (int j = 0; j < WG_MAXR; j++) {
+    const int jj = rg + rgroups * j;
+    if (jj < RSC) {
+#pragma unroll
+      for (int a = 0; a < WG_KPT; a++) part[(long long)blockIdx.x * V + (long long)(kg * WG_KPT + a) * RSC + jj] = (double)acc[a][j];
+    }
+  }
+  __shared__ double scratch[NTH];
+  if (combine_splits(tk, part, gpart, V, G, blockIdx.x, (int)V, out, scratch)) {
+    for (long long v = threadIdx.x; v < V; v += NTH) dw[v] = (float)__ldcg(out + v);
+  }
+  orion_signal(sig);
+}
+#undef WG_FETCH
 }  // namespace smallc
 
 }  // namespace
@@ -2081,13 +2214,43 @@ int conv_dgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cuda
                       BDgrad{(const float*)a[1], s}, sig, st);
 }
 
+extern "C" uint64_t orion_conv_wgrad_workspace_bytes(uint64_t N, uint64_t H, uint64_t W, uint64_t C, uint64_t K, uint64_t R,
+                                                     uint64_t S, uint64_t stride, uint64_t pad) {
+  ConvShape s{(int)N, (int)H, (int)W, (int)C, (int)K, (int)R, (int)S, (int)stride, (int)pad,
+              (int)((H + 2 * pad - R) / stride + 1), (int)((W + 2 * pad - S) / stride + 1)};
+  uint64_t b = orion_gemm_workspace_bytes(K, R * S * C, (uint64_t)N * s.P * s.Q);
+  if (smallc::wgrad_ok(s)) {
+    const uint64_t b2 = smallc::wgrad_ws_bytes(s);
+    if (b2 > b) b = b2;
+  }
+  return b;
+}
+
 int conv_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
   ConvShape s = conv_shape(a);
+  if (smallc::wgrad_ok(s) && a[14] != 0 && a[15] >= smallc::wgrad_ws_bytes(s)) {
+    static std::atomic<int> attr{0};
+    const int smem = (smallc::WG_QT * s.K + smallc::wg_xwin(s)) * 4;
+    if (!attr.load()) {
+      if (cudaFuncSetAttribute((const void*)smallc::conv_wgrad_smallc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 48 * 1024) !=
+          cudaSuccess)
+        return ORION_E_CUDA;
+      attr.store(1);
+    }
+    g->grid = dim3((unsigned)smallc::wg_ctas(s)); g->block = dim3(smallc::NTH); g->smem = smem;
+    g->func = (const void*)smallc::conv_wgrad_smallc_kernel;
+    return 0;
+  }
   tiled_geom<ADenseT, BWgrad>(g, s.K, (long long)s.R * s.S * s.C, (long long)s.N * s.P * s.Q, a[14], a[15]);
   return 0;
 }
 int conv_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   ConvShape s = conv_shape(a);
+  if (g.func == (const void*)smallc::conv_wgrad_smallc_kernel) {
+    smallc::conv_wgrad_smallc_kernel<<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s,
+                                                                       (unsigned char*)a[14], sig);
+    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+  }
   long long M = s.K, N = (long long)s.R * s.S * s.C, K = (long long)s.N * s.P * s.Q;
   // A(m = kout, k = npq) = dy[npq * K + kout]
   return launch_tiled(g, M, N, K, (float*)a[2], N, nullptr, (float*)a[14], ADenseT{(const float*)a[1], s.K},

@@ -4,8 +4,9 @@
 //
 //  * gemm_bf16: y = x W^T + b on the 5th-gen tensor cores (tcgen05.mma kind::f16, bf16 operands,
 //    fp32 accumulator in TMEM), operands staged by cp.async into the UMMA K-major core-matrix
-//    layout, a 6-stage mbarrier pipeline, one elected MMA thread; epilogue TMEM -> registers ->
-//    bias -> bf16 (round to nearest even).
+//    layout, an 8-10-stage mbarrier pipeline, one elected MMA thread; BERT's few-tile shapes are
+//    split over K across a thread-block cluster and reduced in rank order through distributed
+//    shared memory; epilogue TMEM -> registers -> bias -> bf16 (round to nearest even).
 //  * attention: fused scaled-dot-product attention (the one SDPA kernel PyTorch dispatches),
 //    per (batch, head, 64-query block); Q K^T and P V on mma.sync m16n8k16 bf16 with fp32
 //    accumulators, softmax in fp32 registers, P rounded to bf16 for the second product (what a
@@ -98,11 +99,12 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
 
 template <int BN>
 struct Cfg {
-  static constexpr int STAGES = 6;
   static constexpr int A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2, STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int EPI_LD = BN + 8;   // padded bf16 staging row: conflict-free 16-byte row writes
-  static constexpr int EPI_BYTES = BM * EPI_LD * 2;
-  static constexpr int SMEM = (STAGES * STAGE_BYTES > EPI_BYTES ? STAGES * STAGE_BYTES : EPI_BYTES) + 256 + 1024;
+  static constexpr int STAGES = BN == 64 ? 10 : 8;   // 160 / 192 KB of operand stages per CTA
+  static constexpr int RED_LD = BN + 4;              // padded fp32 partial row (split-K reduction)
+  static constexpr int RED_BYTES = BM * RED_LD * 4;
+  static constexpr int MAIN = STAGES * STAGE_BYTES > RED_BYTES ? STAGES * STAGE_BYTES : RED_BYTES;
+  static constexpr int SMEM = MAIN + 256 + 1024;
   static constexpr int TMEM_COLS = BN < 32 ? 32 : BN;
   // instruction descriptor (kind::f16): D f32 (bits 4-5 = 1), A bf16 (bits 7-9 = 1), B bf16 (bits
   // 10-12 = 1), both K-major, N >> 3 at bits 17-22, M >> 4 at bits 24-28
@@ -115,21 +117,42 @@ struct Cfg {
 __device__ __forceinline__ uint32_t elem_off(int row, int kq, int rows) {
   return (uint32_t)((kq >> 1) * (rows * 32) + (row >> 3) * 256 + (kq & 1) * 128 + (row & 7) * 16);
 }
+__device__ __forceinline__ uint32_t cluster_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ float4 ld_dsmem4(uint32_t local_addr, uint32_t rank) {
+  uint32_t ra;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(local_addr), "r"(rank));
+  float4 v;
+  asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(ra) : "memory");
+  return v;
+}
 
+// Split-K over a thread-block cluster: the `split` CTAs of a cluster (gridDim.z == cluster z) take
+// consecutive K ranges of the same output tile; each parks its fp32 partial tile in its own shared
+// memory, and after a cluster barrier rank 0 sums ranks 0, 1, .. in order through distributed
+// shared memory (ld.shared::cluster), adds the bias, rounds to bf16 and stores. No workspace, no
+// atomics, fixed summation order (the split is a function of the shape only).
 template <int BN>
 __global__ void __launch_bounds__(NTHR, 1) gemm_bf16_kernel(const bf16* __restrict__ A, const bf16* __restrict__ W, bf16* __restrict__ C,
-                                                           const bf16* __restrict__ bias, int M, int N, int K, OrionSig sig) {
+                                                           const bf16* __restrict__ bias, int M, int N, int K, int kps, OrionSig sig) {
   using Cf = Cfg<BN>;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   constexpr int S = Cf::STAGES;
-  constexpr int MAIN = S * Cf::STAGE_BYTES > Cf::EPI_BYTES ? S * Cf::STAGE_BYTES : Cf::EPI_BYTES;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + MAIN);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + Cf::MAIN);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * S + 1);
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + S), done_bar = smem_u32(bars + 2 * S);
   const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
   const int m0 = blockIdx.y * BM, n0 = blockIdx.x * BN;
-  const int nk = (K + BK - 1) / BK;
+  const int split = gridDim.z;
+  const int kbeg = blockIdx.z * kps, kend = min(K, kbeg + kps);
+  const int nk = kend > kbeg ? (kend - kbeg + BK - 1) / BK : 0;
 
   if (tid == 0) {
     for (int s = 0; s < S; s++) { mbar_init(full0 + 8 * s, NPROD); mbar_init(empty0 + 8 * s, 1); }
@@ -146,19 +169,19 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_bf16_kernel(const bf16* __restri
   const uint32_t tmem = *tmem_slot;
 
   if (warp < NPROD / 32) {
-    // producers: thread t copies A row t (4 chunks of 8 bf16) and B rows t (and t + 128 / 64 ..)
-    // of every stage with cp.async (zero-fill beyond M, N, K), S-2 stages in flight
+    // producers: thread t copies A row t (4 chunks of 8 bf16) and B rows t (+128) of every stage
+    // with cp.async (zero-fill beyond M, N, K), S-2 stages in flight
     const int a_row = tid;
     const bool a_ok = m0 + a_row < M;
     const bf16* a_src = A + (long long)(m0 + a_row) * K;
     auto issue = [&](int kt) {
       const int s = kt % S;
       const uint32_t st = smem_u32(smem + s * Cf::STAGE_BYTES);
-      const int k0 = kt * BK;
+      const int k0 = kbeg + kt * BK;
 #pragma unroll
       for (int q = 0; q < 4; q++) {
         const int k = k0 + 8 * q;
-        cp_async16(st + elem_off(a_row, q, BM), a_src + k, a_ok && k < K);
+        cp_async16(st + elem_off(a_row, q, BM), a_src + k, a_ok && k < kend);
       }
 #pragma unroll
       for (int r = tid; r < BN; r += NPROD) {
@@ -167,7 +190,7 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_bf16_kernel(const bf16* __restri
 #pragma unroll
         for (int q = 0; q < 4; q++) {
           const int k = k0 + 8 * q;
-          cp_async16(st + Cf::A_BYTES + elem_off(r, q, BN), src + k, ok && k < K);
+          cp_async16(st + Cf::A_BYTES + elem_off(r, q, BN), src + k, ok && k < kend);
         }
       }
     };
@@ -189,6 +212,7 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_bf16_kernel(const bf16* __restri
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // cp.async writes -> tensor core
       mbar_arrive(full0 + 8 * (kt % S));
     }
+    cp_wait<0>();
   } else if (lane == 0) {
     // MMA issuer (one thread): two K steps of 16 per stage into one fp32 accumulator
     for (int kt = 0; kt < nk; kt++) {
@@ -206,12 +230,11 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_bf16_kernel(const bf16* __restri
     mma_commit(done_bar);
   }
 
-  // epilogue (warps 0-3 = TMEM lanes 0-127 = tile rows): accumulator + bias -> bf16 -> padded
-  // shared tile -> coalesced 16-byte row stores
+  // epilogue (warps 0-3 = TMEM lanes 0-127 = tile rows): fp32 partial tile -> padded shared tile
+  float* red = reinterpret_cast<float*>(smem);
   if (warp < 4) {
     mbar_wait(done_bar, 0);
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
-    bf16* tile = reinterpret_cast<bf16*>(smem);
 #pragma unroll 1
     for (int c0 = 0; c0 < BN; c0 += 32) {
       float v[32];
@@ -221,29 +244,41 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_bf16_kernel(const bf16* __restri
         for (int i = 0; i < 32; i++) v[i] = 0.f;
       }
 #pragma unroll
-      for (int i = 0; i < 32; i++) {
-        const int n = n0 + c0 + i;
-        if (bias != nullptr && n < N) v[i] += bf2f(bias[n]);
-      }
-#pragma unroll
-      for (int i = 0; i < 32; i += 8) *reinterpret_cast<uint4*>(tile + tid * Cf::EPI_LD + c0 + i) = pack8(v + i);
+      for (int i = 0; i < 32; i += 4)
+        *reinterpret_cast<float4*>(red + tid * Cf::RED_LD + c0 + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
     }
-    asm volatile("bar.sync 1, 128;" ::: "memory");
-    constexpr int CPR = BN / 8;   // 16-byte chunks per tile row
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  if (split > 1) cluster_sync(); else __syncthreads();
+  // rank 0 of the cluster: sum partials in rank order, + bias, bf16, coalesced 16-byte row stores
+  if ((split == 1 || cluster_rank() == 0) && tid < 128) {
+    constexpr int CPR = BN / 8;   // 16-byte output chunks per tile row
     const bool vec = (N % 8) == 0;
     for (int e = tid; e < BM * CPR; e += 128) {
       const int r = e / CPR, c = (e % CPR) * 8;
       const int m = m0 + r, n = n0 + c;
       if (m >= M || n >= N) continue;
-      const bf16* srcp = tile + r * Cf::EPI_LD + c;
+      const float* src = red + r * Cf::RED_LD + c;
+      float4 lo = *reinterpret_cast<const float4*>(src), hi = *reinterpret_cast<const float4*>(src + 4);
+      for (int z = 1; z < split; z++) {
+        const uint32_t la = smem_u32(src);
+        const float4 a = ld_dsmem4(la, (uint32_t)z), b = ld_dsmem4(la + 16, (uint32_t)z);
+        lo.x += a.x; lo.y += a.y; lo.z += a.z; lo.w += a.w;
+        hi.x += b.x; hi.y += b.y; hi.z += b.z; hi.w += b.w;
+      }
+      float f[8] = {lo.x, lo.y, lo.z, lo.w, hi.x, hi.y, hi.z, hi.w};
+      if (bias != nullptr) {
+#pragma unroll
+        for (int i = 0; i < 8; i++)
+          if (n + i < N) f[i] += bf2f(bias[n + i]);
+      }
       bf16* dst = C + (long long)m * N + n;
-      if (vec) *reinterpret_cast<uint4*>(dst) = *reinterpret_cast<const uint4*>(srcp);
+      if (vec) *reinterpret_cast<uint4*>(dst) = pack8(f);
       else
-        for (int i = 0; i < 8 && n + i < N; i++) dst[i] = srcp[i];
+        for (int i = 0; i < 8 && n + i < N; i++) dst[i] = __float2bfloat16_rn(f[i]);
     }
   }
-  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-  __syncthreads();
+  if (split > 1) cluster_sync();   // partials stay alive until rank 0 has read them
   if (warp == NPROD / 32) {
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(Cf::TMEM_COLS) : "memory");
@@ -260,9 +295,25 @@ bool prepare() {
   if (ok) done.store(1, std::memory_order_release);
   return ok;
 }
-// Tile width from the shape only (never the SM partition): 128 when that still gives >= one CTA
-// per SM of a whole B200, else 64 (twice the CTAs for the N = 768 projections of BERT-base).
-inline int bn_for(long long M, long long N) { return cdiv(M, BM) * cdiv(N, 128) >= 148 ? 128 : 64; }
+// Shape-only plan (never the SM partition): tile width BN in {64, 128} and cluster split-K s in
+// {1..4} minimising waves x per-CTA stream (k-tiles x bytes per stage) over a 148-SM part, >= 4
+// k-tiles per split.
+struct Plan { int bn, split, kps; };
+inline Plan plan(long long M, long long N, long long K) {
+  const long long kt = cdiv(K, BK);
+  Plan best{64, 1, (int)K};
+  double best_cost = 1e30;
+  for (int bn = 64; bn <= 128; bn *= 2) {
+    const long long tiles = cdiv(M, BM) * cdiv(N, bn);
+    for (int sp = 1; sp <= 4; sp++) {
+      if (sp > 1 && kt / sp < 4) break;
+      const long long kts = cdiv(kt, sp);
+      const double cost = (double)cdiv(tiles * sp, 148) * (double)kts * (double)(BM + bn) + (sp > 1 ? 3.0 * (sp - 1) * (BM + bn) : 0.0);
+      if (cost < best_cost) { best_cost = cost; best = Plan{bn, sp, (int)(kts * BK)}; }
+    }
+  }
+  return best;
+}
 
 }  // namespace tcb
 
@@ -546,10 +597,10 @@ inline bool al16(uint64_t p) { return (p & 15) == 0; }
 int gemm_bf16_geom(const uint64_t* a, LaunchGeom* g) {
   const long long M = (long long)a[4], N = (long long)a[5], K = (long long)a[6];
   if (M <= 0 || N <= 0 || K <= 0 || (K % 8) != 0 || !al16(a[0]) || !al16(a[1]) || !al16(a[2])) return ORION_E_INVAL;
-  const int bn = tcb::bn_for(M, N);
-  g->grid = dim3((unsigned)cdiv(N, bn), (unsigned)cdiv(M, tcb::BM));
+  const tcb::Plan pl = tcb::plan(M, N, K);
+  g->grid = dim3((unsigned)cdiv(N, pl.bn), (unsigned)cdiv(M, tcb::BM), (unsigned)pl.split);
   g->block = dim3(tcb::NTHR);
-  if (bn == 128) {
+  if (pl.bn == 128) {
     if (!tcb::prepare<128>()) return ORION_E_CUDA;
     g->smem = tcb::Cfg<128>::SMEM; g->func = (const void*)tcb::gemm_bf16_kernel<128>;
   } else {
@@ -559,13 +610,21 @@ int gemm_bf16_geom(const uint64_t* a, LaunchGeom* g) {
   return 0;
 }
 int gemm_bf16_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
-  auto A = (const bf16*)a[0]; auto W = (const bf16*)a[1]; auto C = (bf16*)a[2]; auto bias = (const bf16*)a[3];
-  const int M = (int)a[4], N = (int)a[5], K = (int)a[6];
+  const bf16* A = (const bf16*)a[0]; const bf16* W = (const bf16*)a[1]; bf16* C = (bf16*)a[2]; const bf16* bias = (const bf16*)a[3];
+  int M = (int)a[4], N = (int)a[5], K = (int)a[6];
+  int kps = tcb::plan(M, N, K).kps;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = g.grid; cfg.blockDim = g.block; cfg.dynamicSmemBytes = (size_t)g.smem; cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = 1; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = g.grid.z;
+  cfg.attrs = at; cfg.numAttrs = 1;
+  cudaError_t e;
   if (g.func == (const void*)tcb::gemm_bf16_kernel<128>)
-    tcb::gemm_bf16_kernel<128><<<g.grid, g.block, g.smem, s>>>(A, W, C, bias, M, N, K, sig);
+    e = cudaLaunchKernelEx(&cfg, tcb::gemm_bf16_kernel<128>, A, W, C, bias, M, N, K, kps, sig);
   else
-    tcb::gemm_bf16_kernel<64><<<g.grid, g.block, g.smem, s>>>(A, W, C, bias, M, N, K, sig);
-  CHECK_LAUNCH();
+    e = cudaLaunchKernelEx(&cfg, tcb::gemm_bf16_kernel<64>, A, W, C, bias, M, N, K, kps, sig);
+  return e == cudaSuccess ? 0 : ORION_E_CUDA;
 }
 
 // attention: args q, k, v, o, B, S, heads, head_dim, ld

@@ -119,11 +119,13 @@ static inline void log_dec(Instance* I, uint64_t k, int kind, int c, uint32_t ki
 // ------------------------------------------------------------------ policy pieces (Listing 1)
 // different profiles (L28, R1, R4): unknown on either side is compatible
 static inline bool profiles_differ(const Instance* I, uint8_t hp_cls, uint8_t be_cls) {
+  if (I->cfg.flags & ORION_F_NO_PROFILE_TEST) return true;   // ablation (Fig. 14)
   if (I->cfg.flags & ORION_F_HP_UNKNOWN_STRICT) return be_cls == ORION_CLS_U || (hp_cls != ORION_CLS_U && hp_cls != be_cls);
   return hp_cls == ORION_CLS_U || be_cls == ORION_CLS_U || hp_cls != be_cls;
 }
 // SM test (L27, R5): sm_needed < SM_THRESHOLD; FREE_SMS: sm_needed + hp.sm_needed <= num_sms
 static inline bool sm_fits(const Instance* I, const Prof& h, uint32_t sm_needed) {
+  if (I->cfg.flags & ORION_F_NO_SM_TEST) return true;        // ablation (Fig. 14)
   if (I->cfg.flags & ORION_F_FREE_SMS) return (uint64_t)sm_needed + h.sm_needed <= I->num_sms;
   return sm_needed < I->sm_thr;
 }
@@ -213,7 +215,7 @@ static void one_iteration(Instance* I, uint64_t k) {
     }
     int reason = schedule_be(I, busy, op);  // L11
     bool sched = reason == RSN_NONE;
-    const bool throttle = !(I->cfg.flags & ORION_F_THROTTLE_ONLY_HP_BUSY) || busy;  // R7
+    const bool throttle = !(I->cfg.flags & ORION_F_NO_THROTTLE) && (!(I->cfg.flags & ORION_F_THROTTLE_ONLY_HP_BUSY) || busy);  // R7
     if (throttle && I->be_dur > (int64_t)I->dur_thr) {                                // L12 (R6)
       if (be_all_finished(I)) {                                                       // L13
         I->be_dur = 0;                                                                // L14

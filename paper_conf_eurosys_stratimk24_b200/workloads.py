@@ -142,7 +142,7 @@ def conv_wgrad(g, x, dy, dw, stride, pad, label, depthwise=False):
         return g.k("dw_wgrad", [_p(x), _p(dy), _p(dw)] + conv_args(x, dw, dy, stride, pad) + [0, 0], label, ws_at=14)
     if r == 1 and s == 1 and stride == 1 and pad == 0:   # dW[K, C] = dy^T[K, NHW] x[NHW, C]
         return gemm(g, dy, x, dw, None, k, c, n * h * wd, k, c, c, 1, label)
-    g.need_ws(L.lib.orion_gemm_workspace_bytes(k, r * s * c, n * p * q))
+    g.need_ws(L.lib.orion_conv_wgrad_workspace_bytes(n, h, wd, c, k, r, s, stride, pad))
     return g.k("conv_wgrad", [_p(x), _p(dy), _p(dw)] + conv_args(x, dw, dy, stride, pad) + [0, 0], label, ws_at=14)
 
 

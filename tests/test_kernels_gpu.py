@@ -80,6 +80,9 @@ CONV_CASES = [  # N, H, W, C, K, R, stride, pad
     (2, 14, 14, 64, 70, 3, 1, 1),
     (2, 13, 13, 64, 128, 1, 2, 0),   # 1x1 / stride 2 downsample
     (3, 9, 11, 20, 24, 3, 2, 1),
+    (4, 64, 64, 3, 64, 7, 2, 3),     # ResNet stem (direct few-channel wgrad kernel)
+    (2, 224, 224, 3, 64, 7, 2, 3),   # ResNet stem at 224 (several tiles per CTA, ragged Q)
+    (3, 50, 38, 3, 32, 3, 2, 1),     # MobileNetV2 stem class, ragged
 ]
 
 
@@ -100,9 +103,12 @@ def test_conv_fwd_dgrad_wgrad(shape):
     run("conv_dgrad", [dev(dy), dev(wt), dx] + dims + [wd, wd.numel() * 4])
     assert rel(dx, om.conv2d_bwd_data(dy, wt, (n, h, w_, c), st, pad)) < 1e-5
     dw = torch.zeros(k, r, r, c, device="cuda")
-    wsb = ws(L.lib.orion_gemm_workspace_bytes(k, r * r * c, n * p * q))
+    wsb = ws(L.lib.orion_conv_wgrad_workspace_bytes(n, h, w_, c, k, r, r, st, pad))
     run("conv_wgrad", [dev(x), dev(dy), dw] + dims + [wsb, wsb.numel() * 4])
     assert rel(dw, om.conv2d_bwd_weight(x, dy, (k, r, r, c), st, pad)) < 1e-5
+    first = dw.clone()
+    run("conv_wgrad", [dev(x), dev(dy), dw] + dims + [wsb, wsb.numel() * 4])
+    assert torch.equal(first, dw), "non-deterministic conv wgrad"
 
 
 @pytest.mark.parametrize("n,h,c,st", [(2, 15, 32, 1), (3, 16, 96, 2), (2, 7, 960, 1), (1, 9, 8, 2)])

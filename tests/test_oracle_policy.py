@@ -33,7 +33,7 @@ def _op(kid, cls, sm, dur, kind=0, opf=0):
     return (kid, kind, opf, cls, sm, dur)
 
 
-ALL_FLAGS = [0, 1, 2, 4, 8, 16, 1 | 2, 2 | 16, 4 | 8, 31]
+ALL_FLAGS = [0, 1, 2, 4, 8, 16, 1 | 2, 2 | 16, 4 | 8, 31, 64, 128, 256, 64 | 128 | 256, 32 | 64 | 128 | 256, 128 | 2]
 
 
 @pytest.mark.parametrize("flags", ALL_FLAGS)

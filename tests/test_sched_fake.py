@@ -37,7 +37,8 @@ def _producer(o, cid, ops, rng, burst):
 
 @pytest.mark.parametrize("seed,flags,n_be", [(1, 0, 1), (2, 0, 2), (3, L.F_HP_BUSY_REQUEST | L.F_HP_REF_ALL, 1),
                                              (4, L.F_FREE_SMS, 2), (5, L.F_HP_UNKNOWN_STRICT | L.F_THROTTLE_ONLY_HP_BUSY, 1),
-                                             (6, 31, 3)])
+                                             (6, 31, 3), (7, L.POLICIES["priorities"], 2), (8, L.POLICIES["profiles"], 1),
+                                             (9, L.POLICIES["streams"], 2)])
 def test_fake_log_matches_oracle(seed, flags, n_be):
     rng = random.Random(seed)
     o = orion.Orion(backend=L.BACKEND_FAKE, hp_latency_ns=1_000_000, dur_threshold_ppm=25000, flags=flags,
