@@ -109,7 +109,12 @@ enum orion_fn {
      whose first maximum (row-major window order) is x[n,h,w,c]. args: x, dy, dx, N, H, W, C, P, Q.
      C % 4 == 0; P, Q must be the forward's output size (else ORION_E_INVAL). */
   ORION_FN_MAXPOOL_BWD = 30,
-  ORION_FN_COUNT = 31
+  /* fp32 col2im (adjoint of im2col): dx[n,h,w,c] = sum over taps (r, s) with h = p*stride - pad + r,
+     w = q*stride - pad + s of col[(n,p,q)][(r,s,c)]. With col = dy W (GEMM, W = OHWI weights as
+     [K][R*S*C]) it is the data gradient of a strided convolution. args: col, dx, N, H, W, C, R, S,
+     stride, pad, P, Q. C % 4 == 0; P, Q must be the conv's output size (else ORION_E_INVAL). */
+  ORION_FN_COL2IM = 31,
+  ORION_FN_COUNT = 32
 };
 
 /* Number of table entries, and a stable name for each (for profiles and logs). */

@@ -609,3 +609,16 @@ def out_hw(h, k, s, p):
 
 def logsumexp_uniform(c):
     return math.log(c)
+
+
+# ------------------------------------------------------------------------------- col2im
+def col2im(col, x_shape, R, S, stride, pad):
+    """col2im (the adjoint of im2col): dx[n,h,w,c] = sum over (p,q,r,s) with h = p*stride - pad + r,
+    w = q*stride - pad + s of col[n,p,q,r,s,c]. col [N*P*Q, R*S*C] (rows (n,p,q), columns (r,s,c)
+    with c fastest), dx NHWC. With col = dy W (W as [K, R*S*C]) this is the data gradient of a
+    convolution, the form liborion uses for strided convs. torch's fold = col2im."""
+    n, h, w, c = x_shape
+    p, q = (h + 2 * pad - R) // stride + 1, (w + 2 * pad - S) // stride + 1
+    cd = _d(col).view(n, p * q, R, S, c).permute(0, 4, 2, 3, 1).reshape(n, c * R * S, p * q)
+    dx = F.fold(cd, (h, w), (R, S), padding=pad, stride=stride)
+    return _r(_nhwc(dx))

@@ -186,3 +186,4 @@ ENTRY_DECL(gelu)
 ENTRY_DECL(add_bf16)
 ENTRY_DECL(embed)
 ENTRY_DECL(maxpool_bwd)
+ENTRY_DECL(col2im)

@@ -1761,7 +1761,7 @@ Plan plan_gemm(long long M, long long N, long long K) {
     if (tiles < 148) {              // one CTA per SM (~196 KB smem each): fill a 148-SM part once,
       split = 148 / tiles;          // never spilling into a second wave
       if (split > ktiles / 4) split = ktiles / 4;   // >= 4 k-tiles per split
-      if (split > 16) split = 16;                   // bounded ordered reduction (<= 512 KB per tile)
+      if (split > 128) split = 128;                 // ordered two-level reduction (split_finish) beyond 32
       if (split < 1) split = 1;
     }
     pl.split = (int)split;
@@ -1921,15 +1921,19 @@ inline bool fwd_ok(const ConvShape& s) { return s.C == 3 && s.R == 3 && s.S == 3
 // (the next tile's loads held in registers while the current one is multiplied), and each thread
 // owns a 4 (k) x <= WG_MAXR (rsc) register block. Partials (fp64) of the G CTAs (a shape-only
 // count) are combined in CTA order (combine_splits), so results are deterministic.
-constexpr int WG_QT = 32, WG_KPT = 4, WG_MAXR = 12, WG_G = 148;   // one CTA per SM of a full B200 (~166 registers)
+constexpr int WG_QT = 32, WG_KPT = 4, WG_MAXR = 10, WG_G = 296;   // two CTAs per SM of a full B200
 constexpr int WG_PF_DY = WG_QT * MAXK / 4 / NTH, WG_PF_X = 8;   // per-thread prefetch registers
 __host__ __device__ inline int wg_wwin(const ConvShape& s) { return (WG_QT - 1) * s.stride + s.S; }
 __host__ __device__ inline int wg_xwin(const ConvShape& s) { return s.R * wg_wwin(s) * s.C; }
 inline long long wg_tiles(const ConvShape& s) { return (long long)s.N * s.P * ((s.Q + WG_QT - 1) / WG_QT); }
 inline int wg_ctas(const ConvShape& s) { return (int)(wg_tiles(s) < WG_G ? wg_tiles(s) : WG_G); }
+// register-block width (rsc per thread) of the launch: 10 for the ResNet stem (147 / 16 groups)
+inline int wg_nr(const ConvShape& s) { return (s.R * s.S * s.C + NTH / (s.K / WG_KPT) - 1) / (NTH / (s.K / WG_KPT)); }
+// Taken for the large stems (R*S*C >= 64, e.g. ResNet's 7x7x3); the 3x3x3 MobileNetV2 stem has too
+// few products per staged value and stays on the tiled split-K path.
 inline bool wgrad_ok(const ConvShape& s) {
   const int kg = s.K / WG_KPT, rsc = s.R * s.S * s.C;
-  return s.C <= 4 && s.K % WG_KPT == 0 && s.K <= MAXK && (kg & (kg - 1)) == 0 && rsc <= (NTH / kg) * WG_MAXR &&
+  return s.C <= 4 && s.K % WG_KPT == 0 && s.K <= MAXK && (kg & (kg - 1)) == 0 && rsc >= 64 && wg_nr(s) >= 8 && wg_nr(s) <= WG_MAXR &&
          wg_xwin(s) <= NTH * WG_PF_X && s.stride <= 2;
 }
 inline uint64_t wgrad_ws_bytes(const ConvShape& s) {
@@ -1938,30 +1942,31 @@ inline uint64_t wgrad_ws_bytes(const ConvShape& s) {
   return WS_TICKET_BYTES + (uint64_t)(G + combine_rows(G) + 1) * V * 8;
 }
 
-__global__ void __launch_bounds__(NTH, 1) conv_wgrad_smallc_kernel(const float* __restrict__ x, const float* __restrict__ dy,
-                                                                float* __restrict__ dw, ConvShape s, unsigned char* ws, OrionSig sig) {
+template <int NR>
+__global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc_kernel(const float* __restrict__ x, const float* __restrict__ dy,
+                                                                   float* __restrict__ dw, ConvShape s, unsigned char* ws, OrionSig sig) {
   extern __shared__ __align__(16) float wsm[];
   const int K = s.K, RSC = s.R * s.S * s.C, WW = wg_wwin(s), XW = wg_xwin(s);
   float* dys = wsm;                      // [WG_QT][K]
   float* xs = wsm + WG_QT * K;           // [R][WW][C]
   const int kgroups = K / WG_KPT, rgroups = NTH / kgroups;
   const int kg = threadIdx.x % kgroups, rg = threadIdx.x / kgroups;
-  int off[WG_MAXR];
+  int off[NR];
 #pragma unroll
-  for (int i = 0; i < WG_MAXR; i++) {
+  for (int i = 0; i < NR; i++) {
     const int j = rg + rgroups * i;
     if (j < RSC) {
       const int c = j % s.C, t = j / s.C, u = t % s.S, r = t / s.S;
       off[i] = (r * WW + u) * s.C + c;
     } else {
-      off[i] = -1;
+      off[i] = 0;   // padding slot: accumulates garbage that is never stored (no branch in the hot loop)
     }
   }
-  float acc[WG_KPT][WG_MAXR];
+  float acc[WG_KPT][NR];
 #pragma unroll
   for (int a = 0; a < WG_KPT; a++)
 #pragma unroll
-    for (int i = 0; i < WG_MAXR; i++) acc[a][i] = 0.f;
+    for (int i = 0; i < NR; i++) acc[a][i] = 0.f;
   const int qtiles = (s.Q + WG_QT - 1) / WG_QT;
   const long long T = (long long)s.N * s.P * qtiles;
   float4 pdy[WG_PF_DY];
@@ -2011,14 +2016,12 @@ __global__ void __launch_bounds__(NTH, 1) conv_wgrad_smallc_kernel(const float* 
       const float4 d = *reinterpret_cast<const float4*>(dys + i * K + kg * WG_KPT);
       const float* xr = xs + i * xstep;
 #pragma unroll
-      for (int j = 0; j < WG_MAXR; j++) {
-        if (off[j] >= 0) {
-          const float xv = xr[off[j]];
-          acc[0][j] = fmaf(d.x, xv, acc[0][j]);
-          acc[1][j] = fmaf(d.y, xv, acc[1][j]);
-          acc[2][j] = fmaf(d.z, xv, acc[2][j]);
-          acc[3][j] = fmaf(d.w, xv, acc[3][j]);
-        }
+      for (int j = 0; j < NR; j++) {
+        const float xv = xr[off[j]];
+        acc[0][j] = fmaf(d.x, xv, acc[0][j]);
+        acc[1][j] = fmaf(d.y, xv, acc[1][j]);
+        acc[2][j] = fmaf(d.z, xv, acc[2][j]);
+        acc[3][j] = fmaf(d.w, xv, acc[3][j]);
       }
     }
   }
@@ -2030,7 +2033,7 @@ __global__ void __launch_bounds__(NTH, 1) conv_wgrad_smallc_kernel(const float* 
   double* gpart = part + (long long)G * V;
   double* out = gpart + (long long)combine_rows(G) * V;
 #pragma unroll
-  for (int j = 0; j < WG_MAXR; j++) {
+  for (int j = 0; j < NR; j++) {
     const int jj = rg + rgroups * j;
     if (jj < RSC) {
 #pragma unroll
@@ -2044,6 +2047,13 @@ __global__ void __launch_bounds__(NTH, 1) conv_wgrad_smallc_kernel(const float* 
   orion_signal(sig);
 }
 #undef WG_FETCH
+inline const void* wgrad_fn(const ConvShape& s) {
+  switch (wg_nr(s)) {
+    case 8: return (const void*)conv_wgrad_smallc_kernel<8>;
+    case 9: return (const void*)conv_wgrad_smallc_kernel<9>;
+    default: return (const void*)conv_wgrad_smallc_kernel<10>;
+  }
+}
 }  // namespace smallc
 
 }  // namespace
@@ -2229,16 +2239,9 @@ extern "C" uint64_t orion_conv_wgrad_workspace_bytes(uint64_t N, uint64_t H, uin
 int conv_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
   ConvShape s = conv_shape(a);
   if (smallc::wgrad_ok(s) && a[14] != 0 && a[15] >= smallc::wgrad_ws_bytes(s)) {
-    static std::atomic<int> attr{0};
-    const int smem = (smallc::WG_QT * s.K + smallc::wg_xwin(s)) * 4;
-    if (!attr.load()) {
-      if (cudaFuncSetAttribute((const void*)smallc::conv_wgrad_smallc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 48 * 1024) !=
-          cudaSuccess)
-        return ORION_E_CUDA;
-      attr.store(1);
-    }
-    g->grid = dim3((unsigned)smallc::wg_ctas(s)); g->block = dim3(smallc::NTH); g->smem = smem;
-    g->func = (const void*)smallc::conv_wgrad_smallc_kernel;
+    g->grid = dim3((unsigned)smallc::wg_ctas(s)); g->block = dim3(smallc::NTH);
+    g->smem = (smallc::WG_QT * s.K + smallc::wg_xwin(s)) * 4;   // <= 24 KB
+    g->func = smallc::wgrad_fn(s);
     return 0;
   }
   tiled_geom<ADenseT, BWgrad>(g, s.K, (long long)s.R * s.S * s.C, (long long)s.N * s.P * s.Q, a[14], a[15]);
@@ -2246,9 +2249,14 @@ int conv_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
 }
 int conv_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   ConvShape s = conv_shape(a);
-  if (g.func == (const void*)smallc::conv_wgrad_smallc_kernel) {
-    smallc::conv_wgrad_smallc_kernel<<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s,
-                                                                       (unsigned char*)a[14], sig);
+  if (smallc::wgrad_ok(s) && g.func == smallc::wgrad_fn(s)) {
+    const float* x = (const float*)a[0]; const float* dy = (const float*)a[1]; float* dw = (float*)a[2];
+    unsigned char* ws = (unsigned char*)a[14];
+    switch (smallc::wg_nr(s)) {
+      case 8: smallc::conv_wgrad_smallc_kernel<8><<<g.grid, g.block, g.smem, st>>>(x, dy, dw, s, ws, sig); break;
+      case 9: smallc::conv_wgrad_smallc_kernel<9><<<g.grid, g.block, g.smem, st>>>(x, dy, dw, s, ws, sig); break;
+      default: smallc::conv_wgrad_smallc_kernel<10><<<g.grid, g.block, g.smem, st>>>(x, dy, dw, s, ws, sig); break;
+    }
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
   long long M = s.K, N = (long long)s.R * s.S * s.C, K = (long long)s.N * s.P * s.Q;

@@ -34,6 +34,7 @@ const KernelEntry g_kernels[ORION_FN_COUNT] = {
     E(add_bf16, add_bf16, 4),
     E(embed, embed, 9),
     E(maxpool_bwd, maxpool_bwd, 9),
+    E(col2im, col2im, 12),
 };
 #undef E
 

@@ -3,10 +3,8 @@
 // ResNet training client (BE of config 3).
 //
 //  * gemm_bf16: y = x W^T + b on the 5th-gen tensor cores (tcgen05.mma kind::f16, bf16 operands,
-//    fp32 accumulator in TMEM), operands staged by cp.async into the UMMA K-major core-matrix
-//    layout, an 8-10-stage mbarrier pipeline, one elected MMA thread; BERT's few-tile shapes are
-//    split over K across a thread-block cluster and reduced in rank order through distributed
-//    shared memory; epilogue TMEM -> registers -> bias -> bf16 (round to nearest even).
+//    fp32 accumulator in TMEM), operands brought in by TMA (128-byte swizzle) through a 6-8 stage
+//    mbarrier ring, one elected MMA thread; epilogue TMEM -> registers -> bias -> bf16 (RNE).
 //  * attention: fused scaled-dot-product attention (the one SDPA kernel PyTorch dispatches),
 //    per (batch, head, 64-query block); Q K^T and P V on mma.sync m16n8k16 bf16 with fp32
 //    accumulators, softmax in fp32 registers, P rounded to bf16 for the second product (what a
@@ -17,6 +15,7 @@
 //    windows whose first maximum it is, in fixed order; no atomics, so deterministic.
 // Every kernel computes each output in one thread (or one warp) in a fixed order: outputs are
 // bitwise identical solo and collocated.
+#include <cuda.h>
 #include <cuda_bf16.h>
 #include <float.h>
 #include <atomic>
@@ -46,15 +45,24 @@ __device__ __forceinline__ uint4 pack8(const float* f) {
 }
 
 // =============================================================================== gemm_bf16
+// TMA-fed tcgen05 GEMM: one thread issues two 2-D tensor copies per stage (A: 128 x 64 bf16, W:
+// BN x 64 bf16, 128-byte swizzle, zero fill out of bounds) onto an mbarrier with an expected byte
+// count; one thread issues 4 tcgen05.mma (K = 16 each) per stage from the swizzled tiles and
+// commits the stage back to the producer; four epilogue warps read the fp32 accumulator from
+// TMEM, add the bias (staged in shared memory once), round to bf16 and store through a padded
+// shared tile with coalesced 16-byte row stores. One output tile per CTA, fixed k order.
 namespace tcb {
 
-constexpr int BM = 128, BK = 32, NPROD = 128, NTHR = 160;   // 4 producer / epilogue warps + 1 MMA warp
+constexpr int BM = 128, BK = 64, NTHR = 192;   // warps 0-3 epilogue, 4 TMA producer, 5 MMA issuer / TMEM owner
+constexpr int TMA_WARP = 4, MMA_WARP = 5;
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint32_t a, uint32_t cnt) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(cnt) : "memory");
 }
-__device__ __forceinline__ void mbar_arrive(uint32_t a) { asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(a) : "memory"); }
+__device__ __forceinline__ void mbar_expect(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
 __device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity) {
   uint32_t ok = 0;
   while (!ok) {
@@ -62,18 +70,15 @@ __device__ __forceinline__ void mbar_wait(uint32_t a, uint32_t parity) {
                  : "=r"(ok) : "r"(a), "r"(parity) : "memory");
   }
 }
-__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, bool ok) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(dst), "l"(ok ? src : (const void*)&cp_async16), "r"(ok ? 16 : 0)
-               : "memory");
+__device__ __forceinline__ void tma2d(uint32_t dst, const CUtensorMap* tm, int c0, int c1, uint32_t bar) {
+  asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(dst), "l"(tm),
+               "r"(c0), "r"(c1), "r"(bar) : "memory");
 }
-__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N_>
-__device__ __forceinline__ void cp_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N_) : "memory"); }
-// UMMA shared-memory descriptor, K-major, no swizzle (version 1): LBO = byte distance between the
-// two 16-byte K halves of a 32-byte K step, SBO = distance between 8-row core-matrix groups.
-__device__ __forceinline__ uint64_t sdesc(uint32_t addr, uint32_t lbo, uint32_t sbo) {
-  return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) | ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) |
-         (1ull << 46);
+// UMMA descriptor, K-major SWIZZLE_128B: 8-row atoms of 128-byte rows (64 bf16), SBO = 1024 B between
+// atoms, LBO unused (1), version 1 (bit 46), layout type 2 (bits 61-63); K step j (16 bf16 = 32 B)
+// advances the start address by 32 B inside the swizzle atom.
+__device__ __forceinline__ uint64_t sdesc128(uint32_t addr) {
+  return (uint64_t)((addr >> 4) & 0x3FFF) | (1ull << 16) | ((uint64_t)(1024 >> 4) << 32) | (1ull << 46) | (2ull << 61);
 }
 __device__ __forceinline__ void mma_bf16(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
   asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}"
@@ -100,141 +105,78 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
 template <int BN>
 struct Cfg {
   static constexpr int A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2, STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES = BN == 64 ? 10 : 8;   // 160 / 192 KB of operand stages per CTA
-  static constexpr int RED_LD = BN + 4;              // padded fp32 partial row (split-K reduction)
-  static constexpr int RED_BYTES = BM * RED_LD * 4;
-  static constexpr int MAIN = STAGES * STAGE_BYTES > RED_BYTES ? STAGES * STAGE_BYTES : RED_BYTES;
-  static constexpr int SMEM = MAIN + 256 + 1024;
-  static constexpr int TMEM_COLS = BN < 32 ? 32 : BN;
+  static constexpr int STAGES = (192 * 1024) / STAGE_BYTES;   // 6 (BN 128) / 8 (BN 64)
+  static constexpr int EPI_LD = BN + 8;                        // padded bf16 staging row
+  static constexpr int EPI_BYTES = BM * EPI_LD * 2;
+  static constexpr int MAIN = STAGES * STAGE_BYTES > EPI_BYTES ? STAGES * STAGE_BYTES : EPI_BYTES;
+  static constexpr int SMEM = MAIN + BN * 4 + 256 + 1024;
+  static constexpr int TMEM_COLS = BN;
+  static constexpr uint32_t TX = STAGE_BYTES;
   // instruction descriptor (kind::f16): D f32 (bits 4-5 = 1), A bf16 (bits 7-9 = 1), B bf16 (bits
   // 10-12 = 1), both K-major, N >> 3 at bits 17-22, M >> 4 at bits 24-28
   static constexpr uint32_t IDESC = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
 };
 
-// Byte offset of chunk kq (8 consecutive bf16 = 16 bytes; 4 chunks per 32-element stage row) of
-// operand row `row` in a stage buffer of `rows` rows: MMA K step j = kq / 2 (16 bf16 = 32 bytes,
-// rows x 32 B), core matrices of 8 rows x 16 B: row-group stride 256 B, K-half stride 128 B.
-__device__ __forceinline__ uint32_t elem_off(int row, int kq, int rows) {
-  return (uint32_t)((kq >> 1) * (rows * 32) + (row >> 3) * 256 + (kq & 1) * 128 + (row & 7) * 16);
-}
-__device__ __forceinline__ uint32_t cluster_rank() {
-  uint32_t r;
-  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
-  return r;
-}
-__device__ __forceinline__ void cluster_sync() {
-  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-__device__ __forceinline__ float4 ld_dsmem4(uint32_t local_addr, uint32_t rank) {
-  uint32_t ra;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(local_addr), "r"(rank));
-  float4 v;
-  asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(ra) : "memory");
-  return v;
-}
-
-// Split-K over a thread-block cluster: the `split` CTAs of a cluster (gridDim.z == cluster z) take
-// consecutive K ranges of the same output tile; each parks its fp32 partial tile in its own shared
-// memory, and after a cluster barrier rank 0 sums ranks 0, 1, .. in order through distributed
-// shared memory (ld.shared::cluster), adds the bias, rounds to bf16 and stores. No workspace, no
-// atomics, fixed summation order (the split is a function of the shape only).
 template <int BN>
-__global__ void __launch_bounds__(NTHR, 1) gemm_bf16_kernel(const bf16* __restrict__ A, const bf16* __restrict__ W, bf16* __restrict__ C,
-                                                           const bf16* __restrict__ bias, int M, int N, int K, int kps, OrionSig sig) {
+__global__ void __launch_bounds__(NTHR, 1) gemm_bf16_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmW,
+                                                           bf16* __restrict__ C, const bf16* __restrict__ bias, int M, int N, int K,
+                                                           OrionSig sig) {
   using Cf = Cfg<BN>;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   constexpr int S = Cf::STAGES;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + Cf::MAIN);
+  float* bias_s = reinterpret_cast<float*>(smem + Cf::MAIN);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + Cf::MAIN + BN * 4);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * S + 1);
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + S), done_bar = smem_u32(bars + 2 * S);
   const int tid = threadIdx.x, warp = tid / 32, lane = tid % 32;
   const int m0 = blockIdx.y * BM, n0 = blockIdx.x * BN;
-  const int split = gridDim.z;
-  const int kbeg = blockIdx.z * kps, kend = min(K, kbeg + kps);
-  const int nk = kend > kbeg ? (kend - kbeg + BK - 1) / BK : 0;
+  const int nk = (K + BK - 1) / BK;
 
   if (tid == 0) {
-    for (int s = 0; s < S; s++) { mbar_init(full0 + 8 * s, NPROD); mbar_init(empty0 + 8 * s, 1); }
+    for (int s = 0; s < S; s++) { mbar_init(full0 + 8 * s, 1); mbar_init(empty0 + 8 * s, 1); }
     mbar_init(done_bar, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == NPROD / 32) {
+  if (warp == MMA_WARP) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)), "r"(Cf::TMEM_COLS) : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
+  if (tid < BN) bias_s[tid] = (bias != nullptr && n0 + tid < N) ? bf2f(bias[n0 + tid]) : 0.f;
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   const uint32_t tmem = *tmem_slot;
 
-  if (warp < NPROD / 32) {
-    // producers: thread t copies A row t (4 chunks of 8 bf16) and B rows t (+128) of every stage
-    // with cp.async (zero-fill beyond M, N, K), S-2 stages in flight
-    const int a_row = tid;
-    const bool a_ok = m0 + a_row < M;
-    const bf16* a_src = A + (long long)(m0 + a_row) * K;
-    auto issue = [&](int kt) {
-      const int s = kt % S;
-      const uint32_t st = smem_u32(smem + s * Cf::STAGE_BYTES);
-      const int k0 = kbeg + kt * BK;
-#pragma unroll
-      for (int q = 0; q < 4; q++) {
-        const int k = k0 + 8 * q;
-        cp_async16(st + elem_off(a_row, q, BM), a_src + k, a_ok && k < kend);
-      }
-#pragma unroll
-      for (int r = tid; r < BN; r += NPROD) {
-        const bool ok = n0 + r < N;
-        const bf16* src = W + (long long)(n0 + r) * K;
-#pragma unroll
-        for (int q = 0; q < 4; q++) {
-          const int k = k0 + 8 * q;
-          cp_async16(st + Cf::A_BYTES + elem_off(r, q, BN), src + k, ok && k < kend);
-        }
-      }
-    };
-    constexpr int L = S - 2;
-#pragma unroll 1
-    for (int kt = 0; kt < L; kt++) {
-      if (kt < nk) issue(kt);
-      cp_commit();
-    }
-#pragma unroll 1
+  if (warp == TMA_WARP && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmW) : "memory");
     for (int kt = 0; kt < nk; kt++) {
-      const int nxt = kt + L;
-      if (nxt < nk) {
-        if (nxt >= S) mbar_wait(empty0 + 8 * (nxt % S), ((uint32_t)(nxt / S) & 1u) ^ 1u);
-        issue(nxt);
-      }
-      cp_commit();
-      cp_wait<L>();
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // cp.async writes -> tensor core
-      mbar_arrive(full0 + 8 * (kt % S));
+      const int s = kt % S;
+      if (kt >= S) mbar_wait(empty0 + 8 * s, ((uint32_t)(kt / S) & 1u) ^ 1u);
+      const uint32_t st = smem_u32(smem + s * Cf::STAGE_BYTES), bar = full0 + 8 * s;
+      mbar_expect(bar, Cf::TX);
+      tma2d(st, &tmA, kt * BK, m0, bar);
+      tma2d(st + Cf::A_BYTES, &tmW, kt * BK, n0, bar);
     }
-    cp_wait<0>();
-  } else if (lane == 0) {
-    // MMA issuer (one thread): two K steps of 16 per stage into one fp32 accumulator
+  } else if (warp == MMA_WARP && lane == 0) {
     for (int kt = 0; kt < nk; kt++) {
       const int s = kt % S;
       mbar_wait(full0 + 8 * s, (uint32_t)(kt / S) & 1u);
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       const uint32_t st = smem_u32(smem + s * Cf::STAGE_BYTES);
 #pragma unroll
-      for (int j = 0; j < BK / 16; j++) {
-        const uint64_t da = sdesc(st + j * BM * 32, 128, 256), db = sdesc(st + Cf::A_BYTES + j * BN * 32, 128, 256);
-        mma_bf16(tmem, da, db, Cf::IDESC, (kt | j) != 0);
-      }
+      for (int j = 0; j < BK / 16; j++)
+        mma_bf16(tmem, sdesc128(st + 32 * j), sdesc128(st + Cf::A_BYTES + 32 * j), Cf::IDESC, (kt | j) != 0);
       mma_commit(empty0 + 8 * s);
     }
     mma_commit(done_bar);
-  }
-
-  // epilogue (warps 0-3 = TMEM lanes 0-127 = tile rows): fp32 partial tile -> padded shared tile
-  float* red = reinterpret_cast<float*>(smem);
-  if (warp < 4) {
+  } else if (warp < 4) {
+    // epilogue (TMEM lanes 32w..32w+31 = tile rows): accumulator + bias -> bf16 -> padded shared
+    // tile -> coalesced 16-byte row stores
     mbar_wait(done_bar, 0);
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    bf16* tile = reinterpret_cast<bf16*>(smem);
 #pragma unroll 1
     for (int c0 = 0; c0 < BN; c0 += 32) {
       float v[32];
@@ -244,42 +186,27 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_bf16_kernel(const bf16* __restri
         for (int i = 0; i < 32; i++) v[i] = 0.f;
       }
 #pragma unroll
-      for (int i = 0; i < 32; i += 4)
-        *reinterpret_cast<float4*>(red + tid * Cf::RED_LD + c0 + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+      for (int i = 0; i < 32; i++) v[i] += bias_s[c0 + i];
+#pragma unroll
+      for (int i = 0; i < 32; i += 8) *reinterpret_cast<uint4*>(tile + tid * Cf::EPI_LD + c0 + i) = pack8(v + i);
     }
-  }
-  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
-  if (split > 1) cluster_sync(); else __syncthreads();
-  // rank 0 of the cluster: sum partials in rank order, + bias, bf16, coalesced 16-byte row stores
-  if ((split == 1 || cluster_rank() == 0) && tid < 128) {
-    constexpr int CPR = BN / 8;   // 16-byte output chunks per tile row
+    asm volatile("bar.sync 1, 128;" ::: "memory");
+    constexpr int CPR = BN / 8;
     const bool vec = (N % 8) == 0;
     for (int e = tid; e < BM * CPR; e += 128) {
       const int r = e / CPR, c = (e % CPR) * 8;
       const int m = m0 + r, n = n0 + c;
       if (m >= M || n >= N) continue;
-      const float* src = red + r * Cf::RED_LD + c;
-      float4 lo = *reinterpret_cast<const float4*>(src), hi = *reinterpret_cast<const float4*>(src + 4);
-      for (int z = 1; z < split; z++) {
-        const uint32_t la = smem_u32(src);
-        const float4 a = ld_dsmem4(la, (uint32_t)z), b = ld_dsmem4(la + 16, (uint32_t)z);
-        lo.x += a.x; lo.y += a.y; lo.z += a.z; lo.w += a.w;
-        hi.x += b.x; hi.y += b.y; hi.z += b.z; hi.w += b.w;
-      }
-      float f[8] = {lo.x, lo.y, lo.z, lo.w, hi.x, hi.y, hi.z, hi.w};
-      if (bias != nullptr) {
-#pragma unroll
-        for (int i = 0; i < 8; i++)
-          if (n + i < N) f[i] += bf2f(bias[n + i]);
-      }
+      const bf16* srcp = tile + r * Cf::EPI_LD + c;
       bf16* dst = C + (long long)m * N + n;
-      if (vec) *reinterpret_cast<uint4*>(dst) = pack8(f);
+      if (vec) *reinterpret_cast<uint4*>(dst) = *reinterpret_cast<const uint4*>(srcp);
       else
-        for (int i = 0; i < 8 && n + i < N; i++) dst[i] = __float2bfloat16_rn(f[i]);
+        for (int i = 0; i < 8 && n + i < N; i++) dst[i] = srcp[i];
     }
   }
-  if (split > 1) cluster_sync();   // partials stay alive until rank 0 has read them
-  if (warp == NPROD / 32) {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == MMA_WARP) {
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(Cf::TMEM_COLS) : "memory");
   }
@@ -295,24 +222,32 @@ bool prepare() {
   if (ok) done.store(1, std::memory_order_release);
   return ok;
 }
-// Shape-only plan (never the SM partition): tile width BN in {64, 128} and cluster split-K s in
-// {1..4} minimising waves x per-CTA stream (k-tiles x bytes per stage) over a 148-SM part, >= 4
-// k-tiles per split.
-struct Plan { int bn, split, kps; };
-inline Plan plan(long long M, long long N, long long K) {
-  const long long kt = cdiv(K, BK);
-  Plan best{64, 1, (int)K};
-  double best_cost = 1e30;
-  for (int bn = 64; bn <= 128; bn *= 2) {
-    const long long tiles = cdiv(M, BM) * cdiv(N, bn);
-    for (int sp = 1; sp <= 4; sp++) {
-      if (sp > 1 && kt / sp < 4) break;
-      const long long kts = cdiv(kt, sp);
-      const double cost = (double)cdiv(tiles * sp, 148) * (double)kts * (double)(BM + bn) + (sp > 1 ? 3.0 * (sp - 1) * (BM + bn) : 0.0);
-      if (cost < best_cost) { best_cost = cost; best = Plan{bn, sp, (int)(kts * BK)}; }
-    }
-  }
-  return best;
+// Tile width from the shape only (never the SM partition): 128 when that still gives >= one CTA
+// per SM of a whole B200, else 64 (twice the CTAs for BERT-base's N = 768 projections).
+inline int bn_for(long long M, long long N) { return cdiv(M, BM) * cdiv(N, 128) >= 148 ? 128 : 64; }
+
+// cuTensorMapEncodeTiled through cudart's driver entry point (liborion does not link libcuda)
+typedef CUresult (*encode_fn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                              const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+inline encode_fn encoder() {
+  static encode_fn fn = [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPointByVersion("cuTensorMapEncodeTiled", &p, 12000, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return (encode_fn) nullptr;
+    return (encode_fn)p;
+  }();
+  return fn;
+}
+// bf16 row-major [rows][K], box {64, box_rows}, 128-byte swizzle, out-of-bounds zero fill
+inline bool map_bf16(CUtensorMap* m, const void* base, long long rows, long long K, int box_rows) {
+  cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)K * 2};
+  cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)box_rows};
+  cuuint32_t es[2] = {1, 1};
+  return encoder()(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
 }  // namespace tcb
@@ -588,6 +523,41 @@ __global__ void __launch_bounds__(TB) maxpool_bwd_kernel(const float* __restrict
   orion_signal(sig);
 }
 
+// =============================================================================== col2im (fp32)
+// dx[n,h,w,c] = sum over taps (r, s) with h = p*stride - pad + r, w = q*stride - pad + s (p, q in
+// range) of col[(n,p,q)][(r,s,c)]: the second half of a strided convolution's data gradient
+// (col = dy W is a dense GEMM). Thread per (n, h, w, 4 channels); taps visited in (r, s) order.
+__global__ void __launch_bounds__(TB) col2im_kernel(const float* __restrict__ col, float* __restrict__ dx, int N, int H, int W, int C, int R,
+                                                   int S, int st, int pad, int P, int Q, OrionSig sig) {
+  const int C4 = C / 4;
+  const long long total = (long long)N * H * W * C4;
+  const long long rsc = (long long)R * S * C;
+  for (long long i = (long long)blockIdx.x * TB + threadIdx.x; i < total; i += (long long)gridDim.x * TB) {
+    const int c = (int)(i % C4) * 4;
+    long long t = i / C4;
+    const int w = (int)(t % W); t /= W;
+    const int h = (int)(t % H);
+    const int n = (int)(t / H);
+    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int r = 0; r < R; r++) {
+      const int ph = h + pad - r;
+      if (ph < 0 || ph % st) continue;
+      const int p = ph / st;
+      if (p >= P) continue;
+      for (int s = 0; s < S; s++) {
+        const int pw = w + pad - s;
+        if (pw < 0 || pw % st) continue;
+        const int q = pw / st;
+        if (q >= Q) continue;
+        const float4 v = __ldg(reinterpret_cast<const float4*>(col + (((long long)n * P + p) * Q + q) * rsc + ((long long)r * S + s) * C + c));
+        acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+      }
+    }
+    *reinterpret_cast<float4*>(dx + (((long long)n * H + h) * W + w) * C + c) = acc;
+  }
+  orion_signal(sig);
+}
+
 inline bool al16(uint64_t p) { return (p & 15) == 0; }
 
 }  // namespace
@@ -597,10 +567,11 @@ inline bool al16(uint64_t p) { return (p & 15) == 0; }
 int gemm_bf16_geom(const uint64_t* a, LaunchGeom* g) {
   const long long M = (long long)a[4], N = (long long)a[5], K = (long long)a[6];
   if (M <= 0 || N <= 0 || K <= 0 || (K % 8) != 0 || !al16(a[0]) || !al16(a[1]) || !al16(a[2])) return ORION_E_INVAL;
-  const tcb::Plan pl = tcb::plan(M, N, K);
-  g->grid = dim3((unsigned)cdiv(N, pl.bn), (unsigned)cdiv(M, tcb::BM), (unsigned)pl.split);
+  if (tcb::encoder() == nullptr) return ORION_E_CUDA;
+  const int bn = tcb::bn_for(M, N);
+  g->grid = dim3((unsigned)cdiv(N, bn), (unsigned)cdiv(M, tcb::BM));
   g->block = dim3(tcb::NTHR);
-  if (pl.bn == 128) {
+  if (bn == 128) {
     if (!tcb::prepare<128>()) return ORION_E_CUDA;
     g->smem = tcb::Cfg<128>::SMEM; g->func = (const void*)tcb::gemm_bf16_kernel<128>;
   } else {
@@ -610,21 +581,16 @@ int gemm_bf16_geom(const uint64_t* a, LaunchGeom* g) {
   return 0;
 }
 int gemm_bf16_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
-  const bf16* A = (const bf16*)a[0]; const bf16* W = (const bf16*)a[1]; bf16* C = (bf16*)a[2]; const bf16* bias = (const bf16*)a[3];
-  int M = (int)a[4], N = (int)a[5], K = (int)a[6];
-  int kps = tcb::plan(M, N, K).kps;
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = g.grid; cfg.blockDim = g.block; cfg.dynamicSmemBytes = (size_t)g.smem; cfg.stream = s;
-  cudaLaunchAttribute at[1];
-  at[0].id = cudaLaunchAttributeClusterDimension;
-  at[0].val.clusterDim.x = 1; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = g.grid.z;
-  cfg.attrs = at; cfg.numAttrs = 1;
-  cudaError_t e;
-  if (g.func == (const void*)tcb::gemm_bf16_kernel<128>)
-    e = cudaLaunchKernelEx(&cfg, tcb::gemm_bf16_kernel<128>, A, W, C, bias, M, N, K, kps, sig);
+  const long long M = (long long)a[4], N = (long long)a[5], K = (long long)a[6];
+  const bool wide = g.func == (const void*)tcb::gemm_bf16_kernel<128>;
+  CUtensorMap ma, mw;
+  if (!tcb::map_bf16(&ma, (const void*)a[0], M, K, tcb::BM) || !tcb::map_bf16(&mw, (const void*)a[1], N, K, wide ? 128 : 64))
+    return ORION_E_CUDA;
+  if (wide)
+    tcb::gemm_bf16_kernel<128><<<g.grid, g.block, g.smem, s>>>(ma, mw, (bf16*)a[2], (const bf16*)a[3], (int)M, (int)N, (int)K, sig);
   else
-    e = cudaLaunchKernelEx(&cfg, tcb::gemm_bf16_kernel<64>, A, W, C, bias, M, N, K, kps, sig);
-  return e == cudaSuccess ? 0 : ORION_E_CUDA;
+    tcb::gemm_bf16_kernel<64><<<g.grid, g.block, g.smem, s>>>(ma, mw, (bf16*)a[2], (const bf16*)a[3], (int)M, (int)N, (int)K, sig);
+  CHECK_LAUNCH();
 }
 
 // attention: args q, k, v, o, B, S, heads, head_dim, ld
@@ -721,5 +687,21 @@ int maxpool_bwd_geom(const uint64_t* a, LaunchGeom* g) {
 int maxpool_bwd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   maxpool_bwd_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (const float*)a[1], (float*)a[2], (int)a[3], (int)a[4], (int)a[5],
                                                 (int)a[6], (int)a[7], (int)a[8], sig);
+  CHECK_LAUNCH();
+}
+
+// col2im: args col, dx, N, H, W, C, R, S, stride, pad, P, Q   (C % 4 == 0)
+int col2im_geom(const uint64_t* a, LaunchGeom* g) {
+  const long long N = (long long)a[2], H = (long long)a[3], W = (long long)a[4], C = (long long)a[5];
+  const long long R = (long long)a[6], S = (long long)a[7], st = (long long)a[8], pad = (long long)a[9];
+  if (N <= 0 || H <= 0 || W <= 0 || C <= 0 || C % 4 || R <= 0 || S <= 0 || st <= 0 || pad < 0 || !al16(a[0]) || !al16(a[1]))
+    return ORION_E_INVAL;
+  if ((long long)a[10] != (H + 2 * pad - R) / st + 1 || (long long)a[11] != (W + 2 * pad - S) / st + 1) return ORION_E_INVAL;
+  vec_geom(g, (uint64_t)(N * H * W * C / 4), (const void*)col2im_kernel);
+  return 0;
+}
+int col2im_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
+  col2im_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (float*)a[1], (int)a[2], (int)a[3], (int)a[4], (int)a[5], (int)a[6], (int)a[7],
+                                           (int)a[8], (int)a[9], (int)a[10], (int)a[11], sig);
   CHECK_LAUNCH();
 }

@@ -153,6 +153,10 @@ def check_op(fn, a, R, snap=None, R_in=None):
         n, h, w, c, p, q = a[3:9]
         x, dy = T(a[0], n * h * w * c, (n, h, w, c)), T(a[1], n * p * q * c, (n, p, q, c))
         return rel(R.get(a[2], n * h * w * c, (n, h, w, c)), om.maxpool3x3s2_bwd(x, dy))
+    if fn == "col2im":
+        n, h, w, c, r, s_, st, pad, p, q = a[2:12]
+        col = T(a[0], n * p * q * r * s_ * c, (n * p * q, r * s_ * c))
+        return rel(R.get(a[1], n * h * w * c, (n, h, w, c)), om.col2im(col, (n, h, w, c), r, s_, st, pad))
     if fn == "colsum":
         M, N = a[2], a[3]
         return rel(R.get(a[1], N), om._r(T(a[0], M * N, (M, N)).double().sum(0)))

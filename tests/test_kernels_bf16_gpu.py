@@ -115,3 +115,15 @@ def test_maxpool_bwd(n, h, w, c):
     xt = torch.relu(x - 1.0)
     run("maxpool_bwd", [xt.cuda(), dy.cuda(), dx, n, h, w, c, p, q])
     assert rel(dx, om.maxpool3x3s2_bwd(xt, dy)) < 1e-6
+
+
+@pytest.mark.parametrize("n,h,w,c,k,st,pad", [(2, 56, 56, 256, 1, 2, 0), (2, 14, 14, 64, 3, 2, 1), (1, 9, 8, 4, 7, 2, 3),
+                                               (2, 13, 11, 8, 3, 2, 1)], ids=str)
+def test_col2im(n, h, w, c, k, st, pad):
+    """fp32 col2im (strided conv data gradient, second half): vs the oracle's fold, and the pair
+    GEMM + col2im vs the oracle's conv data gradient."""
+    p, q = (h + 2 * pad - k) // st + 1, (w + 2 * pad - k) // st + 1
+    col = si.normal((n * p * q, k * k * c), 63)
+    dx = torch.full((n, h, w, c), float("nan"), device="cuda")
+    run("col2im", [col.cuda(), dx, n, h, w, c, k, k, st, pad, p, q], twice=dx)
+    assert rel(dx, om.col2im(col, (n, h, w, c), k, k, st, pad)) < 1e-6

@@ -197,3 +197,28 @@ def test_resnet_train_step_vs_torchvision():
             torch.testing.assert_close(newP[k].double(), bufs[_rn_rename(k)], rtol=1e-5, atol=1e-6)
     k = "fc.w"
     torch.testing.assert_close(newP[k].double(), P[k].double() - 0.01 * named[_rn_rename(k)].grad, rtol=1e-5, atol=1e-7)
+
+
+# ------------------------------------------------------------------------------------ col2im
+@pytest.mark.parametrize("stride,pad,k", [(2, 1, 3), (2, 0, 1), (1, 1, 3), (2, 3, 7)])
+def test_col2im_is_conv_data_gradient(stride, pad, k):
+    """col2im(dy W) equals the convolution data gradient (adjoint identity), and an explicit loop."""
+    n, h, w, c, kout = 2, 9, 8, 4, 5
+    p, q = (h + 2 * pad - k) // stride + 1, (w + 2 * pad - k) // stride + 1
+    dy = _rand(n, p, q, kout, seed=71)
+    wt = _rand(kout, k, k, c, seed=72)
+    col = (dy.double().reshape(-1, kout) @ wt.double().reshape(kout, -1))
+    dx = om.col2im(col, (n, h, w, c), k, k, stride, pad)
+    ref = om.conv2d_bwd_data(dy, wt, (n, h, w, c), stride, pad)
+    torch.testing.assert_close(dx.double(), ref.double(), atol=1e-5, rtol=1e-5)
+    colv = col.view(n, p, q, k, k, c)
+    loop = torch.zeros(n, h, w, c, dtype=D)
+    for b in range(n):
+        for i in range(p):
+            for j in range(q):
+                for r in range(k):
+                    for s in range(k):
+                        hh, ww = i * stride - pad + r, j * stride - pad + s
+                        if 0 <= hh < h and 0 <= ww < w:
+                            loop[b, hh, ww] += colv[b, i, j, r, s]
+    torch.testing.assert_close(dx.double(), loop, atol=1e-5, rtol=1e-5)
