@@ -84,6 +84,8 @@ def test_be_rn50_one_iteration_vs_oracle(cfg3):
     assert not bad, sorted(bad.items(), key=lambda x: -x[1])[:10]
     for name in newP:
         floor = 1e-2 if name.endswith(".rmean") else 1e-30
+        if name.endswith(".beta"):   # starts at 0: the update is -lr * grad, floored like the gradient above
+            floor = 0.01 * float(g_ref[name.replace(".beta", ".gamma")].norm())
         tol = 1e-3 if name in stem else (3e-4 if name.endswith(".beta") else 1e-5)
         assert rel(G.p[name], newP[name], floor) < tol, name
     assert torch.equal(G.vflat, G.gflat)
