@@ -622,3 +622,117 @@ def col2im(col, x_shape, R, S, stride, pad):
     cd = _d(col).view(n, p * q, R, S, c).permute(0, 4, 2, 3, 1).reshape(n, c * R * S, p * q)
     dx = F.fold(cd, (h, w), (R, S), padding=pad, stride=stride)
     return _r(_nhwc(dx))
+
+
+# ============================================================ Transformer encoder training (fp32)
+# BE of BASELINE config 4 (reading R32): torch.nn.TransformerEncoderLayer stack,
+# post-LN (norm_first=False), ReLU FFN, dropout 0, batch_first; packed in-projection
+# (in_proj_weight [3d, d], as nn.MultiheadAttention); MSE loss to a target; SGD(momentum).
+# Every op computes in fp64 and rounds its output to fp32 (the unfused GPU op stream).
+
+def encoder_spec(layers=6, d=512, ffn=2048):
+    s = []
+    for i in range(layers):
+        p = f"enc{i}"
+        s += [(f"{p}.in.w", (3 * d, d), ("uniform_fan_in", d)), (f"{p}.in.b", (3 * d,), ("const", 0.0)),
+              (f"{p}.out.w", (d, d), ("uniform_fan_in", d)), (f"{p}.out.b", (d,), ("const", 0.0)),
+              (f"{p}.ln1.gamma", (d,), ("const", 1.0)), (f"{p}.ln1.beta", (d,), ("const", 0.0)),
+              (f"{p}.ff1.w", (ffn, d), ("uniform_fan_in", d)), (f"{p}.ff1.b", (ffn,), ("uniform_fan_in", d)),
+              (f"{p}.ff2.w", (d, ffn), ("uniform_fan_in", ffn)), (f"{p}.ff2.b", (d,), ("uniform_fan_in", ffn)),
+              (f"{p}.ln2.gamma", (d,), ("const", 1.0)), (f"{p}.ln2.beta", (d,), ("const", 0.0))]
+    return s
+
+
+def layernorm_fwd(x, gamma, beta, eps=1e-5):
+    """LayerNorm over the last dim (biased variance). Returns y, mean, rstd (the saved statistics
+    of the fused PyTorch kernel), each rounded to fp32."""
+    xd = _d(x)
+    mean = xd.mean(-1)
+    var = ((xd - mean[..., None]) ** 2).mean(-1)
+    rstd = 1.0 / torch.sqrt(var + eps)
+    y = (xd - mean[..., None]) * rstd[..., None] * _d(gamma) + _d(beta)
+    return _r(y), _r(mean), _r(rstd)
+
+
+def layernorm_bwd(x, dy, gamma, mean, rstd):
+    """Backward of LayerNorm from the saved fp32 mean / rstd: xhat = (x - mean) rstd;
+    dgamma = sum_rows dy xhat; dbeta = sum_rows dy; dx = rstd (g - mean(g) - xhat mean(g xhat))
+    with g = dy gamma."""
+    xd, dyd = _d(x), _d(dy)
+    xh = (xd - _d(mean)[..., None]) * _d(rstd)[..., None]
+    g = dyd * _d(gamma)
+    dx = _d(rstd)[..., None] * (g - g.mean(-1, keepdim=True) - xh * (g * xh).mean(-1, keepdim=True))
+    red = tuple(range(x.dim() - 1))
+    return _r(dx), _r((dyd * xh).sum(red)), _r(dyd.sum(red))
+
+
+def mha_fwd(q, k, v, heads):
+    """Scaled dot-product attention (no mask) per head on [B, S, H] views; fp32 output."""
+    return attention(q, k, v, heads, store=F32)
+
+
+def mha_bwd(q, k, v, do, heads):
+    """Backward of softmax(Q K^T / sqrt d) V per head: P recomputed in fp64;
+    dV = P^T dO, dP = dO V^T, dS = P (dP - rowsum(P dP)), dQ = dS K / sqrt d, dK = dS^T Q / sqrt d."""
+    b, sq, hd = q.shape
+    d = hd // heads
+
+    def split(t):
+        return _d(t).view(b, sq, heads, d).permute(0, 2, 1, 3)
+    Q, K, V, dO = split(q), split(k), split(v), split(do)
+    sc = Q @ K.transpose(-1, -2) / math.sqrt(d)
+    P = torch.softmax(sc, dim=-1)
+    dV = P.transpose(-1, -2) @ dO
+    dP = dO @ V.transpose(-1, -2)
+    dS = P * (dP - (P * dP).sum(-1, keepdim=True))
+    dQ = dS @ K / math.sqrt(d)
+    dK = dS.transpose(-1, -2) @ Q / math.sqrt(d)
+
+    def merge(t):
+        return _r(t.permute(0, 2, 1, 3).reshape(b, sq, hd))
+    return merge(dQ), merge(dK), merge(dV)
+
+
+def encoder_train_step(P, V, x, t, first, layers=6, heads=8, lr=0.01, momentum=0.9, eps=1e-5, masks=None):
+    """One training iteration of the post-LN encoder stack on x [B, S, d] with MSE to t.
+    masks (optional): {name: fp32 tensor} — the values the GPU's ReLU backward decided on (its FFN
+    pre-activations), as in the other training oracles. Returns (loss, newP, newV, grads)."""
+    b, sq, dm = x.shape
+    rows = b * sq
+    g = {}
+    recs = []
+    h = x.reshape(rows, dm)
+    for i in range(layers):
+        p = f"enc{i}"
+        qkv = linear_fwd(h, P[f"{p}.in.w"], P[f"{p}.in.b"])                 # [rows, 3d]
+        q, k, v = (qkv[:, j * dm:(j + 1) * dm].reshape(b, sq, dm) for j in range(3))
+        a = mha_fwd(q, k, v, heads).reshape(rows, dm)
+        o = linear_fwd(a, P[f"{p}.out.w"], P[f"{p}.out.b"])
+        s1 = add(h, o)
+        h1, m1, r1 = layernorm_fwd(s1, P[f"{p}.ln1.gamma"], P[f"{p}.ln1.beta"], eps)
+        f = linear_fwd(h1, P[f"{p}.ff1.w"], P[f"{p}.ff1.b"])
+        fa = relu(f)
+        f2 = linear_fwd(fa, P[f"{p}.ff2.w"], P[f"{p}.ff2.b"])
+        s2 = add(h1, f2)
+        h2, m2, r2 = layernorm_fwd(s2, P[f"{p}.ln2.gamma"], P[f"{p}.ln2.beta"], eps)
+        recs.append((h, q, k, v, a, s1, h1, m1, r1, f, fa, s2, m2, r2))
+        h = h2
+    loss, dh = mse_fwd_bwd(h, t.reshape(rows, dm))
+    for i in reversed(range(layers)):
+        p = f"enc{i}"
+        hin, q, k, v, a, s1, h1, m1, r1, f, fa, s2, m2, r2 = recs[i]
+        ds2, g[f"{p}.ln2.gamma"], g[f"{p}.ln2.beta"] = layernorm_bwd(s2, dh, P[f"{p}.ln2.gamma"], m2, r2)
+        dfa, g[f"{p}.ff2.w"], g[f"{p}.ff2.b"] = linear_bwd(fa, P[f"{p}.ff2.w"], ds2)
+        df = relu_bwd(masks[f"{p}.ff1"] if masks is not None else f, dfa)
+        dh1_ff, g[f"{p}.ff1.w"], g[f"{p}.ff1.b"] = linear_bwd(h1, P[f"{p}.ff1.w"], df)
+        dh1 = add(ds2, dh1_ff)
+        ds1, g[f"{p}.ln1.gamma"], g[f"{p}.ln1.beta"] = layernorm_bwd(s1, dh1, P[f"{p}.ln1.gamma"], m1, r1)
+        da, g[f"{p}.out.w"], g[f"{p}.out.b"] = linear_bwd(a, P[f"{p}.out.w"], ds1)
+        dq, dk, dv = mha_bwd(q, k, v, da.reshape(b, sq, dm), heads)
+        dqkv = torch.cat([dq.reshape(rows, dm), dk.reshape(rows, dm), dv.reshape(rows, dm)], dim=1)
+        dhin_attn, g[f"{p}.in.w"], g[f"{p}.in.b"] = linear_bwd(hin, P[f"{p}.in.w"], dqkv)
+        dh = add(ds1, dhin_attn)
+    newP, newV = dict(P), {}
+    for n in sorted(g):
+        newP[n], newV[n] = sgd(P[n], g[n], V.get(n), lr, momentum, first)
+    return loss, newP, newV, g

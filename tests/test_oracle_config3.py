@@ -222,3 +222,69 @@ def test_col2im_is_conv_data_gradient(stride, pad, k):
                         if 0 <= hh < h and 0 <= ww < w:
                             loop[b, hh, ww] += colv[b, i, j, r, s]
     torch.testing.assert_close(dx.double(), loop, atol=1e-5, rtol=1e-5)
+
+
+# ------------------------------------------------------------- Transformer encoder training
+def test_layernorm_bwd_fd():
+    x = _rand(5, 12, seed=81, dtype=D) * 2 + 1
+    gm, bt = _rand(12, seed=82, dtype=D), _rand(12, seed=83, dtype=D)
+    dy = _rand(5, 12, seed=84, dtype=D)
+    y, m, r = om.layernorm_fwd(x, gm, bt)
+    dx, dg, db = om.layernorm_bwd(x, dy, gm, m.double(), r.double())
+    xr = x.clone().requires_grad_(True)
+    gr, br = gm.clone().requires_grad_(True), bt.clone().requires_grad_(True)
+    torch.nn.functional.layer_norm(xr, (12,), gr, br, 1e-5).backward(dy)
+    torch.testing.assert_close(dx.double(), xr.grad, atol=2e-6, rtol=2e-5)
+    torch.testing.assert_close(dg.double(), gr.grad, atol=2e-6, rtol=2e-5)
+    torch.testing.assert_close(db.double(), br.grad, atol=2e-6, rtol=2e-5)
+
+
+def test_mha_bwd_vs_autograd():
+    B, S, heads, d = 2, 5, 2, 3
+    q, k, v, do = (_rand(B, S, heads * d, seed=s, dtype=D) for s in (85, 86, 87, 88))
+    dq, dk, dv = om.mha_bwd(q, k, v, do, heads)
+    qr, kr, vr = (t.clone().requires_grad_(True) for t in (q, k, v))
+    om_out = []
+
+    def f(q_, k_, v_):
+        Q, K, V = (t.view(B, S, heads, d).permute(0, 2, 1, 3) for t in (q_, k_, v_))
+        o = torch.softmax(Q @ K.transpose(-1, -2) / math.sqrt(d), -1) @ V
+        return o.permute(0, 2, 1, 3).reshape(B, S, heads * d)
+    f(qr, kr, vr).backward(do)
+    for a, b_ in ((dq, qr.grad), (dk, kr.grad), (dv, vr.grad)):
+        torch.testing.assert_close(a.double(), b_, atol=1e-6, rtol=1e-5)
+
+
+def test_encoder_train_step_vs_torch():
+    """2-layer post-LN encoder (d 32, 4 heads, FFN 64), batch 2, seq 6: loss, every gradient and
+    the SGD update against torch.nn.TransformerEncoderLayer in fp64 with autograd."""
+    L_, dm, heads, ffn = 2, 32, 4, 64
+    P = si.make_params(om.encoder_spec(L_, dm, ffn))
+    x, t = si.normal((2, 6, dm), si.BE_SEED, sub=1), si.normal((2, 6, dm), si.BE_SEED, sub=2)
+    loss, newP, _, g = om.encoder_train_step(P, {}, x, t, first=True, layers=L_, heads=heads)
+    mods = [torch.nn.TransformerEncoderLayer(dm, heads, ffn, dropout=0.0, activation="relu", batch_first=True,
+                                             norm_first=False).double() for _ in range(L_)]
+    names = {"in.w": "self_attn.in_proj_weight", "in.b": "self_attn.in_proj_bias", "out.w": "self_attn.out_proj.weight",
+             "out.b": "self_attn.out_proj.bias", "ln1.gamma": "norm1.weight", "ln1.beta": "norm1.bias",
+             "ff1.w": "linear1.weight", "ff1.b": "linear1.bias", "ff2.w": "linear2.weight", "ff2.b": "linear2.bias",
+             "ln2.gamma": "norm2.weight", "ln2.beta": "norm2.bias"}
+    for i, m in enumerate(mods):
+        sd = m.state_dict()
+        for k2, tk in names.items():
+            sd[tk] = P[f"enc{i}.{k2}"].double()
+        m.load_state_dict(sd)
+    h = x.double()
+    for m in mods:
+        h = m(h)
+    L = ((h - t.double()) ** 2).mean()
+    L.backward()
+    assert abs(float(loss) - float(L)) < 1e-5 * float(L)
+    for i, m in enumerate(mods):
+        named = dict(m.named_parameters())
+        for k2, tk in names.items():
+            ref = named[tk].grad
+            err = float((g[f"enc{i}.{k2}"].double() - ref).norm() / max(float(ref.norm()), 1e-12))
+            assert err < 1e-4, (i, k2, err)
+    k2 = "enc0.ff1.w"
+    torch.testing.assert_close(newP[k2].double(), P[k2].double() - 0.01 * dict(mods[0].named_parameters())["linear1.weight"].grad,
+                               rtol=1e-5, atol=1e-7)
