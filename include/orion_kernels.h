@@ -114,7 +114,27 @@ enum orion_fn {
      [K][R*S*C]) it is the data gradient of a strided convolution. args: col, dx, N, H, W, C, R, S,
      stride, pad, P, Q. C % 4 == 0; P, Q must be the conv's output size (else ORION_E_INVAL). */
   ORION_FN_COL2IM = 31,
-  ORION_FN_COUNT = 32
+  /* ---- fp32 Transformer-encoder training (BE of BASELINE config 4; reading R32): post-LN
+     torch.nn.TransformerEncoderLayer. LayerNorm over the last dim (C % 128 == 0, C <= 512), saving
+     the row mean and rstd = 1/sqrt(var + eps). args: x, y, gamma, beta, mean, rstd, rows, C, eps_bits */
+  ORION_FN_LAYERNORM_F32 = 32,
+  /* Its backward from the saved statistics: dx, dgamma = sum dy*xhat, dbeta = sum dy (column sums in
+     fp64, CTA partials combined in order). args: x, dy, dx, gamma, mean, rstd, dgamma, dbeta, rows, C,
+     workspace, ws_bytes (orion_layernorm_bwd_workspace_bytes(rows, C)) */
+  ORION_FN_LAYERNORM_F32_BWD = 33,
+  /* Attention forward, fp32: per batch b and head h, O = softmax(Q K^T / sqrt(d)) V over the head's
+     d = 64 columns. q, k, v rows of stride ld_in (e.g. the packed [rows, 3d] in-projection), o of
+     stride ld_out. S % 32 == 0, S <= 256. args: q, k, v, o, B, S, heads, d, ld_in, ld_out */
+  ORION_FN_ATTENTION_F32 = 34,
+  /* Attention backward, op 1: dQ = dS K / sqrt(d) with dS = P (dO V^T - rowsum(P dO V^T)); writes the
+     per-row statistics (max, 1/sum, rowsum) to stats [B][heads][S][3] for op 2.
+     args: q, k, v, dO, dq, stats, B, S, heads, d, ld_in, ld_out (q, k, v, dq of stride ld_in: gradients
+     share their input's layout, e.g. the packed [rows, 3d] buffer; dO of stride ld_out) */
+  ORION_FN_ATTENTION_F32_BWD_DQ = 35,
+  /* Attention backward, op 2: dV = P^T dO, dK = dS^T Q / sqrt(d) from the stats of op 1.
+     args: q, k, v, dO, stats, dk, dv, B, S, heads, d, ld_in, ld_out (dk, dv of stride ld_in, dO of ld_out) */
+  ORION_FN_ATTENTION_F32_BWD_DKV = 36,
+  ORION_FN_COUNT = 37
 };
 
 /* Number of table entries, and a stable name for each (for profiles and logs). */
@@ -135,6 +155,7 @@ uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t K);
 uint64_t orion_conv_wgrad_workspace_bytes(uint64_t N, uint64_t H, uint64_t W, uint64_t C, uint64_t K, uint64_t R, uint64_t S,
                                           uint64_t stride, uint64_t pad);
 uint64_t orion_bn_workspace_bytes(uint64_t rows, uint64_t C);
+uint64_t orion_layernorm_bwd_workspace_bytes(uint64_t rows, uint64_t C);
 uint64_t orion_dw_wgrad_workspace_bytes(uint64_t N, uint64_t C, uint64_t P, uint64_t Q);
 
 #ifdef __cplusplus

@@ -81,6 +81,7 @@ _sig = {
     "orion_gemm_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64]),
     "orion_conv_wgrad_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64] * 9),
     "orion_bn_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64, ctypes.c_uint64]),
+    "orion_layernorm_bwd_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64, ctypes.c_uint64]),
     "orion_dw_wgrad_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64]),
 }
 for _name, (_res, _args) in _sig.items():

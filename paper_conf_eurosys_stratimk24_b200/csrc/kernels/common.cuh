@@ -187,3 +187,8 @@ ENTRY_DECL(add_bf16)
 ENTRY_DECL(embed)
 ENTRY_DECL(maxpool_bwd)
 ENTRY_DECL(col2im)
+ENTRY_DECL(layernorm_f32)
+ENTRY_DECL(layernorm_f32_bwd)
+ENTRY_DECL(attention_f32)
+ENTRY_DECL(attention_f32_bwd_dq)
+ENTRY_DECL(attention_f32_bwd_dkv)

@@ -35,6 +35,11 @@ const KernelEntry g_kernels[ORION_FN_COUNT] = {
     E(embed, embed, 9),
     E(maxpool_bwd, maxpool_bwd, 9),
     E(col2im, col2im, 12),
+    E(layernorm_f32, layernorm_f32, 9),
+    E(layernorm_f32_bwd, layernorm_f32_bwd, 12),
+    E(attention_f32, attention_f32, 10),
+    E(attention_f32_bwd_dq, attention_f32_bwd_dq, 12),
+    E(attention_f32_bwd_dkv, attention_f32_bwd_dkv, 13),
 };
 #undef E
 

@@ -272,6 +272,7 @@ def mlp_train_graph(host_params, xs, ts, lr=0.01, width=512, layers=3, device="c
 
 # ====================================================================== ResNet-50 inference (HP)
 RESNET50_LAYERS = [(64, 3, 1), (128, 4, 2), (256, 6, 2), (512, 3, 2)]
+RESNET101_LAYERS = [(64, 3, 1), (128, 4, 2), (256, 23, 2), (512, 3, 2)]
 
 
 def resnet_spec(layers=RESNET50_LAYERS, num_classes=1000):
@@ -793,3 +794,135 @@ def bert_infer_graph(host_params, batch=8, seq=128, layers=12, heads=12, hidden=
     g.x = ids
     g.params = P
     return g.finalize()
+
+
+# ============================================================ Transformer encoder training (BE, config 4)
+def encoder_spec(layers=6, d=512, ffn=2048):
+    """torch.nn.TransformerEncoderLayer parameters (packed in-projection [3d, d]); torch's init
+    reading: U(+-1/sqrt(fan_in)) weights, zero attention biases, LN (1, 0)."""
+    s = []
+    for i in range(layers):
+        p = f"enc{i}"
+        s += [(f"{p}.in.w", (3 * d, d), ("uniform_fan_in", d)), (f"{p}.in.b", (3 * d,), ("const", 0.0)),
+              (f"{p}.out.w", (d, d), ("uniform_fan_in", d)), (f"{p}.out.b", (d,), ("const", 0.0)),
+              (f"{p}.ln1.gamma", (d,), ("const", 1.0)), (f"{p}.ln1.beta", (d,), ("const", 0.0)),
+              (f"{p}.ff1.w", (ffn, d), ("uniform_fan_in", d)), (f"{p}.ff1.b", (ffn,), ("uniform_fan_in", d)),
+              (f"{p}.ff2.w", (d, ffn), ("uniform_fan_in", ffn)), (f"{p}.ff2.b", (d,), ("uniform_fan_in", ffn)),
+              (f"{p}.ln2.gamma", (d,), ("const", 1.0)), (f"{p}.ln2.beta", (d,), ("const", 0.0))]
+    return s
+
+
+def encoder_train_graph(host_params, xs, ts, layers=6, d=512, heads=8, ffn=2048, lr=0.01, momentum=0.9, device="cuda"):
+    """BE (config 4): one training iteration of a post-LN Transformer-encoder stack (fp32, MSE to a
+    target, SGD momentum), op by op: packed in-projection GEMM, attention, out-projection, residual
+    add, LayerNorm, FFN (ReLU), residual add, LayerNorm; backward in reverse with the two-op
+    attention backward. One op-list variant per pre-staged (x, t) batch."""
+    g = Graph("encoder_train", device)
+    spec = encoder_spec(layers, d, ffn)
+    P = FlatParams(g, spec, host_params, grads=True, momentum=True)
+    b, sq, _ = xs[0].shape
+    rows = b * sq
+    xb = [g.buf(f"x{i}", (rows, d)) for i in range(len(xs))]
+    tb = [g.buf(f"t{i}", (rows, d)) for i in range(len(ts))]
+    with torch.no_grad():
+        for dst, src in zip(xb + tb, list(xs) + list(ts)):
+            dst.copy_(src.reshape(rows, d).to(dst.device))
+    loss = g.buf("loss", (1,))
+    cnt = [0]
+
+    def new(cols):
+        cnt[0] += 1
+        return g.buf(f"t{cnt[0]}", (rows, cols))
+    L_ = []
+    for i in range(layers):
+        L_.append(dict(qkv=new(3 * d), a=new(d), o=new(d), s1=new(d), h1=new(d), m1=g.buf(f"m1_{i}", (rows,)),
+                       r1=g.buf(f"r1_{i}", (rows,)), f=new(ffn), fa=new(ffn), f2=new(d), s2=new(d), h2=new(d),
+                       m2=g.buf(f"m2_{i}", (rows,)), r2=g.buf(f"r2_{i}", (rows,))))
+    dh, ds2, dfa, df, dh1ff, dh1, ds1, da, dqkv, dha = (new(c) for c in (d, d, ffn, ffn, d, d, d, d, 3 * d, d))
+    dhs = [new(d) for _ in range(layers)]
+    stats = g.buf("attn_stats", (b * heads * sq * 3,))
+    g.need_ws(L.lib.orion_layernorm_bwd_workspace_bytes(rows, d))
+    g.need_ws(L.WS_TICKET_BYTES + 8 * 148 * 8)
+    eps = f32bits(1e-5)
+
+    def lin(x, name, out):
+        linear_fwd(g, x, P.p[f"{name}.w"], P.p[f"{name}.b"], out, name)
+
+    def lin_bwd(x, name, dy, dx):
+        w = P.p[f"{name}.w"]
+        fout, fin = w.shape
+        gemm(g, dy, x, P.g[f"{name}.w"], None, fout, fin, rows, fout, fin, fin, 1, f"{name}.wgrad")
+        g.k("colsum", [_p(dy), _p(P.g[f"{name}.b"]), rows, fout], f"{name}.bgrad")
+        if dx is not None:
+            gemm(g, dy, w, dx, None, rows, fin, fout, fout, fin, fin, 0, f"{name}.dgrad")
+
+    def ln_bwd(x, dy, dx, name, m, r):
+        g.k("layernorm_f32_bwd", [_p(x), _p(dy), _p(dx), _p(P.p[f"{name}.gamma"]), _p(m), _p(r), _p(P.g[f"{name}.gamma"]),
+                                  _p(P.g[f"{name}.beta"]), rows, d, 0, 0], f"{name}.bwd", ws_at=10)
+
+    variants, ws_ops = [], None
+    for vi in range(len(xs)):
+        g.ops, g._ws_ops = [], []
+        h = xb[vi]
+        for i in range(layers):
+            p, R = f"enc{i}", L_[i]
+            lin(h, f"{p}.in", R["qkv"])
+            qkv = R["qkv"].data_ptr()
+            g.k("attention_f32", [qkv, qkv + 4 * d, qkv + 8 * d, _p(R["a"]), b, sq, heads, d // heads, 3 * d, d], f"{p}.attn")
+            lin(R["a"], f"{p}.out", R["o"])
+            g.k("add", [_p(h), _p(R["o"]), _p(R["s1"]), rows * d], f"{p}.add1")
+            g.k("layernorm_f32", [_p(R["s1"]), _p(R["h1"]), _p(P.p[f"{p}.ln1.gamma"]), _p(P.p[f"{p}.ln1.beta"]), _p(R["m1"]),
+                                  _p(R["r1"]), rows, d, eps], f"{p}.ln1")
+            lin(R["h1"], f"{p}.ff1", R["f"])
+            g.k("relu", [_p(R["f"]), _p(R["fa"]), rows * ffn], f"{p}.relu")
+            lin(R["fa"], f"{p}.ff2", R["f2"])
+            g.k("add", [_p(R["h1"]), _p(R["f2"]), _p(R["s2"]), rows * d], f"{p}.add2")
+            g.k("layernorm_f32", [_p(R["s2"]), _p(R["h2"]), _p(P.p[f"{p}.ln2.gamma"]), _p(P.p[f"{p}.ln2.beta"]), _p(R["m2"]),
+                                  _p(R["r2"]), rows, d, eps], f"{p}.ln2")
+            R["in"] = h
+            h = R["h2"]
+        g.k("mse", [_p(h), _p(tb[vi]), _p(loss), _p(dh), rows * d, 0, 0], "mse", ws_at=5)
+        dcur = dh
+        for i in reversed(range(layers)):
+            p, R = f"enc{i}", L_[i]
+            ln_bwd(R["s2"], dcur, ds2, f"{p}.ln2", R["m2"], R["r2"])
+            lin_bwd(R["fa"], f"{p}.ff2", ds2, dfa)
+            g.k("relu_bwd", [_p(R["f"]), _p(dfa), _p(df), rows * ffn], f"{p}.relu_bwd")
+            lin_bwd(R["h1"], f"{p}.ff1", df, dh1ff)
+            g.k("add", [_p(ds2), _p(dh1ff), _p(dh1), rows * d], f"{p}.add2_bwd")
+            ln_bwd(R["s1"], dh1, ds1, f"{p}.ln1", R["m1"], R["r1"])
+            lin_bwd(R["a"], f"{p}.out", ds1, da)
+            qkv, dq = R["qkv"].data_ptr(), dqkv.data_ptr()
+            g.k("attention_f32_bwd_dq", [qkv, qkv + 4 * d, qkv + 8 * d, _p(da), dq, _p(stats), b, sq, heads, d // heads, 3 * d, d],
+                f"{p}.attn_bwd_dq")
+            g.k("attention_f32_bwd_dkv", [qkv, qkv + 4 * d, qkv + 8 * d, _p(da), _p(stats), dq + 4 * d, dq + 8 * d, b, sq, heads,
+                                          d // heads, 3 * d, d], f"{p}.attn_bwd_dkv")
+            lin_bwd(R["in"], f"{p}.in", dqkv, dha)
+            g.k("add", [_p(ds1), _p(dha), _p(dhs[i]), rows * d], f"{p}.add1_bwd")
+            dcur = dhs[i]
+        g.k("sgd", [_p(P.flat), _p(P.gflat), _p(P.vflat), P.total, f32bits(lr), f32bits(momentum)], "sgd")
+        variants.append(g.ops)
+        ws_ops = g._ws_ops
+    g.variants = []
+    for ops in variants:
+        g.ops, g._ws_ops = ops, list(ws_ops)
+        g.finalize()
+        g.variants.append(list(g.ops))
+    g.ops = g.variants[0]
+    g.loss = loss
+    g.params = P
+    g.relu_in = {f"enc{i}.ff1": L_[i]["f"] for i in range(layers)}
+    return g
+
+
+# ============================================================ training as the HP client (config 4)
+def as_hp_training(graph, x_host, device="cuda"):
+    """Wrap a one-variant training graph as an HP client op list: H2D of the iteration's input batch
+    first, D2H of the loss last (the request boundaries, R2 / R19); each 'request' is one training
+    iteration (throughput mode). Returns (ops list, input buffer)."""
+    xbuf = graph.bufs["x0"]
+    ops = [(L.OP_MEMCPY_H2D, [xbuf.data_ptr(), 0, xbuf.numel() * 4], "h2d_batch")] + list(graph.variants[0])
+    ops.append((L.OP_MEMCPY_D2H, [0, graph.loss.data_ptr(), 4], "d2h_loss"))
+    graph.ops = ops
+    graph.variants = [ops]
+    return graph

@@ -157,6 +157,31 @@ def check_op(fn, a, R, snap=None, R_in=None):
         n, h, w, c, r, s_, st, pad, p, q = a[2:12]
         col = T(a[0], n * p * q * r * s_ * c, (n * p * q, r * s_ * c))
         return rel(R.get(a[1], n * h * w * c, (n, h, w, c)), om.col2im(col, (n, h, w, c), r, s_, st, pad))
+    if fn == "layernorm_f32":
+        rows, C = a[6], a[7]
+        y, m, r = om.layernorm_fwd(T(a[0], rows * C, (rows, C)), T(a[2], C), T(a[3], C), _u2f(a[8]))
+        return max(rel(R.get(a[1], rows * C, (rows, C)), y), rel(R.get(a[4], rows), m, 1e-3), rel(R.get(a[5], rows), r))
+    if fn == "layernorm_f32_bwd":
+        rows, C = a[8], a[9]
+        dx, dg, db = om.layernorm_bwd(T(a[0], rows * C, (rows, C)), T(a[1], rows * C, (rows, C)), T(a[3], C), T(a[4], rows), T(a[5], rows))
+        return max(rel(R.get(a[2], rows * C, (rows, C)), dx), rel(R.get(a[6], C), dg, 1e-3), rel(R.get(a[7], C), db, 1e-3))
+    if fn in ("attention_f32", "attention_f32_bwd_dq", "attention_f32_bwd_dkv"):
+        np_ = {"attention_f32": 4, "attention_f32_bwd_dq": 6, "attention_f32_bwd_dkv": 7}[fn]
+        B, S, H, d, ldi, ldo = a[np_:np_ + 6]
+        hd = H * d
+
+        def view(ptr, ld):   # [B, S, hd] view of rows of stride ld starting at ptr
+            return R_in.get(ptr, (B * S - 1) * ld + hd, None).cpu().as_strided((B, S, hd), (S * ld, ld, 1))
+
+        def out(ptr, ld):
+            return R.get(ptr, (B * S - 1) * ld + hd, None).cpu().as_strided((B, S, hd), (S * ld, ld, 1))
+        q, k, v = view(a[0], ldi), view(a[1], ldi), view(a[2], ldi)
+        if fn == "attention_f32":
+            return rel(out(a[3], ldo), om.mha_fwd(q, k, v, H))
+        dq, dk, dv = om.mha_bwd(q, k, v, view(a[3], ldo), H)
+        if fn == "attention_f32_bwd_dq":
+            return rel(out(a[4], ldi), dq)
+        return max(rel(out(a[5], ldi), dk), rel(out(a[6], ldi), dv))
     if fn == "colsum":
         M, N = a[2], a[3]
         return rel(R.get(a[1], N), om._r(T(a[0], M * N, (M, N)).double().sum(0)))
