@@ -476,7 +476,11 @@ def train_train(args, rank, world, local, metric):
     # binary search of SM_THRESHOLD on HP throughput
     lo, hi = 0, max(r["sm_needed"] for r in rows_be) + 1
     probes = []
-    while hi - lo > max(4, (hi - lo) // 16) and len(probes) < 6:
+    _, h_, b_ = colloc(hi, max(8, n // 4))          # the most aggressive threshold first
+    probes.append((hi, h_ / hp_ded, b_))
+    if h_ >= 0.9 * hp_ded:
+        lo = hi
+    while hi - lo > 2 and len(probes) < 7:
         mid = (lo + hi) // 2
         _, h_, b_ = colloc(mid, max(8, n // 4))
         probes.append((mid, h_ / hp_ded, b_))

@@ -1419,6 +1419,7 @@ struct V {
 using V44 = V<4, 4, 64, 128, 128>;
 using V84 = V<8, 4, 32, 192, 64>;
 using V48 = V<4, 8, 32, 64, 192>;
+using V88 = V<8, 8, 16, 256, 256>;   // 256 x 64 / 64 x 256 / 128 x 128 (ResNet's 1x1 weight gradients)
 
 template <class VV, int TMB, int TNB, int R>
 __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float* __restrict__ A, long long lda,
@@ -1732,13 +1733,14 @@ int atb_variant(long long M, long long N, long long K) {
   if (atb::V44::fits(M, N)) return 5;
   if (atb::V84::fits(M, N)) return 6;
   if (atb::V48::fits(M, N)) return 7;
+  if (atb::V88::fits(M, N)) return 8;
   return -1;
 }
 bool atb_ok(long long M, long long N, long long K) { return atb_variant(M, N, K) >= 0; }
 
 Plan plan_atb(long long M, long long N, long long K) {
   Plan pl;
-  pl.cfg = atb_variant(M, N, K); pl.bm = (int)M; pl.bn = (int)N; pl.bk = pl.cfg == 5 ? 64 : 32;
+  pl.cfg = atb_variant(M, N, K); pl.bm = (int)M; pl.bn = (int)N; pl.bk = pl.cfg == 5 ? 64 : (pl.cfg == 8 ? 16 : 32);
   long long split = cdiv(148 * 4, 1);
   long long kmax = K / (4 * pl.bk);
   if (split > kmax) split = kmax;
@@ -2114,14 +2116,17 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
           cudaFuncSetAttribute((const void*)atb::gemm_atb_kernel<atb::V84, 8, 4, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                atb::V84::smem_bytes(192, 64)) != cudaSuccess ||
           cudaFuncSetAttribute((const void*)atb::gemm_atb_kernel<atb::V48, 4, 8, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               atb::V48::smem_bytes(64, 192)) != cudaSuccess)
+                               atb::V48::smem_bytes(64, 192)) != cudaSuccess ||
+          cudaFuncSetAttribute((const void*)atb::gemm_atb_kernel<atb::V88, 8, 8, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               atb::V88::smem_bytes(256, 256)) != cudaSuccess)
         return ORION_E_CUDA;
       attr.store(1);
     }
     g->grid = dim3(1, 1, (unsigned)pl.split); g->block = dim3(atb::NTH);
     if (pl.cfg == 5) { g->smem = atb::V44::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V44, 4, 4, 64>; }
     else if (pl.cfg == 6) { g->smem = atb::V84::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V84, 8, 4, 32>; }
-    else { g->smem = atb::V48::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V48, 4, 8, 32>; }
+    else if (pl.cfg == 7) { g->smem = atb::V48::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V48, 4, 8, 32>; }
+    else { g->smem = atb::V88::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V88, 8, 8, 16>; }
     return 0;
   }
   switch (flags) {
@@ -2168,6 +2173,10 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
   }
   if (g.func == (const void*)atb::gemm_atb_kernel<atb::V48, 4, 8, 32>) {
     atb::gemm_atb_kernel<atb::V48, 4, 8, 32><<<g.grid, g.block, g.smem, s>>>(make_params(M, N, K, C, ldc, bias, (int)g.grid.z, ws, 32), A, lda, B, ldb, sig);
+    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+  }
+  if (g.func == (const void*)atb::gemm_atb_kernel<atb::V88, 8, 8, 16>) {
+    atb::gemm_atb_kernel<atb::V88, 8, 8, 16><<<g.grid, g.block, g.smem, s>>>(make_params(M, N, K, C, ldc, bias, (int)g.grid.z, ws, 16), A, lda, B, ldb, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
   switch (flags) {

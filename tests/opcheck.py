@@ -182,6 +182,10 @@ def check_op(fn, a, R, snap=None, R_in=None):
         if fn == "attention_f32_bwd_dq":
             return rel(out(a[4], ldi), dq)
         return max(rel(out(a[5], ldi), dk), rel(out(a[6], ldi), dv))
+    if fn == "mse":
+        n = a[4]
+        loss, dy = om.mse_fwd_bwd(T(a[0], n), T(a[1], n))
+        return max(rel(R.get(a[2], 1), loss.reshape(1)), rel(R.get(a[3], n), dy))
     if fn == "colsum":
         M, N = a[2], a[3]
         return rel(R.get(a[1], N), om._r(T(a[0], M * N, (M, N)).double().sum(0)))

@@ -46,7 +46,9 @@ def ws(nbytes):
                                          (144, 24, 75264, 1), (192, 32, 75264, 1), (32, 192, 75264, 1), (150, 22, 5000, 1),
                                          # multi-tile tcgen05 kernel (>= 296 tiles): ragged M / N / K, unaligned K
                                          (40000, 96, 16, 2), (30000, 144, 20, 0), (20000, 200, 40, 2), (40000, 64, 33, 2),
-                                         (301056, 24, 144, 0), (38000, 33, 24, 0), (18816, 384, 64, 2), (4704, 1280, 320, 0)],
+                                         (301056, 24, 144, 0), (38000, 33, 24, 0), (18816, 384, 64, 2), (4704, 1280, 320, 0),
+                                         # skinny A^T B 8x8 register-block variant (ResNet 1x1 weight gradients)
+                                         (256, 64, 50000, 1), (64, 256, 50176, 1), (128, 128, 20000, 1), (250, 60, 9999, 1)],
                          ids=lambda v: str(v))
 def test_gemm_shapes(M, N, K, flags):
     test_gemm(M, N, K, flags)
