@@ -357,6 +357,12 @@ def main():
             traffic = json.load(open(tp)).get(top_row["label"])
         except Exception:
             traffic = None
+    if traffic is None:
+        # dram__bytes_read.sum + dram__bytes_write.sum of this op's solo launch in the committed
+        # per-op ncu capture (tools/ncu_times.sh; profiles/<config>_be_ncu.csv)
+        ncu_rows = PR.load_ncu_csv(ncu_be)
+        if top_kid in ncu_rows and ncu_rows[top_kid][2] > 0:
+            traffic = ncu_rows[top_kid][2]
     # ---- e2e: BE inputs copied from pinned host each iteration (H2D) + loss read back (D2H)
     e2e = None
     if not args.no_e2e:

@@ -1938,6 +1938,7 @@ inline bool wgrad_ok(const ConvShape& s) {
   return s.C <= 4 && s.K % WG_KPT == 0 && s.K <= MAXK && (kg & (kg - 1)) == 0 && rsc >= 64 && wg_nr(s) >= 8 && wg_nr(s) <= WG_MAXR &&
          wg_xwin(s) <= NTH * WG_PF_X && s.stride <= 2;
 }
+inline bool wgrad2_ok(const ConvShape& s);
 inline uint64_t wgrad_ws_bytes(const ConvShape& s) {
   const int G = wg_ctas(s);
   const uint64_t V = (uint64_t)s.K * s.R * s.S * s.C;
@@ -2049,6 +2050,131 @@ __global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc_kernel(const float* 
   orion_signal(sig);
 }
 #undef WG_FETCH
+
+// Variant for the 3x3x3 / 32-filter stem (MobileNetV2): the 864 outputs are few and each value is
+// used by few products, so a whole warp covers all outputs of one pixel — lane = (k-quad kg < 8,
+// rsc subset rs < 4), 4 x 7 register block — and the 8 warps of a CTA take interleaved pixels of the
+// staged 32-pixel tile; warp partials are summed in warp order, CTA partials (fp64) in CTA order.
+constexpr int W2_NR = 7;
+inline bool wgrad2_ok(const ConvShape& s) {
+  return s.C <= 4 && s.K == 32 && s.R * s.S * s.C <= 4 * W2_NR && wg_xwin(s) <= NTH * WG_PF_X && s.stride <= 2;
+}
+__global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc2_kernel(const float* __restrict__ x, const float* __restrict__ dy,
+                                                                    float* __restrict__ dw, ConvShape s, unsigned char* ws, OrionSig sig) {
+  extern __shared__ __align__(16) float wsm[];
+  constexpr int K = 32;
+  const int RSC = s.R * s.S * s.C, WW = wg_wwin(s), XW = wg_xwin(s);
+  float* dys = wsm;                      // [WG_QT][K]
+  float* xs = wsm + WG_QT * K;           // [R][WW][C]
+  const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
+  const int kg = lane % 8, rs = lane / 8;
+  int off[W2_NR];
+#pragma unroll
+  for (int i = 0; i < W2_NR; i++) {
+    const int j = rs + 4 * i;
+    if (j < RSC) {
+      const int c = j % s.C, t = j / s.C, u = t % s.S, r = t / s.S;
+      off[i] = (r * WW + u) * s.C + c;
+    } else {
+      off[i] = 0;   // padding slot, never stored
+    }
+  }
+  float acc[4][W2_NR];
+#pragma unroll
+  for (int a = 0; a < 4; a++)
+#pragma unroll
+    for (int i = 0; i < W2_NR; i++) acc[a][i] = 0.f;
+  const int qtiles = (s.Q + WG_QT - 1) / WG_QT;
+  const long long T = (long long)s.N * s.P * qtiles;
+  constexpr int PF_DY = WG_QT * K / 4 / NTH;   // 1 float4 per thread
+  float4 pdy[PF_DY];
+  float px[WG_PF_X];
+#define W2_FETCH(TT)                                                                                                    \
+  {                                                                                                                     \
+    const long long t_ = (TT);                                                                                          \
+    const int qt = (int)(t_ % qtiles); const long long np = t_ / qtiles;                                                \
+    const int p = (int)(np % s.P), n = (int)(np / s.P);                                                                 \
+    const int q0 = qt * WG_QT, qn = min(WG_QT, s.Q - q0);                                                               \
+    const float4* src = reinterpret_cast<const float4*>(dy + (((long long)n * s.P + p) * s.Q + q0) * K);                \
+    _Pragma("unroll") for (int e = 0; e < PF_DY; e++) {                                                                 \
+      const int idx = threadIdx.x + e * NTH;                                                                            \
+      pdy[e] = (idx * 4 < qn * K) ? __ldg(src + idx) : make_float4(0.f, 0.f, 0.f, 0.f);                                  \
+    }                                                                                                                   \
+    const int h0 = p * s.stride - s.pad, w0 = q0 * s.stride - s.pad;                                                    \
+    _Pragma("unroll") for (int e = 0; e < WG_PF_X; e++) {                                                               \
+      const int idx = threadIdx.x + e * NTH;                                                                            \
+      float v = 0.f;                                                                                                    \
+      if (idx < XW) {                                                                                                   \
+        const int c = idx % s.C, t2 = idx / s.C, u = t2 % WW, r = t2 / WW;                                              \
+        const int h = h0 + r, w = w0 + u;                                                                               \
+        if ((unsigned)h < (unsigned)s.H && (unsigned)w < (unsigned)s.W) v = __ldg(x + (((long long)n * s.H + h) * s.W + w) * s.C + c); \
+      }                                                                                                                 \
+      px[e] = v;                                                                                                        \
+    }                                                                                                                   \
+  }
+  long long t = blockIdx.x;
+  if (t < T) W2_FETCH(t);
+  for (; t < T; t += gridDim.x) {
+    __syncthreads();
+#pragma unroll
+    for (int e = 0; e < PF_DY; e++) reinterpret_cast<float4*>(dys)[threadIdx.x + e * NTH] = pdy[e];
+#pragma unroll
+    for (int e = 0; e < WG_PF_X; e++) {
+      const int idx = threadIdx.x + e * NTH;
+      if (idx < XW) xs[idx] = px[e];
+    }
+    __syncthreads();
+    if (t + gridDim.x < T) W2_FETCH(t + gridDim.x);
+    const int xstep = s.stride * s.C;
+#pragma unroll
+    for (int i = warp; i < WG_QT; i += NTH / 32) {
+      const float4 d = *reinterpret_cast<const float4*>(dys + i * K + kg * 4);
+      const float* xr = xs + i * xstep;
+#pragma unroll
+      for (int j = 0; j < W2_NR; j++) {
+        const float xv = xr[off[j]];
+        acc[0][j] = fmaf(d.x, xv, acc[0][j]);
+        acc[1][j] = fmaf(d.y, xv, acc[1][j]);
+        acc[2][j] = fmaf(d.z, xv, acc[2][j]);
+        acc[3][j] = fmaf(d.w, xv, acc[3][j]);
+      }
+    }
+  }
+  __syncthreads();
+  // warp partials -> shared [8][K * RSC] (reusing the staging area), summed in warp order
+  const int V = K * RSC;
+  float* wp = wsm;
+#pragma unroll
+  for (int j = 0; j < W2_NR; j++) {
+    const int jj = rs + 4 * j;
+    if (jj < RSC) {
+#pragma unroll
+      for (int a = 0; a < 4; a++) wp[warp * V + (kg * 4 + a) * RSC + jj] = acc[a][j];
+    }
+  }
+  __syncthreads();
+  unsigned int* tk = reinterpret_cast<unsigned int*>(ws);
+  double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
+  const int G = gridDim.x;
+  for (int v = threadIdx.x; v < V; v += NTH) {
+    double sum = 0.0;
+    for (int w = 0; w < NTH / 32; w++) sum += (double)wp[w * V + v];
+    part[(long long)blockIdx.x * V + v] = sum;
+  }
+  double* gpart = part + (long long)G * V;
+  double* out = gpart + (long long)combine_rows(G) * V;
+  __shared__ double scratch[NTH];
+  if (combine_splits(tk, part, gpart, V, G, blockIdx.x, V, out, scratch)) {
+    for (int v = threadIdx.x; v < V; v += NTH) dw[v] = (float)__ldcg(out + v);
+  }
+  orion_signal(sig);
+}
+#undef W2_FETCH
+inline int wgrad2_smem(const ConvShape& s) {
+  const int stage = WG_QT * 32 + wg_xwin(s), red = (NTH / 32) * 32 * s.R * s.S * s.C;
+  return (stage > red ? stage : red) * 4;
+}
+
 inline const void* wgrad_fn(const ConvShape& s) {
   switch (wg_nr(s)) {
     case 8: return (const void*)conv_wgrad_smallc_kernel<8>;
@@ -2238,7 +2364,7 @@ extern "C" uint64_t orion_conv_wgrad_workspace_bytes(uint64_t N, uint64_t H, uin
   ConvShape s{(int)N, (int)H, (int)W, (int)C, (int)K, (int)R, (int)S, (int)stride, (int)pad,
               (int)((H + 2 * pad - R) / stride + 1), (int)((W + 2 * pad - S) / stride + 1)};
   uint64_t b = orion_gemm_workspace_bytes(K, R * S * C, (uint64_t)N * s.P * s.Q);
-  if (smallc::wgrad_ok(s)) {
+  if (smallc::wgrad_ok(s) || smallc::wgrad2_ok(s)) {
     const uint64_t b2 = smallc::wgrad_ws_bytes(s);
     if (b2 > b) b = b2;
   }
@@ -2247,6 +2373,19 @@ extern "C" uint64_t orion_conv_wgrad_workspace_bytes(uint64_t N, uint64_t H, uin
 
 int conv_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
   ConvShape s = conv_shape(a);
+  if (smallc::wgrad2_ok(s) && a[14] != 0 && a[15] >= smallc::wgrad_ws_bytes(s)) {
+    static std::atomic<int> attr{0};
+    if (!attr.load()) {
+      if (cudaFuncSetAttribute((const void*)smallc::conv_wgrad_smallc2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024) !=
+          cudaSuccess)
+        return ORION_E_CUDA;
+      attr.store(1);
+    }
+    g->grid = dim3((unsigned)smallc::wg_ctas(s)); g->block = dim3(smallc::NTH);
+    g->smem = smallc::wgrad2_smem(s);
+    g->func = (const void*)smallc::conv_wgrad_smallc2_kernel;
+    return 0;
+  }
   if (smallc::wgrad_ok(s) && a[14] != 0 && a[15] >= smallc::wgrad_ws_bytes(s)) {
     g->grid = dim3((unsigned)smallc::wg_ctas(s)); g->block = dim3(smallc::NTH);
     g->smem = (smallc::WG_QT * s.K + smallc::wg_xwin(s)) * 4;   // <= 24 KB
@@ -2258,6 +2397,11 @@ int conv_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
 }
 int conv_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   ConvShape s = conv_shape(a);
+  if (g.func == (const void*)smallc::conv_wgrad_smallc2_kernel) {
+    smallc::conv_wgrad_smallc2_kernel<<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s,
+                                                                       (unsigned char*)a[14], sig);
+    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+  }
   if (smallc::wgrad_ok(s) && g.func == smallc::wgrad_fn(s)) {
     const float* x = (const float*)a[0]; const float* dy = (const float*)a[1]; float* dw = (float*)a[2];
     unsigned char* ws = (unsigned char*)a[14];
