@@ -87,6 +87,18 @@ def op_work(fn, a):
     if f == "embed":
         B, S, H = a[5], a[6], a[7]
         return 2 * B * S * H, 2 * (2 * B * S * H + S * H + H) + 4 * B * S
+    if f == "col2im":
+        n, h, w, c, r, s_, st, pad, p, q = a[2:12]
+        return n * p * q * r * s_ * c, 4 * (n * p * q * r * s_ * c + n * h * w * c)
+    if f == "layernorm_f32":
+        return 8 * a[6] * a[7], 4 * (2 * a[6] * a[7] + 2 * a[6] + 2 * a[7])
+    if f == "layernorm_f32_bwd":
+        return 12 * a[8] * a[9], 4 * (3 * a[8] * a[9] + 2 * a[8] + 3 * a[9])
+    if f in ("attention_f32", "attention_f32_bwd_dq", "attention_f32_bwd_dkv"):
+        k0 = {"attention_f32": 4, "attention_f32_bwd_dq": 6, "attention_f32_bwd_dkv": 7}[f]
+        B, S, H, d = a[k0], a[k0 + 1], a[k0 + 2], a[k0 + 3]
+        mul = {"attention_f32": (4, 4), "attention_f32_bwd_dq": (6, 5), "attention_f32_bwd_dkv": (8, 6)}[f]
+        return mul[0] * B * H * S * S * d, 4 * mul[1] * B * S * H * d
     if f == "maxpool_bwd":
         n, h, w, c, p, q = a[3:9]
         return 9 * n * p * q * c, 4 * (2 * n * h * w * c + n * p * q * c)

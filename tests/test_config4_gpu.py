@@ -46,11 +46,10 @@ def test_encoder_ops_teacher_forced():
     R = opcheck.Resolver(tensors)
     R_in = opcheck.Resolver(tensors, read_alias={Pm.flat.data_ptr(): Pm.flat.clone()})
     s = torch.cuda.current_stream().cuda_stream
-    for fn, args, lab in g.ops:
-        orion.kernel_launch(fn, args, s)
-    torch.cuda.synchronize()
     errs = []
-    for i, (fn, args, lab) in enumerate(g.ops):
+    for i, (fn, args, lab) in enumerate(g.ops):   # gradient buffers are shared across layers: check each op right away
+        orion.kernel_launch(fn, args, s)
+        torch.cuda.synchronize()
         if fn == "sgd":
             continue
         e = opcheck.check_op(fn, args, R, None, R_in)
