@@ -2055,17 +2055,19 @@ __global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc_kernel(const float* 
 // used by few products, so a whole warp covers all outputs of one pixel — lane = (k-quad kg < 8,
 // rsc subset rs < 4), 4 x 7 register block — and the 8 warps of a CTA take interleaved pixels of the
 // staged 32-pixel tile; warp partials are summed in warp order, CTA partials (fp64) in CTA order.
-constexpr int W2_NR = 7;
+constexpr int W2_NR = 7, W2_QT = 112, W2_PF_X = 8;   // a whole MobileNetV2 stem output row per tile
+__host__ __device__ inline int w2_wwin(const ConvShape& s) { return (W2_QT - 1) * s.stride + s.S; }
+__host__ __device__ inline int w2_xwin(const ConvShape& s) { return s.R * w2_wwin(s) * s.C; }
 inline bool wgrad2_ok(const ConvShape& s) {
-  return s.C <= 4 && s.K == 32 && s.R * s.S * s.C <= 4 * W2_NR && wg_xwin(s) <= NTH * WG_PF_X && s.stride <= 2;
+  return s.C <= 4 && s.K == 32 && s.R * s.S * s.C <= 4 * W2_NR && w2_xwin(s) <= NTH * W2_PF_X && s.stride <= 2;
 }
 __global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc2_kernel(const float* __restrict__ x, const float* __restrict__ dy,
                                                                     float* __restrict__ dw, ConvShape s, unsigned char* ws, OrionSig sig) {
   extern __shared__ __align__(16) float wsm[];
   constexpr int K = 32;
-  const int RSC = s.R * s.S * s.C, WW = wg_wwin(s), XW = wg_xwin(s);
-  float* dys = wsm;                      // [WG_QT][K]
-  float* xs = wsm + WG_QT * K;           // [R][WW][C]
+  const int RSC = s.R * s.S * s.C, WW = w2_wwin(s), XW = w2_xwin(s);
+  float* dys = wsm;                      // [W2_QT][K]
+  float* xs = wsm + W2_QT * K;           // [R][WW][C]
   const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
   const int kg = lane % 8, rs = lane / 8;
   int off[W2_NR];
@@ -2084,24 +2086,24 @@ __global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc2_kernel(const float*
   for (int a = 0; a < 4; a++)
 #pragma unroll
     for (int i = 0; i < W2_NR; i++) acc[a][i] = 0.f;
-  const int qtiles = (s.Q + WG_QT - 1) / WG_QT;
+  const int qtiles = (s.Q + W2_QT - 1) / W2_QT;
   const long long T = (long long)s.N * s.P * qtiles;
-  constexpr int PF_DY = WG_QT * K / 4 / NTH;   // 1 float4 per thread
+  constexpr int PF_DY = (W2_QT * K / 4 + NTH - 1) / NTH;   // 4 float4 per thread
   float4 pdy[PF_DY];
-  float px[WG_PF_X];
+  float px[W2_PF_X];
 #define W2_FETCH(TT)                                                                                                    \
   {                                                                                                                     \
     const long long t_ = (TT);                                                                                          \
     const int qt = (int)(t_ % qtiles); const long long np = t_ / qtiles;                                                \
     const int p = (int)(np % s.P), n = (int)(np / s.P);                                                                 \
-    const int q0 = qt * WG_QT, qn = min(WG_QT, s.Q - q0);                                                               \
+    const int q0 = qt * W2_QT, qn = min(W2_QT, s.Q - q0);                                                               \
     const float4* src = reinterpret_cast<const float4*>(dy + (((long long)n * s.P + p) * s.Q + q0) * K);                \
     _Pragma("unroll") for (int e = 0; e < PF_DY; e++) {                                                                 \
       const int idx = threadIdx.x + e * NTH;                                                                            \
       pdy[e] = (idx * 4 < qn * K) ? __ldg(src + idx) : make_float4(0.f, 0.f, 0.f, 0.f);                                  \
     }                                                                                                                   \
     const int h0 = p * s.stride - s.pad, w0 = q0 * s.stride - s.pad;                                                    \
-    _Pragma("unroll") for (int e = 0; e < WG_PF_X; e++) {                                                               \
+    _Pragma("unroll") for (int e = 0; e < W2_PF_X; e++) {                                                               \
       const int idx = threadIdx.x + e * NTH;                                                                            \
       float v = 0.f;                                                                                                    \
       if (idx < XW) {                                                                                                   \
@@ -2117,17 +2119,18 @@ __global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc2_kernel(const float*
   for (; t < T; t += gridDim.x) {
     __syncthreads();
 #pragma unroll
-    for (int e = 0; e < PF_DY; e++) reinterpret_cast<float4*>(dys)[threadIdx.x + e * NTH] = pdy[e];
+    for (int e = 0; e < PF_DY; e++)
+      if (threadIdx.x + e * NTH < W2_QT * K / 4) reinterpret_cast<float4*>(dys)[threadIdx.x + e * NTH] = pdy[e];
 #pragma unroll
-    for (int e = 0; e < WG_PF_X; e++) {
+    for (int e = 0; e < W2_PF_X; e++) {
       const int idx = threadIdx.x + e * NTH;
       if (idx < XW) xs[idx] = px[e];
     }
     __syncthreads();
     if (t + gridDim.x < T) W2_FETCH(t + gridDim.x);
     const int xstep = s.stride * s.C;
-#pragma unroll
-    for (int i = warp; i < WG_QT; i += NTH / 32) {
+#pragma unroll 2
+    for (int i = warp; i < W2_QT; i += NTH / 32) {
       const float4 d = *reinterpret_cast<const float4*>(dys + i * K + kg * 4);
       const float* xr = xs + i * xstep;
 #pragma unroll
@@ -2170,8 +2173,12 @@ __global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc2_kernel(const float*
   orion_signal(sig);
 }
 #undef W2_FETCH
+inline int w2_ctas(const ConvShape& s) {
+  const long long t = (long long)s.N * s.P * ((s.Q + W2_QT - 1) / W2_QT);
+  return (int)(t < WG_G ? t : WG_G);
+}
 inline int wgrad2_smem(const ConvShape& s) {
-  const int stage = WG_QT * 32 + wg_xwin(s), red = (NTH / 32) * 32 * s.R * s.S * s.C;
+  const int stage = W2_QT * 32 + w2_xwin(s), red = (NTH / 32) * 32 * s.R * s.S * s.C;
   return (stage > red ? stage : red) * 4;
 }
 
@@ -2381,7 +2388,7 @@ int conv_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
         return ORION_E_CUDA;
       attr.store(1);
     }
-    g->grid = dim3((unsigned)smallc::wg_ctas(s)); g->block = dim3(smallc::NTH);
+    g->grid = dim3((unsigned)smallc::w2_ctas(s)); g->block = dim3(smallc::NTH);
     g->smem = smallc::wgrad2_smem(s);
     g->func = (const void*)smallc::conv_wgrad_smallc2_kernel;
     return 0;

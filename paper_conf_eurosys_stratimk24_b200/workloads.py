@@ -34,6 +34,12 @@ class Graph:
 
     # ---- buffers
     def buf(self, name, shape, dtype=F32, zero=True):
+        """A named device buffer. Asking again for an existing name returns the same tensor (the op
+        lists hold raw pointers, so a buffer must never be replaced while the graph lives)."""
+        old = self.bufs.get(name)
+        if old is not None:
+            assert tuple(old.shape) == tuple(shape) and old.dtype == dtype, f"buffer {name} redefined"
+            return old
         t = torch.zeros(shape, dtype=dtype, device=self.device) if zero else torch.empty(shape, dtype=dtype, device=self.device)
         self.bufs[name] = t
         return t
@@ -825,7 +831,7 @@ def encoder_train_graph(host_params, xs, ts, layers=6, d=512, heads=8, ffn=2048,
     b, sq, _ = xs[0].shape
     rows = b * sq
     xb = [g.buf(f"x{i}", (rows, d)) for i in range(len(xs))]
-    tb = [g.buf(f"t{i}", (rows, d)) for i in range(len(ts))]
+    tb = [g.buf(f"tgt{i}", (rows, d)) for i in range(len(ts))]
     with torch.no_grad():
         for dst, src in zip(xb + tb, list(xs) + list(ts)):
             dst.copy_(src.reshape(rows, d).to(dst.device))

@@ -94,3 +94,16 @@ def test_variants_share_one_live_workspace():
         for fn, args, lab in v:
             if fn == "mse":
                 assert args[5] == gm._ws.data_ptr()
+
+
+def test_graph_buffers_never_replaced():
+    """Op lists hold raw device pointers: a second request for a named buffer (e.g. a per-op scratch
+    built once per op-list variant) must return the same tensor, never free the first one."""
+    from paper_conf_eurosys_stratimk24_b200 import workloads as W
+    g = W.Graph("t", device="cpu")
+    a = g.buf("col.x", (4, 4))
+    b = g.buf("col.x", (4, 4))
+    assert a.data_ptr() == b.data_ptr()
+    import pytest
+    with pytest.raises(AssertionError):
+        g.buf("col.x", (2, 4))

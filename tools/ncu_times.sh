@@ -2,7 +2,7 @@
 # Per-launch device time of every op of one client (solo runner), under ncu (serialised, cold-ish caches).
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
-OURS='(gemm_|gemv_bt_kernel|conv_fwd_smallc|unary_kernel|binary_kernel|bn_|dw_|maxpool_kernel|maxpool_bwd_kernel|attention_kernel|layernorm_kernel|gelu_kernel|add_bf16_kernel|embed_kernel|col2im_kernel|ln_fwd_kernel|ln_bwd_kernel|attn_|avgpool|ce_kernel|mse_kernel|sgd_kernel|colsum_kernel|smallc_kernel)'
+OURS='(gemm_|gemv_bt_kernel|conv_fwd_smallc|unary_kernel|binary_kernel|bn_|dw_|maxpool_kernel|maxpool_bwd_kernel|attention_kernel|layernorm_kernel|gelu_kernel|add_bf16_kernel|embed_kernel|col2im_kernel|ln_fwd_kernel|ln_bwd_kernel|attn_|avgpool|ce_kernel|mse_kernel|sgd_kernel|colsum_kernel|smallc_kernel|smallc2_kernel)'
 for c in ${CLIENTS:-hp be}; do
   timeout -s KILL 900 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,launch__grid_size --clock-control none --csv --page raw \
      --kernel-name-base function -k "regex:$OURS" --log-file gpurun_out/ncu_times_${CONFIG:-rn50_mnv2}_${c}.csv python tools/profile/solo_runner.py --config ${CONFIG:-rn50_mnv2} --client $c > gpurun_out/ncu_times_${CONFIG:-rn50_mnv2}_${c}.out 2>&1
