@@ -18,10 +18,11 @@ struct DwShape { int N, H, W, C, stride, P, Q; };
 // registers. S = stride (compile-time 1 or 2).
 constexpr int ROW_WARPS = 8;
 constexpr int DW_U = 4;
+constexpr int DW_UW = 8;   // wgrad: twice the loads in flight per window block (latency-bound, ncu r01)
 
-template <int S>
+template <int S, int U = DW_U>
 struct Win {
-  static constexpr int NC = (DW_U - 1) * S + 3;   // input columns per block of U outputs
+  static constexpr int NC = (U - 1) * S + 3;   // input columns per block of U outputs
   float v[3][NC];
   // columns col0 .. col0+NC-1 of the 3 input rows (zero outside the image / missing rows)
   __device__ __forceinline__ void load(const float* const (&rowp)[3], const bool (&rv)[3], int col0, int W, int C) {
@@ -212,14 +213,14 @@ __global__ void __launch_bounds__(DW_THREADS) dw_wgrad_rows_kernel(const float* 
       float f[9];
 #pragma unroll
       for (int t = 0; t < 9; t++) f[t] = 0.f;
-      for (int q0 = 0; q0 < s.Q; q0 += DW_U) {
-        Win<S> win;
+      for (int q0 = 0; q0 < s.Q; q0 += DW_UW) {
+        Win<S, DW_UW> win;
         win.load(xr, rv, q0 * S - 1, s.W, s.C);
-        float g[DW_U];
+        float g[DW_UW];
 #pragma unroll
-        for (int u = 0; u < DW_U; u++) g[u] = (q0 + u < s.Q) ? __ldg(gr + (long long)(q0 + u) * s.C) : 0.f;
+        for (int u = 0; u < DW_UW; u++) g[u] = (q0 + u < s.Q) ? __ldg(gr + (long long)(q0 + u) * s.C) : 0.f;
 #pragma unroll
-        for (int u = 0; u < DW_U; u++)
+        for (int u = 0; u < DW_UW; u++)
 #pragma unroll
           for (int r = 0; r < 3; r++)
 #pragma unroll
