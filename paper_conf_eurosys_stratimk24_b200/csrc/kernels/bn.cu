@@ -201,20 +201,32 @@ __global__ void __launch_bounds__(BN_THREADS) bn_apply_kernel(const float* __res
                                                               const float* __restrict__ beta, const float* __restrict__ mean,
                                                               const float* __restrict__ invstd, long long total, int C, OrionSig sig) {
   if ((C & 3) == 0) {
-    long long nv = total / 4;
-    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nv; i += (long long)gridDim.x * blockDim.x) {
-      int c = (int)((i * 4) % C);
-      float4 xv = __ldg(reinterpret_cast<const float4*>(x) + i);
-      float4 m = __ldg(reinterpret_cast<const float4*>(mean + c));
-      float4 is = __ldg(reinterpret_cast<const float4*>(invstd + c));
-      float4 g = __ldg(reinterpret_cast<const float4*>(gamma + c));
-      float4 b = __ldg(reinterpret_cast<const float4*>(beta + c));
-      float4 o;
-      o.x = fmaf(xv.x - m.x, is.x * g.x, b.x);
-      o.y = fmaf(xv.y - m.y, is.y * g.y, b.y);
-      o.z = fmaf(xv.z - m.z, is.z * g.z, b.z);
-      o.w = fmaf(xv.w - m.w, is.w * g.w, b.w);
-      reinterpret_cast<float4*>(y)[i] = o;
+    // fixed channel quad per thread (per-channel vectors loaded once), lanes stride over rows
+    const int q = C / 4;
+    const long long rows = total / C;
+    const long long gt = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const long long L = ((long long)gridDim.x * blockDim.x) / q;
+    const int cq = (int)(gt % q);
+    const long long lane = gt / q;
+    if (lane < L) {
+      const int c = cq * 4;
+      const float4 m = __ldg(reinterpret_cast<const float4*>(mean + c));
+      const float4 is = __ldg(reinterpret_cast<const float4*>(invstd + c));
+      const float4 g = __ldg(reinterpret_cast<const float4*>(gamma + c));
+      const float4 b = __ldg(reinterpret_cast<const float4*>(beta + c));
+      const float4 sc = make_float4(is.x * g.x, is.y * g.y, is.z * g.z, is.w * g.w);
+      auto one = [&](const float4& xv) {
+        return make_float4(fmaf(xv.x - m.x, sc.x, b.x), fmaf(xv.y - m.y, sc.y, b.y), fmaf(xv.z - m.z, sc.z, b.z), fmaf(xv.w - m.w, sc.w, b.w));
+      };
+      const float4* x4 = reinterpret_cast<const float4*>(x);
+      float4* y4 = reinterpret_cast<float4*>(y);
+      long long r = lane;
+      for (; r + 3 * L < rows; r += 4 * L) {
+        const long long i0 = r * q + cq, i1 = (r + L) * q + cq, i2 = (r + 2 * L) * q + cq, i3 = (r + 3 * L) * q + cq;
+        const float4 a0 = __ldg(x4 + i0), a1 = __ldg(x4 + i1), a2 = __ldg(x4 + i2), a3 = __ldg(x4 + i3);
+        y4[i0] = one(a0); y4[i1] = one(a1); y4[i2] = one(a2); y4[i3] = one(a3);
+      }
+      for (; r < rows; r += L) y4[r * q + cq] = one(__ldg(x4 + r * q + cq));
     }
   } else {
     for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
@@ -239,19 +251,40 @@ __global__ void __launch_bounds__(BN_THREADS) bn_bwd_dx_kernel(const float* __re
   const long long total = rows * C;
   const double invN = 1.0 / (double)rows;
   if ((C & 3) == 0) {
-    const long long nv = total / 4;
-    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nv; i += (long long)gridDim.x * blockDim.x) {
-      const int c = (int)((i * 4) % C);
-      float4 xv = __ldg(reinterpret_cast<const float4*>(x) + i), gv = __ldg(reinterpret_cast<const float4*>(dy) + i);
-      float4 ga = __ldg(reinterpret_cast<const float4*>(gamma + c)), mu = __ldg(reinterpret_cast<const float4*>(mean + c));
-      float4 is = __ldg(reinterpret_cast<const float4*>(invstd + c)), dg = __ldg(reinterpret_cast<const float4*>(dgamma + c));
-      float4 db = __ldg(reinterpret_cast<const float4*>(dbeta + c));
-      float4 o;
-      o.x = bn_dx1(xv.x, gv.x, ga.x, mu.x, is.x, dg.x, db.x, invN);
-      o.y = bn_dx1(xv.y, gv.y, ga.y, mu.y, is.y, dg.y, db.y, invN);
-      o.z = bn_dx1(xv.z, gv.z, ga.z, mu.z, is.z, dg.z, db.z, invN);
-      o.w = bn_dx1(xv.w, gv.w, ga.w, mu.w, is.w, dg.w, db.w, invN);
-      reinterpret_cast<float4*>(dx)[i] = o;
+    // thread -> fixed channel quad cq (its 5 per-channel vectors loaded once) and row lane; lanes
+    // stride over rows, so a warp's 32 float4 loads are consecutive in memory; 2 rows in flight
+    const int q = C / 4;
+    const long long gt = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const long long L = ((long long)gridDim.x * blockDim.x) / q;
+    const int cq = (int)(gt % q);
+    const long long lane = gt / q;
+    if (lane < L) {
+      const int c = cq * 4;
+      const float4 ga = __ldg(reinterpret_cast<const float4*>(gamma + c)), mu = __ldg(reinterpret_cast<const float4*>(mean + c));
+      const float4 is = __ldg(reinterpret_cast<const float4*>(invstd + c)), dg = __ldg(reinterpret_cast<const float4*>(dgamma + c));
+      const float4 db = __ldg(reinterpret_cast<const float4*>(dbeta + c));
+      auto one = [&](const float4& xv, const float4& gv) {
+        float4 o;
+        o.x = bn_dx1(xv.x, gv.x, ga.x, mu.x, is.x, dg.x, db.x, invN);
+        o.y = bn_dx1(xv.y, gv.y, ga.y, mu.y, is.y, dg.y, db.y, invN);
+        o.z = bn_dx1(xv.z, gv.z, ga.z, mu.z, is.z, dg.z, db.z, invN);
+        o.w = bn_dx1(xv.w, gv.w, ga.w, mu.w, is.w, dg.w, db.w, invN);
+        return o;
+      };
+      const float4* x4 = reinterpret_cast<const float4*>(x);
+      const float4* g4 = reinterpret_cast<const float4*>(dy);
+      float4* d4 = reinterpret_cast<float4*>(dx);
+      long long r = lane;
+      for (; r + L < rows; r += 2 * L) {
+        const long long i0 = r * q + cq, i1 = (r + L) * q + cq;
+        const float4 x0 = __ldg(x4 + i0), g0 = __ldg(g4 + i0), x1 = __ldg(x4 + i1), g1 = __ldg(g4 + i1);
+        d4[i0] = one(x0, g0);
+        d4[i1] = one(x1, g1);
+      }
+      if (r < rows) {
+        const long long i0 = r * q + cq;
+        d4[i0] = one(__ldg(x4 + i0), __ldg(g4 + i0));
+      }
     }
   } else {
     for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
