@@ -1728,6 +1728,9 @@ struct Plan { int cfg; int split; int bm, bn, bk; };
 
 // Skinny A^T B (cfg 5/6/7 = variants V44/V84/V48): the whole M x N fits one CTA's register
 // blocks (<= 256 of them), long K.
+// First fitting variant in this order (measured: the 8x8 variant's 16-row stages cost more than its
+// higher FMA-per-load ratio gains on MobileNetV2's narrow weight gradients, so it only takes the
+// shapes no other variant fits: ResNet's 256 x 64 / 64 x 256 / 128 x 128).
 int atb_variant(long long M, long long N, long long K) {
   if (K < 4096) return -1;
   if (atb::V44::fits(M, N)) return 5;
