@@ -329,6 +329,24 @@ def main():
     col = C.latency_stats(rc)
     be_col, be_n = C.be_throughput(rc, rc["t0"], rc["t_hp_end"])
     clocks = clk.summary()
+    # combined utilisation of the pair (analytic): algorithmic HBM bytes and FLOPs of
+    # the work completed in the window / (window x peak), collocated vs each client alone
+    hp_b, hp_f = sum(r["bytes"] for r in rows_hp), sum(r["flops"] for r in rows_hp)
+    be_b, be_f = sum(r["bytes"] for r in rows_be), sum(r["flops"] for r in rows_be)
+    win_s = (rc["t_hp_end"] - rc["t0"]) / 1e9
+    n_hp_done = len(rc["t_done"])
+    pk_u, _ = peaks()
+    tc_peak = pk_u.get("bf16_tflops_sustained", pk_u["bf16_tflops"]) * 1e12 / (6.0 if W_.get("dtype", "f32") == "f32" else 1.0)
+    hbm_peak = pk_u["hbm_gbs"] * 1e9
+    util = {
+        "collocated": {"hbm_gbs": (n_hp_done * hp_b + be_n * be_b) / win_s / 1e9,
+                       "hbm_frac": (n_hp_done * hp_b + be_n * be_b) / win_s / hbm_peak,
+                       "flop_frac": (n_hp_done * hp_f + be_n * be_f) / win_s / tc_peak},
+        "hp_alone": {"hbm_gbs": ded["n"] * hp_b / ((rd["t_done"][-1] - rd["t0"]) / 1e9) / 1e9,
+                     "flop_frac": ded["n"] * hp_f / ((rd["t_done"][-1] - rd["t0"]) / 1e9) / tc_peak},
+        "be_alone": {"hbm_gbs": be_ded * be_b / 1e9, "hbm_frac": be_ded * be_b / hbm_peak, "flop_frac": be_ded * be_f / tc_peak},
+        "basis": "algorithmic bytes/FLOPs per op (profiler.op_work) x completed requests / iterations; flop peak = the "
+                 "algorithmic ceiling of the path's tensor pipe (bf16, or bf16/6 for fp32 on 3xTF32)"}
     # roofline of the dominant kernel from its live launches inside the timed region
     tr = rc.get("trace_ms", [])
     flops, nbytes = top_row["flops"], top_row["bytes"]
@@ -425,6 +443,7 @@ def main():
         "gpu_launches": int(world * args.steps * n_hp_k + sum(r["be_n"] for r in allr) * n_be_k),
         "clocks": clocks,
         "scheduler": rc["stats"],
+        "utilisation": util,
     }
     print(json.dumps(line), flush=True)
 
