@@ -1728,15 +1728,14 @@ struct Plan { int cfg; int split; int bm, bn, bk; };
 
 // Skinny A^T B (cfg 5/6/7 = variants V44/V84/V48): the whole M x N fits one CTA's register
 // blocks (<= 256 of them), long K.
-// First fitting variant in this order (measured: the 8x8 variant's 16-row stages cost more than its
-// higher FMA-per-load ratio gains on MobileNetV2's narrow weight gradients, so it only takes the
-// shapes no other variant fits: ResNet's 256 x 64 / 64 x 256 / 128 x 128).
+// First fitting variant in this order. The 8x8 variant (V88) is compiled but not routed: measured
+// slower than the alternatives everywhere (MobileNetV2's narrow weight gradients 2x; ResNet-50's
+// 64 x 256 layer-1 weight gradient 369 us vs 282 us on the split-K tensor-core path), ncu r01.
 int atb_variant(long long M, long long N, long long K) {
   if (K < 4096) return -1;
   if (atb::V44::fits(M, N)) return 5;
   if (atb::V84::fits(M, N)) return 6;
   if (atb::V48::fits(M, N)) return 7;
-  if (atb::V88::fits(M, N)) return 8;
   return -1;
 }
 bool atb_ok(long long M, long long N, long long K) { return atb_variant(M, N, K) >= 0; }
