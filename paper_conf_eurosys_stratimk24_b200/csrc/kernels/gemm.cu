@@ -1419,7 +1419,6 @@ struct V {
 using V44 = V<4, 4, 64, 128, 128>;
 using V84 = V<8, 4, 32, 192, 64>;
 using V48 = V<4, 8, 32, 64, 192>;
-using V88 = V<8, 8, 16, 256, 256>;   // 256 x 64 / 64 x 256 / 128 x 128 (ResNet's 1x1 weight gradients)
 
 template <class VV, int TMB, int TNB, int R>
 __global__ void __launch_bounds__(NTH) gemm_atb_kernel(GemmParams p, const float* __restrict__ A, long long lda,
@@ -1728,9 +1727,8 @@ struct Plan { int cfg; int split; int bm, bn, bk; };
 
 // Skinny A^T B (cfg 5/6/7 = variants V44/V84/V48): the whole M x N fits one CTA's register
 // blocks (<= 256 of them), long K.
-// First fitting variant in this order. The 8x8 variant (V88) is compiled but not routed: measured
-// slower than the alternatives everywhere (MobileNetV2's narrow weight gradients 2x; ResNet-50's
-// 64 x 256 layer-1 weight gradient 369 us vs 282 us on the split-K tensor-core path), ncu r01.
+// First fitting variant in this order. (An 8x8 register-block variant was measured slower than these
+// and than the split-K tensor-core path on ResNet-50's 64 x 256 weight gradients, ncu r01.)
 int atb_variant(long long M, long long N, long long K) {
   if (K < 4096) return -1;
   if (atb::V44::fits(M, N)) return 5;
@@ -1742,7 +1740,7 @@ bool atb_ok(long long M, long long N, long long K) { return atb_variant(M, N, K)
 
 Plan plan_atb(long long M, long long N, long long K) {
   Plan pl;
-  pl.cfg = atb_variant(M, N, K); pl.bm = (int)M; pl.bn = (int)N; pl.bk = pl.cfg == 5 ? 64 : (pl.cfg == 8 ? 16 : 32);
+  pl.cfg = atb_variant(M, N, K); pl.bm = (int)M; pl.bn = (int)N; pl.bk = pl.cfg == 5 ? 64 : 32;
   long long split = cdiv(148 * 4, 1);
   long long kmax = K / (4 * pl.bk);
   if (split > kmax) split = kmax;
@@ -2251,17 +2249,14 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
           cudaFuncSetAttribute((const void*)atb::gemm_atb_kernel<atb::V84, 8, 4, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                atb::V84::smem_bytes(192, 64)) != cudaSuccess ||
           cudaFuncSetAttribute((const void*)atb::gemm_atb_kernel<atb::V48, 4, 8, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               atb::V48::smem_bytes(64, 192)) != cudaSuccess ||
-          cudaFuncSetAttribute((const void*)atb::gemm_atb_kernel<atb::V88, 8, 8, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               atb::V88::smem_bytes(256, 256)) != cudaSuccess)
+                               atb::V48::smem_bytes(64, 192)) != cudaSuccess)
         return ORION_E_CUDA;
       attr.store(1);
     }
     g->grid = dim3(1, 1, (unsigned)pl.split); g->block = dim3(atb::NTH);
     if (pl.cfg == 5) { g->smem = atb::V44::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V44, 4, 4, 64>; }
     else if (pl.cfg == 6) { g->smem = atb::V84::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V84, 8, 4, 32>; }
-    else if (pl.cfg == 7) { g->smem = atb::V48::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V48, 4, 8, 32>; }
-    else { g->smem = atb::V88::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V88, 8, 8, 16>; }
+    else { g->smem = atb::V48::smem_bytes((int)M, (int)N); g->func = (const void*)atb::gemm_atb_kernel<atb::V48, 4, 8, 32>; }
     return 0;
   }
   switch (flags) {
@@ -2308,10 +2303,6 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
   }
   if (g.func == (const void*)atb::gemm_atb_kernel<atb::V48, 4, 8, 32>) {
     atb::gemm_atb_kernel<atb::V48, 4, 8, 32><<<g.grid, g.block, g.smem, s>>>(make_params(M, N, K, C, ldc, bias, (int)g.grid.z, ws, 32), A, lda, B, ldb, sig);
-    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
-  }
-  if (g.func == (const void*)atb::gemm_atb_kernel<atb::V88, 8, 8, 16>) {
-    atb::gemm_atb_kernel<atb::V88, 8, 8, 16><<<g.grid, g.block, g.smem, s>>>(make_params(M, N, K, C, ldc, bias, (int)g.grid.z, ws, 16), A, lda, B, ldb, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
   switch (flags) {
