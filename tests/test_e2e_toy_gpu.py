@@ -111,3 +111,24 @@ def test_toy_three_be_clients(toy):
         b.graph.params.reset()
         C.run_session(be=b, be_iters=K)
         assert torch.equal(b.graph.params.flat.cpu(), p_col)
+
+
+@pytest.mark.parametrize("policy", ["priorities", "profiles", "streams", "orion_noprio"])
+def test_toy_policy_ablation_log(toy, policy):
+    """The ablation switches (Fig. 14) on real kernels: the decision log of each
+    policy variant equals the oracle replay of its own tape, and outputs stay bitwise identical to
+    the default policy's solo run (scheduling never changes results)."""
+    hp, be = toy["hp"], toy["be"]
+    be.graph.params.reset()
+    hp.out.zero_()
+    res = C.run_session(hp=hp, be=be, arrivals_ns=toy["arrivals"][:60], log_capacity=1 << 22, hp_latency_ns=20_000,
+                        flags=L.POLICIES[policy])
+    hdr, prefix, tape, decs = lf.split_log(res["log"])
+    assert decs == po.replay(prefix)
+    kinds = {d[1] for d in lf.decode_decisions(decs)}
+    if policy in ("priorities", "streams"):
+        assert not kinds & {5, 6, 7, 8}, kinds      # no defers, no resets: every BE op admitted at once
+    out_col = hp.out[:60].clone()
+    hp.out.zero_()
+    C.run_session(hp=hp, arrivals_ns=toy["arrivals"][:60])
+    assert torch.equal(hp.out[:60], out_col)
