@@ -142,15 +142,16 @@ __global__ void __launch_bounds__(BN_THREADS) bn_bwd_reduce_kernel(const float* 
       sgx.w = fma((double)g.w, ((double)v.w - mu.w) * is.w, sgx.w);
     };
     long long r = r0 + rl;
-    for (; r + 7LL * rl_n < r1; r += 8LL * rl_n) {   // 16 128-bit loads in flight per thread
-      float4 g[8], v[8];
-#pragma unroll
-      for (int i = 0; i < 8; i++) {
-        g[i] = __ldg(reinterpret_cast<const float4*>(gp + (r + i * (long long)rl_n) * C));
-        v[i] = __ldg(reinterpret_cast<const float4*>(xp + (r + i * (long long)rl_n) * C));
-      }
-#pragma unroll
-      for (int i = 0; i < 8; i++) acc(g[i], v[i]);
+    for (; r + 3LL * rl_n < r1; r += 4LL * rl_n) {
+      float4 g0 = __ldg(reinterpret_cast<const float4*>(gp + r * C));
+      float4 g1 = __ldg(reinterpret_cast<const float4*>(gp + (r + rl_n) * C));
+      float4 g2 = __ldg(reinterpret_cast<const float4*>(gp + (r + 2LL * rl_n) * C));
+      float4 g3 = __ldg(reinterpret_cast<const float4*>(gp + (r + 3LL * rl_n) * C));
+      float4 v0 = __ldg(reinterpret_cast<const float4*>(xp + r * C));
+      float4 v1 = __ldg(reinterpret_cast<const float4*>(xp + (r + rl_n) * C));
+      float4 v2 = __ldg(reinterpret_cast<const float4*>(xp + (r + 2LL * rl_n) * C));
+      float4 v3 = __ldg(reinterpret_cast<const float4*>(xp + (r + 3LL * rl_n) * C));
+      acc(g0, v0); acc(g1, v1); acc(g2, v2); acc(g3, v3);
     }
     for (; r < r1; r += rl_n)
       acc(__ldg(reinterpret_cast<const float4*>(gp + r * C)), __ldg(reinterpret_cast<const float4*>(xp + r * C)));
