@@ -40,7 +40,7 @@ def peaks():
 
 
 # --------------------------------------------------------------------------------- workloads
-def build_config(name, rank):
+def build_config(name, rank, be_sub=0):
     from paper_conf_eurosys_stratimk24_b200 import workloads as W
     from synth import inputs as si
     if name == "toy":
@@ -60,8 +60,8 @@ def build_config(name, rank):
         hp_inputs = [si.token_ids((8, 128), 30522, si.HP_SEED, sub=r).reshape(-1).view(torch.float32) for r in range(16)]
         hpg = W.bert_infer_graph(Pb, batch=8, seq=128)
         Prn = si.make_params(W.resnet_train_spec())
-        xs = [si.normal((64, 224, 224, 3), si.BE_SEED, sub=i) for i in range(8)]
-        labels = [si.labels(64, 1000, si.BE_SEED, sub=i) for i in range(8)]
+        xs = [si.normal((64, 224, 224, 3), si.BE_SEED, sub=be_sub + i) for i in range(8)]
+        labels = [si.labels(64, 1000, si.BE_SEED, sub=be_sub + i) for i in range(8)]
         beg = W.resnet_train_graph(Prn, xs, labels)
         return dict(hpg=hpg, beg=beg, hp_inputs=hp_inputs, rate=4.0, be_inputs=xs, dtype="bf16 (HP) + f32 (BE)",
                     cfg={"workload": "HP BERT-base inference b8 s128 bf16 (Poisson 4 rps) + BE ResNet-50 training b64, 1 B200 per instance",
@@ -71,8 +71,8 @@ def build_config(name, rank):
     hp_inputs = [si.normal((4, 224, 224, 3), si.HP_SEED, sub=r) for r in range(16)]
     hpg = W.resnet_infer_graph(Prn, batch=4)
     Pmn = si.make_params(W.mnv2_spec())
-    xs = [si.normal((96, 224, 224, 3), si.BE_SEED, sub=i) for i in range(8)]
-    labels = [si.labels(96, 1000, si.BE_SEED, sub=i) for i in range(8)]
+    xs = [si.normal((96, 224, 224, 3), si.BE_SEED, sub=be_sub + i) for i in range(8)]
+    labels = [si.labels(96, 1000, si.BE_SEED, sub=be_sub + i) for i in range(8)]
     beg = W.mnv2_train_graph(Pmn, xs, labels)
     return dict(hpg=hpg, beg=beg, hp_inputs=hp_inputs, rate=15.0, be_inputs=xs,
                 cfg={"workload": "HP ResNet-50 inference b4 (Poisson 15 rps) + BE MobileNetV2 training b96, 1 B200 per instance",
@@ -231,6 +231,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--rate", type=float, default=0.0, help="override HP arrival rate (rps)")
+    ap.add_argument("--n-be", type=int, default=1, help="number of BE clients (R11; default 1)")
     ap.add_argument("--policy", default="orion", choices=["orion", "orion_noprio", "profiles", "priorities", "streams"],
                     help="policy ablation (Fig. 14) / Streams baselines (P:1003-1014); orion = the full policy")
     args = ap.parse_args()
@@ -274,6 +275,15 @@ def main():
     beg.params.reset()
     hp = C.HPClient(hpg, W_["hp_inputs"], max(args.steps, 64), prof_hp, 0)
     be = C.BEClient(beg, prof_be, 10000)
+    # --n-be > 1: more BE clients of the same model on their own data (R11: one shared DUR budget,
+    # round robin); BE throughput is summed over the clients, dedicated = the BE clients without HP
+    extra_be = []
+    for j in range(1, args.n_be):
+        gj = build_config(args.config, rank, be_sub=8 * j)["beg"]
+        pj, _ = PR.build_profiles(gj, 10000 * (j + 1), reps=3, ncu_csv=None)
+        gj.params.reset()
+        extra_be.append(C.BEClient(gj, pj, 10000 * (j + 1)))
+    be_all = [be] + extra_be if extra_be else be
     n_hp_k = sum(1 for o in hp.ops if o.kind == L.OP_KERNEL)
     n_be_k = sum(1 for o in be.variants[0] if o.kind == L.OP_KERNEL)
     sched_cpu = 2 + 4 * local if (os.cpu_count() or 1) >= 8 else -1
@@ -303,9 +313,10 @@ def main():
     rb = session(be=be, be_iters=3)
     per_it = (time.time() - t0) / 3
     n_it = int(max(5, min(200, 6.0 / max(per_it, 1e-6))))
-    rb = session(be=be, be_iters=n_it)
-    tb = rb["be_t_end"]
-    be_ded = (len(tb) - 1) / ((tb[-1] - tb[0]) / 1e9) if len(tb) > 1 else float("nan")
+    rb = session(be=be_all, be_iters=n_it)
+    be_ded = 0.0
+    for tb in rb.get("be_t_end_all", [rb["be_t_end"]]):
+        be_ded += (len(tb) - 1) / ((tb[-1] - tb[0]) / 1e9) if len(tb) > 1 else float("nan")
     # ---- dominant BE kernel (largest share of solo time) for the roofline
     shares = {}
     for r in rows_be:
@@ -319,7 +330,7 @@ def main():
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         e0.record()
-        rc = session(hp=hp, be=be, arrivals_ns=arrivals, hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm,
+        rc = session(hp=hp, be=be_all, arrivals_ns=arrivals, hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm,
                      be_partition_sms=args.be_partition, trace_kernel_id=top_kid)
         torch.cuda.synchronize()
         e1.record()
@@ -327,7 +338,10 @@ def main():
     barrier()
     win_ms = e0.elapsed_time(e1)
     col = C.latency_stats(rc)
-    be_col, be_n = C.be_throughput(rc, rc["t0"], rc["t_hp_end"])
+    be_col, be_n = 0.0, 0
+    for tb in rc.get("be_t_end_all", [rc["be_t_end"]]):
+        c_, n_ = C.be_throughput({"be_t_end": tb}, rc["t0"], rc["t_hp_end"])
+        be_col, be_n = be_col + c_, be_n + n_
     clocks = clk.summary()
     # combined utilisation of the pair (analytic): algorithmic HBM bytes and FLOPs of
     # the work completed in the window / (window x peak), collocated vs each client alone
@@ -383,7 +397,7 @@ def main():
             traffic = ncu_rows[top_kid][2]
     # ---- e2e: BE inputs copied from pinned host each iteration (H2D) + loss read back (D2H)
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and not extra_be:
         variants, pinned, loss_host, be_h2d = with_be_h2d(beg, W_["be_inputs"])
         from paper_conf_eurosys_stratimk24_b200.workloads import Graph  # noqa: F401
         be_e2e = C.BEClient.__new__(C.BEClient)
@@ -423,7 +437,7 @@ def main():
         "data": "synthetic (seeded; DESIGN.md §5)",
         "config": dict(W_["cfg"], parallelism=f"replicas x{world} (independent Orion instance per GPU)",
                        hp_rate_rps=rate, dur_threshold_pct=args.dur_ppm / 1e4, be_partition_sms=args.be_partition,
-                       policy=args.policy,
+                       policy=args.policy, n_be_clients=args.n_be,
                        l2=f"inputs > L2 (BE batch {W_['be_inputs'][0].numel() * 4 / 1e6:.1f} MB x 8 staged; no flush)"),
         "hp": {"p50_ms": col["p50_ns"] / 1e6, "p99_ms": col["p99_ns"] / 1e6, "dedicated_p50_ms": ded["p50_ns"] / 1e6,
                "dedicated_p99_ms": ded["p99_ns"] / 1e6, "p99_vs_dedicated": col["p99_ns"] / ded["p99_ns"],
