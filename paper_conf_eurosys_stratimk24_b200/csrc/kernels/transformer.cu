@@ -105,7 +105,7 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, float* v) {
 template <int BN>
 struct Cfg {
   static constexpr int A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2, STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES = (192 * 1024) / STAGE_BYTES;   // 6 (BN 128) / 8 (BN 64)
+  static constexpr int STAGES = (192 * 1024) / STAGE_BYTES;   // 4 (BN 256) / 6 (BN 128) / 8 (BN 64)
   static constexpr int EPI_LD = BN + 8;                        // padded bf16 staging row
   static constexpr int EPI_BYTES = BM * EPI_LD * 2;
   static constexpr int MAIN = STAGES * STAGE_BYTES > EPI_BYTES ? STAGES * STAGE_BYTES : EPI_BYTES;
@@ -142,7 +142,7 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_bf16_kernel(const __grid_constan
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)), "r"(Cf::TMEM_COLS) : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
-  if (tid < BN) bias_s[tid] = (bias != nullptr && n0 + tid < N) ? bf2f(bias[n0 + tid]) : 0.f;
+  for (int i = tid; i < BN; i += NTHR) bias_s[i] = (bias != nullptr && n0 + i < N) ? bf2f(bias[n0 + i]) : 0.f;
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
   __syncthreads();
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
@@ -224,7 +224,12 @@ bool prepare() {
 }
 // Tile width from the shape only (never the SM partition): 128 when that still gives >= one CTA
 // per SM of a whole B200, else 64 (twice the CTAs for BERT-base's N = 768 projections).
-inline int bn_for(long long M, long long N) { return cdiv(M, BM) * cdiv(N, 128) >= 148 ? 128 : 64; }
+// 256-wide tiles (the widest UMMA N: most MMA work per staged A tile) when they still give >= 96
+// CTAs (BERT's FFN up-projection), else 128 when that gives >= one CTA per SM, else 64.
+inline int bn_for(long long M, long long N) {
+  if (cdiv(M, BM) * cdiv(N, 256) >= 96) return 256;
+  return cdiv(M, BM) * cdiv(N, 128) >= 148 ? 128 : 64;
+}
 
 // cuTensorMapEncodeTiled through cudart's driver entry point (liborion does not link libcuda)
 typedef CUresult (*encode_fn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
@@ -571,7 +576,10 @@ int gemm_bf16_geom(const uint64_t* a, LaunchGeom* g) {
   const int bn = tcb::bn_for(M, N);
   g->grid = dim3((unsigned)cdiv(N, bn), (unsigned)cdiv(M, tcb::BM));
   g->block = dim3(tcb::NTHR);
-  if (bn == 128) {
+  if (bn == 256) {
+    if (!tcb::prepare<256>()) return ORION_E_CUDA;
+    g->smem = tcb::Cfg<256>::SMEM; g->func = (const void*)tcb::gemm_bf16_kernel<256>;
+  } else if (bn == 128) {
     if (!tcb::prepare<128>()) return ORION_E_CUDA;
     g->smem = tcb::Cfg<128>::SMEM; g->func = (const void*)tcb::gemm_bf16_kernel<128>;
   } else {
@@ -582,11 +590,13 @@ int gemm_bf16_geom(const uint64_t* a, LaunchGeom* g) {
 }
 int gemm_bf16_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   const long long M = (long long)a[4], N = (long long)a[5], K = (long long)a[6];
-  const bool wide = g.func == (const void*)tcb::gemm_bf16_kernel<128>;
+  const int bn = g.func == (const void*)tcb::gemm_bf16_kernel<256> ? 256 : g.func == (const void*)tcb::gemm_bf16_kernel<128> ? 128 : 64;
   CUtensorMap ma, mw;
-  if (!tcb::map_bf16(&ma, (const void*)a[0], M, K, tcb::BM) || !tcb::map_bf16(&mw, (const void*)a[1], N, K, wide ? 128 : 64))
+  if (!tcb::map_bf16(&ma, (const void*)a[0], M, K, tcb::BM) || !tcb::map_bf16(&mw, (const void*)a[1], N, K, bn))
     return ORION_E_CUDA;
-  if (wide)
+  if (bn == 256)
+    tcb::gemm_bf16_kernel<256><<<g.grid, g.block, g.smem, s>>>(ma, mw, (bf16*)a[2], (const bf16*)a[3], (int)M, (int)N, (int)K, sig);
+  else if (bn == 128)
     tcb::gemm_bf16_kernel<128><<<g.grid, g.block, g.smem, s>>>(ma, mw, (bf16*)a[2], (const bf16*)a[3], (int)M, (int)N, (int)K, sig);
   else
     tcb::gemm_bf16_kernel<64><<<g.grid, g.block, g.smem, s>>>(ma, mw, (bf16*)a[2], (const bf16*)a[3], (int)M, (int)N, (int)K, sig);
