@@ -14,12 +14,18 @@ def test_specs_match_oracle():
     assert W.resnet_spec() == om.resnet_spec()
     assert W.mnv2_spec() == om.mnv2_spec()
     assert W.mnv2_blocks() == om.mnv2_blocks()
+    assert W.bert_spec(layers=2) == om.bert_spec(layers=2)
+    assert W.resnet_train_spec() == om.resnet_train_spec()
+    assert W.resnet_train_spec(W.RESNET101_LAYERS) == om.resnet_train_spec(om.RESNET101_LAYERS)
+    assert W.encoder_spec(2) == om.encoder_spec(2)
 
 
 NARGS = {"gemm": 13, "colsum": 4, "relu": 3, "relu_bwd": 4, "relu6": 3, "relu6_bwd": 4, "add": 4, "mse": 6, "sgd": 6,
          "conv_fwd": 16, "conv_dgrad": 16, "conv_wgrad": 16, "dw_fwd": 14, "dw_dgrad": 14, "dw_wgrad": 16,
          "bn_eval": 9, "bn_stats": 11, "bn_apply": 8, "bn_bwd_reduce": 10, "bn_bwd_dx": 10, "maxpool": 8,
-         "avgpool": 5, "avgpool_bwd": 5, "ce": 7}
+         "avgpool": 5, "avgpool_bwd": 5, "ce": 7, "gemm_bf16": 7, "attention": 9, "layernorm": 7, "gelu": 3, "add_bf16": 4,
+         "embed": 9, "maxpool_bwd": 9, "col2im": 12, "layernorm_f32": 9, "layernorm_f32_bwd": 12, "attention_f32": 10,
+         "attention_f32_bwd_dq": 12, "attention_f32_bwd_dkv": 13}
 
 
 def _check(g):
@@ -107,3 +113,24 @@ def test_graph_buffers_never_replaced():
     import pytest
     with pytest.raises(AssertionError):
         g.buf("col.x", (2, 4))
+
+
+def test_config3_config4_graphs():
+    """BERT (bf16), ResNet-50 / -101 training and the encoder: every op carries its args, the HP
+    graphs start with an H2D and end with a D2H memop, and the analytic work of every op is defined
+    (the profiler's roofline / classifier needs it)."""
+    from paper_conf_eurosys_stratimk24_b200 import profiler as PR
+    gb = W.bert_infer_graph(si.make_params(W.bert_spec(layers=2)), batch=2, seq=32, layers=2, device="cpu")
+    gr = W.resnet_train_graph(si.make_params(W.resnet_train_spec()), [si.normal((1, 64, 64, 3), 2)], [si.labels(1, 1000, 2)], device="cpu")
+    ge = W.encoder_train_graph(si.make_params(W.encoder_spec(2)), [si.normal((2, 32, 512), 2)], [si.normal((2, 32, 512), 3)],
+                               layers=2, device="cpu")
+    x = si.normal((1, 64, 64, 3), 1)
+    gh = W.as_hp_training(W.resnet_train_graph(si.make_params(W.resnet_train_spec(W.RESNET101_LAYERS)), [x], [si.labels(1, 1000, 1)],
+                                               layers=W.RESNET101_LAYERS, device="cpu"), x)
+    for g in (gb, gr, ge, gh):
+        _check(g)
+        for i, fn, args, lab in g.kernel_ops():
+            flops, nbytes = PR.op_work(fn, args)
+            assert nbytes > 0, (lab, fn)
+    for g in (gb, gh):
+        assert g.ops[0][0] == L.OP_MEMCPY_H2D and g.ops[-1][0] == L.OP_MEMCPY_D2H
