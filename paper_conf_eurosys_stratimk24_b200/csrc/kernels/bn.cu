@@ -174,18 +174,31 @@ __global__ void __launch_bounds__(BN_THREADS) bn_eval_kernel(const float* __rest
                                                              const float* __restrict__ beta, const float* __restrict__ rm,
                                                              const float* __restrict__ rv, long long total, int C, float eps, OrionSig sig) {
   if ((C & 3) == 0) {
-    const long long nv = total / 4;
-    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nv; i += (long long)gridDim.x * blockDim.x) {
-      const int c = (int)((i * 4) % C);
-      float4 xv = __ldg(reinterpret_cast<const float4*>(x) + i);
-      float4 g = __ldg(reinterpret_cast<const float4*>(gamma + c)), b = __ldg(reinterpret_cast<const float4*>(beta + c));
-      float4 m = __ldg(reinterpret_cast<const float4*>(rm + c)), v = __ldg(reinterpret_cast<const float4*>(rv + c));
-      float4 o;
-      o.x = fmaf(xv.x - m.x, g.x * rsqrtf(v.x + eps), b.x);
-      o.y = fmaf(xv.y - m.y, g.y * rsqrtf(v.y + eps), b.y);
-      o.z = fmaf(xv.z - m.z, g.z * rsqrtf(v.z + eps), b.z);
-      o.w = fmaf(xv.w - m.w, g.w * rsqrtf(v.w + eps), b.w);
-      reinterpret_cast<float4*>(y)[i] = o;
+    // fixed channel quad per thread: the per-channel scale g * rsqrt(var + eps) (the same fp32
+    // operations as the scalar path, so bit-identical to it) is formed once, lanes stride over rows
+    const int q = C / 4;
+    const long long rows = total / C;
+    const long long gt = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    const long long L = ((long long)gridDim.x * blockDim.x) / q;
+    const int cq = (int)(gt % q);
+    const long long lane = gt / q;
+    if (lane < L) {
+      const int c = cq * 4;
+      const float4 g = __ldg(reinterpret_cast<const float4*>(gamma + c)), b = __ldg(reinterpret_cast<const float4*>(beta + c));
+      const float4 m = __ldg(reinterpret_cast<const float4*>(rm + c)), v = __ldg(reinterpret_cast<const float4*>(rv + c));
+      const float4 sc = make_float4(g.x * rsqrtf(v.x + eps), g.y * rsqrtf(v.y + eps), g.z * rsqrtf(v.z + eps), g.w * rsqrtf(v.w + eps));
+      auto one = [&](const float4& xv) {
+        return make_float4(fmaf(xv.x - m.x, sc.x, b.x), fmaf(xv.y - m.y, sc.y, b.y), fmaf(xv.z - m.z, sc.z, b.z), fmaf(xv.w - m.w, sc.w, b.w));
+      };
+      const float4* x4 = reinterpret_cast<const float4*>(x);
+      float4* y4 = reinterpret_cast<float4*>(y);
+      long long r = lane;
+      for (; r + 3 * L < rows; r += 4 * L) {
+        const long long i0 = r * q + cq, i1 = (r + L) * q + cq, i2 = (r + 2 * L) * q + cq, i3 = (r + 3 * L) * q + cq;
+        const float4 a0 = __ldg(x4 + i0), a1 = __ldg(x4 + i1), a2 = __ldg(x4 + i2), a3 = __ldg(x4 + i3);
+        y4[i0] = one(a0); y4[i1] = one(a1); y4[i2] = one(a2); y4[i3] = one(a3);
+      }
+      for (; r < rows; r += L) y4[r * q + cq] = one(__ldg(x4 + r * q + cq));
     }
   } else {
     for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
@@ -260,15 +273,29 @@ __global__ void __launch_bounds__(BN_THREADS) bn_bwd_dx_kernel(const float* __re
     const long long lane = gt / q;
     if (lane < L) {
       const int c = cq * 4;
-      const float4 ga = __ldg(reinterpret_cast<const float4*>(gamma + c)), mu = __ldg(reinterpret_cast<const float4*>(mean + c));
-      const float4 is = __ldg(reinterpret_cast<const float4*>(invstd + c)), dg = __ldg(reinterpret_cast<const float4*>(dgamma + c));
-      const float4 db = __ldg(reinterpret_cast<const float4*>(dbeta + c));
+      // dx = A dy + B x + K per channel, A = gamma invstd, B = -A invstd dgamma / N,
+      // K = -A dbeta / N - B mean (the expression above expanded; coefficients in fp64 once per
+      // thread, so an element costs 2 conversions in, 2 DFMA and 1 conversion out)
+      double A[4], B[4], K[4];
+      {
+        const float4 ga = __ldg(reinterpret_cast<const float4*>(gamma + c)), mu = __ldg(reinterpret_cast<const float4*>(mean + c));
+        const float4 is = __ldg(reinterpret_cast<const float4*>(invstd + c)), dg = __ldg(reinterpret_cast<const float4*>(dgamma + c));
+        const float4 db = __ldg(reinterpret_cast<const float4*>(dbeta + c));
+        const float gv[4] = {ga.x, ga.y, ga.z, ga.w}, mv[4] = {mu.x, mu.y, mu.z, mu.w}, iv[4] = {is.x, is.y, is.z, is.w};
+        const float dgv[4] = {dg.x, dg.y, dg.z, dg.w}, dbv[4] = {db.x, db.y, db.z, db.w};
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+          A[k] = (double)gv[k] * (double)iv[k];
+          B[k] = -A[k] * (double)iv[k] * (double)dgv[k] * invN;
+          K[k] = -A[k] * (double)dbv[k] * invN - B[k] * (double)mv[k];
+        }
+      }
       auto one = [&](const float4& xv, const float4& gv) {
         float4 o;
-        o.x = bn_dx1(xv.x, gv.x, ga.x, mu.x, is.x, dg.x, db.x, invN);
-        o.y = bn_dx1(xv.y, gv.y, ga.y, mu.y, is.y, dg.y, db.y, invN);
-        o.z = bn_dx1(xv.z, gv.z, ga.z, mu.z, is.z, dg.z, db.z, invN);
-        o.w = bn_dx1(xv.w, gv.w, ga.w, mu.w, is.w, dg.w, db.w, invN);
+        o.x = (float)fma(A[0], (double)gv.x, fma(B[0], (double)xv.x, K[0]));
+        o.y = (float)fma(A[1], (double)gv.y, fma(B[1], (double)xv.y, K[1]));
+        o.z = (float)fma(A[2], (double)gv.z, fma(B[2], (double)xv.z, K[2]));
+        o.w = (float)fma(A[3], (double)gv.w, fma(B[3], (double)xv.w, K[3]));
         return o;
       };
       const float4* x4 = reinterpret_cast<const float4*>(x);
@@ -295,9 +322,10 @@ __global__ void __launch_bounds__(BN_THREADS) bn_bwd_dx_kernel(const float* __re
   orion_signal(sig);
 }
 
-void ew(LaunchGeom* g, uint64_t n, const void* f) {
+void ew(LaunchGeom* g, uint64_t n, const void* f, std::atomic<int>& occ) {
   uint64_t ctas = cdiv(n ? n : 1, BN_THREADS);
-  if (ctas > 148 * 8) ctas = 148 * 8;
+  const uint64_t wave = 148ull * resident_ctas_per_sm(f, BN_THREADS, occ);
+  if (ctas > wave) ctas = wave;
   g->grid = dim3((unsigned)ctas); g->block = dim3(BN_THREADS); g->smem = 0; g->func = f;
 }
 
@@ -308,7 +336,8 @@ extern "C" uint64_t orion_bn_workspace_bytes(uint64_t rows, uint64_t C) { return
 #define CHECK_LAUNCH() return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA
 
 // BN eval: x, y, gamma, beta, rm, rv, rows, C, eps_bits
-int bn_eval_geom(const uint64_t* a, LaunchGeom* g) { ew(g, (a[7] & 3) == 0 ? a[6] * a[7] / 4 : a[6] * a[7], (const void*)bn_eval_kernel); return 0; }
+std::atomic<int> bn_eval_occ{0};
+int bn_eval_geom(const uint64_t* a, LaunchGeom* g) { ew(g, (a[7] & 3) == 0 ? a[6] * a[7] / 4 : a[6] * a[7], (const void*)bn_eval_kernel, bn_eval_occ); return 0; }
 int bn_eval_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   bn_eval_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (float*)a[1], (const float*)a[2], (const float*)a[3], (const float*)a[4],
                                             (const float*)a[5], (long long)(a[6] * a[7]), (int)a[7], u2f(a[8]), sig);
@@ -330,7 +359,8 @@ int bn_stats_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaSt
 }
 
 // BN apply: x, y, gamma, beta, mean, invstd, rows, C
-int bn_apply_geom(const uint64_t* a, LaunchGeom* g) { ew(g, (a[7] & 3) == 0 ? a[6] * a[7] / 4 : a[6] * a[7], (const void*)bn_apply_kernel); return 0; }
+std::atomic<int> bn_apply_occ{0};
+int bn_apply_geom(const uint64_t* a, LaunchGeom* g) { ew(g, (a[7] & 3) == 0 ? a[6] * a[7] / 4 : a[6] * a[7], (const void*)bn_apply_kernel, bn_apply_occ); return 0; }
 int bn_apply_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   bn_apply_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (float*)a[1], (const float*)a[2], (const float*)a[3], (const float*)a[4],
                                              (const float*)a[5], (long long)(a[6] * a[7]), (int)a[7], sig);
@@ -353,7 +383,8 @@ int bn_bwd_reduce_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, c
 }
 
 // BN bwd dx: x, dy, dx, gamma, mean, invstd, dgamma, dbeta, rows, C
-int bn_bwd_dx_geom(const uint64_t* a, LaunchGeom* g) { ew(g, (a[9] & 3) == 0 ? a[8] * a[9] / 4 : a[8] * a[9], (const void*)bn_bwd_dx_kernel); return 0; }
+std::atomic<int> bn_bwd_dx_occ{0};
+int bn_bwd_dx_geom(const uint64_t* a, LaunchGeom* g) { ew(g, (a[9] & 3) == 0 ? a[8] * a[9] / 4 : a[8] * a[9], (const void*)bn_bwd_dx_kernel, bn_bwd_dx_occ); return 0; }
 int bn_bwd_dx_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   bn_bwd_dx_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (const float*)a[1], (float*)a[2], (const float*)a[3], (const float*)a[4],
                                               (const float*)a[5], (const float*)a[6], (const float*)a[7], (long long)a[8], (int)a[9], sig);

@@ -5,6 +5,23 @@
 #include "orion.h"
 #include "orion_kernels.h"
 
+#include <atomic>
+
+// Resident CTAs per SM of a grid-stride kernel, from the occupancy query (cached per kernel in
+// `slot`; 8 when the query fails, e.g. no device). The memory-bound grid-stride kernels cap their
+// grid at one full wave of 148 SMs x this, so no CTA waits for a tail wave (results never depend
+// on the grid size).
+inline int resident_ctas_per_sm(const void* f, int threads, std::atomic<int>& slot) {
+  int b = slot.load(std::memory_order_relaxed);
+  if (b > 0) return b;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, f, threads, 0) != cudaSuccess || b < 1 || b > 8) {
+    (void)cudaGetLastError();
+    b = 8;
+  }
+  slot.store(b, std::memory_order_relaxed);
+  return b;
+}
+
 // Completion signal fused into every kernel: the last CTA of a launch publishes `seq` (the
 // client's completed-op count) to a host-mapped counter, so the scheduler observes completion by a
 // plain load instead of a CUDA event query (P:778-786 uses cudaEventQuery).

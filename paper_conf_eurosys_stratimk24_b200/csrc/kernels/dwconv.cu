@@ -296,9 +296,10 @@ DwShape dw_shape(const uint64_t* a) {
 }
 bool dw_ok(const uint64_t* a) { return (a[6] % 4) == 0 && a[7] == a[6] && a[8] == 3 && a[9] == 3 && a[11] == 1; }
 
-void ew(LaunchGeom* g, uint64_t n, const void* f) {
+void ew(LaunchGeom* g, uint64_t n, const void* f, std::atomic<int>& occ) {
   uint64_t ctas = cdiv(n ? n : 1, DW_THREADS);
-  if (ctas > 148 * 8) ctas = 148 * 8;
+  const uint64_t wave = 148ull * resident_ctas_per_sm(f, DW_THREADS, occ);
+  if (ctas > wave) ctas = wave;
   g->grid = dim3((unsigned)ctas); g->block = dim3(DW_THREADS); g->smem = 0; g->func = f;
 }
 
@@ -342,12 +343,13 @@ int dw_fwd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStre
     dw_fwd_rows_kernel<2><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
   CHECK_LAUNCH();
 }
+std::atomic<int> dw_dgrad_occ{0};
 int dw_dgrad_geom(const uint64_t* a, LaunchGeom* g) {
   if (!dw_ok(a)) return ORION_E_INVAL;
   DwShape s = dw_shape(a);
   if (s.stride == 1) rows_geom(g, (long long)s.N * s.H * ((s.C + 31) / 32), (const void*)dw_dgrad_rows_s1_kernel);
   else if (s.stride == 2) rows_geom(g, (long long)s.N * s.H * ((s.C + 31) / 32), (const void*)dw_dgrad_rows_s2_kernel);
-  else ew(g, (uint64_t)s.N * s.H * s.W * (s.C / 4), (const void*)dw_dgrad_kernel);
+  else ew(g, (uint64_t)s.N * s.H * s.W * (s.C / 4), (const void*)dw_dgrad_kernel, dw_dgrad_occ);
   return 0;
 }
 int dw_dgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
