@@ -191,15 +191,16 @@ __global__ void __launch_bounds__(DW_THREADS) dw_dgrad_rows_s2_kernel(const floa
 // blocks as above), fp32 per row and fp64 across rows; warps combine in smem in fixed order, CTAs
 // write per-split partials, the last CTA of the channel block sums them in split order.
 template <int S>
-__global__ void __launch_bounds__(DW_THREADS) dw_wgrad_rows_kernel(const float* __restrict__ x, const float* __restrict__ dy,
+__global__ void __launch_bounds__(DW_THREADS, S == 1 ? 3 : 2) dw_wgrad_rows_kernel(const float* __restrict__ x, const float* __restrict__ dy,
                                                                    float* __restrict__ dw, DwShape s, unsigned char* ws, OrionSig sig) {
   __shared__ double sh[ROW_WARPS][9][32];
   const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
   const int c = blockIdx.x * 32 + lane;
   const long long nrows = (long long)s.N * s.P;
-  double acc[9];
+  // the fp64 row sums live in this lane's own shared-memory slots (no registers; same order)
+  double* acc = &sh[warp][0][lane];
 #pragma unroll
-  for (int t = 0; t < 9; t++) acc[t] = 0.0;
+  for (int t = 0; t < 9; t++) acc[t * 32] = 0.0;
   if (c < s.C) {
     for (long long row = (long long)blockIdx.y * ROW_WARPS + warp; row < nrows; row += (long long)gridDim.y * ROW_WARPS) {
       const int p = (int)(row % s.P), n = (int)(row / s.P);
@@ -229,11 +230,9 @@ __global__ void __launch_bounds__(DW_THREADS) dw_wgrad_rows_kernel(const float* 
             for (int t = 0; t < 3; t++) f[r * 3 + t] = fmaf(g[u], win.v[r][u * S + t], f[r * 3 + t]);
       }
 #pragma unroll
-      for (int t = 0; t < 9; t++) acc[t] += (double)f[t];
+      for (int t = 0; t < 9; t++) acc[t * 32] += (double)f[t];
     }
   }
-#pragma unroll
-  for (int t = 0; t < 9; t++) sh[warp][t][lane] = acc[t];
   __syncthreads();
   unsigned int* tickets = reinterpret_cast<unsigned int*>(ws);
   double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
