@@ -100,11 +100,13 @@ constexpr uint64_t WS_TICKET_BYTES = 65536;
 // order. The split into chunks depends on (n, V, blockDim) only, so the result is deterministic.
 // scratch: >= blockDim doubles of shared memory. dst may be global or shared; on return (after
 // a barrier) dst is complete.
-__device__ __forceinline__ double sum_chunk(const double* src, long long stride, int z0, int z1, int v) {
+// (src may be fp32 or fp64 partials; the sums are fp64 either way)
+template <class Src>
+__device__ __forceinline__ double sum_chunk(const Src* src, long long stride, int z0, int z1, int v) {
   double s = 0.0;
   int z = z0;
   for (; z + 7 < z1; z += 8) {
-    double a[8];
+    Src a[8];
 #pragma unroll
     for (int i = 0; i < 8; i++) a[i] = __ldcg(src + (long long)(z + i) * stride + v);
 #pragma unroll
@@ -113,7 +115,8 @@ __device__ __forceinline__ double sum_chunk(const double* src, long long stride,
   for (; z < z1; z++) s += __ldcg(src + (long long)z * stride + v);
   return s;
 }
-__device__ inline void sum_rows_ordered(const double* src, long long stride, int n, int V, double* dst, double* scratch) {
+template <class Src>
+__device__ inline void sum_rows_ordered(const Src* src, long long stride, int n, int V, double* dst, double* scratch) {
   const int nt = blockDim.x, t = threadIdx.x;
   if (V >= nt / 2) {
     for (int v = t; v < V; v += nt) dst[v] = sum_chunk(src, stride, 0, n, v);
@@ -148,7 +151,8 @@ __host__ __device__ __forceinline__ int combine_group(int nz) {
 __host__ __device__ __forceinline__ int combine_rows(int nz) {   // gpart rows needed (0: one level)
   return nz <= 16 ? 0 : (nz + combine_group(nz) - 1) / combine_group(nz);
 }
-__device__ inline bool combine_splits(unsigned int* tk, const double* part, double* gpart, long long stride, int nz, int z, int V,
+template <class Src>
+__device__ inline bool combine_splits(unsigned int* tk, const Src* part, double* gpart, long long stride, int nz, int z, int V,
                                       double* out, double* scratch) {
   if (nz <= 16) {
     if (!last_cta_of(tk, (unsigned)nz)) return false;
@@ -163,6 +167,12 @@ __device__ inline bool combine_splits(unsigned int* tk, const double* part, doub
   sum_rows_ordered(gpart, stride, ng, V, out, scratch);
   return true;
 }
+
+// Streaming weight-gradient GEMM (wgs.cu), taken by gemm flags = 1 when its TMA constraints hold.
+uint64_t wgs_ws_bytes(long long M, long long N, long long K);
+bool wgs_try_geom(const uint64_t* a, LaunchGeom* g);
+bool wgs_is(const void* f);
+int wgs_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
 
 // Kernel table (table.cu)
 extern const KernelEntry g_kernels[ORION_FN_COUNT];

@@ -2202,6 +2202,8 @@ extern "C" uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t 
     uint64_t b2 = ws_bytes_for(plan_atb((long long)M, (long long)N, (long long)K), (long long)M, (long long)N);
     if (b2 > b) b = b2;
   }
+  const uint64_t b3 = wgs_ws_bytes((long long)M, (long long)N, (long long)K);   // ... or the streaming one
+  if (b3 > b) b = b3;
   return b;
 }
 
@@ -2239,6 +2241,7 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     g->grid = dim3((unsigned)cdiv(M, rows::rpc((int)N))); g->block = dim3(rows::NTH); g->smem = rows::smem_bytes((int)K, (int)N); g->func = f;
     return 0;
   }
+  if (flags == 1 && wgs_try_geom(a, g)) return 0;   // TMA-fed streaming A^T B (wgs.cu)
   if (flags == 1 && atb_ok(M, N, K)) {
     Plan pl = plan_atb(M, N, K);
     if (pl.split > 1 && (a[11] == 0 || a[12] < ws_bytes_for(pl, M, N))) pl.split = 1;
@@ -2281,6 +2284,7 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
     gemv_bt_kernel<<<g.grid, g.block, 0, s>>>(A, lda, B, ldb, C, ldc, bias, (int)M, (int)N, (int)K, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
+  if (wgs_is(g.func)) return wgs_launch(a, g, sig, s);
   if (tmk::is(g.func)) return tmk::launch(g, M, N, K, C, ldc, bias, A, lda, B, ldb, flags == 0, sig, s);
   if (tcm::is<ADense, BDenseT>(g.func))
     return tcm::launch(g, M, N, K, C, ldc, bias, ADense{A, lda}, BDenseT{B, ldb}, sig, s);

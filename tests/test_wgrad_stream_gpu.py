@@ -1,0 +1,92 @@
+"""Streaming weight-gradient GEMM (csrc/kernels/wgs.cu; gemm flags = 1, no bias): dW = dy^T x of the
+1x1 convolutions of MobileNetV2 / ResNet training (cuDNN's weight-gradient kernels in the paper's
+runs) against the fp64 oracle product, at sizes that span several tiles, ragged rows,
+ragged tiles in both operand roles, and at the full BASELINE size of the dominant op
+(features.2.expand: dW[96, 16] over 96*112*112 rows).
+
+Checks per case:
+  * per-tensor relative L2 <= 1e-5 (single fp32 op);
+  * elementwise |C - ref| <= 4 u sqrt(K) (|A|^T |B|) + 1e-30: the probabilistic rounding bound of a
+    length-K fp32 dot product (u = 2^-24), which the kernel's partial sums (fp32 row groups of
+    <= K terms, fp64 split combine) satisfy; it catches a localized tile / tail error that a
+    per-tensor norm would average away;
+  * the streaming kernel really ran (288-thread CTAs from orion_kernel_geometry), and a second
+    launch reproduces the bytes (fixed reduction order)."""
+import math
+
+import pytest
+import torch
+
+from oracle import model as om
+from synth import inputs as si
+
+pytestmark = pytest.mark.gpu
+
+if torch.cuda.is_available():
+    import paper_conf_eurosys_stratimk24_b200 as orion
+    from paper_conf_eurosys_stratimk24_b200 import _lib as L
+    from paper_conf_eurosys_stratimk24_b200.runtime import kernel_geometry
+
+U = 2.0 ** -24
+
+
+def elem_bound(A, B, K):
+    """4 u sqrt(K) (|A|^T |B|): the rounding-error bound of each output's length-K fp32 dot product."""
+    return 4.0 * U * math.sqrt(K) * (A.double().abs().t() @ B.double().abs())
+
+
+def check_wgrad(M, N, K, seed=31, expect_stream=True):
+    A = si.normal((K, M), seed)        # dy [rows][M]
+    B = si.normal((K, N), seed + 1)    # x  [rows][N]
+    ref = A.double().t() @ B.double()
+    C = torch.zeros(M, N, device="cuda")
+    nws = L.lib.orion_gemm_workspace_bytes(M, N, K)
+    w = torch.zeros(int(nws) // 4 + 64, dtype=torch.float32, device="cuda")
+    Ad, Bd = A.cuda(), B.cuda()
+    args = [Ad.data_ptr(), Bd.data_ptr(), C.data_ptr(), 0, M, N, K, M, N, N, 1, w.data_ptr(), w.numel() * 4]
+    _, _, threads, _ = kernel_geometry("gemm", args)
+    assert (threads == 288) == expect_stream, f"kernel selection: {threads} threads"
+    s = torch.cuda.current_stream().cuda_stream
+    orion.kernel_launch("gemm", args, s)
+    torch.cuda.synchronize()
+    got = C.double().cpu()
+    rel = float((got - ref).norm() / ref.norm())
+    assert rel < 1e-5, rel
+    err = (got - ref).abs()
+    bound = elem_bound(A, B, K) + 1e-30
+    worst = float((err / bound).max())
+    assert worst <= 1.0, f"elementwise error {worst:.3f} x the fp32 dot-product bound"
+    first = C.clone()
+    orion.kernel_launch("gemm", args, s)
+    torch.cuda.synchronize()
+    assert torch.equal(first, C), "non-deterministic weight gradient"
+    return rel, worst
+
+
+# (M, N, K): MobileNetV2-b96 weight-gradient shapes (rows reduced where the fp64 product would be
+# slow) plus ragged rows (K % stage rows != 0), ragged tiles, both operand roles, split = 1
+WGS_CASES = [
+    (96, 16, 1204224),      # features.2.expand at full size (dominant BE op, BASELINE config 2)
+    (16, 32, 300037),       # features.1.project class, lane operand = x (transposed write)
+    (24, 96, 100003),       # features.2.project class
+    (144, 24, 75264),       # features.3/4.expand (two lane tiles, ragged)
+    (24, 144, 75271),       # features.3.project
+    (32, 144, 20000),
+    (192, 32, 18816), (32, 192, 18816),
+    (384, 64, 18816), (64, 384, 4704),
+    (576, 96, 4704), (96, 576, 4704),
+    (960, 160, 4704), (160, 960, 4704),
+    (1280, 320, 4704),      # features.18 (200 tiles, split 1)
+    (20, 12, 999),          # tiny, ragged everything
+    (100, 36, 70001),
+]
+
+
+@pytest.mark.parametrize("M,N,K", WGS_CASES, ids=lambda v: str(v))
+def test_wgrad_stream(M, N, K):
+    check_wgrad(M, N, K)
+
+
+@pytest.mark.parametrize("M,N,K", [(18, 16, 50000), (96, 16, 200)])   # M % 4 != 0 / short K: other kernels
+def test_wgrad_fallback(M, N, K):
+    check_wgrad(M, N, K, expect_stream=False)

@@ -1,5 +1,7 @@
 #!/bin/bash
 mkdir -p gpurun_out
+# probe binaries are build outputs (git-ignored): compile them here
+for b in probe mma_rate tma_tf32; do nvcc -O3 -std=c++17 -gencode arch=compute_100a,code=sm_100a -o tools/probe/$b tools/probe/$b.cu -lcuda || exit 1; done
 { nproc; lscpu | head -20; nvidia-smi; nvidia-smi topo -m; free -g; } > gpurun_out/box_info.txt 2>&1
 ./tools/probe/probe > gpurun_out/probe.txt 2>&1
 python - >> gpurun_out/probe.txt 2>&1 <<'PY'

@@ -1,10 +1,11 @@
 """Print the per-op device-time summary written by tools/ncu_times.sh."""
 import collections
 import csv
+import os
 import sys
 
 for c in (sys.argv[1:] or ["hp", "be"]):
-    rows = list(csv.DictReader(open(f"gpurun_out/times_{c}.csv")))
+    rows = list(csv.DictReader(open(f"gpurun_out/times_{os.environ.get('CONFIG', 'rn50_mnv2')}_{c}.csv")))
     tot = sum(float(r["dur_ns"]) for r in rows)
     by = collections.defaultdict(float)
     for r in rows:
