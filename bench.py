@@ -515,22 +515,17 @@ def train_train(args, rank, world, local, metric):
         r = session(hp=hp, be=be, arrivals_ns=np.zeros(nreq, dtype=np.int64), hp_latency_ns=iter_ns,
                     dur_threshold_ppm=args.dur_ppm, sm_threshold=thr, trace_kernel_id=trace)
         return r, hp_its(r), C.be_throughput(r, r["t0"], r["t_hp_end"])[0]
-    # binary search of SM_THRESHOLD on HP throughput
-    lo, hi = 0, max(r["sm_needed"] for r in rows_be) + 1
-    probes = []
-    _, h_, b_ = colloc(hi, max(8, n // 4))          # the most aggressive threshold first
-    probes.append((hi, h_ / hp_ded, b_))
-    if h_ >= HP_KEEP * hp_ded:
-        lo = hi
-    while hi - lo > 2 and len(probes) < 7:
-        mid = (lo + hi) // 2
-        _, h_, b_ = colloc(mid, max(8, n // 4))
-        probes.append((mid, h_ / hp_ded, b_))
-        if h_ >= HP_KEEP * hp_ded:
-            lo = mid
-        else:
-            hi = mid
-    tuned = max(lo, 1)
+    # binary search of SM_THRESHOLD on HP throughput (tuning.py, tested on the FAKE backend)
+    from paper_conf_eurosys_stratimk24_b200 import tuning as TU
+    be_at = {}
+
+    def measure(thr):
+        _, h_, b_ = colloc(thr, max(8, n // 4))
+        be_at[thr] = b_
+        return h_ / hp_ded
+    lo, probes_ = TU.search_sm_threshold(measure, max(r["sm_needed"] for r in rows_be), keep=HP_KEEP, max_probes=7)
+    probes = [(t, f, be_at[t]) for t, f in probes_]
+    tuned = max(lo, 1)   # threshold 0 would mean "the default (#SMs)" in orion_config; 1 admits nothing beside a busy HP
     top = max(rows_be, key=lambda r: r["dur_ns"])
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)

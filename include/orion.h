@@ -107,7 +107,10 @@ typedef struct {
   uint32_t trace_kernel_id_plus1; /* CUDA backend: 0 = off; else record a CUDA event pair around every
                                      launch of kernel_id (trace_kernel_id_plus1 - 1) on its own stream
                                      (bench roofline: live launch durations, read by orion_trace_read) */
-  uint32_t reserved[6];
+  uint32_t fake_contention;   /* FAKE backend: 1 = model SM contention between concurrently running
+                                 kernels (each runs at 148 / total sm_needed of real time while the
+                                 running kernels ask for more than 148 SMs); 0 = independent streams */
+  uint32_t reserved[5];
 } orion_config;
 
 /* Create an instance on `cuda_device` (ignored by the FAKE backend). Returns ORION_E_NODEV if the
@@ -157,6 +160,16 @@ int orion_trace_read(orion_t h, float* ms_out, uint32_t cap, uint32_t* n);
 int orion_run_requests(orion_t h, int client_id, const orion_op* ops, uint32_t n_ops,
                        const int64_t* arrivals_ns, uint32_t n_req, uint32_t in_cycle, uint32_t out_cycle,
                        int64_t* t_arrival_ns, int64_t* t_done_ns);
+
+/* The "native" arm of R20 (P:1355-1360 reports Orion's overhead against direct execution): the
+ * same open-loop request stream as orion_run_requests, but the calling thread launches every op
+ * itself, in order, on the client's stream -- no ring, no scheduler, no policy. Only valid on an
+ * instance that was never started (ORION_E_STATE otherwise) with a single registered client
+ * in use; completion is observed through the same per-stream counters, so the latencies are
+ * directly comparable with orion_run_requests. Arguments and outputs as orion_run_requests. */
+int orion_run_requests_direct(orion_t h, int client_id, const orion_op* ops, uint32_t n_ops,
+                              const int64_t* arrivals_ns, uint32_t n_req, uint32_t in_cycle, uint32_t out_cycle,
+                              int64_t* t_arrival_ns, int64_t* t_done_ns);
 
 /* Closed-loop training client: iteration i submits variant (i % n_variants) of
  * the op list (ops is n_variants x n_ops, row-major) and waits for it to complete before the

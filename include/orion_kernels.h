@@ -147,6 +147,26 @@ int orion_kernel_launch(uint32_t fn, const uint64_t* args, uint32_t nargs, void*
    CTAs per SM (cudaOccupancyMaxActiveBlocksPerMultiprocessor), for sm_needed (R17). */
 int orion_kernel_geometry(uint32_t fn, const uint64_t* args, uint32_t nargs, uint64_t* grid_ctas,
                           int32_t* blocks_per_sm, int32_t* threads_per_cta, int32_t* smem_bytes);
+/* Which pipe an operator's arithmetic runs on, as launched (the roofline ridge of the profiler's
+   classifier depends on it, reading R16 / P:838-847): */
+enum orion_pipe {
+  ORION_PIPE_FMA = 0,     /* FP32 FFMA / ALU / load-store (SIMT kernels) */
+  ORION_PIPE_TF32X3 = 1,  /* tcgen05 kind::tf32, 3 MMAs per fp32 product (3xTF32) */
+  ORION_PIPE_BF16 = 2     /* bf16 tensor pipe (tcgen05 kind::f16 or mma.sync bf16) */
+};
+/* Everything the offline profiler needs about one launch ("the number of blocks, the
+   number of threads per block, the number of registers per thread, and the amount of shared memory
+   that the kernel requires"), for the op as it would launch. Returns 0 or ORION_E_INVAL / E_CUDA. */
+typedef struct {
+  uint64_t grid_ctas;        /* total CTAs of the launch */
+  int32_t threads_per_cta;
+  int32_t regs_per_thread;   /* cudaFuncAttributes.numRegs */
+  int32_t static_smem;       /* cudaFuncAttributes.sharedSizeBytes */
+  int32_t dynamic_smem;      /* dynamic shared memory per CTA of this launch */
+  int32_t blocks_per_sm;     /* cudaOccupancyMaxActiveBlocksPerMultiprocessor */
+  int32_t pipe;              /* enum orion_pipe */
+} orion_kernel_info_t;
+int orion_kernel_info(uint32_t fn, const uint64_t* args, uint32_t nargs, orion_kernel_info_t* out);
 /* Workspace sizes (bytes) of the ops that split their reductions. Workspaces must be zeroed once
    at allocation; a client's ops may share one (they run in stream order; tickets self-reset). */
 uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t K);

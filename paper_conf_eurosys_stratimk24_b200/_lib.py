@@ -45,8 +45,16 @@ class Config(ctypes.Structure):
                 ("hp_latency_ns", ctypes.c_uint64), ("flags", ctypes.c_uint32), ("queue_capacity", ctypes.c_uint32),
                 ("backend", ctypes.c_uint32), ("sched_cpu", ctypes.c_int32), ("log_capacity", ctypes.c_uint64),
                 ("fake_time_scale_pct", ctypes.c_uint32), ("trace_kernel_id_plus1", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32 * 6)]
+                ("fake_contention", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 5)]
 
+
+class KernelInfo(ctypes.Structure):   # orion_kernel_info_t
+    _fields_ = [("grid_ctas", ctypes.c_uint64), ("threads_per_cta", ctypes.c_int32), ("regs_per_thread", ctypes.c_int32),
+                ("static_smem", ctypes.c_int32), ("dynamic_smem", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
+                ("pipe", ctypes.c_int32)]
+
+
+PIPE_FMA, PIPE_TF32X3, PIPE_BF16 = 0, 1, 2
 
 assert ctypes.sizeof(Op) == 224 and ctypes.sizeof(Profile) == 24
 
@@ -67,6 +75,8 @@ _sig = {
     "orion_strerror": (ctypes.c_char_p, [ctypes.c_int]),
     "orion_run_requests": (ctypes.c_int, [_h, ctypes.c_int, ctypes.POINTER(Op), ctypes.c_uint32, ctypes.c_void_p,
                                           ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p]),
+    "orion_run_requests_direct": (ctypes.c_int, [_h, ctypes.c_int, ctypes.POINTER(Op), ctypes.c_uint32, ctypes.c_void_p,
+                                                 ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_void_p, ctypes.c_void_p]),
     "orion_run_iterations": (ctypes.c_int, [_h, ctypes.c_int, ctypes.POINTER(Op), ctypes.c_uint32, ctypes.c_uint32,
                                             ctypes.c_void_p, ctypes.c_uint64, ctypes.c_void_p, ctypes.c_uint64,
                                             ctypes.POINTER(ctypes.c_uint64)]),
@@ -78,6 +88,8 @@ _sig = {
     "orion_kernel_geometry": (ctypes.c_int, [ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint64), ctypes.c_uint32,
                                              ctypes.POINTER(ctypes.c_uint64), ctypes.POINTER(ctypes.c_int32),
                                              ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_int32)]),
+    "orion_kernel_info": (ctypes.c_int, [ctypes.c_uint32, ctypes.POINTER(ctypes.c_uint64), ctypes.c_uint32,
+                                         ctypes.POINTER(KernelInfo)]),
     "orion_gemm_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64]),
     "orion_conv_wgrad_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64] * 9),
     "orion_bn_workspace_bytes": (ctypes.c_uint64, [ctypes.c_uint64, ctypes.c_uint64]),

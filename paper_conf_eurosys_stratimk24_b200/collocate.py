@@ -86,15 +86,30 @@ def run_session(hp=None, be=None, arrivals_ns=None, be_iters=0, log_capacity=0, 
             th.start()
     else:
         res["t0"] = o_now = L.lib.orion_now_ns()
+    try:
+        if hp is not None:
+            ta, td = o.run_requests(hp_id, hp.ops, arrivals_ns, in_cycle=hp.inp.shape[0], out_cycle=hp.n_req)
+            res["t_arrival"], res["t_done"] = ta, td
+            res["t_hp_end"] = L.lib.orion_now_ns()
+    except BaseException:
+        # an HP driver error must not leave the BE threads spinning in native code: stop them,
+        # join them and tear the instance down before the error propagates
+        stop.value = 1
+        for th in ths:
+            th.join()
+        try:
+            o.stop()
+        except Exception:
+            pass
+        o.destroy()
+        raise
     if hp is not None:
-        ta, td = o.run_requests(hp_id, hp.ops, arrivals_ns, in_cycle=hp.inp.shape[0], out_cycle=hp.n_req)
-        res["t_arrival"], res["t_done"] = ta, td
-        res["t_hp_end"] = L.lib.orion_now_ns()
         stop.value = 1
     for th in ths:
         th.join()
     if "be_err" in res:
         o.stop()
+        o.destroy()
         raise res["be_err"]
     if bes:
         res["be_t_end"] = res["be_t_end_all"][0]
@@ -108,6 +123,20 @@ def run_session(hp=None, be=None, arrivals_ns=None, be_iters=0, log_capacity=0, 
     o.destroy()
     del o_now
     return res
+
+
+def run_direct(hp, arrivals_ns, device=0):
+    """The native arm (R20; P:1355-1360 measures Orion's overhead against it): the HP request stream
+    launched directly on one stream by the client thread, no scheduler. Same completion counters and
+    clock as run_session, so latencies compare one to one."""
+    o = Orion(device=device, backend=L.BACKEND_CUDA)
+    try:
+        cid = o.register_client(L.HP)
+        torch.cuda.synchronize()
+        ta, td = o.run_requests_direct(cid, hp.ops, arrivals_ns, in_cycle=hp.inp.shape[0], out_cycle=hp.n_req)
+    finally:
+        o.destroy()
+    return {"t_arrival": ta, "t_done": td}
 
 
 def latency_stats(res):

@@ -1,5 +1,9 @@
 // FAKE backend: each "stream" is a CPU thread that completes the ops launched on it in FIFO order
 // after their profiled duration (scaled), then publishes done = seq + 1. No GPU, no CUDA calls.
+// Optional SM-contention model (orion_config.fake_contention, CPU tests of the SM_THRESHOLD
+// search): a running kernel occupies min(sm_needed, 148) "SMs"; while the kernels running on all
+// streams together ask for more than 148, each progresses at 148 / demand of real time (SMs time-
+// shared), so a BE kernel admitted beside the HP slows the HP exactly when the two do not fit.
 #include <time.h>
 
 #include <atomic>
@@ -15,7 +19,8 @@ namespace orion {
 struct StreamHandle {
   std::mutex mu;
   std::condition_variable cv;
-  std::deque<std::pair<uint64_t, uint64_t>> q;  // (seq, duration ns)
+  struct Job { uint64_t seq, dur_ns; uint32_t sm; };
+  std::deque<Job> q;
   alignas(64) std::atomic<uint64_t> done{0};
   bool quit = false;
   std::thread th;
@@ -28,14 +33,36 @@ static int64_t mono_ns() {
 }
 
 struct FakeBackend : Backend {
+  static constexpr int64_t kSms = 148;
   uint32_t scale_pct;
-  explicit FakeBackend(const orion_config& c) : scale_pct(c.fake_time_scale_pct ? c.fake_time_scale_pct : 100) {}
-  uint32_t num_sms() override { return 148; }
+  bool contention;
+  std::atomic<int64_t> demand{0};   // SMs asked for by the kernels running now (contention model)
+  explicit FakeBackend(const orion_config& c)
+      : scale_pct(c.fake_time_scale_pct ? c.fake_time_scale_pct : 100), contention(c.fake_contention != 0) {}
+  uint32_t num_sms() override { return (uint32_t)kSms; }
+  void run(const StreamHandle::Job& job) {
+    if (!contention || job.sm == 0) {
+      const int64_t until = mono_ns() + (int64_t)job.dur_ns;
+      while (mono_ns() < until) std::this_thread::yield();
+      return;
+    }
+    const int64_t sm = job.sm < kSms ? (int64_t)job.sm : kSms;
+    demand.fetch_add(sm);
+    double progress = 0.0;
+    int64_t t = mono_ns();
+    while (progress < (double)job.dur_ns) {
+      std::this_thread::yield();
+      const int64_t t2 = mono_ns(), d = demand.load();
+      progress += (double)(t2 - t) * (d > kSms ? (double)kSms / (double)d : 1.0);
+      t = t2;
+    }
+    demand.fetch_sub(sm);
+  }
   int create_stream(int, StreamHandle** out) override {
     StreamHandle* s = new StreamHandle();
-    s->th = std::thread([s]() {
+    s->th = std::thread([this, s]() {
       for (;;) {
-        std::pair<uint64_t, uint64_t> job;
+        StreamHandle::Job job;
         {
           std::unique_lock<std::mutex> lk(s->mu);
           s->cv.wait(lk, [s] { return s->quit || !s->q.empty(); });
@@ -43,9 +70,8 @@ struct FakeBackend : Backend {
           job = s->q.front();
           s->q.pop_front();
         }
-        const int64_t until = mono_ns() + (int64_t)job.second;
-        while (mono_ns() < until) std::this_thread::yield();
-        s->done.store(job.first + 1, std::memory_order_release);
+        run(job);
+        s->done.store(job.seq + 1, std::memory_order_release);
       }
     });
     *out = s;
@@ -62,10 +88,11 @@ struct FakeBackend : Backend {
   }
   void* native_stream(StreamHandle*) override { return nullptr; }
   int launch(StreamHandle* s, const orion_op& op, uint64_t seq) override {
-    uint64_t d = op.kind == ORION_OP_KERNEL ? op.prof.dur_ns * scale_pct / 100 : 0;
+    const bool kern = op.kind == ORION_OP_KERNEL;
+    const uint64_t d = kern ? op.prof.dur_ns * scale_pct / 100 : 0;
     {
       std::lock_guard<std::mutex> lk(s->mu);
-      s->q.emplace_back(seq, d);
+      s->q.push_back(StreamHandle::Job{seq, d, kern ? op.prof.sm_needed : 0u});
     }
     s->cv.notify_one();
     return 0;

@@ -52,6 +52,7 @@ struct LaunchGeom {
   dim3 grid{1, 1, 1}, block{1, 1, 1};
   int smem = 0;
   const void* func = nullptr;
+  int pipe = 0;   // ORION_PIPE_*: the pipe the chosen kernel's arithmetic runs on (profiler ridge, R16)
   unsigned long long ctas() const { return (unsigned long long)grid.x * grid.y * grid.z; }
 };
 

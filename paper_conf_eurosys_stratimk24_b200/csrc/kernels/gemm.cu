@@ -1058,6 +1058,7 @@ void geom(LaunchGeom* g, long long M, long long N) {
   g->grid = dim3((unsigned)cdiv(tiles, tpc_of(tiles))); g->block = dim3(NTHR);
   if (bn_for(N) == 128) { prepare<128, LA, LB>(); g->smem = Cfg<128>::SMEM; g->func = (const void*)gemm_tcm_kernel<128, LA, LB>; }
   else { prepare<64, LA, LB>(); g->smem = Cfg<64>::SMEM; g->func = (const void*)gemm_tcm_kernel<64, LA, LB>; }
+  g->pipe = ORION_PIPE_TF32X3;
 }
 template <class LA, class LB>
 bool is(const void* f) { return f == (const void*)gemm_tcm_kernel<128, LA, LB> || f == (const void*)gemm_tcm_kernel<64, LA, LB>; }
@@ -1361,6 +1362,7 @@ void geom_t(LaunchGeom* g, long long tiles) {
   prepare<BN, BMN>();
   g->grid = dim3((unsigned)cdiv(tiles, tcm::tpc_of(tiles))); g->block = dim3(NTHR); g->smem = Cfg<BN, BMN>::SMEM;
   g->func = (const void*)gemm_tmk_kernel<BN, BMN>;
+  g->pipe = ORION_PIPE_TF32X3;
 }
 inline void geom(LaunchGeom* g, long long M, long long N, bool bmn) {
   const long long tiles = tcm::tiles_of(M, N);
@@ -1822,8 +1824,8 @@ void tiled_geom(LaunchGeom* g, long long M, long long N, long long K, uint64_t w
   if (pl.split > 1 && (ws_ptr == 0 || ws_bytes < ws_bytes_for(pl, M, N))) pl.split = 1;
   g->grid = dim3((unsigned)cdiv(N, pl.bn), (unsigned)cdiv(M, pl.bm), (unsigned)pl.split);
   g->func = kernel_for<LA, LB>(pl.cfg);
-  if (pl.cfg == 3) { tc_prepare<128, LA, LB>(); g->block = dim3(tc::NTHR); g->smem = tc::TcCfg<128>::SMEM; }
-  else if (pl.cfg == 4) { tc_prepare<64, LA, LB>(); g->block = dim3(tc::NTHR); g->smem = tc::TcCfg<64>::SMEM; }
+  if (pl.cfg == 3) { tc_prepare<128, LA, LB>(); g->block = dim3(tc::NTHR); g->smem = tc::TcCfg<128>::SMEM; g->pipe = ORION_PIPE_TF32X3; }
+  else if (pl.cfg == 4) { tc_prepare<64, LA, LB>(); g->block = dim3(tc::NTHR); g->smem = tc::TcCfg<64>::SMEM; g->pipe = ORION_PIPE_TF32X3; }
   else { g->block = dim3(NT); g->smem = 0; }
 }
 

@@ -86,4 +86,28 @@ int orion_kernel_geometry(uint32_t fn, const uint64_t* args, uint32_t nargs, uin
   return 0;
 }
 
+int orion_kernel_info(uint32_t fn, const uint64_t* args, uint32_t nargs, orion_kernel_info_t* out) {
+  if (fn >= ORION_FN_COUNT || args == nullptr || out == nullptr) return ORION_E_INVAL;
+  const KernelEntry& e = g_kernels[fn];
+  if ((int)nargs < e.nargs) return ORION_E_INVAL;
+  LaunchGeom g;
+  int r = e.geom(args, &g);
+  if (r) return r;
+  cudaFuncAttributes fa;
+  if (cudaFuncGetAttributes(&fa, g.func) != cudaSuccess) { (void)cudaGetLastError(); return ORION_E_CUDA; }
+  out->grid_ctas = g.ctas();
+  out->threads_per_cta = (int32_t)(g.block.x * g.block.y * g.block.z);
+  out->regs_per_thread = fa.numRegs;
+  out->static_smem = (int32_t)fa.sharedSizeBytes;
+  out->dynamic_smem = g.smem;
+  out->pipe = g.pipe;
+  int b = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, g.func, out->threads_per_cta, g.smem) != cudaSuccess) {
+    (void)cudaGetLastError();
+    return ORION_E_CUDA;
+  }
+  out->blocks_per_sm = b;
+  return 0;
+}
+
 }  // extern "C"

@@ -578,13 +578,13 @@ int gemm_bf16_geom(const uint64_t* a, LaunchGeom* g) {
   g->block = dim3(tcb::NTHR);
   if (bn == 256) {
     if (!tcb::prepare<256>()) return ORION_E_CUDA;
-    g->smem = tcb::Cfg<256>::SMEM; g->func = (const void*)tcb::gemm_bf16_kernel<256>;
+    g->smem = tcb::Cfg<256>::SMEM; g->func = (const void*)tcb::gemm_bf16_kernel<256>; g->pipe = ORION_PIPE_BF16;
   } else if (bn == 128) {
     if (!tcb::prepare<128>()) return ORION_E_CUDA;
-    g->smem = tcb::Cfg<128>::SMEM; g->func = (const void*)tcb::gemm_bf16_kernel<128>;
+    g->smem = tcb::Cfg<128>::SMEM; g->func = (const void*)tcb::gemm_bf16_kernel<128>; g->pipe = ORION_PIPE_BF16;
   } else {
     if (!tcb::prepare<64>()) return ORION_E_CUDA;
-    g->smem = tcb::Cfg<64>::SMEM; g->func = (const void*)tcb::gemm_bf16_kernel<64>;
+    g->smem = tcb::Cfg<64>::SMEM; g->func = (const void*)tcb::gemm_bf16_kernel<64>; g->pipe = ORION_PIPE_BF16;
   }
   return 0;
 }
@@ -622,6 +622,7 @@ int attention_geom(const uint64_t* a, LaunchGeom* g) {
   g->block = dim3(attn::NTH);
   g->smem = 0;
   g->func = f;
+  g->pipe = ORION_PIPE_BF16;   // QK^T and PV on mma.sync bf16 (tensor pipe)
   return 0;
 }
 int attention_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {

@@ -549,6 +549,50 @@ int orion_run_requests(orion_t h, int client_id, const orion_op* ops, uint32_t n
   return ORION_OK;
 }
 
+int orion_run_requests_direct(orion_t h, int client_id, const orion_op* ops, uint32_t n_ops, const int64_t* arrivals_ns, uint32_t n_req,
+                              uint32_t in_cycle, uint32_t out_cycle, int64_t* t_arrival_ns, int64_t* t_done_ns) {
+  if (!h || !ops || !n_ops || !arrivals_ns || client_id < 0 || client_id >= (int)h->clients.size()) return ORION_E_INVAL;
+  if (h->state.load() != CREATED) return ORION_E_STATE;
+  if (h->failed.load()) return ORION_E_CUDA;
+  if (in_cycle == 0) in_cycle = 1;
+  if (out_cycle == 0) out_cycle = 1;
+  Client* c = h->clients[client_id].get();
+  h->backend->thread_init();
+  orion_op op;
+  uint32_t next_done = 0;
+  std::vector<uint64_t> end_seq(n_req, 0);
+  auto poll = [&]() {
+    const uint64_t d = h->backend->read_done(c->stream);
+    int64_t t = -1;
+    while (next_done < n_req && end_seq[next_done] != 0 && d >= end_seq[next_done]) {
+      if (t < 0) t = now_ns();
+      if (t_done_ns) t_done_ns[next_done] = t;
+      next_done++;
+    }
+  };
+  const int64_t start = now_ns();
+  for (uint32_t r = 0; r < n_req; r++) {
+    const int64_t due = start + arrivals_ns[r];
+    while (now_ns() < due) { poll(); cpu_relax(); }
+    for (uint32_t i = 0; i < n_ops; i++) {
+      op = ops[i];
+      if (op.kind == ORION_OP_MEMCPY_H2D) op.args[1] = ops[i].args[1] + (uint64_t)(r % in_cycle) * ops[i].args[2];
+      if (op.kind == ORION_OP_MEMCPY_D2H) op.args[0] = ops[i].args[0] + (uint64_t)(r % out_cycle) * ops[i].args[2];
+      const uint64_t seq = c->submitted++;
+      if (h->backend->launch(c->stream, op, seq) != 0) { h->failed.store(1); return ORION_E_CUDA; }
+    }
+    if (t_arrival_ns) t_arrival_ns[r] = due;
+    end_seq[r] = c->submitted;
+    poll();
+  }
+  while (next_done < n_req) {
+    poll();
+    if (h->failed.load(std::memory_order_relaxed)) return ORION_E_CUDA;
+    cpu_relax();
+  }
+  return ORION_OK;
+}
+
 int orion_run_iterations(orion_t h, int client_id, const orion_op* ops, uint32_t n_ops, uint32_t n_variants, const volatile int32_t* stop,
                          uint64_t max_iters, int64_t* t_end_ns, uint64_t cap_iters, uint64_t* iters_out) {
   if (!h || !ops || !n_ops || client_id < 0 || client_id >= (int)h->clients.size()) return ORION_E_INVAL;

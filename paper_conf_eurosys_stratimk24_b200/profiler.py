@@ -18,15 +18,26 @@ import os
 import torch
 
 from . import _lib as L
-from .runtime import kernel_launch, kernel_geometry
+from .runtime import kernel_launch, kernel_geometry, kernel_info
 
 # B200 peaks (MEASURED_PEAKS.json; FFMA peak derived: 148 SMs x 128 FMA x 2 x 1.965 GHz)
 HBM_GBS = 6554.2
 FFMA_TFLOPS = 148 * 128 * 2 * 1.965e9 / 1e12
-RIDGE_FFMA = FFMA_TFLOPS * 1e12 / (HBM_GBS * 1e9)   # flop per DRAM byte
+RIDGE_FFMA = FFMA_TFLOPS * 1e12 / (HBM_GBS * 1e9)   # flop per DRAM byte (11.4)
 BF16_TFLOPS = 1669.2                                  # dense bf16 tensor pipe (MEASURED_PEAKS.json)
 RIDGE_BF16 = BF16_TFLOPS * 1e12 / (HBM_GBS * 1e9)
-TENSOR_OPS = ("gemm_bf16", "attention")               # ops on the bf16 tensor pipe: their own ridge
+# fp32 GEMM / conv on tcgen05 kind::tf32 with three MMAs per product (3xTF32): tf32 dense = bf16 x
+# the guide's nominal 1/2, so the algorithmic fp32 ceiling is bf16 / 6 -> ridge 42.4
+TF32X3_TFLOPS = BF16_TFLOPS / 6.0
+RIDGE_TF32X3 = TF32X3_TFLOPS * 1e12 / (HBM_GBS * 1e9)
+RIDGE_OF_PIPE = {L.PIPE_FMA: RIDGE_FFMA, L.PIPE_TF32X3: RIDGE_TF32X3, L.PIPE_BF16: RIDGE_BF16}
+
+# sm_100 per-SM limits for the closed-form occupancy (R17): threads, warps, CTAs,
+# registers (allocated per warp in units of 256), shared memory (228 KB per SM, 1 KB reserved per
+# CTA, 128-byte allocation granularity)
+SM_MAX_THREADS, SM_MAX_WARPS, SM_MAX_CTAS = 2048, 64, 32
+SM_REGS, REG_ALLOC_UNIT = 65536, 256
+SM_SMEM, CTA_SMEM_RESERVED, SMEM_ALLOC_UNIT = 233472, 1024, 128
 
 
 def op_work(fn, a):
@@ -115,9 +126,38 @@ def classify(c_pct=None, m_pct=None, flops=0, dram_bytes=0, ridge=RIDGE_FFMA):
     return L.CLS_U
 
 
+def occupancy_limits(threads, regs, smem):
+    """blocks_per_sm of a kernel from its launch resources, limit by limit ("limited by
+    the number of threads, the number of registers, or the amount of shared memory"); the same
+    quantities ncu reports as launch__occupancy_limit_{warps,registers,shared_mem,blocks}."""
+    warps = -(-threads // 32)
+    lim_warps = SM_MAX_WARPS // warps
+    per_warp = -(-(regs * 32) // REG_ALLOC_UNIT) * REG_ALLOC_UNIT
+    lim_regs = (SM_REGS // per_warp) // warps if regs > 0 else SM_MAX_CTAS
+    per_cta = -(-smem // SMEM_ALLOC_UNIT) * SMEM_ALLOC_UNIT + CTA_SMEM_RESERVED
+    lim_smem = SM_SMEM // per_cta
+    return {"warps": lim_warps, "registers": lim_regs, "shared_mem": lim_smem, "blocks": SM_MAX_CTAS}
+
+
+def blocks_per_sm_closed_form(threads, regs, smem):
+    return min(occupancy_limits(threads, regs, smem).values())
+
+
+def sm_needed_closed_form(num_blocks, threads, regs, smem):
+    """sm_needed = ceil(num_blocks / blocks_per_sm) (P:869-870)."""
+    return int(math.ceil(num_blocks / max(blocks_per_sm_closed_form(threads, regs, smem), 1)))
+
+
 def sm_needed(fn, args, num_sms=148):
+    """R17 on the op as launched: the occupancy API's blocks_per_sm (== the closed form above,
+    cross-checked on the GPU by tests/test_profiler_gpu.py)."""
     grid, bps, _, _ = kernel_geometry(fn, args)
     return int(math.ceil(grid / max(bps, 1)))
+
+
+def ridge_of(fn, args):
+    """Roofline ridge (flop per DRAM byte) of the pipe the op's kernel runs on as launched."""
+    return RIDGE_OF_PIPE[kernel_info(fn, args)["pipe"]]
 
 
 def time_ops(graph, reps=10, warmup=2, stream=None):
@@ -172,11 +212,11 @@ def build_profiles(graph, kid_base=0, reps=10, ncu_csv=None):
             # arithmetic intensity over max(measured DRAM bytes, compulsory bytes): on B200 the 126 MB
             # L2 often holds an op's inputs, and DRAM bytes alone would call a memory-bound op
             # compute-bound (DESIGN.md §3 R16)
-            cls = classify(c, m, flops, max(dram, nbytes), RIDGE_BF16 if fn in TENSOR_OPS else RIDGE_FFMA)
+            cls = classify(c, m, flops, max(dram, nbytes), ridge_of(fn, args))
             dur = int(ndur) if ndur > 0 else dur   # device time of the kernel alone
             src = "ncu"
         else:
-            cls = classify(None, None, flops, nbytes, RIDGE_BF16 if fn in TENSOR_OPS else RIDGE_FFMA)
+            cls = classify(None, None, flops, nbytes, ridge_of(fn, args))
             src = "analytic"
         sm = sm_needed(fn, args)
         table[kid] = (cls, sm, dur)

@@ -41,12 +41,13 @@ class Orion:
 
     def __init__(self, device=0, backend=L.BACKEND_CUDA, num_sms=0, sm_threshold=0, dur_threshold_ppm=25000,
                  hp_latency_ns=0, be_partition_sms=0, flags=0, queue_capacity=4096, sched_cpu=-1, log_capacity=0,
-                 fake_time_scale_pct=100, trace_kernel_id=None):
+                 fake_time_scale_pct=100, trace_kernel_id=None, fake_contention=False):
         cfg = Config()
         cfg.num_sms, cfg.sm_threshold, cfg.dur_threshold_ppm = num_sms, sm_threshold, dur_threshold_ppm
         cfg.be_partition_sms, cfg.hp_latency_ns, cfg.flags = be_partition_sms, hp_latency_ns, flags
         cfg.queue_capacity, cfg.backend, cfg.sched_cpu = queue_capacity, backend, sched_cpu
         cfg.log_capacity, cfg.fake_time_scale_pct = log_capacity, fake_time_scale_pct
+        cfg.fake_contention = 1 if fake_contention else 0
         cfg.trace_kernel_id_plus1 = 0 if trace_kernel_id is None else trace_kernel_id + 1
         self.h = ctypes.c_void_p()
         check(L.lib.orion_create(device, ctypes.byref(cfg), ctypes.byref(self.h)), "orion_create")
@@ -128,6 +129,17 @@ class Orion:
                                        ta.ctypes.data, td.ctypes.data), "orion_run_requests")
         return ta, td
 
+    def run_requests_direct(self, cid, ops, arrivals_ns, in_cycle=1, out_cycle=1):
+        """The native arm (orion_run_requests_direct: direct launches, no scheduler; instance never started)."""
+        arr = op_array(ops)
+        arrivals = np.ascontiguousarray(arrivals_ns, dtype=np.int64)
+        n = len(arrivals)
+        ta = np.zeros(n, dtype=np.int64)
+        td = np.zeros(n, dtype=np.int64)
+        check(L.lib.orion_run_requests_direct(self.h, cid, arr, len(ops), arrivals.ctypes.data, n, in_cycle, out_cycle,
+                                              ta.ctypes.data, td.ctypes.data), "orion_run_requests_direct")
+        return ta, td
+
     def run_iterations(self, cid, variants, stop_flag=None, max_iters=0, cap=1 << 16):
         """Native closed-loop training driver (orion_run_iterations). variants: list of op lists."""
         n_ops = len(variants[0])
@@ -169,3 +181,13 @@ def kernel_geometry(fn, args):
     check(L.lib.orion_kernel_geometry(L.FN[fn] if isinstance(fn, str) else fn, a, len(args), ctypes.byref(grid),
                                       ctypes.byref(bps), ctypes.byref(thr), ctypes.byref(smem)), f"kernel_geometry({fn})")
     return grid.value, bps.value, thr.value, smem.value
+
+
+def kernel_info(fn, args):
+    """orion_kernel_info: launch geometry, registers, shared memory, occupancy and pipe of one op as it
+    would launch (the offline profiler's inputs)."""
+    a = (ctypes.c_uint64 * len(args))(*[int(x) & 0xFFFFFFFFFFFFFFFF for x in args])
+    info = L.KernelInfo()
+    check(L.lib.orion_kernel_info(L.FN[fn] if isinstance(fn, str) else fn, a, len(args), ctypes.byref(info)),
+          f"kernel_info({fn})")
+    return {k: getattr(info, k) for k, _ in info._fields_}

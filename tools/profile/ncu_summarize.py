@@ -25,19 +25,29 @@ def parse(path):
     return out
 
 
+# the profiler's further inputs (P:838-847 throughputs, P:859-870 occupancy limits): CSV column <- ncu metric
+EXTRA = [("tc_pct", "sm__pipe_tc_cycles_active.avg.pct_of_peak_sustained_elapsed"),
+         ("tensor_pct", "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed"),
+         ("fma_pct", "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_elapsed"),
+         ("block", "launch__block_size"), ("regs", "launch__registers_per_thread"),
+         ("occ_blocks", "launch__occupancy_limit_blocks"), ("occ_regs", "launch__occupancy_limit_registers"),
+         ("occ_smem", "launch__occupancy_limit_shared_mem"), ("occ_warps", "launch__occupancy_limit_warps")]
+
+
 def main(ncu_log, oplist, base, out_csv):
     launches = parse(ncu_log)
     ops = [l.rstrip("\n").split("\t") for l in open(oplist)]
     assert len(launches) == len(ops), (len(launches), len(ops))
     with open(out_csv, "w", newline="") as f:
         w = csv.writer(f)
-        w.writerow(["kernel_id", "label", "fn", "dur_ns", "sm_pct", "mem_pct", "dram_bytes", "dram_gbs", "grid"])
+        w.writerow(["kernel_id", "label", "fn", "dur_ns", "sm_pct", "mem_pct", "dram_bytes", "dram_gbs", "grid"] +
+                   [c for c, _ in EXTRA])
         for (idx, fn, lab), m in zip(ops, launches):
             dur = m.get("gpu__time_duration.sum", 0.0)
             dram = m.get("dram__bytes_read.sum", 0.0) + m.get("dram__bytes_write.sum", 0.0)
             w.writerow([int(idx) + base, lab, fn, dur, m.get("sm__throughput.avg.pct_of_peak_sustained_elapsed", 0.0),
                         m.get("gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed", 0.0), dram,
-                        dram / dur if dur else 0.0, m.get("launch__grid_size", 0)])
+                        dram / dur if dur else 0.0, m.get("launch__grid_size", 0)] + [m.get(k, "") for _, k in EXTRA])
 
 
 if __name__ == "__main__":
