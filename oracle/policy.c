@@ -24,7 +24,7 @@
 
 #define MAXC 16
 #ifndef ORACLE_MUTANT
-#define ORACLE_MUTANT 0   /* tests compile deliberate mistakes (1..8) to prove the pins catch them */
+#define ORACLE_MUTANT 0   /* tests compile deliberate mistakes (1..10) to prove the pins catch them */
 #endif
 #define KIND_KERNEL 0
 #define CLS_U 0
@@ -188,7 +188,7 @@ static int hp_busy_now(const o_cfg *c, const o_state *s) {
     if (o->opflags & OPF_REQ_BEGIN) begin = i;
     if ((o->opflags & OPF_REQ_END) && begin != UINT64_MAX) {
       /* request spans [begin, i] */
-      if (begin < s->popped[h] && i >= s->done[h]) return 1;
+      if ((ORACLE_MUTANT == 10 ? i < s->popped[h] : begin < s->popped[h]) && i >= s->done[h]) return 1;
       begin = UINT64_MAX;
     }
   }
@@ -208,7 +208,7 @@ static int schedule_be(const o_cfg *c, const o_state *s, int hp_busy, const o_op
     return R_NONE;
   }
   int h = c->hp, any_sm = 0, any_prof = 0;
-  for (uint64_t i = s->done[h]; i < s->popped[h]; i++) {
+  for (uint64_t i = (ORACLE_MUTANT == 9 ? s->popped[h] - 1 : s->done[h]); i < s->popped[h]; i++) {
     const o_op *ho = &c->ops[h][i];
     const o_op *hr = ho->kind == KIND_KERNEL ? ho : &U_PROF;
     if (!((int64_t)op->sm_needed < thr(c, hr))) any_sm = 1;
@@ -391,6 +391,23 @@ static void check_iter(o_brute *b, const o_state *pre, const o_state *post, cons
       if (r->kind == D_ADMIT_COLOC && !(c->flags & F_HP_REF_ALL)) {
         const o_op *h = &post->hp_ref;
         if (!((int64_t)op->sm_needed < thr(c, h) && differ(c, h->cls, op->cls))) bfail(b, "I3 (coloc admit violates SM/profile)", k);
+      }
+      /* I3 under HP_REF_ALL (R3 switch): the tests hold against every HP op in flight at the
+         admission, i.e. seq in [done sampled this iteration, popped after this iteration's HP
+         launch); with none in flight (a busy request between ops) against the last popped one */
+      if (r->kind == D_ADMIT_COLOC && (c->flags & F_HP_REF_ALL)) {
+        const int hh = c->hp;
+        if (pre->done[hh] >= post->popped[hh]) {
+          const o_op *h = &post->hp_ref;
+          if (!((int64_t)op->sm_needed < thr(c, h) && differ(c, h->cls, op->cls))) bfail(b, "I3 (coloc admit violates SM/profile, REF_ALL)", k);
+        } else {
+          for (uint64_t q = pre->done[hh]; q < post->popped[hh]; q++) {
+            const o_op *hq = &c->ops[hh][q];
+            o_op hu = {0u, 0, 0, CLS_U, 0, 0};
+            const o_op *h = hq->kind == KIND_KERNEL ? hq : &hu;
+            if (!((int64_t)op->sm_needed < thr(c, h) && differ(c, h->cls, op->cls))) bfail(b, "I3 (coloc admit violates SM/profile vs an in-flight HP op)", k);
+          }
+        }
       }
       /* I4: admission happens with be_dur <= thr, or after a RESET in this iteration */
       int throttle = !(c->flags & F_NO_THROTTLE) && (!(c->flags & F_THROTTLE_ONLY_HP_BUSY) || hp_busy_pre || hp_launches);

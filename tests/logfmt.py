@@ -101,11 +101,15 @@ def parse_golden(path):
             ops[w[1]] = []
         elif w[0] == "op":
             cname, oname, cls, sm, dur = w[1], w[2], w[3], int(w[4]), int(w[5])
+            # optional request marks (HP_BUSY_REQUEST): REQ_BEGIN, REQ_END or REQ_BEGIN|REQ_END
+            opf = 0
+            for m in (w[6].split("|") if len(w) > 6 else []):
+                opf |= {"REQ_BEGIN": 1, "REQ_END": 2}[m]
             kid = kid_of.setdefault(oname, len(kid_of) + 1)
             if cls in ("MEMCPY",):
-                ops[cname].append((kid, KIND["MEMCPY"], 0, 0, 0, 0))
+                ops[cname].append((kid, KIND["MEMCPY"], opf, 0, 0, 0))
             else:
-                ops[cname].append((kid, 0, 0, CLS[cls], sm, dur))
+                ops[cname].append((kid, 0, opf, CLS[cls], sm, dur))
         elif w[0] == "tape":
             tape.append((int(w[1]), T_VIS if w[2] == "VIS" else T_DONE, names[w[3]], int(w[4])))
         elif w[0] == "kend":

@@ -123,7 +123,9 @@ def test_k_end_truncates():
 
 MUTANTS = {1: "SM test <= instead of <", 2: "profile test inverted", 3: "unknown treated as its own class",
            4: "DUR test >= instead of >", 5: "reset without drain", 6: "be_dur not accumulated",
-           7: "hp_busy never set", 8: "no BE round-robin rotation"}
+           7: "hp_busy never set", 8: "no BE round-robin rotation",
+           9: "HP_REF_ALL checks only the newest in-flight HP op",
+           10: "HP_BUSY_REQUEST ignores a request whose last op is not popped yet"}
 
 
 @pytest.mark.parametrize("m", sorted(MUTANTS))
