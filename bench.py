@@ -222,7 +222,7 @@ def cpu_oracle_sample(cfg_name, budget_s=15.0):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=300, help="HP requests timed under collocation")
+    ap.add_argument("--steps", type=int, default=20, help="timed steps (REQ_PER_STEP HP requests each, per mode and rate)")
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="orion", choices=["orion", "reference"])
     ap.add_argument("--config", default="rn50_mnv2", choices=["rn50_mnv2", "toy", "bert_rn50", "rn101_enc"])
@@ -230,6 +230,7 @@ def main():
     ap.add_argument("--be-partition", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-stress", action="store_true", help="skip the stress-rate (rho 0.3 / 0.6) runs")
     ap.add_argument("--rate", type=float, default=0.0, help="override HP arrival rate (rps)")
     ap.add_argument("--n-be", type=int, default=1, help="number of BE clients (R11; default 1)")
     ap.add_argument("--policy", default="orion", choices=["orion", "orion_noprio", "profiles", "priorities", "streams"],
@@ -262,21 +263,80 @@ def main():
 
     if args.config == "rn101_enc":
         return train_train(args, rank, world, local, metric)
+    return infer_train(args, rank, world, local, metric)
+
+
+REQ_PER_STEP = 50       # HP requests per timed step (each rate, each mode): K = 20 -> 1000 requests
+REPEATS = 3             # dedicated / collocated runs interleaved D, C, D, C, D, C (three repeats)
+STRESS_RHO = (0.3, 0.6)  # stress rates: rho = lambda x L_solo
+
+
+def pct(v, p):
+    """Nearest-rank percentile (R19)."""
+    s = np.sort(np.asarray(v, dtype=np.float64))
+    return float(s[max(0, int(np.ceil(p / 100.0 * len(s))) - 1)]) if len(s) else float("nan")
+
+
+def bootstrap_ratio_ci(col, ded, p=99, n=1000, seed=7):
+    """95 % bootstrap CI of pct(col, p) / pct(ded, p): requests resampled with replacement, the two
+    modes independently (SURVEY §8(d) statistical hygiene)."""
+    rng = np.random.Generator(np.random.PCG64(seed))
+    col, ded = np.asarray(col, dtype=np.float64), np.asarray(ded, dtype=np.float64)
+    r = np.empty(n)
+    for i in range(n):
+        a = col[rng.integers(0, len(col), len(col))]
+        b = ded[rng.integers(0, len(ded), len(ded))]
+        r[i] = pct(a, p) / pct(b, p)
+    return [float(np.percentile(r, 2.5)), float(np.percentile(r, 97.5))]
+
+
+def bootstrap_pct_ci(v, p=99, n=1000, seed=8):
+    rng = np.random.Generator(np.random.PCG64(seed))
+    v = np.asarray(v, dtype=np.float64)
+    r = [pct(v[rng.integers(0, len(v), len(v))], p) for _ in range(n)]
+    return [float(np.percentile(r, 2.5)), float(np.percentile(r, 97.5))]
+
+
+def replay_timing(rl):
+    """The policy oracle (oracle/policy.c, one core) replays the logged run's tape: its decision
+    rate beside the scheduler's (SURVEY §8(d) CPU oracle timing; part of the cpu_baseline leg)."""
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    import logfmt as lf
+    from oracle import policy_ffi as po
+    _, prefix, tape, decs = lf.split_log(rl["log"])
+    n_dec = len(lf.decode_decisions(decs))
+    t0 = time.perf_counter()
+    rep = po.replay(prefix)
+    t_rep = time.perf_counter() - t0
+    win = (rl["t1"] - rl["t0"]) / 1e9
+    return {"decisions": n_dec, "tape_records": len(tape), "bit_exact": rep == decs, "scheduler_window_s": win,
+            "scheduler_decisions_per_s": n_dec / win, "oracle_replay_s": t_rep,
+            "oracle_replay_decisions_per_s": n_dec / max(t_rep, 1e-9), "oracle_cores": 1}
+
+
+def infer_train(args, rank, world, local, metric):
+    """Inf-train configs (BASELINE configs 1-3 and 5): HP open-loop Poisson inference, BE closed-loop
+    training. Per arrival rate (Table 3's, then the stress rates rho = 0.3 and 0.6 of the HP's solo
+    latency) the same request traces run dedicated and collocated, interleaved D, C, D, C, D, C;
+    the collocated runs at Table 3's rate are the timed region (K steps of REQ_PER_STEP requests)."""
+    from paper_conf_eurosys_stratimk24_b200 import collocate as C, profiler as PR, _lib as L, placement as PL
+    from paper_conf_eurosys_stratimk24_b200 import replicas as RP
+    from synth import inputs as si
+    barrier = RP.barrier
     W_ = build_config(args.config, rank)
     rate = args.rate or W_["rate"]
     hpg, beg = W_["hpg"], W_["beg"]
-    # ---- offline profile: solo op durations, sm_needed, class
-    # offline profile: event-timed durations, occupancy sm_needed, class from the committed per-op
+    # ---- offline profile (P:824-879): solo op durations, sm_needed, class from the committed per-op
     # ncu counters (profiles/<config>_<client>_ncu.csv, R16) or the analytic roofline without one
     ncu_hp = os.path.join(ROOT, "profiles", f"{args.config}_hp_ncu.csv")
     ncu_be = os.path.join(ROOT, "profiles", f"{args.config}_be_ncu.csv")
     prof_hp, rows_hp = PR.build_profiles(hpg, 0, reps=5, ncu_csv=ncu_hp)
     prof_be, rows_be = PR.build_profiles(beg, 10000, reps=5, ncu_csv=ncu_be)
     beg.params.reset()
-    hp = C.HPClient(hpg, W_["hp_inputs"], max(args.steps, 64), prof_hp, 0)
+    n_req = max(1, args.steps) * REQ_PER_STEP
+    per_rep = -(-n_req // REPEATS)
+    hp = C.HPClient(hpg, W_["hp_inputs"], max(per_rep, 64), prof_hp, 0)
     be = C.BEClient(beg, prof_be, 10000)
-    # --n-be > 1: more BE clients of the same model on their own data (R11: one shared DUR budget,
-    # round robin); BE throughput is summed over the clients, dedicated = the BE clients without HP
     extra_be = []
     for j in range(1, args.n_be):
         gj = build_config(args.config, rank, be_sub=8 * j)["beg"]
@@ -286,120 +346,140 @@ def main():
     be_all = [be] + extra_be if extra_be else be
     n_hp_k = sum(1 for o in hp.ops if o.kind == L.OP_KERNEL)
     n_be_k = sum(1 for o in be.variants[0] if o.kind == L.OP_KERNEL)
-    sched_cpu = 2 + 4 * local if (os.cpu_count() or 1) >= 8 else -1
-
+    # ---- host cores: scheduler, HP driver, BE driver(s), one each (placement.py)
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", world))
+    cores, place_note = PL.for_this_process(local, local_world, 2 + max(1, args.n_be))
+    sched_cpu, hp_cpu, be_cpus = cores[0], cores[1], cores[2:]
     pol_flags = L.POLICIES[args.policy]
 
     def session(**kw):
-        return C.run_session(sched_cpu=sched_cpu, device=local, flags=pol_flags, **kw)
+        return C.run_session(sched_cpu=sched_cpu, device=local, flags=pol_flags, hp_cpu=hp_cpu, be_cpus=be_cpus, **kw)
 
-    # ---- HP solo request latency -> DUR_THRESHOLD base (R9)
-    spaced = (np.arange(1, 41) * 20e6).astype(np.int64)
+    # ---- HP solo request latency -> DUR_THRESHOLD base (R9: median of 100 solo requests)
+    spaced = (np.arange(1, 101) * 10e6).astype(np.int64)
+    session(hp=hp, arrivals_ns=spaced[:10])                                    # warm the path
     r0 = session(hp=hp, arrivals_ns=spaced)
-    lat0 = np.sort(r0["t_done"] - r0["t_arrival"])
-    hp_lat_ns = int(lat0[len(lat0) // 2])
+    lat0 = r0["t_done"] - r0["t_arrival"]
+    hp_lat_ns = int(np.median(lat0))
+    # ---- scheduler overhead vs direct launches (R20's native arm), same spaced requests
+    C.run_direct(hp, spaced[:10], device=local, hp_cpu=hp_cpu)
+    rn = C.run_direct(hp, spaced, device=local, hp_cpu=hp_cpu)
+    lat_native = rn["t_done"] - rn["t_arrival"]
+    overhead = {"requests": len(spaced), "orion_p50_ms": float(np.median(lat0)) / 1e6,
+                "native_p50_ms": float(np.median(lat_native)) / 1e6,
+                "orion_p99_ms": pct(lat0, 99) / 1e6, "native_p99_ms": pct(lat_native, 99) / 1e6,
+                "p50_overhead": float(np.median(lat0) / np.median(lat_native)) - 1.0}
     # ---- warm-up (untimed)
     if args.warmup:
-        session(hp=hp, be=be, arrivals_ns=si.poisson_arrivals_ns(rate, args.warmup, seed=99, gpu_index=rank),
+        session(hp=hp, be=be, arrivals_ns=si.poisson_arrivals_ns(rate, args.warmup * 4, seed=99, gpu_index=rank),
                 hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm)
-    arrivals = si.poisson_arrivals_ns(rate, args.steps, gpu_index=rank)
-    # ---- dedicated HP (Ideal latency)
-    barrier()
-    rd = session(hp=hp, arrivals_ns=arrivals)
-    ded = C.latency_stats(rd)
+    # ---- dominant BE kernel (largest share of solo time) for the roofline
+    top_row = max(rows_be, key=lambda r: r["dur_ns"])
+    top_kid = top_row["kernel_id"]
+    # ---- interleaved dedicated / collocated runs at each rate
+    rates = [("table3", rate)] + [(f"rho{rho}", rho / (hp_lat_ns / 1e9)) for rho in STRESS_RHO]
+    if args.no_stress:
+        rates = rates[:1]
+    runs = {name: {"ded": [], "col": [], "ratio_per_repeat": []} for name, _ in rates}
+    be_iters, be_time_s, win_ms, trace_ms, stats = 0, 0.0, 0.0, [], None
+    be_iters_all = 0
+    beg.params.reset()
+    with ClockSampler(local) as clk:
+        for name, lam in rates:
+            for rep in range(REPEATS):
+                arr = si.poisson_arrivals_ns(lam, per_rep, seed=si.ARRIVAL_SEED + 17 * rep, gpu_index=rank)
+                rd = session(hp=hp, arrivals_ns=arr)
+                barrier()
+                torch.cuda.synchronize()
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                rc = session(hp=hp, be=be_all, arrivals_ns=arr, hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm,
+                             be_partition_sms=args.be_partition, trace_kernel_id=top_kid if name == "table3" else None)
+                e1.record()
+                torch.cuda.synchronize()
+                barrier()
+                ld, lc = rd["t_done"] - rd["t_arrival"], rc["t_done"] - rc["t_arrival"]
+                runs[name]["ded"] += ld.tolist()
+                runs[name]["col"] += lc.tolist()
+                runs[name]["ratio_per_repeat"].append(pct(lc, 99) / pct(ld, 99))
+                if name == "table3":
+                    win_ms += e0.elapsed_time(e1)
+                    for tb in rc.get("be_t_end_all", [rc["be_t_end"]]):
+                        _, n_ = C.be_throughput({"be_t_end": tb}, rc["t0"], rc["t_hp_end"])
+                        be_iters += n_
+                    be_time_s += (rc["t_hp_end"] - rc["t0"]) / 1e9
+                    trace_ms += list(rc.get("trace_ms", []))
+                    stats = rc["stats"]
+    clocks = clk.summary()
+    be_col = be_iters / max(be_time_s, 1e-9)
+    hp_block = {}
+    for name, lam in rates:
+        d, c = runs[name]["ded"], runs[name]["col"]
+        hp_block[name] = {
+            "rate_rps": lam, "rho": lam * hp_lat_ns / 1e9, "requests": len(c), "repeats": REPEATS,
+            "p50_ms": pct(c, 50) / 1e6, "p99_ms": pct(c, 99) / 1e6,
+            "dedicated_p50_ms": pct(d, 50) / 1e6, "dedicated_p99_ms": pct(d, 99) / 1e6,
+            "p99_vs_dedicated": pct(c, 99) / pct(d, 99), "p50_vs_dedicated": pct(c, 50) / pct(d, 50),
+            "p99_ratio_ci95": bootstrap_ratio_ci(c, d), "p99_ms_ci95": [x / 1e6 for x in bootstrap_pct_ci(c)],
+            "dedicated_p99_ms_ci95": [x / 1e6 for x in bootstrap_pct_ci(d)],
+            "p99_ratio_per_repeat": runs[name]["ratio_per_repeat"]}
+    main_hp = hp_block["table3"]
     # ---- dedicated BE throughput
     beg.params.reset()
     t0 = time.time()
-    rb = session(be=be, be_iters=3)
+    session(be=be, be_iters=3)
     per_it = (time.time() - t0) / 3
-    n_it = int(max(5, min(200, 6.0 / max(per_it, 1e-6))))
+    n_it = int(max(5, min(300, 6.0 / max(per_it, 1e-6))))
     rb = session(be=be_all, be_iters=n_it)
     be_ded = 0.0
     for tb in rb.get("be_t_end_all", [rb["be_t_end"]]):
         be_ded += (len(tb) - 1) / ((tb[-1] - tb[0]) / 1e9) if len(tb) > 1 else float("nan")
-    # ---- dominant BE kernel (largest share of solo time) for the roofline
-    shares = {}
-    for r in rows_be:
-        shares[r["kernel_id"]] = r["dur_ns"]
-    top_kid = max(shares, key=shares.get)
-    top_row = next(r for r in rows_be if r["kernel_id"] == top_kid)
-    # ---- collocated (timed region)
-    beg.params.reset()
-    barrier()
-    torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local) as clk:
-        e0.record()
-        rc = session(hp=hp, be=be_all, arrivals_ns=arrivals, hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm,
-                     be_partition_sms=args.be_partition, trace_kernel_id=top_kid)
-        torch.cuda.synchronize()
-        e1.record()
-        torch.cuda.synchronize()
-    barrier()
-    win_ms = e0.elapsed_time(e1)
-    col = C.latency_stats(rc)
-    be_col, be_n = 0.0, 0
-    for tb in rc.get("be_t_end_all", [rc["be_t_end"]]):
-        c_, n_ = C.be_throughput({"be_t_end": tb}, rc["t0"], rc["t_hp_end"])
-        be_col, be_n = be_col + c_, be_n + n_
-    clocks = clk.summary()
-    # combined utilisation of the pair (analytic): algorithmic HBM bytes and FLOPs of
-    # the work completed in the window / (window x peak), collocated vs each client alone
+    # ---- combined utilisation (analytic): algorithmic bytes / FLOPs of the completed work
     hp_b, hp_f = sum(r["bytes"] for r in rows_hp), sum(r["flops"] for r in rows_hp)
     be_b, be_f = sum(r["bytes"] for r in rows_be), sum(r["flops"] for r in rows_be)
-    win_s = (rc["t_hp_end"] - rc["t0"]) / 1e9
-    n_hp_done = len(rc["t_done"])
     pk_u, _ = peaks()
     tc_peak = pk_u.get("bf16_tflops_sustained", pk_u["bf16_tflops"]) * 1e12 / (6.0 if W_.get("dtype", "f32") == "f32" else 1.0)
     hbm_peak = pk_u["hbm_gbs"] * 1e9
+    n_done = len(runs["table3"]["col"])
     util = {
-        "collocated": {"hbm_gbs": (n_hp_done * hp_b + be_n * be_b) / win_s / 1e9,
-                       "hbm_frac": (n_hp_done * hp_b + be_n * be_b) / win_s / hbm_peak,
-                       "flop_frac": (n_hp_done * hp_f + be_n * be_f) / win_s / tc_peak},
-        "hp_alone": {"hbm_gbs": ded["n"] * hp_b / ((rd["t_done"][-1] - rd["t0"]) / 1e9) / 1e9,
-                     "flop_frac": ded["n"] * hp_f / ((rd["t_done"][-1] - rd["t0"]) / 1e9) / tc_peak},
+        "collocated": {"hbm_gbs": (n_done * hp_b + be_iters * be_b) / be_time_s / 1e9,
+                       "hbm_frac": (n_done * hp_b + be_iters * be_b) / be_time_s / hbm_peak,
+                       "flop_frac": (n_done * hp_f + be_iters * be_f) / be_time_s / tc_peak},
         "be_alone": {"hbm_gbs": be_ded * be_b / 1e9, "hbm_frac": be_ded * be_b / hbm_peak, "flop_frac": be_ded * be_f / tc_peak},
-        "basis": "algorithmic bytes/FLOPs per op (profiler.op_work) x completed requests / iterations; flop peak = the "
-                 "algorithmic ceiling of the path's tensor pipe (bf16, or bf16/6 for fp32 on 3xTF32)"}
-    # roofline of the dominant kernel from its live launches inside the timed region
-    tr = rc.get("trace_ms", [])
+        "be_bytes_per_iteration_GB": be_b / 1e9, "hp_bytes_per_request_GB": hp_b / 1e9,
+        "basis": "algorithmic bytes/FLOPs per op of this implementation's op list (profiler.op_work) x completed "
+                 "requests / iterations; SURVEY §8(d)'s own per-iteration figures (35.7 GB MobileNetV2 b96, 1.16 GB "
+                 "ResNet-50 b4) are the unfused-PyTorch op decomposition; flop peak = the algorithmic ceiling of the "
+                 "path's tensor pipe (bf16, or bf16/6 for fp32 on 3xTF32)"}
+    # ---- roofline of the dominant BE kernel from its live launches inside the timed region
     flops, nbytes = top_row["flops"], top_row["bytes"]
     pk, pk_src = peaks()
-    if tr:
-        avg_s = float(np.mean(tr)) / 1e3
+    roof = {"kernel": top_row["label"], "launches": len(trace_ms), "algorithmic_bytes": nbytes, "algorithmic_flops": flops,
+            "peak_source": pk_src}
+    if trace_ms:
+        avg_s = float(np.mean(trace_ms)) / 1e3
+        pipe = PR.kernel_info(top_row["fn"], dict((i, a) for i, _, a, _ in beg.kernel_ops())[top_kid - 10000])["pipe"] \
+            if hasattr(PR, "kernel_info") else 0
         if top_row["cls"] == "M":
             achieved, peak, unit, bound = nbytes / avg_s / 1e9, pk["hbm_gbs"], "GB/s", "hbm"
-        elif top_row["fn"] in ("gemm_bf16", "attention", "gemm", "conv_fwd", "conv_dgrad", "conv_wgrad"):
-            # timed inside a long collocated window: the sustained bf16 figure (B200_PROFILING.md)
-            tpk = pk.get("bf16_tflops_sustained", pk["bf16_tflops"])
-            if top_row["fn"] in ("gemm_bf16", "attention"):
-                achieved, peak, unit, bound = flops / avg_s / 1e12, tpk, "TFLOP/s", "tensor"
-            else:
-                # 3xTF32 on tcgen05: tf32 dense = bf16 x the guide's nominal 1/2, three MMAs per fp32
-                # product -> algorithmic fp32 peak = bf16 / 6
-                achieved, peak, unit, bound = flops / avg_s / 1e12, tpk / 6.0, "TFLOP/s", "tensor"
+        elif pipe == L.PIPE_BF16:
+            achieved, peak, unit, bound = flops / avg_s / 1e12, pk.get("bf16_tflops_sustained", pk["bf16_tflops"]), "TFLOP/s", "tensor"
+        elif pipe == L.PIPE_TF32X3:
+            # 3xTF32 on tcgen05: tf32 dense = bf16 x the guide's nominal 1/2, three MMAs per fp32 product
+            achieved, peak, unit, bound = flops / avg_s / 1e12, pk.get("bf16_tflops_sustained", pk["bf16_tflops"]) / 6.0, "TFLOP/s", "tensor"
         else:
             achieved, peak, unit, bound = flops / avg_s / 1e12, FFMA_TFLOPS, "TFLOP/s", "alu"
-    else:
-        achieved, peak, unit, bound, avg_s = None, None, None, None, None
+        roof.update(bound=bound, achieved=achieved, peak=peak, unit=unit, frac=achieved / peak, avg_launch_us=avg_s * 1e6)
     traffic = None
-    tp = os.path.join(ROOT, "profiles", f"traffic_{args.config}.json")
-    if os.path.exists(tp):
-        try:
-            traffic = json.load(open(tp)).get(top_row["label"])
-        except Exception:
-            traffic = None
-    if traffic is None:
-        # dram__bytes_read.sum + dram__bytes_write.sum of this op's solo launch in the committed
-        # per-op ncu capture (tools/ncu_times.sh; profiles/<config>_be_ncu.csv)
-        ncu_rows = PR.load_ncu_csv(ncu_be)
-        if top_kid in ncu_rows and ncu_rows[top_kid][2] > 0:
-            traffic = ncu_rows[top_kid][2]
-    # ---- e2e: BE inputs copied from pinned host each iteration (H2D) + loss read back (D2H)
+    ncu_rows = PR.load_ncu_csv(ncu_be)
+    if top_kid in ncu_rows and ncu_rows[top_kid][2] > 0:
+        traffic = ncu_rows[top_kid][2]   # dram read + write bytes of this op's solo launch (committed capture)
+    roof["traffic"] = traffic
+    # ---- e2e: BE inputs copied from pinned host each iteration (H2D) + loss read back (D2H), HP
+    # requests with their H2D input / D2H output, through the same C ABI, at Table 3's rate
     e2e = None
     if not args.no_e2e and not extra_be:
         variants, pinned, loss_host, be_h2d = with_be_h2d(beg, W_["be_inputs"])
-        from paper_conf_eurosys_stratimk24_b200.workloads import Graph  # noqa: F401
         be_e2e = C.BEClient.__new__(C.BEClient)
         be_e2e.graph = beg
         saved = beg.variants
@@ -408,18 +488,23 @@ def main():
         beg.variants = saved
         beg.ops = saved[0]
         beg.params.reset()
+        arr = si.poisson_arrivals_ns(rate, per_rep, gpu_index=rank)
         barrier()
-        re2 = session(hp=hp, be=be_e2e, arrivals_ns=arrivals, hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm,
+        re2 = session(hp=hp, be=be_e2e, arrivals_ns=arr, hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm,
                       be_partition_sms=args.be_partition)
         e2e_its, e2e_n = C.be_throughput(re2, re2["t0"], re2["t_hp_end"])
-        hp_in = hp.inp[0].numel() * 4
-        hp_out = hp.out[0].numel() * 4
-        e2e = {"value": e2e_its, "unit": "it/s", "hp_p99_ms": C.latency_stats(re2)["p99_ns"] / 1e6,
-               "h2d_bytes_per_step": int(hp_in + be_h2d * e2e_n / max(args.steps, 1)),
-               "d2h_bytes_per_step": int(hp_out + 4 * e2e_n / max(args.steps, 1))}
+        hp_in, hp_out = hp.inp[0].numel() * 4, hp.out[0].numel() * 4
+        steps_e2e = per_rep / REQ_PER_STEP
+        e2e = {"value": e2e_its, "unit": "it/s", "requests": per_rep, "hp_p99_ms": C.latency_stats(re2)["p99_ns"] / 1e6,
+               "h2d_bytes_per_step": int((per_rep * hp_in + be_h2d * e2e_n) / steps_e2e),
+               "d2h_bytes_per_step": int((per_rep * hp_out + 4 * e2e_n) / steps_e2e)}
+    # ---- scheduler decision rate on a logged collocated run (the oracle replays the same log below)
+    arr = si.poisson_arrivals_ns(hp_block[rates[-1][0]]["rate_rps"], 200, seed=5, gpu_index=rank)
+    beg.params.reset()
+    rl = session(hp=hp, be=be, arrivals_ns=arr, hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm, log_capacity=1 << 22)
     # ---- aggregate over ranks
-    mine = dict(be_col=be_col, be_ded=be_ded, win_ms=win_ms, p99=col["p99_ns"], p50=col["p50_ns"], p99d=ded["p99_ns"],
-                p50d=ded["p50_ns"], e2e=(e2e or {}).get("value", 0.0), be_n=be_n)
+    mine = dict(be_col=be_col, be_ded=be_ded, win_ms=win_ms, p99=main_hp["p99_ms"], p99d=main_hp["dedicated_p99_ms"],
+                p50=main_hp["p50_ms"], p50d=main_hp["dedicated_p50_ms"], e2e=(e2e or {}).get("value", 0.0), be_n=be_iters)
     allr = RP.gather(mine)
     if rank != 0:
         return
@@ -427,36 +512,34 @@ def main():
     value = agg["value"]
     cpu = None
     if not args.no_cpu_baseline:
-        v, sample, cores = cpu_oracle_sample(args.config)
-        cpu = {"value": v, "unit": "it/s", "cores": cores, "kind": "oracle", "sample": sample}
-    ms_per_step = agg["ms_per_step"]
+        v, sample, ncores = cpu_oracle_sample(args.config)
+        cpu = {"value": v, "unit": "it/s", "cores": ncores, "kind": "oracle", "sample": sample,
+               "replay": replay_timing(rl)}
     line = {
         "metric": metric, "value": value, "unit": "it/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+        "ms_per_step": agg["ms_per_step"], "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
         "dtype": W_.get("dtype", "f32"),
         "data": "synthetic (seeded; DESIGN.md §5)",
         "config": dict(W_["cfg"], parallelism=f"replicas x{world} (independent Orion instance per GPU)",
                        hp_rate_rps=rate, dur_threshold_pct=args.dur_ppm / 1e4, be_partition_sms=args.be_partition,
-                       policy=args.policy, n_be_clients=args.n_be,
+                       policy=args.policy, n_be_clients=args.n_be, requests_per_step=REQ_PER_STEP,
+                       timed_region=f"{REPEATS} collocated runs at the Table-3 rate ({args.steps} steps x {REQ_PER_STEP} "
+                                    f"HP requests), interleaved with dedicated runs of the same traces",
+                       host_cores={"scheduler": sched_cpu, "hp_driver": hp_cpu, "be_drivers": be_cpus, "note": place_note},
                        l2=f"inputs > L2 (BE batch {W_['be_inputs'][0].numel() * 4 / 1e6:.1f} MB x 8 staged; no flush)"),
-        "hp": {"p50_ms": col["p50_ns"] / 1e6, "p99_ms": col["p99_ns"] / 1e6, "dedicated_p50_ms": ded["p50_ns"] / 1e6,
-               "dedicated_p99_ms": ded["p99_ns"] / 1e6, "p99_vs_dedicated": col["p99_ns"] / ded["p99_ns"],
-               "p50_vs_dedicated": col["p50_ns"] / ded["p50_ns"], "solo_latency_ms": hp_lat_ns / 1e6,
-               "requests": col["n"], "per_rank_p99_ratio": agg["hp_p99_ratio_per_rank"],
-               "worst_rank_p99_ratio": agg["hp_p99_ratio_max"]},
+        "hp": dict(main_hp, solo_latency_ms=hp_lat_ns / 1e6, per_rank_p99_ratio=agg["hp_p99_ratio_per_rank"],
+                   worst_rank_p99_ratio=agg["hp_p99_ratio_max"], stress={k: v for k, v in hp_block.items() if k != "table3"},
+                   scheduler_overhead=overhead),
         "be": {"collocated_its": value, "dedicated_its": agg["be_dedicated"],
                "fraction_of_dedicated": value / max(agg["be_dedicated"], 1e-9),
                "iterations_in_window": agg["be_iterations"]},
         "target": {"hp_p99_ratio_max": 1.15, "be_fraction_min": 0.5},
-        "roofline": {"kernel": top_row["label"], "bound": bound, "achieved": achieved, "peak": peak, "unit": unit,
-                     "frac": (achieved / peak) if achieved and peak else None, "traffic": traffic,
-                     "launches": len(tr), "avg_launch_us": avg_s * 1e6 if avg_s else None,
-                     "algorithmic_bytes": nbytes, "algorithmic_flops": flops, "peak_source": pk_src},
+        "roofline": roof,
         "cpu_baseline": cpu,
         "e2e": e2e,
-        "gpu_launches": int(world * args.steps * n_hp_k + sum(r["be_n"] for r in allr) * n_be_k),
+        "gpu_launches": int(world * n_req * n_hp_k + sum(r["be_n"] for r in allr) * n_be_k),
         "clocks": clocks,
-        "scheduler": rc["stats"],
+        "scheduler": stats,
         "utilisation": util,
     }
     print(json.dumps(line), flush=True)
@@ -490,11 +573,12 @@ def train_train(args, rank, world, local, metric):
     beg.params.reset()
     hp = C.HPClient(hpg, [x], 64, prof_hp, 0)
     be = C.BEClient(beg, prof_be, 10000)
-    sched_cpu = 2 + 4 * local if (os.cpu_count() or 1) >= 8 else -1
+    from paper_conf_eurosys_stratimk24_b200 import placement as PL
+    cores, place_note = PL.for_this_process(local, int(os.environ.get("LOCAL_WORLD_SIZE", world)), 3)
     pol = L.POLICIES[args.policy]
 
     def session(**kw):
-        return C.run_session(sched_cpu=sched_cpu, device=local, flags=pol, **kw)
+        return C.run_session(sched_cpu=cores[0], device=local, flags=pol, hp_cpu=cores[1], be_cpus=cores[2:], **kw)
 
     def hp_its(res):
         td = res["t_done"]
@@ -561,7 +645,8 @@ def train_train(args, rank, world, local, metric):
             "config": {"workload": "train-train: HP ResNet-101 training b32 (throughput mode) + BE Transformer-encoder training "
                                    "(6 x d512, 8 heads, FFN 2048, b8 s192), 1 B200 per instance",
                        "parallelism": f"replicas x{world}", "policy": args.policy, "dur_threshold_pct": args.dur_ppm / 1e4,
-                       "sm_threshold_tuned": tuned, "l2": "BE batches 3.1 MB x 8 staged; HP batch 19.3 MB"},
+                       "sm_threshold_tuned": tuned, "l2": "BE batches 3.1 MB x 8 staged; HP batch 19.3 MB",
+                       "host_cores": {"scheduler": cores[0], "hp_driver": cores[1], "be_drivers": cores[2:], "note": place_note}},
             "hp": {"throughput_its": hp_col, "dedicated_its": hp_ded, "fraction_of_dedicated": hp_col / hp_ded,
                    "default_sm_threshold": {"hp_fraction": hp_def / hp_ded, "be_its": be_def},
                    "sm_threshold_search": [{"sm_threshold": p[0], "hp_fraction": p[1], "be_its": p[2]} for p in probes]},

@@ -103,6 +103,24 @@ def bn_train_fwd(x, gamma, beta, rmean, rvar, eps=1e-5, momentum=0.1):
     return _r(y), _r(mean), _r(invstd), _r(rm), _r(rv)
 
 
+def bn_bwd_abs(x, dy, mean, invstd):
+    """Absolute-term sums of bn_bwd's parameter gradients: sum |dy * xhat| and sum |dy| per
+    channel. Not a result of the method: the scale of the rounding-error bound of each gradient
+    element (|fl(sum t) - sum t| <= c u sum |t|), used by the parity tests' error model
+    (DESIGN.md §8)."""
+    c = x.shape[-1]
+    xhat = (_d(x).reshape(-1, c) - _d(mean)) * _d(invstd)
+    dyd = _d(dy).reshape(-1, c).abs()
+    return (dyd * xhat.abs()).sum(0), dyd.sum(0)
+
+
+def conv2d_bwd_weight_abs(x, dy, w_shape, stride=1, pad=0, groups=1):
+    """sum |x| |dy| over the same (image, tap) pairs as conv2d_bwd_weight: its error-bound scale."""
+    o, kh, kw, ig = w_shape
+    dw = torch.nn.grad.conv2d_weight(_nchw(_d(x).abs()), (o, ig, kh, kw), _nchw(_d(dy).abs()), stride, pad, 1, groups)
+    return dw.permute(0, 2, 3, 1).contiguous()
+
+
 def bn_bwd(x, dy, gamma, mean, invstd):
     """Backward of training-mode BN given the saved (fp32) batch mean / invstd.
     xhat = (x-mean)*invstd; dbeta = sum dy; dgamma = sum dy*xhat;
@@ -323,7 +341,7 @@ def mnv2_trainable(spec):
     return [n for n, _, _ in spec if not (n.endswith(".rmean") or n.endswith(".rvar"))]
 
 
-def mnv2_train_step(P, V, x, labels, first, lr=0.01, momentum=0.9, eps=1e-5, bn_momentum=0.1, masks=None):
+def mnv2_train_step(P, V, x, labels, first, lr=0.01, momentum=0.9, eps=1e-5, bn_momentum=0.1, masks=None, trace=None):
     """One training iteration of torchvision MobileNetV2 (dropout p=0, reading R22) with
     CE loss and SGD(momentum). P: params + BN running stats (dict of fp32 tensors);
     V: momentum buffers (dict). Returns (loss, newP, newV, grads).
@@ -331,14 +349,24 @@ def mnv2_train_step(P, V, x, labels, first, lr=0.01, momentum=0.9, eps=1e-5, bn_
     masks (optional): {bn name: fp32 tensor} — the values on which the ReLU6 backward takes its
     pass/stop decision (0 < y < 6). A decision is an integer decided by floating point; to compare
     a fp32 GPU backward with this fp64 oracle both must decide on the same value, so
-    parity tests pass the GPU's own BN outputs here. All arithmetic stays the oracle's."""
+    parity tests pass the GPU's own BN outputs here, after auditing them against the oracle's own
+    (trace["bn_out"]). All arithmetic stays the oracle's.
+
+    trace (optional dict, test instrumentation): filled with "bn_out" {bn name: the oracle's own BN
+    output, on which its free-running ReLU6 decides} and "abs" {gradient name: the absolute-term sum
+    of every gradient element, the scale of its rounding-error bound}."""
     newP = dict(P)
+    if trace is not None:
+        trace.setdefault("bn_out", {})
+        trace.setdefault("abs", {})
 
     def conv_bn(h, cname, bname, k, stride, groups, act):
         z = conv2d_fwd(h, P[f"{cname}.w"], stride, k // 2, groups)
         y, mean, invstd, rm, rv = bn_train_fwd(z, P[f"{bname}.gamma"], P[f"{bname}.beta"],
                                                P[f"{bname}.rmean"], P[f"{bname}.rvar"], eps, bn_momentum)
         newP[f"{bname}.rmean"], newP[f"{bname}.rvar"] = rm, rv
+        if trace is not None:
+            trace["bn_out"][bname] = y
         rec = (cname, bname, k, stride, groups, act, h, z, y, mean, invstd)
         return (relu6(y) if act else y), rec
 
@@ -350,6 +378,9 @@ def mnv2_train_step(P, V, x, labels, first, lr=0.01, momentum=0.9, eps=1e-5, bn_
         dz, g[f"{bname}.gamma"], g[f"{bname}.beta"] = bn_bwd(z, dy, P[f"{bname}.gamma"], mean, invstd)
         w = P[f"{cname}.w"]
         g[f"{cname}.w"] = conv2d_bwd_weight(hin, dz, tuple(w.shape), stride, k // 2, groups)
+        if trace is not None:
+            trace["abs"][f"{bname}.gamma"], trace["abs"][f"{bname}.beta"] = bn_bwd_abs(z, dy, mean, invstd)
+            trace["abs"][f"{cname}.w"] = conv2d_bwd_weight_abs(hin, dz, tuple(w.shape), stride, k // 2, groups)
         return conv2d_bwd_data(dz, w, tuple(hin.shape), stride, k // 2, groups) if need_dx else None
 
     # ---- forward
@@ -373,6 +404,9 @@ def mnv2_train_step(P, V, x, labels, first, lr=0.01, momentum=0.9, eps=1e-5, bn_
 
     # ---- backward (reverse op order)
     dpooled, g["classifier.w"], g["classifier.b"] = linear_bwd(pooled, P["classifier.w"], dlogits)
+    if trace is not None:
+        trace["abs"]["classifier.w"] = _d(dlogits).abs().t() @ _d(pooled).abs()
+        trace["abs"]["classifier.b"] = _d(dlogits).abs().sum(0)
     dh = avgpool_bwd(dpooled, feat_shape)
     dh = conv_bn_bwd(last, dh)
     for res, r in reversed(recs):
@@ -417,14 +451,20 @@ def maxpool3x3s2_bwd(x, dy):
 
 # -------------------------------------------------------------------- ResNet training
 def resnet_train_step(P, V, x, labels, first, layers=RESNET50_LAYERS, lr=0.01, momentum=0.9, eps=1e-5,
-                      bn_momentum=0.1, masks=None):
+                      bn_momentum=0.1, masks=None, trace=None):
     """One training iteration of TorchVision ResNet v1.5 (train-mode BN, CE, SGD momentum), the
     BE client of BASELINE config 3 (ResNet-50, batch 64) and HP of config 4 (ResNet-101).
     Ops in PyTorch eager order, each rounded to fp32 (R22-R24). masks (optional): {name: fp32
     tensor} of the values the GPU's ReLU backward decides on (its BN / residual-sum outputs), as in
-    mnv2_train_step (DESIGN.md §8). Returns (loss, newP, newV, grads)."""
+    mnv2_train_step; the max-pool backward then also picks its first maxima on
+    relu(masks["bn1"]), the GPU's own max-pool input. trace (optional dict): filled with "relu_in"
+    {name: the oracle's own ReLU input} and "abs" {gradient: absolute-term sums}, as in
+    mnv2_train_step. Returns (loss, newP, newV, grads)."""
     newP = dict(P)
     g = {}
+    if trace is not None:
+        trace.setdefault("relu_in", {})
+        trace.setdefault("abs", {})
 
     def cb(h, cname, bname, stride, pad):
         z = conv2d_fwd(h, P[f"{cname}.w"], stride, pad)
@@ -438,9 +478,14 @@ def resnet_train_step(P, V, x, labels, first, layers=RESNET50_LAYERS, lr=0.01, m
         dz, g[f"{bname}.gamma"], g[f"{bname}.beta"] = bn_bwd(z, dy, P[f"{bname}.gamma"], mean, invstd)
         w = P[f"{cname}.w"]
         g[f"{cname}.w"] = conv2d_bwd_weight(hin, dz, tuple(w.shape), stride, pad)
+        if trace is not None:
+            trace["abs"][f"{bname}.gamma"], trace["abs"][f"{bname}.beta"] = bn_bwd_abs(z, dy, mean, invstd)
+            trace["abs"][f"{cname}.w"] = conv2d_bwd_weight_abs(hin, dz, tuple(w.shape), stride, pad)
         return conv2d_bwd_data(dz, w, tuple(hin.shape), stride, pad) if need_dx else None
 
     def m(name, val):
+        if trace is not None:
+            trace["relu_in"][name] = val
         return masks[name] if masks is not None else val
 
     # ---- forward
@@ -473,6 +518,9 @@ def resnet_train_step(P, V, x, labels, first, layers=RESNET50_LAYERS, lr=0.01, m
 
     # ---- backward (reverse op order)
     dpooled, g["fc.w"], g["fc.b"] = linear_bwd(pooled, P["fc.w"], dlogits)
+    if trace is not None:
+        trace["abs"]["fc.w"] = _d(dlogits).abs().t() @ _d(pooled).abs()
+        trace["abs"]["fc.b"] = _d(dlogits).abs().sum(0)
     dh = avgpool_bwd(dpooled, feat_shape)
     for p, r1, y1, r2, y2, r3, rd, sm in reversed(blocks):
         dsm = relu_bwd(m(f"{p}.sum", sm), dh)
@@ -483,7 +531,7 @@ def resnet_train_step(P, V, x, labels, first, layers=RESNET50_LAYERS, lr=0.01, m
         d = cb_bwd(r1, d)
         didn = cb_bwd(rd, dsm) if rd is not None else dsm
         dh = add(d, didn)
-    da = maxpool3x3s2_bwd(a, dh)
+    da = maxpool3x3s2_bwd(relu(masks["bn1"]) if masks is not None else a, dh)
     dy = relu_bwd(m("bn1", y), da)
     cb_bwd(stem, dy, need_dx=False)
 
@@ -693,13 +741,30 @@ def mha_bwd(q, k, v, do, heads):
     return merge(dQ), merge(dK), merge(dV)
 
 
-def encoder_train_step(P, V, x, t, first, layers=6, heads=8, lr=0.01, momentum=0.9, eps=1e-5, masks=None):
+def encoder_train_step(P, V, x, t, first, layers=6, heads=8, lr=0.01, momentum=0.9, eps=1e-5, masks=None, trace=None):
     """One training iteration of the post-LN encoder stack on x [B, S, d] with MSE to t.
     masks (optional): {name: fp32 tensor} — the values the GPU's ReLU backward decided on (its FFN
-    pre-activations), as in the other training oracles. Returns (loss, newP, newV, grads)."""
+    pre-activations), as in the other training oracles. trace (optional dict):
+    "relu_in" {name: the oracle's own FFN pre-activation} and "abs" {gradient: absolute-term sums}.
+    Returns (loss, newP, newV, grads)."""
     b, sq, dm = x.shape
     rows = b * sq
     g = {}
+    if trace is not None:
+        trace.setdefault("relu_in", {})
+        trace.setdefault("abs", {})
+
+    def lin_abs(name, xin, dy):
+        if trace is not None:
+            trace["abs"][f"{name}.w"] = _d(dy).abs().t() @ _d(xin).abs()
+            trace["abs"][f"{name}.b"] = _d(dy).abs().sum(0)
+
+    def ln_abs(name, xin, dy, mean, rstd):
+        if trace is not None:
+            xh = ((_d(xin) - _d(mean)[..., None]) * _d(rstd)[..., None]).abs()
+            red = tuple(range(xin.dim() - 1))
+            trace["abs"][f"{name}.gamma"] = (_d(dy).abs() * xh).sum(red)
+            trace["abs"][f"{name}.beta"] = _d(dy).abs().sum(red)
     recs = []
     h = x.reshape(rows, dm)
     for i in range(layers):
@@ -722,15 +787,23 @@ def encoder_train_step(P, V, x, t, first, layers=6, heads=8, lr=0.01, momentum=0
         p = f"enc{i}"
         hin, q, k, v, a, s1, h1, m1, r1, f, fa, s2, m2, r2 = recs[i]
         ds2, g[f"{p}.ln2.gamma"], g[f"{p}.ln2.beta"] = layernorm_bwd(s2, dh, P[f"{p}.ln2.gamma"], m2, r2)
+        ln_abs(f"{p}.ln2", s2, dh, m2, r2)
         dfa, g[f"{p}.ff2.w"], g[f"{p}.ff2.b"] = linear_bwd(fa, P[f"{p}.ff2.w"], ds2)
+        lin_abs(f"{p}.ff2", fa, ds2)
+        if trace is not None:
+            trace["relu_in"][f"{p}.ff1"] = f
         df = relu_bwd(masks[f"{p}.ff1"] if masks is not None else f, dfa)
         dh1_ff, g[f"{p}.ff1.w"], g[f"{p}.ff1.b"] = linear_bwd(h1, P[f"{p}.ff1.w"], df)
+        lin_abs(f"{p}.ff1", h1, df)
         dh1 = add(ds2, dh1_ff)
         ds1, g[f"{p}.ln1.gamma"], g[f"{p}.ln1.beta"] = layernorm_bwd(s1, dh1, P[f"{p}.ln1.gamma"], m1, r1)
+        ln_abs(f"{p}.ln1", s1, dh1, m1, r1)
         da, g[f"{p}.out.w"], g[f"{p}.out.b"] = linear_bwd(a, P[f"{p}.out.w"], ds1)
+        lin_abs(f"{p}.out", a, ds1)
         dq, dk, dv = mha_bwd(q, k, v, da.reshape(b, sq, dm), heads)
         dqkv = torch.cat([dq.reshape(rows, dm), dk.reshape(rows, dm), dv.reshape(rows, dm)], dim=1)
         dhin_attn, g[f"{p}.in.w"], g[f"{p}.in.b"] = linear_bwd(hin, P[f"{p}.in.w"], dqkv)
+        lin_abs(f"{p}.in", hin, dqkv)
         dh = add(ds1, dhin_attn)
     newP, newV = dict(P), {}
     for n in sorted(g):

@@ -7,6 +7,7 @@ Dedicated runs (the "Ideal" baseline) use the same binary with the 
 absent (R20).
 """
 import ctypes
+import os
 import threading
 
 import numpy as np
@@ -54,10 +55,12 @@ class BEClient:
 
 def run_session(hp=None, be=None, arrivals_ns=None, be_iters=0, log_capacity=0, hp_latency_ns=0,
                 dur_threshold_ppm=25000, sm_threshold=0, be_partition_sms=0, flags=0, sched_cpu=-1,
-                backend=L.BACKEND_CUDA, device=0, trace_kernel_id=None):
+                backend=L.BACKEND_CUDA, device=0, trace_kernel_id=None, hp_cpu=None, be_cpus=None):
     """Run one session. HP (if given) issues len(arrivals_ns) requests open loop; BE (a client or a
     list of clients, each on its own thread and stream) runs closed loop until HP finishes (or
     be_iters iterations if HP is absent / be_iters > 0 and no HP).
+    hp_cpu / be_cpus: host cores the HP driver (this thread, for the session) and the BE driver
+    threads pin themselves to (placement.py), so no two busy-polling threads share a core.
     Returns dict with HP arrival/completion ns, BE iteration end times, window, log bytes, stats."""
     o = Orion(device=device, backend=backend, hp_latency_ns=hp_latency_ns, dur_threshold_ppm=dur_threshold_ppm,
               sm_threshold=sm_threshold, be_partition_sms=be_partition_sms, flags=flags, sched_cpu=sched_cpu,
@@ -76,6 +79,8 @@ def run_session(hp=None, be=None, arrivals_ns=None, be_iters=0, log_capacity=0, 
         res["be_t_end_all"] = [None] * len(bes)
 
         def be_main(j):
+            if be_cpus:
+                os.sched_setaffinity(0, {be_cpus[j % len(be_cpus)]})
             try:
                 res["be_t_end_all"][j] = o.run_iterations(be_ids[j], bes[j].variants, stop_flag=stop, max_iters=max_iters)
             except Exception as e:  # surfaced below
@@ -86,8 +91,11 @@ def run_session(hp=None, be=None, arrivals_ns=None, be_iters=0, log_capacity=0, 
             th.start()
     else:
         res["t0"] = o_now = L.lib.orion_now_ns()
+    prev_mask = os.sched_getaffinity(0) if hp_cpu is not None else None
     try:
         if hp is not None:
+            if hp_cpu is not None:
+                os.sched_setaffinity(0, {hp_cpu})
             ta, td = o.run_requests(hp_id, hp.ops, arrivals_ns, in_cycle=hp.inp.shape[0], out_cycle=hp.n_req)
             res["t_arrival"], res["t_done"] = ta, td
             res["t_hp_end"] = L.lib.orion_now_ns()
@@ -103,6 +111,9 @@ def run_session(hp=None, be=None, arrivals_ns=None, be_iters=0, log_capacity=0, 
             pass
         o.destroy()
         raise
+    finally:
+        if prev_mask is not None:
+            os.sched_setaffinity(0, prev_mask)
     if hp is not None:
         stop.value = 1
     for th in ths:
@@ -125,16 +136,20 @@ def run_session(hp=None, be=None, arrivals_ns=None, be_iters=0, log_capacity=0, 
     return res
 
 
-def run_direct(hp, arrivals_ns, device=0):
+def run_direct(hp, arrivals_ns, device=0, hp_cpu=None):
     """The native arm (R20; P:1355-1360 measures Orion's overhead against it): the HP request stream
     launched directly on one stream by the client thread, no scheduler. Same completion counters and
     clock as run_session, so latencies compare one to one."""
     o = Orion(device=device, backend=L.BACKEND_CUDA)
+    prev = os.sched_getaffinity(0)
     try:
         cid = o.register_client(L.HP)
         torch.cuda.synchronize()
+        if hp_cpu is not None:
+            os.sched_setaffinity(0, {hp_cpu})
         ta, td = o.run_requests_direct(cid, hp.ops, arrivals_ns, in_cycle=hp.inp.shape[0], out_cycle=hp.n_req)
     finally:
+        os.sched_setaffinity(0, prev)
         o.destroy()
     return {"t_arrival": ta, "t_done": td}
 

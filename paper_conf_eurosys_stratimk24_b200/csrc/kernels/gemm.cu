@@ -600,7 +600,8 @@ template <int BN, class LA, class LB>
 __global__ void __launch_bounds__(NTHR, 1) gemm_tc_kernel(GemmParams p, LA la, LB lb, OrionSig sig) {
   using Cfg = TcCfg<BN>;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
-  unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // offset the shared array itself (not a uintptr_t round trip), so accesses stay LDS/STS
+  unsigned char* smem = smem_raw + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_raw) & 1023u)) & 1023u);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + Cfg::STAGES * Cfg::STAGE_BYTES);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * Cfg::STAGES + 1);
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + Cfg::STAGES), done_bar = smem_u32(bars + 2 * Cfg::STAGES);
@@ -839,7 +840,8 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tcm_kernel(Params p, LA la, LB l
   constexpr int TMEM_COLS = C_::TMEM_COLS;
   constexpr uint32_t IDESC = C_::IDESC;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
-  unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // offset the shared array itself (not a uintptr_t round trip), so accesses stay LDS/STS
+  unsigned char* smem = smem_raw + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_raw) & 1023u)) & 1023u);
   unsigned char* raw = smem + STAGES * STAGE_BYTES;
   float* epi = reinterpret_cast<float*>(raw + RAW_STAGES * RAW_BYTES);
   uint64_t* bars = reinterpret_cast<uint64_t*>(raw + RAW_STAGES * RAW_BYTES + EPI_BYTES);
@@ -1142,7 +1144,8 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_tmk_kernel(const __grid_constant
   using C_ = Cfg<BN_, BMN>;
   constexpr int BN = C_::BN, A_BYTES = C_::A_BYTES, B_BYTES = C_::B_BYTES, STAGE_BYTES = C_::STAGE_BYTES, STAGES = C_::STAGES;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
-  unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // offset the shared array itself (not a uintptr_t round trip), so accesses stay LDS/STS
+  unsigned char* smem = smem_raw + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_raw) & 1023u)) & 1023u);
   unsigned char* epi = smem + STAGES * STAGE_BYTES;
   uint64_t* bars = reinterpret_cast<uint64_t*>(epi + EPI_BYTES);
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 3 * STAGES + 4);

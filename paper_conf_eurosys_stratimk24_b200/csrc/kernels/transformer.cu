@@ -123,7 +123,8 @@ __global__ void __launch_bounds__(NTHR, 1) gemm_bf16_kernel(const __grid_constan
                                                            OrionSig sig) {
   using Cf = Cfg<BN>;
   extern __shared__ __align__(1024) unsigned char smem_raw[];
-  unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // offset the shared array itself (not a uintptr_t round trip), so accesses stay LDS/STS
+  unsigned char* smem = smem_raw + ((1024u - ((uint32_t)__cvta_generic_to_shared(smem_raw) & 1023u)) & 1023u);
   constexpr int S = Cf::STAGES;
   float* bias_s = reinterpret_cast<float*>(smem + Cf::MAIN);
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + Cf::MAIN + BN * 4);

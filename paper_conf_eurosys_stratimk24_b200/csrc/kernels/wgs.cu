@@ -64,7 +64,7 @@ inline int smem_bytes(int mi, int nb, int R, int stages) {
   const int red = NCW * V * 4, comb = (V + NTHR) * 8;
   if (red > body) body = red;
   if (comb > body) body = comb;
-  return 256 + body + 128;   // barriers, stage / reduction area, alignment slack
+  return 256 + body;   // barriers, stage / reduction area
 }
 
 // Shape-only plan (never the SM count of the partition): pick the operand roles and register
@@ -126,10 +126,11 @@ template <int MI, int NB>
 __global__ void __maxnreg__(MAXREG) wgs_kernel(const __grid_constant__ CUtensorMap tmL, const __grid_constant__ CUtensorMap tmQ,
                                                      Params p, OrionSig sig) {
   constexpr int TL = 32 * MI, ROWF = TL + NB, V = TL * NB;
+  // (pointers derived from the shared array itself, so the compiler emits LDS, not generic loads;
+  // dynamic shared memory is 128-byte aligned, more than TMA's 16 bytes without swizzle)
   extern __shared__ __align__(128) unsigned char wgs_smem[];
-  unsigned char* base = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(wgs_smem) + 127) & ~uintptr_t(127));
-  uint64_t* bars = reinterpret_cast<uint64_t*>(base);   // full[stages], empty[stages]
-  float* ring = reinterpret_cast<float*>(base + 256);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(wgs_smem);   // full[stages], empty[stages]
+  float* ring = reinterpret_cast<float*>(wgs_smem + 256);
   const int R = p.R, S = p.stages, stage_floats = R * ROWF;
   const uint32_t full0 = smem_u32(bars), empty0 = full0 + 8 * S;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;

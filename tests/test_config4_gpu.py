@@ -2,8 +2,8 @@
 post-LN Transformer-encoder training (fp32) under liborion.
   * teacher-forced per-op parity of the encoder's op list at full width (d 512, 8 heads, FFN 2048,
     batch 8, seq 192; 2 layers) vs the fp64 oracle ops (2e-5);
-  * one encoder iteration end to end vs the oracle (loss 1e-5, gradients 3e-4 with the ReLU
-    decisions taken on the GPU's own pre-activations, updated parameters 1e-5);
+  * two encoder iterations end to end vs the oracle, and two full-size ResNet-101 b32 HP training
+    iterations vs the oracle, ReLU decisions audited (tests/parity.py, DESIGN.md §8);
   * a collocated session (HP ResNet-101 at a reduced batch): decision log == oracle replay byte for
     byte, HP and BE parameters bitwise identical to solo runs of the same iteration counts."""
 import numpy as np
@@ -61,20 +61,49 @@ def test_encoder_ops_teacher_forced():
     assert not bad, sorted(bad, reverse=True)[:10]
 
 
-def test_encoder_one_iteration_vs_oracle():
+def test_encoder_iterations_vs_oracle():
+    """K = 2 encoder iterations (2 layers at full width) vs the fp64 oracle, the GPU's FFN ReLU
+    decisions audited against the oracle's own pre-activations (tests/parity.py)."""
+    import copy
+    import parity as PT
     P, xs, ts, g = _enc()
     be = C.BEClient(g)
     g.params.reset()
-    C.run_session(be=be, be_iters=1)
-    G = g.params
-    masks = {k: v.cpu() for k, v in g.relu_in.items()}
-    loss, newP, _, g_ref = om.encoder_train_step(P, {}, xs[0], ts[0], first=True, layers=2, masks=masks)
-    assert rel(g.loss, loss.reshape(1)) < 1e-5
-    worst = {n: rel(G.g[n], r, 1e-6) for n, r in g_ref.items()}
-    print("worst gradient errors:", sorted(worst.items(), key=lambda x: -x[1])[:6])
-    assert max(worst.values()) < 3e-4
-    for n in newP:
-        assert rel(G.p[n], newP[n]) < 1e-5, n
+
+    def run_one(it):
+        one = copy.copy(be)
+        one.variants = [be.variants[it]]
+        C.run_session(be=one, be_iters=1)
+
+    def step(Pp, V, x, t, first, masks, trace):
+        return om.encoder_train_step(Pp, V, x, t, first=first, layers=2, masks=masks, trace=trace)
+    rep = PT.check_train_iterations(run_one, g, step, xs, ts, P, 2, "relu_in", (0.0,))
+    print("encoder iterations vs oracle:", rep)
+
+
+def test_rn101_hp_training_full_size_vs_oracle():
+    """Config 4's HP at its full size: one ResNet-101 training iteration at batch 32, 224x224 (the
+    HP op list the train-train bench runs), and a second one, vs the fp64 oracle with audited ReLU
+    decisions (tests/parity.py)."""
+    import copy
+    import parity as PT
+    torch.cuda.set_device(0)
+    Pr = si.make_params(W.resnet_train_spec(W.RESNET101_LAYERS))
+    xs = [si.normal((32, 224, 224, 3), si.HP_SEED, sub=i) for i in range(2)]
+    labs = [si.labels(32, 1000, si.HP_SEED, sub=i) for i in range(2)]
+    hpg = W.resnet_train_graph(Pr, xs, labs, layers=W.RESNET101_LAYERS)
+    be = C.BEClient(hpg)
+    hpg.params.reset()
+
+    def run_one(it):
+        one = copy.copy(be)
+        one.variants = [be.variants[it]]
+        C.run_session(be=one, be_iters=1)
+
+    def step(Pp, V, x, lab, first, masks, trace):
+        return om.resnet_train_step(Pp, V, x, lab, first=first, layers=W.RESNET101_LAYERS, masks=masks, trace=trace)
+    rep = PT.check_train_iterations(run_one, hpg, step, xs, labs, Pr, 2, "relu_in", (0.0,))
+    print("ResNet-101 b32 training iterations vs oracle:", rep)
 
 
 def test_rn101_hp_encoder_be_collocated():

@@ -321,3 +321,25 @@ def test_mnv2_train_step_vs_torchvision():
     k = "classifier.w"
     torch.testing.assert_close(newP[k].double(), P[k].double() - 0.01 * named[_mn_rename(k)].grad, rtol=1e-5, atol=1e-7)
     assert worst < 1e-3
+
+
+def test_abs_sum_scales():
+    """The error-model scales (trace["abs"]) are absolute-term sums: they bound |gradient|
+    elementwise (triangle inequality) and equal it when every term has one sign."""
+    g = torch.Generator().manual_seed(5)
+    x = torch.randn(2, 5, 6, 4, generator=g, dtype=torch.float32)
+    dy = torch.randn(2, 5, 6, 3, generator=g, dtype=torch.float32)
+    w_shape = (3, 1, 1, 4)
+    dw = om.conv2d_bwd_weight(x, dy, w_shape).double()
+    A = om.conv2d_bwd_weight_abs(x, dy, w_shape)
+    assert bool((A >= dw.abs() - 1e-6).all())
+    assert torch.allclose(om.conv2d_bwd_weight_abs(x.abs(), dy.abs(), w_shape), om.conv2d_bwd_weight(x.abs(), dy.abs(), w_shape).double(), rtol=1e-6)
+    dw3 = om.conv2d_bwd_weight(x, torch.randn(2, 5, 6, 4, generator=g), (4, 3, 3, 1), 1, 1, groups=4)
+    assert om.conv2d_bwd_weight_abs(x, torch.randn(2, 5, 6, 4, generator=g), (4, 3, 3, 1), 1, 1, groups=4).shape == dw3.shape
+    z = torch.randn(2, 5, 6, 4, generator=g, dtype=torch.float32)
+    dyb = torch.randn(2, 5, 6, 4, generator=g, dtype=torch.float32)
+    mean, invstd = z.double().reshape(-1, 4).mean(0).float(), (1 / z.double().reshape(-1, 4).std(0, unbiased=False)).float()
+    _, dgam, dbet = om.bn_bwd(z, dyb, torch.ones(4), mean, invstd)
+    Ag, Ab = om.bn_bwd_abs(z, dyb, mean, invstd)
+    assert bool((Ag >= dgam.double().abs() - 1e-6).all()) and bool((Ab >= dbet.double().abs() - 1e-6).all())
+    assert torch.allclose(om.bn_bwd_abs(z, dyb.abs(), mean, invstd)[1], om.bn_bwd(z, dyb.abs(), torch.ones(4), mean, invstd)[2].double(), rtol=1e-6)
