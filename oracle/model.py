@@ -323,17 +323,40 @@ def mnv2_blocks(width_mult=1.0):
     return blocks
 
 
-def mnv2_spec(num_classes=1000):
-    s = _conv_spec("features.0", 32, 3, 3) + _bn_spec("features.0.bn", 32, False)
+def mnv2_spec(num_classes=1000, eval_stats=False):
+    """eval_stats: seeded running statistics (the inference clients, reading R22) instead of torch's
+    training start (0, 1)."""
+    e = eval_stats
+    s = _conv_spec("features.0", 32, 3, 3) + _bn_spec("features.0.bn", 32, e)
     for name, cin, hid, cout, stride, expand, res in mnv2_blocks():
         if expand:
-            s += _conv_spec(f"{name}.expand", hid, 1, cin) + _bn_spec(f"{name}.expand_bn", hid, False)
-        s += _conv_spec(f"{name}.dw", hid, 3, 1) + _bn_spec(f"{name}.dw_bn", hid, False)
-        s += _conv_spec(f"{name}.project", cout, 1, hid) + _bn_spec(f"{name}.project_bn", cout, False)
-    s += _conv_spec("features.18", 1280, 1, 320) + _bn_spec("features.18.bn", 1280, False)
+            s += _conv_spec(f"{name}.expand", hid, 1, cin) + _bn_spec(f"{name}.expand_bn", hid, e)
+        s += _conv_spec(f"{name}.dw", hid, 3, 1) + _bn_spec(f"{name}.dw_bn", hid, e)
+        s += _conv_spec(f"{name}.project", cout, 1, hid) + _bn_spec(f"{name}.project_bn", cout, e)
+    s += _conv_spec("features.18", 1280, 1, 320) + _bn_spec("features.18.bn", 1280, e)
     # torchvision MobileNetV2 classifier init: normal(0, 0.01), bias zeros
     s += [("classifier.w", (num_classes, 1280), ("normal", 0.01)), ("classifier.b", (num_classes,), ("const", 0.0))]
     return s
+
+
+def mnv2_infer(P, x):
+    """TorchVision MobileNetV2 inference (eval-mode BN, ReLU6, dropout inactive): x NHWC [N,H,W,3] ->
+    logits. A best-effort inference client of the inf-inf configuration (Table 1 b4)."""
+    def cb(h, cname, bname, k, stride, groups, act):
+        h = conv2d_fwd(h, P[f"{cname}.w"], stride, k // 2, groups)
+        h = bn_eval(h, P[f"{bname}.gamma"], P[f"{bname}.beta"], P[f"{bname}.rmean"], P[f"{bname}.rvar"])
+        return relu6(h) if act else h
+    h = cb(x, "features.0", "features.0.bn", 3, 2, 1, True)
+    for name, cin, hid, cout, stride, expand, res in mnv2_blocks():
+        inp = h
+        if expand:
+            h = cb(h, f"{name}.expand", f"{name}.expand_bn", 1, 1, 1, True)
+        h = cb(h, f"{name}.dw", f"{name}.dw_bn", 3, stride, hid, True)
+        h = cb(h, f"{name}.project", f"{name}.project_bn", 1, 1, 1, False)
+        if res:
+            h = add(h, inp)
+    h = cb(h, "features.18", "features.18.bn", 1, 1, 1, True)
+    return linear_fwd(avgpool_fwd(h), P["classifier.w"], P["classifier.b"])
 
 
 def mnv2_trainable(spec):
@@ -739,6 +762,24 @@ def mha_bwd(q, k, v, do, heads):
     def merge(t):
         return _r(t.permute(0, 2, 1, 3).reshape(b, sq, hd))
     return merge(dQ), merge(dK), merge(dV)
+
+
+def encoder_infer(P, x, layers=6, heads=8, eps=1e-5):
+    """Forward of the post-LN encoder stack (reading R32) in fp32 storage: x [B, S, d] -> the last
+    layer's output [B*S, d]. The "Transformer" inference client of the inf-inf configuration."""
+    b, sq, dm = x.shape
+    rows = b * sq
+    h = x.reshape(rows, dm)
+    for i in range(layers):
+        p = f"enc{i}"
+        qkv = linear_fwd(h, P[f"{p}.in.w"], P[f"{p}.in.b"])
+        q, k, v = (qkv[:, j * dm:(j + 1) * dm].reshape(b, sq, dm) for j in range(3))
+        a = mha_fwd(q, k, v, heads).reshape(rows, dm)
+        s1 = add(h, linear_fwd(a, P[f"{p}.out.w"], P[f"{p}.out.b"]))
+        h1, _, _ = layernorm_fwd(s1, P[f"{p}.ln1.gamma"], P[f"{p}.ln1.beta"], eps)
+        f2 = linear_fwd(relu(linear_fwd(h1, P[f"{p}.ff1.w"], P[f"{p}.ff1.b"])), P[f"{p}.ff2.w"], P[f"{p}.ff2.b"])
+        h, _, _ = layernorm_fwd(add(h1, f2), P[f"{p}.ln2.gamma"], P[f"{p}.ln2.beta"], eps)
+    return h
 
 
 def encoder_train_step(P, V, x, t, first, layers=6, heads=8, lr=0.01, momentum=0.9, eps=1e-5, masks=None, trace=None):

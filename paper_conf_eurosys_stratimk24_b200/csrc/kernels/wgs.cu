@@ -22,8 +22,8 @@ namespace {
 namespace wgs {
 using namespace tmah;
 
-constexpr int NCW = 8;                    // consumer warps = row groups
-constexpr int NTHR = (NCW + 1) * 32;      // + one TMA producer warp
+constexpr int NCW = 8;                    // warps = row groups; lane 0 of warp 0 also issues the TMA loads
+constexpr int NTHR = NCW * 32;            // 8 warps: two CTAs (16 warps, 4 per SM sub-partition) at <= 128 registers
 constexpr int STAGE_BUDGET = 96 * 1024;   // stage ring per CTA: two CTAs per SM
 
 struct Plan {
@@ -43,9 +43,10 @@ struct Params {
   double* gpart;   // [tile][groups][V] fp64 group sums (two-level combine)
 };
 
-// register blocks with <= 72 accumulators (two CTAs of 288 threads per SM: <= 112 registers)
+// register blocks with <= 72 accumulators; two CTAs of 256 threads per SM put 4 warps on each
+// 16 K-register sub-partition: <= 128 registers per thread
 __host__ __device__ constexpr bool blk_ok(int mi, int nb) { return mi * nb <= 72; }
-constexpr int MAXREG = 112;
+constexpr int MAXREG = 128;
 
 inline int pow2_floor(int v) {
   int p = 1;
@@ -142,8 +143,9 @@ __global__ void __maxnreg__(MAXREG) wgs_kernel(const __grid_constant__ CUtensorM
   if (tid == 0) {
     for (int s = 0; s < S; s++) { mbar_init(full0 + 8 * s, 1); mbar_init(empty0 + 8 * s, NCW); }
     fence_barrier_init();
+    prefetch_tmap(&tmL);
+    prefetch_tmap(&tmQ);
   }
-  if (warp == NCW && lane == 0) { prefetch_tmap(&tmL); prefetch_tmap(&tmQ); }
   __syncthreads();
 
   float acc[MI][NB];
@@ -152,52 +154,51 @@ __global__ void __maxnreg__(MAXREG) wgs_kernel(const __grid_constant__ CUtensorM
 #pragma unroll
     for (int j = 0; j < NB; j++) acc[i][j] = 0.f;
 
-  if (warp == NCW) {
-    if (lane == 0) {
-      const uint32_t tx = (uint32_t)stage_floats * 4;
+  // producer (lane 0 of warp 0): stage `it` goes to slot it % S once every warp released the
+  // slot's previous round (empty barrier, phase (it / S - 1) & 1)
+  const uint32_t tx = (uint32_t)stage_floats * 4;
+  auto produce = [&](int it) {
+    const int s = it % S;
+    if (it >= S) mbar_wait(empty0 + 8 * s, ((uint32_t)(it / S) & 1u) ^ 1u);
+    const uint32_t bar = full0 + 8 * s, dst = smem_u32(ring + (size_t)s * stage_floats);
+    mbar_expect(bar, tx);
+    tma_load2d(dst, &tmL, l0, k0 + it * R, bar);
+    tma_load2d(dst + (uint32_t)(R * TL * 4), &tmQ, q0, k0 + it * R, bar);
+  };
+  if (tid == 0)
+    for (int it = 0; it < S - 1 && it < nst; it++) produce(it);
 #pragma unroll 1
-      for (int it = 0; it < nst; it++) {
-        const int s = it % S;
-        if (it >= S) mbar_wait(empty0 + 8 * s, ((uint32_t)(it / S) & 1u) ^ 1u);
-        const uint32_t bar = full0 + 8 * s, dst = smem_u32(ring + (size_t)s * stage_floats);
-        mbar_expect(bar, tx);
-        tma_load2d(dst, &tmL, l0, k0 + it * R, bar);
-        tma_load2d(dst + (uint32_t)(R * TL * 4), &tmQ, q0, k0 + it * R, bar);
-      }
-    }
-  } else {
+  for (int it = 0; it < nst; it++) {
+    if (tid == 0 && it + S - 1 < nst) produce(it + S - 1);   // keeps S - 1 stages in flight
+    const int s = it % S;
+    mbar_wait(full0 + 8 * s, (uint32_t)(it / S) & 1u);
+    const float* Ls = ring + (size_t)s * stage_floats + lane;
+    const float4* Qs = reinterpret_cast<const float4*>(ring + (size_t)s * stage_floats + R * TL);
+    const int rows = min(R, k1 - (k0 + it * R));
 #pragma unroll 1
-    for (int it = 0; it < nst; it++) {
-      const int s = it % S;
-      mbar_wait(full0 + 8 * s, (uint32_t)(it / S) & 1u);
-      const float* Ls = ring + (size_t)s * stage_floats + lane;
-      const float4* Qs = reinterpret_cast<const float4*>(ring + (size_t)s * stage_floats + R * TL);
-      const int rows = min(R, k1 - (k0 + it * R));
-#pragma unroll 1
-      for (int r = warp; r < rows; r += NCW) {
-        float lv[MI];
+    for (int r = warp; r < rows; r += NCW) {
+      float lv[MI];
 #pragma unroll
-        for (int i = 0; i < MI; i++) lv[i] = Ls[r * TL + 32 * i];
+      for (int i = 0; i < MI; i++) lv[i] = Ls[r * TL + 32 * i];
 #pragma unroll
-        for (int j = 0; j < NB / 4; j++) {
-          const float4 q = Qs[r * (NB / 4) + j];
+      for (int j = 0; j < NB / 4; j++) {
+        const float4 q = Qs[r * (NB / 4) + j];
 #pragma unroll
-          for (int i = 0; i < MI; i++) {
-            acc[i][4 * j] = fmaf(lv[i], q.x, acc[i][4 * j]);
-            acc[i][4 * j + 1] = fmaf(lv[i], q.y, acc[i][4 * j + 1]);
-            acc[i][4 * j + 2] = fmaf(lv[i], q.z, acc[i][4 * j + 2]);
-            acc[i][4 * j + 3] = fmaf(lv[i], q.w, acc[i][4 * j + 3]);
-          }
+        for (int i = 0; i < MI; i++) {
+          acc[i][4 * j] = fmaf(lv[i], q.x, acc[i][4 * j]);
+          acc[i][4 * j + 1] = fmaf(lv[i], q.y, acc[i][4 * j + 1]);
+          acc[i][4 * j + 2] = fmaf(lv[i], q.z, acc[i][4 * j + 2]);
+          acc[i][4 * j + 3] = fmaf(lv[i], q.w, acc[i][4 * j + 3]);
         }
       }
-      __syncwarp();
-      if (lane == 0) mbar_arrive(empty0 + 8 * s);
     }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty0 + 8 * s);
   }
   __syncthreads();   // every stage consumed: the ring becomes the reduction area
   // row-group blocks -> shared [warp][i][j][lane], then summed in warp order (element e = (i*NB+j)*32 + lane)
   float* red = ring;
-  if (warp < NCW) {
+  {
 #pragma unroll
     for (int i = 0; i < MI; i++)
 #pragma unroll

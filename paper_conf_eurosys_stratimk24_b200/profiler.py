@@ -33,10 +33,10 @@ RIDGE_TF32X3 = TF32X3_TFLOPS * 1e12 / (HBM_GBS * 1e9)
 RIDGE_OF_PIPE = {L.PIPE_FMA: RIDGE_FFMA, L.PIPE_TF32X3: RIDGE_TF32X3, L.PIPE_BF16: RIDGE_BF16}
 
 # sm_100 per-SM limits for the closed-form occupancy (R17): threads, warps, CTAs,
-# registers (allocated per warp in units of 256), shared memory (228 KB per SM, 1 KB reserved per
-# CTA, 128-byte allocation granularity)
+# registers (64 K per SM in four 16 K sub-partitions, each warp's allocated from one of them in
+# units of 256), shared memory (228 KB per SM, 1 KB reserved per CTA, 128-byte granularity)
 SM_MAX_THREADS, SM_MAX_WARPS, SM_MAX_CTAS = 2048, 64, 32
-SM_REGS, REG_ALLOC_UNIT = 65536, 256
+SM_REGS, SM_PARTITIONS, REG_ALLOC_UNIT = 65536, 4, 256
 SM_SMEM, CTA_SMEM_RESERVED, SMEM_ALLOC_UNIT = 233472, 1024, 128
 
 
@@ -133,7 +133,8 @@ def occupancy_limits(threads, regs, smem):
     warps = -(-threads // 32)
     lim_warps = SM_MAX_WARPS // warps
     per_warp = -(-(regs * 32) // REG_ALLOC_UNIT) * REG_ALLOC_UNIT
-    lim_regs = (SM_REGS // per_warp) // warps if regs > 0 else SM_MAX_CTAS
+    warps_by_regs = (SM_REGS // SM_PARTITIONS // per_warp) * SM_PARTITIONS if regs > 0 else SM_MAX_WARPS
+    lim_regs = warps_by_regs // warps
     per_cta = -(-smem // SMEM_ALLOC_UNIT) * SMEM_ALLOC_UNIT + CTA_SMEM_RESERVED
     lim_smem = SM_SMEM // per_cta
     return {"warps": lim_warps, "registers": lim_regs, "shared_mem": lim_smem, "blocks": SM_MAX_CTAS}

@@ -381,10 +381,12 @@ def mnv2_blocks():
     return blocks
 
 
-def mnv2_spec(num_classes=1000):
+def mnv2_spec(num_classes=1000, eval_stats=False):
+    """eval_stats: seeded running statistics (inference clients, R22) instead of torch's (0, 1) start."""
     def bn(name, c):
-        return [(f"{name}.gamma", (c,), ("const", 1.0)), (f"{name}.beta", (c,), ("const", 0.0)),
-                (f"{name}.rmean", (c,), ("const", 0.0)), (f"{name}.rvar", (c,), ("const", 1.0))]
+        st = [(f"{name}.rmean", (c,), ("normal", 0.1)), (f"{name}.rvar", (c,), ("uniform", 0.5, 1.5))] if eval_stats else \
+             [(f"{name}.rmean", (c,), ("const", 0.0)), (f"{name}.rvar", (c,), ("const", 1.0))]
+        return [(f"{name}.gamma", (c,), ("const", 1.0)), (f"{name}.beta", (c,), ("const", 0.0))] + st
 
     def conv(name, cout, k, cin):
         return [(f"{name}.w", (cout, k, k, cin), ("kaiming_fan_out", cout * k * k))]
@@ -921,6 +923,100 @@ def encoder_train_graph(host_params, xs, ts, layers=6, d=512, heads=8, ffn=2048,
     g.params = P
     g.relu_in = {f"enc{i}.ff1": L_[i]["f"] for i in range(layers)}
     return g
+
+
+# ============================================================ inference clients of the inf-inf config
+def mnv2_infer_graph(host_params, batch=4, hw=224, num_classes=1000, device="cuda"):
+    """Inf-inf BE client (Table 1: MobileNetV2 inference b4): TorchVision MobileNetV2
+    in eval mode, unfused ops (conv, BN, ReLU6, add each a kernel), H2D input and D2H logits."""
+    g = Graph("mnv2_infer", device)
+    spec = mnv2_spec(num_classes, eval_stats=True)
+    P = FlatParams(g, spec, host_params, grads=False)
+    x = g.buf("x", (batch, hw, hw, 3))
+    g.memcpy(L.OP_MEMCPY_H2D, _p(x), 0, x.numel() * 4, "h2d_input")
+    cnt = [0]
+
+    def new(shape):
+        cnt[0] += 1
+        return g.buf(f"t{cnt[0]}", shape)
+
+    def cb(h, cname, bname, k, stride, dw, act):
+        w = P.p[f"{cname}.w"]
+        n, hh, ww, _ = h.shape
+        pad = k // 2
+        ho, wo = (hh + 2 * pad - k) // stride + 1, (ww + 2 * pad - k) // stride + 1
+        cout = w.shape[0]
+        z = new((n, ho, wo, cout))
+        conv_fwd(g, h, w, z, stride, pad, cname, depthwise=dw)
+        y = new(z.shape)
+        g.k("bn_eval", [_p(z), _p(y), _p(P.p[f"{bname}.gamma"]), _p(P.p[f"{bname}.beta"]), _p(P.p[f"{bname}.rmean"]),
+                        _p(P.p[f"{bname}.rvar"]), n * ho * wo, cout, EPS_BITS], bname)
+        if not act:
+            return y
+        a = new(y.shape)
+        g.k("relu6", [_p(y), _p(a), y.numel()], f"{bname}.relu6")
+        return a
+
+    h = cb(x, "features.0", "features.0.bn", 3, 2, False, True)
+    for name, cin, hid, cout, stride, expand, res in mnv2_blocks():
+        inp = h
+        if expand:
+            h = cb(h, f"{name}.expand", f"{name}.expand_bn", 1, 1, False, True)
+        h = cb(h, f"{name}.dw", f"{name}.dw_bn", 3, stride, True, True)
+        h = cb(h, f"{name}.project", f"{name}.project_bn", 1, 1, False, False)
+        if res:
+            r = new(h.shape)
+            g.k("add", [_p(h), _p(inp), _p(r), h.numel()], f"{name}.add")
+            h = r
+    h = cb(h, "features.18", "features.18.bn", 1, 1, False, True)
+    n, hh, ww, c = h.shape
+    pooled = new((n, c))
+    g.k("avgpool", [_p(h), _p(pooled), n, hh * ww, c], "avgpool")
+    logits = new((n, num_classes))
+    linear_fwd(g, pooled, P.p["classifier.w"], P.p["classifier.b"], logits, "classifier")
+    g.memcpy(L.OP_MEMCPY_D2H, 0, _p(logits), logits.numel() * 4, "d2h_logits")
+    g.out, g.x, g.params = logits, x, P
+    return g.finalize()
+
+
+def encoder_infer_graph(host_params, batch=4, seq=192, layers=6, d=512, heads=8, ffn=2048, device="cuda"):
+    """Inf-inf BE client: the "Transformer" (reading R32: post-LN encoder, 6 x d512 / 8 heads /
+    FFN 2048) inference at Table 1's batch 4, fp32, the forward op list of encoder_train_graph;
+    H2D of the input embeddings first, D2H of the last layer's output last."""
+    g = Graph("encoder_infer", device)
+    spec = encoder_spec(layers, d, ffn)
+    P = FlatParams(g, spec, host_params, grads=False)
+    rows = batch * seq
+    x = g.buf("x", (rows, d))
+    g.memcpy(L.OP_MEMCPY_H2D, _p(x), 0, x.numel() * 4, "h2d_input")
+    cnt = [0]
+
+    def new(cols):
+        cnt[0] += 1
+        return g.buf(f"t{cnt[0]}", (rows, cols))
+    eps = f32bits(1e-5)
+    mrow, rrow = g.buf("ln_mean", (rows,)), g.buf("ln_rstd", (rows,))
+    h = x
+    for i in range(layers):
+        p = f"enc{i}"
+        qkv, a, o, s1, h1, f, fa, f2, s2, h2 = new(3 * d), new(d), new(d), new(d), new(d), new(ffn), new(ffn), new(d), new(d), new(d)
+        linear_fwd(g, h, P.p[f"{p}.in.w"], P.p[f"{p}.in.b"], qkv, f"{p}.in")
+        q = qkv.data_ptr()
+        g.k("attention_f32", [q, q + 4 * d, q + 8 * d, _p(a), batch, seq, heads, d // heads, 3 * d, d], f"{p}.attn")
+        linear_fwd(g, a, P.p[f"{p}.out.w"], P.p[f"{p}.out.b"], o, f"{p}.out")
+        g.k("add", [_p(h), _p(o), _p(s1), rows * d], f"{p}.add1")
+        g.k("layernorm_f32", [_p(s1), _p(h1), _p(P.p[f"{p}.ln1.gamma"]), _p(P.p[f"{p}.ln1.beta"]), _p(mrow), _p(rrow), rows, d, eps],
+            f"{p}.ln1")
+        linear_fwd(g, h1, P.p[f"{p}.ff1.w"], P.p[f"{p}.ff1.b"], f, f"{p}.ff1")
+        g.k("relu", [_p(f), _p(fa), rows * ffn], f"{p}.relu")
+        linear_fwd(g, fa, P.p[f"{p}.ff2.w"], P.p[f"{p}.ff2.b"], f2, f"{p}.ff2")
+        g.k("add", [_p(h1), _p(f2), _p(s2), rows * d], f"{p}.add2")
+        g.k("layernorm_f32", [_p(s2), _p(h2), _p(P.p[f"{p}.ln2.gamma"]), _p(P.p[f"{p}.ln2.beta"]), _p(mrow), _p(rrow), rows, d, eps],
+            f"{p}.ln2")
+        h = h2
+    g.memcpy(L.OP_MEMCPY_D2H, 0, _p(h), h.numel() * 4, "d2h_output")
+    g.out, g.x, g.params = h, x, P
+    return g.finalize()
 
 
 # ============================================================ training as the HP client (config 4)

@@ -288,3 +288,28 @@ def test_encoder_train_step_vs_torch():
     k2 = "enc0.ff1.w"
     torch.testing.assert_close(newP[k2].double(), P[k2].double() - 0.01 * dict(mods[0].named_parameters())["linear1.weight"].grad,
                                rtol=1e-5, atol=1e-7)
+
+
+def test_encoder_infer_vs_torch():
+    """Inf-inf BE client ("Transformer" inference, R32): the encoder forward vs
+    torch.nn.TransformerEncoderLayer stack in eval mode, fp64."""
+    L_, dm, heads, ffn = 2, 32, 4, 64
+    P = si.make_params(om.encoder_spec(L_, dm, ffn))
+    x = si.normal((2, 6, dm), si.BE_SEED, sub=3)
+    y = om.encoder_infer(P, x, layers=L_, heads=heads)
+    mods = [torch.nn.TransformerEncoderLayer(dm, heads, ffn, dropout=0.0, activation="relu", batch_first=True,
+                                             norm_first=False).double().eval() for _ in range(L_)]
+    names = {"in.w": "self_attn.in_proj_weight", "in.b": "self_attn.in_proj_bias", "out.w": "self_attn.out_proj.weight",
+             "out.b": "self_attn.out_proj.bias", "ln1.gamma": "norm1.weight", "ln1.beta": "norm1.bias",
+             "ff1.w": "linear1.weight", "ff1.b": "linear1.bias", "ff2.w": "linear2.weight", "ff2.b": "linear2.bias",
+             "ln2.gamma": "norm2.weight", "ln2.beta": "norm2.bias"}
+    for i, m in enumerate(mods):
+        sd = m.state_dict()
+        for k2, tk in names.items():
+            sd[tk] = P[f"enc{i}.{k2}"].double()
+        m.load_state_dict(sd)
+    h = x.double()
+    with torch.no_grad():
+        for m in mods:
+            h = m(h)
+    assert float((y.double() - h.reshape(-1, dm)).norm() / h.norm()) < 1e-5

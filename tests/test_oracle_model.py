@@ -343,3 +343,28 @@ def test_abs_sum_scales():
     Ag, Ab = om.bn_bwd_abs(z, dyb, mean, invstd)
     assert bool((Ag >= dgam.double().abs() - 1e-6).all()) and bool((Ab >= dbet.double().abs() - 1e-6).all())
     assert torch.allclose(om.bn_bwd_abs(z, dyb.abs(), mean, invstd)[1], om.bn_bwd(z, dyb.abs(), torch.ones(4), mean, invstd)[2].double(), rtol=1e-6)
+
+
+def test_mnv2_infer_vs_torchvision():
+    """Inf-inf BE client: MobileNetV2 inference with seeded eval statistics vs torchvision, fp64."""
+    tv = pytest.importorskip("torchvision")
+    P = si.make_params(om.mnv2_spec(num_classes=10, eval_stats=True))
+    m = tv.models.mobilenet_v2(num_classes=10).double().eval()
+    _to_tv(P, m, _mn_rename)
+    x = si.normal((2, 64, 64, 3), 3)
+    y = om.mnv2_infer(P, x)
+    with torch.no_grad():
+        ref = m(x.double().permute(0, 3, 1, 2))
+    assert float((y.double() - ref).norm() / ref.norm()) < 1e-5
+
+
+def test_resnet101_infer_vs_torchvision():
+    tv = pytest.importorskip("torchvision")
+    P = si.make_params(om.resnet_spec(om.RESNET101_LAYERS))
+    m = tv.models.resnet101().double().eval()
+    _to_tv(P, m, _rn_rename)
+    x = si.normal((1, 64, 64, 3), 4)
+    y = om.resnet_infer(P, x, om.RESNET101_LAYERS)
+    with torch.no_grad():
+        ref = m(x.double().permute(0, 3, 1, 2))
+    assert float((y.double() - ref).norm() / ref.norm()) < 1e-5

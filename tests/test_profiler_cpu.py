@@ -65,5 +65,10 @@ def test_occupancy_granularities():
     # shared memory: 128-byte granularity + 1 KB reserved per CTA; 227 KB is one CTA per SM
     assert PR.occupancy_limits(128, 32, 227 * 1024)["shared_mem"] == 1
     assert PR.occupancy_limits(128, 32, 100 * 1024 + 1)["shared_mem"] == 2
+    # registers come from four 16 K sub-partitions: 9 warps of 112 registers (3584 per warp) fit 4
+    # warps per partition = 16 per SM -> one 288-thread CTA, not the two 64 K / (9 x 3584) suggests
+    # (measured: cudaOccupancyMaxActiveBlocksPerMultiprocessor = 1 for wgs_kernel at 109 registers)
+    assert PR.occupancy_limits(288, 109, 98 * 1024)["registers"] == 1
+    assert PR.occupancy_limits(256, 119, 98 * 1024)["registers"] == 2
     # a kernel that needs more SMs than the GPU has is never admitted beside the HP (L27, R5)
-    assert PR.sm_needed_closed_form(296, 288, 112, 97 * 1024) == 148
+    assert PR.sm_needed_closed_form(296, 256, 119, 97 * 1024) == 148

@@ -18,6 +18,23 @@ def test_specs_match_oracle():
     assert W.resnet_train_spec() == om.resnet_train_spec()
     assert W.resnet_train_spec(W.RESNET101_LAYERS) == om.resnet_train_spec(om.RESNET101_LAYERS)
     assert W.encoder_spec(2) == om.encoder_spec(2)
+    assert W.mnv2_spec(eval_stats=True) == om.mnv2_spec(eval_stats=True)
+    assert W.resnet_spec(W.RESNET101_LAYERS) == om.resnet_spec(om.RESNET101_LAYERS)
+    assert W.bert_spec(layers=2, hidden=1024, heads=16, ffn=4096) == om.bert_spec(layers=2, hidden=1024, heads=16, ffn=4096)
+
+
+def test_infinf_client_graphs():
+    """Inf-inf BE inference clients: H2D input first, D2H output last, every kernel op well formed."""
+    g = W.mnv2_infer_graph(si.make_params(W.mnv2_spec(10, eval_stats=True)), batch=1, hw=32, num_classes=10, device="cpu")
+    _check(g)
+    kern = [o for o in g.ops if isinstance(o[0], str)]
+    assert g.ops[0][2] == "h2d_input" and g.ops[-1][2] == "d2h_logits"
+    assert sum(1 for o in kern if o[0] == "bn_eval") == 52 and sum(1 for o in kern if o[0] == "dw_fwd") == 17
+    assert sum(1 for o in kern if o[0] == "add") == 10
+    e = W.encoder_infer_graph(si.make_params(W.encoder_spec(2)), batch=1, seq=32, layers=2, device="cpu")
+    _check(e)
+    assert [o[0] for o in e.ops if isinstance(o[0], str)].count("attention_f32") == 2
+    assert e.ops[0][2] == "h2d_input" and e.ops[-1][2] == "d2h_output"
 
 
 NARGS = {"gemm": 13, "colsum": 4, "relu": 3, "relu_bwd": 4, "relu6": 3, "relu6_bwd": 4, "add": 4, "mse": 6, "sgd": 6,
