@@ -80,6 +80,41 @@ def build_config(name, rank, be_sub=0):
                      "image": "224x224x3 NHWC fp32", "arrivals": "poisson 15 rps (PAPER Table 3)"})
 
 
+# Inf-inf (Fig. 13; Table 3 "Inf-Inf Poisson" rates, Table 1 inference batch sizes):
+# HP ResNet-50 b4 beside four BE inference clients, all open-loop Poisson.
+INFINF = [  # (name, rps, builder)
+    ("resnet50", 50.0), ("mobilenet_v2", 65.0), ("resnet101", 25.0), ("bert_large", 5.0), ("transformer", 12.0)]
+
+
+def build_infinf_client(name, n_inputs=16, seed_sub=0):
+    """(graph, host inputs, host params, output view fn) of one inf-inf client (reading R34,
+    DESIGN.md §3). The GPU tests compute the oracle's outputs from the same params and inputs."""
+    from paper_conf_eurosys_stratimk24_b200 import workloads as W
+    from synth import inputs as si
+    if name in ("resnet50", "resnet101"):
+        layers = W.RESNET50_LAYERS if name == "resnet50" else W.RESNET101_LAYERS
+        P = si.make_params(W.resnet_spec(layers))
+        g = W.resnet_infer_graph(P, batch=4, layers=layers)
+        xs = [si.normal((4, 224, 224, 3), si.HP_SEED, sub=seed_sub + r) for r in range(n_inputs)]
+        return g, xs, P, (lambda t: t.view(4, 1000))
+    if name == "mobilenet_v2":
+        P = si.make_params(W.mnv2_spec(eval_stats=True))
+        g = W.mnv2_infer_graph(P, batch=4)
+        xs = [si.normal((4, 224, 224, 3), si.HP_SEED, sub=seed_sub + 100 + r) for r in range(n_inputs)]
+        return g, xs, P, (lambda t: t.view(4, 1000))
+    if name == "bert_large":
+        P = si.make_params(W.bert_spec(layers=24, hidden=1024, heads=16, ffn=4096))
+        g = W.bert_infer_graph(P, batch=2, seq=128, layers=24, heads=16, hidden=1024, ffn=4096)
+        ids = [si.token_ids((2, 128), 30522, si.HP_SEED, sub=seed_sub + 200 + r) for r in range(n_inputs)]
+        return g, [t.reshape(-1).view(torch.float32) for t in ids], P, (lambda t: t.view(torch.bfloat16).view(2, 128, 1024))
+    if name == "transformer":
+        P = si.make_params(W.encoder_spec(6))
+        g = W.encoder_infer_graph(P, batch=4, seq=192)
+        xs = [si.normal((4, 192, 512), si.HP_SEED, sub=seed_sub + 300 + r) for r in range(n_inputs)]
+        return g, xs, P, (lambda t: t.view(4 * 192, 512))
+    raise ValueError(name)
+
+
 def build_client(name, client):
     """One client's graph only (the offline profiler's solo runner)."""
     from paper_conf_eurosys_stratimk24_b200 import workloads as W
@@ -225,7 +260,7 @@ def main():
     ap.add_argument("--steps", type=int, default=20, help="timed steps (REQ_PER_STEP HP requests each, per mode and rate)")
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", default="orion", choices=["orion", "reference"])
-    ap.add_argument("--config", default="rn50_mnv2", choices=["rn50_mnv2", "toy", "bert_rn50", "rn101_enc"])
+    ap.add_argument("--config", default="rn50_mnv2", choices=["rn50_mnv2", "toy", "bert_rn50", "rn101_enc", "infinf"])
     ap.add_argument("--dur-ppm", type=int, default=25000)
     ap.add_argument("--be-partition", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
@@ -263,6 +298,8 @@ def main():
 
     if args.config == "rn101_enc":
         return train_train(args, rank, world, local, metric)
+    if args.config == "infinf":
+        return infer_infer(args, rank, world, local, metric)
     return infer_train(args, rank, world, local, metric)
 
 
@@ -542,6 +579,92 @@ def infer_train(args, rank, world, local, metric):
         "scheduler": stats,
         "utilisation": util,
     }
+    print(json.dumps(line), flush=True)
+
+
+def infer_infer(args, rank, world, local, metric):
+    """Inf-inf (Fig. 13): HP ResNet-50 b4 with four BE inference
+    clients (MobileNetV2 b4, ResNet-101 b4, BERT-large b2 bf16, Transformer encoder b4), all open-loop
+    Poisson at Table 3's Inf-Inf rates (reading R34). Per repeat: every client alone on its trace
+    (dedicated), then all five together (collocated, timed); three repeats interleaved. Reports every
+    client's p50 / p99 vs dedicated with bootstrap CIs; value = BE requests/s served collocated."""
+    from paper_conf_eurosys_stratimk24_b200 import collocate as C, profiler as PR, _lib as L, placement as PL
+    from paper_conf_eurosys_stratimk24_b200 import replicas as RP
+    from synth import inputs as si
+    n_hp = max(1, args.steps) * REQ_PER_STEP
+    per_rep = -(-n_hp // REPEATS)
+    dur_s = per_rep / INFINF[0][1]
+    clients = []
+    for j, (name, rps) in enumerate(INFINF):
+        g, xs, _, _ = build_infinf_client(name, n_inputs=8)
+        prof, rows = PR.build_profiles(g, 10000 * j, reps=3)
+        n_j = max(4, int(round(rps * dur_s)))
+        clients.append(dict(name=name, rps=rps, n=n_j, rows=rows, c=C.HPClient(g, xs, n_j, prof, 10000 * j)))
+    cores, note = PL.for_this_process(local, int(os.environ.get("LOCAL_WORLD_SIZE", world)), 1 + len(INFINF))
+    sched_cpu, hp_cpu, be_cpus = cores[0], cores[1], cores[2:]
+    pol = L.POLICIES[args.policy]
+
+    def session(**kw):
+        return C.run_inference_session(sched_cpu=sched_cpu, device=local, flags=pol, hp_cpu=hp_cpu, be_cpus=be_cpus, **kw)
+    hp = clients[0]
+    spaced = (np.arange(1, 101) * 10e6).astype(np.int64)
+    session(hp=hp["c"], hp_arrivals=spaced[:10])
+    r0 = session(hp=hp["c"], hp_arrivals=spaced)
+    hp_lat_ns = int(np.median(r0["hp"][1] - r0["hp"][0]))
+    lat = {cl["name"]: {"ded": [], "col": []} for cl in clients}
+    win_ms, be_done, be_time = 0.0, 0, 0.0
+    with ClockSampler(local) as clk:
+        for rep in range(REPEATS):
+            arr = [si.poisson_arrivals_ns(cl["rps"], cl["n"], seed=si.ARRIVAL_SEED + 17 * rep + j, gpu_index=rank)
+                   for j, cl in enumerate(clients)]
+            for j, cl in enumerate(clients):          # dedicated: each client alone on its own trace
+                r = session(hp=cl["c"], hp_arrivals=arr[j]) if j == 0 else session(bes=[cl["c"]], be_arrivals=[arr[j]])
+                ta, td = r["hp"] if j == 0 else r["be"][0]
+                lat[cl["name"]]["ded"] += (td - ta).tolist()
+            RP.barrier()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            rc = session(hp=hp["c"], hp_arrivals=arr[0], bes=[cl["c"] for cl in clients[1:]], be_arrivals=arr[1:],
+                         hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm)
+            e1.record()
+            torch.cuda.synchronize()
+            RP.barrier()
+            win_ms += e0.elapsed_time(e1)
+            ta, td = rc["hp"]
+            lat[hp["name"]]["col"] += (td - ta).tolist()
+            for j, cl in enumerate(clients[1:]):
+                ta, td = rc["be"][j]
+                lat[cl["name"]]["col"] += (td - ta).tolist()
+                be_done += len(td)
+            be_time += (rc["t1"] - rc["t0"]) / 1e9
+            stats = rc["stats"]
+    per_client = {}
+    for cl in clients:
+        d, c = lat[cl["name"]]["ded"], lat[cl["name"]]["col"]
+        per_client[cl["name"]] = {
+            "role": "HP" if cl is hp else "BE", "rate_rps": cl["rps"], "requests": len(c),
+            "p50_ms": pct(c, 50) / 1e6, "p99_ms": pct(c, 99) / 1e6, "dedicated_p50_ms": pct(d, 50) / 1e6,
+            "dedicated_p99_ms": pct(d, 99) / 1e6, "p99_vs_dedicated": pct(c, 99) / pct(d, 99),
+            "p99_ratio_ci95": bootstrap_ratio_ci(c, d)}
+    value = be_done / max(be_time, 1e-9)
+    allr = RP.gather(dict(value=value, win_ms=win_ms, hp=per_client[hp["name"]]["p99_vs_dedicated"]))
+    if rank != 0:
+        return
+    line = {"metric": metric, "value": sum(r["value"] for r in allr), "unit": "req/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": max(r["win_ms"] for r in allr) / max(args.steps, 1), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f32 + bf16 (BERT)", "data": "synthetic (seeded; DESIGN.md §5)",
+            "config": {"workload": "inf-inf: HP ResNet-50 b4 + BE MobileNetV2 b4, ResNet-101 b4, BERT-large b2 s128 (bf16), "
+                                   "Transformer encoder b4 s192, all Poisson (Table 3 Inf-Inf rates), 1 B200 per instance",
+                       "parallelism": f"replicas x{world}", "policy": args.policy, "dur_threshold_pct": args.dur_ppm / 1e4,
+                       "hp_solo_latency_ms": hp_lat_ns / 1e6, "repeats": REPEATS,
+                       "host_cores": {"scheduler": sched_cpu, "hp_driver": hp_cpu, "be_drivers": be_cpus, "note": note}},
+            "clients": per_client, "hp": per_client[hp["name"]],
+            "be": {"requests_per_s": value, "unit": "BE requests completed per second in the collocated windows"},
+            "target": {"paper": "HP p99 within 9% of ideal on A100 with 4 BE inference clients (P:1305-1308)"},
+            "roofline": None, "cpu_baseline": None, "e2e": None,
+            "gpu_launches": int(sum(len(lat[cl["name"]]["col"]) * sum(1 for o in cl["c"].ops if o.kind == L.OP_KERNEL) for cl in clients)),
+            "clocks": clk.summary(), "scheduler": stats}
     print(json.dumps(line), flush=True)
 
 

@@ -165,6 +165,7 @@ typedef struct {
   int32_t dynamic_smem;      /* dynamic shared memory per CTA of this launch */
   int32_t blocks_per_sm;     /* cudaOccupancyMaxActiveBlocksPerMultiprocessor */
   int32_t pipe;              /* enum orion_pipe */
+  char kernel[120];          /* the kernel the op launches (mangled device-function name, truncated) */
 } orion_kernel_info_t;
 int orion_kernel_info(uint32_t fn, const uint64_t* args, uint32_t nargs, orion_kernel_info_t* out);
 /* Workspace sizes (bytes) of the ops that split their reductions. Workspaces must be zeroed once

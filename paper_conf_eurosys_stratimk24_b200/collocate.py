@@ -171,3 +171,65 @@ def be_throughput(res, t_from=None, t_to=None):
     t_to = res["t1"] if t_to is None else t_to
     n = int(((t >= t_from) & (t <= t_to)).sum())
     return n / ((t_to - t_from) / 1e9), n
+
+
+def run_inference_session(hp=None, hp_arrivals=None, bes=(), be_arrivals=(), log_capacity=0, hp_latency_ns=0,
+                          dur_threshold_ppm=25000, sm_threshold=0, be_partition_sms=0, flags=0, sched_cpu=-1,
+                          backend=L.BACKEND_CUDA, device=0, hp_cpu=None, be_cpus=None):
+    """Inf-inf session (Fig. 13): one HP and several BE *inference* clients, every one
+    open loop with its own arrival trace, each driven by orion_run_requests on its own thread
+    (BE requests go through Listing 1's BE path like any BE op; R11 rotates the BE clients). Any
+    client may be absent (the dedicated runs). Returns {"hp": (t_arrival, t_done) or None,
+    "be": [(t_arrival, t_done), ...], "t0", "t1", "stats", "log"}."""
+    o = Orion(device=device, backend=backend, hp_latency_ns=hp_latency_ns, dur_threshold_ppm=dur_threshold_ppm,
+              sm_threshold=sm_threshold, be_partition_sms=be_partition_sms, flags=flags, sched_cpu=sched_cpu,
+              log_capacity=log_capacity)
+    try:
+        hp_id = o.register_client(L.HP) if hp is not None else None
+        be_ids = [o.register_client(L.BE) for _ in bes]
+        torch.cuda.synchronize()
+        o.start()
+    except BaseException:
+        o.destroy()
+        raise
+    res = {"hp": None, "be": [None] * len(bes)}
+    errs = []
+
+    def be_main(j):
+        if be_cpus:
+            os.sched_setaffinity(0, {be_cpus[j % len(be_cpus)]})
+        try:
+            c = bes[j]
+            res["be"][j] = o.run_requests(be_ids[j], c.ops, be_arrivals[j], in_cycle=c.inp.shape[0], out_cycle=c.n_req)
+        except Exception as e:   # surfaced below
+            errs.append(e)
+    ths = [threading.Thread(target=be_main, args=(j,)) for j in range(len(bes))]
+    res["t0"] = L.lib.orion_now_ns()
+    for th in ths:
+        th.start()
+    prev_mask = os.sched_getaffinity(0) if hp_cpu is not None else None
+    try:
+        if hp is not None:
+            if hp_cpu is not None:
+                os.sched_setaffinity(0, {hp_cpu})
+            res["hp"] = o.run_requests(hp_id, hp.ops, hp_arrivals, in_cycle=hp.inp.shape[0], out_cycle=hp.n_req)
+    except BaseException as e:
+        errs.append(e)
+    finally:
+        if prev_mask is not None:
+            os.sched_setaffinity(0, prev_mask)
+        for th in ths:          # BE request streams are finite: they end on their own
+            th.join()
+    res["t1"] = L.lib.orion_now_ns()
+    try:
+        o.stop()
+    except Exception as e:
+        errs.append(e)
+    if errs:
+        o.destroy()
+        raise errs[0]
+    res["stats"] = o.stats()
+    if log_capacity:
+        res["log"] = o.read_log()
+    o.destroy()
+    return res

@@ -107,6 +107,15 @@ int orion_kernel_info(uint32_t fn, const uint64_t* args, uint32_t nargs, orion_k
     return ORION_E_CUDA;
   }
   out->blocks_per_sm = b;
+  const char* nm = nullptr;
+  out->kernel[0] = 0;
+  if (cudaFuncGetName(&nm, g.func) == cudaSuccess && nm) {
+    size_t i = 0;
+    for (; nm[i] && i + 1 < sizeof(out->kernel); i++) out->kernel[i] = nm[i];
+    out->kernel[i] = 0;
+  } else {
+    (void)cudaGetLastError();
+  }
   return 0;
 }
 

@@ -71,6 +71,19 @@ inline int smem_bytes(int mi, int nb, int R, int stages) {
 // Shape-only plan (never the SM count of the partition): pick the operand roles and register
 // block by a three-term time model (FFMA issue, HBM bytes, L2 re-reads), then split K so that about
 // two CTAs per SM of a 148-SM B200 stream, keeping the partial-tile traffic small.
+inline int split_for(long long M, long long N, long long K, int tiles, int R, int mi, int nb) {
+  // at most one wave of two CTAs per SM (a 148-SM B200 constant, not the partition's count)
+  long long split = tiles >= 296 ? 1 : 296 / tiles;
+  const long long kmax = K / (2LL * R);   // >= 2 stages per split
+  if (split > kmax) split = kmax > 0 ? kmax : 1;
+  // partial tiles (written once, read once) within ~25 % of the operand bytes
+  const long long V = 32LL * mi * nb;
+  const long long pmax = (4 * K * (M + N)) / (32 * tiles * V);
+  if (split > pmax) split = pmax > 0 ? pmax : 1;
+  if (split > 1024) split = 1024;
+  return (int)split;
+}
+
 inline Plan plan(long long M, long long N, long long K) {
   static const int MIS[3] = {1, 2, 3};
   static const int NBS[5] = {8, 16, 24, 32, 4};
@@ -82,9 +95,14 @@ inline Plan plan(long long M, long long N, long long K) {
       for (int nb : NBS) {
         if (!blk_ok(mi, nb)) continue;
         const long long tl = cdiv(DL, 32 * mi), tq = cdiv(DQ, nb), tiles = tl * tq;
+        if (tiles > (1 << 20)) continue;
+        const int R = stage_rows(32 * mi + nb);
+        const long long split = split_for(M, N, K, (int)tiles, R, mi, nb);
+        const long long ctas = tiles * split, waves = cdiv(ctas, 296);
+        const double eff = (double)ctas / (double)(waves * 296);   // fraction of the CTA slots kept busy
         const double issue = (double)tiles * (mi * nb + mi + nb / 4 + 3);   // warp instructions per row
-        const double t_fma = (double)K * issue / (148.0 * 4 * 1.9e9);
-        const double t_hbm = 4.0 * K * (M + N) / 6.5e12;
+        const double t_fma = (double)K * issue / (148.0 * 4 * 1.9e9) / eff;
+        const double t_hbm = 4.0 * K * (M + N) / 6.5e12 / (eff < 0.5 ? 2 * eff : 1.0);
         const double t_l2 = 4.0 * K * tiles * (32 * mi + nb) / 20e12;
         double cost = t_fma > t_hbm ? t_fma : t_hbm;
         if (t_l2 > cost) cost = t_l2;
@@ -92,25 +110,15 @@ inline Plan plan(long long M, long long N, long long K) {
         if (cost < best_cost) {
           best_cost = cost;
           best.trans = trans; best.mi = mi; best.nb = nb; best.tiles_l = (int)tl; best.tiles_q = (int)tq;
+          best.R = R; best.split = (int)split;
         }
       }
   }
-  const int tiles = best.tiles_l * best.tiles_q;
   const int rowf = 32 * best.mi + best.nb;
-  best.R = stage_rows(rowf);
   best.stages = STAGE_BUDGET / (best.R * rowf * 4);
   if (best.stages > 8) best.stages = 8;
   if (best.stages < 2) best.stages = 2;
-  long long split = (296 + tiles / 2) / tiles;
-  if (split < 1) split = 1;
-  const long long kmax = K / (2LL * best.R);   // >= 2 stages per split
-  if (split > kmax) split = kmax > 0 ? kmax : 1;
-  // partial tiles (written once, read once) within ~25 % of the operand bytes
-  const long long V = 32LL * best.mi * best.nb;
-  const long long pmax = (4 * K * (M + N)) / (32 * tiles * V);
-  if (split > pmax) split = pmax > 0 ? pmax : 1;
-  if (split > 1024) split = 1024;
-  long long kps = cdiv(cdiv(K, split), best.R) * best.R;
+  long long kps = cdiv(cdiv(K, best.split), best.R) * best.R;
   best.kps = (int)kps;
   best.split = (int)cdiv(K, kps);
   best.smem = smem_bytes(best.mi, best.nb, best.R, best.stages);

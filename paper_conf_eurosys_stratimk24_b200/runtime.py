@@ -190,4 +190,6 @@ def kernel_info(fn, args):
     info = L.KernelInfo()
     check(L.lib.orion_kernel_info(L.FN[fn] if isinstance(fn, str) else fn, a, len(args), ctypes.byref(info)),
           f"kernel_info({fn})")
-    return {k: getattr(info, k) for k, _ in info._fields_}
+    d = {k: getattr(info, k) for k, _ in info._fields_}
+    d["kernel"] = d["kernel"].decode(errors="replace")
+    return d

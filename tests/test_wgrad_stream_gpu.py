@@ -10,8 +10,8 @@ Checks per case:
     length-K fp32 dot product (u = 2^-24), which the kernel's partial sums (fp32 row groups of
     <= K terms, fp64 split combine) satisfy; it catches a localized tile / tail error that a
     per-tensor norm would average away;
-  * the streaming kernel really ran (288-thread CTAs from orion_kernel_geometry), and a second
-    launch reproduces the bytes (fixed reduction order)."""
+  * the streaming kernel really ran (orion_kernel_info names wgs_kernel), and a second launch
+    reproduces the bytes (fixed reduction order)."""
 import math
 
 import pytest
@@ -25,7 +25,7 @@ pytestmark = pytest.mark.gpu
 if torch.cuda.is_available():
     import paper_conf_eurosys_stratimk24_b200 as orion
     from paper_conf_eurosys_stratimk24_b200 import _lib as L
-    from paper_conf_eurosys_stratimk24_b200.runtime import kernel_geometry
+    from paper_conf_eurosys_stratimk24_b200.runtime import kernel_info
 
 U = 2.0 ** -24
 
@@ -44,8 +44,8 @@ def check_wgrad(M, N, K, seed=31, expect_stream=True):
     w = torch.zeros(int(nws) // 4 + 64, dtype=torch.float32, device="cuda")
     Ad, Bd = A.cuda(), B.cuda()
     args = [Ad.data_ptr(), Bd.data_ptr(), C.data_ptr(), 0, M, N, K, M, N, N, 1, w.data_ptr(), w.numel() * 4]
-    _, _, threads, _ = kernel_geometry("gemm", args)
-    assert (threads == 288) == expect_stream, f"kernel selection: {threads} threads"
+    kern = kernel_info("gemm", args)["kernel"]
+    assert ("wgs_kernel" in kern) == expect_stream, f"kernel selection: {kern}"
     s = torch.cuda.current_stream().cuda_stream
     orion.kernel_launch("gemm", args, s)
     torch.cuda.synchronize()
