@@ -51,18 +51,24 @@ def assert_close(name, got, ref, rel_tol, elem_factor=ELEM_FACTOR, floor=1e-30):
     return r, e
 
 
-def audit_decisions(name, y_gpu, y_oracle, thresholds=(0.0, 6.0), tau=1e-4):
+def audit_decisions(name, y_gpu, y_oracle, thresholds=(0.0, 6.0), rel_tol=1e-4, elem_factor=ELEM_FACTOR,
+                    max_flip_frac=1e-4):
     """The GPU's ReLU6 (thresholds 0, 6) or ReLU (0) decided on y_gpu; the oracle's own free-running
     forward produced y_oracle. Checks:
-      * elementwise forward agreement |y_gpu - y_oracle| <= delta = tau * rms(y_oracle);
+      * the forward values agree like any compared tensor: rel L2 <= rel_tol and max |err| <= delta =
+        elem_factor x rel_tol x rms(y_oracle) (the free-running fp32 forward drifts from the fp64
+        oracle through the layers before it; rounding, not a wrong value, must explain the gap);
       * every element where the two take different decisions has its oracle value within delta of
-        a threshold (so the flip is decided by rounding, not by a wrong value);
+        a threshold, and such flips are rare (<= max_flip_frac of the elements): a systematic error
+        would flip many decisions far from the thresholds.
     Returns (flips, delta)."""
     g, o = _dd(y_gpu).reshape(-1), _dd(y_oracle).reshape(-1)
     rms = float(o.norm()) / math.sqrt(max(o.numel(), 1))
-    delta = tau * rms
+    delta = elem_factor * rel_tol * rms
+    r = float((g - o).norm() / max(float(o.norm()), 1e-30))
+    assert r <= rel_tol, f"{name}: forward rel L2 {r:.3e} > {rel_tol:g}"
     err = float((g - o).abs().max())
-    assert err <= delta, f"{name}: forward max |err| {err:.3e} > delta {delta:.3e} (tau {tau:g} x rms)"
+    assert err <= delta, f"{name}: forward max |err| {err:.3e} > delta {delta:.3e}"
     lo = thresholds[0]
     if len(thresholds) == 2:
         hi = thresholds[1]
@@ -76,6 +82,7 @@ def audit_decisions(name, y_gpu, y_oracle, thresholds=(0.0, 6.0), tau=1e-4):
     if nflip:
         worst = float(near[flip].max())
         assert worst <= delta, f"{name}: decision flip at an oracle value {worst:.3e} from a threshold (delta {delta:.3e})"
+        assert nflip <= max(1, max_flip_frac * o.numel()), f"{name}: {nflip} decision flips of {o.numel()}"
     return nflip, delta
 
 
@@ -88,8 +95,8 @@ def check_train_iterations(run_one, graph, step, xs, labels, P0, K, dec_attr, th
     dec_attr: the graph's dict of the values its ReLU / ReLU6 backward decided on (name -> tensor);
     the oracle's trace key of the same values is "bn_out" or "relu_in"; names with a suffix in
     audit_skip feed no activation and are not audited.
-    Per iteration: decisions audited (forward elementwise within 1e-4 x rms, flips only inside that
-    band); loss rel 1e-5; every gradient element within tau_g of its absolute-term sum, every
+    Per iteration: decisions audited (forward rel L2 1e-4 and elementwise 1e-3 x rms, flips only
+    inside that band and rare); loss rel 1e-5; every gradient element within tau_g of its absolute-term sum, every
     gradient tensor within tau_g x max(1, kappa) in rel L2. After K: momentum (accumulated sums)
     and parameters (K ulps of storage rounding per side + lr x the accumulated bound); BN running
     statistics rel 1e-5 (rmean with an absolute floor of 1e-2: block outputs have exactly zero
