@@ -600,7 +600,8 @@ int orion_run_iterations(orion_t h, int client_id, const orion_op* ops, uint32_t
   if (n_variants == 0) n_variants = 1;
   Client* c = h->clients[client_id].get();
   uint64_t it = 0;
-  while ((max_iters == 0 || it < max_iters) && !(stop && *stop)) {
+  // the stop flag is written by another thread (the controller): an atomic acquire load, not a plain read
+  while ((max_iters == 0 || it < max_iters) && !(stop && __atomic_load_n(stop, __ATOMIC_ACQUIRE))) {
     const orion_op* v = ops + (size_t)(it % n_variants) * n_ops;
     for (uint32_t i = 0; i < n_ops; i++) {
       int rc;
