@@ -83,13 +83,47 @@ __global__ void __launch_bounds__(EW_THREADS) sgd_kernel(float* __restrict__ p, 
   orion_signal(sig);
 }
 
-// ---- column sum (bias gradient): out[n] = sum_m A[m][n], sequential in m
+// ---- column sum (bias gradient): out[n] = sum_m A[m][n]. A CTA owns CS_COLS columns (8 column
+// quads, 128-bit loads when N % 4 == 0) and all M rows, split over 32 row lanes: lane l sums rows
+// l, l + 32, ... in fp32 (8 loads in flight), the lanes are added in lane order in fp64. One pass
+// over A with N / CS_COLS CTAs (the round-1 thread-per-column loop ran 6 CTAs at ~56 GB/s);
+// fixed order, no workspace, deterministic.
+constexpr int CS_QUADS = 8, CS_LANES = EW_THREADS / CS_QUADS, CS_COLS = 4 * CS_QUADS;
 __global__ void __launch_bounds__(EW_THREADS) colsum_kernel(const float* __restrict__ A, float* __restrict__ out, int M, int N, OrionSig sig) {
-  int n = blockIdx.x * blockDim.x + threadIdx.x;
+  __shared__ float4 part[CS_LANES][CS_QUADS];
+  const int q = threadIdx.x % CS_QUADS, lane = threadIdx.x / CS_QUADS;
+  const int n = blockIdx.x * CS_COLS + 4 * q;
+  float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
   if (n < N) {
-    float s = 0.f;
-    for (int m = 0; m < M; m++) s += __ldg(A + (long long)m * N + n);
-    out[n] = s;
+    const bool vec = (N % 4 == 0);
+    auto ld = [&](long long m) -> float4 {
+      const float* p = A + m * N + n;
+      if (vec) return __ldg(reinterpret_cast<const float4*>(p));
+      return make_float4(__ldg(p), n + 1 < N ? __ldg(p + 1) : 0.f, n + 2 < N ? __ldg(p + 2) : 0.f, n + 3 < N ? __ldg(p + 3) : 0.f);
+    };
+    int m = lane;
+    for (; m + 7 * CS_LANES < M; m += 8 * CS_LANES) {
+      float4 v[8];
+#pragma unroll
+      for (int i = 0; i < 8; i++) v[i] = ld(m + (long long)i * CS_LANES);
+#pragma unroll
+      for (int i = 0; i < 8; i++) { s.x += v[i].x; s.y += v[i].y; s.z += v[i].z; s.w += v[i].w; }
+    }
+    for (; m < M; m += CS_LANES) {
+      const float4 v = ld(m);
+      s.x += v.x; s.y += v.y; s.z += v.z; s.w += v.w;
+    }
+  }
+  part[lane][q] = s;
+  __syncthreads();
+  if (threadIdx.x < CS_COLS) {
+    const int qq = threadIdx.x / 4, j = threadIdx.x % 4, col = blockIdx.x * CS_COLS + threadIdx.x;
+    double t = 0.0;
+    for (int l = 0; l < CS_LANES; l++) {
+      const float4 v = part[l][qq];
+      t += (double)(j == 0 ? v.x : j == 1 ? v.y : j == 2 ? v.z : v.w);
+    }
+    if (col < N) out[col] = (float)t;
   }
   orion_signal(sig);
 }
@@ -283,7 +317,7 @@ int sgd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_
 
 // ---- colsum: args A, out, M, N
 int colsum_geom(const uint64_t* a, LaunchGeom* g) {
-  g->grid = dim3((unsigned)cdiv(a[3], EW_THREADS)); g->block = dim3(EW_THREADS); g->smem = 0; g->func = (const void*)colsum_kernel;
+  g->grid = dim3((unsigned)cdiv(a[3], CS_COLS)); g->block = dim3(EW_THREADS); g->smem = 0; g->func = (const void*)colsum_kernel;
   return 0;
 }
 int colsum_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {

@@ -55,7 +55,7 @@ inline int pow2_floor(int v) {
 }
 
 inline int stage_rows(int rowf) {
-  int r = pow2_floor(32768 / (rowf * 4));
+  int r = pow2_floor(16384 / (rowf * 4));   // ~16 KB stages: many small stages keep more loads in flight
   return r < 32 ? 32 : (r > 256 ? 256 : r);
 }
 
@@ -150,6 +150,7 @@ __global__ void __maxnreg__(MAXREG) wgs_kernel(const __grid_constant__ CUtensorM
 
   if (tid == 0) {
     for (int s = 0; s < S; s++) { mbar_init(full0 + 8 * s, 1); mbar_init(empty0 + 8 * s, NCW); }
+    // (released[] below is zeroed before the first arrival)
     fence_barrier_init();
     prefetch_tmap(&tmL);
     prefetch_tmap(&tmQ);
@@ -162,22 +163,25 @@ __global__ void __maxnreg__(MAXREG) wgs_kernel(const __grid_constant__ CUtensorM
 #pragma unroll
     for (int j = 0; j < NB; j++) acc[i][j] = 0.f;
 
-  // producer (lane 0 of warp 0): stage `it` goes to slot it % S once every warp released the
-  // slot's previous round (empty barrier, phase (it / S - 1) & 1)
+  // producer: the slot of stage `it` is refilled with stage it + S by the warp that releases it last
+  // (a per-slot arrival count in shared memory), so all S slots are in flight and no warp waits for
+  // another to issue loads. Stage `it` lands in slot it % S; its full barrier completes phase
+  // (it / S) & 1.
+  __shared__ unsigned int released[8];
+  if (tid < 8) released[tid] = 0u;
+  __syncthreads();
   const uint32_t tx = (uint32_t)stage_floats * 4;
   auto produce = [&](int it) {
     const int s = it % S;
-    if (it >= S) mbar_wait(empty0 + 8 * s, ((uint32_t)(it / S) & 1u) ^ 1u);
     const uint32_t bar = full0 + 8 * s, dst = smem_u32(ring + (size_t)s * stage_floats);
     mbar_expect(bar, tx);
     tma_load2d(dst, &tmL, l0, k0 + it * R, bar);
     tma_load2d(dst + (uint32_t)(R * TL * 4), &tmQ, q0, k0 + it * R, bar);
   };
   if (tid == 0)
-    for (int it = 0; it < S - 1 && it < nst; it++) produce(it);
+    for (int it = 0; it < S && it < nst; it++) produce(it);
 #pragma unroll 1
   for (int it = 0; it < nst; it++) {
-    if (tid == 0 && it + S - 1 < nst) produce(it + S - 1);   // keeps S - 1 stages in flight
     const int s = it % S;
     mbar_wait(full0 + 8 * s, (uint32_t)(it / S) & 1u);
     const float* Ls = ring + (size_t)s * stage_floats + lane;
@@ -201,7 +205,18 @@ __global__ void __maxnreg__(MAXREG) wgs_kernel(const __grid_constant__ CUtensorM
       }
     }
     __syncwarp();
-    if (lane == 0) mbar_arrive(empty0 + 8 * s);
+    if (lane == 0) {
+      // this warp is done reading slot s; the last of the NCW warps to get here refills it (the
+      // empty barrier orders every warp's reads before the async-proxy TMA write)
+      mbar_arrive(empty0 + 8 * s);
+      if (atomicAdd(&released[s], 1u) == NCW - 1) {
+        released[s] = 0u;
+        if (it + S < nst) {
+          mbar_wait(empty0 + 8 * s, (uint32_t)(it / S) & 1u);
+          produce(it + S);
+        }
+      }
+    }
   }
   __syncthreads();   // every stage consumed: the ring becomes the reduction area
   // row-group blocks -> shared [warp][i][j][lane], then summed in warp order (element e = (i*NB+j)*32 + lane)

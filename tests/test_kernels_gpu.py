@@ -213,12 +213,25 @@ def test_losses_sgd_colsum():
     assert rel(out, om._r(A.double().sum(0))) < 1e-6
 
 
+@pytest.mark.parametrize("M,N", [(1536, 2048), (1536, 512), (1537, 1535), (5, 3), (40000, 37), (32, 512)])
+def test_colsum_shapes(M, N):
+    """Bias gradients (encoder b8 s192 FFN / projections; ragged rows and columns, N % 4 != 0)."""
+    import parity as PT
+    A = si.normal((M, N), 69)
+    out = torch.zeros(N, device="cuda")
+    run("colsum", [dev(A), out, M, N])
+    PT.assert_close("colsum", out, om._r(A.double().sum(0)), 1e-6)
+    first = out.clone()
+    run("colsum", [dev(A), out, M, N])
+    assert torch.equal(first, out)
+
+
 def test_geometry_and_sm_needed():
     """sm_needed = ceil(grid / blocks_per_sm) from the kernel's own launch geometry."""
     A = torch.zeros(4096, 256, device="cuda")
     grid, bps, thr, smem = orion.kernel_geometry("gemm", [A.data_ptr(), A.data_ptr(), A.data_ptr(), 0, 1024, 16, 16, 16, 16, 16, 2, 0, 0])
     assert grid == 1024 // 32 and thr == 256 and bps >= 1
-    # a compute-dense shape routes to the tcgen05 kernel (160 threads, ~196 KB dynamic smem)
+    # a compute-dense shape routes to the tcgen05 kernel (288 threads, ~196 KB dynamic smem)
     grid, bps, thr, smem = orion.kernel_geometry("gemm", [A.data_ptr(), A.data_ptr(), A.data_ptr(), 0, 4096, 256, 256, 256, 256, 256, 0, 0, 0])
     assert thr == 288 and smem > 100_000 and bps == 1
     grid, bps, thr, smem = orion.kernel_geometry("relu", [A.data_ptr(), A.data_ptr(), A.numel()])
