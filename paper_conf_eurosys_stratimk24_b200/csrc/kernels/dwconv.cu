@@ -11,244 +11,231 @@ constexpr int DW_THREADS = 256;
 
 struct DwShape { int N, H, W, C, stride, P, Q; };
 
-// Row-blocked depthwise kernels: a warp owns 32 consecutive channels (128-byte coalesced rows of
-// the NHWC tensor) and one output row (n, p); each lane produces U = 4 consecutive outputs per step
-// from a 3 x ((U-1)*S+3) register window of its input columns whose loads are all issued
-// together (memory-level parallelism instead of one dependent load per output). Weights live in
-// registers. S = stride (compile-time 1 or 2).
-constexpr int ROW_WARPS = 8;
-constexpr int DW_U = 4;
-constexpr int DW_UW = 8;   // wgrad: twice the loads in flight per window block (latency-bound, ncu r01)
-constexpr int DW_U1 = 8;   // stride-1 fwd / dgrad: 8 outputs per 3 x 10 window (3.75 loads per output instead of 4.5)
-
-template <int S, int U = DW_U>
-struct Win {
-  static constexpr int NC = (U - 1) * S + 3;   // input columns per block of U outputs
-  float v[3][NC];
-  // columns col0 .. col0+NC-1 of the 3 input rows (zero outside the image / missing rows)
-  __device__ __forceinline__ void load(const float* const (&rowp)[3], const bool (&rv)[3], int col0, int W, int C) {
+// Channel-quad sliding-window kernels (round 2). A thread owns one channel quad (4 channels,
+// 128-bit NHWC loads / stores; C % 4 == 0) of one output row (n, p) and walks the row: the 3 x 3
+// window of input quads slides one column (stride 1) or two (stride 2) per output, so an output quad
+// costs 3 (or 6) 128-bit loads, 36 FFMA and one 128-bit store. Items (row, quad) are laid out quad-
+// fastest so a warp's loads are contiguous 512-byte runs of the NHWC rows. (Round 1 gave each lane
+// one channel and recomputed a 64-bit address and a bounds predicate per scalar load: ~85
+// instructions per output, ncu: issue-bound at 77 % of issue slots, 29 % of DRAM bandwidth.)
+// The three window columns rotate roles through a 3x unrolled step (no register moves).
+__device__ __forceinline__ float4 ld4(const float* p, bool ok) {
+  return ok ? __ldg(reinterpret_cast<const float4*>(p)) : make_float4(0.f, 0.f, 0.f, 0.f);
+}
+__device__ __forceinline__ void fma4(float4& a, const float4& x, const float4& w) {
+  a.x = fmaf(x.x, w.x, a.x); a.y = fmaf(x.y, w.y, a.y); a.z = fmaf(x.z, w.z, a.z); a.w = fmaf(x.w, w.w, a.w);
+}
+// taps t = r * 3 + u of channels c..c+3 (weights [C][3][3]); FLIP reverses the taps (the stride-1
+// data gradient is the forward correlation of dy with the flipped kernel)
+template <bool FLIP>
+__device__ __forceinline__ void load_taps(const float* __restrict__ w, int c, float4 (&k)[9]) {
 #pragma unroll
-    for (int r = 0; r < 3; r++)
-#pragma unroll
-      for (int j = 0; j < NC; j++) {
-        const int col = col0 + j;
-        v[r][j] = (rv[r] && (unsigned)col < (unsigned)W) ? __ldg(rowp[r] + (long long)col * C) : 0.f;
-      }
+  for (int t = 0; t < 9; t++) {
+    const int tt = FLIP ? 8 - t : t;
+    k[t] = make_float4(__ldg(w + (c + 0) * 9 + tt), __ldg(w + (c + 1) * 9 + tt), __ldg(w + (c + 2) * 9 + tt), __ldg(w + (c + 3) * 9 + tt));
   }
-};
+}
 
-template <int S>
-__global__ void __launch_bounds__(DW_THREADS) dw_fwd_rows_kernel(const float* __restrict__ x, const float* __restrict__ w,
-                                                                 float* __restrict__ y, DwShape s, OrionSig sig) {
-  const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
-  const int cblocks = (s.C + 31) / 32;
-  const long long nrows = (long long)s.N * s.P;
-  for (long long item = (long long)blockIdx.x * ROW_WARPS + warp; item < nrows * cblocks; item += (long long)gridDim.x * ROW_WARPS) {
-    const int cb = (int)(item % cblocks);
-    const long long row = item / cblocks;
-    const int p = (int)(row % s.P), n = (int)(row / s.P);
-    const int c = cb * 32 + lane;
-    if (c >= s.C) continue;
-    float wr[9];
-#pragma unroll
-    for (int t = 0; t < 9; t++) wr[t] = __ldg(w + c * 9 + t);
+// y[n,p,q,c] = sum_{r,u} x[n, p*S-1+r, q*S-1+u, c] k[c,r,u]; with FLIP (and S = 1, x = dy) this is
+// the stride-1 data gradient dx[n,h,w,c] = sum_{r,u} dy[n,h+1-r,w+1-u,c] k[c,r,u].
+template <int S, bool FLIP>
+__global__ void __launch_bounds__(DW_THREADS) dw_q4_fwd_kernel(const float* __restrict__ x, const float* __restrict__ w,
+                                                               float* __restrict__ y, int N, int H, int W, int C, int P, int Q,
+                                                               OrionSig sig) {
+  const int C4 = C / 4;
+  const long long items = (long long)N * P * C4;
+  for (long long it = (long long)blockIdx.x * blockDim.x + threadIdx.x; it < items; it += (long long)gridDim.x * blockDim.x) {
+    const int c = (int)(it % C4) * 4;
+    const long long row = it / C4;
+    const int p = (int)(row % P), n = (int)(row / P);
+    float4 k[9];
+    load_taps<FLIP>(w, c, k);
     const float* xr[3];
     bool rv[3];
 #pragma unroll
     for (int r = 0; r < 3; r++) {
-      int h = p * S - 1 + r;
-      rv[r] = (unsigned)h < (unsigned)s.H;
-      xr[r] = x + (((long long)n * s.H + (rv[r] ? h : 0)) * s.W) * s.C + c;
+      const int h = p * S - 1 + r;
+      rv[r] = (unsigned)h < (unsigned)H;
+      xr[r] = x + (((long long)n * H + (rv[r] ? h : 0)) * W) * C + c;
     }
-    float* yr = y + (((long long)n * s.P + p) * s.Q) * s.C + c;
-    constexpr int U = S == 1 ? DW_U1 : DW_U;
-    for (int q0 = 0; q0 < s.Q; q0 += U) {
-      Win<S, U> win;
-      win.load(xr, rv, q0 * S - 1, s.W, s.C);
+    float* yr = y + (((long long)n * P + p) * Q) * C + c;
+    // window columns: a = col q*S-1, b = q*S, cc = q*S+1 (stride 2 also needs q*S+2 = next a)
+    float4 a[3], b[3], e[3];
 #pragma unroll
-      for (int u = 0; u < U; u++) {
-        if (q0 + u < s.Q) {
-          float acc = 0.f;
+    for (int r = 0; r < 3; r++) { a[r] = make_float4(0.f, 0.f, 0.f, 0.f); b[r] = ld4(xr[r], rv[r] && 0 < W); }
+    auto out = [&](const float4 (&c0)[3], const float4 (&c1)[3], const float4 (&c2)[3], int q) {
+      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
-          for (int r = 0; r < 3; r++)
+      for (int r = 0; r < 3; r++) { fma4(acc, c0[r], k[r * 3]); fma4(acc, c1[r], k[r * 3 + 1]); fma4(acc, c2[r], k[r * 3 + 2]); }
+      *reinterpret_cast<float4*>(yr + (long long)q * C) = acc;
+    };
+    if (S == 1) {
+      // a = col q-1, b = col q; load col q+1 into the third slot; roles rotate a -> b -> e
+      int q = 0;
+      for (; q + 2 < Q; q += 3) {
 #pragma unroll
-            for (int t = 0; t < 3; t++) acc = fmaf(win.v[r][u * S + t], wr[r * 3 + t], acc);
-          yr[(long long)(q0 + u) * s.C] = acc;
-        }
+        for (int r = 0; r < 3; r++) e[r] = ld4(xr[r] + (long long)(q + 1) * C, rv[r] && q + 1 < W);
+        out(a, b, e, q);
+#pragma unroll
+        for (int r = 0; r < 3; r++) a[r] = ld4(xr[r] + (long long)(q + 2) * C, rv[r] && q + 2 < W);
+        out(b, e, a, q + 1);
+#pragma unroll
+        for (int r = 0; r < 3; r++) b[r] = ld4(xr[r] + (long long)(q + 3) * C, rv[r] && q + 3 < W);
+        out(e, a, b, q + 2);   // a = col q+2, b = col q+3: exactly the next trip's "q-1" and "q"
+      }
+      for (; q < Q; q++) {
+#pragma unroll
+        for (int r = 0; r < 3; r++) e[r] = ld4(xr[r] + (long long)(q + 1) * C, rv[r] && q + 1 < W);
+        out(a, b, e, q);
+#pragma unroll
+        for (int r = 0; r < 3; r++) { a[r] = b[r]; b[r] = e[r]; }
+      }
+    } else {
+      // stride 2: output q reads cols 2q-1 (a), 2q (b), 2q+1 (e); the next output's 2q+1 is e
+      for (int q = 0; q < Q; q++) {
+#pragma unroll
+        for (int r = 0; r < 3; r++) e[r] = ld4(xr[r] + (long long)(2 * q + 1) * C, rv[r] && 2 * q + 1 < W);
+        out(a, b, e, q);
+#pragma unroll
+        for (int r = 0; r < 3; r++) { a[r] = e[r]; b[r] = ld4(xr[r] + (long long)(2 * q + 2) * C, rv[r] && 2 * q + 2 < W); }
       }
     }
   }
   orion_signal(sig);
 }
 
-// Stride-1 dgrad is a correlation with the flipped kernel: dx(h, w) = sum_{r,u} dy(h+1-r, w+1-u) k(r,u).
-__global__ void __launch_bounds__(DW_THREADS) dw_dgrad_rows_s1_kernel(const float* __restrict__ dy, const float* __restrict__ w,
-                                                                      float* __restrict__ dx, DwShape s, OrionSig sig) {
-  const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
-  const int cblocks = (s.C + 31) / 32;
-  const long long nrows = (long long)s.N * s.H;
-  for (long long item = (long long)blockIdx.x * ROW_WARPS + warp; item < nrows * cblocks; item += (long long)gridDim.x * ROW_WARPS) {
-    const int cb = (int)(item % cblocks);
-    const long long row = item / cblocks;
-    const int h = (int)(row % s.H), n = (int)(row / s.H);
-    const int c = cb * 32 + lane;
-    if (c >= s.C) continue;
-    float wr[9];
-#pragma unroll
-    for (int t = 0; t < 9; t++) wr[t] = __ldg(w + c * 9 + t);
-    const float* gr[3];
-    bool rv[3];
-#pragma unroll
-    for (int r = 0; r < 3; r++) {   // kernel row r reads dy row p = h + 1 - r
-      int pp = h + 1 - r;
-      rv[r] = (unsigned)pp < (unsigned)s.P;
-      gr[r] = dy + (((long long)n * s.P + (rv[r] ? pp : 0)) * s.Q) * s.C + c;
-    }
-    float* dr = dx + (((long long)n * s.H + h) * s.W) * s.C + c;
-    for (int w0 = 0; w0 < s.W; w0 += DW_U1) {
-      Win<1, DW_U1> win;               // dy columns w0-1 .. w0+U
-      win.load(gr, rv, w0 - 1, s.Q, s.C);
-#pragma unroll
-      for (int u = 0; u < DW_U1; u++) {
-        if (w0 + u < s.W) {
-          // column index in win for dy column (w0+u)+1-t is u + 2 - t
-          float acc = 0.f;
-#pragma unroll
-          for (int r = 0; r < 3; r++)
-#pragma unroll
-            for (int t = 0; t < 3; t++) acc = fmaf(win.v[r][u + 2 - t], wr[r * 3 + t], acc);
-          dr[(long long)(w0 + u) * s.C] = acc;
-        }
-      }
-    }
-  }
-  orion_signal(sig);
-}
-
-// Stride-2 dgrad, row-blocked: for input row h only kernel rows r with (h+1-r) even contribute
-// (one row for even h, two for odd h), and along w the pair (w = 2j, 2j+1) reads dy columns j and
-// j+1 only: dx(2j) = sum_r dy(p_r, j) k(r,1); dx(2j+1) = sum_r dy(p_r, j+1) k(r,0) + dy(p_r, j) k(r,2).
-__global__ void __launch_bounds__(DW_THREADS) dw_dgrad_rows_s2_kernel(const float* __restrict__ dy, const float* __restrict__ w,
-                                                                      float* __restrict__ dx, DwShape s, OrionSig sig) {
-  const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
-  const int cblocks = (s.C + 31) / 32;
-  const long long nrows = (long long)s.N * s.H;
-  for (long long item = (long long)blockIdx.x * ROW_WARPS + warp; item < nrows * cblocks; item += (long long)gridDim.x * ROW_WARPS) {
-    const int cb = (int)(item % cblocks);
-    const long long row = item / cblocks;
-    const int h = (int)(row % s.H), n = (int)(row / s.H);
-    const int c = cb * 32 + lane;
-    if (c >= s.C) continue;
-    // up to two contributing kernel rows
-    int rr[2], pp[2], nr = 0;
-#pragma unroll
-    for (int r = 0; r < 3; r++) {
-      const int ph = h + 1 - r;
-      if (ph >= 0 && (ph & 1) == 0 && ph / 2 < s.P) { rr[nr] = r; pp[nr] = ph / 2; nr++; }
-    }
-    float k0[2], k1[2], k2[2];
+// Stride-2 data gradient: input row h takes kernel rows r with (h+1-r) even (dy row (h+1-r)/2);
+// along w the pair (2j, 2j+1) reads dy columns j and j+1:
+//   dx(2j) = sum_r dy(p_r, j) k(r,1);  dx(2j+1) = sum_r dy(p_r, j+1) k(r,0) + dy(p_r, j) k(r,2).
+// Thread = (n, h, channel quad); dy column j+1 of one pair is column j of the next.
+__global__ void __launch_bounds__(DW_THREADS) dw_q4_dgrad_s2_kernel(const float* __restrict__ dy, const float* __restrict__ w,
+                                                                    float* __restrict__ dx, int N, int H, int W, int C, int P, int Q,
+                                                                    OrionSig sig) {
+  const int C4 = C / 4;
+  const long long items = (long long)N * H * C4;
+  for (long long it = (long long)blockIdx.x * blockDim.x + threadIdx.x; it < items; it += (long long)gridDim.x * blockDim.x) {
+    const int c = (int)(it % C4) * 4;
+    const long long row = it / C4;
+    const int h = (int)(row % H), n = (int)(row / H);
+    // odd h: kernel rows 0 and 2 (dy rows (h+1)/2 and (h-1)/2); even h: kernel row 1 (dy row h/2)
+    const bool odd = h & 1;
+    const int rsel[2] = {odd ? 0 : 1, 2};
+    const int prow[2] = {odd ? (h + 1) / 2 : h / 2, (h - 1) / 2};
+    bool on[2];
+    on[0] = prow[0] < P;
+    on[1] = odd && prow[1] >= 0 && prow[1] < P;
+    float4 k0[2], k1[2], k2[2];
     const float* gr[2];
 #pragma unroll
     for (int i = 0; i < 2; i++) {
-      const bool on = i < nr;
-      k0[i] = on ? __ldg(w + c * 9 + rr[i] * 3 + 0) : 0.f;
-      k1[i] = on ? __ldg(w + c * 9 + rr[i] * 3 + 1) : 0.f;
-      k2[i] = on ? __ldg(w + c * 9 + rr[i] * 3 + 2) : 0.f;
-      gr[i] = dy + (((long long)n * s.P + (on ? pp[i] : 0)) * s.Q) * s.C + c;
+      const int r = rsel[i];
+      gr[i] = dy + (((long long)n * P + (on[i] ? prow[i] : 0)) * Q) * C + c;
+      k0[i] = make_float4(__ldg(w + c * 9 + r * 3), __ldg(w + (c + 1) * 9 + r * 3), __ldg(w + (c + 2) * 9 + r * 3), __ldg(w + (c + 3) * 9 + r * 3));
+      k1[i] = make_float4(__ldg(w + c * 9 + r * 3 + 1), __ldg(w + (c + 1) * 9 + r * 3 + 1), __ldg(w + (c + 2) * 9 + r * 3 + 1),
+                          __ldg(w + (c + 3) * 9 + r * 3 + 1));
+      k2[i] = make_float4(__ldg(w + c * 9 + r * 3 + 2), __ldg(w + (c + 1) * 9 + r * 3 + 2), __ldg(w + (c + 2) * 9 + r * 3 + 2),
+                          __ldg(w + (c + 3) * 9 + r * 3 + 2));
     }
-    auto ld = [&](int i, int col) -> float {
-      return (i < nr && (unsigned)col < (unsigned)s.Q) ? __ldg(gr[i] + (long long)col * s.C) : 0.f;
-    };
-    float* dr = dx + (((long long)n * s.H + h) * s.W) * s.C + c;
-    const int npairs = (s.W + 1) / 2;
-    for (int j0 = 0; j0 < npairs; j0 += DW_U) {
-      float col[2][DW_U + 1];
+    float* dr = dx + (((long long)n * H + h) * W) * C + c;
+    float4 cur[2];
 #pragma unroll
-      for (int i = 0; i < 2; i++)
+    for (int i = 0; i < 2; i++) cur[i] = ld4(gr[i], on[i] && 0 < Q);
+    const int npairs = (W + 1) / 2;
+    for (int j = 0; j < npairs; j++) {
+      float4 nxt[2];
 #pragma unroll
-        for (int u = 0; u <= DW_U; u++) col[i][u] = ld(i, j0 + u);
+      for (int i = 0; i < 2; i++) nxt[i] = ld4(gr[i] + (long long)(j + 1) * C, on[i] && j + 1 < Q);
+      float4 e = make_float4(0.f, 0.f, 0.f, 0.f), o = make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
-      for (int u = 0; u < DW_U; u++) {
-        const int we = 2 * (j0 + u);
-        if (we < s.W) {
-          float e = 0.f, o = 0.f;
+      for (int i = 0; i < 2; i++) { fma4(e, cur[i], k1[i]); fma4(o, nxt[i], k0[i]); fma4(o, cur[i], k2[i]); }
+      *reinterpret_cast<float4*>(dr + (long long)(2 * j) * C) = e;
+      if (2 * j + 1 < W) *reinterpret_cast<float4*>(dr + (long long)(2 * j + 1) * C) = o;
 #pragma unroll
-          for (int i = 0; i < 2; i++) {
-            e = fmaf(col[i][u], k1[i], e);
-            o = fmaf(col[i][u + 1], k0[i], o);
-            o = fmaf(col[i][u], k2[i], o);
-          }
-          dr[(long long)we * s.C] = e;
-          if (we + 1 < s.W) dr[(long long)(we + 1) * s.C] = o;
-        }
-      }
+      for (int i = 0; i < 2; i++) cur[i] = nxt[i];
     }
   }
   orion_signal(sig);
 }
 
-// wgrad: a warp accumulates the 9 taps of its 32 channels over whole output rows (register window
-// blocks as above), fp32 per row and fp64 across rows; warps combine in smem in fixed order, CTAs
-// write per-split partials, the last CTA of the channel block sums them in split order.
+// wgrad: dW[c,r,u] = sum_{n,p,q} dy[n,p,q,c] x[n, p*S-1+r, q*S-1+u, c]. CTA = a block of CQ channel
+// quads (quad = tid % CQ) x RL row lanes (tid / CQ); a thread walks whole output rows of its quad
+// with the sliding x window, accumulating the 36 products of a row in fp32, then adds the row into
+// its fp64 slots in shared memory (same order every run). Row lanes are combined in lane order,
+// CTAs write per-split partials, the last CTA of the channel block sums them in split order.
+constexpr int WQ_MAXQ = 64;   // channel quads per CTA (C <= 256 per block)
 template <int S>
-__global__ void __launch_bounds__(DW_THREADS, S == 1 ? 3 : 2) dw_wgrad_rows_kernel(const float* __restrict__ x, const float* __restrict__ dy,
-                                                                   float* __restrict__ dw, DwShape s, unsigned char* ws, OrionSig sig) {
-  __shared__ double sh[ROW_WARPS][9][32];
-  const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
-  const int c = blockIdx.x * 32 + lane;
-  const long long nrows = (long long)s.N * s.P;
-  // the fp64 row sums live in this lane's own shared-memory slots (no registers; same order)
-  double* acc = &sh[warp][0][lane];
-#pragma unroll
-  for (int t = 0; t < 9; t++) acc[t * 32] = 0.0;
-  if (c < s.C) {
-    for (long long row = (long long)blockIdx.y * ROW_WARPS + warp; row < nrows; row += (long long)gridDim.y * ROW_WARPS) {
-      const int p = (int)(row % s.P), n = (int)(row / s.P);
+__global__ void __launch_bounds__(DW_THREADS, 2) dw_q4_wgrad_kernel(const float* __restrict__ x, const float* __restrict__ dy,
+                                                                    float* __restrict__ dwt, int N, int H, int W, int C, int P, int Q,
+                                                                    int cq_n, unsigned char* ws, OrionSig sig) {
+  extern __shared__ double wq_sh[];   // [rl][36][cq_n] fp64 row-sum slots, later [36 * cq_n] combine area
+  const int rl_n = DW_THREADS / cq_n;
+  const int cq = threadIdx.x % cq_n, rl = threadIdx.x / cq_n;
+  const int c = (blockIdx.x * cq_n + cq) * 4;
+  const bool active = rl < rl_n && c < C;
+  double* slot = wq_sh + (size_t)rl * 36 * cq_n + cq;
+  if (rl < rl_n)
+    for (int t = 0; t < 36; t++) slot[(size_t)t * cq_n] = 0.0;
+  const long long nrows = (long long)N * P;
+  if (active) {
+    for (long long row = (long long)blockIdx.y * rl_n + rl; row < nrows; row += (long long)gridDim.y * rl_n) {
+      const int p = (int)(row % P), n = (int)(row / P);
       const float* xr[3];
       bool rv[3];
 #pragma unroll
       for (int r = 0; r < 3; r++) {
-        int h = p * S - 1 + r;
-        rv[r] = (unsigned)h < (unsigned)s.H;
-        xr[r] = x + (((long long)n * s.H + (rv[r] ? h : 0)) * s.W) * s.C + c;
+        const int h = p * S - 1 + r;
+        rv[r] = (unsigned)h < (unsigned)H;
+        xr[r] = x + (((long long)n * H + (rv[r] ? h : 0)) * W) * C + c;
       }
-      const float* gr = dy + (((long long)n * s.P + p) * s.Q) * s.C + c;
-      float f[9];
+      const float* gr = dy + (((long long)n * P + p) * Q) * C + c;
+      float4 f[9];
 #pragma unroll
-      for (int t = 0; t < 9; t++) f[t] = 0.f;
-      for (int q0 = 0; q0 < s.Q; q0 += DW_UW) {
-        Win<S, DW_UW> win;
-        win.load(xr, rv, q0 * S - 1, s.W, s.C);
-        float g[DW_UW];
+      for (int t = 0; t < 9; t++) f[t] = make_float4(0.f, 0.f, 0.f, 0.f);
+      float4 a[3], b[3], e[3];
 #pragma unroll
-        for (int u = 0; u < DW_UW; u++) g[u] = (q0 + u < s.Q) ? __ldg(gr + (long long)(q0 + u) * s.C) : 0.f;
+      for (int r = 0; r < 3; r++) { a[r] = make_float4(0.f, 0.f, 0.f, 0.f); b[r] = ld4(xr[r], rv[r] && 0 < W); }
+      for (int q = 0; q < Q; q++) {
 #pragma unroll
-        for (int u = 0; u < DW_UW; u++)
+        for (int r = 0; r < 3; r++) e[r] = ld4(xr[r] + (long long)(q * S + 1) * C, rv[r] && q * S + 1 < W);
+        const float4 g = __ldg(reinterpret_cast<const float4*>(gr + (long long)q * C));
 #pragma unroll
-          for (int r = 0; r < 3; r++)
+        for (int r = 0; r < 3; r++) { fma4(f[r * 3], g, a[r]); fma4(f[r * 3 + 1], g, b[r]); fma4(f[r * 3 + 2], g, e[r]); }
+        if (S == 1) {
 #pragma unroll
-            for (int t = 0; t < 3; t++) f[r * 3 + t] = fmaf(g[u], win.v[r][u * S + t], f[r * 3 + t]);
+          for (int r = 0; r < 3; r++) { a[r] = b[r]; b[r] = e[r]; }
+        } else {
+#pragma unroll
+          for (int r = 0; r < 3; r++) { a[r] = e[r]; b[r] = ld4(xr[r] + (long long)(q * S + 2) * C, rv[r] && q * S + 2 < W); }
+        }
       }
 #pragma unroll
-      for (int t = 0; t < 9; t++) acc[t * 32] += (double)f[t];
+      for (int t = 0; t < 9; t++) {
+        slot[(size_t)(t * 4 + 0) * cq_n] += (double)f[t].x;
+        slot[(size_t)(t * 4 + 1) * cq_n] += (double)f[t].y;
+        slot[(size_t)(t * 4 + 2) * cq_n] += (double)f[t].z;
+        slot[(size_t)(t * 4 + 3) * cq_n] += (double)f[t].w;
+      }
     }
   }
   __syncthreads();
   unsigned int* tickets = reinterpret_cast<unsigned int*>(ws);
   double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
-  if (warp == 0 && c < s.C) {
-    for (int t = 0; t < 9; t++) {
-      double v = 0.0;
-      for (int wv = 0; wv < ROW_WARPS; wv++) v += sh[wv][t][lane];
-      part[((long long)blockIdx.y * s.C + c) * 9 + t] = v;
-    }
+  const int c0 = blockIdx.x * cq_n * 4;
+  const int nch = min(cq_n * 4, C - c0);
+  // partial of this split: part[split][c][tap] (tap = r*3+u), row lanes summed in lane order
+  for (int v = threadIdx.x; v < nch * 9; v += DW_THREADS) {
+    const int cc = v / 9, t = v % 9, q4 = cc / 4, j = cc % 4;
+    double sum = 0.0;
+    for (int l = 0; l < rl_n; l++) sum += wq_sh[((size_t)l * 36 + t * 4 + j) * cq_n + q4];
+    part[((long long)blockIdx.y * C + c0 + cc) * 9 + t] = sum;
   }
-  __shared__ double out[9 * 32];
-  const int rs = gridDim.y, c0 = blockIdx.x * 32;
-  const int V = 9 * min(32, s.C - c0);
-  if (combine_splits(tickets + blockIdx.x * (combine_rows(rs) + 1), part + 9LL * c0, part + 9LL * rs * s.C + 9LL * c0, 9LL * s.C, rs,
-                     blockIdx.y, V, out, &sh[0][0][0])) {
-    for (int v = threadIdx.x; v < V; v += blockDim.x) dw[9LL * c0 + v] = (float)out[v];
+  const int rs = gridDim.y;
+  const int V = 9 * nch;
+  double* out = wq_sh;   // reuse (the partials above are in global memory now)
+  __syncthreads();
+  if (combine_splits(tickets + blockIdx.x * (combine_rows(rs) + 1), part + 9LL * c0, part + 9LL * rs * C + 9LL * c0, 9LL * C, rs,
+                     blockIdx.y, V, out, out + V)) {
+    for (int v = threadIdx.x; v < V; v += DW_THREADS) dwt[9LL * c0 + v] = (float)out[v];
   }
   orion_signal(sig);
 }
@@ -304,17 +291,23 @@ void ew(LaunchGeom* g, uint64_t n, const void* f, std::atomic<int>& occ) {
   g->grid = dim3((unsigned)ctas); g->block = dim3(DW_THREADS); g->smem = 0; g->func = f;
 }
 
-void rows_geom(LaunchGeom* g, long long items, const void* f) {
-  long long ctas = cdiv(items, ROW_WARPS);
-  if (ctas > 148 * 8) ctas = 148 * 8;
+std::atomic<int> dwq_occ[4];
+void q4_geom(LaunchGeom* g, long long items, const void* f, std::atomic<int>& occ) {
+  long long ctas = cdiv(items, DW_THREADS);
+  const long long wave = 148LL * resident_ctas_per_sm(f, DW_THREADS, occ);   // one resident wave (shape heuristic)
+  if (ctas > wave) ctas = wave;
   if (ctas < 1) ctas = 1;
   g->grid = dim3((unsigned)ctas); g->block = dim3(DW_THREADS); g->smem = 0; g->func = f;
 }
 
+int wq_cq(int C) { const int q = C / 4; return q < WQ_MAXQ ? q : WQ_MAXQ; }
+int wq_smem(int C) { const int cq = wq_cq(C); const int rl = DW_THREADS / cq; return rl * 36 * cq * 8; }
+
 int wg_splits(const DwShape& s) {
-  long long cblocks = (s.C + 31) / 32;
-  long long rs = cdiv(148 * 8, cblocks);
-  long long max_rs = cdiv((long long)s.N * s.P, ROW_WARPS);
+  const int cq = wq_cq(s.C);
+  long long cblocks = cdiv(s.C / 4, cq);
+  long long rs = cdiv(148 * 2, cblocks);                     // ~two CTAs per SM of a 148-SM part
+  long long max_rs = cdiv((long long)s.N * s.P, DW_THREADS / cq);
   if (rs > max_rs) rs = max_rs;
   if (rs < 1) rs = 1;
   return (int)rs;
@@ -323,6 +316,7 @@ int wg_splits(const DwShape& s) {
 }  // namespace
 
 extern "C" uint64_t orion_dw_wgrad_workspace_bytes(uint64_t N, uint64_t C, uint64_t P, uint64_t Q) {
+  if (C % 4) C += 4 - C % 4;
   DwShape s{(int)N, 0, 0, (int)C, 1, (int)P, (int)Q};
   const int rs = wg_splits(s);
   return WS_TICKET_BYTES + (uint64_t)(rs + combine_rows(rs)) * C * 9 * 8;
@@ -334,32 +328,37 @@ int dw_fwd_geom(const uint64_t* a, LaunchGeom* g) {
   if (!dw_ok(a)) return ORION_E_INVAL;
   DwShape s = dw_shape(a);
   if (s.stride != 1 && s.stride != 2) return ORION_E_INVAL;
-  rows_geom(g, (long long)s.N * s.P * ((s.C + 31) / 32), s.stride == 1 ? (const void*)dw_fwd_rows_kernel<1> : (const void*)dw_fwd_rows_kernel<2>);
+  const long long items = (long long)s.N * s.P * (s.C / 4);
+  if (s.stride == 1) q4_geom(g, items, (const void*)dw_q4_fwd_kernel<1, false>, dwq_occ[0]);
+  else q4_geom(g, items, (const void*)dw_q4_fwd_kernel<2, false>, dwq_occ[1]);
   return 0;
 }
 int dw_fwd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
-  if (g.func == (const void*)dw_fwd_rows_kernel<1>)
-    dw_fwd_rows_kernel<1><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
+  DwShape s = dw_shape(a);
+  if (g.func == (const void*)dw_q4_fwd_kernel<1, false>)
+    dw_q4_fwd_kernel<1, false><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q, sig);
   else
-    dw_fwd_rows_kernel<2><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
+    dw_q4_fwd_kernel<2, false><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q, sig);
   CHECK_LAUNCH();
 }
 std::atomic<int> dw_dgrad_occ{0};
 int dw_dgrad_geom(const uint64_t* a, LaunchGeom* g) {
   if (!dw_ok(a)) return ORION_E_INVAL;
   DwShape s = dw_shape(a);
-  if (s.stride == 1) rows_geom(g, (long long)s.N * s.H * ((s.C + 31) / 32), (const void*)dw_dgrad_rows_s1_kernel);
-  else if (s.stride == 2) rows_geom(g, (long long)s.N * s.H * ((s.C + 31) / 32), (const void*)dw_dgrad_rows_s2_kernel);
+  if (s.stride == 1) q4_geom(g, (long long)s.N * s.H * (s.C / 4), (const void*)dw_q4_fwd_kernel<1, true>, dwq_occ[2]);
+  else if (s.stride == 2) q4_geom(g, (long long)s.N * s.H * (s.C / 4), (const void*)dw_q4_dgrad_s2_kernel, dwq_occ[3]);
   else ew(g, (uint64_t)s.N * s.H * s.W * (s.C / 4), (const void*)dw_dgrad_kernel, dw_dgrad_occ);
   return 0;
 }
 int dw_dgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
-  if (g.func == (const void*)dw_dgrad_rows_s1_kernel)
-    dw_dgrad_rows_s1_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
-  else if (g.func == (const void*)dw_dgrad_rows_s2_kernel)
-    dw_dgrad_rows_s2_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
+  DwShape s = dw_shape(a);
+  if (g.func == (const void*)dw_q4_fwd_kernel<1, true>)   // stride-1 dgrad = correlation of dy with the flipped kernel
+    dw_q4_fwd_kernel<1, true><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.P, s.Q, s.C, s.H, s.W,
+                                                          sig);
+  else if (g.func == (const void*)dw_q4_dgrad_s2_kernel)
+    dw_q4_dgrad_s2_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q, sig);
   else
-    dw_dgrad_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a), sig);
+    dw_dgrad_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s, sig);
   CHECK_LAUNCH();
 }
 // wgrad args: x, dy, dw, N, H, W, C, C, 3, 3, stride, 1, P, Q, ws, ws_bytes
@@ -368,16 +367,28 @@ int dw_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
   DwShape s = dw_shape(a);
   if (a[14] == 0 || a[15] < orion_dw_wgrad_workspace_bytes(s.N, s.C, s.P, s.Q)) return ORION_E_INVAL;
   if (s.stride != 1 && s.stride != 2) return ORION_E_INVAL;
-  g->grid = dim3((s.C + 31) / 32, wg_splits(s)); g->block = dim3(DW_THREADS); g->smem = 0;
-  g->func = s.stride == 1 ? (const void*)dw_wgrad_rows_kernel<1> : (const void*)dw_wgrad_rows_kernel<2>;
+  static std::atomic<int> attr{0};
+  if (!attr.load()) {
+    if (cudaFuncSetAttribute((const void*)dw_q4_wgrad_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024) != cudaSuccess ||
+        cudaFuncSetAttribute((const void*)dw_q4_wgrad_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024) != cudaSuccess) {
+      (void)cudaGetLastError();
+      return ORION_E_CUDA;
+    }
+    attr.store(1);
+  }
+  const int cq = wq_cq(s.C);
+  g->grid = dim3((unsigned)cdiv(s.C / 4, cq), (unsigned)wg_splits(s)); g->block = dim3(DW_THREADS); g->smem = wq_smem(s.C);
+  g->func = s.stride == 1 ? (const void*)dw_q4_wgrad_kernel<1> : (const void*)dw_q4_wgrad_kernel<2>;
   return 0;
 }
 int dw_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
-  if (g.func == (const void*)dw_wgrad_rows_kernel<1>)
-    dw_wgrad_rows_kernel<1><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a),
-                                                        (unsigned char*)a[14], sig);
+  DwShape s = dw_shape(a);
+  const int cq = wq_cq(s.C);
+  if (g.func == (const void*)dw_q4_wgrad_kernel<1>)
+    dw_q4_wgrad_kernel<1><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q,
+                                                          cq, (unsigned char*)a[14], sig);
   else
-    dw_wgrad_rows_kernel<2><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], dw_shape(a),
-                                                        (unsigned char*)a[14], sig);
+    dw_q4_wgrad_kernel<2><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q,
+                                                          cq, (unsigned char*)a[14], sig);
   CHECK_LAUNCH();
 }

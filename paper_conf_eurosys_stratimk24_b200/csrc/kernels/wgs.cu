@@ -15,6 +15,8 @@
 //    the last CTA of every tile sums the K splits in split order in fp64 (combine_splits).
 // The tile shape, the K split and the stage size are functions of (M, N, K) only, so results are
 // bitwise reproducible and independent of the SM partition the kernel runs in.
+#include <cstdlib>
+
 #include "common.cuh"
 #include "tma.cuh"
 
@@ -54,8 +56,19 @@ inline int pow2_floor(int v) {
   return p;
 }
 
+// stage size (KB) of the ring: a tuning knob (ORION_WGS_STAGE_KB, read once; default 32), never a
+// function of the partition, so results stay independent of where the kernel runs
+inline int stage_kb() {
+  static const int kb = [] {
+    const char* e = getenv("ORION_WGS_STAGE_KB");
+    const int v = e ? atoi(e) : 32;
+    return v >= 4 && v <= 48 ? v : 32;
+  }();
+  return kb;
+}
+
 inline int stage_rows(int rowf) {
-  int r = pow2_floor(16384 / (rowf * 4));   // ~16 KB stages: many small stages keep more loads in flight
+  int r = pow2_floor(stage_kb() * 1024 / (rowf * 4));
   return r < 32 ? 32 : (r > 256 ? 256 : r);
 }
 

@@ -1,0 +1,78 @@
+"""Warm per-launch CUDA-event times of the BE operators at MobileNetV2-b96 shapes (weight-gradient
+GEMMs, depthwise fwd / dgrad / wgrad), with algorithmic GB/s. Inputs > L2 for the large shapes.
+Usage: python tools/bench_kernels.py [wgs|dw|all]"""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+import paper_conf_eurosys_stratimk24_b200 as orion  # noqa: E402
+from paper_conf_eurosys_stratimk24_b200 import _lib as L  # noqa: E402
+from paper_conf_eurosys_stratimk24_b200.runtime import kernel_info  # noqa: E402
+
+
+def timeit(fn, args, reps=20):
+    s = torch.cuda.current_stream().cuda_stream
+    for _ in range(3):
+        orion.kernel_launch(fn, args, s)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0.record()
+    for _ in range(reps):
+        orion.kernel_launch(fn, args, s)
+    e1.record()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / reps * 1e3
+
+
+def ws(nbytes):
+    return torch.zeros(int(nbytes) // 4 + 64, device="cuda")
+
+
+WGS = [(96, 16, 1204224), (16, 32, 1204224), (24, 96, 301056), (144, 24, 301056), (24, 144, 301056), (32, 144, 75264),
+       (192, 32, 75264), (32, 192, 75264), (64, 192, 18816), (384, 64, 18816), (64, 384, 18816), (576, 96, 18816),
+       (96, 576, 18816), (160, 576, 4704), (960, 160, 4704), (160, 960, 4704), (320, 960, 4704), (1280, 320, 4704)]
+DW = [(96, 112, 32, 1), (96, 112, 96, 2), (96, 56, 144, 1), (96, 56, 144, 2), (96, 28, 192, 1), (96, 28, 192, 2),
+      (96, 14, 384, 1), (96, 14, 576, 1), (96, 14, 576, 2), (96, 7, 960, 1)]
+
+
+def wgs():
+    tot = 0.0
+    for M, N, K in WGS:
+        A, B, C = torch.randn(K, M, device="cuda"), torch.randn(K, N, device="cuda"), torch.zeros(M, N, device="cuda")
+        w = ws(L.lib.orion_gemm_workspace_bytes(M, N, K))
+        a = [A.data_ptr(), B.data_ptr(), C.data_ptr(), 0, M, N, K, M, N, N, 1, w.data_ptr(), w.numel() * 4]
+        t = timeit("gemm", a)
+        tot += t
+        info = kernel_info("gemm", a)
+        print(f"wgrad M={M:5d} N={N:5d} K={K:8d} {t:7.1f} us {4 * K * (M + N) / t / 1e3:6.0f} GB/s "
+              f"{2 * M * N * K / t / 1e6:6.1f} TF  grid {info['grid_ctas']} regs {info['regs_per_thread']} {info['kernel'][:40]}")
+    print(f"wgrad total {tot:.1f} us")
+
+
+def dw():
+    tot = 0.0
+    for n, h, c, st in DW:
+        p = (h - 1) // st + 1
+        x, dy = torch.randn(n, h, h, c, device="cuda"), torch.randn(n, p, p, c, device="cuda")
+        wt = torch.randn(c, 3, 3, 1, device="cuda")
+        y, dx, dwt = torch.zeros(n, p, p, c, device="cuda"), torch.zeros(n, h, h, c, device="cuda"), torch.zeros(c, 9, device="cuda")
+        dims = [n, h, h, c, c, 3, 3, st, 1, p, p]
+        w = ws(L.lib.orion_dw_wgrad_workspace_bytes(n, c, p, p))
+        byt = (x.numel() + dy.numel()) * 4
+        t1 = timeit("dw_fwd", [x.data_ptr(), wt.data_ptr(), y.data_ptr()] + dims)
+        t2 = timeit("dw_dgrad", [dy.data_ptr(), wt.data_ptr(), dx.data_ptr()] + dims)
+        t3 = timeit("dw_wgrad", [x.data_ptr(), dy.data_ptr(), dwt.data_ptr()] + dims + [w.data_ptr(), w.numel() * 4])
+        tot += t1 + t2 + t3
+        print(f"dw n={n} h={h:4d} c={c:4d} s={st}  fwd {t1:7.1f} us {byt / t1 / 1e3:5.0f} GB/s  dgrad {t2:7.1f} us "
+              f"{byt / t2 / 1e3:5.0f} GB/s  wgrad {t3:7.1f} us {byt / t3 / 1e3:5.0f} GB/s")
+    print(f"dw total {tot:.1f} us")
+
+
+if __name__ == "__main__":
+    torch.cuda.set_device(0)
+    what = sys.argv[1] if len(sys.argv) > 1 else "all"
+    if what in ("wgs", "all"):
+        wgs()
+    if what in ("dw", "all"):
+        dw()
