@@ -11,93 +11,76 @@ constexpr int DW_THREADS = 256;
 
 struct DwShape { int N, H, W, C, stride, P, Q; };
 
-// Channel-quad sliding-window kernels (round 2). A thread owns one channel quad (4 channels,
-// 128-bit NHWC loads / stores; C % 4 == 0) of one output row (n, p) and walks the row: the 3 x 3
-// window of input quads slides one column (stride 1) or two (stride 2) per output, so an output quad
-// costs 3 (or 6) 128-bit loads, 36 FFMA and one 128-bit store. Items (row, quad) are laid out quad-
-// fastest so a warp's loads are contiguous 512-byte runs of the NHWC rows. (Round 1 gave each lane
-// one channel and recomputed a 64-bit address and a bounds predicate per scalar load: ~85
-// instructions per output, ncu: issue-bound at 77 % of issue slots, 29 % of DRAM bandwidth.)
-// The three window columns rotate roles through a 3x unrolled step (no register moves).
+// Channel-quad kernels (round 2). A thread owns one channel quad (4 channels: 128-bit NHWC loads and
+// stores; C % 4 == 0) and a segment of U consecutive outputs of one output row. It issues all the
+// loads of its (U-1)*S+3-column input window at once (memory-level parallelism inside the thread),
+// then forms the U output quads from registers: per output quad (U = 4, stride 1) 4.5 128-bit loads,
+// 36 FFMA, one 128-bit store. The CTA stages the weights once as [tap][quad] float4s in shared
+// memory. Items are (quad, segment, row) with the quad fastest, so a warp's loads are contiguous runs
+// of NHWC rows. (Round 1 gave each lane one channel and recomputed a 64-bit address and a bounds
+// predicate per scalar load: ~85 instructions per output; ncu: issue-bound at 77 % of issue slots,
+// 29 % of DRAM bandwidth.)
 __device__ __forceinline__ float4 ld4(const float* p, bool ok) {
   return ok ? __ldg(reinterpret_cast<const float4*>(p)) : make_float4(0.f, 0.f, 0.f, 0.f);
 }
 __device__ __forceinline__ void fma4(float4& a, const float4& x, const float4& w) {
   a.x = fmaf(x.x, w.x, a.x); a.y = fmaf(x.y, w.y, a.y); a.z = fmaf(x.z, w.z, a.z); a.w = fmaf(x.w, w.w, a.w);
 }
-// taps t = r * 3 + u of channels c..c+3 (weights [C][3][3]); FLIP reverses the taps (the stride-1
-// data gradient is the forward correlation of dy with the flipped kernel)
+// weights [C][3][3] -> shared [tap][C/4] float4 (FLIP: taps reversed, t -> 8 - t)
 template <bool FLIP>
-__device__ __forceinline__ void load_taps(const float* __restrict__ w, int c, float4 (&k)[9]) {
-#pragma unroll
-  for (int t = 0; t < 9; t++) {
-    const int tt = FLIP ? 8 - t : t;
-    k[t] = make_float4(__ldg(w + (c + 0) * 9 + tt), __ldg(w + (c + 1) * 9 + tt), __ldg(w + (c + 2) * 9 + tt), __ldg(w + (c + 3) * 9 + tt));
+__device__ __forceinline__ void stage_taps(const float* __restrict__ w, int C, float4* wsm) {
+  const int C4 = C / 4;
+  for (int i = threadIdx.x; i < 9 * C4; i += blockDim.x) {
+    const int t = i / C4, q = i % C4, c = q * 4, tt = FLIP ? 8 - t : t;
+    wsm[i] = make_float4(__ldg(w + (c + 0) * 9 + tt), __ldg(w + (c + 1) * 9 + tt), __ldg(w + (c + 2) * 9 + tt), __ldg(w + (c + 3) * 9 + tt));
   }
+  __syncthreads();
 }
+inline int dwq_smem(int C) { return 9 * (C / 4) * 16; }
 
 // y[n,p,q,c] = sum_{r,u} x[n, p*S-1+r, q*S-1+u, c] k[c,r,u]; with FLIP (and S = 1, x = dy) this is
 // the stride-1 data gradient dx[n,h,w,c] = sum_{r,u} dy[n,h+1-r,w+1-u,c] k[c,r,u].
-template <int S, bool FLIP>
+template <int S, bool FLIP, int U>
 __global__ void __launch_bounds__(DW_THREADS) dw_q4_fwd_kernel(const float* __restrict__ x, const float* __restrict__ w,
                                                                float* __restrict__ y, int N, int H, int W, int C, int P, int Q,
                                                                OrionSig sig) {
-  const int C4 = C / 4;
-  const long long items = (long long)N * P * C4;
+  extern __shared__ float4 dwq_w[];
+  stage_taps<FLIP>(w, C, dwq_w);
+  constexpr int NC = (U - 1) * S + 3;
+  const int C4 = C / 4, nseg = (Q + U - 1) / U;
+  const long long items = (long long)N * P * nseg * C4;
   for (long long it = (long long)blockIdx.x * blockDim.x + threadIdx.x; it < items; it += (long long)gridDim.x * blockDim.x) {
-    const int c = (int)(it % C4) * 4;
-    const long long row = it / C4;
+    const int quad = (int)(it % C4);
+    long long t2 = it / C4;
+    const int q0 = (int)(t2 % nseg) * U;
+    const long long row = t2 / nseg;
     const int p = (int)(row % P), n = (int)(row / P);
-    float4 k[9];
-    load_taps<FLIP>(w, c, k);
-    const float* xr[3];
-    bool rv[3];
+    const int c = quad * 4;
+    float4 v[3][NC];
 #pragma unroll
     for (int r = 0; r < 3; r++) {
       const int h = p * S - 1 + r;
-      rv[r] = (unsigned)h < (unsigned)H;
-      xr[r] = x + (((long long)n * H + (rv[r] ? h : 0)) * W) * C + c;
+      const bool rv = (unsigned)h < (unsigned)H;
+      const float* xr = x + (((long long)n * H + (rv ? h : 0)) * W) * C + c;
+#pragma unroll
+      for (int j = 0; j < NC; j++) {
+        const int col = q0 * S - 1 + j;
+        v[r][j] = ld4(xr + (long long)col * C, rv && (unsigned)col < (unsigned)W);
+      }
     }
-    float* yr = y + (((long long)n * P + p) * Q) * C + c;
-    // window columns: a = col q*S-1, b = q*S, cc = q*S+1 (stride 2 also needs q*S+2 = next a)
-    float4 a[3], b[3], e[3];
+    float4 k[9];
 #pragma unroll
-    for (int r = 0; r < 3; r++) { a[r] = make_float4(0.f, 0.f, 0.f, 0.f); b[r] = ld4(xr[r], rv[r] && 0 < W); }
-    auto out = [&](const float4 (&c0)[3], const float4 (&c1)[3], const float4 (&c2)[3], int q) {
-      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int t = 0; t < 9; t++) k[t] = dwq_w[t * C4 + quad];
+    float* yr = y + (((long long)n * P + p) * Q + q0) * C + c;
 #pragma unroll
-      for (int r = 0; r < 3; r++) { fma4(acc, c0[r], k[r * 3]); fma4(acc, c1[r], k[r * 3 + 1]); fma4(acc, c2[r], k[r * 3 + 2]); }
-      *reinterpret_cast<float4*>(yr + (long long)q * C) = acc;
-    };
-    if (S == 1) {
-      // a = col q-1, b = col q; load col q+1 into the third slot; roles rotate a -> b -> e
-      int q = 0;
-      for (; q + 2 < Q; q += 3) {
+    for (int u = 0; u < U; u++) {
+      if (q0 + u < Q) {
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
-        for (int r = 0; r < 3; r++) e[r] = ld4(xr[r] + (long long)(q + 1) * C, rv[r] && q + 1 < W);
-        out(a, b, e, q);
+        for (int r = 0; r < 3; r++)
 #pragma unroll
-        for (int r = 0; r < 3; r++) a[r] = ld4(xr[r] + (long long)(q + 2) * C, rv[r] && q + 2 < W);
-        out(b, e, a, q + 1);
-#pragma unroll
-        for (int r = 0; r < 3; r++) b[r] = ld4(xr[r] + (long long)(q + 3) * C, rv[r] && q + 3 < W);
-        out(e, a, b, q + 2);   // a = col q+2, b = col q+3: exactly the next trip's "q-1" and "q"
-      }
-      for (; q < Q; q++) {
-#pragma unroll
-        for (int r = 0; r < 3; r++) e[r] = ld4(xr[r] + (long long)(q + 1) * C, rv[r] && q + 1 < W);
-        out(a, b, e, q);
-#pragma unroll
-        for (int r = 0; r < 3; r++) { a[r] = b[r]; b[r] = e[r]; }
-      }
-    } else {
-      // stride 2: output q reads cols 2q-1 (a), 2q (b), 2q+1 (e); the next output's 2q+1 is e
-      for (int q = 0; q < Q; q++) {
-#pragma unroll
-        for (int r = 0; r < 3; r++) e[r] = ld4(xr[r] + (long long)(2 * q + 1) * C, rv[r] && 2 * q + 1 < W);
-        out(a, b, e, q);
-#pragma unroll
-        for (int r = 0; r < 3; r++) { a[r] = e[r]; b[r] = ld4(xr[r] + (long long)(2 * q + 2) * C, rv[r] && 2 * q + 2 < W); }
+          for (int t = 0; t < 3; t++) fma4(acc, v[r][u * S + t], k[r * 3 + t]);
+        *reinterpret_cast<float4*>(yr + (long long)u * C) = acc;
       }
     }
   }
@@ -107,51 +90,52 @@ __global__ void __launch_bounds__(DW_THREADS) dw_q4_fwd_kernel(const float* __re
 // Stride-2 data gradient: input row h takes kernel rows r with (h+1-r) even (dy row (h+1-r)/2);
 // along w the pair (2j, 2j+1) reads dy columns j and j+1:
 //   dx(2j) = sum_r dy(p_r, j) k(r,1);  dx(2j+1) = sum_r dy(p_r, j+1) k(r,0) + dy(p_r, j) k(r,2).
-// Thread = (n, h, channel quad); dy column j+1 of one pair is column j of the next.
+// Thread = (channel quad, segment of U pairs, input row): U+1 dy columns of <= 2 rows loaded at once.
+template <int U>
 __global__ void __launch_bounds__(DW_THREADS) dw_q4_dgrad_s2_kernel(const float* __restrict__ dy, const float* __restrict__ w,
                                                                     float* __restrict__ dx, int N, int H, int W, int C, int P, int Q,
                                                                     OrionSig sig) {
-  const int C4 = C / 4;
-  const long long items = (long long)N * H * C4;
+  extern __shared__ float4 dwq_w[];
+  stage_taps<false>(w, C, dwq_w);
+  const int C4 = C / 4, npairs = (W + 1) / 2, nseg = (npairs + U - 1) / U;
+  const long long items = (long long)N * H * nseg * C4;
   for (long long it = (long long)blockIdx.x * blockDim.x + threadIdx.x; it < items; it += (long long)gridDim.x * blockDim.x) {
-    const int c = (int)(it % C4) * 4;
-    const long long row = it / C4;
+    const int quad = (int)(it % C4);
+    long long t2 = it / C4;
+    const int j0 = (int)(t2 % nseg) * U;
+    const long long row = t2 / nseg;
     const int h = (int)(row % H), n = (int)(row / H);
+    const int c = quad * 4;
     // odd h: kernel rows 0 and 2 (dy rows (h+1)/2 and (h-1)/2); even h: kernel row 1 (dy row h/2)
     const bool odd = h & 1;
     const int rsel[2] = {odd ? 0 : 1, 2};
     const int prow[2] = {odd ? (h + 1) / 2 : h / 2, (h - 1) / 2};
-    bool on[2];
-    on[0] = prow[0] < P;
-    on[1] = odd && prow[1] >= 0 && prow[1] < P;
-    float4 k0[2], k1[2], k2[2];
-    const float* gr[2];
+    const bool on[2] = {prow[0] < P, odd && prow[1] >= 0 && prow[1] < P};
+    float4 g[2][U + 1];
 #pragma unroll
     for (int i = 0; i < 2; i++) {
-      const int r = rsel[i];
-      gr[i] = dy + (((long long)n * P + (on[i] ? prow[i] : 0)) * Q) * C + c;
-      k0[i] = make_float4(__ldg(w + c * 9 + r * 3), __ldg(w + (c + 1) * 9 + r * 3), __ldg(w + (c + 2) * 9 + r * 3), __ldg(w + (c + 3) * 9 + r * 3));
-      k1[i] = make_float4(__ldg(w + c * 9 + r * 3 + 1), __ldg(w + (c + 1) * 9 + r * 3 + 1), __ldg(w + (c + 2) * 9 + r * 3 + 1),
-                          __ldg(w + (c + 3) * 9 + r * 3 + 1));
-      k2[i] = make_float4(__ldg(w + c * 9 + r * 3 + 2), __ldg(w + (c + 1) * 9 + r * 3 + 2), __ldg(w + (c + 2) * 9 + r * 3 + 2),
-                          __ldg(w + (c + 3) * 9 + r * 3 + 2));
+      const float* gr = dy + (((long long)n * P + (on[i] ? prow[i] : 0)) * Q) * C + c;
+#pragma unroll
+      for (int j = 0; j <= U; j++) g[i][j] = ld4(gr + (long long)(j0 + j) * C, on[i] && j0 + j < Q);
+    }
+    float4 k0[2], k1[2], k2[2];
+#pragma unroll
+    for (int i = 0; i < 2; i++) {
+      k0[i] = dwq_w[(rsel[i] * 3 + 0) * C4 + quad];
+      k1[i] = dwq_w[(rsel[i] * 3 + 1) * C4 + quad];
+      k2[i] = dwq_w[(rsel[i] * 3 + 2) * C4 + quad];
     }
     float* dr = dx + (((long long)n * H + h) * W) * C + c;
-    float4 cur[2];
 #pragma unroll
-    for (int i = 0; i < 2; i++) cur[i] = ld4(gr[i], on[i] && 0 < Q);
-    const int npairs = (W + 1) / 2;
-    for (int j = 0; j < npairs; j++) {
-      float4 nxt[2];
+    for (int u = 0; u < U; u++) {
+      const int we = 2 * (j0 + u);
+      if (we < W) {
+        float4 e = make_float4(0.f, 0.f, 0.f, 0.f), o = make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
-      for (int i = 0; i < 2; i++) nxt[i] = ld4(gr[i] + (long long)(j + 1) * C, on[i] && j + 1 < Q);
-      float4 e = make_float4(0.f, 0.f, 0.f, 0.f), o = make_float4(0.f, 0.f, 0.f, 0.f);
-#pragma unroll
-      for (int i = 0; i < 2; i++) { fma4(e, cur[i], k1[i]); fma4(o, nxt[i], k0[i]); fma4(o, cur[i], k2[i]); }
-      *reinterpret_cast<float4*>(dr + (long long)(2 * j) * C) = e;
-      if (2 * j + 1 < W) *reinterpret_cast<float4*>(dr + (long long)(2 * j + 1) * C) = o;
-#pragma unroll
-      for (int i = 0; i < 2; i++) cur[i] = nxt[i];
+        for (int i = 0; i < 2; i++) { fma4(e, g[i][u], k1[i]); fma4(o, g[i][u + 1], k0[i]); fma4(o, g[i][u], k2[i]); }
+        *reinterpret_cast<float4*>(dr + (long long)we * C) = e;
+        if (we + 1 < W) *reinterpret_cast<float4*>(dr + (long long)(we + 1) * C) = o;
+      }
     }
   }
   orion_signal(sig);
@@ -191,22 +175,25 @@ __global__ void __launch_bounds__(DW_THREADS, 2) dw_q4_wgrad_kernel(const float*
       float4 f[9];
 #pragma unroll
       for (int t = 0; t < 9; t++) f[t] = make_float4(0.f, 0.f, 0.f, 0.f);
-      float4 a[3], b[3], e[3];
+      // segments of WU outputs: the (WU-1)*S+3 window columns and WU dy quads loaded at once
+      constexpr int WU = 2, NC = (WU - 1) * S + 3;
+      for (int q0 = 0; q0 < Q; q0 += WU) {
+        float4 v[3][NC], g[WU];
 #pragma unroll
-      for (int r = 0; r < 3; r++) { a[r] = make_float4(0.f, 0.f, 0.f, 0.f); b[r] = ld4(xr[r], rv[r] && 0 < W); }
-      for (int q = 0; q < Q; q++) {
+        for (int r = 0; r < 3; r++)
 #pragma unroll
-        for (int r = 0; r < 3; r++) e[r] = ld4(xr[r] + (long long)(q * S + 1) * C, rv[r] && q * S + 1 < W);
-        const float4 g = __ldg(reinterpret_cast<const float4*>(gr + (long long)q * C));
+          for (int j = 0; j < NC; j++) {
+            const int col = q0 * S - 1 + j;
+            v[r][j] = ld4(xr[r] + (long long)col * C, rv[r] && (unsigned)col < (unsigned)W);
+          }
 #pragma unroll
-        for (int r = 0; r < 3; r++) { fma4(f[r * 3], g, a[r]); fma4(f[r * 3 + 1], g, b[r]); fma4(f[r * 3 + 2], g, e[r]); }
-        if (S == 1) {
+        for (int u = 0; u < WU; u++) g[u] = ld4(gr + (long long)(q0 + u) * C, q0 + u < Q);
 #pragma unroll
-          for (int r = 0; r < 3; r++) { a[r] = b[r]; b[r] = e[r]; }
-        } else {
+        for (int u = 0; u < WU; u++)
 #pragma unroll
-          for (int r = 0; r < 3; r++) { a[r] = e[r]; b[r] = ld4(xr[r] + (long long)(q * S + 2) * C, rv[r] && q * S + 2 < W); }
-        }
+          for (int r = 0; r < 3; r++)
+#pragma unroll
+            for (int t = 0; t < 3; t++) fma4(f[r * 3 + t], g[u], v[r][u * S + t]);
       }
 #pragma unroll
       for (int t = 0; t < 9; t++) {
@@ -282,7 +269,7 @@ DwShape dw_shape(const uint64_t* a) {
   s.N = (int)a[3]; s.H = (int)a[4]; s.W = (int)a[5]; s.C = (int)a[6]; s.stride = (int)a[10]; s.P = (int)a[12]; s.Q = (int)a[13];
   return s;
 }
-bool dw_ok(const uint64_t* a) { return (a[6] % 4) == 0 && a[7] == a[6] && a[8] == 3 && a[9] == 3 && a[11] == 1; }
+bool dw_ok(const uint64_t* a) { return (a[6] % 4) == 0 && a[6] <= 2048 && a[7] == a[6] && a[8] == 3 && a[9] == 3 && a[11] == 1; }
 
 void ew(LaunchGeom* g, uint64_t n, const void* f, std::atomic<int>& occ) {
   uint64_t ctas = cdiv(n ? n : 1, DW_THREADS);
@@ -291,13 +278,33 @@ void ew(LaunchGeom* g, uint64_t n, const void* f, std::atomic<int>& occ) {
   g->grid = dim3((unsigned)ctas); g->block = dim3(DW_THREADS); g->smem = 0; g->func = f;
 }
 
+constexpr int DWQ_U1 = 4, DWQ_U2 = 2, DWQ_UP = 4;   // outputs (pairs) per thread item: stride 1 / stride 2 / s2 dgrad
 std::atomic<int> dwq_occ[4];
-void q4_geom(LaunchGeom* g, long long items, const void* f, std::atomic<int>& occ) {
+// shared memory for the staged weights of up to C = 2048 channels (set once per kernel)
+bool dwq_prepare() {
+  static std::atomic<int> done{0};
+  if (done.load(std::memory_order_acquire)) return true;
+  const void* fs[4] = {(const void*)dw_q4_fwd_kernel<1, false, DWQ_U1>, (const void*)dw_q4_fwd_kernel<2, false, DWQ_U2>,
+                       (const void*)dw_q4_fwd_kernel<1, true, DWQ_U1>, (const void*)dw_q4_dgrad_s2_kernel<DWQ_UP>};
+  for (const void* f : fs)
+    if (cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, dwq_smem(2048)) != cudaSuccess) {
+      (void)cudaGetLastError();
+      return false;
+    }
+  done.store(1, std::memory_order_release);
+  return true;
+}
+void q4_geom(LaunchGeom* g, long long items, const void* f, std::atomic<int>& occ, int smem) {
   long long ctas = cdiv(items, DW_THREADS);
-  const long long wave = 148LL * resident_ctas_per_sm(f, DW_THREADS, occ);   // one resident wave (shape heuristic)
+  int b = occ.load(std::memory_order_relaxed);   // resident CTAs per SM (occupancy query with this smem)
+  if (b <= 0) {
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, f, DW_THREADS, smem) != cudaSuccess || b < 1) { (void)cudaGetLastError(); b = 4; }
+    occ.store(b, std::memory_order_relaxed);
+  }
+  const long long wave = 148LL * b;   // one resident wave (shape heuristic, not the partition's count)
   if (ctas > wave) ctas = wave;
   if (ctas < 1) ctas = 1;
-  g->grid = dim3((unsigned)ctas); g->block = dim3(DW_THREADS); g->smem = 0; g->func = f;
+  g->grid = dim3((unsigned)ctas); g->block = dim3(DW_THREADS); g->smem = smem; g->func = f;
 }
 
 int wq_cq(int C) { const int q = C / 4; return q < WQ_MAXQ ? q : WQ_MAXQ; }
@@ -328,35 +335,43 @@ int dw_fwd_geom(const uint64_t* a, LaunchGeom* g) {
   if (!dw_ok(a)) return ORION_E_INVAL;
   DwShape s = dw_shape(a);
   if (s.stride != 1 && s.stride != 2) return ORION_E_INVAL;
-  const long long items = (long long)s.N * s.P * (s.C / 4);
-  if (s.stride == 1) q4_geom(g, items, (const void*)dw_q4_fwd_kernel<1, false>, dwq_occ[0]);
-  else q4_geom(g, items, (const void*)dw_q4_fwd_kernel<2, false>, dwq_occ[1]);
+  if (!dwq_prepare()) return ORION_E_CUDA;
+  const long long items = (long long)s.N * s.P * (s.C / 4) * cdiv(s.Q, s.stride == 1 ? DWQ_U1 : DWQ_U2);
+  if (s.stride == 1) q4_geom(g, items, (const void*)dw_q4_fwd_kernel<1, false, DWQ_U1>, dwq_occ[0], dwq_smem(s.C));
+  else q4_geom(g, items, (const void*)dw_q4_fwd_kernel<2, false, DWQ_U2>, dwq_occ[1], dwq_smem(s.C));
   return 0;
 }
 int dw_fwd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   DwShape s = dw_shape(a);
-  if (g.func == (const void*)dw_q4_fwd_kernel<1, false>)
-    dw_q4_fwd_kernel<1, false><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q, sig);
+  if (g.func == (const void*)dw_q4_fwd_kernel<1, false, DWQ_U1>)
+    dw_q4_fwd_kernel<1, false, DWQ_U1><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C,
+                                                                       s.P, s.Q, sig);
   else
-    dw_q4_fwd_kernel<2, false><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q, sig);
+    dw_q4_fwd_kernel<2, false, DWQ_U2><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C,
+                                                                       s.P, s.Q, sig);
   CHECK_LAUNCH();
 }
 std::atomic<int> dw_dgrad_occ{0};
 int dw_dgrad_geom(const uint64_t* a, LaunchGeom* g) {
   if (!dw_ok(a)) return ORION_E_INVAL;
   DwShape s = dw_shape(a);
-  if (s.stride == 1) q4_geom(g, (long long)s.N * s.H * (s.C / 4), (const void*)dw_q4_fwd_kernel<1, true>, dwq_occ[2]);
-  else if (s.stride == 2) q4_geom(g, (long long)s.N * s.H * (s.C / 4), (const void*)dw_q4_dgrad_s2_kernel, dwq_occ[3]);
+  if ((s.stride == 1 || s.stride == 2) && !dwq_prepare()) return ORION_E_CUDA;
+  if (s.stride == 1)
+    q4_geom(g, (long long)s.N * s.H * (s.C / 4) * cdiv(s.W, DWQ_U1), (const void*)dw_q4_fwd_kernel<1, true, DWQ_U1>, dwq_occ[2], dwq_smem(s.C));
+  else if (s.stride == 2)
+    q4_geom(g, (long long)s.N * s.H * (s.C / 4) * cdiv((s.W + 1) / 2, DWQ_UP), (const void*)dw_q4_dgrad_s2_kernel<DWQ_UP>, dwq_occ[3],
+            dwq_smem(s.C));
   else ew(g, (uint64_t)s.N * s.H * s.W * (s.C / 4), (const void*)dw_dgrad_kernel, dw_dgrad_occ);
   return 0;
 }
 int dw_dgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   DwShape s = dw_shape(a);
-  if (g.func == (const void*)dw_q4_fwd_kernel<1, true>)   // stride-1 dgrad = correlation of dy with the flipped kernel
-    dw_q4_fwd_kernel<1, true><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.P, s.Q, s.C, s.H, s.W,
-                                                          sig);
-  else if (g.func == (const void*)dw_q4_dgrad_s2_kernel)
-    dw_q4_dgrad_s2_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q, sig);
+  if (g.func == (const void*)dw_q4_fwd_kernel<1, true, DWQ_U1>)   // stride-1 dgrad = correlation of dy with the flipped kernel
+    dw_q4_fwd_kernel<1, true, DWQ_U1><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.P, s.Q, s.C,
+                                                                      s.H, s.W, sig);
+  else if (g.func == (const void*)dw_q4_dgrad_s2_kernel<DWQ_UP>)
+    dw_q4_dgrad_s2_kernel<DWQ_UP><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P,
+                                                                  s.Q, sig);
   else
     dw_dgrad_kernel<<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s, sig);
   CHECK_LAUNCH();

@@ -113,23 +113,34 @@ def test_conv_fwd_dgrad_wgrad(shape):
     assert torch.equal(first, dw), "non-deterministic conv wgrad"
 
 
-@pytest.mark.parametrize("n,h,c,st", [(2, 15, 32, 1), (3, 16, 96, 2), (2, 7, 960, 1), (1, 9, 8, 2)])
-def test_depthwise(n, h, c, st):
-    x = si.normal((n, h, h, c), 31)
+@pytest.mark.parametrize("n,h,wd,c,st", [(2, 15, 15, 32, 1), (3, 16, 16, 96, 2), (2, 7, 7, 960, 1), (1, 9, 9, 8, 2),
+                                          (2, 14, 11, 144, 1), (2, 13, 10, 144, 2), (1, 5, 4, 12, 1), (1, 6, 7, 4, 2),
+                                          (3, 28, 28, 192, 2), (1, 1, 1, 16, 1), (1, 2, 3, 8, 2)])
+def test_depthwise(n, h, wd, c, st):
+    """Depthwise 3x3 fwd / dgrad / wgrad (MobileNetV2 shapes incl. C = 144, stride 2, non-square and
+    ragged widths that exercise the 3x unrolled window rotation and its remainder)."""
+    import parity as PT
+    x = si.normal((n, h, wd, c), 31)
     wt = si.normal((c, 3, 3, 1), 32)
-    p = (h + 2 - 3) // st + 1
-    dy = si.normal((n, p, p, c), 33)
-    dims = [n, h, h, c, c, 3, 3, st, 1, p, p]
-    y = torch.zeros(n, p, p, c, device="cuda")
+    p, q = (h + 2 - 3) // st + 1, (wd + 2 - 3) // st + 1
+    dy = si.normal((n, p, q, c), 33)
+    dims = [n, h, wd, c, c, 3, 3, st, 1, p, q]
+    y = torch.zeros(n, p, q, c, device="cuda")
     run("dw_fwd", [dev(x), dev(wt), y] + dims)
-    assert rel(y, om.conv2d_fwd(x, wt, st, 1, c)) < 1e-5
-    dx = torch.zeros(n, h, h, c, device="cuda")
+    PT.assert_close("dw_fwd", y, om.conv2d_fwd(x, wt, st, 1, c), 1e-5)
+    dx = torch.zeros(n, h, wd, c, device="cuda")
     run("dw_dgrad", [dev(dy), dev(wt), dx] + dims)
-    assert rel(dx, om.conv2d_bwd_data(dy, wt, (n, h, h, c), st, 1, c)) < 1e-5
+    PT.assert_close("dw_dgrad", dx, om.conv2d_bwd_data(dy, wt, (n, h, wd, c), st, 1, c), 1e-5)
     dw = torch.zeros(c, 3, 3, 1, device="cuda")
-    wsb = ws(L.lib.orion_dw_wgrad_workspace_bytes(n, c, p, p))
-    run("dw_wgrad", [dev(x), dev(dy), dw] + dims + [wsb, wsb.numel() * 4])
-    assert rel(dw, om.conv2d_bwd_weight(x, dy, (c, 3, 3, 1), st, 1, c)) < 1e-5
+    wsb = ws(L.lib.orion_dw_wgrad_workspace_bytes(n, c, p, q))
+    args = [dev(x), dev(dy), dw] + dims + [wsb, wsb.numel() * 4]
+    run("dw_wgrad", args)
+    ref = om.conv2d_bwd_weight(x, dy, (c, 3, 3, 1), st, 1, c)
+    assert PT.cond_elem(dw, ref, om.conv2d_bwd_weight_abs(x, dy, (c, 3, 3, 1), st, 1, c)) < 1e-5
+    assert PT.rel(dw, ref) < 1e-5
+    first = dw.clone()
+    run("dw_wgrad", args)
+    assert torch.equal(first, dw), "non-deterministic depthwise wgrad"
 
 
 @pytest.mark.parametrize("rows,C", [(4 * 56 * 56, 64), (96 * 7 * 7, 1280), (1000, 24), (12345, 16), (96 * 112 * 112, 32)])
