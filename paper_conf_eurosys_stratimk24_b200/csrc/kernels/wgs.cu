@@ -200,22 +200,45 @@ __global__ void __maxnreg__(MAXREG) wgs_kernel(const __grid_constant__ CUtensorM
     const float* Ls = ring + (size_t)s * stage_floats + lane;
     const float4* Qs = reinterpret_cast<const float4*>(ring + (size_t)s * stage_floats + R * TL);
     const int rows = min(R, k1 - (k0 + it * R));
-#pragma unroll 1
-    for (int r = warp; r < rows; r += NCW) {
-      float lv[MI];
+    // two rows per trip when the register block leaves room (both rows' loads issued before the
+    // first row's FMAs: the LDS latency of one row hides behind the other's arithmetic); the
+    // accumulation order is unchanged (row r, then row r + NCW)
+    constexpr int RU = MI * NB <= 48 ? 2 : 1;
+    auto fma_row = [&](const float (&lv)[MI], const float4 (&qv)[NB / 4]) {
+#pragma unroll
+      for (int j = 0; j < NB / 4; j++)
+#pragma unroll
+        for (int i = 0; i < MI; i++) {
+          acc[i][4 * j] = fmaf(lv[i], qv[j].x, acc[i][4 * j]);
+          acc[i][4 * j + 1] = fmaf(lv[i], qv[j].y, acc[i][4 * j + 1]);
+          acc[i][4 * j + 2] = fmaf(lv[i], qv[j].z, acc[i][4 * j + 2]);
+          acc[i][4 * j + 3] = fmaf(lv[i], qv[j].w, acc[i][4 * j + 3]);
+        }
+    };
+    auto ld_row = [&](int r, float (&lv)[MI], float4 (&qv)[NB / 4]) {
 #pragma unroll
       for (int i = 0; i < MI; i++) lv[i] = Ls[r * TL + 32 * i];
 #pragma unroll
-      for (int j = 0; j < NB / 4; j++) {
-        const float4 q = Qs[r * (NB / 4) + j];
-#pragma unroll
-        for (int i = 0; i < MI; i++) {
-          acc[i][4 * j] = fmaf(lv[i], q.x, acc[i][4 * j]);
-          acc[i][4 * j + 1] = fmaf(lv[i], q.y, acc[i][4 * j + 1]);
-          acc[i][4 * j + 2] = fmaf(lv[i], q.z, acc[i][4 * j + 2]);
-          acc[i][4 * j + 3] = fmaf(lv[i], q.w, acc[i][4 * j + 3]);
-        }
+      for (int j = 0; j < NB / 4; j++) qv[j] = Qs[r * (NB / 4) + j];
+    };
+    int r = warp;
+    if (RU == 2) {
+#pragma unroll 1
+      for (; r + NCW < rows; r += 2 * NCW) {
+        float lv0[MI], lv1[MI];
+        float4 q0[NB / 4], q1[NB / 4];
+        ld_row(r, lv0, q0);
+        ld_row(r + NCW, lv1, q1);
+        fma_row(lv0, q0);
+        fma_row(lv1, q1);
       }
+    }
+#pragma unroll 1
+    for (; r < rows; r += NCW) {
+      float lv[MI];
+      float4 qv[NB / 4];
+      ld_row(r, lv, qv);
+      fma_row(lv, qv);
     }
     __syncwarp();
     if (lane == 0) {
