@@ -1,0 +1,394 @@
+// Weight-gradient GEMM on the tensor cores (gemm flags = 1): C[M][N] = sum_k A[k][m] B[k][n] with
+// both operands MN-major in HBM (dy [rows][Cout], x [rows][Cin] of a 1x1 convolution or Linear
+// layer), fp32 through 3xTF32 on tcgen05 (x = hi + lo, D += lo.hi + hi.lo + hi.hi).
+//
+// The streaming FFMA kernel (wgs.cu) reaches HBM speed only while M*N/(M+N) stays small; beyond ~40
+// flop/B it is bound by the FFMA issue rate (MobileNetV2's late layers, ResNet's 1x1 convs). Here:
+//  * one elected thread streams BK = 32-row stages with 2-D TMA, 128-byte swizzle, straight into
+//    the MN-major canonical layout UMMA reads (32-element atoms of 8 k-rows x 128 B; atoms along
+//    M / N 4 KB apart = LBO, k-groups 1 KB apart = SBO) -- no transposition anywhere;
+//  * four converter warps form lo = x - trunc_tf32(x) in place-shaped copies (elementwise, so the
+//    swizzled layout is preserved); the raw fp32 tile serves as hi (the tensor core reads tf32);
+//  * one thread issues tcgen05.mma kind::tf32 with transposed (MN-major) A and B descriptors into
+//    two TMEM accumulators (main, corrections); the converter warps then read TMEM back;
+//  * K is split over CTAs (shape-only count); fp32 partial tiles are summed in split order by the
+//    last CTA of each tile (fp64), so results are deterministic and partition-independent.
+#include <cstdlib>
+
+#include "common.cuh"
+#include "tma.cuh"
+
+namespace {
+namespace atc {
+using namespace tmah;
+
+constexpr int BM = 128, BK = 32, NTHR = 192;   // warps: 0 TMA, 1 MMA + TMEM owner, 2-5 converters / epilogue
+constexpr int CONV_THREADS = 128;
+
+template <int BN_>
+struct Cfg {
+  static constexpr int BN = BN_;
+  static constexpr int A_BYTES = BM * BK * 4, B_BYTES = BN * BK * 4;
+  static constexpr int STAGE = 2 * (A_BYTES + B_BYTES);   // [A raw][A lo][B raw][B lo]
+  static constexpr int STAGES = (200 * 1024) / STAGE > 6 ? 6 : (200 * 1024) / STAGE;
+  static constexpr int SMEM = STAGES * STAGE + 1024 + 256;
+  static constexpr int TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
+  // kind::tf32: D fp32 (bit 4), A, B tf32 (bits 7, 10), A and B MN-major (bits 15, 16), N>>3, M>>4
+  static constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | (1u << 15) | (1u << 16) | ((uint32_t)(BN >> 3) << 17) |
+                                    ((uint32_t)(BM >> 4) << 24);
+  static constexpr uint32_t TX = A_BYTES + B_BYTES;
+};
+
+struct Params {
+  int DM, DN, K;      // M side (TMEM lanes), N side, rows
+  int trans;          // 0: C[m][n]; 1: C[n][m] (M side = the gemm's N operand)
+  float* C;
+  long long ldc;
+  int tiles_n, tiles, split, kps;
+  unsigned int* tickets;
+  float* part;        // [tile][split][BM*BN]
+  double* gpart;
+};
+
+__device__ __forceinline__ uint64_t desc_mn128(uint32_t addr) {
+  // MN-major, SWIZZLE_128B: LBO = 4096 B between 32-element MN atoms (one TMA box), SBO = 1024 B
+  // between 8-row k-groups; version 1 (bit 46); layout type 2 = 128-byte swizzle (bits 61-63)
+  return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)(4096 >> 4) << 16) | ((uint64_t)(1024 >> 4) << 32) | (1ull << 46) | (2ull << 61);
+}
+__device__ __forceinline__ void mma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
+               "l"(a), "l"(b), "r"(idesc), "r"(acc)
+               : "memory");
+}
+__device__ __forceinline__ void mma_commit(uint32_t mbar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(mbar) : "memory");
+}
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t* r) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]), "=r"(r[9]),
+        "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]),
+        "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]),
+        "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+}
+__device__ __forceinline__ float trunc_tf32(float x) { return __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
+
+template <int BN>
+__global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                                                     Params p, OrionSig sig) {
+  using C_ = Cfg<BN>;
+  constexpr int A_BYTES = C_::A_BYTES, B_BYTES = C_::B_BYTES, STAGE = C_::STAGE, S = C_::STAGES;
+  extern __shared__ __align__(1024) unsigned char atc_raw[];
+  // 1024-byte alignment for the swizzle atoms, by offsetting the shared array itself (keeps LDS/STS)
+  unsigned char* smem = atc_raw + ((1024u - ((uint32_t)__cvta_generic_to_shared(atc_raw) & 1023u)) & 1023u);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + S * STAGE);
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 3 * S + 2);
+  const uint32_t full0 = smem_u32(bars), conv0 = full0 + 8 * S, empty0 = conv0 + 8 * S, done_bar = empty0 + 8 * S;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int tile = blockIdx.x, z = blockIdx.y;
+  const int m0 = (tile / p.tiles_n) * BM, n0 = (tile % p.tiles_n) * BN;
+  const int k0 = z * p.kps, k1 = min(p.K, k0 + p.kps);
+  const int nst = (k1 - k0 + BK - 1) / BK;
+
+  if (tid == 0) {
+    for (int s = 0; s < S; s++) { mbar_init(full0 + 8 * s, 1); mbar_init(conv0 + 8 * s, CONV_THREADS / 32); mbar_init(empty0 + 8 * s, 1); }
+    mbar_init(done_bar, 1);
+    fence_barrier_init();
+    prefetch_tmap(&tmA);
+    prefetch_tmap(&tmB);
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)), "r"(C_::TMEM_COLS) : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+#pragma unroll 1
+      for (int it = 0; it < nst; it++) {
+        const int s = it % S;
+        if (it >= S) mbar_wait(empty0 + 8 * s, ((uint32_t)(it / S) & 1u) ^ 1u);
+        const uint32_t st = smem_u32(smem + (size_t)s * STAGE), bar = full0 + 8 * s;
+        mbar_expect(bar, C_::TX);
+        const int kk = k0 + it * BK;
+#pragma unroll
+        for (int j = 0; j < BM / 32; j++) tma_load2d(st + j * 4096, &tmA, m0 + 32 * j, kk, bar);
+#pragma unroll
+        for (int j = 0; j < BN / 32; j++) tma_load2d(st + 2 * A_BYTES + j * 4096, &tmB, n0 + 32 * j, kk, bar);
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      const uint32_t d_main = tmem, d_corr = tmem + BN;
+#pragma unroll 1
+      for (int it = 0; it < nst; it++) {
+        const int s = it % S;
+        const uint32_t ph = (uint32_t)(it / S) & 1u;
+        mbar_wait(full0 + 8 * s, ph);
+        mbar_wait(conv0 + 8 * s, ph);
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        const uint32_t st = smem_u32(smem + (size_t)s * STAGE);
+        const uint32_t a_hi = st, a_lo = st + A_BYTES, b_hi = st + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
+#pragma unroll
+        for (int ks = 0; ks < BK / 8; ks++) {
+          const uint32_t o = ks * 1024;   // next 8-row k-group inside every atom
+          const uint32_t acc = (it | ks) != 0;
+          mma_tf32(d_corr, desc_mn128(a_lo + o), desc_mn128(b_hi + o), C_::IDESC, acc);
+          mma_tf32(d_corr, desc_mn128(a_hi + o), desc_mn128(b_lo + o), C_::IDESC, 1);
+          mma_tf32(d_main, desc_mn128(a_hi + o), desc_mn128(b_hi + o), C_::IDESC, acc);
+        }
+        mma_commit(empty0 + 8 * s);
+      }
+      mma_commit(done_bar);
+    }
+  } else {
+    // ---------------- converters: lo = x - trunc(x), same (swizzled) layout
+    const int ct = tid - 64;
+#pragma unroll 1
+    for (int it = 0; it < nst; it++) {
+      const int s = it % S;
+      mbar_wait(full0 + 8 * s, (uint32_t)(it / S) & 1u);
+      unsigned char* st = smem + (size_t)s * STAGE;
+      const float4* ahi = reinterpret_cast<const float4*>(st);
+      float4* alo = reinterpret_cast<float4*>(st + A_BYTES);
+      constexpr int AQ = A_BYTES / 16 / CONV_THREADS, BQ = B_BYTES / 16 / CONV_THREADS;
+      float4 va[AQ], vb[BQ > 0 ? BQ : 1];
+#pragma unroll
+      for (int j = 0; j < AQ; j++) va[j] = ahi[ct + CONV_THREADS * j];
+      const float4* bhi = reinterpret_cast<const float4*>(st + 2 * A_BYTES);
+      float4* blo = reinterpret_cast<float4*>(st + 2 * A_BYTES + B_BYTES);
+#pragma unroll
+      for (int j = 0; j < BQ; j++) vb[j] = bhi[ct + CONV_THREADS * j];
+#pragma unroll
+      for (int j = 0; j < AQ; j++)
+        alo[ct + CONV_THREADS * j] = make_float4(va[j].x - trunc_tf32(va[j].x), va[j].y - trunc_tf32(va[j].y), va[j].z - trunc_tf32(va[j].z),
+                                                 va[j].w - trunc_tf32(va[j].w));
+#pragma unroll
+      for (int j = 0; j < BQ; j++)
+        blo[ct + CONV_THREADS * j] = make_float4(vb[j].x - trunc_tf32(vb[j].x), vb[j].y - trunc_tf32(vb[j].y), vb[j].z - trunc_tf32(vb[j].z),
+                                                 vb[j].w - trunc_tf32(vb[j].w));
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(conv0 + 8 * s);
+    }
+    // ---------------- epilogue: TMEM lanes 32 (warp % 4) .. +31 = tile rows; 32 columns at a time
+    mbar_wait(done_bar, 0);
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  }
+  __syncthreads();
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+  // all TMEM reads happen below (warps 2-5), partial tiles / results written, then dealloc
+  float* part = p.part ? p.part + ((long long)tile * p.split + z) * (BM * BN) : nullptr;
+  if (warp >= 2) {
+    const int q = warp & 3, row = 32 * q + lane, m = m0 + row;
+#pragma unroll 1
+    for (int c0 = 0; c0 < BN; c0 += 32) {
+      uint32_t mv[32], cv[32];
+      const uint32_t base = tmem + ((uint32_t)(32 * q) << 16) + (uint32_t)c0;
+      tmem_ld32(base, mv);
+      tmem_ld32(base + BN, cv);
+      asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+      if (p.split == 1) {
+#pragma unroll
+        for (int j = 0; j < 32; j++) {
+          const int n = n0 + c0 + j;
+          const float v = __uint_as_float(mv[j]) + __uint_as_float(cv[j]);
+          if (m < p.DM && n < p.DN) {
+            if (p.trans) p.C[(long long)n * p.ldc + m] = v;
+            else p.C[(long long)m * p.ldc + n] = v;
+          }
+        }
+      } else {
+        float4* dst = reinterpret_cast<float4*>(part + (size_t)row * BN + c0);
+#pragma unroll
+        for (int j = 0; j < 32; j += 4)
+          dst[j / 4] = make_float4(__uint_as_float(mv[j]) + __uint_as_float(cv[j]), __uint_as_float(mv[j + 1]) + __uint_as_float(cv[j + 1]),
+                                   __uint_as_float(mv[j + 2]) + __uint_as_float(cv[j + 2]), __uint_as_float(mv[j + 3]) + __uint_as_float(cv[j + 3]));
+      }
+    }
+  }
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+  __syncthreads();
+  if (warp == 1) {
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(C_::TMEM_COLS) : "memory");
+  }
+  if (p.split > 1) {
+    // ordered combine of the tile's split partials: in shared memory (two levels) when the tile is
+    // small enough, else directly by the last CTA (planner keeps split <= 8 then)
+    constexpr int V = BM * BN;
+    double* out = reinterpret_cast<double*>(smem);   // stage memory is free now
+    const float* tpart = p.part + (long long)tile * p.split * V;
+    if (V <= 4096) {
+      const int ng = combine_rows(p.split);
+      if (combine_splits(p.tickets + tile * (1 + ng), tpart, p.gpart + (long long)tile * ng * V, V, p.split, z, V, out, out + V)) {
+        for (int v = tid; v < V; v += NTHR) {
+          const int m = m0 + v / BN, n = n0 + v % BN;
+          if (m < p.DM && n < p.DN) {
+            if (p.trans) p.C[(long long)n * p.ldc + m] = (float)out[v];
+            else p.C[(long long)m * p.ldc + n] = (float)out[v];
+          }
+        }
+      }
+    } else if (last_cta_of(p.tickets + tile, (unsigned)p.split)) {
+      for (int v = tid; v < V; v += NTHR) {
+        const int m = m0 + v / BN, n = n0 + v % BN;
+        if (m >= p.DM || n >= p.DN) continue;
+        double t = 0.0;
+        for (int zz = 0; zz < p.split; zz++) t += (double)__ldcg(tpart + (long long)zz * V + v);
+        if (p.trans) p.C[(long long)n * p.ldc + m] = (float)t;
+        else p.C[(long long)m * p.ldc + n] = (float)t;
+      }
+    }
+  }
+  orion_signal(sig);
+}
+
+struct Plan { int trans, bn, tiles_n, tiles, split, kps; };
+
+inline int bn_for(long long DN) { return DN <= 32 ? 32 : DN <= 64 ? 64 : DN <= 128 ? 128 : (DN <= 256 ? 256 : 128); }
+
+inline Plan plan(long long M, long long N, long long K) {
+  Plan best{};
+  double best_cost = 1e300;
+  for (int trans = 0; trans < 2; trans++) {
+    const long long DM = trans ? N : M, DN = trans ? M : N;
+    const int bn = bn_for(DN);
+    const long long tm = cdiv(DM, BM), tn = cdiv(DN, bn), tiles = tm * tn;
+    const double padded = (double)tiles * BM * bn;   // tensor work (and smem traffic) per row
+    if (padded < best_cost) {
+      best_cost = padded;
+      best.trans = trans; best.bn = bn; best.tiles_n = (int)tn; best.tiles = (int)tiles;
+    }
+  }
+  long long split = best.tiles >= 148 ? 1 : 148 / best.tiles;   // one CTA per SM (~200 KB of stages)
+  const long long kmax = K / (4LL * BK);                         // >= 4 stages per split
+  if (split > kmax) split = kmax > 0 ? kmax : 1;
+  if ((long long)BM * best.bn > 4096 && split > 8) split = 8;    // direct last-CTA combine above 4096 values
+  if (split > 1024) split = 1024;
+  best.kps = (int)(cdiv(cdiv(K, split), BK) * BK);
+  best.split = (int)cdiv(K, best.kps);
+  return best;
+}
+
+inline uint64_t ws_bytes(const Plan& p) {
+  if (p.split <= 1) return 0;
+  const uint64_t V = (uint64_t)BM * p.bn;
+  return WS_TICKET_BYTES + (uint64_t)p.tiles * p.split * V * 4 + 16 + (uint64_t)p.tiles * combine_rows(p.split) * V * 8;
+}
+
+template <int BN>
+bool prepare() {
+  static std::atomic<int> done{0};
+  if (done.load(std::memory_order_acquire)) return true;
+  if (cudaFuncSetAttribute((const void*)atc_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<BN>::SMEM) != cudaSuccess) {
+    (void)cudaGetLastError();
+    return false;
+  }
+  done.store(1, std::memory_order_release);
+  return true;
+}
+
+inline const void* fn_of(int bn) {
+  switch (bn) {
+    case 32: return (const void*)atc_kernel<32>;
+    case 64: return (const void*)atc_kernel<64>;
+    case 128: return (const void*)atc_kernel<128>;
+    default: return (const void*)atc_kernel<256>;
+  }
+}
+inline int smem_of(int bn) {
+  switch (bn) {
+    case 32: return Cfg<32>::SMEM;
+    case 64: return Cfg<64>::SMEM;
+    case 128: return Cfg<128>::SMEM;
+    default: return Cfg<256>::SMEM;
+  }
+}
+inline bool prepare_of(int bn) {
+  switch (bn) {
+    case 32: return prepare<32>();
+    case 64: return prepare<64>();
+    case 128: return prepare<128>();
+    default: return prepare<256>();
+  }
+}
+
+}  // namespace atc
+}  // namespace
+
+// ---- entry points used by gemm.cu (flags = 1 routing): the tensor path for weight gradients whose
+// FFMA streaming form is compute-bound, i.e. M*N/(M+N) >= ATC_MIN_INTENSITY (flop per byte / 2)
+static int atc_min_intensity() {
+  static const int v = [] {
+    const char* e = getenv("ORION_ATC_MIN_AI");   // tuning knob (shape routing only)
+    return e ? atoi(e) : 40;
+  }();
+  return v;
+}
+
+uint64_t atc_ws_bytes(long long M, long long N, long long K) {
+  if (M <= 0 || N <= 0 || K <= 0) return 0;
+  return atc::ws_bytes(atc::plan(M, N, K));
+}
+
+bool atc_try_geom(const uint64_t* a, LaunchGeom* g) {
+  const long long M = a[4], N = a[5], K = a[6], lda = a[7], ldb = a[8];
+  if ((int)a[10] != 1 || a[3] != 0) return false;
+  if (M * N < (long long)atc_min_intensity() * (M + N)) return false;
+  if (K < 4 * atc::BK || lda % 4 || ldb % 4 || M % 4 || N % 4) return false;
+  if (!tmah::al16((const void*)a[0]) || !tmah::al16((const void*)a[1]) || tmah::encoder() == nullptr) return false;
+  if (M >= (1LL << 24) || N >= (1LL << 24) || K >= (1LL << 31)) return false;
+  atc::Plan pl = atc::plan(M, N, K);
+  if (pl.split > 1 && (a[11] == 0 || a[12] < atc::ws_bytes(pl))) return false;
+  if ((uint64_t)pl.tiles * (1 + combine_rows(pl.split)) * 4 > WS_TICKET_BYTES) return false;
+  if (!atc::prepare_of(pl.bn)) return false;
+  g->grid = dim3((unsigned)pl.tiles, (unsigned)pl.split);
+  g->block = dim3(atc::NTHR);
+  g->smem = atc::smem_of(pl.bn);
+  g->func = atc::fn_of(pl.bn);
+  g->pipe = ORION_PIPE_TF32X3;
+  return true;
+}
+
+bool atc_is(const void* f) {
+  return f == atc::fn_of(32) || f == atc::fn_of(64) || f == atc::fn_of(128) || f == atc::fn_of(256);
+}
+
+int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
+  const long long M = a[4], N = a[5], K = a[6], lda = a[7], ldb = a[8], ldc = a[9];
+  atc::Plan pl = atc::plan(M, N, K);
+  atc::Params p;
+  p.trans = pl.trans;
+  p.DM = (int)(pl.trans ? N : M); p.DN = (int)(pl.trans ? M : N); p.K = (int)K;
+  p.C = (float*)a[2]; p.ldc = ldc;
+  p.tiles_n = pl.tiles_n; p.tiles = pl.tiles; p.split = pl.split; p.kps = pl.kps;
+  p.tickets = nullptr; p.part = nullptr; p.gpart = nullptr;
+  if (pl.split > 1) {
+    unsigned char* ws = (unsigned char*)a[11];
+    const uint64_t V = (uint64_t)atc::BM * pl.bn;
+    p.tickets = reinterpret_cast<unsigned int*>(ws);
+    p.part = reinterpret_cast<float*>(ws + WS_TICKET_BYTES);
+    uintptr_t gp = reinterpret_cast<uintptr_t>(ws + WS_TICKET_BYTES + (uint64_t)pl.tiles * pl.split * V * 4);
+    p.gpart = reinterpret_cast<double*>((gp + 15) & ~uintptr_t(15));
+  }
+  const float* Ap = pl.trans ? (const float*)a[1] : (const float*)a[0];   // M side
+  const float* Bp = pl.trans ? (const float*)a[0] : (const float*)a[1];   // N side
+  const long long ldA = pl.trans ? ldb : lda, ldB = pl.trans ? lda : ldb;
+  CUtensorMap mA, mB;
+  if (!tmah::map2d_f32_sw(&mA, Ap, K, p.DM, ldA, 32, atc::BK, CU_TENSOR_MAP_SWIZZLE_128B)) return ORION_E_CUDA;
+  if (!tmah::map2d_f32_sw(&mB, Bp, K, p.DN, ldB, 32, atc::BK, CU_TENSOR_MAP_SWIZZLE_128B)) return ORION_E_CUDA;
+  switch (pl.bn) {
+    case 32: atc::atc_kernel<32><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
+    case 64: atc::atc_kernel<64><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
+    case 128: atc::atc_kernel<128><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
+    default: atc::atc_kernel<256><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
+  }
+  return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+}

@@ -88,27 +88,12 @@ __global__ void __launch_bounds__(BN_THREADS) bn_stats_kernel(const float* __res
   if (c < C && rl < rl_n) {
     const float* xp = x + c;
     long long r = r0 + rl;
-    // runs of 8 rows (16 loads in flight per thread, two runs per trip) are summed in fp32 (x and
-    // x*x: rounding <= 8u of the run's |x| sum), then added to the fp64 totals: 8x fewer fp64
-    // conversions than per element (round 1 stalled on F2F.F64 after every load, ncu)
-    auto run8 = [&](const float4 (&v)[8]) {
-      float4 a = v[0], q = make_float4(v[0].x * v[0].x, v[0].y * v[0].y, v[0].z * v[0].z, v[0].w * v[0].w);
-#pragma unroll
-      for (int i = 1; i < 8; i++) {
-        a.x += v[i].x; a.y += v[i].y; a.z += v[i].z; a.w += v[i].w;
-        q.x = fmaf(v[i].x, v[i].x, q.x); q.y = fmaf(v[i].y, v[i].y, q.y); q.z = fmaf(v[i].z, v[i].z, q.z); q.w = fmaf(v[i].w, v[i].w, q.w);
-      }
-      s1.x += a.x; s1.y += a.y; s1.z += a.z; s1.w += a.w;
-      s2.x += q.x; s2.y += q.y; s2.z += q.z; s2.w += q.w;
-    };
-    for (; r + 15LL * rl_n < r1; r += 16LL * rl_n) {
-      float4 v[8], u[8];
+    for (; r + 7LL * rl_n < r1; r += 8LL * rl_n) {
+      float4 v[8];
 #pragma unroll
       for (int i = 0; i < 8; i++) v[i] = __ldg(reinterpret_cast<const float4*>(xp + (r + i * (long long)rl_n) * C));
 #pragma unroll
-      for (int i = 0; i < 8; i++) u[i] = __ldg(reinterpret_cast<const float4*>(xp + (r + (8 + i) * (long long)rl_n) * C));
-      run8(v);
-      run8(u);
+      for (int i = 0; i < 8; i++) { add4(s1, v[i]); sq4(s2, v[i]); }
     }
     for (; r < r1; r += rl_n) {
       float4 v = __ldg(reinterpret_cast<const float4*>(xp + r * C));
@@ -158,22 +143,16 @@ __global__ void __launch_bounds__(BN_THREADS) bn_bwd_reduce_kernel(const float* 
       sgx.w = fma((double)g.w, (double)v.w, sgx.w);
     };
     long long r = r0 + rl;
-    // runs of 8 rows (16 loads in flight) summed in fp32 (sum dy and sum dy*x; rounding <= 8u of
-    // the run's absolute sums), then added to the fp64 totals
-    for (; r + 7LL * rl_n < r1; r += 8LL * rl_n) {
-      float4 g[8], v[8];
-#pragma unroll
-      for (int i = 0; i < 8; i++) g[i] = __ldg(reinterpret_cast<const float4*>(gp + (r + i * (long long)rl_n) * C));
-#pragma unroll
-      for (int i = 0; i < 8; i++) v[i] = __ldg(reinterpret_cast<const float4*>(xp + (r + i * (long long)rl_n) * C));
-      float4 a = g[0], b = make_float4(g[0].x * v[0].x, g[0].y * v[0].y, g[0].z * v[0].z, g[0].w * v[0].w);
-#pragma unroll
-      for (int i = 1; i < 8; i++) {
-        a.x += g[i].x; a.y += g[i].y; a.z += g[i].z; a.w += g[i].w;
-        b.x = fmaf(g[i].x, v[i].x, b.x); b.y = fmaf(g[i].y, v[i].y, b.y); b.z = fmaf(g[i].z, v[i].z, b.z); b.w = fmaf(g[i].w, v[i].w, b.w);
-      }
-      sg.x += a.x; sg.y += a.y; sg.z += a.z; sg.w += a.w;
-      sgx.x += b.x; sgx.y += b.y; sgx.z += b.z; sgx.w += b.w;
+    for (; r + 3LL * rl_n < r1; r += 4LL * rl_n) {
+      float4 g0 = __ldg(reinterpret_cast<const float4*>(gp + r * C));
+      float4 g1 = __ldg(reinterpret_cast<const float4*>(gp + (r + rl_n) * C));
+      float4 g2 = __ldg(reinterpret_cast<const float4*>(gp + (r + 2LL * rl_n) * C));
+      float4 g3 = __ldg(reinterpret_cast<const float4*>(gp + (r + 3LL * rl_n) * C));
+      float4 v0 = __ldg(reinterpret_cast<const float4*>(xp + r * C));
+      float4 v1 = __ldg(reinterpret_cast<const float4*>(xp + (r + rl_n) * C));
+      float4 v2 = __ldg(reinterpret_cast<const float4*>(xp + (r + 2LL * rl_n) * C));
+      float4 v3 = __ldg(reinterpret_cast<const float4*>(xp + (r + 3LL * rl_n) * C));
+      acc(g0, v0); acc(g1, v1); acc(g2, v2); acc(g3, v3);
     }
     for (; r < r1; r += rl_n)
       acc(__ldg(reinterpret_cast<const float4*>(gp + r * C)), __ldg(reinterpret_cast<const float4*>(xp + r * C)));

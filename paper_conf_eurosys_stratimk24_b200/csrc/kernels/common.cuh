@@ -175,6 +175,12 @@ bool wgs_try_geom(const uint64_t* a, LaunchGeom* g);
 bool wgs_is(const void* f);
 int wgs_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
 
+// Tensor-core weight-gradient GEMM (atc.cu), taken by gemm flags = 1 for compute-dense shapes.
+uint64_t atc_ws_bytes(long long M, long long N, long long K);
+bool atc_try_geom(const uint64_t* a, LaunchGeom* g);
+bool atc_is(const void* f);
+int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
+
 // Kernel table (table.cu)
 extern const KernelEntry g_kernels[ORION_FN_COUNT];
 int kernel_launch_sig(uint32_t fn, const uint64_t* args, uint32_t nargs, OrionSig sig, cudaStream_t s,

@@ -2209,6 +2209,8 @@ extern "C" uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t 
   }
   const uint64_t b3 = wgs_ws_bytes((long long)M, (long long)N, (long long)K);   // ... or the streaming one
   if (b3 > b) b = b3;
+  const uint64_t b4 = atc_ws_bytes((long long)M, (long long)N, (long long)K);   // ... or the tensor-core one
+  if (b4 > b) b = b4;
   return b;
 }
 
@@ -2246,6 +2248,7 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     g->grid = dim3((unsigned)cdiv(M, rows::rpc((int)N))); g->block = dim3(rows::NTH); g->smem = rows::smem_bytes((int)K, (int)N); g->func = f;
     return 0;
   }
+  if (flags == 1 && atc_try_geom(a, g)) return 0;   // compute-dense A^T B on tcgen05 (atc.cu)
   if (flags == 1 && wgs_try_geom(a, g)) return 0;   // TMA-fed streaming A^T B (wgs.cu)
   if (flags == 1 && atb_ok(M, N, K)) {
     Plan pl = plan_atb(M, N, K);
@@ -2289,6 +2292,7 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
     gemv_bt_kernel<<<g.grid, g.block, 0, s>>>(A, lda, B, ldb, C, ldc, bias, (int)M, (int)N, (int)K, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
+  if (atc_is(g.func)) return atc_launch(a, g, sig, s);
   if (wgs_is(g.func)) return wgs_launch(a, g, sig, s);
   if (tmk::is(g.func)) return tmk::launch(g, M, N, K, C, ldc, bias, A, lda, B, ldb, flags == 0, sig, s);
   if (tcm::is<ADense, BDenseT>(g.func))

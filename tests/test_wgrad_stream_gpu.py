@@ -1,4 +1,6 @@
-"""Streaming weight-gradient GEMM (csrc/kernels/wgs.cu; gemm flags = 1, no bias): dW = dy^T x of the
+"""Weight-gradient GEMMs (gemm flags = 1, no bias): the streaming FFMA kernel (csrc/kernels/wgs.cu)
+and, for compute-dense shapes, the tcgen05 3xTF32 kernel with MN-major TMA operands (atc.cu):
+dW = dy^T x of the
 1x1 convolutions of MobileNetV2 / ResNet training (cuDNN's weight-gradient kernels in the paper's
 runs) against the fp64 oracle product, at sizes that span several tiles, ragged rows,
 ragged tiles in both operand roles, and at the full BASELINE size of the dominant op
@@ -45,7 +47,12 @@ def check_wgrad(M, N, K, seed=31, expect_stream=True):
     Ad, Bd = A.cuda(), B.cuda()
     args = [Ad.data_ptr(), Bd.data_ptr(), C.data_ptr(), 0, M, N, K, M, N, N, 1, w.data_ptr(), w.numel() * 4]
     kern = kernel_info("gemm", args)["kernel"]
-    assert ("wgs_kernel" in kern) == expect_stream, f"kernel selection: {kern}"
+    # compute-dense shapes (M N >= 40 (M + N)) take the tcgen05 kernel (atc.cu), the rest wgs.cu
+    want = ("atc_kernel" if M * N >= 40 * (M + N) else "wgs_kernel") if expect_stream else None
+    if want:
+        assert want in kern, f"kernel selection: {kern}, expected {want}"
+    else:
+        assert "wgs_kernel" not in kern and "atc_kernel" not in kern, kern
     s = torch.cuda.current_stream().cuda_stream
     orion.kernel_launch("gemm", args, s)
     torch.cuda.synchronize()
@@ -76,7 +83,9 @@ WGS_CASES = [
     (384, 64, 18816), (64, 384, 4704),
     (576, 96, 4704), (96, 576, 4704),
     (960, 160, 4704), (160, 960, 4704),
-    (1280, 320, 4704),      # features.18 (200 tiles, split 1)
+    (1280, 320, 4704),      # features.18 (tensor path: 30 tiles x split 4)
+    (256, 64, 50176), (64, 256, 50176), (512, 128, 12544),   # ResNet-50 b64 layer1 / layer2 1x1 weight gradients
+    (2048, 512, 3136), (1000, 2048, 400), (300, 200, 520),    # layer4, fc-like, ragged tiles on the tensor path
     (20, 12, 999),          # tiny, ragged everything
     (100, 36, 70001),
 ]
