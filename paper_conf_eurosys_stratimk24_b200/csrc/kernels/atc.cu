@@ -48,12 +48,16 @@ struct Params {
   unsigned int* tickets;
   float* part;        // [tile][split][BM*BN]
   double* gpart;
+  double* fin;        // [tile][BM*BN] fp64 sums of the splits
+  int dbg;            // ORION_ATC_DBG (bring-up only): 1 = write stage-0 A tile as decoded from smem
 };
 
 __device__ __forceinline__ uint64_t desc_mn128(uint32_t addr) {
-  // MN-major, SWIZZLE_128B: LBO = 4096 B between 32-element MN atoms (one TMA box), SBO = 1024 B
-  // between 8-row k-groups; version 1 (bit 46); layout type 2 = 128-byte swizzle (bits 61-63)
-  return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)(4096 >> 4) << 16) | ((uint64_t)(1024 >> 4) << 32) | (1ull << 46) | (2ull << 61);
+  // MN-major tf32 operands need the 128-byte swizzle with 32-byte atoms (SWIZZLE_128B_BASE32B,
+  // layout type 1; TMA CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B): atoms of 4 k-rows x 128 B (32 tf32
+  // along M / N). LBO = 4096 B between MN atoms (one TMA box), SBO = 512 B between 4-row k-groups;
+  // version 1 (bit 46). (The 16-byte-granular SWIZZLE_128B layout reads as zeros for MN-major tf32.)
+  return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)(4096 >> 4) << 16) | ((uint64_t)(512 >> 4) << 32) | (1ull << 46) | (1ull << 61);
 }
 __device__ __forceinline__ void mma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
   asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
@@ -135,13 +139,22 @@ __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CU
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t st = smem_u32(smem + (size_t)s * STAGE);
         const uint32_t a_hi = st, a_lo = st + A_BYTES, b_hi = st + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
+        uint32_t idesc = C_::IDESC;
+        if (p.dbg == 2) idesc &= ~((1u << 15) | (1u << 16));
 #pragma unroll
         for (int ks = 0; ks < BK / 8; ks++) {
           const uint32_t o = ks * 1024;   // next 8-row k-group inside every atom
           const uint32_t acc = (it | ks) != 0;
-          mma_tf32(d_corr, desc_mn128(a_lo + o), desc_mn128(b_hi + o), C_::IDESC, acc);
-          mma_tf32(d_corr, desc_mn128(a_hi + o), desc_mn128(b_lo + o), C_::IDESC, 1);
-          mma_tf32(d_main, desc_mn128(a_hi + o), desc_mn128(b_hi + o), C_::IDESC, acc);
+          if (p.dbg == 3) {   // bring-up: K-major SW128 descriptors (wrong data, must still write)
+            auto dk = [](uint32_t addr) {
+              return (uint64_t)((addr >> 4) & 0x3FFF) | (1ull << 16) | ((uint64_t)(1024 >> 4) << 32) | (1ull << 46) | (2ull << 61);
+            };
+            mma_tf32(d_main, dk(a_hi + 32 * ks), dk(b_hi + 32 * ks), idesc & ~((1u << 15) | (1u << 16)), acc);
+            continue;
+          }
+          mma_tf32(d_corr, desc_mn128(a_lo + o), desc_mn128(b_hi + o), idesc, acc);
+          mma_tf32(d_corr, desc_mn128(a_hi + o), desc_mn128(b_lo + o), idesc, 1);
+          mma_tf32(d_main, desc_mn128(a_hi + o), desc_mn128(b_hi + o), idesc, acc);
         }
         mma_commit(empty0 + 8 * s);
       }
@@ -185,7 +198,16 @@ __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CU
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   // all TMEM reads happen below (warps 2-5), partial tiles / results written, then dealloc
   float* part = p.part ? p.part + ((long long)tile * p.split + z) * (BM * BN) : nullptr;
-  if (warp >= 2) {
+  if (p.dbg == 1 && warp >= 2) {
+    // C[m][k] = A element (m, k) of stage 0 read back through the SW128 MN-major atom layout
+    const int q = warp & 3, row = 32 * q + lane;
+    const unsigned char* st = smem;
+    for (int k = 0; k < BK; k++) {
+      const int atom = row / 32, mi = row % 32;
+      const uint32_t off = atom * 4096 + (k / 8) * 1024 + (k % 8) * 128 + ((((mi * 4) / 16) ^ (k % 8)) << 4) + (mi * 4) % 16;
+      if (m0 + row < p.DM && k < p.DN) p.C[(long long)(m0 + row) * p.ldc + k] = *reinterpret_cast<const float*>(st + off);
+    }
+  } else if (warp >= 2) {
     const int q = warp & 3, row = 32 * q + lane, m = m0 + row;
 #pragma unroll 1
     for (int c0 = 0; c0 < BN; c0 += 32) {
@@ -220,30 +242,20 @@ __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CU
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(C_::TMEM_COLS) : "memory");
   }
   if (p.split > 1) {
-    // ordered combine of the tile's split partials: in shared memory (two levels) when the tile is
-    // small enough, else directly by the last CTA (planner keeps split <= 8 then)
+    // ordered two-level combine of the tile's split partials (combine_splits, fp64); the sums land
+    // in this tile's slice of the workspace, from which the last CTA writes C
     constexpr int V = BM * BN;
-    double* out = reinterpret_cast<double*>(smem);   // stage memory is free now
+    const int ng = combine_rows(p.split);
     const float* tpart = p.part + (long long)tile * p.split * V;
-    if (V <= 4096) {
-      const int ng = combine_rows(p.split);
-      if (combine_splits(p.tickets + tile * (1 + ng), tpart, p.gpart + (long long)tile * ng * V, V, p.split, z, V, out, out + V)) {
-        for (int v = tid; v < V; v += NTHR) {
-          const int m = m0 + v / BN, n = n0 + v % BN;
-          if (m < p.DM && n < p.DN) {
-            if (p.trans) p.C[(long long)n * p.ldc + m] = (float)out[v];
-            else p.C[(long long)m * p.ldc + n] = (float)out[v];
-          }
-        }
-      }
-    } else if (last_cta_of(p.tickets + tile, (unsigned)p.split)) {
+    double* fin = p.fin + (long long)tile * V;
+    double* scratch = reinterpret_cast<double*>(smem);   // (used only for V < blockDim / 2)
+    if (combine_splits(p.tickets + tile * (1 + ng), tpart, p.gpart + (long long)tile * ng * V, V, p.split, z, V, fin, scratch)) {
       for (int v = tid; v < V; v += NTHR) {
         const int m = m0 + v / BN, n = n0 + v % BN;
-        if (m >= p.DM || n >= p.DN) continue;
-        double t = 0.0;
-        for (int zz = 0; zz < p.split; zz++) t += (double)__ldcg(tpart + (long long)zz * V + v);
-        if (p.trans) p.C[(long long)n * p.ldc + m] = (float)t;
-        else p.C[(long long)m * p.ldc + n] = (float)t;
+        if (m < p.DM && n < p.DN) {
+          if (p.trans) p.C[(long long)n * p.ldc + m] = (float)fin[v];
+          else p.C[(long long)m * p.ldc + n] = (float)fin[v];
+        }
       }
     }
   }
@@ -270,7 +282,9 @@ inline Plan plan(long long M, long long N, long long K) {
   long long split = best.tiles >= 148 ? 1 : 148 / best.tiles;   // one CTA per SM (~200 KB of stages)
   const long long kmax = K / (4LL * BK);                         // >= 4 stages per split
   if (split > kmax) split = kmax > 0 ? kmax : 1;
-  if ((long long)BM * best.bn > 4096 && split > 8) split = 8;    // direct last-CTA combine above 4096 values
+  // partial tiles (written once, read once) within ~25 % of the operand bytes
+  const long long pmax = (4 * K * (M + N)) / (32LL * best.tiles * BM * best.bn);
+  if (split > pmax) split = pmax > 0 ? pmax : 1;
   if (split > 1024) split = 1024;
   best.kps = (int)(cdiv(cdiv(K, split), BK) * BK);
   best.split = (int)cdiv(K, best.kps);
@@ -280,7 +294,7 @@ inline Plan plan(long long M, long long N, long long K) {
 inline uint64_t ws_bytes(const Plan& p) {
   if (p.split <= 1) return 0;
   const uint64_t V = (uint64_t)BM * p.bn;
-  return WS_TICKET_BYTES + (uint64_t)p.tiles * p.split * V * 4 + 16 + (uint64_t)p.tiles * combine_rows(p.split) * V * 8;
+  return WS_TICKET_BYTES + (uint64_t)p.tiles * p.split * V * 4 + 16 + (uint64_t)p.tiles * (combine_rows(p.split) + 1) * V * 8;
 }
 
 template <int BN>
@@ -369,7 +383,8 @@ int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_
   p.DM = (int)(pl.trans ? N : M); p.DN = (int)(pl.trans ? M : N); p.K = (int)K;
   p.C = (float*)a[2]; p.ldc = ldc;
   p.tiles_n = pl.tiles_n; p.tiles = pl.tiles; p.split = pl.split; p.kps = pl.kps;
-  p.tickets = nullptr; p.part = nullptr; p.gpart = nullptr;
+  p.tickets = nullptr; p.part = nullptr; p.gpart = nullptr; p.fin = nullptr;
+  { const char* e = getenv("ORION_ATC_DBG"); p.dbg = e ? atoi(e) : 0; }
   if (pl.split > 1) {
     unsigned char* ws = (unsigned char*)a[11];
     const uint64_t V = (uint64_t)atc::BM * pl.bn;
@@ -377,13 +392,14 @@ int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_
     p.part = reinterpret_cast<float*>(ws + WS_TICKET_BYTES);
     uintptr_t gp = reinterpret_cast<uintptr_t>(ws + WS_TICKET_BYTES + (uint64_t)pl.tiles * pl.split * V * 4);
     p.gpart = reinterpret_cast<double*>((gp + 15) & ~uintptr_t(15));
+    p.fin = p.gpart + (uint64_t)pl.tiles * combine_rows(pl.split) * V;
   }
   const float* Ap = pl.trans ? (const float*)a[1] : (const float*)a[0];   // M side
   const float* Bp = pl.trans ? (const float*)a[0] : (const float*)a[1];   // N side
   const long long ldA = pl.trans ? ldb : lda, ldB = pl.trans ? lda : ldb;
   CUtensorMap mA, mB;
-  if (!tmah::map2d_f32_sw(&mA, Ap, K, p.DM, ldA, 32, atc::BK, CU_TENSOR_MAP_SWIZZLE_128B)) return ORION_E_CUDA;
-  if (!tmah::map2d_f32_sw(&mB, Bp, K, p.DN, ldB, 32, atc::BK, CU_TENSOR_MAP_SWIZZLE_128B)) return ORION_E_CUDA;
+  if (!tmah::map2d_f32_sw(&mA, Ap, K, p.DM, ldA, 32, atc::BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
+  if (!tmah::map2d_f32_sw(&mB, Bp, K, p.DN, ldB, 32, atc::BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
   switch (pl.bn) {
     case 32: atc::atc_kernel<32><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
     case 64: atc::atc_kernel<64><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
