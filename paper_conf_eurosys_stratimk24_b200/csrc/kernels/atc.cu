@@ -13,6 +13,7 @@
 //    two TMEM accumulators (main, corrections); the converter warps then read TMEM back;
 //  * K is split over CTAs (shape-only count); fp32 partial tiles are summed in split order by the
 //    last CTA of each tile (fp64), so results are deterministic and partition-independent.
+#include <cmath>
 #include <cstdlib>
 
 #include "common.cuh"
@@ -279,12 +280,16 @@ inline Plan plan(long long M, long long N, long long K) {
       best.trans = trans; best.bn = bn; best.tiles_n = (int)tn; best.tiles = (int)tiles;
     }
   }
-  long long split = best.tiles >= 148 ? 1 : 148 / best.tiles;   // one CTA per SM (~200 KB of stages)
+  // split K so that the streaming time per CTA (operand bytes / CTAs) and the serial ordered combine
+  // of a tile's partials (split x tile bytes, read by its last CTAs) balance: split ~ sqrt(operand
+  // bytes / (tiles x tile bytes)), at most one CTA per SM of a 148-SM part (~200 KB of stages each)
+  const double ob = 4.0 * (double)K * (double)(M + N), tb = 4.0 * BM * best.bn;
+  long long split = (long long)(sqrt(ob / ((double)best.tiles * tb)) + 0.5);
+  const long long smax = best.tiles >= 148 ? 1 : 148 / best.tiles;
+  if (split > smax) split = smax;
+  if (split < 1) split = 1;
   const long long kmax = K / (4LL * BK);                         // >= 4 stages per split
   if (split > kmax) split = kmax > 0 ? kmax : 1;
-  // partial tiles (written once, read once) within ~25 % of the operand bytes
-  const long long pmax = (4 * K * (M + N)) / (32LL * best.tiles * BM * best.bn);
-  if (split > pmax) split = pmax > 0 ? pmax : 1;
   if (split > 1024) split = 1024;
   best.kps = (int)(cdiv(cdiv(K, split), BK) * BK);
   best.split = (int)cdiv(K, best.kps);
