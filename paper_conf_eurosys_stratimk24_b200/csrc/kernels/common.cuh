@@ -116,11 +116,38 @@ __device__ __forceinline__ double sum_chunk(const Src* src, long long stride, in
   for (; z < z1; z++) s += __ldcg(src + (long long)z * stride + v);
   return s;
 }
+// sum_rows_ordered: every value is summed over the rows in row order (unchanged results); a thread
+// owns SR_VB consecutive values and keeps 8 rows x SR_VB loads in flight per batch, so a large V
+// costs V / (SR_VB * blockDim) batches instead of V / blockDim dependent row walks.
+constexpr int SR_VB = 4;
 template <class Src>
 __device__ inline void sum_rows_ordered(const Src* src, long long stride, int n, int V, double* dst, double* scratch) {
   const int nt = blockDim.x, t = threadIdx.x;
   if (V >= nt / 2) {
-    for (int v = t; v < V; v += nt) dst[v] = sum_chunk(src, stride, 0, n, v);
+    for (int v0 = t * SR_VB; v0 < V; v0 += nt * SR_VB) {
+      double acc[SR_VB];
+#pragma unroll
+      for (int j = 0; j < SR_VB; j++) acc[j] = 0.0;
+      int z = 0;
+      for (; z + 7 < n; z += 8) {
+        Src a[8][SR_VB];
+#pragma unroll
+        for (int i = 0; i < 8; i++)
+#pragma unroll
+          for (int j = 0; j < SR_VB; j++) a[i][j] = v0 + j < V ? __ldcg(src + (long long)(z + i) * stride + v0 + j) : Src(0);
+#pragma unroll
+        for (int i = 0; i < 8; i++)
+#pragma unroll
+          for (int j = 0; j < SR_VB; j++) acc[j] += a[i][j];
+      }
+      for (; z < n; z++)
+#pragma unroll
+        for (int j = 0; j < SR_VB; j++)
+          if (v0 + j < V) acc[j] += __ldcg(src + (long long)z * stride + v0 + j);
+#pragma unroll
+      for (int j = 0; j < SR_VB; j++)
+        if (v0 + j < V) dst[v0 + j] = acc[j];
+    }
   } else {
     int T = nt / V;
     if (T > n) T = n > 0 ? n : 1;
