@@ -23,15 +23,17 @@ namespace {
 namespace atc {
 using namespace tmah;
 
-constexpr int BM = 128, BK = 32, NTHR = 192;   // warps: 0 TMA, 1 MMA + TMEM owner, 2-5 converters / epilogue
+constexpr int BM = 128, BK = 16, NTHR = 192;   // warps: 0 TMA, 1 MMA + TMEM owner, 2-5 converters / epilogue
+// (16-row stages: deep rings -- 6-8 stages -- keep the loads of one CTA per SM in flight)
 constexpr int CONV_THREADS = 128;
+constexpr int BOX_BYTES = 32 * BK * 4;   // one TMA box: 32 elements (128 B) x BK rows = one MN atom column
 
 template <int BN_>
 struct Cfg {
   static constexpr int BN = BN_;
   static constexpr int A_BYTES = BM * BK * 4, B_BYTES = BN * BK * 4;
   static constexpr int STAGE = 2 * (A_BYTES + B_BYTES);   // [A raw][A lo][B raw][B lo]
-  static constexpr int STAGES = (200 * 1024) / STAGE > 6 ? 6 : (200 * 1024) / STAGE;
+  static constexpr int STAGES = (200 * 1024) / STAGE > 8 ? 8 : (200 * 1024) / STAGE;
   static constexpr int SMEM = STAGES * STAGE + 1024 + 256;
   static constexpr int TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
   // kind::tf32: D fp32 (bit 4), A, B tf32 (bits 7, 10), A and B MN-major (bits 15, 16), N>>3, M>>4
@@ -50,15 +52,14 @@ struct Params {
   float* part;        // [tile][split][BM*BN]
   double* gpart;
   double* fin;        // [tile][BM*BN] fp64 sums of the splits
-  int dbg;            // ORION_ATC_DBG (bring-up only): 1 = write stage-0 A tile as decoded from smem
 };
 
 __device__ __forceinline__ uint64_t desc_mn128(uint32_t addr) {
   // MN-major tf32 operands need the 128-byte swizzle with 32-byte atoms (SWIZZLE_128B_BASE32B,
   // layout type 1; TMA CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B): atoms of 4 k-rows x 128 B (32 tf32
-  // along M / N). LBO = 4096 B between MN atoms (one TMA box), SBO = 512 B between 4-row k-groups;
+  // along M / N). LBO = BOX_BYTES between MN atoms (one TMA box), SBO = 512 B between 4-row k-groups;
   // version 1 (bit 46). (The 16-byte-granular SWIZZLE_128B layout reads as zeros for MN-major tf32.)
-  return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)(4096 >> 4) << 16) | ((uint64_t)(512 >> 4) << 32) | (1ull << 46) | (1ull << 61);
+  return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)(BOX_BYTES >> 4) << 16) | ((uint64_t)(512 >> 4) << 32) | (1ull << 46) | (1ull << 61);
 }
 __device__ __forceinline__ void mma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
   asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
@@ -123,9 +124,9 @@ __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CU
         mbar_expect(bar, C_::TX);
         const int kk = k0 + it * BK;
 #pragma unroll
-        for (int j = 0; j < BM / 32; j++) tma_load2d(st + j * 4096, &tmA, m0 + 32 * j, kk, bar);
+        for (int j = 0; j < BM / 32; j++) tma_load2d(st + j * BOX_BYTES, &tmA, m0 + 32 * j, kk, bar);
 #pragma unroll
-        for (int j = 0; j < BN / 32; j++) tma_load2d(st + 2 * A_BYTES + j * 4096, &tmB, n0 + 32 * j, kk, bar);
+        for (int j = 0; j < BN / 32; j++) tma_load2d(st + 2 * A_BYTES + j * BOX_BYTES, &tmB, n0 + 32 * j, kk, bar);
       }
     }
   } else if (warp == 1) {
@@ -140,19 +141,11 @@ __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CU
         asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
         const uint32_t st = smem_u32(smem + (size_t)s * STAGE);
         const uint32_t a_hi = st, a_lo = st + A_BYTES, b_hi = st + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
-        uint32_t idesc = C_::IDESC;
-        if (p.dbg == 2) idesc &= ~((1u << 15) | (1u << 16));
+        const uint32_t idesc = C_::IDESC;
 #pragma unroll
         for (int ks = 0; ks < BK / 8; ks++) {
-          const uint32_t o = ks * 1024;   // next 8-row k-group inside every atom
+          const uint32_t o = ks * 1024;   // next 8 rows (two 4-row atoms) inside every MN atom column
           const uint32_t acc = (it | ks) != 0;
-          if (p.dbg == 3) {   // bring-up: K-major SW128 descriptors (wrong data, must still write)
-            auto dk = [](uint32_t addr) {
-              return (uint64_t)((addr >> 4) & 0x3FFF) | (1ull << 16) | ((uint64_t)(1024 >> 4) << 32) | (1ull << 46) | (2ull << 61);
-            };
-            mma_tf32(d_main, dk(a_hi + 32 * ks), dk(b_hi + 32 * ks), idesc & ~((1u << 15) | (1u << 16)), acc);
-            continue;
-          }
           mma_tf32(d_corr, desc_mn128(a_lo + o), desc_mn128(b_hi + o), idesc, acc);
           mma_tf32(d_corr, desc_mn128(a_hi + o), desc_mn128(b_lo + o), idesc, 1);
           mma_tf32(d_main, desc_mn128(a_hi + o), desc_mn128(b_hi + o), idesc, acc);
@@ -199,16 +192,7 @@ __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CU
   asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
   // all TMEM reads happen below (warps 2-5), partial tiles / results written, then dealloc
   float* part = p.part ? p.part + ((long long)tile * p.split + z) * (BM * BN) : nullptr;
-  if (p.dbg == 1 && warp >= 2) {
-    // C[m][k] = A element (m, k) of stage 0 read back through the SW128 MN-major atom layout
-    const int q = warp & 3, row = 32 * q + lane;
-    const unsigned char* st = smem;
-    for (int k = 0; k < BK; k++) {
-      const int atom = row / 32, mi = row % 32;
-      const uint32_t off = atom * 4096 + (k / 8) * 1024 + (k % 8) * 128 + ((((mi * 4) / 16) ^ (k % 8)) << 4) + (mi * 4) % 16;
-      if (m0 + row < p.DM && k < p.DN) p.C[(long long)(m0 + row) * p.ldc + k] = *reinterpret_cast<const float*>(st + off);
-    }
-  } else if (warp >= 2) {
+  if (warp >= 2) {
     const int q = warp & 3, row = 32 * q + lane, m = m0 + row;
 #pragma unroll 1
     for (int c0 = 0; c0 < BN; c0 += 32) {
@@ -265,7 +249,7 @@ __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CU
 
 struct Plan { int trans, bn, tiles_n, tiles, split, kps; };
 
-inline int bn_for(long long DN) { return DN <= 32 ? 32 : DN <= 64 ? 64 : DN <= 128 ? 128 : (DN <= 256 ? 256 : 128); }
+inline int bn_for(long long DN) { return DN <= 32 ? 32 : DN <= 64 ? 64 : 128; }   // BN <= 128: >= 6 stages
 
 inline Plan plan(long long M, long long N, long long K) {
   Plan best{};
@@ -318,24 +302,21 @@ inline const void* fn_of(int bn) {
   switch (bn) {
     case 32: return (const void*)atc_kernel<32>;
     case 64: return (const void*)atc_kernel<64>;
-    case 128: return (const void*)atc_kernel<128>;
-    default: return (const void*)atc_kernel<256>;
+    default: return (const void*)atc_kernel<128>;
   }
 }
 inline int smem_of(int bn) {
   switch (bn) {
     case 32: return Cfg<32>::SMEM;
     case 64: return Cfg<64>::SMEM;
-    case 128: return Cfg<128>::SMEM;
-    default: return Cfg<256>::SMEM;
+    default: return Cfg<128>::SMEM;
   }
 }
 inline bool prepare_of(int bn) {
   switch (bn) {
     case 32: return prepare<32>();
     case 64: return prepare<64>();
-    case 128: return prepare<128>();
-    default: return prepare<256>();
+    default: return prepare<128>();
   }
 }
 
@@ -377,7 +358,7 @@ bool atc_try_geom(const uint64_t* a, LaunchGeom* g) {
 }
 
 bool atc_is(const void* f) {
-  return f == atc::fn_of(32) || f == atc::fn_of(64) || f == atc::fn_of(128) || f == atc::fn_of(256);
+  return f == atc::fn_of(32) || f == atc::fn_of(64) || f == atc::fn_of(128);
 }
 
 int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
@@ -389,7 +370,6 @@ int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_
   p.C = (float*)a[2]; p.ldc = ldc;
   p.tiles_n = pl.tiles_n; p.tiles = pl.tiles; p.split = pl.split; p.kps = pl.kps;
   p.tickets = nullptr; p.part = nullptr; p.gpart = nullptr; p.fin = nullptr;
-  { const char* e = getenv("ORION_ATC_DBG"); p.dbg = e ? atoi(e) : 0; }
   if (pl.split > 1) {
     unsigned char* ws = (unsigned char*)a[11];
     const uint64_t V = (uint64_t)atc::BM * pl.bn;
@@ -408,8 +388,7 @@ int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_
   switch (pl.bn) {
     case 32: atc::atc_kernel<32><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
     case 64: atc::atc_kernel<64><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
-    case 128: atc::atc_kernel<128><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
-    default: atc::atc_kernel<256><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
+    default: atc::atc_kernel<128><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
   }
   return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
 }
