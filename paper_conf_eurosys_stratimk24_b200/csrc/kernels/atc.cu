@@ -11,8 +11,8 @@
 //    swizzled layout is preserved); the raw fp32 tile serves as hi (the tensor core reads tf32);
 //  * one thread issues tcgen05.mma kind::tf32 with transposed (MN-major) A and B descriptors into
 //    two TMEM accumulators (main, corrections); the converter warps then read TMEM back;
-//  * K is split over CTAs (shape-only count); fp32 partial tiles are summed in split order by the
-//    last CTA of each tile (fp64), so results are deterministic and partition-independent.
+//  * K is split over CTAs (shape-only count); the fp32 partial tiles are summed in split order (fp64)
+//    by a second, many-CTA launch of the op, so results are deterministic and partition-independent.
 #include <cmath>
 #include <cstdlib>
 
@@ -48,10 +48,7 @@ struct Params {
   float* C;
   long long ldc;
   int tiles_n, tiles, split, kps;
-  unsigned int* tickets;
-  float* part;        // [tile][split][BM*BN]
-  double* gpart;
-  double* fin;        // [tile][BM*BN] fp64 sums of the splits
+  float* part;        // [tile][split][BM*BN] fp32 partial tiles (split > 1)
 };
 
 __device__ __forceinline__ uint64_t desc_mn128(uint32_t addr) {
@@ -226,21 +223,42 @@ __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CU
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(C_::TMEM_COLS) : "memory");
   }
-  if (p.split > 1) {
-    // ordered two-level combine of the tile's split partials (combine_splits, fp64); the sums land
-    // in this tile's slice of the workspace, from which the last CTA writes C
-    constexpr int V = BM * BN;
-    const int ng = combine_rows(p.split);
-    const float* tpart = p.part + (long long)tile * p.split * V;
-    double* fin = p.fin + (long long)tile * V;
-    double* scratch = reinterpret_cast<double*>(smem);   // (used only for V < blockDim / 2)
-    if (combine_splits(p.tickets + tile * (1 + ng), tpart, p.gpart + (long long)tile * ng * V, V, p.split, z, V, fin, scratch)) {
-      for (int v = tid; v < V; v += NTHR) {
-        const int m = m0 + v / BN, n = n0 + v % BN;
-        if (m < p.DM && n < p.DN) {
-          if (p.trans) p.C[(long long)n * p.ldc + m] = (float)fin[v];
-          else p.C[(long long)m * p.ldc + n] = (float)fin[v];
-        }
+  if (p.split == 1) orion_signal(sig);   // else the combine kernel below signals
+}
+
+// Ordered combine of the split partials (a second launch of the op, many CTAs: the serial last-CTA
+// combine of round 2's first version cost ~25 us per launch): thread = 4 consecutive elements of
+// one tile, partials added in split order in fp64 with 8 splits' loads in flight; writes C.
+constexpr int CMB_THREADS = 256;
+template <int BN>
+__global__ void __launch_bounds__(CMB_THREADS) atc_combine_kernel(Params p, OrionSig sig) {
+  constexpr int V = BM * BN, V4 = V / 4, per_tile = (V4 + CMB_THREADS - 1) / CMB_THREADS;
+  const int tile = blockIdx.x / per_tile;
+  const int v4 = (blockIdx.x % per_tile) * CMB_THREADS + threadIdx.x;
+  if (v4 < V4) {
+    const float4* src = reinterpret_cast<const float4*>(p.part + (long long)tile * p.split * V) + v4;
+    double a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;
+    int z = 0;
+    for (; z + 7 < p.split; z += 8) {
+      float4 t[8];
+#pragma unroll
+      for (int i = 0; i < 8; i++) t[i] = __ldcg(src + (long long)(z + i) * V4);
+#pragma unroll
+      for (int i = 0; i < 8; i++) { a0 += t[i].x; a1 += t[i].y; a2 += t[i].z; a3 += t[i].w; }
+    }
+    for (; z < p.split; z++) {
+      const float4 t = __ldcg(src + (long long)z * V4);
+      a0 += t.x; a1 += t.y; a2 += t.z; a3 += t.w;
+    }
+    const int m0 = (tile / p.tiles_n) * BM, n0 = (tile % p.tiles_n) * BN;
+    const int v = 4 * v4, m = m0 + v / BN, nb = n0 + v % BN;
+    const double a[4] = {a0, a1, a2, a3};
+#pragma unroll
+    for (int j = 0; j < 4; j++) {
+      const int n = nb + j;
+      if (m < p.DM && n < p.DN) {
+        if (p.trans) p.C[(long long)n * p.ldc + m] = (float)a[j];
+        else p.C[(long long)m * p.ldc + n] = (float)a[j];
       }
     }
   }
@@ -267,8 +285,10 @@ inline Plan plan(long long M, long long N, long long K) {
   // split K so that the streaming time per CTA (operand bytes / CTAs) and the serial ordered combine
   // of a tile's partials (split x tile bytes, read by its last CTAs) balance: split ~ sqrt(operand
   // bytes / (tiles x tile bytes)), at most one CTA per SM of a 148-SM part (~200 KB of stages each)
+  // one CTA per SM of a 148-SM part (~200 KB of stages each); the partial tiles (written once,
+  // read once by the parallel combine) stay within ~25 % of the operand bytes
   const double ob = 4.0 * (double)K * (double)(M + N), tb = 4.0 * BM * best.bn;
-  long long split = (long long)(sqrt(ob / ((double)best.tiles * tb)) + 0.5);
+  long long split = (long long)(ob / (8.0 * (double)best.tiles * tb));
   const long long smax = best.tiles >= 148 ? 1 : 148 / best.tiles;
   if (split > smax) split = smax;
   if (split < 1) split = 1;
@@ -283,8 +303,9 @@ inline Plan plan(long long M, long long N, long long K) {
 inline uint64_t ws_bytes(const Plan& p) {
   if (p.split <= 1) return 0;
   const uint64_t V = (uint64_t)BM * p.bn;
-  return WS_TICKET_BYTES + (uint64_t)p.tiles * p.split * V * 4 + 16 + (uint64_t)p.tiles * (combine_rows(p.split) + 1) * V * 8;
+  return WS_TICKET_BYTES + (uint64_t)p.tiles * p.split * V * 4;
 }
+inline unsigned combine_ctas(const Plan& p) { return (unsigned)(p.tiles * cdiv((uint64_t)BM * p.bn / 4, CMB_THREADS)); }
 
 template <int BN>
 bool prepare() {
@@ -347,9 +368,9 @@ bool atc_try_geom(const uint64_t* a, LaunchGeom* g) {
   if (M >= (1LL << 24) || N >= (1LL << 24) || K >= (1LL << 31)) return false;
   atc::Plan pl = atc::plan(M, N, K);
   if (pl.split > 1 && (a[11] == 0 || a[12] < atc::ws_bytes(pl))) return false;
-  if ((uint64_t)pl.tiles * (1 + combine_rows(pl.split)) * 4 > WS_TICKET_BYTES) return false;
   if (!atc::prepare_of(pl.bn)) return false;
   g->grid = dim3((unsigned)pl.tiles, (unsigned)pl.split);
+  g->sig_ctas = pl.split > 1 ? atc::combine_ctas(pl) : 0;
   g->block = dim3(atc::NTHR);
   g->smem = atc::smem_of(pl.bn);
   g->func = atc::fn_of(pl.bn);
@@ -369,15 +390,12 @@ int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_
   p.DM = (int)(pl.trans ? N : M); p.DN = (int)(pl.trans ? M : N); p.K = (int)K;
   p.C = (float*)a[2]; p.ldc = ldc;
   p.tiles_n = pl.tiles_n; p.tiles = pl.tiles; p.split = pl.split; p.kps = pl.kps;
-  p.tickets = nullptr; p.part = nullptr; p.gpart = nullptr; p.fin = nullptr;
+  p.part = nullptr;
   if (pl.split > 1) {
     unsigned char* ws = (unsigned char*)a[11];
     const uint64_t V = (uint64_t)atc::BM * pl.bn;
-    p.tickets = reinterpret_cast<unsigned int*>(ws);
+    (void)V;
     p.part = reinterpret_cast<float*>(ws + WS_TICKET_BYTES);
-    uintptr_t gp = reinterpret_cast<uintptr_t>(ws + WS_TICKET_BYTES + (uint64_t)pl.tiles * pl.split * V * 4);
-    p.gpart = reinterpret_cast<double*>((gp + 15) & ~uintptr_t(15));
-    p.fin = p.gpart + (uint64_t)pl.tiles * combine_rows(pl.split) * V;
   }
   const float* Ap = pl.trans ? (const float*)a[1] : (const float*)a[0];   // M side
   const float* Bp = pl.trans ? (const float*)a[0] : (const float*)a[1];   // N side
@@ -385,10 +403,21 @@ int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_
   CUtensorMap mA, mB;
   if (!tmah::map2d_f32_sw(&mA, Ap, K, p.DM, ldA, 32, atc::BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
   if (!tmah::map2d_f32_sw(&mB, Bp, K, p.DN, ldB, 32, atc::BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
+  // split > 1: the tile kernel runs unsignalled, the combine kernel signals (g.sig_ctas CTAs)
+  const OrionSig none{nullptr, nullptr, 0, 0};
+  const OrionSig s1 = pl.split > 1 ? none : sig;
   switch (pl.bn) {
-    case 32: atc::atc_kernel<32><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
-    case 64: atc::atc_kernel<64><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
-    default: atc::atc_kernel<128><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, sig); break;
+    case 32: atc::atc_kernel<32><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, s1); break;
+    case 64: atc::atc_kernel<64><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, s1); break;
+    default: atc::atc_kernel<128><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, s1); break;
+  }
+  if (pl.split > 1) {
+    const unsigned cg = atc::combine_ctas(pl);
+    switch (pl.bn) {
+      case 32: atc::atc_combine_kernel<32><<<cg, atc::CMB_THREADS, 0, s>>>(p, sig); break;
+      case 64: atc::atc_combine_kernel<64><<<cg, atc::CMB_THREADS, 0, s>>>(p, sig); break;
+      default: atc::atc_combine_kernel<128><<<cg, atc::CMB_THREADS, 0, s>>>(p, sig); break;
+    }
   }
   return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
 }

@@ -53,6 +53,10 @@ struct LaunchGeom {
   int smem = 0;
   const void* func = nullptr;
   int pipe = 0;   // ORION_PIPE_*: the pipe the chosen kernel's arithmetic runs on (profiler ridge, R16)
+  // CTAs that run orion_signal (0 = all of grid): an op that launches a second, signalling kernel
+  // after an unsignalled one (split-K partials + their ordered combine) reports the second's grid
+  unsigned long long sig_ctas = 0;
+  unsigned long long signal_ctas() const { return sig_ctas ? sig_ctas : ctas(); }
   unsigned long long ctas() const { return (unsigned long long)grid.x * grid.y * grid.z; }
 };
 

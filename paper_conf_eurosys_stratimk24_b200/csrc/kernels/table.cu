@@ -50,8 +50,8 @@ int kernel_launch_sig(uint32_t fn, const uint64_t* args, uint32_t nargs, OrionSi
   LaunchGeom g;
   int r = e.geom(args, &g);
   if (r) return r;
-  if (ctas_out) *ctas_out = g.ctas();
-  if (sig.ticket) sig.target += g.ctas();
+  if (ctas_out) *ctas_out = g.signal_ctas();
+  if (sig.ticket) sig.target += g.signal_ctas();
   return e.launch(args, g, sig, s);
 }
 
