@@ -286,14 +286,19 @@ inline Plan plan(long long M, long long N, long long K) {
   // of a tile's partials (split x tile bytes, read by its last CTAs) balance: split ~ sqrt(operand
   // bytes / (tiles x tile bytes)), at most one CTA per SM of a 148-SM part (~200 KB of stages each)
   // one CTA per SM of a 148-SM part (~200 KB of stages each); the partial tiles (written once,
-  // read once by the parallel combine) stay within ~25 % of the operand bytes
+  // read once by the parallel combine) stay within the operand bytes
   const double ob = 4.0 * (double)K * (double)(M + N), tb = 4.0 * BM * best.bn;
-  long long split = (long long)(ob / (8.0 * (double)best.tiles * tb));
+  long long split = (long long)(ob / (2.0 * (double)best.tiles * tb));
   const long long smax = best.tiles >= 148 ? 1 : 148 / best.tiles;
   if (split > smax) split = smax;
   if (split < 1) split = 1;
   const long long kmax = K / (4LL * BK);                         // >= 4 stages per split
   if (split > kmax) split = kmax > 0 ? kmax : 1;
+  // accuracy: the tensor core accumulates a split's rows in fp32 inside TMEM; chains of <= 2048 rows
+  // keep 3xTF32 within the single-op bound (rel 1e-5; one K = 4704 chain measured 1.13e-5), the
+  // splits themselves are added in fp64
+  const long long kchain = (K + 2047) / 2048;
+  if (split < kchain) split = kchain;
   if (split > 1024) split = 1024;
   best.kps = (int)(cdiv(cdiv(K, split), BK) * BK);
   best.split = (int)cdiv(K, best.kps);
