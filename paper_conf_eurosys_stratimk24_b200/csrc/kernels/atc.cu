@@ -49,6 +49,9 @@ struct Params {
   long long ldc;
   int tiles_n, tiles, split, kps;
   float* part;        // [tile][split][BM*BN] fp32 partial tiles (split > 1)
+  // convolution weight gradient (CONV): rows are blocks of PB x QB output positions of one image;
+  // x boxes of column col take tap (col / C) shifted by the stride (4-D TMA, zero fill = padding)
+  int cv_C, cv_S, stride, pad, QB, PB, npb, nqb;
 };
 
 __device__ __forceinline__ uint64_t desc_mn128(uint32_t addr) {
@@ -78,7 +81,7 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t* r) {
 }
 __device__ __forceinline__ float trunc_tf32(float x) { return __uint_as_float(__float_as_uint(x) & 0xFFFFE000u); }
 
-template <int BN>
+template <int BN, bool CONV>
 __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                                                      Params p, OrionSig sig) {
   using C_ = Cfg<BN>;
@@ -120,10 +123,29 @@ __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CU
         const uint32_t st = smem_u32(smem + (size_t)s * STAGE), bar = full0 + 8 * s;
         mbar_expect(bar, C_::TX);
         const int kk = k0 + it * BK;
+        if (!CONV) {
 #pragma unroll
-        for (int j = 0; j < BM / 32; j++) tma_load2d(st + j * BOX_BYTES, &tmA, m0 + 32 * j, kk, bar);
+          for (int j = 0; j < BM / 32; j++) tma_load2d(st + j * BOX_BYTES, &tmA, m0 + 32 * j, kk, bar);
 #pragma unroll
-        for (int j = 0; j < BN / 32; j++) tma_load2d(st + 2 * A_BYTES + j * BOX_BYTES, &tmB, n0 + 32 * j, kk, bar);
+          for (int j = 0; j < BN / 32; j++) tma_load2d(st + 2 * A_BYTES + j * BOX_BYTES, &tmB, n0 + 32 * j, kk, bar);
+        } else {
+          // stage = position block b: image n, output rows p0.., columns q0..
+          const int b = kk / BK, qb = b % p.nqb, t2 = b / p.nqb, pb = t2 % p.npb, n = t2 / p.npb;
+          const int p0 = pb * p.PB, q0 = qb * p.QB;
+          // dy side: column = output channel; x side: column = (tap, input channel)
+          auto box = [&](bool is_x, const CUtensorMap* tm, uint32_t dst, int col) {
+            if (!is_x) {
+              tma_load4d(dst, tm, col, q0, p0, n, bar);
+            } else {
+              const int tap = col / p.cv_C, c = col - tap * p.cv_C, r = tap / p.cv_S, sx = tap - r * p.cv_S;
+              tma_load4d(dst, tm, c, q0 * p.stride + sx - p.pad, p0 * p.stride + r - p.pad, n, bar);
+            }
+          };
+#pragma unroll
+          for (int j = 0; j < BM / 32; j++) box(p.trans != 0, &tmA, st + j * BOX_BYTES, m0 + 32 * j);
+#pragma unroll
+          for (int j = 0; j < BN / 32; j++) box(p.trans == 0, &tmB, st + 2 * A_BYTES + j * BOX_BYTES, n0 + 32 * j);
+        }
       }
     }
   } else if (warp == 1) {
@@ -312,11 +334,11 @@ inline uint64_t ws_bytes(const Plan& p) {
 }
 inline unsigned combine_ctas(const Plan& p) { return (unsigned)(p.tiles * cdiv((uint64_t)BM * p.bn / 4, CMB_THREADS)); }
 
-template <int BN>
+template <int BN, bool CONV>
 bool prepare() {
   static std::atomic<int> done{0};
   if (done.load(std::memory_order_acquire)) return true;
-  if (cudaFuncSetAttribute((const void*)atc_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<BN>::SMEM) != cudaSuccess) {
+  if (cudaFuncSetAttribute((const void*)atc_kernel<BN, CONV>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<BN>::SMEM) != cudaSuccess) {
     (void)cudaGetLastError();
     return false;
   }
@@ -324,11 +346,11 @@ bool prepare() {
   return true;
 }
 
-inline const void* fn_of(int bn) {
+inline const void* fn_of(int bn, bool conv = false) {
   switch (bn) {
-    case 32: return (const void*)atc_kernel<32>;
-    case 64: return (const void*)atc_kernel<64>;
-    default: return (const void*)atc_kernel<128>;
+    case 32: return conv ? (const void*)atc_kernel<32, true> : (const void*)atc_kernel<32, false>;
+    case 64: return conv ? (const void*)atc_kernel<64, true> : (const void*)atc_kernel<64, false>;
+    default: return conv ? (const void*)atc_kernel<128, true> : (const void*)atc_kernel<128, false>;
   }
 }
 inline int smem_of(int bn) {
@@ -338,12 +360,76 @@ inline int smem_of(int bn) {
     default: return Cfg<128>::SMEM;
   }
 }
-inline bool prepare_of(int bn) {
+inline bool prepare_of(int bn, bool conv = false) {
   switch (bn) {
-    case 32: return prepare<32>();
-    case 64: return prepare<64>();
-    default: return prepare<128>();
+    case 32: return conv ? prepare<32, true>() : prepare<32, false>();
+    case 64: return conv ? prepare<64, true>() : prepare<64, false>();
+    default: return conv ? prepare<128, true>() : prepare<128, false>();
   }
+}
+
+// launch the tile kernel (+ the ordered combine when split > 1)
+template <bool CONV>
+int launch_pair(const LaunchGeom& g, const Plan& pl, const CUtensorMap& mA, const CUtensorMap& mB, const Params& p, OrionSig sig,
+                cudaStream_t s) {
+  const OrionSig none{nullptr, nullptr, 0, 0};
+  const OrionSig s1 = pl.split > 1 ? none : sig;   // split > 1: the combine kernel signals
+  switch (pl.bn) {
+    case 32: atc_kernel<32, CONV><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, s1); break;
+    case 64: atc_kernel<64, CONV><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, s1); break;
+    default: atc_kernel<128, CONV><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, s1); break;
+  }
+  if (pl.split > 1) {
+    const unsigned cg = combine_ctas(pl);
+    switch (pl.bn) {
+      case 32: atc_combine_kernel<32><<<cg, CMB_THREADS, 0, s>>>(p, sig); break;
+      case 64: atc_combine_kernel<64><<<cg, CMB_THREADS, 0, s>>>(p, sig); break;
+      default: atc_combine_kernel<128><<<cg, CMB_THREADS, 0, s>>>(p, sig); break;
+    }
+  }
+  return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+}
+
+// ---- convolution weight gradient: dW[K][R][S][C] = sum over (n, p, q) of dy[n,p,q,k] x-window
+struct ConvGeo { int N, H, W, C, K, R, S, stride, pad, P, Q; };
+inline void conv_blocks(const ConvGeo& c, int& QB, int& PB, int& npb, int& nqb) {
+  // 16 positions per stage: QB x PB with the least zero-filled padding of the P x Q grid
+  double best = 1e30;
+  for (int qb = 16; qb >= 1; qb /= 2) {
+    const int pb = BK / qb;
+    const double w = (double)cdiv(c.Q, qb) * qb * cdiv(c.P, pb) * pb;
+    if (w < best - 1e-9) { best = w; QB = qb; PB = pb; }
+  }
+  npb = (int)cdiv(c.P, PB);
+  nqb = (int)cdiv(c.Q, QB);
+}
+inline Plan plan_conv(const ConvGeo& c) {
+  int QB, PB, npb, nqb;
+  conv_blocks(c, QB, PB, npb, nqb);
+  const long long rows = (long long)c.N * npb * nqb * BK;
+  const long long RSC = (long long)c.R * c.S * c.C;
+  Plan best{};
+  double best_cost = 1e300;
+  for (int trans = 0; trans < 2; trans++) {
+    const long long DM = trans ? RSC : c.K, DN = trans ? c.K : RSC;
+    const int bn = bn_for(DN);
+    const long long tm = cdiv(DM, BM), tn = cdiv(DN, bn), tiles = tm * tn;
+    const double padded = (double)tiles * BM * bn;
+    if (padded < best_cost) { best_cost = padded; best.trans = trans; best.bn = bn; best.tiles_n = (int)tn; best.tiles = (int)tiles; }
+  }
+  const double ob = 4.0 * (double)c.N * c.P * c.Q * (double)(c.K + RSC), tb = 4.0 * BM * best.bn;
+  long long split = (long long)(ob / (2.0 * (double)best.tiles * tb));
+  const long long smax = best.tiles >= 148 ? 1 : 148 / best.tiles;
+  if (split > smax) split = smax;
+  if (split < 1) split = 1;
+  const long long kmax = rows / (4LL * BK);
+  if (split > kmax) split = kmax > 0 ? kmax : 1;
+  const long long kchain = (rows + 2047) / 2048;
+  if (split < kchain) split = kchain;
+  if (split > 1024) split = 1024;
+  best.kps = (int)(cdiv(cdiv(rows, split), BK) * BK);
+  best.split = (int)cdiv(rows, best.kps);
+  return best;
 }
 
 }  // namespace atc
@@ -387,6 +473,68 @@ bool atc_is(const void* f) {
   return f == atc::fn_of(32) || f == atc::fn_of(64) || f == atc::fn_of(128);
 }
 
+// ---- conv weight gradient entry points (gemm.cu conv_wgrad routing)
+// args: x, dy, dw, N, H, W, C, K, R, S, stride, pad, P, Q, workspace, ws_bytes
+static atc::ConvGeo conv_geo(const uint64_t* a) {
+  atc::ConvGeo c;
+  c.N = (int)a[3]; c.H = (int)a[4]; c.W = (int)a[5]; c.C = (int)a[6]; c.K = (int)a[7]; c.R = (int)a[8]; c.S = (int)a[9];
+  c.stride = (int)a[10]; c.pad = (int)a[11]; c.P = (int)a[12]; c.Q = (int)a[13];
+  return c;
+}
+
+uint64_t atc_conv_ws_bytes(uint64_t N, uint64_t H, uint64_t W, uint64_t C, uint64_t K, uint64_t R, uint64_t S, uint64_t stride,
+                           uint64_t pad) {
+  atc::ConvGeo c{(int)N, (int)H, (int)W, (int)C, (int)K, (int)R, (int)S, (int)stride, (int)pad,
+                 (int)((H + 2 * pad - R) / stride + 1), (int)((W + 2 * pad - S) / stride + 1)};
+  if (C % 32 || K % 4) return 0;
+  return atc::ws_bytes(atc::plan_conv(c));
+}
+
+bool atc_conv_try_geom(const uint64_t* a, LaunchGeom* g) {
+  const atc::ConvGeo c = conv_geo(a);
+  if (c.C % 32 || c.K % 4 || c.stride < 1 || c.stride > 8 || c.P <= 0 || c.Q <= 0) return false;
+  if (!tmah::al16((const void*)a[0]) || !tmah::al16((const void*)a[1]) || tmah::encoder() == nullptr) return false;
+  if ((long long)c.N * c.H * c.W * c.C >= (1LL << 40)) return false;
+  atc::Plan pl = atc::plan_conv(c);
+  if (pl.split > 1 && (a[14] == 0 || a[15] < atc::ws_bytes(pl))) return false;
+  if (!atc::prepare_of(pl.bn, true)) return false;
+  g->grid = dim3((unsigned)pl.tiles, (unsigned)pl.split);
+  g->block = dim3(atc::NTHR);
+  g->smem = atc::smem_of(pl.bn);
+  g->func = atc::fn_of(pl.bn, true);
+  g->pipe = ORION_PIPE_TF32X3;
+  g->sig_ctas = pl.split > 1 ? atc::combine_ctas(pl) : 0;
+  return true;
+}
+
+bool atc_conv_is(const void* f) {
+  return f == atc::fn_of(32, true) || f == atc::fn_of(64, true) || f == atc::fn_of(128, true);
+}
+
+int atc_conv_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
+  const atc::ConvGeo c = conv_geo(a);
+  atc::Plan pl = atc::plan_conv(c);
+  atc::Params p;
+  int QB, PB, npb, nqb;
+  atc::conv_blocks(c, QB, PB, npb, nqb);
+  const long long RSC = (long long)c.R * c.S * c.C;
+  p.trans = pl.trans;
+  p.DM = (int)(pl.trans ? RSC : c.K); p.DN = (int)(pl.trans ? c.K : RSC);
+  p.K = (int)((long long)c.N * npb * nqb * atc::BK);
+  p.C = (float*)a[2]; p.ldc = RSC;
+  p.tiles_n = pl.tiles_n; p.tiles = pl.tiles; p.split = pl.split; p.kps = pl.kps;
+  p.part = pl.split > 1 ? reinterpret_cast<float*>((unsigned char*)a[14] + WS_TICKET_BYTES) : nullptr;
+  p.C = (float*)a[2];
+  p.cv_C = c.C; p.cv_S = c.S; p.stride = c.stride; p.pad = c.pad; p.QB = QB; p.PB = PB; p.npb = npb; p.nqb = nqb;
+  CUtensorMap mx, mdy;
+  const long long dx_dims[4] = {c.C, c.W, c.H, c.N}, dy_dims[4] = {c.K, c.Q, c.P, c.N};
+  const int box[4] = {32, QB, PB, 1};
+  if (!tmah::map4d_f32(&mx, (const float*)a[0], dx_dims, box, c.stride, c.stride, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
+  if (!tmah::map4d_f32(&mdy, (const float*)a[1], dy_dims, box, 1, 1, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
+  // M side: x when trans (M = R*S*C), else dy (M = K)
+  return pl.trans ? atc::launch_pair<true>(g, pl, mx, mdy, p, sig, s) : atc::launch_pair<true>(g, pl, mdy, mx, p, sig, s);
+}
+
 int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   const long long M = a[4], N = a[5], K = a[6], lda = a[7], ldb = a[8], ldc = a[9];
   atc::Plan pl = atc::plan(M, N, K);
@@ -408,21 +556,5 @@ int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_
   CUtensorMap mA, mB;
   if (!tmah::map2d_f32_sw(&mA, Ap, K, p.DM, ldA, 32, atc::BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
   if (!tmah::map2d_f32_sw(&mB, Bp, K, p.DN, ldB, 32, atc::BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
-  // split > 1: the tile kernel runs unsignalled, the combine kernel signals (g.sig_ctas CTAs)
-  const OrionSig none{nullptr, nullptr, 0, 0};
-  const OrionSig s1 = pl.split > 1 ? none : sig;
-  switch (pl.bn) {
-    case 32: atc::atc_kernel<32><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, s1); break;
-    case 64: atc::atc_kernel<64><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, s1); break;
-    default: atc::atc_kernel<128><<<g.grid, g.block, g.smem, s>>>(mA, mB, p, s1); break;
-  }
-  if (pl.split > 1) {
-    const unsigned cg = atc::combine_ctas(pl);
-    switch (pl.bn) {
-      case 32: atc::atc_combine_kernel<32><<<cg, atc::CMB_THREADS, 0, s>>>(p, sig); break;
-      case 64: atc::atc_combine_kernel<64><<<cg, atc::CMB_THREADS, 0, s>>>(p, sig); break;
-      default: atc::atc_combine_kernel<128><<<cg, atc::CMB_THREADS, 0, s>>>(p, sig); break;
-    }
-  }
-  return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+  return atc::launch_pair<false>(g, pl, mA, mB, p, sig, s);
 }

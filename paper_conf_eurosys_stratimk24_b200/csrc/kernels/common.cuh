@@ -211,6 +211,11 @@ uint64_t atc_ws_bytes(long long M, long long N, long long K);
 bool atc_try_geom(const uint64_t* a, LaunchGeom* g);
 bool atc_is(const void* f);
 int atc_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
+uint64_t atc_conv_ws_bytes(uint64_t N, uint64_t H, uint64_t W, uint64_t C, uint64_t K, uint64_t R, uint64_t S, uint64_t stride,
+                           uint64_t pad);
+bool atc_conv_try_geom(const uint64_t* a, LaunchGeom* g);
+bool atc_conv_is(const void* f);
+int atc_conv_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
 
 // Kernel table (table.cu)
 extern const KernelEntry g_kernels[ORION_FN_COUNT];

@@ -2381,6 +2381,8 @@ extern "C" uint64_t orion_conv_wgrad_workspace_bytes(uint64_t N, uint64_t H, uin
     const uint64_t b2 = smallc::wgrad_ws_bytes(s);
     if (b2 > b) b = b2;
   }
+  const uint64_t b3 = atc_conv_ws_bytes(N, H, W, C, K, R, S, stride, pad);   // tcgen05 path (atc.cu)
+  if (b3 > b) b = b3;
   return b;
 }
 
@@ -2405,10 +2407,12 @@ int conv_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
     g->func = smallc::wgrad_fn(s);
     return 0;
   }
+  if (atc_conv_try_geom(a, g)) return 0;   // TMA 4-D boxes straight into tcgen05 (atc.cu)
   tiled_geom<ADenseT, BWgrad>(g, s.K, (long long)s.R * s.S * s.C, (long long)s.N * s.P * s.Q, a[14], a[15]);
   return 0;
 }
 int conv_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
+  if (atc_conv_is(g.func)) return atc_conv_launch(a, g, sig, st);
   ConvShape s = conv_shape(a);
   if (g.func == (const void*)smallc::conv_wgrad_smallc2_kernel) {
     smallc::conv_wgrad_smallc2_kernel<<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s,

@@ -70,6 +70,24 @@ inline bool map2d_f32_sw(CUtensorMap* m, const float* base, long long rows, long
   return e(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)base, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
+// 4-D fp32 map of an NHWC-like tensor dims {d0 (contiguous), d1, d2, d3} with element strides
+// {1, es1, es2, 1} (traversal strides: a box walks every es-th element of that dimension)
+inline bool map4d_f32(CUtensorMap* m, const float* base, const long long (&dims)[4], const int (&box)[4], int es1, int es2,
+                      CUtensorMapSwizzle sw) {
+  encode_fn e = encoder();
+  if (!e) return false;
+  cuuint64_t gd[4] = {(cuuint64_t)dims[0], (cuuint64_t)dims[1], (cuuint64_t)dims[2], (cuuint64_t)dims[3]};
+  cuuint64_t gs[3] = {(cuuint64_t)dims[0] * 4, (cuuint64_t)dims[0] * dims[1] * 4, (cuuint64_t)dims[0] * dims[1] * dims[2] * 4};
+  cuuint32_t bx[4] = {(cuuint32_t)box[0], (cuuint32_t)box[1], (cuuint32_t)box[2], (cuuint32_t)box[3]};
+  cuuint32_t es[4] = {1, (cuuint32_t)es1, (cuuint32_t)es2, 1};
+  return e(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, (void*)base, gd, gs, bx, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
+           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+__device__ __forceinline__ void tma_load4d(uint32_t dst, const CUtensorMap* tm, int c0, int c1, int c2, int c3, uint32_t bar) {
+  asm volatile("cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], [%6];" ::"r"(dst),
+               "l"(tm), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(bar)
+               : "memory");
+}
 inline bool al16(const void* q) { return (reinterpret_cast<uintptr_t>(q) & 15) == 0; }
 
 }  // namespace tmah

@@ -99,3 +99,40 @@ def test_wgrad_stream(M, N, K):
 @pytest.mark.parametrize("M,N,K", [(18, 16, 50000), (96, 16, 200)])   # M % 4 != 0 / short K: other kernels
 def test_wgrad_fallback(M, N, K):
     check_wgrad(M, N, K, expect_stream=False)
+
+
+CONV_WG = [  # N, H, W, C, K, R, stride, pad: ResNet weight gradients on the tcgen05 path (C % 32 == 0)
+    (2, 56, 56, 64, 64, 3, 1, 1),     # layer1 3x3
+    (2, 28, 28, 128, 128, 3, 1, 1),   # layer2 3x3
+    (2, 56, 56, 128, 128, 3, 2, 1),   # layer2.0 3x3 stride 2 (v1.5)
+    (2, 7, 7, 512, 512, 3, 1, 1),     # layer4 3x3 (ragged 7 x 7 position blocks)
+    (2, 56, 56, 256, 512, 1, 2, 0),   # layer2.0 downsample 1x1 stride 2
+    (3, 9, 11, 32, 36, 3, 2, 1),      # ragged everything
+]
+
+
+@pytest.mark.parametrize("n,h,w,c,k,r,st,pad", CONV_WG, ids=lambda v: str(v))
+def test_conv_wgrad_tensor_path(n, h, w, c, k, r, st, pad):
+    """dW = sum over positions of dy x-window via 4-D TMA boxes (zero fill = padding) on tcgen05."""
+    import parity as PT
+    x = si.normal((n, h, w, c), 41)
+    p, q = (h + 2 * pad - r) // st + 1, (w + 2 * pad - r) // st + 1
+    dy = si.normal((n, p, q, k), 42)
+    dw = torch.zeros(k, r, r, c, device="cuda")
+    nws = L.lib.orion_conv_wgrad_workspace_bytes(n, h, w, c, k, r, r, st, pad)
+    wsb = torch.zeros(int(nws) // 4 + 64, device="cuda")
+    xd, dyd = x.cuda(), dy.cuda()
+    args = [xd.data_ptr(), dyd.data_ptr(), dw.data_ptr(), n, h, w, c, k, r, r, st, pad, p, q, wsb.data_ptr(), wsb.numel() * 4]
+    assert "atc_kernel" in kernel_info("conv_wgrad", args)["kernel"]
+    s = torch.cuda.current_stream().cuda_stream
+    orion.kernel_launch("conv_wgrad", args, s)
+    torch.cuda.synchronize()
+    ref = om.conv2d_bwd_weight(x, dy, (k, r, r, c), st, pad)
+    A = om.conv2d_bwd_weight_abs(x, dy, (k, r, r, c), st, pad)
+    assert PT.rel(dw, ref) < 1e-5
+    K = n * p * q
+    assert PT.cond_elem(dw, ref, A) <= 4 * U * math.sqrt(K)
+    first = dw.clone()
+    orion.kernel_launch("conv_wgrad", args, s)
+    torch.cuda.synchronize()
+    assert torch.equal(first, dw)
