@@ -493,6 +493,11 @@ uint64_t atc_conv_ws_bytes(uint64_t N, uint64_t H, uint64_t W, uint64_t C, uint6
 bool atc_conv_try_geom(const uint64_t* a, LaunchGeom* g) {
   const atc::ConvGeo c = conv_geo(a);
   if (c.C % 32 || c.K % 4 || c.stride < 1 || c.stride > 8 || c.P <= 0 || c.Q <= 0) return false;
+  {
+    int QB, PB, npb, nqb;
+    atc::conv_blocks(c, QB, PB, npb, nqb);
+    if (QB * c.stride > 256 || PB * c.stride > 256) return false;   // TMA box dimension limit
+  }
   if (!tmah::al16((const void*)a[0]) || !tmah::al16((const void*)a[1]) || tmah::encoder() == nullptr) return false;
   if ((long long)c.N * c.H * c.W * c.C >= (1LL << 40)) return false;
   atc::Plan pl = atc::plan_conv(c);
@@ -529,7 +534,10 @@ int atc_conv_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaSt
   CUtensorMap mx, mdy;
   const long long dx_dims[4] = {c.C, c.W, c.H, c.N}, dy_dims[4] = {c.K, c.Q, c.P, c.N};
   const int box[4] = {32, QB, PB, 1};
-  if (!tmah::map4d_f32(&mx, (const float*)a[0], dx_dims, box, c.stride, c.stride, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
+  // with traversal strides the box spans stride x as many x elements (TMA loads ceil(box / stride)
+  // of them per dimension), so the x box covers QB * stride columns and PB * stride rows
+  const int xbox[4] = {32, QB * c.stride, PB * c.stride, 1};
+  if (!tmah::map4d_f32(&mx, (const float*)a[0], dx_dims, xbox, c.stride, c.stride, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
   if (!tmah::map4d_f32(&mdy, (const float*)a[1], dy_dims, box, 1, 1, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
   // M side: x when trans (M = R*S*C), else dy (M = K)
   return pl.trans ? atc::launch_pair<true>(g, pl, mx, mdy, p, sig, s) : atc::launch_pair<true>(g, pl, mdy, mx, p, sig, s);
