@@ -166,6 +166,7 @@ typedef struct {
   int32_t blocks_per_sm;     /* cudaOccupancyMaxActiveBlocksPerMultiprocessor */
   int32_t pipe;              /* enum orion_pipe */
   char kernel[120];          /* the kernel the op launches (mangled device-function name, truncated) */
+  int32_t launches;          /* kernels one launch of the op issues (2: split partials + ordered combine) */
 } orion_kernel_info_t;
 int orion_kernel_info(uint32_t fn, const uint64_t* args, uint32_t nargs, orion_kernel_info_t* out);
 /* Workspace sizes (bytes) of the ops that split their reductions. Workspaces must be zeroed once

@@ -51,7 +51,7 @@ class Config(ctypes.Structure):
 class KernelInfo(ctypes.Structure):   # orion_kernel_info_t
     _fields_ = [("grid_ctas", ctypes.c_uint64), ("threads_per_cta", ctypes.c_int32), ("regs_per_thread", ctypes.c_int32),
                 ("static_smem", ctypes.c_int32), ("dynamic_smem", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
-                ("pipe", ctypes.c_int32), ("kernel", ctypes.c_char * 120)]
+                ("pipe", ctypes.c_int32), ("kernel", ctypes.c_char * 120), ("launches", ctypes.c_int32)]
 
 
 PIPE_FMA, PIPE_TF32X3, PIPE_BF16 = 0, 1, 2

@@ -101,6 +101,7 @@ int orion_kernel_info(uint32_t fn, const uint64_t* args, uint32_t nargs, orion_k
   out->static_smem = (int32_t)fa.sharedSizeBytes;
   out->dynamic_smem = g.smem;
   out->pipe = g.pipe;
+  out->launches = g.sig_ctas ? 2 : 1;
   int b = 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, g.func, out->threads_per_cta, g.smem) != cudaSuccess) {
     (void)cudaGetLastError();

@@ -77,7 +77,7 @@ def test_encoder_iterations_vs_oracle():
 
     def step(Pp, V, x, t, first, masks, trace):
         return om.encoder_train_step(Pp, V, x, t, first=first, layers=2, masks=masks, trace=trace)
-    rep = PT.check_train_iterations(run_one, g, step, xs, ts, P, 2, "relu_in", (0.0,))
+    rep = PT.check_train_iterations(run_one, g, step, xs, ts, P, 2, "relu_in", (0.0,), trace_order="backward")
     print("encoder iterations vs oracle:", rep)
 
 
@@ -102,7 +102,7 @@ def test_rn101_hp_training_full_size_vs_oracle():
 
     def step(Pp, V, x, lab, first, masks, trace):
         return om.resnet_train_step(Pp, V, x, lab, first=first, layers=W.RESNET101_LAYERS, masks=masks, trace=trace)
-    rep = PT.check_train_iterations(run_one, hpg, step, xs, labs, Pr, 2, "relu_in", (0.0,))
+    rep = PT.check_train_iterations(run_one, hpg, step, xs, labs, Pr, 2, "relu_in", (0.0,), trace_order="backward")
     print("ResNet-101 b32 training iterations vs oracle:", rep)
 
 

@@ -77,7 +77,8 @@ def test_be_rn50_iterations_vs_oracle(cfg3):
 
     def step(P, V, x, lab, first, masks, trace):
         return om.resnet_train_step(P, V, x, lab, first=first, masks=masks, trace=trace)
-    rep = PT.check_train_iterations(run_one, be.graph, step, cfg3["xs"], cfg3["labels"], Prn, 2, "relu_in", (0.0,))
+    rep = PT.check_train_iterations(run_one, be.graph, step, cfg3["xs"], cfg3["labels"], Prn, 2, "relu_in", (0.0,),
+                                    trace_order="backward")
     print("ResNet-50 b64 BE iterations vs oracle:", rep)
 
 

@@ -35,9 +35,22 @@ EXTRA = [("tc_pct", "sm__pipe_tc_cycles_active.avg.pct_of_peak_sustained_elapsed
 
 
 def main(ncu_log, oplist, base, out_csv):
-    launches = parse(ncu_log)
+    raw = parse(ncu_log)
     ops = [l.rstrip("\n").split("\t") for l in open(oplist)]
-    assert len(launches) == len(ops), (len(launches), len(ops))
+    # an op may issue several kernels (4th oplist column): sum their durations / bytes, keep the
+    # first kernel's grid and counters (the op's main kernel)
+    launches, i = [], 0
+    for op in ops:
+        k = int(op[3]) if len(op) > 3 else 1
+        group = raw[i:i + k]
+        i += k
+        m = dict(group[0]) if group else {}
+        for extra in group[1:]:
+            for key in ("gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum"):
+                m[key] = m.get(key, 0.0) + extra.get(key, 0.0)
+        launches.append(m)
+    assert i == len(raw), (i, len(raw))
+    ops = [op[:3] for op in ops]
     with open(out_csv, "w", newline="") as f:
         w = csv.writer(f)
         w.writerow(["kernel_id", "label", "fn", "dur_ns", "sm_pct", "mem_pct", "dram_bytes", "dram_gbs", "grid"] +

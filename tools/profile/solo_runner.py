@@ -12,6 +12,7 @@ import torch  # noqa: E402
 
 import bench  # noqa: E402
 import paper_conf_eurosys_stratimk24_b200 as orion  # noqa: E402
+from paper_conf_eurosys_stratimk24_b200.runtime import kernel_info  # noqa: E402
 
 
 def main():
@@ -31,8 +32,8 @@ def main():
     torch.cuda.synchronize()
     with open(os.path.join(ROOT, "gpurun_out", f"oplist_{a.config}_{a.client}.txt"), "w") as f:
         for i, (fn, args, lab) in enumerate(g.ops):
-            if isinstance(fn, str):
-                f.write(f"{i}\t{fn}\t{lab}\n")
+            if isinstance(fn, str):   # kernels per op launch (2 = split partials + ordered combine)
+                f.write(f"{i}\t{fn}\t{lab}\t{kernel_info(fn, args)['launches']}\n")
 
 
 if __name__ == "__main__":
