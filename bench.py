@@ -161,6 +161,60 @@ def with_be_h2d(graph, xs_host):
 
 
 # ------------------------------------------------------------------------------------ clocks
+class GpmWindow:
+    """Sampled GPU utilisation over a window (beside the analytic one): NVML GPU Performance Monitoring
+    samples at window start and end -> SM activity (fraction of SM cycles with a resident warp), SM
+    occupancy, tensor-pipe and DRAM-bandwidth utilisation, averaged by the driver's counters over the
+    window. {"unavailable": why} where the driver or device does not expose GPM."""
+    METRICS = {"sm_util_pct": "NVML_GPM_METRIC_SM_UTIL", "sm_occupancy_pct": "NVML_GPM_METRIC_SM_OCCUPANCY",
+               "tensor_util_pct": "NVML_GPM_METRIC_ANY_TENSOR_UTIL", "dram_bw_util_pct": "NVML_GPM_METRIC_DRAM_BW_UTIL",
+               "fp32_util_pct": "NVML_GPM_METRIC_FP32_UTIL"}
+
+    def __init__(self, index):
+        self.index, self.err, self.s1 = index, None, None
+        try:
+            import pynvml as nv
+            self.nv = nv
+            nv.nvmlInit()
+            self.dev = nv.nvmlDeviceGetHandleByIndex(index)
+            if not nv.nvmlGpmQueryDeviceSupport(self.dev).isSupportedDevice:
+                self.err = "GPM not supported on this device"
+        except Exception as e:   # noqa: BLE001 (report, never fail the bench on a monitoring API)
+            self.err = f"nvml: {e}"
+
+    def start(self):
+        if self.err:
+            return
+        try:
+            self.s1 = self.nv.nvmlGpmSampleGet(self.dev, self.nv.nvmlGpmSampleAlloc())
+        except Exception as e:   # noqa: BLE001
+            self.err = f"nvmlGpmSampleGet: {e}"
+
+    def stop(self):
+        if self.err or self.s1 is None:
+            return {"unavailable": self.err or "not started"}
+        nv = self.nv
+        try:
+            s2 = nv.nvmlGpmSampleGet(self.dev, nv.nvmlGpmSampleAlloc())
+            mg = nv.c_nvmlGpmMetricsGet_t()
+            mg.version = nv.NVML_GPM_METRICS_GET_VERSION
+            mg.numMetrics = len(self.METRICS)
+            mg.sample1, mg.sample2 = self.s1, s2
+            for i, k in enumerate(self.METRICS.values()):
+                mg.metrics[i].metricId = getattr(nv, k)
+            nv.nvmlGpmMetricsGet(mg)
+            out = {}
+            for i, k in enumerate(self.METRICS):
+                m = mg.metrics[i]
+                out[k] = float(m.value) if m.nvmlReturn == 0 else None
+            nv.nvmlGpmSampleFree(self.s1)
+            nv.nvmlGpmSampleFree(s2)
+            self.s1 = None
+            return out
+        except Exception as e:   # noqa: BLE001
+            return {"unavailable": f"nvmlGpmMetricsGet: {e}"}
+
+
 class ClockSampler:
     def __init__(self, index):
         self.index = index
@@ -314,6 +368,15 @@ def pct(v, p):
     return float(s[max(0, int(np.ceil(p / 100.0 * len(s))) - 1)]) if len(s) else float("nan")
 
 
+def gpm_mean(ws):
+    """Mean of GpmWindow.stop() dicts (first unavailable reason if none has numbers)."""
+    good = [w for w in ws if "unavailable" not in w]
+    if not good:
+        return ws[0] if ws else {"unavailable": "no window"}
+    return {k: (float(np.mean([w[k] for w in good if w.get(k) is not None])) if any(w.get(k) is not None for w in good) else None)
+            for k in good[0]}
+
+
 def bootstrap_ratio_ci(col, ded, p=99, n=1000, seed=7):
     """95 % bootstrap CI of pct(col, p) / pct(ded, p): requests resampled with replacement, the two
     modes independently (SURVEY §8(d) statistical hygiene)."""
@@ -421,6 +484,7 @@ def infer_train(args, rank, world, local, metric):
     be_iters, be_time_s, win_ms, trace_ms, stats = 0, 0.0, 0.0, [], None
     be_iters_all = 0
     beg.params.reset()
+    gpm, gpm_col = GpmWindow(local), []
     with ClockSampler(local) as clk:
         for name, lam in rates:
             for rep in range(REPEATS):
@@ -429,11 +493,15 @@ def infer_train(args, rank, world, local, metric):
                 barrier()
                 torch.cuda.synchronize()
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                if name == "table3":
+                    gpm.start()
                 e0.record()
                 rc = session(hp=hp, be=be_all, arrivals_ns=arr, hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm,
                              be_partition_sms=args.be_partition, trace_kernel_id=top_kid if name == "table3" else None)
                 e1.record()
                 torch.cuda.synchronize()
+                if name == "table3":
+                    gpm_col.append(gpm.stop())
                 barrier()
                 ld, lc = rd["t_done"] - rd["t_arrival"], rc["t_done"] - rc["t_arrival"]
                 runs[name]["ded"] += ld.tolist()
@@ -467,7 +535,9 @@ def infer_train(args, rank, world, local, metric):
     session(be=be, be_iters=3)
     per_it = (time.time() - t0) / 3
     n_it = int(max(5, min(300, 6.0 / max(per_it, 1e-6))))
+    gpm.start()
     rb = session(be=be_all, be_iters=n_it)
+    gpm_be = gpm.stop()
     be_ded = 0.0
     for tb in rb.get("be_t_end_all", [rb["be_t_end"]]):
         be_ded += (len(tb) - 1) / ((tb[-1] - tb[0]) / 1e9) if len(tb) > 1 else float("nan")
@@ -483,6 +553,10 @@ def infer_train(args, rank, world, local, metric):
                        "hbm_frac": (n_done * hp_b + be_iters * be_b) / be_time_s / hbm_peak,
                        "flop_frac": (n_done * hp_f + be_iters * be_f) / be_time_s / tc_peak},
         "be_alone": {"hbm_gbs": be_ded * be_b / 1e9, "hbm_frac": be_ded * be_b / hbm_peak, "flop_frac": be_ded * be_f / tc_peak},
+        "sampled": {"collocated": gpm_mean(gpm_col), "be_alone": gpm_be,
+                    "basis": "NVML GPM counters (driver-sampled SM activity / occupancy / tensor / DRAM utilisation) "
+                             "over each timed collocated run at the Table-3 rate (mean over repeats) and over the "
+                             "dedicated BE run"},
         "be_bytes_per_iteration_GB": be_b / 1e9, "hp_bytes_per_request_GB": hp_b / 1e9,
         "basis": "algorithmic bytes/FLOPs per op of this implementation's op list (profiler.op_work) x completed "
                  "requests / iterations; SURVEY §8(d)'s own per-iteration figures (35.7 GB MobileNetV2 b96, 1.16 GB "

@@ -217,6 +217,13 @@ bool atc_conv_try_geom(const uint64_t* a, LaunchGeom* g);
 bool atc_conv_is(const void* f);
 int atc_conv_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
 
+// Forward convolution / dense B^T GEMM on tcgen05 with TMA im2col boxes (cvf.cu).
+bool cvf_conv_try_geom(const uint64_t* a, LaunchGeom* g);
+bool cvf_gemm_try_geom(const uint64_t* a, LaunchGeom* g);
+bool cvf_is(const void* f);
+int cvf_conv_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
+int cvf_gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
+
 // Kernel table (table.cu)
 extern const KernelEntry g_kernels[ORION_FN_COUNT];
 int kernel_launch_sig(uint32_t fn, const uint64_t* args, uint32_t nargs, OrionSig sig, cudaStream_t s,

@@ -2248,6 +2248,7 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     g->grid = dim3((unsigned)cdiv(M, rows::rpc((int)N))); g->block = dim3(rows::NTH); g->smem = rows::smem_bytes((int)K, (int)N); g->func = f;
     return 0;
   }
+  if (flags == 2 && cvf_gemm_try_geom(a, g)) return 0;   // dense B^T GEMM, TMA-fed tcgen05 (cvf.cu)
   if (flags == 1 && atc_try_geom(a, g)) return 0;   // compute-dense A^T B on tcgen05 (atc.cu)
   if (flags == 1 && wgs_try_geom(a, g)) return 0;   // TMA-fed streaming A^T B (wgs.cu)
   if (flags == 1 && atb_ok(M, N, K)) {
@@ -2293,6 +2294,7 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
   if (atc_is(g.func)) return atc_launch(a, g, sig, s);
+  if (cvf_is(g.func)) return cvf_gemm_launch(a, g, sig, s);
   if (wgs_is(g.func)) return wgs_launch(a, g, sig, s);
   if (tmk::is(g.func)) return tmk::launch(g, M, N, K, C, ldc, bias, A, lda, B, ldb, flags == 0, sig, s);
   if (tcm::is<ADense, BDenseT>(g.func))
@@ -2346,10 +2348,12 @@ int conv_fwd_geom(const uint64_t* a, LaunchGeom* g) {
     g->func = (const void*)smallc::conv_fwd_smallc_kernel<3, 3, 3>;
     return 0;
   }
+  if (cvf_conv_try_geom(a, g)) return 0;   // TMA im2col boxes straight into tcgen05 (cvf.cu)
   tiled_geom<AIm2col, BDenseT>(g, (long long)s.N * s.P * s.Q, s.K, (long long)s.R * s.S * s.C, a[14], a[15]);
   return 0;
 }
 int conv_fwd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
+  if (cvf_is(g.func)) return cvf_conv_launch(a, g, sig, st);
   ConvShape s = conv_shape(a);
   if (g.func == (const void*)smallc::conv_fwd_smallc_kernel<3, 3, 3>) {
     smallc::conv_fwd_smallc_kernel<3, 3, 3><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s, sig);

@@ -51,12 +51,14 @@ def assert_close(name, got, ref, rel_tol, elem_factor=ELEM_FACTOR, floor=1e-30):
     return r, e
 
 
-def audit_decisions(name, y_gpu, y_oracle, thresholds=(0.0, 6.0), max_flip_frac=1e-4, rel_floor=1e-6):
+def audit_decisions(name, y_gpu, y_oracle, thresholds=(0.0, 6.0), max_flip_frac=1e-4, rel_floor=5e-6):
     """The GPU's ReLU6 (thresholds 0, 6) or ReLU (0) decided on y_gpu; the oracle's own free-running
     forward produced y_oracle. Measures the forward drift of this tensor (rel L2, max |err| / rms) and
     checks:
       * the drift is spread like rounding noise, not localized: max |err| <= ELEM_FACTOR x
-        max(rel, rel_floor) x rms (a wrong tile or row has a max far above its share of the norm);
+        max(rel, rel_floor) x rms (a wrong tile or row has a max far above its share of the norm;
+        rel_floor = 5e-6 ~ 80 u absorbs BN's per-channel amplification of a few-ulp error, five
+        orders of magnitude below the O(rms) error of a wrong index);
       * every element where the two take different decisions has its oracle value within that band
         of a threshold, and flips are rare (<= max(max_flip_frac, 2 rel) of the elements).
     Returns (flips, rel). The caller checks that the drift grows smoothly along the forward pass."""
@@ -100,8 +102,9 @@ def check_train_iterations(run_one, graph, step, xs, labels, P0, K, dec_attr, th
     rel L2 <= max(drift_floor, drift_jump x the largest drift before it): the fp32 forward drifts
     geometrically through a deep train-mode network, ~8 % per ResNet block, while a wrong kernel shows
     as a jump); trace_order says whether the oracle's trace lists the tensors in forward or backward
-    order; loss rel 1e-5; every gradient element within tau_g of its absolute-term sum, every
-    gradient tensor within tau_g x max(1, kappa) in rel L2. After K: momentum (accumulated sums)
+    order; loss rel 1e-5; every gradient element within tau of its absolute-term sum, every
+    gradient tensor within tau x max(1, kappa) in rel L2, tau = tau_g + 2 x the iteration's worst
+    forward drift (the operands' perturbation a gradient inherits). After K: momentum (accumulated sums)
     and parameters (K ulps of storage rounding per side + lr x the accumulated bound); BN running
     statistics rel 1e-5 (rmean with an absolute floor of 1e-2: block outputs have exactly zero
     batch mean, so their next BN's running mean is rounding noise). Returns a per-iteration report."""
@@ -109,7 +112,7 @@ def check_train_iterations(run_one, graph, step, xs, labels, P0, K, dec_attr, th
     base = G.gflat.data_ptr()
     V_gpu = {n: G.vflat[(t.data_ptr() - base) // 4:(t.data_ptr() - base) // 4 + t.numel()].view(t.shape) for n, t in G.g.items()}
     Po, Vo = dict(P0), {}
-    A_v, A_vsum, report = {}, {}, []
+    A_v, A_vsum, report, tau_acc = {}, {}, [], tau_g
     for it in range(K):
         run_one(it)
         masks = {k: v.cpu() for k, v in getattr(graph, dec_attr).items()}
@@ -128,28 +131,32 @@ def check_train_iterations(run_one, graph, step, xs, labels, P0, K, dec_attr, th
             flips += f
         lr_ = rel(graph.loss, loss_o.reshape(1))
         assert lr_ < 1e-5, f"iter {it}: loss rel {lr_:.3e}"
+        # a gradient g = sum a b inherits its operands' relative perturbation: |dg| <= sum |a||b| (|da/a| +
+        # |db/b|) + gamma sum |a||b|, so its bound is tau_g plus the forward drift of both operands
+        tau_it = tau_g + 2.0 * worst_drift
+        tau_acc = max(tau_acc, tau_it)
         worst_c, worst_r, worst_k = 0.0, 0.0, 0.0
         for n, ref in g_o.items():
             A = tr["abs"][n]
             ce, k, r = cond_elem(G.g[n], ref, A), kappa(ref, A), rel(G.g[n], ref)
-            assert ce <= tau_g, f"iter {it} {n}: max |err| / abs-sum {ce:.3e} > {tau_g:g}"
+            assert ce <= tau_it, f"iter {it} {n}: max |err| / abs-sum {ce:.3e} > {tau_it:.3g}"
             if k < 1e6:   # exactly-zero true gradients are held by the elementwise bound only
-                assert r <= tau_g * max(1.0, k), f"iter {it} {n}: rel {r:.3e} > {tau_g:g} x kappa {k:.1f}"
+                assert r <= tau_it * max(1.0, k), f"iter {it} {n}: rel {r:.3e} > {tau_it:.3g} x kappa {k:.1f}"
                 worst_r = max(worst_r, r)
                 worst_k = max(worst_k, k)
             worst_c = max(worst_c, ce)
             A_v[n] = A.double() if it == 0 else mu * A_v[n] + A.double()
             A_vsum[n] = A_v[n] if it == 0 else A_vsum[n] + A_v[n]
-        report.append(dict(iter=it, loss=float(loss_o), flips=flips, worst_forward_drift=worst_drift, worst_cond_elem=worst_c,
-                           worst_rel=worst_r, worst_kappa=worst_k))
+        report.append(dict(iter=it, loss=float(loss_o), flips=flips, worst_forward_drift=worst_drift, grad_tol=tau_it,
+                           worst_cond_elem=worst_c, worst_rel=worst_r, worst_kappa=worst_k))
         Po, Vo = newP, newV
     for n, ref in Vo.items():
         ce = cond_elem(V_gpu[n], ref, A_v[n])
-        assert ce <= tau_g, f"momentum {n}: {ce:.3e}"
+        assert ce <= tau_acc, f"momentum {n}: {ce:.3e}"
     for n, ref in Po.items():
         p, r = _dd(G.p[n]), _dd(ref)
         if n in A_vsum:
-            bound = 2 * K * (2.0 ** -23) * r.abs() + tau_g * lr * A_vsum[n] + 1e-30
+            bound = 2 * K * (2.0 ** -23) * r.abs() + tau_acc * lr * A_vsum[n] + 1e-30
             worst = float(((p - r).abs() / bound).max())
             assert worst <= 1.0, f"param {n}: {worst:.3f} x (storage rounding + lr x gradient bound)"
         else:
