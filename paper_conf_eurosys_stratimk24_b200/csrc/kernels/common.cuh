@@ -34,16 +34,16 @@ struct OrionSig {
 
 __device__ __forceinline__ void orion_signal(const OrionSig& sig) {
   if (sig.ticket == nullptr) return;  // direct launch (no scheduler)
-  // bar.sync orders the CTA's writes before thread 0; its gpu-scope fence is cumulative over what
-  // it observed through the barrier (the release pattern CUTLASS semaphores use)
+  // Completion only: the counter tells the scheduler THAT the launch finished (HP busy test, BE
+  // in-flight accounting); no consumer reads the kernel's data through it (later kernels and the
+  // D2H memops see the data by stream order), so no memory fence is needed -- a gpu- and a
+  // system-scope fence per kernel cost microseconds on the HP critical path (tools/diag_launch.py).
+  // bar.sync: every thread of this CTA has finished before its CTA is counted.
   __syncthreads();
   if (threadIdx.x == 0 && threadIdx.y == 0 && threadIdx.z == 0) {
-    __threadfence();
-    unsigned long long t = atomicAdd(sig.ticket, 1ull) + 1ull;
-    if (t == sig.target) {
-      __threadfence_system();
-      asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(sig.done), "l"(sig.seq) : "memory");
-    }
+    unsigned long long t;
+    asm volatile("atom.relaxed.gpu.global.add.u64 %0, [%1], 1;" : "=l"(t) : "l"(sig.ticket) : "memory");
+    if (t + 1ull == sig.target) asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(sig.done), "l"(sig.seq) : "memory");
   }
 }
 

@@ -12,7 +12,8 @@
 //    SWIZZLE_128B layout. A slab of B is one box of the [K][R*S][C] weights. No thread computes an
 //    address per element.
 //  * warps 4-7 form lo = x - trunc_tf32(x) of both operands (elementwise, layout-preserving); warp 8
-//    lane 0 issues TMA; warp 9 lane 0 issues the MMAs into two TMEM accumulators (main, corr).
+//    lane 0 issues TMA; warp 9 lane 0 issues the MMAs into three TMEM accumulators (hi*hi of even
+//    and of odd slabs, corrections).
 //  * small problems (HP inference: a few dozen tiles) split the slabs over a thread-block cluster of
 //    <= 8 CTAs along z; the partial tiles meet in distributed shared memory and each CTA sums a
 //    row slice of all of them in rank order, so the result is deterministic, needs no workspace and
@@ -22,6 +23,7 @@
 //    (kernels are not preemptible).
 #include <algorithm>
 #include <atomic>
+#include <cstdlib>
 
 #include "common.cuh"
 #include "tma.cuh"
@@ -40,7 +42,9 @@ struct Cfg {
   static constexpr int STAGES = (196 * 1024) / STAGE > 6 ? 6 : (196 * 1024) / STAGE;
   static constexpr int TS = BN + 4;                       // staging row stride (floats), conflict-free
   static constexpr int SMEM = STAGES * STAGE + 1024 + 256;
-  static constexpr int TMEM_COLS = 2 * BN;
+  // accumulators: hi*hi of even slabs, of odd slabs, and the correction products (3 BN columns): the
+  // tensor core's fp32 accumulation truncates, so shorter chains keep the bias down
+  static constexpr int TMEM_COLS = 3 * BN <= 256 ? 256 : 512;
   // kind::tf32: D fp32 (bit 4), A, B tf32 (bits 7, 10), both K-major, N>>3 at 17, M>>4 at 24
   static constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
   static_assert(BM * TS * 4 <= STAGES * STAGE, "staging tile fits in the stage ring");
@@ -56,6 +60,7 @@ struct Params {
   float* y;
   long long ldy;
   const float* bias;
+  int dbg;   // measurement switches (ORION_CVF_DEBUG): 1 converters idle, 2 no MMAs, 4 no TMA loads, 8 no epilogue
 };
 
 // UMMA descriptor, K-major SWIZZLE_128B: 8-row atoms of 128-byte rows, SBO = 1024 B, layout type 2
@@ -146,6 +151,7 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
         const int s = it % S;
         if (it >= S) mbar_wait(empty0 + 8 * s, ((uint32_t)(it / S) & 1u) ^ 1u);
         const uint32_t st = smem_u32(smem + s * STAGE), bar = full0 + 8 * s;
+        if (p.dbg & 4) { mbar_arrive(bar); continue; }
         mbar_expect(bar, tx);
         const int slab = s0 + it, tap = slab / p.CB, cb = slab - tap * p.CB;
         const int r = tap / p.S, sx = tap - r * p.S;
@@ -168,6 +174,11 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
       float4* alo = reinterpret_cast<float4*>(st + A_BYTES);
       const float4* bhi = reinterpret_cast<const float4*>(st + 2 * A_BYTES);
       float4* blo = reinterpret_cast<float4*>(st + 2 * A_BYTES + B_BYTES);
+      if (p.dbg & 1) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive(conv0 + 8 * s);
+        continue;
+      }
       float4 va[8], vb[BN / 16];
 #pragma unroll
       for (int j = 0; j < 8; j++) {
@@ -197,35 +208,44 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
       asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
       const uint32_t st = smem_u32(smem + s * STAGE);
       const uint32_t a_hi = st, a_lo = st + A_BYTES, b_hi = st + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
-      const uint32_t d_main = tmem, d_corr = tmem + BN;
+      const uint32_t d_main = tmem + (uint32_t)((it & 1) * BN), d_corr = tmem + 2 * BN;
 #pragma unroll
-      for (int j = 0; j < BK / 8; j++) {
+      for (int j = 0; j < ((p.dbg & 2) ? 0 : BK / 8); j++) {
         const uint64_t dah = sdesc128(a_hi + 32 * j), dal = sdesc128(a_lo + 32 * j);
         const uint64_t dbh = sdesc128(b_hi + 32 * j), dbl = sdesc128(b_lo + 32 * j);
         mma_tf32(d_corr, dal, dbh, C_::IDESC, (it | j) != 0);
         mma_tf32(d_corr, dah, dbl, C_::IDESC, 1);
-        mma_tf32(d_main, dah, dbh, C_::IDESC, (it | j) != 0);
+        mma_tf32(d_main, dah, dbh, C_::IDESC, ((it >> 1) | j) != 0);
       }
       mma_commit(empty0 + 8 * s);
     }
     mma_commit(done_bar);
-  } else if (warp < 4) {
+  } else if (warp < 4 && !(p.dbg & 8)) {
     // TMEM -> registers -> staging tile [128][TS] (the stage ring is idle once done_bar fired)
     mbar_wait(done_bar, 0);
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     float* tilep = reinterpret_cast<float*>(smem);
 #pragma unroll 1
     for (int c0 = 0; c0 < BN; c0 += 32) {
-      uint32_t mv[32], cv[32];
+      uint32_t ev[32], ov[32], cv[32];
       const uint32_t base = tmem + ((uint32_t)(32 * warp) << 16) + (uint32_t)c0;
-      tmem_ld32(base, mv);
-      tmem_ld32(base + BN, cv);
+      tmem_ld32(base, ev);
+      tmem_ld32(base + 2 * BN, cv);
+      if (nsl > 1) tmem_ld32(base + BN, ov);
       asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+      if (nsl <= 1) {
 #pragma unroll
-      for (int j = 0; j < 32; j += 4)
-        *reinterpret_cast<float4*>(tilep + tid * TS + c0 + j) =
-            make_float4(__uint_as_float(mv[j]) + __uint_as_float(cv[j]), __uint_as_float(mv[j + 1]) + __uint_as_float(cv[j + 1]),
-                        __uint_as_float(mv[j + 2]) + __uint_as_float(cv[j + 2]), __uint_as_float(mv[j + 3]) + __uint_as_float(cv[j + 3]));
+        for (int j = 0; j < 32; j++) ov[j] = 0u;   // +0.0f: the odd chain is empty
+      }
+#pragma unroll
+      for (int j = 0; j < 32; j += 4) {
+        float4 v;
+        v.x = (__uint_as_float(ev[j]) + __uint_as_float(ov[j])) + __uint_as_float(cv[j]);
+        v.y = (__uint_as_float(ev[j + 1]) + __uint_as_float(ov[j + 1])) + __uint_as_float(cv[j + 1]);
+        v.z = (__uint_as_float(ev[j + 2]) + __uint_as_float(ov[j + 2])) + __uint_as_float(cv[j + 2]);
+        v.w = (__uint_as_float(ev[j + 3]) + __uint_as_float(ov[j + 3])) + __uint_as_float(cv[j + 3]);
+        *reinterpret_cast<float4*>(tilep + tid * TS + c0 + j) = v;
+      }
     }
   }
   asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
@@ -233,7 +253,7 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
   if (p.split > 1) cluster_sync();   // every partial tile of the cluster is staged
 
   // ---------------- sum the partial tiles of this CTA's row slice in rank order, store
-  {
+  if (!(p.dbg & 8)) {
     const int per = (p.rows + p.split - 1) / p.split;
     const int r_lo = z * per, r_hi = min(p.rows, r_lo + per);
     constexpr int QPR = BN / 4;
@@ -301,6 +321,37 @@ inline bool shape_ok(const Shape& s) {
   return encoder() != nullptr;
 }
 
+template <int BN>
+bool prepare() {
+  static std::atomic<int> done{0};
+  if (done.load(std::memory_order_acquire)) return true;
+  const bool okk = cudaFuncSetAttribute((const void*)cvf_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<BN>::SMEM) == cudaSuccess;
+  if (okk) done.store(1, std::memory_order_release);
+  return okk;
+}
+
+// clusters of `split` CTAs the device runs at once (cudaOccupancyMaxActiveClusters; measured once per
+// (BN, split)): GPC sizes, not the SM count, bound a cluster wave (e.g. 15 clusters of 8 on 148 SMs)
+inline int max_clusters(int BN, int split) {
+  static std::atomic<int> cache[2][MAX_SPLIT + 1];
+  const int b = BN == 128 ? 1 : 0;
+  int v = cache[b][split].load(std::memory_order_relaxed);
+  if (v > 0) return v;
+  int n = 0;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(1, 1, (unsigned)split); cfg.blockDim = dim3(NTHR);
+  cfg.dynamicSmemBytes = BN == 128 ? Cfg<128>::SMEM : Cfg<64>::SMEM;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = 1; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = (unsigned)split;
+  cfg.attrs = at; cfg.numAttrs = 1;
+  const bool ok = BN == 128 ? prepare<128>() && cudaOccupancyMaxActiveClusters(&n, cvf_kernel<128>, &cfg) == cudaSuccess
+                            : prepare<64>() && cudaOccupancyMaxActiveClusters(&n, cvf_kernel<64>, &cfg) == cudaSuccess;
+  if (!ok || n <= 0) { (void)cudaGetLastError(); n = 148 / split; }
+  cache[b][split].store(n, std::memory_order_relaxed);
+  return n;
+}
+
 inline Plan plan(const Shape& s) {
   Plan pl;
   if (s.Q <= 128) {
@@ -316,25 +367,21 @@ inline Plan plan(const Shape& s) {
   pl.nqb = (int)cdivl(s.Q, pl.QB);
   pl.nnb = (int)cdivl(s.NI, pl.NB);
   const long long tiles_m = (long long)pl.nqb * pl.npb * pl.nnb;
-  pl.BN = (s.K > 64 && tiles_m * cdivl(s.K, 128) >= 120) ? 128 : 64;
+  static const int force_bn = getenv("ORION_CVF_BN") ? atoi(getenv("ORION_CVF_BN")) : 0;   // tuning knobs
+  static const int max_split = getenv("ORION_CVF_MAXSPLIT") ? std::max(1, std::min(MAX_SPLIT, atoi(getenv("ORION_CVF_MAXSPLIT")))) : MAX_SPLIT;
+  pl.BN = force_bn == 64 || force_bn == 128 ? force_bn : (s.K > 64 && tiles_m * cdivl(s.K, 128) >= 120) ? 128 : 64;
   pl.tiles_n = (int)cdivl(s.K, pl.BN);
   pl.tiles = (int)(tiles_m * pl.tiles_n);
   pl.nk = (int)(s.R * s.S * cdivl(s.C, 32));
   int split = 1;
-  if (pl.tiles < 148) split = std::max(1, std::min({MAX_SPLIT, 148 / pl.tiles, pl.nk / 2}));
+  if (pl.tiles < 148) split = std::max(1, std::min({max_split, 148 / pl.tiles, pl.nk / 2}));
+  // a cluster of `split` CTAs needs `split` free SMs in one GPC: keep all clusters in one wave
+  while (split > 1 && pl.tiles > max_clusters(pl.BN, split)) split--;
   pl.kps = (int)cdivl(pl.nk, split);
   pl.split = (int)cdivl(pl.nk, pl.kps);
   return pl;
 }
 
-template <int BN>
-bool prepare() {
-  static std::atomic<int> done{0};
-  if (done.load(std::memory_order_acquire)) return true;
-  const bool okk = cudaFuncSetAttribute((const void*)cvf_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<BN>::SMEM) == cudaSuccess;
-  if (okk) done.store(1, std::memory_order_release);
-  return okk;
-}
 
 inline bool geom(const Shape& s, LaunchGeom* g) {
   if (!shape_ok(s)) return false;
@@ -386,6 +433,8 @@ int launch_t(const Shape& s, const Plan& pl, const LaunchGeom& g, OrionSig sig, 
   p.stride = (int)s.stride; p.pad = (int)s.pad; p.S = (int)s.S; p.CB = (int)cdivl(s.C, 32); p.taps = (int)(s.R * s.S);
   p.Kout = (int)s.K; p.tiles_n = pl.tiles_n; p.nk = pl.nk; p.kps = pl.kps; p.split = pl.split;
   p.y = s.y; p.ldy = s.ldy; p.bias = s.bias;
+  static const int dbg = getenv("ORION_CVF_DEBUG") ? atoi(getenv("ORION_CVF_DEBUG")) : 0;
+  p.dbg = dbg;
   if (pl.split == 1) {
     cvf_kernel<BN><<<g.grid, g.block, g.smem, st>>>(ma, mb, p, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;

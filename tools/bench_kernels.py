@@ -1,6 +1,6 @@
 """Warm per-launch CUDA-event times of the BE operators at MobileNetV2-b96 shapes (weight-gradient
 GEMMs, depthwise fwd / dgrad / wgrad), with algorithmic GB/s. Inputs > L2 for the large shapes.
-Usage: python tools/bench_kernels.py [wgs|dw|all]"""
+Also the HP ResNet-50 b4 forward convolutions / 1x1 GEMMs (conv). Usage: python tools/bench_kernels.py [wgs|dw|conv|all]"""
 import os
 import sys
 
@@ -12,6 +12,23 @@ from paper_conf_eurosys_stratimk24_b200.runtime import kernel_info  # noqa: E402
 
 
 def timeit(fn, args, reps=20):
+    if os.environ.get("BENCH_GRAPH"):   # device-bound: replay a captured graph of `reps` launches
+        st = torch.cuda.Stream()
+        for _ in range(3):
+            orion.kernel_launch(fn, args, st.cuda_stream)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=st):
+            for _ in range(reps):
+                orion.kernel_launch(fn, args, st.cuda_stream)
+        g.replay()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        g.replay()
+        e1.record()
+        torch.cuda.synchronize()
+        return e0.elapsed_time(e1) / reps * 1e3
     s = torch.cuda.current_stream().cuda_stream
     for _ in range(3):
         orion.kernel_launch(fn, args, s)
@@ -35,6 +52,46 @@ WGS = [(96, 16, 1204224), (16, 32, 1204224), (24, 96, 301056), (144, 24, 301056)
 DW = [(96, 112, 32, 1), (96, 112, 96, 2), (96, 56, 144, 1), (96, 56, 144, 2), (96, 28, 192, 1), (96, 28, 192, 2),
       (96, 14, 384, 1), (96, 14, 576, 1), (96, 14, 576, 2), (96, 7, 960, 1)]
 
+
+
+HP_CONV = [(4, 56, 56, 64, 64, 3, 1, 1), (4, 56, 56, 128, 128, 3, 2, 1), (4, 28, 28, 128, 128, 3, 1, 1), (4, 28, 28, 256, 256, 3, 2, 1),
+           (4, 14, 14, 256, 256, 3, 1, 1), (4, 14, 14, 512, 512, 3, 2, 1), (4, 7, 7, 512, 512, 3, 1, 1),
+           (4, 56, 56, 256, 512, 1, 2, 0), (4, 28, 28, 512, 1024, 1, 2, 0), (4, 14, 14, 1024, 2048, 1, 2, 0)]
+HP_GEMM = [(12544, 64, 64), (12544, 64, 256), (12544, 256, 64), (12544, 128, 256), (3136, 512, 128), (3136, 128, 512),
+           (3136, 256, 512), (784, 1024, 256), (784, 256, 1024), (784, 512, 1024), (196, 2048, 512), (196, 512, 2048)]
+
+
+def conv():
+    tot = 0.0
+    for n, h, w_, c, k, r, st, pad in HP_CONV:
+        p, q = (h + 2 * pad - r) // st + 1, (w_ + 2 * pad - r) // st + 1
+        x, wt, y = torch.randn(n, h, w_, c, device="cuda"), torch.randn(k, r, r, c, device="cuda"), torch.zeros(n, p, q, k, device="cuda")
+        wf = ws(L.lib.orion_gemm_workspace_bytes(n * p * q, k, r * r * c))
+        a = [x.data_ptr(), wt.data_ptr(), y.data_ptr(), n, h, w_, c, k, r, r, st, pad, p, q, wf.data_ptr(), wf.numel() * 4]
+        t = timeit("conv_fwd", a)
+        tot += t
+        info = kernel_info("conv_fwd", a)
+        print(f"conv {n}x{h}x{w_}x{c}->{k} r{r} s{st} {t:7.1f} us {2 * n * p * q * k * r * r * c / t / 1e6:6.1f} TF  grid {info['grid_ctas']} "
+              f"{info['kernel'][:40]}")
+    for M, N, K in HP_GEMM:
+        A, B, C = torch.randn(M, K, device="cuda"), torch.randn(N, K, device="cuda"), torch.zeros(M, N, device="cuda")
+        w = ws(L.lib.orion_gemm_workspace_bytes(M, N, K))
+        a = [A.data_ptr(), B.data_ptr(), C.data_ptr(), 0, M, N, K, K, K, N, 2, w.data_ptr(), w.numel() * 4]
+        t = timeit("gemm", a)
+        tot += t
+        info = kernel_info("gemm", a)
+        print(f"gemm M={M:5d} N={N:5d} K={K:5d} {t:7.1f} us {2 * M * N * K / t / 1e6:6.1f} TF  grid {info['grid_ctas']} {info['kernel'][:40]}")
+    print(f"conv+gemm total {tot:.1f} us")
+
+
+def floor():
+    """Graph-replayed duration of trivial launches: the per-kernel floor the HP path pays."""
+    x = torch.zeros(1024, device="cuda")
+    t = timeit("relu", [x.data_ptr(), x.data_ptr(), x.numel()])
+    print(f"relu 1024 floats {t:6.2f} us")
+    x = torch.zeros(4 * 56 * 56 * 64, device="cuda")
+    t = timeit("relu", [x.data_ptr(), x.data_ptr(), x.numel()])
+    print(f"relu 4x56x56x64 {t:6.2f} us")
 
 def wgs():
     tot = 0.0
@@ -76,3 +133,7 @@ if __name__ == "__main__":
         wgs()
     if what in ("dw", "all"):
         dw()
+    if what in ("conv", "all"):
+        conv()
+    if what in ("floor", "all"):
+        floor()

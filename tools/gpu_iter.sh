@@ -17,7 +17,7 @@ if [ -n "$CLIENTS" ]; then
   head -60 gpurun_out/show_times.txt
 fi
 if [ -n "$FOCUS" ]; then
-  OURS='(gemm_|gemv_bt_kernel|conv_fwd_smallc|unary_kernel|binary_kernel|bn_|dw_|maxpool_kernel|maxpool_bwd_kernel|attention_kernel|layernorm_kernel|gelu_kernel|add_bf16_kernel|embed_kernel|col2im_kernel|ln_fwd_kernel|ln_bwd_kernel|attn_|avgpool|ce_kernel|mse_kernel|sgd_kernel|colsum_kernel|smallc_kernel|smallc2_kernel|wgs_kernel|atc_)'
+  OURS='(gemm_|gemv_bt_kernel|conv_fwd_smallc|unary_kernel|binary_kernel|bn_|dw_|maxpool_kernel|maxpool_bwd_kernel|attention_kernel|layernorm_kernel|gelu_kernel|add_bf16_kernel|embed_kernel|col2im_kernel|ln_fwd_kernel|ln_bwd_kernel|attn_|avgpool|ce_kernel|mse_kernel|sgd_kernel|colsum_kernel|smallc_kernel|smallc2_kernel|wgs_kernel|atc_|cvf_kernel)'
   timeout -s KILL 600 ncu --set full --import-source on --clock-control none --kernel-name-base function -k "regex:$OURS" -c ${FOCUS_COUNT:-1} \
     -o gpurun_out/focus_${FOCUS//./_} python tools/profile/solo_runner.py --config ${CONFIG:-rn50_mnv2} --client ${FOCUS_CLIENT:-be} --only "$FOCUS" > gpurun_out/focus.log 2>&1
   ncu -i gpurun_out/focus_${FOCUS//./_}.ncu-rep --page details > gpurun_out/focus_${FOCUS//./_}.txt 2>&1
