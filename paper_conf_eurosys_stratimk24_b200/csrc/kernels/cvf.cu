@@ -128,6 +128,10 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
   const int q0 = qb * p.QB, p0 = pb * p.PB, n0 = nb * p.NB, k0 = kb * BN;
   const int s0 = z * p.kps, nsl = min(p.nk, s0 + p.kps) - s0;
   const uint32_t tx = (uint32_t)(p.QB * p.PB * p.NB * 128 + BN * 128);
+  // no K split: the epilogue writes rows straight from TMEM (one 128-byte run per thread per
+  // 32-column chunk), skipping the staging tile and the reduction pass
+  const bool direct = p.split == 1;
+  const bool dvec = (p.ldy & 3) == 0 && (reinterpret_cast<uintptr_t>(p.y) & 15) == 0;
 
   if (tid == 0) {
     for (int s = 0; s < S; s++) { mbar_init(full0 + 8 * s, 1); mbar_init(conv0 + 8 * s, NCONV / 32); mbar_init(empty0 + 8 * s, 1); }
@@ -225,6 +229,12 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
     mbar_wait(done_bar, 0);
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     float* tilep = reinterpret_cast<float*>(smem);
+    float* drow = nullptr;   // direct mode: this thread's (tile row = TMEM lane) output row
+    if (direct && tid < p.rows) {
+      const int q = tid % p.QB, t = tid / p.QB, pp = t % p.PB, nn = t / p.PB;
+      const int qa = q0 + q, pa = p0 + pp, na = n0 + nn;
+      if (qa < p.Q && pa < p.P && na < p.NI) drow = p.y + ((long long)(na * p.P + pa) * p.Q + qa) * p.ldy;
+    }
 #pragma unroll 1
     for (int c0 = 0; c0 < BN; c0 += 32) {
       uint32_t ev[32], ov[32], cv[32];
@@ -236,6 +246,23 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
       if (nsl <= 1) {
 #pragma unroll
         for (int j = 0; j < 32; j++) ov[j] = 0u;   // +0.0f: the odd chain is empty
+      }
+      if (direct) {   // no split: this thread's output row straight from registers (+ bias)
+        if (drow) {
+#pragma unroll
+          for (int j = 0; j < 32; j += 4) {
+            const int n = k0 + c0 + j;
+            float t[4];
+#pragma unroll
+            for (int i = 0; i < 4; i++)
+              t[i] = ((__uint_as_float(ev[j + i]) + __uint_as_float(ov[j + i])) + __uint_as_float(cv[j + i])) +
+                     (p.bias && n + i < p.Kout ? __ldg(p.bias + n + i) : 0.f);
+            if (dvec && n + 3 < p.Kout) *reinterpret_cast<float4*>(drow + n) = make_float4(t[0], t[1], t[2], t[3]);
+            else
+              for (int i = 0; i < 4 && n + i < p.Kout; i++) drow[n + i] = t[i];
+          }
+        }
+        continue;
       }
 #pragma unroll
       for (int j = 0; j < 32; j += 4) {
@@ -253,7 +280,7 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
   if (p.split > 1) cluster_sync();   // every partial tile of the cluster is staged
 
   // ---------------- sum the partial tiles of this CTA's row slice in rank order, store
-  if (!(p.dbg & 8)) {
+  if (!(p.dbg & 8) && !direct) {
     const int per = (p.rows + p.split - 1) / p.split;
     const int r_lo = z * per, r_hi = min(p.rows, r_lo + per);
     constexpr int QPR = BN / 4;
@@ -272,12 +299,17 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
       if (p.split == 1) {
         v = *reinterpret_cast<const float4*>(tilep + r * TS + c);
       } else {
+        // all remote loads in flight at once (one DSMEM latency, not split of them), then the
+        // fixed rank-order sum
         const uint32_t off = tbase + (uint32_t)((r * TS + c) * 4);
-        v = ld_dsmem4(off, 0);
-        for (int zz = 1; zz < p.split; zz++) {
-          const float4 w = ld_dsmem4(off, (uint32_t)zz);
-          v.x += w.x; v.y += w.y; v.z += w.z; v.w += w.w;
-        }
+        float4 w[MAX_SPLIT];
+#pragma unroll
+        for (int zz = 0; zz < MAX_SPLIT; zz++)
+          if (zz < p.split) w[zz] = ld_dsmem4(off, (uint32_t)zz);
+        v = w[0];
+#pragma unroll
+        for (int zz = 1; zz < MAX_SPLIT; zz++)
+          if (zz < p.split) { v.x += w[zz].x; v.y += w[zz].y; v.z += w[zz].z; v.w += w[zz].w; }
       }
       float* dst = p.y + ((long long)(na * p.P + pa) * p.Q + qa) * p.ldy + n;
       if (p.bias) {
@@ -369,7 +401,9 @@ inline Plan plan(const Shape& s) {
   const long long tiles_m = (long long)pl.nqb * pl.npb * pl.nnb;
   static const int force_bn = getenv("ORION_CVF_BN") ? atoi(getenv("ORION_CVF_BN")) : 0;   // tuning knobs
   static const int max_split = getenv("ORION_CVF_MAXSPLIT") ? std::max(1, std::min(MAX_SPLIT, atoi(getenv("ORION_CVF_MAXSPLIT")))) : MAX_SPLIT;
-  pl.BN = force_bn == 64 || force_bn == 128 ? force_bn : (s.K > 64 && tiles_m * cdivl(s.K, 128) >= 120) ? 128 : 64;
+  // BN = 128 whenever the layer has 128+ output channels: one N=128 MMA costs little more than an
+  // N=64 one (measured sweep over the HP ResNet-50 shapes, tools/bench_kernels.py conv)
+  pl.BN = force_bn == 64 || force_bn == 128 ? force_bn : s.K >= 128 ? 128 : 64;
   pl.tiles_n = (int)cdivl(s.K, pl.BN);
   pl.tiles = (int)(tiles_m * pl.tiles_n);
   pl.nk = (int)(s.R * s.S * cdivl(s.C, 32));
