@@ -220,13 +220,15 @@ class ClockSampler:
         self.index = index
         self.proc = None
         self.lines = []
+        self.stamps = []
 
     def __enter__(self):
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,power.draw,"
                  "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap,"
+                 "utilization.gpu,utilization.memory",
                  "--format=csv,noheader,nounits", "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.th = threading.Thread(target=self._read, daemon=True)
             self.th.start()
@@ -237,6 +239,24 @@ class ClockSampler:
     def _read(self):
         for line in self.proc.stdout:
             self.lines.append(line.strip())
+            self.stamps.append(time.time())
+
+    def util_between(self, windows):
+        """Mean nvidia-smi utilization.gpu / .memory (% of time a kernel / a memory access was active,
+        200 ms samples) over the samples taken inside the given (t0, t1) wall-clock windows."""
+        g, m = [], []
+        for t, l in zip(self.stamps, self.lines):
+            if not any(a <= t <= b for a, b in windows):
+                continue
+            f = [x.strip() for x in l.split(",")]
+            try:
+                g.append(float(f[7]))
+                m.append(float(f[8]))
+            except (IndexError, ValueError):
+                continue
+        if not g:
+            return {"unavailable": "no nvidia-smi utilization samples in the window"}
+        return {"gpu_busy_pct": float(np.mean(g)), "mem_busy_pct": float(np.mean(m)), "samples": len(g)}
 
     def __exit__(self, *a):
         if self.proc:
@@ -484,8 +504,9 @@ def infer_train(args, rank, world, local, metric):
     be_iters, be_time_s, win_ms, trace_ms, stats = 0, 0.0, 0.0, [], None
     be_iters_all = 0
     beg.params.reset()
-    gpm, gpm_col = GpmWindow(local), []
-    with ClockSampler(local) as clk:
+    gpm, gpm_col, col_windows = GpmWindow(local), [], []
+    clk = ClockSampler(local)
+    with clk:
         for name, lam in rates:
             for rep in range(REPEATS):
                 arr = si.poisson_arrivals_ns(lam, per_rep, seed=si.ARRIVAL_SEED + 17 * rep, gpu_index=rank)
@@ -495,6 +516,7 @@ def infer_train(args, rank, world, local, metric):
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 if name == "table3":
                     gpm.start()
+                    w0 = time.time()
                 e0.record()
                 rc = session(hp=hp, be=be_all, arrivals_ns=arr, hp_latency_ns=hp_lat_ns, dur_threshold_ppm=args.dur_ppm,
                              be_partition_sms=args.be_partition, trace_kernel_id=top_kid if name == "table3" else None)
@@ -502,6 +524,7 @@ def infer_train(args, rank, world, local, metric):
                 torch.cuda.synchronize()
                 if name == "table3":
                     gpm_col.append(gpm.stop())
+                    col_windows.append((w0, time.time()))
                 barrier()
                 ld, lc = rd["t_done"] - rd["t_arrival"], rc["t_done"] - rc["t_arrival"]
                 runs[name]["ded"] += ld.tolist()
@@ -535,9 +558,13 @@ def infer_train(args, rank, world, local, metric):
     session(be=be, be_iters=3)
     per_it = (time.time() - t0) / 3
     n_it = int(max(5, min(300, 6.0 / max(per_it, 1e-6))))
+    usamp = ClockSampler(local).__enter__()
     gpm.start()
+    wb0 = time.time()
     rb = session(be=be_all, be_iters=n_it)
+    wb1 = time.time()
     gpm_be = gpm.stop()
+    usamp.__exit__(None, None, None)
     be_ded = 0.0
     for tb in rb.get("be_t_end_all", [rb["be_t_end"]]):
         be_ded += (len(tb) - 1) / ((tb[-1] - tb[0]) / 1e9) if len(tb) > 1 else float("nan")
@@ -553,10 +580,12 @@ def infer_train(args, rank, world, local, metric):
                        "hbm_frac": (n_done * hp_b + be_iters * be_b) / be_time_s / hbm_peak,
                        "flop_frac": (n_done * hp_f + be_iters * be_f) / be_time_s / tc_peak},
         "be_alone": {"hbm_gbs": be_ded * be_b / 1e9, "hbm_frac": be_ded * be_b / hbm_peak, "flop_frac": be_ded * be_f / tc_peak},
-        "sampled": {"collocated": gpm_mean(gpm_col), "be_alone": gpm_be,
-                    "basis": "NVML GPM counters (driver-sampled SM activity / occupancy / tensor / DRAM utilisation) "
-                             "over each timed collocated run at the Table-3 rate (mean over repeats) and over the "
-                             "dedicated BE run"},
+        "sampled": {"collocated": dict(clk.util_between(col_windows), gpm=gpm_mean(gpm_col)),
+                    "be_alone": dict(usamp.util_between([(wb0, wb1)]), gpm=gpm_be),
+                    "basis": "nvidia-smi utilization.gpu / .memory sampled every 200 ms (fraction of time a kernel / "
+                             "a memory access was active) inside each timed collocated run at the Table-3 rate and "
+                             "inside the dedicated BE run; plus NVML GPM SM activity / occupancy / tensor / DRAM "
+                             "counters where the driver exposes them"},
         "be_bytes_per_iteration_GB": be_b / 1e9, "hp_bytes_per_request_GB": hp_b / 1e9,
         "basis": "algorithmic bytes/FLOPs per op of this implementation's op list (profiler.op_work) x completed "
                  "requests / iterations; SURVEY §8(d)'s own per-iteration figures (35.7 GB MobileNetV2 b96, 1.16 GB "

@@ -47,6 +47,7 @@ struct Cfg {
   static constexpr int TMEM_COLS = 3 * BN <= 256 ? 256 : 512;
   // kind::tf32: D fp32 (bit 4), A, B tf32 (bits 7, 10), both K-major, N>>3 at 17, M>>4 at 24
   static constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+  static constexpr uint32_t IDESC_BT = IDESC | (1u << 16);   // B MN-major (transposed)
   static_assert(BM * TS * 4 <= STAGES * STAGE, "staging tile fits in the stage ring");
 };
 
@@ -66,6 +67,12 @@ struct Params {
 // UMMA descriptor, K-major SWIZZLE_128B: 8-row atoms of 128-byte rows, SBO = 1024 B, layout type 2
 __device__ __forceinline__ uint64_t sdesc128(uint32_t addr) {
   return (uint64_t)((addr >> 4) & 0x3FFF) | (1ull << 16) | ((uint64_t)(1024 >> 4) << 32) | (1ull << 46) | (2ull << 61);
+}
+// UMMA descriptor, MN-major tf32 (B given [K][N]): SWIZZLE_128B with 32-byte atoms (layout type 1,
+// TMA CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B), 4-row k-groups 512 B apart, 32-column MN atoms one
+// 32 x 32 box (4 KB) apart; k-step j = rows 8j..8j+7 = start + 1024 j
+__device__ __forceinline__ uint64_t sdesc_mn(uint32_t addr) {
+  return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)(4096 >> 4) << 16) | ((uint64_t)(512 >> 4) << 32) | (1ull << 46) | (1ull << 61);
 }
 __device__ __forceinline__ void mma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
   asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
@@ -110,7 +117,7 @@ __device__ __forceinline__ float4 ld_dsmem4(uint32_t local, uint32_t rank) {
   return v;
 }
 
-template <int BN>
+template <int BN, bool BMN>
 __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                                                      Params p, OrionSig sig) {
   using C_ = Cfg<BN>;
@@ -160,7 +167,10 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
         const int slab = s0 + it, tap = slab / p.CB, cb = slab - tap * p.CB;
         const int r = tap / p.S, sx = tap - r * p.S;
         tma_load4d(st, &tmA, cb * 32, q0 * p.stride + sx - p.pad, p0 * p.stride + r - p.pad, n0, bar);
-        if (p.taps == 1) tma_load2d(st + 2 * A_BYTES, &tmB, cb * 32, k0, bar);
+        if (BMN) {   // B [K][N]: BN / 32 MN-major boxes of 32 k-rows
+#pragma unroll
+          for (int j = 0; j < BN / 32; j++) tma_load2d(st + 2 * A_BYTES + 4096 * j, &tmB, k0 + 32 * j, cb * 32, bar);
+        } else if (p.taps == 1) tma_load2d(st + 2 * A_BYTES, &tmB, cb * 32, k0, bar);
         else tma_load3d(st + 2 * A_BYTES, &tmB, cb * 32, tap, k0, bar);
       }
     }
@@ -216,10 +226,12 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
 #pragma unroll
       for (int j = 0; j < ((p.dbg & 2) ? 0 : BK / 8); j++) {
         const uint64_t dah = sdesc128(a_hi + 32 * j), dal = sdesc128(a_lo + 32 * j);
-        const uint64_t dbh = sdesc128(b_hi + 32 * j), dbl = sdesc128(b_lo + 32 * j);
-        mma_tf32(d_corr, dal, dbh, C_::IDESC, (it | j) != 0);
-        mma_tf32(d_corr, dah, dbl, C_::IDESC, 1);
-        mma_tf32(d_main, dah, dbh, C_::IDESC, ((it >> 1) | j) != 0);
+        const uint64_t dbh = BMN ? sdesc_mn(b_hi + 1024 * j) : sdesc128(b_hi + 32 * j);
+        const uint64_t dbl = BMN ? sdesc_mn(b_lo + 1024 * j) : sdesc128(b_lo + 32 * j);
+        constexpr uint32_t ID = BMN ? C_::IDESC_BT : C_::IDESC;
+        mma_tf32(d_corr, dal, dbh, ID, (it | j) != 0);
+        mma_tf32(d_corr, dah, dbl, ID, 1);
+        mma_tf32(d_main, dah, dbh, ID, ((it >> 1) | j) != 0);
       }
       mma_commit(empty0 + 8 * s);
     }
@@ -340,6 +352,7 @@ struct Shape {   // one forward convolution (or B^T GEMM as a 1x1 convolution ov
   long long NI, H, W, C, K, R, S, stride, pad, P, Q;
   long long ldx, ldw, ldy;   // GEMM strides (conv: C, R*S*C, K)
   bool gemm;
+  bool bmn;                  // GEMM with B given [K][N] (flags = 0), not [N][K]
 };
 struct Plan { int BN, QB, PB, NB, nqb, npb, nnb, tiles, tiles_n, nk, kps, split; };
 
@@ -353,11 +366,11 @@ inline bool shape_ok(const Shape& s) {
   return encoder() != nullptr;
 }
 
-template <int BN>
+template <int BN, bool BMN = false>
 bool prepare() {
   static std::atomic<int> done{0};
   if (done.load(std::memory_order_acquire)) return true;
-  const bool okk = cudaFuncSetAttribute((const void*)cvf_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<BN>::SMEM) == cudaSuccess;
+  const bool okk = cudaFuncSetAttribute((const void*)cvf_kernel<BN, BMN>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<BN>::SMEM) == cudaSuccess;
   if (okk) done.store(1, std::memory_order_release);
   return okk;
 }
@@ -377,8 +390,8 @@ inline int max_clusters(int BN, int split) {
   at[0].id = cudaLaunchAttributeClusterDimension;
   at[0].val.clusterDim.x = 1; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = (unsigned)split;
   cfg.attrs = at; cfg.numAttrs = 1;
-  const bool ok = BN == 128 ? prepare<128>() && cudaOccupancyMaxActiveClusters(&n, cvf_kernel<128>, &cfg) == cudaSuccess
-                            : prepare<64>() && cudaOccupancyMaxActiveClusters(&n, cvf_kernel<64>, &cfg) == cudaSuccess;
+  const bool ok = BN == 128 ? prepare<128>() && cudaOccupancyMaxActiveClusters(&n, cvf_kernel<128, false>, &cfg) == cudaSuccess
+                            : prepare<64>() && cudaOccupancyMaxActiveClusters(&n, cvf_kernel<64, false>, &cfg) == cudaSuccess;
   if (!ok || n <= 0) { (void)cudaGetLastError(); n = 148 / split; }
   cache[b][split].store(n, std::memory_order_relaxed);
   return n;
@@ -420,20 +433,25 @@ inline Plan plan(const Shape& s) {
 inline bool geom(const Shape& s, LaunchGeom* g) {
   if (!shape_ok(s)) return false;
   const Plan pl = plan(s);
-  if (pl.BN == 128 ? !prepare<128>() : !prepare<64>()) return false;
+  const bool okp = s.bmn ? (pl.BN == 128 ? prepare<128, true>() : prepare<64, true>()) : (pl.BN == 128 ? prepare<128>() : prepare<64>());
+  if (!okp) return false;
   g->grid = dim3((unsigned)pl.tiles, 1, (unsigned)pl.split);
   g->block = dim3(NTHR);
   g->smem = pl.BN == 128 ? Cfg<128>::SMEM : Cfg<64>::SMEM;
-  g->func = pl.BN == 128 ? (const void*)cvf_kernel<128> : (const void*)cvf_kernel<64>;
+  g->func = s.bmn ? (pl.BN == 128 ? (const void*)cvf_kernel<128, true> : (const void*)cvf_kernel<64, true>)
+                  : (pl.BN == 128 ? (const void*)cvf_kernel<128, false> : (const void*)cvf_kernel<64, false>);
   g->pipe = ORION_PIPE_TF32X3;
   return true;
 }
 
-inline bool is(const void* f) { return f == (const void*)cvf_kernel<128> || f == (const void*)cvf_kernel<64>; }
+inline bool is(const void* f) {
+  return f == (const void*)cvf_kernel<128, false> || f == (const void*)cvf_kernel<64, false> || f == (const void*)cvf_kernel<128, true> ||
+         f == (const void*)cvf_kernel<64, true>;
+}
 
-template <int BN>
+template <int BN, bool BMN>
 int launch_t(const Shape& s, const Plan& pl, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
-  if (!prepare<BN>()) return ORION_E_CUDA;
+  if (!prepare<BN, BMN>()) return ORION_E_CUDA;
   CUtensorMap ma, mb;
   // activations: {C, W, H, N} (GEMM: {K, M, 1, 1}); box {32, QB*stride, PB*stride, NB}, traversal strides
   // (stride, stride): TMA gathers QB x PB x NB positions of one tap (ceil(box / stride) per dim)
@@ -449,7 +467,9 @@ int launch_t(const Shape& s, const Plan& pl, const LaunchGeom& g, OrionSig sig, 
           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return ORION_E_CUDA;
   }
-  if (s.R * s.S == 1) {
+  if (BMN) {   // B [C (reduction)][K (outputs)] row-major: 32 x 32 MN-major boxes
+    if (!map2d_f32_sw(&mb, s.w, s.C, s.K, s.ldw, 32, 32, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B)) return ORION_E_CUDA;
+  } else if (s.R * s.S == 1) {
     if (!map2d_f32_sw(&mb, s.w, s.K, s.C, s.ldw, 32, BN, CU_TENSOR_MAP_SWIZZLE_128B)) return ORION_E_CUDA;
   } else {
     encode_fn e = encoder();
@@ -470,7 +490,7 @@ int launch_t(const Shape& s, const Plan& pl, const LaunchGeom& g, OrionSig sig, 
   static const int dbg = getenv("ORION_CVF_DEBUG") ? atoi(getenv("ORION_CVF_DEBUG")) : 0;
   p.dbg = dbg;
   if (pl.split == 1) {
-    cvf_kernel<BN><<<g.grid, g.block, g.smem, st>>>(ma, mb, p, sig);
+    cvf_kernel<BN, BMN><<<g.grid, g.block, g.smem, st>>>(ma, mb, p, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
   cudaLaunchConfig_t cfg = {};
@@ -479,12 +499,13 @@ int launch_t(const Shape& s, const Plan& pl, const LaunchGeom& g, OrionSig sig, 
   at[0].id = cudaLaunchAttributeClusterDimension;
   at[0].val.clusterDim.x = 1; at[0].val.clusterDim.y = 1; at[0].val.clusterDim.z = (unsigned)pl.split;
   cfg.attrs = at; cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, cvf_kernel<BN>, ma, mb, p, sig) == cudaSuccess ? 0 : ORION_E_CUDA;
+  return cudaLaunchKernelEx(&cfg, cvf_kernel<BN, BMN>, ma, mb, p, sig) == cudaSuccess ? 0 : ORION_E_CUDA;
 }
 
 inline int launch(const Shape& s, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   const Plan pl = plan(s);
-  return pl.BN == 128 ? launch_t<128>(s, pl, g, sig, st) : launch_t<64>(s, pl, g, sig, st);
+  if (s.bmn) return pl.BN == 128 ? launch_t<128, true>(s, pl, g, sig, st) : launch_t<64, true>(s, pl, g, sig, st);
+  return pl.BN == 128 ? launch_t<128, false>(s, pl, g, sig, st) : launch_t<64, false>(s, pl, g, sig, st);
 }
 
 // conv_fwd args: x, w, y, N, H, W, C, K, R, S, stride, pad, P, Q, workspace, ws_bytes
@@ -494,19 +515,19 @@ inline Shape conv_shape(const uint64_t* a) {
   s.NI = (long long)a[3]; s.H = (long long)a[4]; s.W = (long long)a[5]; s.C = (long long)a[6]; s.K = (long long)a[7];
   s.R = (long long)a[8]; s.S = (long long)a[9]; s.stride = (long long)a[10]; s.pad = (long long)a[11];
   s.P = (long long)a[12]; s.Q = (long long)a[13];
-  s.ldx = s.C; s.ldw = s.R * s.S * s.C; s.ldy = s.K; s.gemm = false;
+  s.ldx = s.C; s.ldw = s.R * s.S * s.C; s.ldy = s.K; s.gemm = false; s.bmn = false;
   if (s.R == 1 && s.S == 1 && s.stride == 1 && s.pad == 0) {   // pointwise: one GEMM over all positions
     s.gemm = true; s.Q = s.NI * s.P * s.Q; s.P = 1; s.NI = 1; s.H = 1; s.W = s.Q;
   }
   return s;
 }
-// gemm args (flags = 2): A [M][lda], B^T [N][ldb], C [M][ldc], bias
+// gemm args (flags = 2: B^T [N][ldb]; flags = 0: B [K][ldb]): A [M][lda], C [M][ldc], bias
 inline Shape gemm_shape(const uint64_t* a) {
   Shape s;
   s.x = (const float*)a[0]; s.w = (const float*)a[1]; s.y = (float*)a[2]; s.bias = (const float*)a[3];
   s.Q = (long long)a[4]; s.K = (long long)a[5]; s.C = (long long)a[6];
   s.NI = 1; s.P = 1; s.H = 1; s.W = s.Q; s.R = 1; s.S = 1; s.stride = 1; s.pad = 0;
-  s.ldx = (long long)a[7]; s.ldw = (long long)a[8]; s.ldy = (long long)a[9]; s.gemm = true;
+  s.ldx = (long long)a[7]; s.ldw = (long long)a[8]; s.ldy = (long long)a[9]; s.gemm = true; s.bmn = (int)a[10] == 0;
   return s;
 }
 
@@ -519,7 +540,7 @@ bool cvf_conv_try_geom(const uint64_t* a, LaunchGeom* g) {
 }
 bool cvf_gemm_try_geom(const uint64_t* a, LaunchGeom* g) {
   static const bool off = getenv("ORION_CVF_OFF") != nullptr;
-  if (off || (int)a[10] != 2) return false;
+  if (off || ((int)a[10] != 2 && (int)a[10] != 0)) return false;
   return cvf::geom(cvf::gemm_shape(a), g);
 }
 bool cvf_is(const void* f) { return cvf::is(f); }

@@ -2248,7 +2248,7 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     g->grid = dim3((unsigned)cdiv(M, rows::rpc((int)N))); g->block = dim3(rows::NTH); g->smem = rows::smem_bytes((int)K, (int)N); g->func = f;
     return 0;
   }
-  if (flags == 2 && cvf_gemm_try_geom(a, g)) return 0;   // dense B^T GEMM, TMA-fed tcgen05 (cvf.cu)
+  if ((flags == 2 || flags == 0) && cvf_gemm_try_geom(a, g)) return 0;   // dense GEMM, TMA-fed tcgen05 (cvf.cu)
   if (flags == 1 && atc_try_geom(a, g)) return 0;   // compute-dense A^T B on tcgen05 (atc.cu)
   if (flags == 1 && wgs_try_geom(a, g)) return 0;   // TMA-fed streaming A^T B (wgs.cu)
   if (flags == 1 && atb_ok(M, N, K)) {

@@ -104,3 +104,33 @@ def test_gemm_bt_tensor_path(M, N, K, bias):
     first = C.clone()
     _launch("gemm", args)
     assert torch.equal(first, C)
+
+
+GEMM_NN = [  # M, N, K: C = A B with B given [K][N] (flags = 0): 1x1-conv / Linear data gradients
+    (4704, 160, 960),    # MobileNetV2 b96 features.16 expand data gradient (7x7 maps)
+    (4704, 960, 320),    # features.18 data gradient
+    (784, 1024, 512),
+    (1000, 100, 36),     # ragged K / N
+    (129, 200, 64),
+]
+
+
+@pytest.mark.parametrize("M,N,K", GEMM_NN, ids=lambda v: str(v))
+def test_gemm_nn_tensor_path(M, N, K):
+    """MN-major B straight from TMA (128-byte swizzle with 32-byte atoms) into the transposed-B MMA."""
+    A = si.normal((M, K), 71)
+    B = si.normal((K, N), 72) * 0.1
+    C = torch.full((M, N), float("nan"), device="cuda")
+    Ad, Bd = A.cuda(), B.cuda()
+    nws = L.lib.orion_gemm_workspace_bytes(M, N, K)
+    w = torch.zeros(int(nws) // 4 + 64, device="cuda")
+    args = [Ad.data_ptr(), Bd.data_ptr(), C.data_ptr(), 0, M, N, K, K, N, N, 0, w.data_ptr(), w.numel() * 4]
+    kern = kernel_info("gemm", args)["kernel"]
+    _launch("gemm", args)
+    ref = om.linear_fwd(A, B.t().contiguous(), None)
+    absref = om.linear_fwd(A.abs(), B.abs().t().contiguous(), None)
+    _check(C, ref, absref, K)
+    assert "cvf_kernel" in kern or "tmk" in kern, kern   # streaming shapes (>= 296 tiles) keep the multi-tile kernel
+    first = C.clone()
+    _launch("gemm", args)
+    assert torch.equal(first, C)
