@@ -116,6 +116,26 @@ __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CU
 
   if (warp == 0) {
     if (lane == 0) {
+      // CONV: the tile's box columns are fixed for the whole CTA -- decode each one's (channel, tap
+      // offset) once; the position block advances by counters. (Per-stage integer divisions on this
+      // single issuing thread made it the bottleneck: 1.4 us per stage, ncu.)
+      int ca[BM / 32], qa[BM / 32], pa[BM / 32], cb_[BN / 32], qb_[BN / 32], pb_[BN / 32];
+      int qb = 0, pb = 0, nimg = 0;
+      if (CONV) {
+        auto decode = [&](bool is_x, int col, int& c, int& dq, int& dp) {
+          if (!is_x) { c = col; dq = 0; dp = 0; return; }
+          const int tap = col / p.cv_C, r = tap / p.cv_S, sx = tap - r * p.cv_S;
+          c = col - tap * p.cv_C; dq = sx - p.pad; dp = r - p.pad;
+        };
+#pragma unroll
+        for (int j = 0; j < BM / 32; j++) decode(p.trans != 0, m0 + 32 * j, ca[j], qa[j], pa[j]);
+#pragma unroll
+        for (int j = 0; j < BN / 32; j++) decode(p.trans == 0, n0 + 32 * j, cb_[j], qb_[j], pb_[j]);
+        const int b0 = k0 / BK;
+        qb = b0 % p.nqb;
+        const int t2 = b0 / p.nqb;
+        pb = t2 % p.npb; nimg = t2 / p.npb;
+      }
 #pragma unroll 1
       for (int it = 0; it < nst; it++) {
         const int s = it % S;
@@ -129,22 +149,18 @@ __global__ void __launch_bounds__(NTHR, 1) atc_kernel(const __grid_constant__ CU
 #pragma unroll
           for (int j = 0; j < BN / 32; j++) tma_load2d(st + 2 * A_BYTES + j * BOX_BYTES, &tmB, n0 + 32 * j, kk, bar);
         } else {
-          // stage = position block b: image n, output rows p0.., columns q0..
-          const int b = kk / BK, qb = b % p.nqb, t2 = b / p.nqb, pb = t2 % p.npb, n = t2 / p.npb;
+          // stage = position block (image nimg, output rows p0.., columns q0..); dy boxes take the
+          // block itself, x boxes the block shifted by the tap (zero fill = padding)
           const int p0 = pb * p.PB, q0 = qb * p.QB;
-          // dy side: column = output channel; x side: column = (tap, input channel)
-          auto box = [&](bool is_x, const CUtensorMap* tm, uint32_t dst, int col) {
-            if (!is_x) {
-              tma_load4d(dst, tm, col, q0, p0, n, bar);
-            } else {
-              const int tap = col / p.cv_C, c = col - tap * p.cv_C, r = tap / p.cv_S, sx = tap - r * p.cv_S;
-              tma_load4d(dst, tm, c, q0 * p.stride + sx - p.pad, p0 * p.stride + r - p.pad, n, bar);
-            }
-          };
+          const int qs = q0 * p.stride, ps = p0 * p.stride;
+          const bool ax = p.trans != 0;
 #pragma unroll
-          for (int j = 0; j < BM / 32; j++) box(p.trans != 0, &tmA, st + j * BOX_BYTES, m0 + 32 * j);
+          for (int j = 0; j < BM / 32; j++)
+            tma_load4d(st + j * BOX_BYTES, &tmA, ca[j], ax ? qs + qa[j] : q0, ax ? ps + pa[j] : p0, nimg, bar);
 #pragma unroll
-          for (int j = 0; j < BN / 32; j++) box(p.trans == 0, &tmB, st + 2 * A_BYTES + j * BOX_BYTES, n0 + 32 * j);
+          for (int j = 0; j < BN / 32; j++)
+            tma_load4d(st + 2 * A_BYTES + j * BOX_BYTES, &tmB, cb_[j], ax ? q0 : qs + qb_[j], ax ? p0 : ps + pb_[j], nimg, bar);
+          if (++qb == p.nqb) { qb = 0; if (++pb == p.npb) { pb = 0; ++nimg; } }
         }
       }
     }

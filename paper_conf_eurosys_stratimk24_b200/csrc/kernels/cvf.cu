@@ -157,21 +157,21 @@ __global__ void __launch_bounds__(NTHR, 1) cvf_kernel(const __grid_constant__ CU
 
   if (warp == TMA_WARP) {
     if (lane == 0) {
+      int tap = s0 / p.CB, cb = s0 - tap * p.CB, r = tap / p.S, sx = tap - r * p.S;   // slab s0
 #pragma unroll 1
       for (int it = 0; it < nsl; it++) {
         const int s = it % S;
         if (it >= S) mbar_wait(empty0 + 8 * s, ((uint32_t)(it / S) & 1u) ^ 1u);
         const uint32_t st = smem_u32(smem + s * STAGE), bar = full0 + 8 * s;
-        if (p.dbg & 4) { mbar_arrive(bar); continue; }
+        if (p.dbg & 4) { mbar_arrive(bar); continue; }   // (counters unused in this measurement mode)
         mbar_expect(bar, tx);
-        const int slab = s0 + it, tap = slab / p.CB, cb = slab - tap * p.CB;
-        const int r = tap / p.S, sx = tap - r * p.S;
         tma_load4d(st, &tmA, cb * 32, q0 * p.stride + sx - p.pad, p0 * p.stride + r - p.pad, n0, bar);
         if (BMN) {   // B [K][N]: BN / 32 MN-major boxes of 32 k-rows
 #pragma unroll
           for (int j = 0; j < BN / 32; j++) tma_load2d(st + 2 * A_BYTES + 4096 * j, &tmB, k0 + 32 * j, cb * 32, bar);
         } else if (p.taps == 1) tma_load2d(st + 2 * A_BYTES, &tmB, cb * 32, k0, bar);
         else tma_load3d(st + 2 * A_BYTES, &tmB, cb * 32, tap, k0, bar);
+        if (++cb == p.CB) { cb = 0; ++tap; if (++sx == p.S) { sx = 0; ++r; } }   // next slab, no divisions
       }
     }
   } else if (warp >= 4 && warp < TMA_WARP) {

@@ -93,6 +93,27 @@ def floor():
     t = timeit("relu", [x.data_ptr(), x.data_ptr(), x.numel()])
     print(f"relu 4x56x56x64 {t:6.2f} us")
 
+
+BE_CWG = [(64, 56, 56, 64, 64, 3, 1, 1), (64, 56, 56, 128, 128, 3, 2, 1), (64, 28, 28, 128, 128, 3, 1, 1), (64, 14, 14, 256, 256, 3, 1, 1),
+          (64, 7, 7, 512, 512, 3, 1, 1), (64, 56, 56, 256, 512, 1, 2, 0), (64, 28, 28, 512, 1024, 1, 2, 0)]
+
+
+def cwg():
+    """BE ResNet-50 b64 convolution weight gradients (config 3's dominant BE kernels)."""
+    tot = 0.0
+    for n, h, w_, c, k, r, st, pad in BE_CWG:
+        p, q = (h + 2 * pad - r) // st + 1, (w_ + 2 * pad - r) // st + 1
+        x, dy, dw = torch.randn(n, h, w_, c, device="cuda"), torch.randn(n, p, q, k, device="cuda"), torch.zeros(k, r, r, c, device="cuda")
+        wf = ws(L.lib.orion_conv_wgrad_workspace_bytes(n, h, w_, c, k, r, r, st, pad))
+        a = [x.data_ptr(), dy.data_ptr(), dw.data_ptr(), n, h, w_, c, k, r, r, st, pad, p, q, wf.data_ptr(), wf.numel() * 4]
+        t = timeit("conv_wgrad", a)
+        tot += t
+        info = kernel_info("conv_wgrad", a)
+        fl = 2 * n * p * q * k * r * r * c
+        print(f"wgrad {n}x{h}x{w_}x{c}->{k} r{r} s{st} {t:8.1f} us {fl / t / 1e6:6.1f} TF ({fl / t / 1e6 / 228:4.2f} of 3xTF32) "
+              f"grid {info['grid_ctas']} {info['kernel'][:40]}")
+    print(f"conv wgrad total {tot:.1f} us")
+
 def wgs():
     tot = 0.0
     for M, N, K in WGS:
@@ -137,3 +158,5 @@ if __name__ == "__main__":
         conv()
     if what in ("floor", "all"):
         floor()
+    if what in ("cwg", "all"):
+        cwg()
