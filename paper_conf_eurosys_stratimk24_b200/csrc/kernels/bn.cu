@@ -3,6 +3,8 @@
 // canonical memory-bound kernel. Reductions accumulate in fp64 per thread, combine
 // row-lanes in a fixed order in shared memory, write per-split partials and let the last CTA of
 // each channel block sum the splits in split order: deterministic, partition-independent.
+#include <cstdlib>
+
 #include "common.cuh"
 
 namespace {
@@ -23,8 +25,12 @@ BnSplit bn_split(long long rows, int C) {
   s.cg4 = q < 64 ? q : 64;
   s.rl = BN_THREADS / s.cg4;
   s.cblocks = (int)cdiv(q, s.cg4);
-  long long rs = cdiv(148 * 4, s.cblocks);      // shape-only: ~4 CTAs per SM of a 148-SM part
-  long long max_rs = cdiv(rows, 16LL * s.rl);   // >= 16 rows per row lane (2 trips of 8 loads)
+  // ~2 CTAs per SM: measured best over MobileNetV2's 12 BN shapes (tools/bench_kernels.py bn: 741 us
+  // vs 830 at 4 per SM, 886 at 1 per SM for the stats + backward-reduce pairs)
+  static const long long cta_target = getenv("ORION_BN_CTAS") ? atoll(getenv("ORION_BN_CTAS")) : 148 * 2;   // tuning knob
+  static const long long min_rows = getenv("ORION_BN_MINROWS") ? atoll(getenv("ORION_BN_MINROWS")) : 16;
+  long long rs = cdiv(cta_target, s.cblocks);   // shape-only (a 148-SM constant, not the partition)
+  long long max_rs = cdiv(rows, min_rows * s.rl);   // >= 16 rows per row lane (2 trips of 8 loads)
   if (rs > max_rs) rs = max_rs;
   if (rs < 1) rs = 1;
   if (rs > 1024) rs = 1024;

@@ -114,6 +114,30 @@ def cwg():
               f"grid {info['grid_ctas']} {info['kernel'][:40]}")
     print(f"conv wgrad total {tot:.1f} us")
 
+
+BN_SHAPES = [(96 * 112 * 112, 32), (96 * 112 * 112, 96), (96 * 56 * 56, 144), (96 * 56 * 56, 24), (96 * 28 * 28, 192), (96 * 28 * 28, 32),
+             (96 * 14 * 14, 384), (96 * 14 * 14, 64), (96 * 14 * 14, 576), (96 * 7 * 7, 960), (96 * 7 * 7, 160), (96 * 7 * 7, 1280)]
+
+
+def bn():
+    """MobileNetV2 b96 BN statistics / backward reduction shapes (rows, C)."""
+    tot = 0.0
+    for rows, c in BN_SHAPES:
+        x, dy = torch.randn(rows, c, device="cuda"), torch.randn(rows, c, device="cuda")
+        mean, inv, rm, rv = (torch.zeros(c, device="cuda") for _ in range(4))
+        dg, db = torch.zeros(c, device="cuda"), torch.zeros(c, device="cuda")
+        w = ws(L.lib.orion_bn_workspace_bytes(rows, c) if hasattr(L.lib, "orion_bn_workspace_bytes") else 64 << 20)
+        eps = __import__("struct").unpack("<I", __import__("struct").pack("<f", 1e-5))[0]
+        mom = __import__("struct").unpack("<I", __import__("struct").pack("<f", 0.1))[0]
+        a1 = [x.data_ptr(), mean.data_ptr(), inv.data_ptr(), rm.data_ptr(), rv.data_ptr(), rows, c, eps, mom, w.data_ptr(), w.numel() * 4]
+        a2 = [x.data_ptr(), dy.data_ptr(), mean.data_ptr(), inv.data_ptr(), dg.data_ptr(), db.data_ptr(), rows, c, w.data_ptr(), w.numel() * 4]
+        t1, t2 = timeit("bn_stats", a1), timeit("bn_bwd_reduce", a2)
+        tot += t1 + t2
+        g1 = kernel_info("bn_stats", a1)["grid_ctas"]
+        print(f"bn rows={rows:8d} C={c:5d} stats {t1:6.1f} us {4 * rows * c / t1 / 1e3:5.0f} GB/s (grid {g1})  "
+              f"bwd_reduce {t2:6.1f} us {8 * rows * c / t2 / 1e3:5.0f} GB/s")
+    print(f"bn total {tot:.1f} us")
+
 def wgs():
     tot = 0.0
     for M, N, K in WGS:
@@ -160,3 +184,5 @@ if __name__ == "__main__":
         floor()
     if what in ("cwg", "all"):
         cwg()
+    if what in ("bn", "all"):
+        bn()
