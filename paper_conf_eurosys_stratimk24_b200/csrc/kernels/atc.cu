@@ -28,12 +28,16 @@ constexpr int BM = 128, BK = 16, NTHR = 192;   // warps: 0 TMA, 1 MMA + TMEM own
 constexpr int CONV_THREADS = 128;
 constexpr int BOX_BYTES = 32 * BK * 4;   // one TMA box: 32 elements (128 B) x BK rows = one MN atom column
 
+#ifndef ATC_MAX_STAGES
+#define ATC_MAX_STAGES 8
+#endif
+constexpr int MAX_STAGES = ATC_MAX_STAGES;   // ring depth cap (small-N tiles: more 16-row stages in flight)
 template <int BN_>
 struct Cfg {
   static constexpr int BN = BN_;
   static constexpr int A_BYTES = BM * BK * 4, B_BYTES = BN * BK * 4;
   static constexpr int STAGE = 2 * (A_BYTES + B_BYTES);   // [A raw][A lo][B raw][B lo]
-  static constexpr int STAGES = (200 * 1024) / STAGE > 8 ? 8 : (200 * 1024) / STAGE;
+  static constexpr int STAGES = (200 * 1024) / STAGE > MAX_STAGES ? MAX_STAGES : (200 * 1024) / STAGE;
   static constexpr int SMEM = STAGES * STAGE + 1024 + 256;
   static constexpr int TMEM_COLS = 2 * BN < 32 ? 32 : 2 * BN;
   // kind::tf32: D fp32 (bit 4), A, B tf32 (bits 7, 10), A and B MN-major (bits 15, 16), N>>3, M>>4
