@@ -72,3 +72,38 @@ def test_occupancy_granularities():
     assert PR.occupancy_limits(256, 119, 98 * 1024)["registers"] == 2
     # a kernel that needs more SMs than the GPU has is never admitted beside the HP (L27, R5)
     assert PR.sm_needed_closed_form(296, 256, 119, 97 * 1024) == 148
+
+
+def _ncu_tables():
+    import csv
+    import glob
+    import os
+    root = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles")
+    for path in sorted(glob.glob(os.path.join(root, "*_ncu.csv"))):
+        rows = list(csv.DictReader(open(path)))
+        if rows and "occ_regs" in rows[0] and rows[0]["occ_regs"] not in ("", None):
+            yield os.path.basename(path), rows
+
+
+def test_occupancy_closed_form_matches_ncu():
+    """R17 pinned to the hardware: for every launch of the committed per-op ncu tables (one solo
+    launch per op on a B200, tools/ncu_times.sh with NCU_PROFILE=1), the closed-form limits from
+    the launch's block size, registers per thread and shared memory equal ncu's
+    launch__occupancy_limit_{warps,registers,blocks[,shared_mem]} -- the quantities P:863-868 names."""
+    n = 0
+    for name, rows in _ncu_tables():
+        for r in rows:
+            block, regs = int(float(r["block"])), int(float(r["regs"]))
+            smem = None
+            if r.get("smem_dyn") not in (None, "") and r.get("smem_static") not in (None, ""):
+                smem = int(float(r["smem_dyn"])) + int(float(r["smem_static"]))
+            lim = PR.occupancy_limits(block, regs, smem or 0)
+            assert lim["warps"] == int(float(r["occ_warps"])), (name, r["label"])
+            assert lim["registers"] == int(float(r["occ_regs"])), (name, r["label"], block, regs)
+            assert lim["blocks"] == int(float(r["occ_blocks"])), (name, r["label"])
+            if smem is not None:
+                assert lim["shared_mem"] == int(float(r["occ_smem"])), (name, r["label"], smem)
+            n += 1
+    if n == 0:
+        pytest.skip("no committed ncu table carries the occupancy limits")
+    assert n >= 100

@@ -31,7 +31,8 @@ EXTRA = [("tc_pct", "sm__pipe_tc_cycles_active.avg.pct_of_peak_sustained_elapsed
          ("fma_pct", "sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_elapsed"),
          ("block", "launch__block_size"), ("regs", "launch__registers_per_thread"),
          ("occ_blocks", "launch__occupancy_limit_blocks"), ("occ_regs", "launch__occupancy_limit_registers"),
-         ("occ_smem", "launch__occupancy_limit_shared_mem"), ("occ_warps", "launch__occupancy_limit_warps")]
+         ("occ_smem", "launch__occupancy_limit_shared_mem"), ("occ_warps", "launch__occupancy_limit_warps"),
+         ("smem_dyn", "launch__shared_mem_per_block_dynamic"), ("smem_static", "launch__shared_mem_per_block_static")]
 
 
 def main(ncu_log, oplist, base, out_csv):
