@@ -76,6 +76,16 @@ __host__ __device__ __forceinline__ float u2f(uint64_t v) {
 
 __host__ __device__ __forceinline__ uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
 
+// Packed fp32 FMA (sm_100a FFMA2): d.x += a * b.x, d.y += a * b.y, each lane rounded once exactly as
+// fmaf would (same results bit for bit), one issue slot for two FMAs. The scalar a is broadcast to
+// both lanes (SASS: FFMA2 Rd, Ra.F32, Rb.F32x2, Rd.F32x2).
+__device__ __forceinline__ void ffma2(float2& d, float a, float2 b) {
+  asm("{\n\t.reg .b64 a2, b2, d2;\n\tmov.b64 a2, {%2, %2};\n\tmov.b64 b2, {%3, %4};\n\tmov.b64 d2, {%0, %1};\n\t"
+      "fma.rn.f32x2 d2, a2, b2, d2;\n\tmov.b64 {%0, %1}, d2;\n\t}"
+      : "+f"(d.x), "+f"(d.y)
+      : "f"(a), "f"(b.x), "f"(b.y));
+}
+
 // Last-CTA-of-a-group detection for deterministic two-phase reductions: every CTA of the group
 // calls this after writing its partials; returns true in exactly one CTA (the last), which then
 // reduces the partials in a fixed order. The ticket is reset by the last CTA.
@@ -216,6 +226,12 @@ uint64_t atc_conv_ws_bytes(uint64_t N, uint64_t H, uint64_t W, uint64_t C, uint6
 bool atc_conv_try_geom(const uint64_t* a, LaunchGeom* g);
 bool atc_conv_is(const void* f);
 int atc_conv_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
+
+// Streaming tensor-core weight-gradient GEMM (ats.cu): long K, narrow operands, 3xTF32 on tcgen05.
+uint64_t ats_ws_bytes(long long M, long long N, long long K);
+bool ats_try_geom(const uint64_t* a, LaunchGeom* g);
+bool ats_is(const void* f);
+int ats_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s);
 
 // Forward convolution / dense B^T GEMM on tcgen05 with TMA im2col boxes (cvf.cu).
 bool cvf_conv_try_geom(const uint64_t* a, LaunchGeom* g);

@@ -2214,6 +2214,8 @@ extern "C" uint64_t orion_gemm_workspace_bytes(uint64_t M, uint64_t N, uint64_t 
   if (b3 > b) b = b3;
   const uint64_t b4 = atc_ws_bytes((long long)M, (long long)N, (long long)K);   // ... or the tensor-core one
   if (b4 > b) b = b4;
+  const uint64_t b5 = ats_ws_bytes((long long)M, (long long)N, (long long)K);   // ... or the streaming tensor-core one
+  if (b5 > b) b = b5;
   return b;
 }
 
@@ -2252,6 +2254,7 @@ int gemm_geom(const uint64_t* a, LaunchGeom* g) {
     return 0;
   }
   if ((flags == 2 || flags == 0) && cvf_gemm_try_geom(a, g)) return 0;   // dense GEMM, TMA-fed tcgen05 (cvf.cu)
+  if (flags == 1 && ats_try_geom(a, g)) return 0;   // long-K narrow A^T B streamed into tcgen05 (ats.cu)
   if (flags == 1 && atc_try_geom(a, g)) return 0;   // compute-dense A^T B on tcgen05 (atc.cu)
   if (flags == 1 && wgs_try_geom(a, g)) return 0;   // TMA-fed streaming A^T B (wgs.cu)
   if (flags == 1 && atb_ok(M, N, K)) {
@@ -2297,6 +2300,7 @@ int gemm_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
   if (atc_is(g.func)) return atc_launch(a, g, sig, s);
+  if (ats_is(g.func)) return ats_launch(a, g, sig, s);
   if (cvf_is(g.func)) return cvf_gemm_launch(a, g, sig, s);
   if (wgs_is(g.func)) return wgs_launch(a, g, sig, s);
   if (tmk::is(g.func)) return tmk::launch(g, M, N, K, C, ldc, bias, A, lda, B, ldb, flags == 0, sig, s);

@@ -170,11 +170,13 @@ __global__ void __maxnreg__(MAXREG) wgs_kernel(const __grid_constant__ CUtensorM
   }
   __syncthreads();
 
-  float acc[MI][NB];
+  // accumulator pairs (columns 2j, 2j+1 of the broadcast operand): packed FFMA2, two FMAs per issue
+  // slot (same per-lane rounding as fmaf: results bit-identical to the scalar form)
+  float2 acc[MI][NB / 2];
 #pragma unroll
   for (int i = 0; i < MI; i++)
 #pragma unroll
-    for (int j = 0; j < NB; j++) acc[i][j] = 0.f;
+    for (int j = 0; j < NB / 2; j++) acc[i][j] = make_float2(0.f, 0.f);
 
   // producer: the slot of stage `it` is refilled with stage it + S by the warp that releases it last
   // (a per-slot arrival count in shared memory), so all S slots are in flight and no warp waits for
@@ -209,10 +211,8 @@ __global__ void __maxnreg__(MAXREG) wgs_kernel(const __grid_constant__ CUtensorM
       for (int j = 0; j < NB / 4; j++)
 #pragma unroll
         for (int i = 0; i < MI; i++) {
-          acc[i][4 * j] = fmaf(lv[i], qv[j].x, acc[i][4 * j]);
-          acc[i][4 * j + 1] = fmaf(lv[i], qv[j].y, acc[i][4 * j + 1]);
-          acc[i][4 * j + 2] = fmaf(lv[i], qv[j].z, acc[i][4 * j + 2]);
-          acc[i][4 * j + 3] = fmaf(lv[i], qv[j].w, acc[i][4 * j + 3]);
+          ffma2(acc[i][2 * j], lv[i], make_float2(qv[j].x, qv[j].y));
+          ffma2(acc[i][2 * j + 1], lv[i], make_float2(qv[j].z, qv[j].w));
         }
     };
     auto ld_row = [&](int r, float (&lv)[MI], float4 (&qv)[NB / 4]) {
@@ -261,7 +261,7 @@ __global__ void __maxnreg__(MAXREG) wgs_kernel(const __grid_constant__ CUtensorM
 #pragma unroll
     for (int i = 0; i < MI; i++)
 #pragma unroll
-      for (int j = 0; j < NB; j++) red[((warp * MI + i) * NB + j) * 32 + lane] = acc[i][j];
+      for (int j = 0; j < NB; j++) red[((warp * MI + i) * NB + j) * 32 + lane] = (j & 1) ? acc[i][j / 2].y : acc[i][j / 2].x;
   }
   __syncthreads();
   auto coord = [&](int e, int& m, int& n) {   // tile element e -> output (m, n)

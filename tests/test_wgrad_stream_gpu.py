@@ -136,3 +136,20 @@ def test_conv_wgrad_tensor_path(n, h, w, c, k, r, st, pad):
     orion.kernel_launch("conv_wgrad", args, s)
     torch.cuda.synchronize()
     assert torch.equal(first, dw)
+
+
+def test_ats_tensor_streaming_path():
+    """The streaming tcgen05 weight-gradient kernel (ats.cu, 3xTF32 with <= 2048-row TMEM chains and
+    fp32 chain sums) is off by default (slower than wgs / atc on B200: tf32 MMAs with N <= 64 cost
+    ~45 cycles each); it stays held to the same numerics and determinism bar, forced on
+    in a child process (the routing knob is read once per process)."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, ORION_ATS_MIN_ROWS="1")
+    cases = ["96", "16", "1204224", "144", "24", "75264", "40", "40", "50000", "100", "36", "65536"]
+    r = subprocess.run([sys.executable, os.path.join(root, "tools", "check_wgrad.py")] + cases, env=env, cwd=root,
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout + r.stderr
+    assert r.stdout.count("ats_kernel") == 4, r.stdout

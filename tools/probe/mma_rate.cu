@@ -18,7 +18,13 @@ __device__ __forceinline__ void mma(uint32_t d, uint64_t a, uint64_t b, uint32_t
     asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\ttcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d), "l"(a), "l"(b), "r"(idesc), "r"(acc) : "memory");
 }
 
-template <int KIND, int N, int NACC>
+// MN-major tf32 operand descriptor: 128-byte swizzle with 32-byte atoms (layout type 1), LBO 4 KB
+// between MN atoms, SBO 512 B between 4-row k-groups (the weight-gradient kernels' layout)
+__device__ __forceinline__ uint64_t desc_mn(uint32_t addr) {
+  return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)(4096 >> 4) << 16) | ((uint64_t)(512 >> 4) << 32) | (1ull << 46) | (1ull << 61);
+}
+
+template <int KIND, int N, int NACC, bool MN = false>
 __global__ void __launch_bounds__(128, 1) k_mma(int iters, unsigned long long* out) {
   extern __shared__ __align__(1024) unsigned char sm[];
   __shared__ uint32_t slot;
@@ -39,9 +45,10 @@ __global__ void __launch_bounds__(128, 1) k_mma(int iters, unsigned long long* o
   const uint32_t tmem = slot;
   if (threadIdx.x == 0) {
     constexpr uint32_t ab = KIND == 0 ? 2u : 1u;
-    const uint32_t idesc = (1u << 4) | (ab << 7) | (ab << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
-    const uint32_t base = smem_u32(sm);
-    const uint64_t da = sdesc(base, 128, 256), db = sdesc(base + 32768, 128, 256);
+    const uint32_t mn = MN ? ((1u << 15) | (1u << 16)) : 0u;
+    const uint32_t idesc = (1u << 4) | (ab << 7) | (ab << 10) | mn | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+    const uint32_t base = (smem_u32(sm) + 1023u) & ~1023u;
+    const uint64_t da = MN ? desc_mn(base) : sdesc(base, 128, 256), db = MN ? desc_mn(base + 32768) : sdesc(base + 32768, 128, 256);
     long long t0 = clock64();
     for (int i = 0; i < iters; i++) {
 #pragma unroll
@@ -80,11 +87,11 @@ __global__ void k_cvt(int iters, float* out, unsigned long long* cyc) {
   if (threadIdx.x == 0) cyc[blockIdx.x] = (unsigned long long)(t1 - t0);
 }
 
-template <int KIND, int N, int NACC>
+template <int KIND, int N, int NACC, bool MN = false>
 void run(const char* name) {
   unsigned long long* d;
   cudaMalloc(&d, 148 * 8);
-  auto f = k_mma<KIND, N, NACC>;
+  auto f = k_mma<KIND, N, NACC, MN>;
   cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, 65536);
   const int iters = 2000;
   f<<<148, 128, 65536>>>(iters, d);
@@ -98,6 +105,12 @@ void run(const char* name) {
 }
 
 int main() {
+  run<0, 32, 1>("tf32 N=32  same acc");
+  run<0, 32, 4>("tf32 N=32  4 accs");
+  run<0, 32, 1, true>("tf32 MN-major N=32 same acc");
+  run<0, 32, 4, true>("tf32 MN-major N=32 4 accs");
+  run<0, 64, 4, true>("tf32 MN-major N=64 4 accs");
+  run<0, 128, 3, true>("tf32 MN-major N=128 3 accs");
   run<0, 64, 1>("tf32 N=64  same acc");
   run<0, 64, 4>("tf32 N=64  4 accs");
   run<0, 128, 1>("tf32 N=128 same acc");
