@@ -85,6 +85,13 @@ __device__ __forceinline__ void ffma2(float2& d, float a, float2 b) {
       : "+f"(d.x), "+f"(d.y)
       : "f"(a), "f"(b.x), "f"(b.y));
 }
+// d.x += a.x * b.x, d.y += a.y * b.y (packed, each lane rounded once like fmaf)
+__device__ __forceinline__ void ffma2v(float2& d, float2 a, float2 b) {
+  asm("{\n\t.reg .b64 a2, b2, d2;\n\tmov.b64 a2, {%2, %3};\n\tmov.b64 b2, {%4, %5};\n\tmov.b64 d2, {%0, %1};\n\t"
+      "fma.rn.f32x2 d2, a2, b2, d2;\n\tmov.b64 {%0, %1}, d2;\n\t}"
+      : "+f"(d.x), "+f"(d.y)
+      : "f"(a.x), "f"(a.y), "f"(b.x), "f"(b.y));
+}
 
 // Last-CTA-of-a-group detection for deterministic two-phase reductions: every CTA of the group
 // calls this after writing its partials; returns true in exactly one CTA (the last), which then

@@ -3,6 +3,8 @@
 // rows (one warp = 32 channels x one row); stride-2 dgrad gathers per output pixel (4 channels per
 // thread). wgrad reductions: fp32 per row, fp64 across rows, fixed-order CTA combine, ordered
 // split reduction (combine_splits) per channel block.
+#include <cstdlib>
+
 #include "common.cuh"
 
 namespace {
@@ -40,47 +42,80 @@ inline int dwq_smem(int C) { return 9 * (C / 4) * 16; }
 
 // y[n,p,q,c] = sum_{r,u} x[n, p*S-1+r, q*S-1+u, c] k[c,r,u]; with FLIP (and S = 1, x = dy) this is
 // the stride-1 data gradient dx[n,h,w,c] = sum_{r,u} dy[n,h+1-r,w+1-u,c] k[c,r,u].
+//
+// Round 3: a thread walks DOWN a band of output rows (fixed channel quad and segment of U outputs)
+// with a rolling register window of the three input rows the taps read, so each input row is loaded
+// once per segment (one new row per output row at stride 1, two at stride 2) instead of once per
+// output row that reads it: 1.5 instead of 4.5 128-bit loads per output at stride 1, U = 4.
+// Output rows per band: 16 for tall stride-1 maps (measured: 1.5 loads per output, 75 -> 63 us on
+// MobileNetV2's 112x112x32 layer); stride 2 reuses only one of three input rows per step, so it keeps
+// one row per item (more independent loads in flight; measured as fast as the band walk or faster).
+__host__ __device__ inline int dw_bh(int P, int S) {
+  if (S != 1) return 1;
+  return P >= 32 ? 16 : (P > 16 ? (P + 1) / 2 : P);
+}
 template <int S, bool FLIP, int U>
-__global__ void __launch_bounds__(DW_THREADS) dw_q4_fwd_kernel(const float* __restrict__ x, const float* __restrict__ w,
+__global__ void __launch_bounds__(DW_THREADS, 2) dw_q4_fwd_kernel(const float* __restrict__ x, const float* __restrict__ w,
                                                                float* __restrict__ y, int N, int H, int W, int C, int P, int Q,
                                                                OrionSig sig) {
   extern __shared__ float4 dwq_w[];
   stage_taps<FLIP>(w, C, dwq_w);
   constexpr int NC = (U - 1) * S + 3;
-  const int C4 = C / 4, nseg = (Q + U - 1) / U;
-  const long long items = (long long)N * P * nseg * C4;
+  const int C4 = C / 4, nseg = (Q + U - 1) / U, BH = dw_bh(P, S), nband = (P + BH - 1) / BH;
+  const long long items = (long long)N * nband * nseg * C4;
   for (long long it = (long long)blockIdx.x * blockDim.x + threadIdx.x; it < items; it += (long long)gridDim.x * blockDim.x) {
     const int quad = (int)(it % C4);
     long long t2 = it / C4;
     const int q0 = (int)(t2 % nseg) * U;
-    const long long row = t2 / nseg;
-    const int p = (int)(row % P), n = (int)(row / P);
-    const int c = quad * 4;
-    float4 v[3][NC];
-#pragma unroll
-    for (int r = 0; r < 3; r++) {
-      const int h = p * S - 1 + r;
+    t2 /= nseg;
+    const int band = (int)(t2 % nband), n = (int)(t2 / nband);
+    const int p0 = band * BH, p1 = min(P, p0 + BH);
+    const int c = quad * 4, w0 = q0 * S - 1;
+    const float* xn = x + (long long)n * H * W * C + c;
+    float4 win[3][NC];
+    auto load_row = [&](float4 (&dst)[NC], int h) {
       const bool rv = (unsigned)h < (unsigned)H;
-      const float* xr = x + (((long long)n * H + (rv ? h : 0)) * W) * C + c;
+      const float* xr = xn + (long long)(rv ? h : 0) * W * C;
 #pragma unroll
-      for (int j = 0; j < NC; j++) {
-        const int col = q0 * S - 1 + j;
-        v[r][j] = ld4(xr + (long long)col * C, rv && (unsigned)col < (unsigned)W);
-      }
+      for (int j = 0; j < NC; j++) dst[j] = ld4(xr + (long long)(w0 + j) * C, rv && (unsigned)(w0 + j) < (unsigned)W);
+    };
+    if (S == 1) {
+      load_row(win[0], p0 - 1);
+      load_row(win[1], p0);
+    } else {
+      load_row(win[2], 2 * p0 - 1);
     }
-    float4 k[9];
+#pragma unroll 1
+    for (int p = p0; p < p1; p++) {
+      if (S == 1) {
+        load_row(win[2], p + 1);
+      } else {
 #pragma unroll
-    for (int t = 0; t < 9; t++) k[t] = dwq_w[t * C4 + quad];
-    float* yr = y + (((long long)n * P + p) * Q + q0) * C + c;
+        for (int j = 0; j < NC; j++) win[0][j] = win[2][j];
+        load_row(win[1], 2 * p);
+        load_row(win[2], 2 * p + 1);
+      }
+      // tap rows outer (three taps live at a time), same per-output order r, t as before
+      float4 acc[U];
 #pragma unroll
-    for (int u = 0; u < U; u++) {
-      if (q0 + u < Q) {
-        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int u = 0; u < U; u++) acc[u] = make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
-        for (int r = 0; r < 3; r++)
+      for (int r = 0; r < 3; r++) {
+        float4 k[3];
 #pragma unroll
-          for (int t = 0; t < 3; t++) fma4(acc, v[r][u * S + t], k[r * 3 + t]);
-        *reinterpret_cast<float4*>(yr + (long long)u * C) = acc;
+        for (int t = 0; t < 3; t++) k[t] = dwq_w[(r * 3 + t) * C4 + quad];
+#pragma unroll
+        for (int u = 0; u < U; u++)
+#pragma unroll
+          for (int t = 0; t < 3; t++) fma4(acc[u], win[r][u * S + t], k[t]);
+      }
+      float* yr = y + (((long long)n * P + p) * Q + q0) * C + c;
+#pragma unroll
+      for (int u = 0; u < U; u++)
+        if (q0 + u < Q) *reinterpret_cast<float4*>(yr + (long long)u * C) = acc[u];
+      if (S == 1) {
+#pragma unroll
+        for (int j = 0; j < NC; j++) { win[0][j] = win[1][j]; win[1][j] = win[2][j]; }
       }
     }
   }
@@ -141,67 +176,110 @@ __global__ void __launch_bounds__(DW_THREADS) dw_q4_dgrad_s2_kernel(const float*
   orion_signal(sig);
 }
 
-// wgrad: dW[c,r,u] = sum_{n,p,q} dy[n,p,q,c] x[n, p*S-1+r, q*S-1+u, c]. CTA = a block of CQ channel
-// quads (quad = tid % CQ) x RL row lanes (tid / CQ); a thread walks whole output rows of its quad
-// with the sliding x window, accumulating the 36 products of a row in fp32, then adds the row into
-// its fp64 slots in shared memory (same order every run). Row lanes are combined in lane order,
-// CTAs write per-split partials, the last CTA of the channel block sums them in split order.
-constexpr int WQ_MAXQ = 64;   // channel quads per CTA (C <= 256 per block)
+// wgrad: dW[c,r,u] = sum_{n,p,q} dy[n,p,q,c] x[n, p*S-1+r, q*S-1+u, c]. A thread owns one channel
+// quad and a segment of WU_ output columns of one image and walks DOWN a band of BH output rows
+// with a rolling register window of the three x rows the taps read: per output row it loads only
+// the new x rows (one for stride 1, two for stride 2) and the dy quads, so every x row is read once
+// per segment (the round-2 row walker re-read each x row for three output rows and kept one
+// segment's loads in flight per thread). The 36 tap sums accumulate in fp32 over the band (packed
+// FFMA2), the CTA's lanes are summed in lane order in fp64, CTAs write per-split partials and the
+// last CTA of the channel block sums them in split order (combine_splits): deterministic.
+constexpr int WG_U = 2, WG_MAXQ = 64;
+
+// output rows per band of the weight-gradient walker (measured A/B in one process, MobileNetV2 b96):
+// 16 for the 112-row maps (103 us vs 107 / 118 at 32 / 64), 32 at stride 1 and the whole map at
+// stride 2 for the 56-row ones (123 vs 141 us; 102 vs 127 us); the whole map below 32 rows
+__host__ __device__ inline int wg_bh(int P, int S) {
+  if (P >= 100) return 16;
+  if (P >= 32) return S == 1 ? 32 : P;
+  return P;
+}
+
+// lanes enumerate (segment, band, image), segment fastest; a CTA covers 256 / cq consecutive lanes
+struct WgPlan { int cq, lanes, cblocks, nseg, nband, bh, rs; };
+inline WgPlan wg_plan(int N, int C, int P, int Q, int S) {
+  WgPlan w;
+  const int C4 = C / 4;
+  w.cq = C4 < WG_MAXQ ? C4 : WG_MAXQ;
+  w.lanes = DW_THREADS / w.cq;
+  w.cblocks = (int)cdiv(C4, w.cq);
+  w.nseg = (int)cdiv(Q, WG_U);
+  w.bh = wg_bh(P, S);
+  w.nband = (int)cdiv(P, w.bh);
+  w.rs = (int)cdiv((long long)N * w.nband * w.nseg, w.lanes);
+  return w;
+}
+
 template <int S>
-__global__ void __launch_bounds__(DW_THREADS, 2) dw_q4_wgrad_kernel(const float* __restrict__ x, const float* __restrict__ dy,
-                                                                    float* __restrict__ dwt, int N, int H, int W, int C, int P, int Q,
-                                                                    int cq_n, unsigned char* ws, OrionSig sig) {
-  extern __shared__ double wq_sh[];   // [rl][36][cq_n] fp64 row-sum slots, later [36 * cq_n] combine area
-  const int rl_n = DW_THREADS / cq_n;
-  const int cq = threadIdx.x % cq_n, rl = threadIdx.x / cq_n;
+__global__ void __launch_bounds__(DW_THREADS, 2) dw_wgrad_band_kernel(const float* __restrict__ x, const float* __restrict__ dy,
+                                                                      float* __restrict__ dwt, int N, int H, int W, int C, int P, int Q,
+                                                                      int cq_n, int nseg, int nband, int BH, unsigned char* ws, OrionSig sig) {
+  constexpr int NC = (WG_U - 1) * S + 3;   // x window columns of a segment
+  extern __shared__ float wb_sh[];         // [lane][36][cq_n] fp32 band sums, later the fp64 combine area
+  const int lanes = DW_THREADS / cq_n;
+  const int cq = threadIdx.x % cq_n, lane = threadIdx.x / cq_n;
   const int c = (blockIdx.x * cq_n + cq) * 4;
-  const bool active = rl < rl_n && c < C;
-  double* slot = wq_sh + (size_t)rl * 36 * cq_n + cq;
-  if (rl < rl_n)
-    for (int t = 0; t < 36; t++) slot[(size_t)t * cq_n] = 0.0;
-  const long long nrows = (long long)N * P;
-  if (active) {
-    for (long long row = (long long)blockIdx.y * rl_n + rl; row < nrows; row += (long long)gridDim.y * rl_n) {
-      const int p = (int)(row % P), n = (int)(row / P);
-      const float* xr[3];
-      bool rv[3];
+  const long long Lg = (long long)blockIdx.y * lanes + lane;   // (segment fastest, band, image)
+  const int seg = (int)(Lg % nseg);
+  const long long t1 = Lg / nseg;
+  const int band = (int)(t1 % nband), n = (int)(t1 / nband);
+  float2 f[9][2];   // tap t: channels (c, c+1) and (c+2, c+3)
 #pragma unroll
-      for (int r = 0; r < 3; r++) {
-        const int h = p * S - 1 + r;
-        rv[r] = (unsigned)h < (unsigned)H;
-        xr[r] = x + (((long long)n * H + (rv[r] ? h : 0)) * W) * C + c;
+  for (int t = 0; t < 9; t++) { f[t][0] = make_float2(0.f, 0.f); f[t][1] = make_float2(0.f, 0.f); }
+  if (lane < lanes && c < C && n < N) {
+    const int p0 = band * BH, p1 = min(P, p0 + BH), q0 = seg * WG_U, w0 = q0 * S - 1;
+    const float* xn = x + (long long)n * H * W * C + c;
+    const float* gn = dy + (long long)n * P * Q * C + c;
+    float4 win[3][NC];
+    auto load_row = [&](float4 (&dst)[NC], int h) {
+      const bool okh = (unsigned)h < (unsigned)H;
+      const float* xr = xn + (long long)(okh ? h : 0) * W * C;
+#pragma unroll
+      for (int j = 0; j < NC; j++) dst[j] = ld4(xr + (long long)(w0 + j) * C, okh && (unsigned)(w0 + j) < (unsigned)W);
+    };
+    // rows p*S-1, p*S, p*S+1 of output row p: window rows 0..2
+    if (S == 1) {
+      load_row(win[0], p0 - 1);
+      load_row(win[1], p0);
+    } else {
+      load_row(win[2], 2 * p0 - 1);
+    }
+#pragma unroll 1
+    for (int p = p0; p < p1; p++) {
+      if (S == 1) {
+        load_row(win[2], p + 1);
+      } else {
+#pragma unroll
+        for (int j = 0; j < NC; j++) win[0][j] = win[2][j];
+        load_row(win[1], 2 * p);
+        load_row(win[2], 2 * p + 1);
       }
-      const float* gr = dy + (((long long)n * P + p) * Q) * C + c;
-      float4 f[9];
+      float4 g[WG_U];
+      const float* gr = gn + (long long)p * Q * C;
 #pragma unroll
-      for (int t = 0; t < 9; t++) f[t] = make_float4(0.f, 0.f, 0.f, 0.f);
-      // segments of WU outputs: the (WU-1)*S+3 window columns and WU dy quads loaded at once
-      constexpr int WU = 2, NC = (WU - 1) * S + 3;
-      for (int q0 = 0; q0 < Q; q0 += WU) {
-        float4 v[3][NC], g[WU];
+      for (int u = 0; u < WG_U; u++) g[u] = ld4(gr + (long long)(q0 + u) * C, q0 + u < Q);
+#pragma unroll
+      for (int u = 0; u < WG_U; u++)
 #pragma unroll
         for (int r = 0; r < 3; r++)
 #pragma unroll
-          for (int j = 0; j < NC; j++) {
-            const int col = q0 * S - 1 + j;
-            v[r][j] = ld4(xr[r] + (long long)col * C, rv[r] && (unsigned)col < (unsigned)W);
+          for (int t = 0; t < 3; t++) {
+            const float4 v = win[r][u * S + t];
+            ffma2v(f[r * 3 + t][0], make_float2(g[u].x, g[u].y), make_float2(v.x, v.y));
+            ffma2v(f[r * 3 + t][1], make_float2(g[u].z, g[u].w), make_float2(v.z, v.w));
           }
+      if (S == 1) {
 #pragma unroll
-        for (int u = 0; u < WU; u++) g[u] = ld4(gr + (long long)(q0 + u) * C, q0 + u < Q);
-#pragma unroll
-        for (int u = 0; u < WU; u++)
-#pragma unroll
-          for (int r = 0; r < 3; r++)
-#pragma unroll
-            for (int t = 0; t < 3; t++) fma4(f[r * 3 + t], g[u], v[r][u * S + t]);
+        for (int j = 0; j < NC; j++) { win[0][j] = win[1][j]; win[1][j] = win[2][j]; }
       }
+    }
+  }
+  // lane sums: [lane][v][cq] fp32, v = tap*4 + channel-in-quad
+  if (lane < lanes) {
 #pragma unroll
-      for (int t = 0; t < 9; t++) {
-        slot[(size_t)(t * 4 + 0) * cq_n] += (double)f[t].x;
-        slot[(size_t)(t * 4 + 1) * cq_n] += (double)f[t].y;
-        slot[(size_t)(t * 4 + 2) * cq_n] += (double)f[t].z;
-        slot[(size_t)(t * 4 + 3) * cq_n] += (double)f[t].w;
-      }
+    for (int t = 0; t < 9; t++) {
+      float* d = wb_sh + ((size_t)lane * 36 + t * 4) * cq_n + cq;
+      d[0] = f[t][0].x; d[(size_t)cq_n] = f[t][0].y; d[2 * (size_t)cq_n] = f[t][1].x; d[3 * (size_t)cq_n] = f[t][1].y;
     }
   }
   __syncthreads();
@@ -209,22 +287,27 @@ __global__ void __launch_bounds__(DW_THREADS, 2) dw_q4_wgrad_kernel(const float*
   double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
   const int c0 = blockIdx.x * cq_n * 4;
   const int nch = min(cq_n * 4, C - c0);
-  // partial of this split: part[split][c][tap] (tap = r*3+u), row lanes summed in lane order
+  // partial of this split: part[split][c][tap] (tap = r*3+u), lanes summed in lane order (fp64)
   for (int v = threadIdx.x; v < nch * 9; v += DW_THREADS) {
     const int cc = v / 9, t = v % 9, q4 = cc / 4, j = cc % 4;
     double sum = 0.0;
-    for (int l = 0; l < rl_n; l++) sum += wq_sh[((size_t)l * 36 + t * 4 + j) * cq_n + q4];
+    for (int l = 0; l < lanes; l++) sum += (double)wb_sh[((size_t)l * 36 + t * 4 + j) * cq_n + q4];
     part[((long long)blockIdx.y * C + c0 + cc) * 9 + t] = sum;
   }
   const int rs = gridDim.y;
   const int V = 9 * nch;
-  double* out = wq_sh;   // reuse (the partials above are in global memory now)
   __syncthreads();
+  double* out = reinterpret_cast<double*>(wb_sh);   // reuse (the partials above are in global memory now)
   if (combine_splits(tickets + blockIdx.x * (combine_rows(rs) + 1), part + 9LL * c0, part + 9LL * rs * C + 9LL * c0, 9LL * C, rs,
                      blockIdx.y, V, out, out + V)) {
     for (int v = threadIdx.x; v < V; v += DW_THREADS) dwt[9LL * c0 + v] = (float)out[v];
   }
   orion_signal(sig);
+}
+inline int wg_smem(const WgPlan& w) {
+  const int lanesum = DW_THREADS * 36 * 4;                    // fp32 [lane][36][cq]
+  const int comb = (9 * 4 * w.cq + DW_THREADS) * 8;           // fp64 combine area + scratch
+  return lanesum > comb ? lanesum : comb;
 }
 
 // dx[n,h,w,c] = sum_{r,u} dy[n,p,q,c] * w[c,r,u] with h = p*stride - 1 + r
@@ -307,25 +390,13 @@ void q4_geom(LaunchGeom* g, long long items, const void* f, std::atomic<int>& oc
   g->grid = dim3((unsigned)ctas); g->block = dim3(DW_THREADS); g->smem = smem; g->func = f;
 }
 
-int wq_cq(int C) { const int q = C / 4; return q < WQ_MAXQ ? q : WQ_MAXQ; }
-int wq_smem(int C) { const int cq = wq_cq(C); const int rl = DW_THREADS / cq; return rl * 36 * cq * 8; }
-
-int wg_splits(const DwShape& s) {
-  const int cq = wq_cq(s.C);
-  long long cblocks = cdiv(s.C / 4, cq);
-  long long rs = cdiv(148 * 2, cblocks);                     // ~two CTAs per SM of a 148-SM part
-  long long max_rs = cdiv((long long)s.N * s.P, DW_THREADS / cq);
-  if (rs > max_rs) rs = max_rs;
-  if (rs < 1) rs = 1;
-  return (int)rs;
-}
-
 }  // namespace
 
 extern "C" uint64_t orion_dw_wgrad_workspace_bytes(uint64_t N, uint64_t C, uint64_t P, uint64_t Q) {
   if (C % 4) C += 4 - C % 4;
-  DwShape s{(int)N, 0, 0, (int)C, 1, (int)P, (int)Q};
-  const int rs = wg_splits(s);
+  // (the stride is not an argument: size for the larger of the two plans)
+  const WgPlan w1 = wg_plan((int)N, (int)C, (int)P, (int)Q, 1), w2 = wg_plan((int)N, (int)C, (int)P, (int)Q, 2);
+  const int rs = w1.rs > w2.rs ? w1.rs : w2.rs;
   return WS_TICKET_BYTES + (uint64_t)(rs + combine_rows(rs)) * C * 9 * 8;
 }
 
@@ -336,7 +407,8 @@ int dw_fwd_geom(const uint64_t* a, LaunchGeom* g) {
   DwShape s = dw_shape(a);
   if (s.stride != 1 && s.stride != 2) return ORION_E_INVAL;
   if (!dwq_prepare()) return ORION_E_CUDA;
-  const long long items = (long long)s.N * s.P * (s.C / 4) * cdiv(s.Q, s.stride == 1 ? DWQ_U1 : DWQ_U2);
+  const int U = s.stride == 1 ? DWQ_U1 : DWQ_U2;
+  const long long items = (long long)s.N * cdiv(s.P, dw_bh(s.P, s.stride)) * (s.C / 4) * cdiv(s.Q, U);
   if (s.stride == 1) q4_geom(g, items, (const void*)dw_q4_fwd_kernel<1, false, DWQ_U1>, dwq_occ[0], dwq_smem(s.C));
   else q4_geom(g, items, (const void*)dw_q4_fwd_kernel<2, false, DWQ_U2>, dwq_occ[1], dwq_smem(s.C));
   return 0;
@@ -357,7 +429,8 @@ int dw_dgrad_geom(const uint64_t* a, LaunchGeom* g) {
   DwShape s = dw_shape(a);
   if ((s.stride == 1 || s.stride == 2) && !dwq_prepare()) return ORION_E_CUDA;
   if (s.stride == 1)
-    q4_geom(g, (long long)s.N * s.H * (s.C / 4) * cdiv(s.W, DWQ_U1), (const void*)dw_q4_fwd_kernel<1, true, DWQ_U1>, dwq_occ[2], dwq_smem(s.C));
+    q4_geom(g, (long long)s.N * cdiv(s.H, dw_bh(s.H, 1)) * (s.C / 4) * cdiv(s.W, DWQ_U1),
+            (const void*)dw_q4_fwd_kernel<1, true, DWQ_U1>, dwq_occ[2], dwq_smem(s.C));
   else if (s.stride == 2)
     q4_geom(g, (long long)s.N * s.H * (s.C / 4) * cdiv((s.W + 1) / 2, DWQ_UP), (const void*)dw_q4_dgrad_s2_kernel<DWQ_UP>, dwq_occ[3],
             dwq_smem(s.C));
@@ -382,28 +455,29 @@ int dw_wgrad_geom(const uint64_t* a, LaunchGeom* g) {
   DwShape s = dw_shape(a);
   if (a[14] == 0 || a[15] < orion_dw_wgrad_workspace_bytes(s.N, s.C, s.P, s.Q)) return ORION_E_INVAL;
   if (s.stride != 1 && s.stride != 2) return ORION_E_INVAL;
+  const WgPlan w = wg_plan(s.N, s.C, s.P, s.Q, s.stride);
+  if ((uint64_t)w.cblocks * (combine_rows(w.rs) + 1) * 4 > WS_TICKET_BYTES || w.rs > 65535) return ORION_E_INVAL;
   static std::atomic<int> attr{0};
   if (!attr.load()) {
-    if (cudaFuncSetAttribute((const void*)dw_q4_wgrad_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024) != cudaSuccess ||
-        cudaFuncSetAttribute((const void*)dw_q4_wgrad_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024) != cudaSuccess) {
+    if (cudaFuncSetAttribute((const void*)dw_wgrad_band_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024) != cudaSuccess ||
+        cudaFuncSetAttribute((const void*)dw_wgrad_band_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 64 * 1024) != cudaSuccess) {
       (void)cudaGetLastError();
       return ORION_E_CUDA;
     }
     attr.store(1);
   }
-  const int cq = wq_cq(s.C);
-  g->grid = dim3((unsigned)cdiv(s.C / 4, cq), (unsigned)wg_splits(s)); g->block = dim3(DW_THREADS); g->smem = wq_smem(s.C);
-  g->func = s.stride == 1 ? (const void*)dw_q4_wgrad_kernel<1> : (const void*)dw_q4_wgrad_kernel<2>;
+  g->grid = dim3((unsigned)w.cblocks, (unsigned)w.rs); g->block = dim3(DW_THREADS); g->smem = wg_smem(w);
+  g->func = s.stride == 1 ? (const void*)dw_wgrad_band_kernel<1> : (const void*)dw_wgrad_band_kernel<2>;
   return 0;
 }
 int dw_wgrad_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   DwShape s = dw_shape(a);
-  const int cq = wq_cq(s.C);
-  if (g.func == (const void*)dw_q4_wgrad_kernel<1>)
-    dw_q4_wgrad_kernel<1><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q,
-                                                          cq, (unsigned char*)a[14], sig);
+  const WgPlan w = wg_plan(s.N, s.C, s.P, s.Q, s.stride);
+  if (g.func == (const void*)dw_wgrad_band_kernel<1>)
+    dw_wgrad_band_kernel<1><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q,
+                                                            w.cq, w.nseg, w.nband, w.bh, (unsigned char*)a[14], sig);
   else
-    dw_q4_wgrad_kernel<2><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q,
-                                                          cq, (unsigned char*)a[14], sig);
+    dw_wgrad_band_kernel<2><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s.N, s.H, s.W, s.C, s.P, s.Q,
+                                                            w.cq, w.nseg, w.nband, w.bh, (unsigned char*)a[14], sig);
   CHECK_LAUNCH();
 }

@@ -163,7 +163,9 @@ inline int lnb_smem(int C) { return (LN_T / 32) * 2 * C * 8 + LN_T * 8; }
 
 // ========================================================================== attention fp32
 // Per (batch, head): D = 64 columns at h*64 of [B, S, ld] rows; S <= 256, S % 32 == 0.
-constexpr int AD = 64, AQB = 64, AT = 128, AMAXK = 8;   // keys per lane: S / 32 <= 8
+constexpr int AD = 64, AQB = 64, AT = 256, AMAXK = 8;   // keys per lane: S / 32 <= 8
+constexpr int AW = AT / 32;                             // warps per CTA (AQB / AW rows each)
+constexpr int ACH = 4;                                  // independent partial sums per long reduction
 
 // forward: O_i = sum_j softmax_j(q_i . k_j / sqrt d) v_j
 __global__ void __launch_bounds__(AT) attn_fwd_kernel(const float* __restrict__ q, const float* __restrict__ k, const float* __restrict__ v,
@@ -172,7 +174,7 @@ __global__ void __launch_bounds__(AT) attn_fwd_kernel(const float* __restrict__ 
   float* Ks = asm_;                       // [S][AD + 1]
   float* Vs = Ks + S * (AD + 1);          // [S][AD]
   float* Qs = Vs + S * AD;                // [4 warps][AD]
-  float* Ps = Qs + 4 * AD;                // [4 warps][S]
+  float* Ps = Qs + AW * AD;               // [AW warps][S]
   const int b = blockIdx.z, h = blockIdx.y, lane = threadIdx.x % 32, warp = threadIdx.x / 32;
   const long long ib = (long long)b * S * ldi + h * AD, ob = (long long)b * S * ldo + h * AD;
   for (int e = threadIdx.x; e < S * AD / 4; e += AT) {
@@ -183,7 +185,7 @@ __global__ void __launch_bounds__(AT) attn_fwd_kernel(const float* __restrict__ 
   }
   __syncthreads();
   const int nk = S / 32;
-  for (int qi = blockIdx.x * AQB + warp * (AQB / 4); qi < min(S, blockIdx.x * AQB + (warp + 1) * (AQB / 4)); qi++) {
+  for (int qi = blockIdx.x * AQB + warp * (AQB / AW); qi < min(S, blockIdx.x * AQB + (warp + 1) * (AQB / AW)); qi++) {
     Qs[warp * AD + lane] = __ldg(q + ib + (long long)qi * ldi + lane);
     Qs[warp * AD + 32 + lane] = __ldg(q + ib + (long long)qi * ldi + 32 + lane);
     __syncwarp();
@@ -207,12 +209,19 @@ __global__ void __launch_bounds__(AT) attn_fwd_kernel(const float* __restrict__ 
       if (t < nk) { sc[t] = expf(sc[t] - mx); l += sc[t]; Ps[warp * S + lane + 32 * t] = sc[t]; }
     l = warp_sum(l);
     __syncwarp();
-    float o0 = 0.f, o1 = 0.f;
-    for (int j = 0; j < S; j++) {
-      const float p = Ps[warp * S + j];
-      o0 = fmaf(p, Vs[j * AD + lane], o0);
-      o1 = fmaf(p, Vs[j * AD + 32 + lane], o1);
+    // ACH interleaved partial sums per output (the serial 192-term chain was latency-bound)
+    float o0p[ACH], o1p[ACH];
+#pragma unroll
+    for (int i = 0; i < ACH; i++) { o0p[i] = 0.f; o1p[i] = 0.f; }
+    for (int j = 0; j < S; j += ACH) {
+#pragma unroll
+      for (int i = 0; i < ACH; i++) {
+        const float p = Ps[warp * S + j + i];
+        o0p[i] = fmaf(p, Vs[(j + i) * AD + lane], o0p[i]);
+        o1p[i] = fmaf(p, Vs[(j + i) * AD + 32 + lane], o1p[i]);
+      }
     }
+    const float o0 = (o0p[0] + o0p[1]) + (o0p[2] + o0p[3]), o1 = (o1p[0] + o1p[1]) + (o1p[2] + o1p[3]);
     const float rl = 1.f / l;
     o[ob + (long long)qi * ldo + lane] = o0 * rl;
     o[ob + (long long)qi * ldo + 32 + lane] = o1 * rl;
@@ -230,9 +239,9 @@ __global__ void __launch_bounds__(AT) attn_bwd_dq_kernel(const float* __restrict
   extern __shared__ __align__(16) float asm_[];
   float* Ks = asm_;                       // [S][AD + 1]
   float* Vs = Ks + S * (AD + 1);          // [S][AD + 1]
-  float* Qs = Vs + S * (AD + 1);          // [4][AD]  (q row)
-  float* Gs = Qs + 4 * AD;                // [4][AD]  (dO row)
-  float* Ps = Gs + 4 * AD;                // [4][S]   (dS row)
+  float* Qs = Vs + S * (AD + 1);          // [AW][AD]  (q row)
+  float* Gs = Qs + AW * AD;               // [AW][AD]  (dO row)
+  float* Ps = Gs + AW * AD;               // [AW][S]   (dS row)
   const int b = blockIdx.z, h = blockIdx.y, lane = threadIdx.x % 32, warp = threadIdx.x / 32;
   const long long ib = (long long)b * S * ldi + h * AD, ob = (long long)b * S * ldo + h * AD;
   for (int e = threadIdx.x; e < S * AD / 4; e += AT) {
@@ -245,7 +254,7 @@ __global__ void __launch_bounds__(AT) attn_bwd_dq_kernel(const float* __restrict
   }
   __syncthreads();
   const int nk = S / 32;
-  for (int qi = blockIdx.x * AQB + warp * (AQB / 4); qi < min(S, blockIdx.x * AQB + (warp + 1) * (AQB / 4)); qi++) {
+  for (int qi = blockIdx.x * AQB + warp * (AQB / AW); qi < min(S, blockIdx.x * AQB + (warp + 1) * (AQB / AW)); qi++) {
     Qs[warp * AD + lane] = __ldg(q + ib + (long long)qi * ldi + lane);
     Qs[warp * AD + 32 + lane] = __ldg(q + ib + (long long)qi * ldi + 32 + lane);
     Gs[warp * AD + lane] = __ldg(dO + ob + (long long)qi * ldo + lane);
@@ -280,12 +289,18 @@ __global__ void __launch_bounds__(AT) attn_bwd_dq_kernel(const float* __restrict
     for (int t = 0; t < AMAXK; t++)
       if (t < nk) Ps[warp * S + lane + 32 * t] = sc[t] * (dp[t] - dl);
     __syncwarp();
-    float g0 = 0.f, g1 = 0.f;
-    for (int j = 0; j < S; j++) {
-      const float ds = Ps[warp * S + j];
-      g0 = fmaf(ds, Ks[j * (AD + 1) + lane], g0);
-      g1 = fmaf(ds, Ks[j * (AD + 1) + 32 + lane], g1);
+    float g0p[ACH], g1p[ACH];
+#pragma unroll
+    for (int i = 0; i < ACH; i++) { g0p[i] = 0.f; g1p[i] = 0.f; }
+    for (int j = 0; j < S; j += ACH) {
+#pragma unroll
+      for (int i = 0; i < ACH; i++) {
+        const float ds = Ps[warp * S + j + i];
+        g0p[i] = fmaf(ds, Ks[(j + i) * (AD + 1) + lane], g0p[i]);
+        g1p[i] = fmaf(ds, Ks[(j + i) * (AD + 1) + 32 + lane], g1p[i]);
+      }
     }
+    const float g0 = (g0p[0] + g0p[1]) + (g0p[2] + g0p[3]), g1 = (g1p[0] + g1p[1]) + (g1p[2] + g1p[3]);
     dq[ib + (long long)qi * ldi + lane] = g0 * scale;
     dq[ib + (long long)qi * ldi + 32 + lane] = g1 * scale;
     if (lane == 0) {
@@ -306,9 +321,9 @@ __global__ void __launch_bounds__(AT) attn_bwd_dkv_kernel(const float* __restric
   float* Qs = asm_;                       // [S][AD + 1]
   float* Gs = Qs + S * (AD + 1);          // [S][AD + 1]  (dO)
   float* St = Gs + S * (AD + 1);          // [S][3]
-  float* Ks = St + S * 3;                 // [4][AD]
-  float* Vw = Ks + 4 * AD;                // [4][AD]
-  float* Pw = Vw + 4 * AD;                // [4][2][S]
+  float* Ks = St + S * 3;                 // [AW][AD]
+  float* Vw = Ks + AW * AD;               // [AW][AD]
+  float* Pw = Vw + AW * AD;               // [AW][2][S]
   const int b = blockIdx.z, h = blockIdx.y, lane = threadIdx.x % 32, warp = threadIdx.x / 32;
   const long long ib = (long long)b * S * ldi + h * AD, ob = (long long)b * S * ldo + h * AD;
   for (int e = threadIdx.x; e < S * AD / 4; e += AT) {
@@ -322,7 +337,7 @@ __global__ void __launch_bounds__(AT) attn_bwd_dkv_kernel(const float* __restric
   for (int e = threadIdx.x; e < S * 3; e += AT) St[e] = __ldg(stats + ((long long)b * H + h) * S * 3 + e);
   __syncthreads();
   const int nq = S / 32;
-  for (int kj = blockIdx.x * AQB + warp * (AQB / 4); kj < min(S, blockIdx.x * AQB + (warp + 1) * (AQB / 4)); kj++) {
+  for (int kj = blockIdx.x * AQB + warp * (AQB / AW); kj < min(S, blockIdx.x * AQB + (warp + 1) * (AQB / AW)); kj++) {
     Ks[warp * AD + lane] = __ldg(k + ib + (long long)kj * ldi + lane);
     Ks[warp * AD + 32 + lane] = __ldg(k + ib + (long long)kj * ldi + 32 + lane);
     Vw[warp * AD + lane] = __ldg(v + ib + (long long)kj * ldi + lane);
@@ -343,14 +358,22 @@ __global__ void __launch_bounds__(AT) attn_bwd_dkv_kernel(const float* __restric
       }
     }
     __syncwarp();
-    float v0 = 0.f, v1 = 0.f, k0 = 0.f, k1 = 0.f;
-    for (int i = 0; i < S; i++) {
-      const float p = Pw[(warp * 2) * S + i], ds = Pw[(warp * 2 + 1) * S + i];
-      v0 = fmaf(p, Gs[i * (AD + 1) + lane], v0);
-      v1 = fmaf(p, Gs[i * (AD + 1) + 32 + lane], v1);
-      k0 = fmaf(ds, Qs[i * (AD + 1) + lane], k0);
-      k1 = fmaf(ds, Qs[i * (AD + 1) + 32 + lane], k1);
+    float v0p[ACH], v1p[ACH], k0p[ACH], k1p[ACH];
+#pragma unroll
+    for (int e = 0; e < ACH; e++) { v0p[e] = 0.f; v1p[e] = 0.f; k0p[e] = 0.f; k1p[e] = 0.f; }
+    for (int i0 = 0; i0 < S; i0 += ACH) {
+#pragma unroll
+      for (int e = 0; e < ACH; e++) {
+        const int i = i0 + e;
+        const float p = Pw[(warp * 2) * S + i], ds = Pw[(warp * 2 + 1) * S + i];
+        v0p[e] = fmaf(p, Gs[i * (AD + 1) + lane], v0p[e]);
+        v1p[e] = fmaf(p, Gs[i * (AD + 1) + 32 + lane], v1p[e]);
+        k0p[e] = fmaf(ds, Qs[i * (AD + 1) + lane], k0p[e]);
+        k1p[e] = fmaf(ds, Qs[i * (AD + 1) + 32 + lane], k1p[e]);
+      }
     }
+    const float v0 = (v0p[0] + v0p[1]) + (v0p[2] + v0p[3]), v1 = (v1p[0] + v1p[1]) + (v1p[2] + v1p[3]);
+    const float k0 = (k0p[0] + k0p[1]) + (k0p[2] + k0p[3]), k1 = (k1p[0] + k1p[1]) + (k1p[2] + k1p[3]);
     dv[ib + (long long)kj * ldi + lane] = v0;
     dv[ib + (long long)kj * ldi + 32 + lane] = v1;
     dk[ib + (long long)kj * ldi + lane] = k0 * scale;
@@ -359,9 +382,9 @@ __global__ void __launch_bounds__(AT) attn_bwd_dkv_kernel(const float* __restric
   }
   orion_signal(sig);
 }
-inline int attn_fwd_smem(int S) { return (S * (AD + 1) + S * AD + 4 * AD + 4 * S) * 4; }
-inline int attn_dq_smem(int S) { return (2 * S * (AD + 1) + 8 * AD + 4 * S) * 4; }
-inline int attn_dkv_smem(int S) { return (2 * S * (AD + 1) + 3 * S + 8 * AD + 8 * S) * 4; }
+inline int attn_fwd_smem(int S) { return (S * (AD + 1) + S * AD + AW * AD + AW * S) * 4; }
+inline int attn_dq_smem(int S) { return (2 * S * (AD + 1) + 2 * AW * AD + AW * S) * 4; }
+inline int attn_dkv_smem(int S) { return (2 * S * (AD + 1) + 3 * S + 2 * AW * AD + 2 * AW * S) * 4; }
 bool attn_prepare() {
   static std::atomic<int> done{0};
   if (done.load()) return true;

@@ -1878,13 +1878,18 @@ int launch_tiled(const LaunchGeom& g, long long M, long long N, long long K, flo
 namespace smallc {
 constexpr int NTH = 256, MAXK = 64;
 
-template <int R, int S, int C>
+template <int R, int S, int C, int K>
 __global__ void __launch_bounds__(NTH) conv_fwd_smallc_kernel(const float* __restrict__ x, const float* __restrict__ w,
                                                               float* __restrict__ y, ConvShape s, OrionSig sig) {
   constexpr int RSC = R * S * C;
-  __shared__ float ws_[MAXK * RSC];
-  for (int i = threadIdx.x; i < s.K * RSC; i += NTH) ws_[i] = __ldg(w + i);
+  // weights transposed to [rsc][k]: one warp-uniform 128-bit load feeds four outputs' FMAs, issued
+  // as two packed FFMA2 (each output still sums its RSC products in rsc order, as fmaf would).
+  // (Measured: as fast as the scalar form -- the kernel is bound by its L1 traffic, ncu "Mem Busy"
+  // 91 %; a shared-memory-staged variant with coalesced row stores was slower, 171 vs 118 us.)
+  __shared__ __align__(16) float wt[RSC * K];
+  for (int i = threadIdx.x; i < K * RSC; i += NTH) wt[(i % RSC) * K + i / RSC] = __ldg(w + i);
   __syncthreads();
+  const float4* wt4 = reinterpret_cast<const float4*>(wt);
   const long long npix = (long long)s.N * s.P * s.Q;
   for (long long pix = (long long)blockIdx.x * NTH + threadIdx.x; pix < npix; pix += (long long)gridDim.x * NTH) {
     const int q = (int)(pix % s.Q); const long long t = pix / s.Q;
@@ -1902,25 +1907,27 @@ __global__ void __launch_bounds__(NTH) conv_fwd_smallc_kernel(const float* __res
         for (int c = 0; c < C; c++) patch[(r * S + u) * C + c] = ok ? __ldg(src + c) : 0.f;
       }
     }
-    float* dst = y + pix * s.K;
-    for (int k0 = 0; k0 < s.K; k0 += 4) {
-      float o[4];
+    float2 acc[K / 2];
 #pragma unroll
-      for (int j = 0; j < 4; j++) {
-        const float* wr = ws_ + (k0 + j) * RSC;
-        float acc = 0.f;
+    for (int j = 0; j < K / 2; j++) acc[j] = make_float2(0.f, 0.f);
 #pragma unroll
-        for (int i = 0; i < RSC; i++) acc = fmaf(patch[i], wr[i], acc);
-        o[j] = acc;
+    for (int i = 0; i < RSC; i++) {
+#pragma unroll
+      for (int kq = 0; kq < K / 4; kq++) {
+        const float4 w4 = wt4[i * (K / 4) + kq];
+        ffma2(acc[2 * kq], patch[i], make_float2(w4.x, w4.y));
+        ffma2(acc[2 * kq + 1], patch[i], make_float2(w4.z, w4.w));
       }
-      *reinterpret_cast<float4*>(dst + k0) = make_float4(o[0], o[1], o[2], o[3]);
     }
+    float4* dst = reinterpret_cast<float4*>(y + pix * K);
+#pragma unroll
+    for (int kq = 0; kq < K / 4; kq++) dst[kq] = make_float4(acc[2 * kq].x, acc[2 * kq].y, acc[2 * kq + 1].x, acc[2 * kq + 1].y);
   }
   orion_signal(sig);
 }
 
 // specialised for the 3x3, 3-channel stem (the only few-channel conv of the workloads)
-inline bool fwd_ok(const ConvShape& s) { return s.C == 3 && s.R == 3 && s.S == 3 && s.K % 4 == 0 && s.K <= MAXK; }
+inline bool fwd_ok(const ConvShape& s) { return s.C == 3 && s.R == 3 && s.S == 3 && s.K == 32; }
 
 // Weight gradient of a few-input-channel stem (ResNet 7x7x3 / MobileNetV2 3x3x3):
 // dw[k][r][s][c] = sum_{n,p,q} dy[n,p,q,k] x[n, p*st-pad+r, q*st-pad+s, c]. As an implicit GEMM the
@@ -2089,11 +2096,11 @@ __global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc2_kernel(const float*
       off[i] = 0;   // padding slot, never stored
     }
   }
-  float acc[4][W2_NR];
+  float2 acc2[2][W2_NR];   // acc2[a2][j] = outputs (k = kg*4 + 2*a2, +1) of rsc slot j
 #pragma unroll
-  for (int a = 0; a < 4; a++)
+  for (int a = 0; a < 2; a++)
 #pragma unroll
-    for (int i = 0; i < W2_NR; i++) acc[a][i] = 0.f;
+    for (int i = 0; i < W2_NR; i++) acc2[a][i] = make_float2(0.f, 0.f);
   const int qtiles = (s.Q + W2_QT - 1) / W2_QT;
   const long long T = (long long)s.N * s.P * qtiles;
   constexpr int PF_DY = (W2_QT * K / 4 + NTH - 1) / NTH;   // 4 float4 per thread
@@ -2144,10 +2151,8 @@ __global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc2_kernel(const float*
 #pragma unroll
       for (int j = 0; j < W2_NR; j++) {
         const float xv = xr[off[j]];
-        acc[0][j] = fmaf(d.x, xv, acc[0][j]);
-        acc[1][j] = fmaf(d.y, xv, acc[1][j]);
-        acc[2][j] = fmaf(d.z, xv, acc[2][j]);
-        acc[3][j] = fmaf(d.w, xv, acc[3][j]);
+        ffma2(acc2[0][j], xv, make_float2(d.x, d.y));   // (k, k+1) pairs: packed FFMA2, same rounding as fmaf
+        ffma2(acc2[1][j], xv, make_float2(d.z, d.w));
       }
     }
   }
@@ -2160,7 +2165,7 @@ __global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc2_kernel(const float*
     const int jj = rs + 4 * j;
     if (jj < RSC) {
 #pragma unroll
-      for (int a = 0; a < 4; a++) wp[warp * V + (kg * 4 + a) * RSC + jj] = acc[a][j];
+      for (int a = 0; a < 4; a++) wp[warp * V + (kg * 4 + a) * RSC + jj] = (a & 1) ? acc2[a / 2][j].y : acc2[a / 2][j].x;
     }
   }
   __syncthreads();
@@ -2352,7 +2357,7 @@ int conv_fwd_geom(const uint64_t* a, LaunchGeom* g) {
   if (smallc::fwd_ok(s)) {
     long long ctas = cdiv((long long)s.N * s.P * s.Q, smallc::NTH);
     g->grid = dim3((unsigned)(ctas < 148 * 16 ? ctas : 148 * 16)); g->block = dim3(smallc::NTH); g->smem = 0;
-    g->func = (const void*)smallc::conv_fwd_smallc_kernel<3, 3, 3>;
+    g->func = (const void*)smallc::conv_fwd_smallc_kernel<3, 3, 3, 32>;
     return 0;
   }
   if (cvf_conv_try_geom(a, g)) return 0;   // TMA im2col boxes straight into tcgen05 (cvf.cu)
@@ -2362,8 +2367,8 @@ int conv_fwd_geom(const uint64_t* a, LaunchGeom* g) {
 int conv_fwd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t st) {
   if (cvf_is(g.func)) return cvf_conv_launch(a, g, sig, st);
   ConvShape s = conv_shape(a);
-  if (g.func == (const void*)smallc::conv_fwd_smallc_kernel<3, 3, 3>) {
-    smallc::conv_fwd_smallc_kernel<3, 3, 3><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s, sig);
+  if (g.func == (const void*)smallc::conv_fwd_smallc_kernel<3, 3, 3, 32>) {
+    smallc::conv_fwd_smallc_kernel<3, 3, 3, 32><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
   long long M = (long long)s.N * s.P * s.Q, N = s.K, K = (long long)s.R * s.S * s.C;

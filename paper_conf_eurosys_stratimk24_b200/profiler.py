@@ -136,7 +136,7 @@ def occupancy_limits(threads, regs, smem):
     warps_by_regs = (SM_REGS // SM_PARTITIONS // per_warp) * SM_PARTITIONS if regs > 0 else SM_MAX_WARPS
     lim_regs = warps_by_regs // warps
     per_cta = -(-smem // SMEM_ALLOC_UNIT) * SMEM_ALLOC_UNIT + CTA_SMEM_RESERVED
-    lim_smem = SM_SMEM // per_cta
+    lim_smem = min(SM_SMEM // per_cta, SM_MAX_CTAS)   # (ncu reports the block cap for smem-free kernels)
     return {"warps": lim_warps, "registers": lim_regs, "shared_mem": lim_smem, "blocks": SM_MAX_CTAS}
 
 

@@ -115,7 +115,9 @@ def test_conv_fwd_dgrad_wgrad(shape):
 
 @pytest.mark.parametrize("n,h,wd,c,st", [(2, 15, 15, 32, 1), (3, 16, 16, 96, 2), (2, 7, 7, 960, 1), (1, 9, 9, 8, 2),
                                           (2, 14, 11, 144, 1), (2, 13, 10, 144, 2), (1, 5, 4, 12, 1), (1, 6, 7, 4, 2),
-                                          (3, 28, 28, 192, 2), (1, 1, 1, 16, 1), (1, 2, 3, 8, 2)])
+                                          (3, 28, 28, 192, 2), (1, 1, 1, 16, 1), (1, 2, 3, 8, 2),
+                                          # several 16-row bands of the weight-gradient walker, ragged last band
+                                          (4, 112, 112, 32, 1), (4, 64, 64, 24, 2), (2, 70, 66, 8, 1), (2, 67, 65, 12, 2)])
 def test_depthwise(n, h, wd, c, st):
     """Depthwise 3x3 fwd / dgrad / wgrad (MobileNetV2 shapes incl. C = 144, stride 2, non-square and
     ragged widths that exercise the 3x unrolled window rotation and its remainder)."""

@@ -138,6 +138,35 @@ def bn():
               f"bwd_reduce {t2:6.1f} us {8 * rows * c / t2 / 1e3:5.0f} GB/s")
     print(f"bn total {tot:.1f} us")
 
+def stem():
+    """MobileNetV2 b96 stem (3x3/2, 3 -> 32 channels): forward and weight gradient."""
+    n, h, c, k = 96, 224, 3, 32
+    p = 112
+    x, wt = torch.randn(n, h, h, c, device="cuda"), torch.randn(k, 3, 3, c, device="cuda")
+    y, dy, dw = torch.zeros(n, p, p, k, device="cuda"), torch.randn(n, p, p, k, device="cuda"), torch.zeros(k, 3, 3, c, device="cuda")
+    dims = [n, h, h, c, k, 3, 3, 2, 1, p, p]
+    wf = ws(max(L.lib.orion_gemm_workspace_bytes(n * p * p, k, 27), L.lib.orion_conv_wgrad_workspace_bytes(n, h, h, c, k, 3, 3, 2, 1)))
+    byt = (x.numel() + y.numel()) * 4
+    t1 = timeit("conv_fwd", [x.data_ptr(), wt.data_ptr(), y.data_ptr()] + dims + [wf.data_ptr(), wf.numel() * 4])
+    t2 = timeit("conv_wgrad", [x.data_ptr(), dy.data_ptr(), dw.data_ptr()] + dims + [wf.data_ptr(), wf.numel() * 4])
+    print(f"stem fwd {t1:7.1f} us {byt / t1 / 1e3:5.0f} GB/s   wgrad {t2:7.1f} us {byt / t2 / 1e3:5.0f} GB/s")
+
+
+def attn():
+    """Config-4 encoder attention (fp32): B 8, S 192, 8 heads of 64; forward and the two backward ops."""
+    B, S, H, d = 8, 192, 8, 64
+    D = H * d
+    q, k, v, o, do = (torch.randn(B, S, D, device="cuda") for _ in range(5))
+    dq, dk, dv = (torch.zeros(B, S, D, device="cuda") for _ in range(3))
+    st = torch.zeros(B, H, S, 3, device="cuda")
+    t1 = timeit("attention_f32", [q.data_ptr(), k.data_ptr(), v.data_ptr(), o.data_ptr(), B, S, H, d, D, D])
+    t2 = timeit("attention_f32_bwd_dq", [q.data_ptr(), k.data_ptr(), v.data_ptr(), do.data_ptr(), dq.data_ptr(), st.data_ptr(), B, S, H, d, D, D])
+    t3 = timeit("attention_f32_bwd_dkv", [q.data_ptr(), k.data_ptr(), v.data_ptr(), do.data_ptr(), st.data_ptr(), dk.data_ptr(), dv.data_ptr(),
+                                           B, S, H, d, D, D])
+    fl = 4 * B * H * S * S * d
+    print(f"attn fwd {t1:7.1f} us ({fl / t1 / 1e6:5.1f} TF)  bwd_dq {t2:7.1f} us  bwd_dkv {t3:7.1f} us")
+
+
 def wgs():
     tot = 0.0
     for M, N, K in WGS:
@@ -176,6 +205,10 @@ if __name__ == "__main__":
     what = sys.argv[1] if len(sys.argv) > 1 else "all"
     if what in ("wgs", "all"):
         wgs()
+    if what in ("stem", "all"):
+        stem()
+    if what in ("attn", "all"):
+        attn()
     if what in ("dw", "all"):
         dw()
     if what in ("conv", "all"):
