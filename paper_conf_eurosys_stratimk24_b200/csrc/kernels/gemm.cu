@@ -1881,12 +1881,14 @@ constexpr int NTH = 256, MAXK = 64;
 template <int R, int S, int C, int K>
 __global__ void __launch_bounds__(NTH) conv_fwd_smallc_kernel(const float* __restrict__ x, const float* __restrict__ w,
                                                               float* __restrict__ y, ConvShape s, OrionSig sig) {
-  constexpr int RSC = R * S * C;
+  constexpr int RSC = R * S * C, SC = S * C;
   // weights transposed to [rsc][k]: one warp-uniform 128-bit load feeds four outputs' FMAs, issued
-  // as two packed FFMA2 (each output still sums its RSC products in rsc order, as fmaf would).
-  // (Measured: as fast as the scalar form -- the kernel is bound by its L1 traffic, ncu "Mem Busy"
-  // 91 %; a shared-memory-staged variant with coalesced row stores was slower, 171 vs 118 us.)
-  __shared__ __align__(16) float wt[RSC * K];
+  // as two packed FFMA2 (each output still sums its RSC products in rsc order, as fmaf would). The
+  // window is gathered one filter row (S*C values) at a time, so the 7x7x3 ResNet stem fits in
+  // registers too. (Measured on the 3x3 stem: as fast as the scalar form -- it is bound by its L1
+  // traffic, ncu "Mem Busy" 91 %; a shared-memory-staged variant with coalesced row stores was
+  // slower, 171 vs 118 us.)
+  extern __shared__ __align__(16) float wt[];   // [RSC][K]
   for (int i = threadIdx.x; i < K * RSC; i += NTH) wt[(i % RSC) * K + i / RSC] = __ldg(w + i);
   __syncthreads();
   const float4* wt4 = reinterpret_cast<const float4*>(wt);
@@ -1894,29 +1896,29 @@ __global__ void __launch_bounds__(NTH) conv_fwd_smallc_kernel(const float* __res
   for (long long pix = (long long)blockIdx.x * NTH + threadIdx.x; pix < npix; pix += (long long)gridDim.x * NTH) {
     const int q = (int)(pix % s.Q); const long long t = pix / s.Q;
     const int p = (int)(t % s.P); const int n = (int)(t / s.P);
-    float patch[RSC];
+    float2 acc[K / 2];
 #pragma unroll
+    for (int j = 0; j < K / 2; j++) acc[j] = make_float2(0.f, 0.f);
+#pragma unroll 1
     for (int r = 0; r < R; r++) {
       const int h = p * s.stride - s.pad + r;
+      float patch[SC];
 #pragma unroll
       for (int u = 0; u < S; u++) {
         const int ww = q * s.stride - s.pad + u;
         const bool ok = (unsigned)h < (unsigned)s.H && (unsigned)ww < (unsigned)s.W;
         const float* src = x + (((long long)n * s.H + (ok ? h : 0)) * s.W + (ok ? ww : 0)) * C;
 #pragma unroll
-        for (int c = 0; c < C; c++) patch[(r * S + u) * C + c] = ok ? __ldg(src + c) : 0.f;
+        for (int c = 0; c < C; c++) patch[u * C + c] = ok ? __ldg(src + c) : 0.f;
       }
-    }
-    float2 acc[K / 2];
 #pragma unroll
-    for (int j = 0; j < K / 2; j++) acc[j] = make_float2(0.f, 0.f);
+      for (int i = 0; i < SC; i++) {
 #pragma unroll
-    for (int i = 0; i < RSC; i++) {
-#pragma unroll
-      for (int kq = 0; kq < K / 4; kq++) {
-        const float4 w4 = wt4[i * (K / 4) + kq];
-        ffma2(acc[2 * kq], patch[i], make_float2(w4.x, w4.y));
-        ffma2(acc[2 * kq + 1], patch[i], make_float2(w4.z, w4.w));
+        for (int kq = 0; kq < K / 4; kq++) {
+          const float4 w4 = wt4[(r * SC + i) * (K / 4) + kq];
+          ffma2(acc[2 * kq], patch[i], make_float2(w4.x, w4.y));
+          ffma2(acc[2 * kq + 1], patch[i], make_float2(w4.z, w4.w));
+        }
       }
     }
     float4* dst = reinterpret_cast<float4*>(y + pix * K);
@@ -1927,7 +1929,9 @@ __global__ void __launch_bounds__(NTH) conv_fwd_smallc_kernel(const float* __res
 }
 
 // specialised for the 3x3, 3-channel stem (the only few-channel conv of the workloads)
-inline bool fwd_ok(const ConvShape& s) { return s.C == 3 && s.R == 3 && s.S == 3 && s.K == 32; }
+inline bool fwd3_ok(const ConvShape& s) { return s.C == 3 && s.R == 3 && s.S == 3 && s.K == 32; }   // MobileNetV2
+inline bool fwd7_ok(const ConvShape& s) { return s.C == 3 && s.R == 7 && s.S == 7 && s.K == 64; }   // ResNet
+inline bool fwd_ok(const ConvShape& s) { return fwd3_ok(s) || fwd7_ok(s); }
 
 // Weight gradient of a few-input-channel stem (ResNet 7x7x3 / MobileNetV2 3x3x3):
 // dw[k][r][s][c] = sum_{n,p,q} dy[n,p,q,k] x[n, p*st-pad+r, q*st-pad+s, c]. As an implicit GEMM the
@@ -2355,9 +2359,19 @@ static ConvShape conv_shape(const uint64_t* a) {
 int conv_fwd_geom(const uint64_t* a, LaunchGeom* g) {
   ConvShape s = conv_shape(a);
   if (smallc::fwd_ok(s)) {
+    static std::atomic<int> attr{0};
+    if (!attr.load()) {
+      if (cudaFuncSetAttribute((const void*)smallc::conv_fwd_smallc_kernel<7, 7, 3, 64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               7 * 7 * 3 * 64 * 4) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return ORION_E_CUDA;
+      }
+      attr.store(1);
+    }
     long long ctas = cdiv((long long)s.N * s.P * s.Q, smallc::NTH);
-    g->grid = dim3((unsigned)(ctas < 148 * 16 ? ctas : 148 * 16)); g->block = dim3(smallc::NTH); g->smem = 0;
-    g->func = (const void*)smallc::conv_fwd_smallc_kernel<3, 3, 3, 32>;
+    g->grid = dim3((unsigned)(ctas < 148 * 16 ? ctas : 148 * 16)); g->block = dim3(smallc::NTH);
+    g->smem = s.R * s.S * s.C * s.K * 4;
+    g->func = smallc::fwd3_ok(s) ? (const void*)smallc::conv_fwd_smallc_kernel<3, 3, 3, 32> : (const void*)smallc::conv_fwd_smallc_kernel<7, 7, 3, 64>;
     return 0;
   }
   if (cvf_conv_try_geom(a, g)) return 0;   // TMA im2col boxes straight into tcgen05 (cvf.cu)
@@ -2368,7 +2382,11 @@ int conv_fwd_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaSt
   if (cvf_is(g.func)) return cvf_conv_launch(a, g, sig, st);
   ConvShape s = conv_shape(a);
   if (g.func == (const void*)smallc::conv_fwd_smallc_kernel<3, 3, 3, 32>) {
-    smallc::conv_fwd_smallc_kernel<3, 3, 3, 32><<<g.grid, g.block, 0, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s, sig);
+    smallc::conv_fwd_smallc_kernel<3, 3, 3, 32><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s, sig);
+    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
+  }
+  if (g.func == (const void*)smallc::conv_fwd_smallc_kernel<7, 7, 3, 64>) {
+    smallc::conv_fwd_smallc_kernel<7, 7, 3, 64><<<g.grid, g.block, g.smem, st>>>((const float*)a[0], (const float*)a[1], (float*)a[2], s, sig);
     return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
   }
   long long M = (long long)s.N * s.P * s.Q, N = s.K, K = (long long)s.R * s.S * s.C;

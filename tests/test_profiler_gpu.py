@@ -43,12 +43,21 @@ def test_closed_form_occupancy_matches_cuda_and_ncu(cfg, client):
         assert cf == info["blocks_per_sm"], (lab, fn, info, PR.occupancy_limits(info["threads_per_cta"], info["regs_per_thread"], smem))
         pipes.setdefault(fn, set()).add(info["pipe"])
         r = ncu.get(i)
-        if r is not None and int(float(r["grid"])) == info["grid_ctas"]:
+        # (a committed row describes the launch as it was built then: compare only rows whose grid,
+        # block size and registers are this build's)
+        if r is not None and int(float(r["grid"])) == info["grid_ctas"] and int(float(r["block"])) == info["threads_per_cta"] \
+                and int(float(r["regs"])) == info["regs_per_thread"]:
             lim = PR.occupancy_limits(info["threads_per_cta"], info["regs_per_thread"], smem)
             assert int(float(r["occ_warps"])) == lim["warps"], (lab, r)
             assert int(float(r["occ_regs"])) == lim["registers"], (lab, r)
-            assert int(float(r["occ_smem"])) == lim["shared_mem"], (lab, r)
+            # ncu's shared-memory limit follows the carveout the driver configured for the launch
+            # (<= the full 228 KB the closed form assumes); the binding limit agrees exactly
+            assert int(float(r["occ_smem"])) <= lim["shared_mem"], (lab, r)
+            ncu_min = min(int(float(r[k])) for k in ("occ_warps", "occ_regs", "occ_blocks", "occ_smem"))
+            assert ncu_min == min(lim.values()) == info["blocks_per_sm"], (lab, r, lim)
             checked_ncu += 1
+    if ncu:
+        assert checked_ncu >= len(ncu) // 2, f"committed ncu table mostly stale ({checked_ncu} of {len(ncu)} rows match this build)"
     # tensor-core operators report a tensor pipe; elementwise ones the FMA/ALU pipe
     for fn in ("relu", "relu6", "bn_apply", "bn_stats", "add", "layernorm", "gelu"):
         if fn in pipes:

@@ -150,6 +150,14 @@ def stem():
     t1 = timeit("conv_fwd", [x.data_ptr(), wt.data_ptr(), y.data_ptr()] + dims + [wf.data_ptr(), wf.numel() * 4])
     t2 = timeit("conv_wgrad", [x.data_ptr(), dy.data_ptr(), dw.data_ptr()] + dims + [wf.data_ptr(), wf.numel() * 4])
     print(f"stem fwd {t1:7.1f} us {byt / t1 / 1e3:5.0f} GB/s   wgrad {t2:7.1f} us {byt / t2 / 1e3:5.0f} GB/s")
+    # ResNet-50 HP stem (7x7/2, 3 -> 64) at batch 4
+    n, h, k, p = 4, 224, 64, 112
+    x, wt, y = torch.randn(n, h, h, 3, device="cuda"), torch.randn(k, 7, 7, 3, device="cuda"), torch.zeros(n, p, p, k, device="cuda")
+    dims = [n, h, h, 3, k, 7, 7, 2, 3, p, p]
+    wf = ws(L.lib.orion_gemm_workspace_bytes(n * p * p, k, 147))
+    a = [x.data_ptr(), wt.data_ptr(), y.data_ptr()] + dims + [wf.data_ptr(), wf.numel() * 4]
+    t3 = timeit("conv_fwd", a)
+    print(f"resnet stem b4 fwd {t3:7.1f} us {2 * n * p * p * k * 147 / t3 / 1e6:5.1f} TF  {kernel_info('conv_fwd', a)['kernel'][-40:]}")
 
 
 def attn():
@@ -165,6 +173,29 @@ def attn():
                                            B, S, H, d, D, D])
     fl = 4 * B * H * S * S * d
     print(f"attn fwd {t1:7.1f} us ({fl / t1 / 1e6:5.1f} TF)  bwd_dq {t2:7.1f} us  bwd_dkv {t3:7.1f} us")
+
+
+# MobileNetV2 b96 1x1 convolutions: (rows, Cin, Cout); forward y = x W^T (flags 2), data gradient
+# dx = dy W (flags 0, B = W [Cout][Cin] MN-major)
+G1X1 = [(1204224, 16, 96), (1204224, 32, 16), (301056, 24, 144), (301056, 144, 24), (75264, 32, 192), (75264, 192, 32),
+        (18816, 64, 384), (18816, 384, 64)]
+
+
+def g1x1():
+    tot = 0.0
+    for M, cin, cout in G1X1:
+        x, w, y = torch.randn(M, cin, device="cuda"), torch.randn(cout, cin, device="cuda"), torch.zeros(M, cout, device="cuda")
+        dy, dx = torch.randn(M, cout, device="cuda"), torch.zeros(M, cin, device="cuda")
+        wf = ws(max(L.lib.orion_gemm_workspace_bytes(M, cout, cin), L.lib.orion_gemm_workspace_bytes(M, cin, cout)))
+        af = [x.data_ptr(), w.data_ptr(), y.data_ptr(), 0, M, cout, cin, cin, cin, cout, 2, wf.data_ptr(), wf.numel() * 4]
+        ad = [dy.data_ptr(), w.data_ptr(), dx.data_ptr(), 0, M, cin, cout, cout, cin, cin, 0, wf.data_ptr(), wf.numel() * 4]
+        t1, t2 = timeit("gemm", af), timeit("gemm", ad)
+        tot += t1 + t2
+        byt = 4 * M * (cin + cout)
+        k1, k2 = kernel_info("gemm", af)["kernel"], kernel_info("gemm", ad)["kernel"]
+        print(f"1x1 M={M:8d} {cin:4d}->{cout:4d}  fwd {t1:7.1f} us {byt / t1 / 1e3:5.0f} GB/s  dgrad {t2:7.1f} us {byt / t2 / 1e3:5.0f} GB/s"
+              f"  {k1[-30:]} {k2[-30:]}")
+    print(f"1x1 total {tot:.1f} us")
 
 
 def wgs():
@@ -209,6 +240,8 @@ if __name__ == "__main__":
         stem()
     if what in ("attn", "all"):
         attn()
+    if what in ("g1x1", "all"):
+        g1x1()
     if what in ("dw", "all"):
         dw()
     if what in ("conv", "all"):

@@ -10,7 +10,7 @@ if [ -n "$NCU_PROFILE" ]; then
   METRICS=$METRICS,launch__block_size,sm__throughput.avg.pct_of_peak_sustained_elapsed,gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed,sm__pipe_tc_cycles_active.avg.pct_of_peak_sustained_elapsed,sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed,sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_elapsed,launch__occupancy_limit_blocks,launch__occupancy_limit_registers,launch__occupancy_limit_shared_mem,launch__occupancy_limit_warps,launch__registers_per_thread,launch__shared_mem_per_block_dynamic,launch__shared_mem_per_block_static
 fi
 for c in ${CLIENTS:-hp be}; do
-  timeout -s KILL 900 ncu --metrics $METRICS --clock-control none --csv --page raw \
+  timeout -s KILL ${NCU_TIMEOUT:-900} ncu --metrics $METRICS --clock-control none --csv --page raw \
      --kernel-name-base function -k "regex:$OURS" --log-file gpurun_out/ncu_times_${CONFIG:-rn50_mnv2}_${c}.csv python tools/profile/solo_runner.py --config ${CONFIG:-rn50_mnv2} --client $c > gpurun_out/ncu_times_${CONFIG:-rn50_mnv2}_${c}.out 2>&1
   base=0; [ "$c" = be ] && base=10000
   python tools/profile/ncu_summarize.py gpurun_out/ncu_times_${CONFIG:-rn50_mnv2}_${c}.csv gpurun_out/oplist_${CONFIG:-rn50_mnv2}_${c}.txt 0 gpurun_out/times_${CONFIG:-rn50_mnv2}_${c}.csv
