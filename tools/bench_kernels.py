@@ -198,6 +198,17 @@ def g1x1():
     print(f"1x1 total {tot:.1f} us")
 
 
+def pool():
+    """ResNet-50 b64 max-pool 3x3/2 forward and backward (config 3's BE, config 4's HP)."""
+    n, h, c, p = 64, 112, 64, 56
+    x, y, dy, dx = (torch.randn(n, h, h, c, device="cuda"), torch.zeros(n, p, p, c, device="cuda"), torch.randn(n, p, p, c, device="cuda"),
+                    torch.zeros(n, h, h, c, device="cuda"))
+    t1 = timeit("maxpool", [x.data_ptr(), y.data_ptr(), n, h, h, c, p, p])
+    t2 = timeit("maxpool_bwd", [x.data_ptr(), dy.data_ptr(), dx.data_ptr(), n, h, h, c, p, p])
+    print(f"maxpool fwd {t1:7.1f} us {(x.numel() + y.numel()) * 4 / t1 / 1e3:5.0f} GB/s   bwd {t2:7.1f} us "
+          f"{(2 * x.numel() + dy.numel()) * 4 / t2 / 1e3:5.0f} GB/s")
+
+
 def wgs():
     tot = 0.0
     for M, N, K in WGS:
@@ -242,6 +253,8 @@ if __name__ == "__main__":
         attn()
     if what in ("g1x1", "all"):
         g1x1()
+    if what in ("pool", "all"):
+        pool()
     if what in ("dw", "all"):
         dw()
     if what in ("conv", "all"):
