@@ -39,12 +39,6 @@ BnSplit bn_split(long long rows, int C) {
   return s;
 }
 
-// loads in flight per thread of the statistics kernel (ORION_BN_STATS_U: 8 or 16; tuning knob, read once)
-inline int bn_stats_u() {
-  static const int u = getenv("ORION_BN_STATS_U") && atoi(getenv("ORION_BN_STATS_U")) == 16 ? 16 : 8;
-  return u;
-}
-
 // workspace: [tickets][split partials rs x C x nvals][group partials combine_rows(rs) x C x nvals]
 uint64_t bn_ws_bytes(long long rows, int C, int nvals) {
   BnSplit s = bn_split(rows, C);
@@ -89,10 +83,7 @@ __device__ bool bn_partial2(const D4& a, const D4& b, int C, int cg4, int rl_n, 
 }
 
 // ---- train statistics: mean, invstd (biased var), running stats (unbiased var, momentum)
-// U = 128-bit loads in flight per thread per trip (a tuning template: 8 or 16; the accumulation order
-// per thread is the row order either way, so results do not depend on it)
-template <int U>
-__global__ void __launch_bounds__(BN_THREADS, 2) bn_stats_kernel(const float* __restrict__ x, float* mean, float* invstd, float* rm, float* rv,
+__global__ void __launch_bounds__(BN_THREADS) bn_stats_kernel(const float* __restrict__ x, float* mean, float* invstd, float* rm, float* rv,
                                                               long long rows, int C, float eps, float momentum, int cg4, int rl_n,
                                                               long long rows_per_split, unsigned char* ws, OrionSig sig) {
   __shared__ double sh[BN_THREADS * 8];
@@ -103,12 +94,12 @@ __global__ void __launch_bounds__(BN_THREADS, 2) bn_stats_kernel(const float* __
   if (c < C && rl < rl_n) {
     const float* xp = x + c;
     long long r = r0 + rl;
-    for (; r + (U - 1LL) * rl_n < r1; r += (long long)U * rl_n) {
-      float4 v[U];
+    for (; r + 7LL * rl_n < r1; r += 8LL * rl_n) {
+      float4 v[8];
 #pragma unroll
-      for (int i = 0; i < U; i++) v[i] = __ldg(reinterpret_cast<const float4*>(xp + (r + i * (long long)rl_n) * C));
+      for (int i = 0; i < 8; i++) v[i] = __ldg(reinterpret_cast<const float4*>(xp + (r + i * (long long)rl_n) * C));
 #pragma unroll
-      for (int i = 0; i < U; i++) { add4(s1, v[i]); sq4(s2, v[i]); }
+      for (int i = 0; i < 8; i++) { add4(s1, v[i]); sq4(s2, v[i]); }
     }
     for (; r < r1; r += rl_n) {
       float4 v = __ldg(reinterpret_cast<const float4*>(xp + r * C));
@@ -364,18 +355,12 @@ int bn_eval_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStr
 int bn_stats_geom(const uint64_t* a, LaunchGeom* g) {
   if ((a[6] & 3) || a[9] == 0 || a[10] < bn_ws_bytes((long long)a[5], (int)a[6], 2)) return ORION_E_INVAL;
   BnSplit sp = bn_split((long long)a[5], (int)a[6]);
-  g->grid = dim3(sp.cblocks, sp.rs); g->block = dim3(BN_THREADS); g->smem = 0;
-  g->func = bn_stats_u() == 16 ? (const void*)bn_stats_kernel<16> : (const void*)bn_stats_kernel<8>;
+  g->grid = dim3(sp.cblocks, sp.rs); g->block = dim3(BN_THREADS); g->smem = 0; g->func = (const void*)bn_stats_kernel;
   return 0;
 }
 int bn_stats_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   BnSplit sp = bn_split((long long)a[5], (int)a[6]);
-  if (g.func == (const void*)bn_stats_kernel<16>) {
-    bn_stats_kernel<16><<<g.grid, g.block, 0, s>>>((const float*)a[0], (float*)a[1], (float*)a[2], (float*)a[3], (float*)a[4], (long long)a[5],
-                                                  (int)a[6], u2f(a[7]), u2f(a[8]), sp.cg4, sp.rl, sp.rows_per_split, (unsigned char*)a[9], sig);
-    return cudaGetLastError() == cudaSuccess ? 0 : ORION_E_CUDA;
-  }
-  bn_stats_kernel<8><<<g.grid, g.block, 0, s>>>((const float*)a[0], (float*)a[1], (float*)a[2], (float*)a[3], (float*)a[4], (long long)a[5],
+  bn_stats_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (float*)a[1], (float*)a[2], (float*)a[3], (float*)a[4], (long long)a[5],
                                              (int)a[6], u2f(a[7]), u2f(a[8]), sp.cg4, sp.rl, sp.rows_per_split, (unsigned char*)a[9], sig);
   CHECK_LAUNCH();
 }
