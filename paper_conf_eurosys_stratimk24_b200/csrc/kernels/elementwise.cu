@@ -238,25 +238,30 @@ __global__ void __launch_bounds__(EW_THREADS) ce_kernel(const float* __restrict_
   orion_signal(sig);
 }
 
-// ---- MaxPool 3x3 / 2, pad 1 (-inf padding), NHWC, thread per output element
+// ---- MaxPool 3x3 / 2, pad 1 (-inf padding), NHWC, thread per output channel quad (128-bit loads;
+// the workloads' C % 4 == 0, checked at geometry time); fmaxf per channel, as the scalar form
 __global__ void __launch_bounds__(EW_THREADS) maxpool_kernel(const float* __restrict__ x, float* __restrict__ y, int N, int H, int W, int C,
                                                              int P, int Q, OrionSig sig) {
-  long long total = (long long)N * P * Q * C;
+  const int C4 = C / 4;
+  long long total = (long long)N * P * Q * C4;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (long long)gridDim.x * blockDim.x) {
-    int c = (int)(i % C); long long t = i / C;
+    int c = (int)(i % C4) * 4; long long t = i / C4;
     int q = (int)(t % Q); t /= Q;
     int p = (int)(t % P); int n = (int)(t / P);
-    float m = -FLT_MAX;
+    float4 m = make_float4(-FLT_MAX, -FLT_MAX, -FLT_MAX, -FLT_MAX);
+#pragma unroll
     for (int r = 0; r < 3; r++) {
       int h = 2 * p - 1 + r;
       if ((unsigned)h >= (unsigned)H) continue;
+#pragma unroll
       for (int s = 0; s < 3; s++) {
         int w = 2 * q - 1 + s;
         if ((unsigned)w >= (unsigned)W) continue;
-        m = fmaxf(m, __ldg(x + (((long long)n * H + h) * W + w) * C + c));
+        const float4 v = __ldg(reinterpret_cast<const float4*>(x + (((long long)n * H + h) * W + w) * C + c));
+        m.x = fmaxf(m.x, v.x); m.y = fmaxf(m.y, v.y); m.z = fmaxf(m.z, v.z); m.w = fmaxf(m.w, v.w);
       }
     }
-    y[i] = m;
+    reinterpret_cast<float4*>(y)[i] = m;
   }
   orion_signal(sig);
 }
@@ -345,7 +350,11 @@ int ce_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t
 }
 
 // ---- maxpool: args x, y, N, H, W, C, P, Q
-int maxpool_geom(const uint64_t* a, LaunchGeom* g) { ew_geom(g, a[2] * a[6] * a[7] * a[5], (const void*)maxpool_kernel); return 0; }
+int maxpool_geom(const uint64_t* a, LaunchGeom* g) {
+  if (a[5] % 4 || (a[0] & 15) || (a[1] & 15)) return ORION_E_INVAL;   // channel quads, 128-bit aligned
+  ew_geom(g, a[2] * a[6] * a[7] * (a[5] / 4), (const void*)maxpool_kernel);
+  return 0;
+}
 int maxpool_launch(const uint64_t* a, const LaunchGeom& g, OrionSig sig, cudaStream_t s) {
   maxpool_kernel<<<g.grid, g.block, 0, s>>>((const float*)a[0], (float*)a[1], (int)a[2], (int)a[3], (int)a[4], (int)a[5], (int)a[6],
                                             (int)a[7], sig);

@@ -1943,11 +1943,15 @@ inline bool fwd_ok(const ConvShape& s) { return fwd3_ok(s) || fwd7_ok(s); }
 // owns a 4 (k) x <= WG_MAXR (rsc) register block. Partials (fp64) of the G CTAs (a shape-only
 // count) are combined in CTA order (combine_splits), so results are deterministic.
 constexpr int WG_QT = 32, WG_KPT = 4, WG_MAXR = 10, WG_G = 296;   // two CTAs per SM of a full B200
+// (Measured and reverted: eight resident waves of the 7x7 stem's weight gradient -- each CTA living
+// ~0.1 ms instead of the whole 0.9 ms op at ResNet-50's training batch -- cost 891 -> 978 us and left
+// config 3's HP p99 where it was, 1.29x vs 1.31x.)
+constexpr int WG1_G = WG_G;
 constexpr int WG_PF_DY = WG_QT * MAXK / 4 / NTH, WG_PF_X = 8;   // per-thread prefetch registers
 __host__ __device__ inline int wg_wwin(const ConvShape& s) { return (WG_QT - 1) * s.stride + s.S; }
 __host__ __device__ inline int wg_xwin(const ConvShape& s) { return s.R * wg_wwin(s) * s.C; }
 inline long long wg_tiles(const ConvShape& s) { return (long long)s.N * s.P * ((s.Q + WG_QT - 1) / WG_QT); }
-inline int wg_ctas(const ConvShape& s) { return (int)(wg_tiles(s) < WG_G ? wg_tiles(s) : WG_G); }
+inline int wg_ctas(const ConvShape& s) { return (int)(wg_tiles(s) < WG1_G ? wg_tiles(s) : WG1_G); }
 // register-block width (rsc per thread) of the launch: 10 for the ResNet stem (147 / 16 groups)
 inline int wg_nr(const ConvShape& s) { return (s.R * s.S * s.C + NTH / (s.K / WG_KPT) - 1) / (NTH / (s.K / WG_KPT)); }
 // Taken for the large stems (R*S*C >= 64, e.g. ResNet's 7x7x3); the 3x3x3 MobileNetV2 stem has too
@@ -1958,10 +1962,14 @@ inline bool wgrad_ok(const ConvShape& s) {
          wg_xwin(s) <= NTH * WG_PF_X && s.stride <= 2;
 }
 inline bool wgrad2_ok(const ConvShape& s);
+inline int w2_ctas(const ConvShape& s);
 inline uint64_t wgrad_ws_bytes(const ConvShape& s) {
-  const int G = wg_ctas(s);
   const uint64_t V = (uint64_t)s.K * s.R * s.S * s.C;
-  return WS_TICKET_BYTES + (uint64_t)(G + combine_rows(G) + 1) * V * 8;
+  const int G = wg_ctas(s), G2 = w2_ctas(s);
+  // 7x7 kernel: fp32 partials + fp64 group rows; 3x3 kernel: fp64 partials + group rows
+  const uint64_t b1 = WS_TICKET_BYTES + ((uint64_t)G * V * 4 + 15) / 16 * 16 + (uint64_t)(combine_rows(G) + 1) * V * 8;
+  const uint64_t b2 = WS_TICKET_BYTES + (uint64_t)(G2 + combine_rows(G2) + 1) * V * 8;
+  return b1 > b2 ? b1 : b2;
 }
 
 template <int NR>
@@ -1984,11 +1992,11 @@ __global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc_kernel(const float* 
       off[i] = 0;   // padding slot: accumulates garbage that is never stored (no branch in the hot loop)
     }
   }
-  float acc[WG_KPT][NR];
+  float2 acc2[WG_KPT / 2][NR];   // (k, k+1) pairs: packed FFMA2, each lane rounded as fmaf
 #pragma unroll
-  for (int a = 0; a < WG_KPT; a++)
+  for (int a = 0; a < WG_KPT / 2; a++)
 #pragma unroll
-    for (int i = 0; i < NR; i++) acc[a][i] = 0.f;
+    for (int i = 0; i < NR; i++) acc2[a][i] = make_float2(0.f, 0.f);
   const int qtiles = (s.Q + WG_QT - 1) / WG_QT;
   const long long T = (long long)s.N * s.P * qtiles;
   float4 pdy[WG_PF_DY];
@@ -2033,33 +2041,32 @@ __global__ void __launch_bounds__(NTH, 2) conv_wgrad_smallc_kernel(const float* 
     __syncthreads();
     if (t + gridDim.x < T) WG_FETCH(t + gridDim.x);    // next tile's loads in flight during the math
     const int xstep = s.stride * s.C;
-#pragma unroll 2
+#pragma unroll 4
     for (int i = 0; i < WG_QT; i++) {                   // zero dy rows beyond Q contribute nothing
       const float4 d = *reinterpret_cast<const float4*>(dys + i * K + kg * WG_KPT);
       const float* xr = xs + i * xstep;
 #pragma unroll
       for (int j = 0; j < NR; j++) {
         const float xv = xr[off[j]];
-        acc[0][j] = fmaf(d.x, xv, acc[0][j]);
-        acc[1][j] = fmaf(d.y, xv, acc[1][j]);
-        acc[2][j] = fmaf(d.z, xv, acc[2][j]);
-        acc[3][j] = fmaf(d.w, xv, acc[3][j]);
+        ffma2(acc2[0][j], xv, make_float2(d.x, d.y));
+        ffma2(acc2[1][j], xv, make_float2(d.z, d.w));
       }
     }
   }
   // partial of this CTA -> workspace (fp64), ordered combine over the G CTAs
   const long long V = (long long)K * RSC;
   unsigned int* tk = reinterpret_cast<unsigned int*>(ws);
-  double* part = reinterpret_cast<double*>(ws + WS_TICKET_BYTES);
+  float* part = reinterpret_cast<float*>(ws + WS_TICKET_BYTES);
   const int G = gridDim.x;
-  double* gpart = part + (long long)G * V;
+  double* gpart = reinterpret_cast<double*>(ws + WS_TICKET_BYTES + ((uint64_t)G * V * 4 + 15) / 16 * 16);
   double* out = gpart + (long long)combine_rows(G) * V;
 #pragma unroll
   for (int j = 0; j < NR; j++) {
     const int jj = rg + rgroups * j;
     if (jj < RSC) {
 #pragma unroll
-      for (int a = 0; a < WG_KPT; a++) part[(long long)blockIdx.x * V + (long long)(kg * WG_KPT + a) * RSC + jj] = (double)acc[a][j];
+      for (int a = 0; a < WG_KPT; a++)
+        part[(long long)blockIdx.x * V + (long long)(kg * WG_KPT + a) * RSC + jj] = (a & 1) ? acc2[a / 2][j].y : acc2[a / 2][j].x;
     }
   }
   __shared__ double scratch[NTH];

@@ -94,7 +94,7 @@ def floor():
     print(f"relu 4x56x56x64 {t:6.2f} us")
 
 
-BE_CWG = [(64, 56, 56, 64, 64, 3, 1, 1), (64, 56, 56, 128, 128, 3, 2, 1), (64, 28, 28, 128, 128, 3, 1, 1), (64, 14, 14, 256, 256, 3, 1, 1),
+BE_CWG = [(64, 224, 224, 3, 64, 7, 2, 3), (64, 56, 56, 64, 64, 3, 1, 1), (64, 56, 56, 128, 128, 3, 2, 1), (64, 28, 28, 128, 128, 3, 1, 1), (64, 14, 14, 256, 256, 3, 1, 1),
           (64, 7, 7, 512, 512, 3, 1, 1), (64, 56, 56, 256, 512, 1, 2, 0), (64, 28, 28, 512, 1024, 1, 2, 0)]
 
 
