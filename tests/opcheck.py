@@ -61,6 +61,12 @@ def check_op(fn, a, R, snap=None, R_in=None):
         if a[3]:
             ref = ref + T(a[3], N).double()
         out = R.get(a[2], M * ldc).view(M, ldc)[:, :N]
+        if fl & 1:
+            # weight gradients reduce over N*H*W rows of mixed-sign terms: the error is normalised by
+            # the absolute-term sum || |A|^T |B| || (a gradient is held to tol * max(1, kappa)
+            # in rel L2, kappa = || |A|^T |B| || / || A^T B ||; the same as rel L2 when nothing cancels)
+            absref = Ad.double().abs() @ Bd.double().abs()
+            return rel(out, om._r(ref)) / max(1.0, float(absref.norm() / max(float(ref.norm()), 1e-30)))
         return rel(out, om._r(ref))
     if fn in ("conv_fwd", "conv_dgrad", "conv_wgrad", "dw_fwd", "dw_dgrad", "dw_wgrad"):
         n, h, w, c, k, r, s, st, pad, p, q = a[3:14]
@@ -73,7 +79,10 @@ def check_op(fn, a, R, snap=None, R_in=None):
             dy, wt = T(a[0], n * p * q * k, (n, p, q, k)), T(a[1], k * r * s * cg, (k, r, s, cg))
             return rel(R.get(a[2], n * h * w * c, (n, h, w, c)), om.conv2d_bwd_data(dy, wt, (n, h, w, c), st, pad, groups))
         x, dy = T(a[0], n * h * w * c, (n, h, w, c)), T(a[1], n * p * q * k, (n, p, q, k))
-        return rel(R.get(a[2], k * r * s * cg, (k, r, s, cg)), om.conv2d_bwd_weight(x, dy, (k, r, s, cg), st, pad, groups))
+        ref = om.conv2d_bwd_weight(x, dy, (k, r, s, cg), st, pad, groups)
+        absref = om.conv2d_bwd_weight_abs(x, dy, (k, r, s, cg), st, pad, groups)
+        kappa = max(1.0, float(absref.double().norm() / max(float(ref.double().norm()), 1e-30)))   # (as for gemm flags & 1)
+        return rel(R.get(a[2], k * r * s * cg, (k, r, s, cg)), ref) / kappa
     if fn in ("relu", "relu6"):
         x = T(a[0], a[2])
         return rel(R.get(a[1], a[2]), (om.relu if fn == "relu" else om.relu6)(x))

@@ -72,3 +72,28 @@ def test_resnet50_train_ops_teacher_forced():
         print("rn50 train", e)
     bad = [e for e in errs if e[0] > 2e-5]
     assert not bad, sorted(bad, reverse=True)[:10]
+
+
+def test_resnet50_train_ops_full_size_sampled():
+    """Config 3's BE client at its full size (ResNet-50 training b64, 224x224): the whole op list runs
+    through the C ABI in order; every 8th op plus every loss / BN-statistics op is checked
+    teacher-forced against the fp64 oracle op (all ops at full size would take ~10 min of fp64 CPU)."""
+    P = si.make_params(W.resnet_train_spec())
+    g = W.resnet_train_graph(P, [si.normal((64, 224, 224, 3), si.BE_SEED, sub=0)], [si.labels(64, 1000, si.BE_SEED, sub=0)])
+    Pm = g.params
+    tensors = [Pm.flat] + list(g.bufs.values()) + list(Pm.p.values()) + list(Pm.g.values()) + [g._ws]
+    R = opcheck.Resolver(tensors)
+    R_in = opcheck.Resolver(tensors, read_alias={Pm.flat.data_ptr(): Pm.flat.clone()})
+    snaps = _launch_all(g, R)
+    errs = []
+    for i, (fn, args, lab) in enumerate(g.ops):
+        if not isinstance(fn, str) or fn == "sgd" or (i % 8 and fn not in ("ce", "bn_stats")):
+            continue
+        e = opcheck.check_op(fn, args, R, snaps.get(i), R_in)
+        assert e is not None, fn
+        errs.append((e, i, lab, fn))
+    for e in sorted(errs, reverse=True)[:8]:
+        print("rn50 train full", e)
+    assert len(errs) >= 100, len(errs)
+    bad = [e for e in errs if e[0] > 2e-5]
+    assert not bad, sorted(bad, reverse=True)[:10]
