@@ -3,7 +3,7 @@
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
 for pol in ${POLICIES:-streams priorities profiles orion orion_noprio}; do
-  timeout -s KILL 900 python bench.py --config ${CONFIG:-rn50_mnv2} --policy $pol --steps ${STEPS:-300} --warmup 5 --no-e2e --no-cpu-baseline \
+  timeout -s KILL 900 python bench.py --config ${CONFIG:-rn50_mnv2} --policy $pol --steps ${STEPS:-20} --warmup 5 --no-e2e --no-cpu-baseline --no-stress \
     > gpurun_out/ablation_${CONFIG:-rn50_mnv2}_$pol.log 2>&1
   python - "$pol" "gpurun_out/ablation_${CONFIG:-rn50_mnv2}_$pol.log" <<'PY'
 import json, sys
