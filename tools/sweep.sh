@@ -7,7 +7,7 @@ SWEEP=${SWEEP:-"--dur-ppm 10000;--dur-ppm 25000;--dur-ppm 50000;--dur-ppm 100000
 IFS=';' read -ra CFGS <<< "$SWEEP"
 for cfg in "${CFGS[@]}"; do
   tag=${CONFIG:-rn50_mnv2}_$(echo "$cfg" | tr -c 'a-z0-9\n' '_')
-  timeout -s KILL 900 python bench.py --config ${CONFIG:-rn50_mnv2} --steps ${STEPS:-150} --warmup 3 --no-e2e --no-cpu-baseline $cfg > gpurun_out/sweep/$tag.log 2>&1
+  timeout -s KILL 900 python bench.py --config ${CONFIG:-rn50_mnv2} --steps ${STEPS:-20} --warmup 3 --no-e2e --no-cpu-baseline --no-stress $cfg > gpurun_out/sweep/$tag.log 2>&1
   python - "$cfg" gpurun_out/sweep/$tag.log <<'PY'
 import json, sys
 line = [l for l in open(sys.argv[2]) if l.startswith("{")]
